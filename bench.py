@@ -1,0 +1,360 @@
+#!/usr/bin/env python
+"""bench.py — the driver's benchmark contract for the CPU-Free Jacobi hot path.
+
+    python bench.py [--gpus N] [--steps K] [--warmup W] [--config c2] [--impl ours|reference]
+
+One "step" is one pass of the whole hot path over the BASELINE.json workload: one
+``jacobi_run(iters)`` call — ONE persistent kernel per GPU running every iteration with the
+halo exchange, flags and grid barriers inside.  At N = 1 the
+workload is BASELINE.json configs[1] (C2: 2D 5-point 16384x16384 fp64, 1000 iterations).
+``value`` = interior cells x iterations x K / max-over-ranks device time (CUDA events on the
+launch stream around each launch), in Gcell-updates/s.  Inputs (2 GiB per buffer) are larger
+than the 126 MB L2, so no flush is needed between steps.
+
+Extra keys: ``roofline`` (the persistent kernel vs the measured HBM copy bandwidth),
+``cpu_baseline`` (the CPU oracle on this host's cores, bounded sample), ``e2e`` (the same
+metric through the C ABI with pinned host buffers: scatter + run + gather per step),
+``cpu_controlled`` (the per-iteration-launch baselines), ``clocks``.
+
+``--impl reference``: there is no reference implementation to install (PAPER.md only), so
+the reference arm is the CPU oracle timed on this host.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import subprocess
+import sys
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+if ROOT not in sys.path:
+    sys.path.insert(0, ROOT)
+
+with open(os.path.join(ROOT, "BASELINE.json")) as _f:
+    _BJ = json.load(_f)
+METRIC = _BJ["metric"]
+UNIT = "Gcell-updates/s"
+
+# Workloads of BASELINE.json "configs".  shape = (nz, ny, nx) incl. boundary.
+CONFIGS = {
+    "c1": dict(shape=(1, 256, 256), iters=1000, scaling="strong",
+               workload="C1: 2D 5-point Jacobi 256x256 fp64, Dirichlet boundary, 1000 iterations"),
+    "c2": dict(shape=(1, 16384, 16384), iters=1000, scaling="strong",
+               workload="C2: 2D 5-point Jacobi 16384x16384 fp64, 1000 iterations, row-slab decomposition"),
+    "c3": dict(shape=(512, 512, 512), iters=1000, scaling="strong",
+               workload="C3: 3D 7-point Jacobi 512^3 fp64, 1000 iterations, z-slab decomposition"),
+    "c4": dict(shape=None, iters=1000, scaling="weak",
+               workload="C4: 3D 7-point Jacobi weak scaling 512x512x(512*P) fp64, 1000 iterations"),
+    "c5a": dict(shape=(128, 128, 128), iters=1000, scaling="strong",
+                workload="C5a: 3D 7-point Jacobi 128^3 fp64 latency sweep, 1000 iterations"),
+    "c5b": dict(shape=(1, 1024, 1024), iters=1000, scaling="strong",
+                workload="C5b: 2D 5-point Jacobi 1024x1024 fp64 latency sweep, 1000 iterations"),
+}
+L2_BYTES = 126 * 1024 * 1024
+
+
+def interior_cells(shape):
+    nz, ny, nx = shape
+    return (nx - 2) * (ny - 2) * (max(nz - 2, 1) if nz > 1 else 1)
+
+
+def measured_hbm():
+    p = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    try:
+        with open(p) as f:
+            return float(json.load(f)["hbm_gbs"]), "measured"
+    except Exception:
+        return 6650.0, "fallback"
+
+
+class ClockSampler:
+    """nvidia-smi clocks / throttle reasons sampled during the timed region."""
+    Q = ("index,clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,"
+         "clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
+         "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, device: int):
+        self.device = device
+        self.proc = None
+
+    def start(self):
+        try:
+            self.proc = subprocess.Popen(["nvidia-smi", "-i", str(self.device), f"--query-gpu={self.Q}",
+                                          "--format=csv,noheader,nounits", "-lms", "200"],
+                                         stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
+        except Exception:
+            self.proc = None
+
+    def stop(self):
+        if not self.proc:
+            return None
+        time.sleep(0.25)
+        self.proc.terminate()
+        out, _ = self.proc.communicate(timeout=10)
+        sm, mx, reasons = [], None, set()
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        for line in out.strip().splitlines():
+            parts = [p.strip() for p in line.split(",")]
+            if len(parts) < 9:
+                continue
+            try:
+                sm.append(float(parts[1]))
+                mx = float(parts[2])
+            except ValueError:
+                continue
+            for n, v in zip(names, parts[5:9]):
+                if v.lower().startswith("active"):
+                    reasons.add(n)
+        if not sm:
+            return None
+        return {"sm_mhz": statistics.median(sm), "sm_max_mhz": mx, "reasons": sorted(reasons),
+                "samples": len(sm)}
+
+
+def dist_env():
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    return world, rank, local
+
+
+def oracle_sample(shape, iters_sample, seed=0x5C24, field=None):
+    """Time the CPU oracle (as it stands) on this host's cores; returns (Gcell/s, seconds, cores)."""
+    import oracle
+    from jacobi_inputs import u12
+    if field is None:
+        field = u12(shape if shape[0] > 1 else shape[1:], seed)
+    cores = os.cpu_count() or 1
+    t0 = time.perf_counter()
+    oracle.jacobi(field, iters_sample, cores)
+    dt = time.perf_counter() - t0
+    return interior_cells(shape) * iters_sample / dt / 1e9, dt, cores
+
+
+def ncu_traffic(config: str, iters: int):
+    """dram bytes per launch from the committed ncu --set full summary of this config, if any."""
+    p = os.path.join(ROOT, "profiles", "ncu_summary.json")
+    try:
+        with open(p) as f:
+            d = json.load(f)
+        e = d[config]
+        return e["dram_bytes_per_iter"] * iters, e
+    except Exception:
+        return None, None
+
+
+def run_reference(args, cfg, shape):
+    world, rank, _ = dist_env()
+    if rank != 0:
+        return 0
+    from jacobi_inputs import u12
+    field = u12(shape if shape[0] > 1 else shape[1:], 0x5C24)
+    k_iter = args.ref_iters
+    for _ in range(args.warmup):
+        oracle_sample(shape, k_iter, field=field)
+    vals, secs = [], []
+    for _ in range(args.steps):
+        v, dt, cores = oracle_sample(shape, k_iter, field=field)
+        vals.append(v)
+        secs.append(dt)
+    value = interior_cells(shape) * k_iter * args.steps / sum(secs) / 1e9
+    sample = f"{k_iter} of {cfg['iters']} iterations of the full {cfg['workload'].split(':')[0]} grid per step"
+    line = {
+        "impl": "reference", "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": args.gpus,
+        "steps": args.steps, "warmup": args.warmup, "ms_per_step": 1e3 * sum(secs) / args.steps,
+        "higher_is_better": True, "scaling": cfg["scaling"], "vs_baseline": None, "dtype": "f64",
+        "data": "synthetic (U12 seed 0x5C24)",
+        "config": {"workload": cfg["workload"], "shape_zyx": list(shape), "iters": cfg["iters"]},
+        "cpu_baseline": {"value": value, "unit": UNIT, "cores": cores, "kind": "oracle", "sample": sample},
+        "e2e": {"value": value, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
+        "note": "no reference code exists (PAPER.md only); the reference arm is the CPU oracle",
+    }
+    print(json.dumps(line), flush=True)
+    return 0
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=3)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--config", default="c2", choices=sorted(CONFIGS))
+    ap.add_argument("--iters", type=int, default=0, help="override iterations per step")
+    ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    ap.add_argument("--ref-iters", type=int, default=2, help="oracle iterations per reference step")
+    ap.add_argument("--no-extras", action="store_true", help="skip e2e / cpu_baseline / baselines")
+    ap.add_argument("--virtual", type=int, default=0, help="(measurement aid) P slabs on one GPU")
+    ap.add_argument("--param", action="append", default=[], help="tuning knob name=value (jacobi_set_param)")
+    args = ap.parse_args()
+    args.warmup = max(args.warmup, 3) if args.impl == "ours" else args.warmup
+
+    world, rank, local = dist_env()
+    cfg = dict(CONFIGS[args.config])
+    if args.iters:
+        cfg["iters"] = args.iters
+    shape = cfg["shape"] or (512 * max(world, 1), 512, 512)
+    iters = cfg["iters"]
+
+    if args.impl == "reference":
+        return run_reference(args, cfg, shape)
+
+    import numpy as np
+    import torch
+    import paper_conf_sc_baydamirlibu24_b200 as jb
+
+    if world > 1:
+        import torch.distributed as dist
+        dist.init_process_group("gloo")
+        j = jb.Jacobi(shape, dist=(rank, world), device=local)
+        jb.exchange_peers(j, nccl=True)
+    else:
+        dist = None
+        j = jb.Jacobi(shape, virtual=args.virtual) if args.virtual else jb.Jacobi(shape, ngpus=1)
+    torch.cuda.set_device(local)
+    for kv in args.param:
+        k, v = kv.split("=")
+        j.set_param(k, int(v))
+
+    def barrier():
+        if dist is not None:
+            dist.barrier()
+
+    def max_over_ranks(x: float) -> float:
+        if dist is None:
+            return x
+        t = torch.tensor([x], dtype=torch.float64)
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        return float(t.item())
+
+    cells = interior_cells(shape)
+    desc = j.describe(0)
+    local_cells = cells // (shape[0] - 2 if shape[0] > 1 else shape[1] - 2) * desc["chunk"] \
+        if world > 1 else cells
+
+    # ---- warm-up + timed region (device time per launch from CUDA events on the launch stream)
+    for _ in range(args.warmup):
+        j.run(iters)
+    barrier()
+    torch.cuda.synchronize()
+    clocks = ClockSampler(local) if rank == 0 else None
+    if clocks:
+        clocks.start()
+    t_wall0 = time.perf_counter()
+    step_ms = []
+    for _ in range(args.steps):
+        j.run(iters)
+        step_ms.append(j.last_time_ms())
+    torch.cuda.synchronize()
+    barrier()
+    t_wall = time.perf_counter() - t_wall0
+    clk = clocks.stop() if clocks else None
+    dev_ms_local = sum(step_ms)
+    dev_ms = max_over_ranks(dev_ms_local)
+    value = cells * iters * args.steps / (dev_ms / 1e3) / 1e9
+
+    # ---- roofline of the dominant (only) kernel: the persistent sweep
+    peak, peak_kind = measured_hbm()
+    launch_ms = dev_ms_local / args.steps
+    alg_bytes = 16 * local_cells * iters  # read once + write once per cell-update
+    achieved = alg_bytes / (launch_ms / 1e3) / 1e9
+    traffic, _ = ncu_traffic(args.config, iters)
+    roofline = {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
+                "frac": achieved / peak, "traffic": traffic, "peak_kind": peak_kind,
+                "kernel": f"jb_sweep<{2 if shape[0] == 1 else 3},false,true> (persistent CPU-Free kernel)",
+                "alg_bytes_per_launch": alg_bytes}
+
+    line = {
+        "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
+        "warmup": args.warmup, "ms_per_step": dev_ms / args.steps, "higher_is_better": True,
+        "scaling": cfg["scaling"], "vs_baseline": None, "dtype": "f64",
+        "data": "synthetic (U12 seed 0x5C24, initialised on the device)",
+        "config": {"workload": cfg["workload"], "shape_zyx": list(shape), "iters": iters,
+                   "parallelism": f"slab{world}" + (f" (virtual {args.virtual} slabs)" if args.virtual else ""),
+                   "l2": ("inputs larger than L2" if 8 * cells > L2_BYTES else "L2-resident (latency config)"),
+                   "tile": {k: desc[k] for k in ("tile_x", "tile_y", "stages", "ctas", "n_top", "n_bot", "k_planes")}},
+        "gpu_launches": args.steps * world,
+        "wall_ms_per_step": 1e3 * t_wall / args.steps,
+        "ms_per_iter": dev_ms / args.steps / iters,
+        "roofline": roofline,
+        "clocks": clk,
+    }
+
+    if not args.no_extras:
+        # ---- CPU-controlled baselines (per-iteration launch + copy/NCCL + host sync), short run
+        base = {}
+        b_iters = min(iters, 200)
+        for name, mode in (("memcpy", jb.MODE_BASELINE_MEMCPY), ("nccl", jb.MODE_BASELINE_NCCL)):
+            if world > 1 and name == "memcpy":
+                continue
+            try:
+                j.set_mode(mode)
+                j.run(b_iters)  # warm
+                j.run(b_iters)
+                ms = max_over_ranks(j.last_time_ms())
+                base[name] = {"value": cells * b_iters / (ms / 1e3) / 1e9, "unit": UNIT,
+                              "ms_per_iter": ms / b_iters, "iters": b_iters}
+            except jb.JacobiError as e:
+                base[name] = {"error": str(e)}
+        j.set_mode(jb.MODE_CPUFREE)
+        line["cpu_controlled"] = base
+
+        # ---- e2e through the C ABI with pinned host buffers (scatter + run + gather per step)
+        from jacobi_inputs import u12_flat
+        nz, ny, nx = shape
+        plane = nx * (ny if nz > 1 else 1)
+        n_out = nz if nz > 1 else ny
+        start, chunk = desc["start"], desc["chunk"]
+        if world > 1:
+            lo, hi = start - 1, start + chunk + 1  # this rank's slab + halos
+        else:
+            lo, hi = 0, n_out
+        nbytes = (hi - lo) * plane * 8
+        h_in = torch.empty((hi - lo) * plane, dtype=torch.float64, pin_memory=True)
+        h_out = torch.empty((hi - lo) * plane, dtype=torch.float64, pin_memory=True)
+        h_in.numpy()[:] = u12_flat(lo * plane, (hi - lo) * plane, 0x5C24)
+        base_in = h_in.data_ptr() - lo * plane * 8
+        base_out = h_out.data_ptr() - lo * plane * 8
+        d2h = (chunk + (1 if start == 1 else 0) + (1 if start + chunk == n_out - 1 else 0)) * plane * 8
+        jb.jacobi_scatter_ptr(j.h, base_in)
+        j.run(iters)
+        jb.jacobi_gather_ptr(j.h, base_out)
+        barrier()
+        t0 = time.perf_counter()
+        for _ in range(args.steps):
+            jb.jacobi_scatter_ptr(j.h, base_in)
+            j.run(iters)
+            jb.jacobi_gather_ptr(j.h, base_out)
+        barrier()
+        e2e_s = max_over_ranks(time.perf_counter() - t0)
+        h2d_total = max_over_ranks(float(nbytes)) if world == 1 else nbytes * world
+        d2h_total = float(d2h) if world == 1 else None
+        if world > 1:
+            d2h_total = max_over_ranks(float(d2h)) * world
+        line["e2e"] = {"value": cells * iters * args.steps / e2e_s / 1e9, "unit": UNIT,
+                       "h2d_bytes_per_step": int(h2d_total), "d2h_bytes_per_step": int(d2h_total),
+                       "ms_per_step": 1e3 * e2e_s / args.steps,
+                       "path": "jacobi_scatter (pinned H2D) + jacobi_run + jacobi_gather (pinned D2H)"}
+
+        # ---- CPU oracle on this host's cores (rank 0, N = 1 only), bounded sample
+        if rank == 0 and world == 1:
+            field = h_in.numpy().reshape(shape if nz > 1 else shape[1:])
+            v1, dt1, cores = oracle_sample(shape, 1, field=field)
+            k = int(max(1, min(50, 10.0 / max(dt1, 1e-3))))
+            v, dt, cores = oracle_sample(shape, k, field=field)
+            line["cpu_baseline"] = {"value": v, "unit": UNIT, "cores": cores, "kind": "oracle",
+                                    "sample": f"{k} of {iters} iterations on the full grid "
+                                              f"({dt:.1f} s, OpenMP over the outer axis)"}
+    if rank == 0:
+        print(json.dumps(line), flush=True)
+    j.close()
+    if dist is not None:
+        dist.barrier()
+        dist.destroy_process_group()
+    return 0
+
+
+if __name__ == "__main__":
+    sys.exit(main())

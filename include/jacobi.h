@@ -1,0 +1,153 @@
+/*
+ * jacobi.h — C ABI of the B200-native CPU-Free Jacobi library (libjacobi_b200.so).
+ *
+ * What the library computes (PAPER.md = /root/reference/PAPER.md):
+ *   The Jacobi method for the Laplace equation with Dirichlet data on the domain boundary
+ *   (§2.1), on a 2D 5-point ("2D5pt", Fig. 4.1) or 3D 7-point ("3D7pt",
+ *   P:535 §6.1.1) grid, for a fixed number of iterations (Listing 4.1), every
+ *   iteration reading only the previous time step (§4.1.1).  The grid is divided
+ *   equally into slabs along its outermost axis (y in 2D, z in 3D) with one halo plane on
+ *   each side, one slab per GPU.
+ *   In the CPU-Free mode (Ch.3-4) every iteration runs inside ONE persistent kernel per GPU
+ *   (§3.1.1): boundary thread blocks wait on a flag from their neighbour, compute
+ *   the edge plane, store it straight into the neighbour GPU's halo over NVLink and raise the
+ *   neighbour's flag (Listing 4.1), interior thread blocks stream
+ *   the bulk, and a device-side grid barrier ends the iteration.
+ *   The CPU-controlled comparison modes launch one kernel per iteration and move halos with
+ *   cudaMemcpyPeerAsync or NCCL send/recv, with a host synchronisation per iteration
+ *   (Listing 2.1a).
+ *
+ * Numerics (readings R1-R4): IEEE fp64, per interior cell
+ *   2D: new = 0.25 * (((u[x+1] + u[x-1]) + u[y+1]) + u[y-1])
+ *   3D: new = fl(1/6) * (((((u[x+1] + u[x-1]) + u[y+1]) + u[y-1]) + u[z+1]) + u[z-1])
+ *   no FMA contraction, no flush-to-zero: results are bitwise identical to the CPU oracle and
+ *   independent of the number of GPUs, the mode and the tiling.
+ *
+ * Field layout seen by the caller (scatter/gather): C-contiguous fp64 array of nx*ny*nz
+ * doubles, x fastest, idx = (z*ny + y)*nx + x; 2D has nz == 1.  Extents INCLUDE the one-cell
+ * Dirichlet layer on every face; only interior cells (1..n-2 on every axis) are ever updated.
+ *
+ * Error behaviour: every int-returning call returns JACOBI_OK (0) or a negative JACOBI_E*
+ * code; after any error the handle remains valid for jacobi_destroy.  A handle is used by one
+ * host thread at a time (not re-entrant).  Calls block until their GPU work is complete.
+ * Ownership: the library owns all device memory and peer mappings it creates; the caller owns
+ * every host array it passes (pageable or pinned; copies are synchronous).
+ */
+#ifndef JACOBI_B200_H
+#define JACOBI_B200_H
+
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+/* ---- error codes --------------------------------------------------------------------- */
+#define JACOBI_OK        0
+#define JACOBI_EINVAL   -1  /* bad argument (extents < 3, stencil/nz mismatch, slab < 2 planes when P > 1, ...) */
+#define JACOBI_ENODEV   -2  /* requested more GPUs than visible / bad device index */
+#define JACOBI_ENOPEER  -3  /* cudaDeviceCanAccessPeer failed for a neighbour pair */
+#define JACOBI_ENOCOOP  -4  /* no cooperative launch, or the persistent grid is not co-resident */
+#define JACOBI_ENOMEM   -5  /* device or host allocation failed */
+#define JACOBI_ECUDA    -6  /* any other CUDA runtime error */
+#define JACOBI_ETIMEOUT -7  /* device watchdog fired: a neighbour never signalled (state undefined) */
+#define JACOBI_ENCCL    -8  /* NCCL unavailable or failed */
+#define JACOBI_ESTATE   -9  /* call not valid in this handle's state (e.g. peers not attached) */
+
+/* ---- modes for jacobi_set_mode --------------------------------------------------------- */
+#define JACOBI_MODE_CPUFREE          0  /* persistent TB-specialised kernel, device-side flags (default) */
+#define JACOBI_MODE_BASELINE_MEMCPY  1  /* per-iteration kernel + cudaMemcpyPeerAsync + host sync */
+#define JACOBI_MODE_BASELINE_NCCL    2  /* per-iteration kernel + ncclSend/ncclRecv + host sync */
+
+/* ---- flags for jacobi_set_mode --------------------------------------------------------- */
+#define JACOBI_FLAG_NO_COMPUTE   1  /* measurement only: skip the stencil
+                                       arithmetic and interior sweep, keep halo copies, flags and
+                                       barriers.  The field is NOT a Jacobi result afterwards. */
+#define JACOBI_FLAG_DROP_SIGNAL  2  /* debug: slab 0 never raises its neighbours' flags (tests the
+                                       watchdog; the run must return JACOBI_ETIMEOUT) */
+
+typedef struct jacobi_ctx *jacobi_t; /* opaque, library-owned */
+
+/* ---- creation ---------------------------------------------------------------------------
+ * All creators validate: nx, ny >= 3; stencil == 5 with nz == 1, or stencil == 7 with nz >= 3;
+ * nslabs >= 1; if nslabs > 1 every slab owns >= 2 outer planes (chunk sizes follow
+ * jacobi_decompose).  The field is initialised on the device with the U12 generator
+ * (seed 0x5C24), so create -> run -> gather needs no host upload. */
+
+/* Single process, one slab per GPU on devices 0..ngpus-1, peer access enabled between
+ * neighbours (P:321-323 UVA load/store).  ngpus == 1 is the 1-GPU path. */
+int jacobi_create(int64_t nx, int64_t ny, int64_t nz, int stencil, int ngpus, jacobi_t *out);
+
+/* Single process, `nslabs` slabs on ONE device, all driven by one cooperative launch in which
+ * each slab gets its own group of thread blocks, grid barrier, flags and "peer" pointers into
+ * the other slabs' buffers.  Exercises the complete multi-GPU protocol on one GPU (the
+ * SURVEY.md §4.2 "virtual PE" backend).  1 <= nslabs <= 8. */
+int jacobi_create_virtual(int64_t nx, int64_t ny, int64_t nz, int stencil, int nslabs,
+                          int device, jacobi_t *out);
+
+/* One process per GPU (torchrun): this process owns slab `rank` of `world_size` on `device`.
+ * Before the first run, exchange jacobi_get_ipc_handle() blobs with the neighbours (any
+ * transport; the Python binding uses torch.distributed) and call jacobi_open_peers().
+ * All dist-mode calls that touch the protocol (run, set_mode) are collective over ranks. */
+int jacobi_create_rank(int64_t nx, int64_t ny, int64_t nz, int stencil, int world_size,
+                       int rank, int device, jacobi_t *out);
+int jacobi_ipc_handle_bytes(void);                     /* size of the blob below */
+int jacobi_get_ipc_handle(jacobi_t h, void *out);      /* CUDA IPC handles of this rank's buffers + flags */
+int jacobi_open_peers(jacobi_t h, const void *top_blob, const void *bottom_blob); /* NULL = no neighbour */
+/* NCCL baseline in dist mode: rank 0 creates a 128-byte ncclUniqueId, every rank passes it to
+ * jacobi_nccl_init (collective).  libnccl.so.2 is loaded with dlopen on first use. */
+int jacobi_nccl_unique_id(void *out128);
+int jacobi_nccl_init(jacobi_t h, const void *id128);
+
+/* ---- running ----------------------------------------------------------------------------- */
+/* Advance the field by `iters` Jacobi iterations in the current mode.  Continues from the
+ * current state: run(a); run(b) == run(a+b) bitwise.  run(0) is a no-op.  Blocks until done. */
+int jacobi_run(jacobi_t h, int64_t iters);
+int jacobi_set_mode(jacobi_t h, int mode, int flags);
+/* Tuning knobs (none changes results): "tile_x", "tile_y", "stages", "boundary_ctas",
+ * "ctas" (persistent grid size per slab group, 0 = all co-resident), "schedule"
+ * (-1 auto, 0 linear, 1 lockstep), "timeout_ms" (watchdog, default 20000).  -1 = default. */
+int jacobi_set_param(jacobi_t h, const char *name, int64_t value);
+int jacobi_get_param(jacobi_t h, const char *name, int64_t *value);
+
+/* ---- data movement -------------------------------------------------------------------- */
+/* Set the whole field (boundary included) from a host array of nx*ny*nz doubles; both
+ * device buffers are written.  In dist mode only this rank's slab (+ its halos) is read. */
+int jacobi_scatter(jacobi_t h, const double *in);
+/* Write the current field into a host array of nx*ny*nz doubles.  In dist mode only this
+ * rank's owned planes (and the global boundary planes it holds) are written. */
+int jacobi_gather(jacobi_t h, double *out);
+
+/* ---- introspection ---------------------------------------------------------------------- */
+/* Device time of the last jacobi_run: max over GPUs and, if ms_per_slab != NULL, one entry
+ * per local slab (CUDA events on each GPU's launch stream around the launch(es)). */
+int jacobi_last_time(jacobi_t h, double *ms_max, double *ms_per_slab);
+int jacobi_iterations(jacobi_t h, int64_t *t);          /* global iteration counter */
+int jacobi_num_slabs(jacobi_t h, int *local, int *total);
+/* Plan of local slab `i`: out[0..15] = start, chunk, pitch, plane_elems, tile_x, tile_y,
+ * units_x, units_y, stages, n_top, n_bot, n_interior, ctas, k_planes, smem_bytes, device. */
+int jacobi_describe(jacobi_t h, int i, int64_t *out16);
+const char *jacobi_strerror(int code);
+int jacobi_destroy(jacobi_t h);                         /* NULL-safe */
+
+/* ---- host-only helpers (no GPU needed) ---------------------------------------------------- */
+/* Slab decomposition of the interior outer indices 1..n_out-2 into nslabs chunks: with
+ * q = (n_out-2) / nslabs, r = (n_out-2) % nslabs, slab g owns q + (g < r) planes starting at
+ * global outer index 1 + g*q + min(g, r)  ("divided equally among GPUs"). */
+int jacobi_decompose(int64_t n_out, int nslabs, int slab, int64_t *start, int64_t *chunk);
+/* The thread-block split of P:398-404 (§4.1.2, garbled formula reconstructed in DESIGN.md
+ * reading R11): boundary_TB = TB_total * w_b / (inner + sides * w_b) per side, rounded up,
+ * >= 1 per side with a neighbour, >= 1 interior block if there is interior work.
+ * out[0..2] = n_top, n_bot, n_interior. */
+int jacobi_tb_split(int ctas, int64_t chunk, int has_top, int has_bottom, int64_t units,
+                    int override_per_side, int *out3);
+/* Geometry chosen for a grid: out[0..7] = pitch, plane_elems, tile_x, tile_y, units_x,
+ * units_y, stage_rows, stage_row_doubles.  tile_x/tile_y <= 0 pick defaults. */
+int jacobi_geometry(int64_t nx, int64_t ny, int64_t nz, int stencil, int tile_x, int tile_y,
+                    int64_t *out8);
+int jacobi_version(void);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* JACOBI_B200_H */

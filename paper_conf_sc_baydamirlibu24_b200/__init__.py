@@ -1,0 +1,339 @@
+"""Thin Python binding of libjacobi_b200.so (include/jacobi.h) — argument marshalling only.
+
+Every step of the hot path runs in the CUDA library; this module never computes the stencil
+and has no CPU fallback: if the extension is missing it raises.  Function names mirror the C
+ABI (``jacobi_create``, ``jacobi_run``, ...); ``Jacobi`` is a small convenience wrapper over a
+handle used by tests, ``bench.py`` and ``__graft_entry__``.  PyTorch is used only as plumbing
+(torch.distributed to exchange CUDA IPC handles / the NCCL unique id between ranks).
+"""
+from __future__ import annotations
+
+import ctypes
+import os
+import re
+
+import numpy as np
+
+_HERE = os.path.dirname(os.path.abspath(__file__))
+LIB_PATH = os.path.join(_HERE, "libjacobi_b200.so")
+HEADER_PATH = os.path.join(os.path.dirname(_HERE), "include", "jacobi.h")
+
+JACOBI_OK = 0
+JACOBI_EINVAL = -1
+JACOBI_ENODEV = -2
+JACOBI_ENOPEER = -3
+JACOBI_ENOCOOP = -4
+JACOBI_ENOMEM = -5
+JACOBI_ECUDA = -6
+JACOBI_ETIMEOUT = -7
+JACOBI_ENCCL = -8
+JACOBI_ESTATE = -9
+
+MODE_CPUFREE = 0
+MODE_BASELINE_MEMCPY = 1
+MODE_BASELINE_NCCL = 2
+FLAG_NO_COMPUTE = 1
+FLAG_DROP_SIGNAL = 2
+
+_c = ctypes
+_i64 = _c.c_int64
+_p = _c.c_void_p
+_SIGS = {
+    "jacobi_create": ([_i64, _i64, _i64, _c.c_int, _c.c_int, _c.POINTER(_p)], _c.c_int),
+    "jacobi_create_virtual": ([_i64, _i64, _i64, _c.c_int, _c.c_int, _c.c_int, _c.POINTER(_p)], _c.c_int),
+    "jacobi_create_rank": ([_i64, _i64, _i64, _c.c_int, _c.c_int, _c.c_int, _c.c_int, _c.POINTER(_p)], _c.c_int),
+    "jacobi_ipc_handle_bytes": ([], _c.c_int),
+    "jacobi_get_ipc_handle": ([_p, _p], _c.c_int),
+    "jacobi_open_peers": ([_p, _p, _p], _c.c_int),
+    "jacobi_nccl_unique_id": ([_p], _c.c_int),
+    "jacobi_nccl_init": ([_p, _p], _c.c_int),
+    "jacobi_run": ([_p, _i64], _c.c_int),
+    "jacobi_set_mode": ([_p, _c.c_int, _c.c_int], _c.c_int),
+    "jacobi_set_param": ([_p, _c.c_char_p, _i64], _c.c_int),
+    "jacobi_get_param": ([_p, _c.c_char_p, _c.POINTER(_i64)], _c.c_int),
+    "jacobi_scatter": ([_p, _p], _c.c_int),
+    "jacobi_gather": ([_p, _p], _c.c_int),
+    "jacobi_last_time": ([_p, _c.POINTER(_c.c_double), _c.POINTER(_c.c_double)], _c.c_int),
+    "jacobi_iterations": ([_p, _c.POINTER(_i64)], _c.c_int),
+    "jacobi_num_slabs": ([_p, _c.POINTER(_c.c_int), _c.POINTER(_c.c_int)], _c.c_int),
+    "jacobi_describe": ([_p, _c.c_int, _c.POINTER(_i64)], _c.c_int),
+    "jacobi_strerror": ([_c.c_int], _c.c_char_p),
+    "jacobi_destroy": ([_p], _c.c_int),
+    "jacobi_decompose": ([_i64, _c.c_int, _c.c_int, _c.POINTER(_i64), _c.POINTER(_i64)], _c.c_int),
+    "jacobi_tb_split": ([_c.c_int, _i64, _c.c_int, _c.c_int, _i64, _c.c_int, _c.POINTER(_c.c_int)], _c.c_int),
+    "jacobi_geometry": ([_i64, _i64, _i64, _c.c_int, _c.c_int, _c.c_int, _c.POINTER(_i64)], _c.c_int),
+    "jacobi_version": ([], _c.c_int),
+}
+
+_lib = None
+
+
+class JacobiError(RuntimeError):
+    def __init__(self, code: int, what: str = ""):
+        self.code = int(code)
+        super().__init__(f"{what}: {strerror(code)} ({code})" if what else f"{strerror(code)} ({code})")
+
+
+def lib() -> ctypes.CDLL:
+    """Load the CUDA extension.  Fails loudly if it has not been built (no fallback)."""
+    global _lib
+    if _lib is None:
+        if not os.path.exists(LIB_PATH):
+            raise RuntimeError(f"CUDA extension missing: {LIB_PATH} (run __graft_entry__.build())")
+        L = ctypes.CDLL(LIB_PATH)
+        for name, (args, res) in _SIGS.items():
+            fn = getattr(L, name)
+            fn.argtypes = args
+            fn.restype = res
+        _lib = L
+    return _lib
+
+
+def header_functions() -> list[str]:
+    """Names of every function declared in include/jacobi.h."""
+    with open(HEADER_PATH) as f:
+        src = f.read()
+    return re.findall(r"^\s*(?:int|const char \*)\s*(jacobi_\w+)\s*\(", src, flags=re.M)
+
+
+def strerror(code: int) -> str:
+    return lib().jacobi_strerror(int(code)).decode()
+
+
+def _check(rc: int, what: str) -> None:
+    if rc != JACOBI_OK:
+        raise JacobiError(rc, what)
+
+
+# ---------------------------------------------------------------- C-ABI mirrors
+def jacobi_create(nx, ny, nz, stencil, ngpus) -> int:
+    h = _p()
+    _check(lib().jacobi_create(nx, ny, nz, stencil, ngpus, _c.byref(h)), "jacobi_create")
+    return h.value
+
+
+def jacobi_create_virtual(nx, ny, nz, stencil, nslabs, device=0) -> int:
+    h = _p()
+    _check(lib().jacobi_create_virtual(nx, ny, nz, stencil, nslabs, device, _c.byref(h)), "jacobi_create_virtual")
+    return h.value
+
+
+def jacobi_create_rank(nx, ny, nz, stencil, world_size, rank, device) -> int:
+    h = _p()
+    _check(lib().jacobi_create_rank(nx, ny, nz, stencil, world_size, rank, device, _c.byref(h)),
+           "jacobi_create_rank")
+    return h.value
+
+
+def jacobi_get_ipc_handle(h) -> bytes:
+    n = lib().jacobi_ipc_handle_bytes()
+    buf = _c.create_string_buffer(n)
+    _check(lib().jacobi_get_ipc_handle(h, buf), "jacobi_get_ipc_handle")
+    return buf.raw
+
+
+def jacobi_open_peers(h, top: bytes | None, bottom: bytes | None) -> None:
+    _check(lib().jacobi_open_peers(h, top, bottom), "jacobi_open_peers")
+
+
+def jacobi_nccl_unique_id() -> bytes:
+    buf = _c.create_string_buffer(128)
+    _check(lib().jacobi_nccl_unique_id(buf), "jacobi_nccl_unique_id")
+    return buf.raw
+
+
+def jacobi_nccl_init(h, uid: bytes) -> None:
+    _check(lib().jacobi_nccl_init(h, uid), "jacobi_nccl_init")
+
+
+def jacobi_run(h, iters: int) -> None:
+    _check(lib().jacobi_run(h, int(iters)), "jacobi_run")
+
+
+def jacobi_set_mode(h, mode: int, flags: int = 0) -> None:
+    _check(lib().jacobi_set_mode(h, int(mode), int(flags)), "jacobi_set_mode")
+
+
+def jacobi_set_param(h, name: str, value: int) -> None:
+    _check(lib().jacobi_set_param(h, name.encode(), int(value)), f"jacobi_set_param({name})")
+
+
+def jacobi_get_param(h, name: str) -> int:
+    v = _i64()
+    _check(lib().jacobi_get_param(h, name.encode(), _c.byref(v)), f"jacobi_get_param({name})")
+    return v.value
+
+
+def _host_ptr(a: np.ndarray, n: int, writable: bool) -> int:
+    if not isinstance(a, np.ndarray) or a.dtype != np.float64 or not a.flags["C_CONTIGUOUS"] or a.size != n:
+        raise ValueError(f"expected a C-contiguous float64 array of {n} elements")
+    if writable and not a.flags["WRITEABLE"]:
+        raise ValueError("output array is read-only")
+    return a.ctypes.data
+
+
+def jacobi_scatter(h, field: np.ndarray, n: int) -> None:
+    _check(lib().jacobi_scatter(h, _host_ptr(field, n, False)), "jacobi_scatter")
+
+
+def jacobi_gather(h, out: np.ndarray, n: int) -> None:
+    _check(lib().jacobi_gather(h, _host_ptr(out, n, True)), "jacobi_gather")
+
+
+def jacobi_scatter_ptr(h, ptr: int) -> None:
+    _check(lib().jacobi_scatter(h, _p(ptr)), "jacobi_scatter")
+
+
+def jacobi_gather_ptr(h, ptr: int) -> None:
+    _check(lib().jacobi_gather(h, _p(ptr)), "jacobi_gather")
+
+
+def jacobi_last_time(h, nslabs: int):
+    mx = _c.c_double()
+    per = (_c.c_double * max(nslabs, 1))()
+    _check(lib().jacobi_last_time(h, _c.byref(mx), per), "jacobi_last_time")
+    return mx.value, list(per)[:nslabs]
+
+
+def jacobi_iterations(h) -> int:
+    t = _i64()
+    _check(lib().jacobi_iterations(h, _c.byref(t)), "jacobi_iterations")
+    return t.value
+
+
+def jacobi_num_slabs(h):
+    a, b = _c.c_int(), _c.c_int()
+    _check(lib().jacobi_num_slabs(h, _c.byref(a), _c.byref(b)), "jacobi_num_slabs")
+    return a.value, b.value
+
+
+DESCRIBE_KEYS = ("start", "chunk", "pitch", "plane_elems", "tile_x", "tile_y", "units_x", "units_y",
+                 "stages", "n_top", "n_bot", "n_interior", "ctas", "k_planes", "smem_bytes", "device")
+
+
+def jacobi_describe(h, i: int) -> dict:
+    o = (_i64 * 16)()
+    _check(lib().jacobi_describe(h, int(i), o), "jacobi_describe")
+    return dict(zip(DESCRIBE_KEYS, list(o)))
+
+
+def jacobi_destroy(h) -> None:
+    _check(lib().jacobi_destroy(h), "jacobi_destroy")
+
+
+def jacobi_decompose(n_out: int, nslabs: int, slab: int):
+    s, c = _i64(), _i64()
+    _check(lib().jacobi_decompose(n_out, nslabs, slab, _c.byref(s), _c.byref(c)), "jacobi_decompose")
+    return s.value, c.value
+
+
+def jacobi_tb_split(ctas, chunk, has_top, has_bottom, units, override_per_side=0):
+    o = (_c.c_int * 3)()
+    _check(lib().jacobi_tb_split(ctas, chunk, int(has_top), int(has_bottom), units, override_per_side, o),
+           "jacobi_tb_split")
+    return tuple(o)
+
+
+GEOMETRY_KEYS = ("pitch", "plane_elems", "tile_x", "tile_y", "units_x", "units_y", "stage_rows", "stage_row_doubles")
+
+
+def jacobi_geometry(nx, ny, nz, stencil, tile_x=0, tile_y=0) -> dict:
+    o = (_i64 * 8)()
+    _check(lib().jacobi_geometry(nx, ny, nz, stencil, tile_x, tile_y, o), "jacobi_geometry")
+    return dict(zip(GEOMETRY_KEYS, list(o)))
+
+
+def jacobi_version() -> int:
+    return lib().jacobi_version()
+
+
+# ---------------------------------------------------------------- convenience wrapper
+class Jacobi:
+    """One handle of the library.  shape = (nz, ny, nx) or (ny, nx) including the boundary."""
+
+    def __init__(self, shape, ngpus: int = 1, virtual: int = 0, device: int = 0, dist=None):
+        shape = tuple(int(s) for s in shape)
+        if len(shape) == 2:
+            shape = (1,) + shape
+        self.shape = shape
+        nz, ny, nx = shape
+        self.nx, self.ny, self.nz = nx, ny, nz
+        self.stencil = 5 if nz == 1 else 7
+        self.n = nx * ny * nz
+        if dist is not None:
+            rank, world = dist
+            self.h = jacobi_create_rank(nx, ny, nz, self.stencil, world, rank, device)
+        elif virtual:
+            self.h = jacobi_create_virtual(nx, ny, nz, self.stencil, virtual, device)
+        else:
+            self.h = jacobi_create(nx, ny, nz, self.stencil, ngpus)
+        self.local_slabs, self.total_slabs = jacobi_num_slabs(self.h)
+
+    def run(self, iters: int) -> "Jacobi":
+        jacobi_run(self.h, iters)
+        return self
+
+    def set_mode(self, mode: int, flags: int = 0) -> "Jacobi":
+        jacobi_set_mode(self.h, mode, flags)
+        return self
+
+    def set_param(self, name: str, value: int) -> "Jacobi":
+        jacobi_set_param(self.h, name, value)
+        return self
+
+    def scatter(self, field: np.ndarray) -> "Jacobi":
+        a = np.ascontiguousarray(field, dtype=np.float64)
+        jacobi_scatter(self.h, a.reshape(-1), self.n)
+        return self
+
+    def gather(self, out: np.ndarray | None = None) -> np.ndarray:
+        if out is None:
+            out = np.empty(self.shape, dtype=np.float64)
+        jacobi_gather(self.h, out.reshape(-1), self.n)
+        return out if self.nz > 1 else out.reshape(self.ny, self.nx)
+
+    def last_time_ms(self) -> float:
+        return jacobi_last_time(self.h, self.local_slabs)[0]
+
+    @property
+    def iterations(self) -> int:
+        return jacobi_iterations(self.h)
+
+    def describe(self, i: int = 0) -> dict:
+        return jacobi_describe(self.h, i)
+
+    def close(self) -> None:
+        if getattr(self, "h", None):
+            jacobi_destroy(self.h)
+            self.h = None
+
+    def __enter__(self):
+        return self
+
+    def __exit__(self, *a):
+        self.close()
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+
+def exchange_peers(j: Jacobi, group=None, nccl: bool = True) -> None:
+    """Dist mode plumbing: all-gather every rank's IPC blob over torch.distributed, attach the
+    neighbours, and (optionally) set up the NCCL communicator of the baseline."""
+    import torch.distributed as dist
+
+    blob = jacobi_get_ipc_handle(j.h)
+    world = dist.get_world_size(group)
+    rank = dist.get_rank(group)
+    blobs = [None] * world
+    dist.all_gather_object(blobs, blob, group=group)
+    top = blobs[rank - 1] if rank > 0 else None
+    bot = blobs[rank + 1] if rank < world - 1 else None
+    jacobi_open_peers(j.h, top, bot)
+    if nccl:
+        uid = [jacobi_nccl_unique_id() if rank == 0 else None]
+        dist.broadcast_object_list(uid, src=0, group=group)
+        jacobi_nccl_init(j.h, uid[0])

@@ -1,0 +1,83 @@
+// jacobi_internal.h — structures shared by the host runtime (runtime.cu, plan.cpp) and the
+// device kernels (kernels.cu).  Product code only; nothing here is shared with oracle/.
+#pragma once
+#include <stdint.h>
+
+#define JB_MAX_SLABS 8          // slabs per launch (virtual mode)
+#define JB_NCW 8                // consumer warps per CTA
+#define JB_NC (JB_NCW * 32)     // consumer threads per CTA
+#define JB_THREADS (JB_NC + 32) // + one producer warp (bulk-copy issue)
+#define JB_MAX_STAGES 32
+#define JB_SMEM_DEFAULT 232448  // B200 opt-in dynamic shared memory per block (227 KB)
+
+// Grid geometry in HBM and the tile shape of the march.
+//   element (x, y, z) of slab plane p lives at  buf + p*plane_elems + y*pitch + (x + 3)
+//   (2D: plane p IS row y = start-1+p, so there is no y*pitch term).  The +3 shift makes the
+//   first interior cell x = 1 16-byte aligned, so 128-bit loads/stores never straddle.
+struct JbGeom {
+  int64_t nx, ny, nz;
+  int64_t pitch;        // doubles per row: round_up(nx + 3, 4)
+  int64_t plane_elems;  // 2D: pitch; 3D: ny * pitch
+  int32_t dim;          // 2 or 3
+  int32_t tx;           // x tile width (power of two >= 8): cells x0 .. x0+tx-1, x0 = 1 + ux*tx
+  int32_t txp_shift;    // log2(tx / 2)
+  int32_t ty;           // rows per tile (3D), 1 in 2D
+  int32_t rh;           // rows per smem stage: 1 (2D) or ty + 2 (3D, y halo rows)
+  int32_t ws;           // smem row stride in doubles: tx + 4
+  int32_t units_x, units_y, units;
+  int32_t stages;       // ring depth
+  int32_t stage_doubles;// rh * ws
+  int32_t pad0;
+};
+
+struct JbSlab {
+  double *buf[2];                 // local slab, planes 0..chunk+1 (0 and chunk+1 are halos)
+  double *peer_top[2];            // top neighbour's plane chunk_top+1 (its bottom halo), per parity
+  double *peer_bot[2];            // bottom neighbour's plane 0 (its top halo), per parity
+  unsigned long long *flag_in_top;   // local; set by the top neighbour to the iteration whose halo it delivered
+  unsigned long long *flag_in_bot;   // local; set by the bottom neighbour
+  unsigned long long *flag_out_top;  // = top neighbour's flag_in_bot
+  unsigned long long *flag_out_bot;  // = bottom neighbour's flag_in_top
+  unsigned int *side_ctr;            // local [2]: boundary CTAs done per side (reset each run)
+  unsigned long long *barrier;       // local grid-barrier counter (reset each run)
+  int64_t chunk;
+  int32_t cta_begin, cta_count;
+  int32_t n_top, n_bot;              // boundary CTAs per side (0: no neighbour on that side)
+  int32_t k_planes;                  // lockstep plane ranges for the interior (0: linear schedule)
+  int32_t slab_id;                   // global slab index g
+};
+
+struct JbParams {
+  JbGeom g;
+  JbSlab s[JB_MAX_SLABS];
+  int32_t nslabs;
+  int32_t flags;
+  int64_t t0;       // global iteration counter at launch
+  int64_t iters;
+  unsigned long long timeout_ns;
+  int *status;      // [0] error code (0 ok), [1] abort flag
+};
+
+// Per-slab control block in device memory (one allocation, IPC-exportable).
+struct JbCtrl {
+  unsigned long long flag_in[2];   // [0] top, [1] bottom
+  unsigned long long barrier;
+  unsigned int side_ctr[2];
+  int status[2];
+  unsigned long long pad[26];      // 256 B total
+};
+
+// ---- host-side planning (plan.cpp) -----------------------------------------------------
+namespace jbplan {
+int64_t pow2ceil(int64_t v);
+void decompose(int64_t n_out, int nslabs, int slab, int64_t *start, int64_t *chunk);
+// Fill geometry for tile sizes (tile_x/tile_y <= 0: defaults); returns 0 or -1.
+int geometry(int64_t nx, int64_t ny, int64_t nz, int dim, int tile_x, int tile_y, int smem_bytes,
+             int stages_req, JbGeom *g);
+void tb_split(int ctas, int64_t inner_planes, int has_top, int has_bot, int64_t units,
+              int override_per_side, int *n_top, int *n_bot, int *n_int);
+// Choose ty (3D) maximising the lockstep utilisation of `n_int` interior CTAs.
+int choose_ty(int64_t ny, int units_x, int n_int, int smem_bytes, int ws);
+int lockstep_k(int units, int n_int, int64_t inner_planes);
+size_t smem_bytes(const JbGeom &g);
+}  // namespace jbplan

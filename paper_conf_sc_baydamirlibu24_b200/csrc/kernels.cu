@@ -1,0 +1,540 @@
+// kernels.cu — sm_100a device code of the CPU-Free Jacobi library.
+//
+// jb_sweep<DIM, NOCOMP, PERSIST> is the whole hot path:
+//   PERSIST = true : the CPU-Free persistent kernel of PAPER.md Listing 4.1.  The time
+//                    loop runs on the device (§3.1.1); thread blocks are specialised
+//                    (§3.1.3): TOP/BOTTOM boundary CTAs wait on a flag from
+//                    their neighbour ("signal_wait_until ... compared to the
+//                    current iteration"), compute the edge plane, store it into the local next
+//                    buffer AND straight into the neighbour GPU's halo through a peer pointer
+//                    (§3.1.4), then set the neighbour's flag to the next
+//                    iteration; INTERIOR CTAs stream the bulk;
+//                    a device-side grid barrier closes the iteration.
+//   PERSIST = false: the discrete one-iteration kernel of the CPU-controlled baseline
+//                    (Listing 2.1a) — same tile code, launched once per iteration.
+//
+// B200 design: one CTA per SM; inside it one producer warp streams planes of a
+// tile from HBM into a shared-memory ring with 1D bulk copies (cp.async.bulk, the TMA engine)
+// completing on mbarriers, and 8 consumer warps march the tile along the outer axis (2.5D), so
+// every cell is read from HBM once and written once per iteration (16 B/cell).  Arithmetic is
+// fp64 in the oracle's order, compiled with -fmad=false (no contraction).
+#include <cuda_runtime.h>
+#include <stdint.h>
+
+#include "../../include/jacobi.h"
+#include "jacobi_internal.h"
+
+namespace {
+
+constexpr double kC6 = 0x1.5555555555555p-3;  // fl(1/6), reading R3
+constexpr unsigned long long kGolden = 0x9E3779B97F4A7C15ull;
+
+enum Role { ROLE_INT = 0, ROLE_TOP = 1, ROLE_BOT = 2 };
+
+// ---------------------------------------------------------------- PTX helpers
+__device__ __forceinline__ uint32_t sptr(const void *p) {
+  return static_cast<uint32_t>(__cvta_generic_to_shared(p));
+}
+__device__ __forceinline__ void mbar_init(uint64_t *b, uint32_t count) {
+  asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(sptr(b)), "r"(count) : "memory");
+}
+__device__ __forceinline__ void mbar_expect_tx(uint64_t *b, uint32_t bytes) {
+  asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(sptr(b)), "r"(bytes)
+               : "memory");
+}
+__device__ __forceinline__ void mbar_arrive(uint64_t *b) {
+  asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(sptr(b)) : "memory");
+}
+__device__ __forceinline__ bool mbar_try_wait(uint64_t *b, uint32_t parity) {
+  uint32_t ok;
+  asm volatile(
+      "{\n .reg .pred p;\n mbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2;\n"
+      " selp.u32 %0, 1, 0, p;\n}\n"
+      : "=r"(ok)
+      : "r"(sptr(b)), "r"(parity)
+      : "memory");
+  return ok != 0;
+}
+__device__ __forceinline__ void mbar_wait(uint64_t *b, uint32_t parity) {
+  while (!mbar_try_wait(b, parity)) {
+  }
+}
+// 1D bulk copy global -> shared (TMA engine), completion counted in bytes on an mbarrier.
+__device__ __forceinline__ void bulk_g2s(void *dst, const void *src, uint32_t bytes, uint64_t *bar) {
+  asm volatile(
+      "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(
+          sptr(dst)),
+      "l"(src), "r"(bytes), "r"(sptr(bar))
+      : "memory");
+}
+__device__ __forceinline__ void fence_proxy_async_global() {
+  asm volatile("fence.proxy.async.global;" ::: "memory");
+}
+__device__ __forceinline__ void fence_mbar_init() {
+  asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+}
+__device__ __forceinline__ void fence_acq_rel_sys() { asm volatile("fence.acq_rel.sys;" ::: "memory"); }
+__device__ __forceinline__ unsigned long long ld_acquire_sys(const unsigned long long *p) {
+  unsigned long long v;
+  asm volatile("ld.acquire.sys.global.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
+  return v;
+}
+__device__ __forceinline__ unsigned long long ld_acquire_gpu(const unsigned long long *p) {
+  unsigned long long v;
+  asm volatile("ld.acquire.gpu.global.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
+  return v;
+}
+__device__ __forceinline__ void st_release_sys(unsigned long long *p, unsigned long long v) {
+  asm volatile("st.release.sys.global.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
+}
+__device__ __forceinline__ void red_release_gpu_add(unsigned long long *p, unsigned long long v) {
+  asm volatile("red.release.gpu.global.add.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
+}
+__device__ __forceinline__ unsigned int atom_acq_rel_gpu_add(unsigned int *p, unsigned int v) {
+  unsigned int old;
+  asm volatile("atom.acq_rel.gpu.global.add.u32 %0, [%1], %2;" : "=r"(old) : "l"(p), "r"(v) : "memory");
+  return old;
+}
+__device__ __forceinline__ unsigned long long globaltimer() {
+  unsigned long long t;
+  asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+  return t;
+}
+__device__ __forceinline__ void named_bar_consumers() {
+  asm volatile("bar.sync 1, %0;" ::"r"(JB_NC) : "memory");
+}
+
+// Spin until *p >= target (acquire at sys or gpu scope).  Watchdog: after timeout_ns set
+// status = ETIMEOUT and the abort flag; also gives up once another CTA raised abort.
+template <bool SYS>
+__device__ bool wait_geq(const unsigned long long *p, unsigned long long target, const JbParams &P) {
+  auto ld = [&]() { return SYS ? ld_acquire_sys(p) : ld_acquire_gpu(p); };
+  if (ld() >= target) return true;
+  const unsigned long long t_start = globaltimer();
+  uint32_t n = 0;
+  volatile int *abort_flag = P.status + 1;
+  while (true) {
+    if (ld() >= target) return true;
+    if ((++n & 127u) == 0) {
+      if (*abort_flag) return false;
+      if (globaltimer() - t_start > P.timeout_ns) {
+        atomicCAS(P.status, 0, JACOBI_ETIMEOUT);
+        atomicExch(P.status + 1, 1);
+        return false;
+      }
+    }
+  }
+}
+
+// ---------------------------------------------------------------- work schedule
+struct Run {
+  int32_t unit;
+  int64_t p0, p1;  // planes computed: p0..p1 (inclusive), marched in order
+};
+
+// Deterministic run list of one CTA for one iteration; producer and consumers enumerate it
+// identically.  kind: 0 none, 1 linear range over (unit, plane) pairs in unit-major order,
+// 2 lockstep (one unit, one plane range), 3 boundary (units ub..ue-1, one plane each).
+struct Sched {
+  int kind;
+  int32_t units;
+  int64_t w, we, npl, lo;
+  int32_t ub, ue;
+  int64_t plane;
+  __device__ bool next(Run &r) {
+    if (kind == 1) {
+      if (w >= we) return false;
+      const int64_t u = w / npl;
+      const int64_t e = min(we, (u + 1) * npl);
+      r.unit = (int32_t)u;
+      r.p0 = lo + (w - u * npl);
+      r.p1 = lo + (e - 1 - u * npl);
+      w = e;
+      return true;
+    }
+    if (kind == 2) {
+      kind = 0;
+      r.unit = ub;
+      r.p0 = w;
+      r.p1 = we;
+      return true;
+    }
+    if (kind == 3) {
+      if (ub >= ue) return false;
+      r.unit = ub++;
+      r.p0 = r.p1 = plane;
+      return true;
+    }
+    return false;
+  }
+};
+
+__device__ Sched make_sched(const JbGeom &g, const JbSlab &S, int role, int ridx, int rcount) {
+  Sched s;
+  s.kind = 0;
+  s.units = g.units;
+  s.w = s.we = s.npl = s.lo = 0;
+  s.ub = s.ue = 0;
+  s.plane = 0;
+  if (role == ROLE_TOP || role == ROLE_BOT) {
+    s.kind = 3;
+    s.ub = (int32_t)((int64_t)g.units * ridx / rcount);
+    s.ue = (int32_t)((int64_t)g.units * (ridx + 1) / rcount);
+    s.plane = role == ROLE_TOP ? 1 : S.chunk;
+    return s;
+  }
+  const int64_t lo = S.n_top ? 2 : 1;
+  const int64_t hi = S.n_bot ? S.chunk - 1 : S.chunk;
+  const int64_t npl = hi - lo + 1;
+  if (npl <= 0 || rcount <= 0) return s;
+  if (S.k_planes > 0) {
+    const int K = S.k_planes;
+    if (ridx >= g.units * K) return s;
+    const int u = ridx % g.units, kr = ridx / g.units;
+    const int64_t a = lo + npl * kr / K, b = lo + npl * (kr + 1) / K - 1;
+    if (b < a) return s;
+    s.kind = 2;
+    s.ub = u;
+    s.w = a;
+    s.we = b;
+    return s;
+  }
+  const int64_t W = (int64_t)g.units * npl;
+  s.kind = 1;
+  s.npl = npl;
+  s.lo = lo;
+  s.w = W * ridx / rcount;
+  s.we = W * (ridx + 1) / rcount;
+  return s;
+}
+
+// Ring position q -> slot / parity.
+struct Ring {
+  uint64_t *full, *empty;
+  double *stages;
+  int S;
+  __device__ __forceinline__ int slot(uint32_t q) const { return (int)(q % (uint32_t)S); }
+  __device__ __forceinline__ uint32_t parity(uint32_t q) const { return (q / (uint32_t)S) & 1u; }
+};
+
+// ---------------------------------------------------------------- producer
+// Load planes pf..pl of tile `unit` from `cur` into consecutive ring stages starting at q.
+__device__ __forceinline__ void produce_planes(const JbGeom &g, const double *cur, int32_t unit,
+                                               int64_t pf, int64_t pl, uint32_t &q, const Ring &R,
+                                               int lane) {
+  const int ux = unit % g.units_x, uy = unit / g.units_x;
+  const int64_t xs = 2 + (int64_t)ux * g.tx;
+  const int64_t xe = min(xs + g.tx + 4, g.pitch);
+  const uint32_t row_bytes = (uint32_t)((xe - xs) * 8);
+  int64_t ya = 0;
+  int nrows = 1;
+  if (g.dim == 3) {
+    ya = (int64_t)uy * g.ty;  // = y0 - 1
+    const int64_t yb = min(ya + 1 + g.ty, g.ny - 1);
+    nrows = (int)(yb - ya + 1);
+  }
+  for (int64_t p = pf; p <= pl; ++p, ++q) {
+    const int s = R.slot(q);
+    if (lane == 0) {
+      if (q >= (uint32_t)R.S) mbar_wait(&R.empty[s], R.parity(q) ^ 1u);
+      mbar_expect_tx(&R.full[s], row_bytes * (uint32_t)nrows);
+    }
+    __syncwarp();
+    if (lane < nrows) {
+      const double *src = cur + p * g.plane_elems + xs + (g.dim == 3 ? (ya + lane) * g.pitch : 0);
+      double *dst = R.stages + (size_t)s * g.stage_doubles + (size_t)lane * g.ws;
+      bulk_g2s(dst, src, row_bytes, &R.full[s]);
+    }
+  }
+}
+
+// ---------------------------------------------------------------- consumers
+__device__ __forceinline__ double2 lds2(const double *p) { return *reinterpret_cast<const double2 *>(p); }
+
+template <int DIM, bool NOCOMP>
+__device__ __forceinline__ void compute_plane(const JbGeom &g, int32_t unit, int64_t p, const double *sm,
+                                              const double *sc, const double *sp, double *nxt,
+                                              double *remote, int ctid) {
+  const int ux = unit % g.units_x, uy = unit / g.units_x;
+  const int64_t x0 = 1 + (int64_t)ux * g.tx;
+  const int vx = (int)min((int64_t)g.tx, g.nx - 1 - x0);  // valid cells in x
+  int64_t y0 = 0;
+  int vy = 1;
+  if (DIM == 3) {
+    y0 = 1 + (int64_t)uy * g.ty;
+    vy = (int)min((int64_t)g.ty, g.ny - 1 - y0);
+  }
+  const int sh = g.txp_shift;
+  const int txp_mask = (1 << sh) - 1;
+  const int total = vy << sh;
+  double *dst_plane = nxt ? nxt + p * g.plane_elems : nullptr;
+  for (int k = ctid; k < total; k += JB_NC) {
+    const int r = k >> sh, kk = k & txp_mask;
+    if (2 * kk >= vx) continue;
+    const int j = 2 + 2 * kk;
+    const int row = (DIM == 3) ? (r + 1) * g.ws : 0;
+    const double *c = sc + row;
+    double o0, o1;
+    if (NOCOMP) {
+      const double2 cc = lds2(c + j);
+      o0 = cc.x;
+      o1 = cc.y;
+    } else if (DIM == 2) {
+      const double2 cc = lds2(c + j);
+      const double w = c[j - 1], e = c[j + 2];
+      const double2 n = lds2(sp + j);  // y+1
+      const double2 s = lds2(sm + j);  // y-1
+      o0 = 0.25 * (((cc.y + w) + n.x) + s.x);
+      o1 = 0.25 * (((e + cc.x) + n.y) + s.y);
+    } else {
+      const double2 cc = lds2(c + j);
+      const double w = c[j - 1], e = c[j + 2];
+      const double2 n = lds2(c + g.ws + j);  // y+1
+      const double2 s = lds2(c - g.ws + j);  // y-1
+      const double2 u = lds2(sp + row + j);  // z+1
+      const double2 d = lds2(sm + row + j);  // z-1
+      o0 = kC6 * (((((cc.y + w) + n.x) + s.x) + u.x) + d.x);
+      o1 = kC6 * (((((e + cc.x) + n.y) + s.y) + u.y) + d.y);
+    }
+    const int64_t off = (DIM == 3 ? (y0 + r) * g.pitch : 0) + 3 + x0 + 2 * kk;
+    const bool pair = (2 * kk + 1) < vx;
+    if (dst_plane) {
+      if (pair) *reinterpret_cast<double2 *>(dst_plane + off) = make_double2(o0, o1);
+      else dst_plane[off] = o0;
+    }
+    if (remote) {
+      if (pair) *reinterpret_cast<double2 *>(remote + off) = make_double2(o0, o1);
+      else remote[off] = o0;
+    }
+  }
+}
+
+__device__ __forceinline__ void release_stage(const Ring &R, uint32_t q, int lane) {
+  __syncwarp();
+  if (lane == 0) mbar_arrive(&R.empty[R.slot(q)]);
+}
+
+// ---------------------------------------------------------------- the kernel
+template <int DIM, bool NOCOMP, bool PERSIST>
+__global__ void __launch_bounds__(JB_THREADS, 1) jb_sweep(const __grid_constant__ JbParams P) {
+  extern __shared__ __align__(128) unsigned char smem[];
+  __shared__ int s_abort;
+  const JbGeom &g = P.g;
+  Ring R;
+  R.S = g.stages;
+  R.full = reinterpret_cast<uint64_t *>(smem);
+  R.empty = R.full + R.S;
+  R.stages = reinterpret_cast<double *>(smem + ((2 * R.S * 8 + 127) & ~127));
+
+  int si = 0;
+  while (si + 1 < P.nslabs && (int)blockIdx.x >= P.s[si + 1].cta_begin) ++si;
+  const JbSlab &SL = P.s[si];
+  const int c = (int)blockIdx.x - SL.cta_begin;
+  int role, ridx, rcount;
+  if (c < SL.n_top) {
+    role = ROLE_TOP; ridx = c; rcount = SL.n_top;
+  } else if (c < SL.n_top + SL.n_bot) {
+    role = ROLE_BOT; ridx = c - SL.n_top; rcount = SL.n_bot;
+  } else {
+    role = ROLE_INT; ridx = c - SL.n_top - SL.n_bot; rcount = SL.cta_count - SL.n_top - SL.n_bot;
+  }
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const bool producer = warp == JB_NCW;
+  const int ctid = threadIdx.x;  // consumer thread id (valid when !producer)
+
+  if (threadIdx.x == 0) {
+    for (int i = 0; i < R.S; ++i) {
+      mbar_init(&R.full[i], 1);
+      mbar_init(&R.empty[i], JB_NCW);
+    }
+    fence_mbar_init();
+    s_abort = 0;
+  }
+  __syncthreads();
+
+  const Sched sched0 = make_sched(g, SL, role, ridx, rcount);
+  const bool drop_signal = (P.flags & JACOBI_FLAG_DROP_SIGNAL) && SL.slab_id == 0;
+  const int side = role == ROLE_TOP ? 0 : 1;
+  uint32_t q = 0;  // ring position (producer and consumers advance it identically)
+
+  for (int64_t t = 0; t < P.iters; ++t) {
+    const int64_t tg = P.t0 + t;
+    const double *cur = SL.buf[tg & 1];
+    double *nxt = SL.buf[(tg + 1) & 1];
+    double *remote = nullptr;
+    if (role == ROLE_TOP) remote = SL.peer_top[(tg + 1) & 1];
+    if (role == ROLE_BOT) remote = SL.peer_bot[(tg + 1) & 1];
+    const bool active = !(NOCOMP && role == ROLE_INT);
+    Sched sched = sched0;
+    Run run;
+
+    if (producer) {
+      if (lane == 0) {
+        fence_proxy_async_global();
+        // wait until the neighbour committed the halo of the previous time step.
+        if (PERSIST && role != ROLE_INT) {
+          const unsigned long long *f = role == ROLE_TOP ? SL.flag_in_top : SL.flag_in_bot;
+          wait_geq<true>(f, (unsigned long long)tg, P);
+          fence_proxy_async_global();
+        }
+      }
+      __syncwarp();
+      if (active) {
+        while (sched.next(run)) {
+          if (NOCOMP) produce_planes(g, cur, run.unit, run.p0, run.p1, q, R, lane);
+          else produce_planes(g, cur, run.unit, run.p0 - 1, run.p1 + 1, q, R, lane);
+        }
+      }
+    } else {
+      if (active) {
+        while (sched.next(run)) {
+          const int64_t L = run.p1 - run.p0 + 1;
+          if (NOCOMP) {
+            for (int64_t i = 0; i < L; ++i, ++q) {
+              mbar_wait(&R.full[R.slot(q)], R.parity(q));
+              const double *sc = R.stages + (size_t)R.slot(q) * g.stage_doubles;
+              compute_plane<DIM, true>(g, run.unit, run.p0 + i, sc, sc, sc, nullptr, remote, ctid);
+              release_stage(R, q, lane);
+            }
+            continue;
+          }
+          mbar_wait(&R.full[R.slot(q)], R.parity(q));
+          mbar_wait(&R.full[R.slot(q + 1)], R.parity(q + 1));
+          for (int64_t i = 0; i < L; ++i) {
+            const uint32_t qm = q + (uint32_t)i, qc = qm + 1, qp = qm + 2;
+            mbar_wait(&R.full[R.slot(qp)], R.parity(qp));
+            const double *sm = R.stages + (size_t)R.slot(qm) * g.stage_doubles;
+            const double *sc = R.stages + (size_t)R.slot(qc) * g.stage_doubles;
+            const double *sp = R.stages + (size_t)R.slot(qp) * g.stage_doubles;
+            compute_plane<DIM, false>(g, run.unit, run.p0 + i, sm, sc, sp, nxt, remote, ctid);
+            release_stage(R, qm, lane);
+          }
+          release_stage(R, q + (uint32_t)L, lane);
+          release_stage(R, q + (uint32_t)L + 1, lane);
+          q += (uint32_t)L + 2;
+        }
+      }
+      // Our generic-proxy stores must be ordered before later bulk (async-proxy) reads.
+      fence_proxy_async_global();
+      // P:364-365 / P:394: signal the neighbour that the halo of iteration tg+1 is in place.
+      if (PERSIST && role != ROLE_INT) {
+        named_bar_consumers();
+        if (ctid == 0 && !drop_signal) {
+          fence_acq_rel_sys();
+          const unsigned int old = atom_acq_rel_gpu_add(&SL.side_ctr[side], 1u);
+          if (old == (unsigned int)(rcount * (t + 1) - 1)) {
+            fence_acq_rel_sys();
+            st_release_sys(role == ROLE_TOP ? SL.flag_out_top : SL.flag_out_bot,
+                           (unsigned long long)(tg + 1));
+          }
+        }
+      }
+    }
+    if (!PERSIST) break;
+
+    // Device-side grid barrier of this slab's CTAs (P:372 grid.sync()).
+    __syncthreads();
+    if (threadIdx.x == 0) {
+      red_release_gpu_add(SL.barrier, 1ull);
+      const bool ok = wait_geq<false>(SL.barrier, (unsigned long long)SL.cta_count * (t + 1), P);
+      s_abort = (!ok || *(volatile int *)(P.status + 1)) ? 1 : 0;
+    }
+    __syncthreads();
+    if (s_abort) return;
+  }
+
+  // End of run: wait for the neighbour's last halo so no remote store is still in flight into
+  // this GPU's buffers when the kernel (and the host's view of the run) completes.
+  if (PERSIST && producer && lane == 0 && role != ROLE_INT && P.iters > 0) {
+    const unsigned long long *f = role == ROLE_TOP ? SL.flag_in_top : SL.flag_in_bot;
+    wait_geq<true>(f, (unsigned long long)(P.t0 + P.iters), P);
+  }
+}
+
+// ---------------------------------------------------------------- init / utility kernels
+__device__ __forceinline__ double u12_value(unsigned long long idx, unsigned long long seed) {
+  unsigned long long z = seed + (idx + 1ull) * kGolden;
+  z = (z ^ (z >> 30)) * 0xBF58476D1CE4E5B9ull;
+  z = (z ^ (z >> 27)) * 0x94D049BB133111EBull;
+  z = z ^ (z >> 31);
+  return __longlong_as_double((long long)(0x3FF0000000000000ull | (z >> 12)));
+}
+
+// Fill planes 0..nplanes-1 of a slab whose plane 0 is global outer index z_first with U12.
+__global__ void jb_init_u12(double *b0, double *b1, int64_t nplanes, JbGeom g, int64_t z_first,
+                            unsigned long long seed) {
+  const int64_t n = nplanes * g.plane_elems;
+  for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n;
+       i += (int64_t)gridDim.x * blockDim.x) {
+    const int64_t p = i / g.plane_elems, rem = i - p * g.plane_elems;
+    int64_t y, pos, idx = -1;
+    if (g.dim == 2) {
+      y = z_first + p;
+      pos = rem;
+      const int64_t x = pos - 3;
+      if (x >= 0 && x < g.nx) idx = y * g.nx + x;
+    } else {
+      y = rem / g.pitch;
+      pos = rem - y * g.pitch;
+      const int64_t x = pos - 3;
+      if (x >= 0 && x < g.nx) idx = ((z_first + p) * g.ny + y) * g.nx + x;
+    }
+    const double v = idx >= 0 ? u12_value((unsigned long long)idx, seed) : 0.0;
+    b0[i] = v;
+    if (b1) b1[i] = v;
+  }
+}
+
+__global__ void jb_flag_max(unsigned long long *flags, int n, unsigned long long v) {
+  if (threadIdx.x < n) atomicMax(flags + threadIdx.x, v);
+}
+
+template <int DIM, bool NOCOMP, bool PERSIST>
+const void *kfn() {
+  return reinterpret_cast<const void *>(&jb_sweep<DIM, NOCOMP, PERSIST>);
+}
+
+const void *sweep_fn(int dim, bool nocomp, bool persist) {
+  if (dim == 2) {
+    if (persist) return nocomp ? kfn<2, true, true>() : kfn<2, false, true>();
+    return nocomp ? kfn<2, true, false>() : kfn<2, false, false>();
+  }
+  if (persist) return nocomp ? kfn<3, true, true>() : kfn<3, false, true>();
+  return nocomp ? kfn<3, true, false>() : kfn<3, false, false>();
+}
+
+}  // namespace
+
+// ---------------------------------------------------------------- host-side launchers
+namespace jbk {
+
+cudaError_t prepare(int dim, bool nocomp, bool persist, size_t smem) {
+  return cudaFuncSetAttribute(sweep_fn(dim, nocomp, persist), cudaFuncAttributeMaxDynamicSharedMemorySize,
+                              (int)smem);
+}
+
+cudaError_t occupancy(int dim, bool nocomp, bool persist, size_t smem, int *blocks_per_sm) {
+  return cudaOccupancyMaxActiveBlocksPerMultiprocessor(blocks_per_sm, sweep_fn(dim, nocomp, persist),
+                                                       JB_THREADS, smem);
+}
+
+cudaError_t launch_sweep(const JbParams &p, bool nocomp, bool persist, int grid, size_t smem,
+                         cudaStream_t st) {
+  void *args[] = {const_cast<JbParams *>(&p)};
+  const void *fn = sweep_fn(p.g.dim, nocomp, persist);
+  if (persist) return cudaLaunchCooperativeKernel(fn, dim3(grid), dim3(JB_THREADS), args, smem, st);
+  return cudaLaunchKernel(fn, dim3(grid), dim3(JB_THREADS), args, smem, st);
+}
+
+cudaError_t launch_init(double *b0, double *b1, int64_t nplanes, const JbGeom &g, int64_t z_first,
+                        unsigned long long seed, cudaStream_t st) {
+  jb_init_u12<<<1184, 256, 0, st>>>(b0, b1, nplanes, g, z_first, seed);
+  return cudaGetLastError();
+}
+
+cudaError_t launch_flag_max(unsigned long long *flags, int n, unsigned long long v, cudaStream_t st) {
+  jb_flag_max<<<1, 32, 0, st>>>(flags, n, v);
+  return cudaGetLastError();
+}
+
+}  // namespace jbk

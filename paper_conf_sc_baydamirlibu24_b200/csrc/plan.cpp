@@ -1,0 +1,179 @@
+// plan.cpp — host-only planning logic of the CPU-Free Jacobi library: slab decomposition
+// ("divided equally among GPUs"), the HBM layout and tile shape, and the thread-block
+// split between boundary and interior blocks (§4.1.2).  No CUDA calls here, so the
+// logic is testable on a CPU-only box through the C ABI (tests/test_host_logic.py).
+#include <algorithm>
+#include <cmath>
+#include <cstring>
+
+#include "jacobi_internal.h"
+#include "../../include/jacobi.h"
+
+namespace jbplan {
+
+int64_t pow2ceil(int64_t v) {
+  int64_t p = 1;
+  while (p < v) p <<= 1;
+  return p;
+}
+
+static int64_t round_up(int64_t v, int64_t m) { return (v + m - 1) / m * m; }
+
+void decompose(int64_t n_out, int nslabs, int slab, int64_t *start, int64_t *chunk) {
+  const int64_t inner = n_out - 2;
+  const int64_t q = inner / nslabs, r = inner % nslabs;
+  *chunk = q + (slab < r ? 1 : 0);
+  *start = 1 + (int64_t)slab * q + std::min<int64_t>(slab, r);
+}
+
+size_t smem_bytes(const JbGeom &g) {
+  size_t bar = (size_t)2 * g.stages * 8;
+  bar = (bar + 127) / 128 * 128;
+  return bar + (size_t)g.stages * g.stage_doubles * 8;
+}
+
+int geometry(int64_t nx, int64_t ny, int64_t nz, int dim, int tile_x, int tile_y, int smem,
+             int stages_req, JbGeom *g) {
+  std::memset(g, 0, sizeof(*g));
+  g->nx = nx; g->ny = ny; g->nz = nz; g->dim = dim;
+  g->pitch = round_up(nx + 3, 4);
+  g->plane_elems = dim == 2 ? g->pitch : ny * g->pitch;
+  const int64_t ix = nx - 2;
+  int64_t tx = tile_x > 0 ? pow2ceil(tile_x) : std::min<int64_t>(dim == 2 ? 1024 : 512, pow2ceil(ix));
+  tx = std::max<int64_t>(tx, 8);
+  if (tx > 4096) return -1;
+  g->tx = (int)tx;
+  int sh = 0;
+  while ((int64_t(1) << sh) < tx / 2) ++sh;
+  g->txp_shift = sh;
+  g->ws = (int)tx + 4;
+  g->units_x = (int)((ix + tx - 1) / tx);
+  if (dim == 2) {
+    g->ty = 1; g->rh = 1; g->units_y = 1;
+  } else {
+    int ty = tile_y > 0 ? tile_y : 8;
+    ty = (int)std::min<int64_t>(ty, ny - 2);
+    ty = std::max(ty, 1);
+    if (ty + 2 > 32) return -1;  // producer warp issues one row per lane
+    g->ty = ty; g->rh = ty + 2;
+    g->units_y = (int)((ny - 2 + ty - 1) / ty);
+  }
+  g->units = g->units_x * g->units_y;
+  g->stage_doubles = g->rh * g->ws;
+  const size_t stage_b = (size_t)g->stage_doubles * 8;
+  int s = (int)((smem - 256) / (stage_b + 16));
+  s = std::min(s, JB_MAX_STAGES);
+  if (stages_req > 0) s = std::min(s, stages_req);
+  if (s < 4) return -1;  // need p-1, p, p+1 resident + one in flight
+  g->stages = s;
+  if (smem_bytes(*g) > (size_t)smem) return -1;
+  return 0;
+}
+
+void tb_split(int ctas, int64_t inner, int has_top, int has_bot, int64_t units, int override_ps,
+              int *n_top, int *n_bot, int *n_int) {
+  const int sides = (has_top ? 1 : 0) + (has_bot ? 1 : 0);
+  if (sides == 0) { *n_top = *n_bot = 0; *n_int = ctas; return; }
+  // Reconstructed P:400: boundary_TB = TB_total * boundary_size / (inner_size + 2*boundary_size).
+  // A boundary plane costs ~2.5 interior planes (it loads p-1, p, p+1 and stores twice).
+  const double wb = 2.5;
+  int ps;
+  if (override_ps > 0) {
+    ps = override_ps;
+  } else {
+    ps = (int)std::ceil((double)ctas * wb / ((double)std::max<int64_t>(inner, 0) + sides * wb));
+  }
+  ps = std::max(ps, 1);
+  ps = (int)std::min<int64_t>(ps, units);
+  if (inner > 0) ps = std::min(ps, std::max(1, (ctas - 1) / sides));
+  else if (override_ps <= 0) ps = (int)std::min<int64_t>(std::max(1, ctas / sides), units);
+  ps = std::min(ps, std::max(1, ctas / sides));
+  *n_top = has_top ? ps : 0;
+  *n_bot = has_bot ? ps : 0;
+  *n_int = ctas - *n_top - *n_bot;
+  if (inner <= 0) *n_int = std::max(*n_int, 0);
+}
+
+int lockstep_k(int units, int n_int, int64_t inner) {
+  if (units <= 0 || n_int < units || inner <= 0) return 0;
+  int64_t k = n_int / units;
+  k = std::min<int64_t>(k, inner);
+  return (int)std::max<int64_t>(k, 1);
+}
+
+int choose_ty(int64_t ny, int units_x, int n_int, int smem, int ws) {
+  // Largest-utilisation ty in [4, 12] whose stage still leaves a >= 5-deep ring.
+  int best = 8;
+  double best_score = -1;
+  for (int ty = 4; ty <= 12; ++ty) {
+    if (ty > ny - 2) break;
+    const size_t stage_b = (size_t)(ty + 2) * ws * 8;
+    if ((size_t)(smem - 256) / (stage_b + 16) < 5) break;
+    const int64_t uy = (ny - 2 + ty - 1) / ty;
+    const int64_t u = uy * units_x;
+    double util;
+    if (u > n_int) {
+      util = 0.5;  // not lockstep-able; linear fallback
+    } else {
+      const int64_t k = n_int / u;
+      util = (double)(u * k) / n_int;
+    }
+    // Prefer fewer halo rows when utilisation ties (reads (ty+2)/ty rows per row from L2).
+    const double score = util - 0.02 * (2.0 / ty);
+    if (score > best_score + 1e-9) { best_score = score; best = ty; }
+  }
+  return best;
+}
+
+}  // namespace jbplan
+
+extern "C" {
+
+int jacobi_decompose(int64_t n_out, int nslabs, int slab, int64_t *start, int64_t *chunk) {
+  if (n_out < 3 || nslabs < 1 || slab < 0 || slab >= nslabs || !start || !chunk) return JACOBI_EINVAL;
+  jbplan::decompose(n_out, nslabs, slab, start, chunk);
+  return JACOBI_OK;
+}
+
+int jacobi_tb_split(int ctas, int64_t chunk, int has_top, int has_bottom, int64_t units,
+                    int override_per_side, int *out3) {
+  if (!out3 || ctas < 1 || chunk < 1 || units < 1) return JACOBI_EINVAL;
+  const int64_t lo = has_top ? 2 : 1, hi = has_bottom ? chunk - 1 : chunk;
+  const int64_t inner = hi - lo + 1;
+  const int sides = (has_top ? 1 : 0) + (has_bottom ? 1 : 0);
+  if (ctas < sides + (inner > 0 ? 1 : 0)) return JACOBI_EINVAL;
+  jbplan::tb_split(ctas, inner, has_top, has_bottom, units, override_per_side, &out3[0], &out3[1], &out3[2]);
+  return JACOBI_OK;
+}
+
+int jacobi_geometry(int64_t nx, int64_t ny, int64_t nz, int stencil, int tile_x, int tile_y,
+                    int64_t *out8) {
+  if (!out8 || nx < 3 || ny < 3) return JACOBI_EINVAL;
+  if (!((stencil == 5 && nz == 1) || (stencil == 7 && nz >= 3))) return JACOBI_EINVAL;
+  JbGeom g;
+  if (jbplan::geometry(nx, ny, nz, stencil == 5 ? 2 : 3, tile_x, tile_y, JB_SMEM_DEFAULT, 0, &g))
+    return JACOBI_EINVAL;
+  out8[0] = g.pitch; out8[1] = g.plane_elems; out8[2] = g.tx; out8[3] = g.ty;
+  out8[4] = g.units_x; out8[5] = g.units_y; out8[6] = g.rh; out8[7] = g.ws;
+  return JACOBI_OK;
+}
+
+const char *jacobi_strerror(int code) {
+  switch (code) {
+    case JACOBI_OK: return "ok";
+    case JACOBI_EINVAL: return "invalid argument";
+    case JACOBI_ENODEV: return "not enough CUDA devices";
+    case JACOBI_ENOPEER: return "peer access between neighbouring GPUs unavailable";
+    case JACOBI_ENOCOOP: return "cooperative launch unavailable or grid not co-resident";
+    case JACOBI_ENOMEM: return "out of memory";
+    case JACOBI_ECUDA: return "CUDA runtime error";
+    case JACOBI_ETIMEOUT: return "device watchdog timeout: a neighbour never signalled";
+    case JACOBI_ENCCL: return "NCCL unavailable or failed";
+    case JACOBI_ESTATE: return "invalid state for this call";
+    default: return "unknown error";
+  }
+}
+
+int jacobi_version(void) { return 100; }
+
+}  // extern "C"

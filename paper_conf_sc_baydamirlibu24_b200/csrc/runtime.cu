@@ -1,0 +1,795 @@
+// runtime.cu — host runtime behind the C ABI in include/jacobi.h.
+//
+// Owns devices, slabs (HBM buffers + control blocks), peer mappings (UVA peer access in one
+// process, CUDA IPC across processes), launches, timing, and the CPU-controlled baselines.
+// All device work is done by the kernels in kernels.cu; the host only orchestrates.
+#include <cuda_runtime.h>
+#include <dlfcn.h>
+#include <nccl.h>
+
+#include <algorithm>
+#include <cstdio>
+#include <cstdlib>
+#include <cstring>
+#include <string>
+#include <vector>
+
+#include "../../include/jacobi.h"
+#include "jacobi_internal.h"
+
+namespace jbk {
+cudaError_t prepare(int dim, bool nocomp, bool persist, size_t smem);
+cudaError_t occupancy(int dim, bool nocomp, bool persist, size_t smem, int *blocks_per_sm);
+cudaError_t launch_sweep(const JbParams &p, bool nocomp, bool persist, int grid, size_t smem,
+                         cudaStream_t st);
+cudaError_t launch_init(double *b0, double *b1, int64_t nplanes, const JbGeom &g, int64_t z_first,
+                        unsigned long long seed, cudaStream_t st);
+cudaError_t launch_flag_max(unsigned long long *flags, int n, unsigned long long v, cudaStream_t st);
+}  // namespace jbk
+
+namespace {
+
+constexpr unsigned long long kSeedBench = 0x5C24ull;
+enum Kind { KIND_SINGLE = 0, KIND_VIRTUAL = 1, KIND_DIST = 2 };
+
+int cuda_err(cudaError_t e) {
+  if (e == cudaSuccess) return JACOBI_OK;
+  if (e == cudaErrorMemoryAllocation) return JACOBI_ENOMEM;
+  if (e == cudaErrorCooperativeLaunchTooLarge) return JACOBI_ENOCOOP;
+  if (getenv("JACOBI_DEBUG")) fprintf(stderr, "[jacobi] CUDA error: %s\n", cudaGetErrorString(e));
+  return JACOBI_ECUDA;
+}
+#define CK(x)                                  \
+  do {                                         \
+    int _rc = cuda_err(x);                     \
+    if (_rc != JACOBI_OK) return _rc;          \
+  } while (0)
+
+// ---------------------------------------------------------------- NCCL (dlopen'ed on demand)
+struct NcclApi {
+  void *lib = nullptr;
+  ncclResult_t (*GetUniqueId)(ncclUniqueId *) = nullptr;
+  ncclResult_t (*CommInitRank)(ncclComm_t *, int, ncclUniqueId, int) = nullptr;
+  ncclResult_t (*CommInitAll)(ncclComm_t *, int, const int *) = nullptr;
+  ncclResult_t (*CommDestroy)(ncclComm_t) = nullptr;
+  ncclResult_t (*Send)(const void *, size_t, ncclDataType_t, int, ncclComm_t, cudaStream_t) = nullptr;
+  ncclResult_t (*Recv)(void *, size_t, ncclDataType_t, int, ncclComm_t, cudaStream_t) = nullptr;
+  ncclResult_t (*GroupStart)() = nullptr;
+  ncclResult_t (*GroupEnd)() = nullptr;
+  bool load() {
+    if (lib) return true;
+    const char *names[] = {"libnccl.so.2", "libnccl.so"};
+    for (const char *n : names) {
+      lib = dlopen(n, RTLD_NOW | RTLD_GLOBAL);
+      if (lib) break;
+    }
+    if (!lib) return false;
+#define LD(f) f = reinterpret_cast<decltype(f)>(dlsym(lib, "nccl" #f))
+    LD(GetUniqueId); LD(CommInitRank); LD(CommInitAll); LD(CommDestroy);
+    LD(Send); LD(Recv); LD(GroupStart); LD(GroupEnd);
+#undef LD
+    return GetUniqueId && CommInitRank && CommInitAll && CommDestroy && Send && Recv && GroupStart && GroupEnd;
+  }
+};
+NcclApi g_nccl;
+
+// ---------------------------------------------------------------- IPC blob (dist mode)
+struct IpcBlob {
+  uint32_t magic;
+  int32_t rank;
+  int64_t chunk;
+  int64_t plane_elems;
+  cudaIpcMemHandle_t buf[2];
+  cudaIpcMemHandle_t ctrl;
+};
+constexpr uint32_t kIpcMagic = 0x4A43424Bu;
+
+}  // namespace
+
+struct Slab {
+  int device = 0;
+  int id = 0;  // global slab index
+  int64_t start = 0, chunk = 0;
+  double *buf[2] = {nullptr, nullptr};
+  JbCtrl *ctrl = nullptr;
+  cudaStream_t stream = nullptr;
+  cudaEvent_t ev0 = nullptr, ev1 = nullptr;
+  bool has_top = false, has_bot = false;
+  double *peer_top[2] = {nullptr, nullptr};
+  double *peer_bot[2] = {nullptr, nullptr};
+  unsigned long long *flag_out_top = nullptr, *flag_out_bot = nullptr;
+  int peer_top_dev = -1, peer_bot_dev = -1;
+  std::vector<void *> ipc_opened;
+  ncclComm_t comm = nullptr;
+  double last_ms = 0;
+  JbSlab desc{};  // last launch descriptor (for jacobi_describe)
+  int grid = 0;
+  size_t smem = 0;
+};
+
+struct jacobi_ctx {
+  int kind = KIND_SINGLE;
+  int64_t nx = 0, ny = 0, nz = 0, n_out = 0;
+  int stencil = 5, dim = 2;
+  int total = 1;  // total slabs P
+  int rank = 0;
+  std::vector<Slab> slabs;
+  int64_t t = 0;
+  int mode = JACOBI_MODE_CPUFREE, flags = 0;
+  int64_t tile_x = -1, tile_y = -1, stages = -1, boundary_ctas = -1, ctas = -1, schedule = -1;
+  int64_t timeout_ms = 20000;
+  bool peers_ready = false;
+  bool nccl_ready = false;
+  double last_ms_max = 0;
+  JbGeom geom{};  // layout geometry (pitch, plane_elems) fixed at create
+};
+
+namespace {
+
+int64_t slab_elems(const jacobi_ctx *h, const Slab &s) { return (s.chunk + 2) * h->geom.plane_elems; }
+
+int validate(int64_t nx, int64_t ny, int64_t nz, int stencil, int nslabs) {
+  if (nx < 3 || ny < 3 || nslabs < 1) return JACOBI_EINVAL;
+  if (!((stencil == 5 && nz == 1) || (stencil == 7 && nz >= 3))) return JACOBI_EINVAL;
+  const int64_t n_out = stencil == 5 ? ny : nz;
+  if (nslabs > 1 && (n_out - 2) / nslabs < 2) return JACOBI_EINVAL;  // every chunk >= 2 planes
+  if (nslabs > 1 && nx + 3 > (int64_t)1 << 40) return JACOBI_EINVAL;
+  return JACOBI_OK;
+}
+
+jacobi_ctx *new_ctx(int64_t nx, int64_t ny, int64_t nz, int stencil, int total) {
+  jacobi_ctx *h = new jacobi_ctx();
+  h->nx = nx; h->ny = ny; h->nz = nz; h->stencil = stencil;
+  h->dim = stencil == 5 ? 2 : 3;
+  h->n_out = h->dim == 2 ? ny : nz;
+  h->total = total;
+  JbGeom g;
+  // Layout only depends on pitch / plane_elems; tile parameters are re-planned per launch.
+  jbplan::geometry(nx, ny, nz, h->dim, 8, 1, JB_SMEM_DEFAULT, 0, &g);
+  h->geom = g;
+  return h;
+}
+
+int alloc_slab(jacobi_ctx *h, Slab &s) {
+  CK(cudaSetDevice(s.device));
+  const size_t bytes = (size_t)slab_elems(h, s) * sizeof(double);
+  CK(cudaMalloc(&s.buf[0], bytes));
+  CK(cudaMalloc(&s.buf[1], bytes));
+  CK(cudaMalloc(&s.ctrl, sizeof(JbCtrl)));
+  CK(cudaMemset(s.ctrl, 0, sizeof(JbCtrl)));
+  CK(cudaStreamCreateWithFlags(&s.stream, cudaStreamNonBlocking));
+  CK(cudaEventCreate(&s.ev0));
+  CK(cudaEventCreate(&s.ev1));
+  // Deterministic U12 initial field, both buffers, padding = 0.
+  CK(jbk::launch_init(s.buf[0], s.buf[1], s.chunk + 2, h->geom, s.start - 1, kSeedBench, s.stream));
+  CK(cudaStreamSynchronize(s.stream));
+  return JACOBI_OK;
+}
+
+void free_slab(Slab &s) {
+  cudaSetDevice(s.device);
+  if (s.comm && g_nccl.CommDestroy) g_nccl.CommDestroy(s.comm);
+  for (void *p : s.ipc_opened) cudaIpcCloseMemHandle(p);
+  s.ipc_opened.clear();
+  if (s.buf[0]) cudaFree(s.buf[0]);
+  if (s.buf[1]) cudaFree(s.buf[1]);
+  if (s.ctrl) cudaFree(s.ctrl);
+  if (s.ev0) cudaEventDestroy(s.ev0);
+  if (s.ev1) cudaEventDestroy(s.ev1);
+  if (s.stream) cudaStreamDestroy(s.stream);
+  s = Slab();
+}
+
+// Link slabs that live in this process (single / virtual mode).
+void link_local(jacobi_ctx *h) {
+  const int64_t pe = h->geom.plane_elems;
+  const int n = (int)h->slabs.size();
+  for (int i = 0; i < n; ++i) {
+    Slab &s = h->slabs[i];
+    s.has_top = i > 0;
+    s.has_bot = i < n - 1;
+    if (s.has_top) {
+      Slab &o = h->slabs[i - 1];
+      for (int p = 0; p < 2; ++p) s.peer_top[p] = o.buf[p] + (o.chunk + 1) * pe;
+      s.flag_out_top = &o.ctrl->flag_in[1];
+      s.peer_top_dev = o.device;
+    }
+    if (s.has_bot) {
+      Slab &o = h->slabs[i + 1];
+      for (int p = 0; p < 2; ++p) s.peer_bot[p] = o.buf[p];
+      s.flag_out_bot = &o.ctrl->flag_in[0];
+      s.peer_bot_dev = o.device;
+    }
+  }
+  h->peers_ready = true;
+}
+
+struct LaunchPlan {
+  JbParams P;
+  int grid = 0;
+  size_t smem = 0;
+  int device = 0;
+  cudaStream_t stream = nullptr;
+  std::vector<int> slab_idx;
+};
+
+// Plan one launch on one device over the local slabs `idx` (1 slab per GPU, or all slabs in
+// virtual mode).  persist=false plans the discrete baseline kernel (no boundary roles).
+int plan_launch(jacobi_ctx *h, const std::vector<int> &idx, bool persist, bool nocomp, LaunchPlan &L) {
+  Slab &s0 = h->slabs[idx[0]];
+  L.device = s0.device;
+  L.stream = s0.stream;
+  L.slab_idx = idx;
+  CK(cudaSetDevice(s0.device));
+  int sms = 0, smem_optin = 0;
+  CK(cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, s0.device));
+  CK(cudaDeviceGetAttribute(&smem_optin, cudaDevAttrMaxSharedMemoryPerBlockOptin, s0.device));
+  smem_optin = std::min(smem_optin, JB_SMEM_DEFAULT) - 1024;  // static smem + reserve
+
+  JbGeom g;
+  // First pass with the default ty to learn units_x / stage size.
+  if (jbplan::geometry(h->nx, h->ny, h->nz, h->dim, (int)h->tile_x, (int)h->tile_y, smem_optin,
+                       (int)h->stages, &g))
+    return JACOBI_EINVAL;
+  const int nslab = (int)idx.size();
+  int total_ctas = sms;  // one CTA per SM (occupancy verified below)
+  if (h->ctas > 0) total_ctas = (int)std::min<int64_t>(h->ctas * nslab, sms);
+  const int per = total_ctas / nslab;
+  if (h->dim == 3 && h->tile_y <= 0) {
+    int ty = jbplan::choose_ty(h->ny, g.units_x, per - (h->total > 1 ? 2 : 0), smem_optin, g.ws);
+    if (jbplan::geometry(h->nx, h->ny, h->nz, h->dim, (int)h->tile_x, ty, smem_optin, (int)h->stages, &g))
+      return JACOBI_EINVAL;
+  }
+  L.smem = jbplan::smem_bytes(g);
+  CK(jbk::prepare(h->dim, nocomp, persist, L.smem));
+  int occ = 0;
+  CK(jbk::occupancy(h->dim, nocomp, persist, L.smem, &occ));
+  if (occ < 1) return JACOBI_ENOCOOP;
+  L.grid = total_ctas;
+
+  JbParams &P = L.P;
+  std::memset(&P, 0, sizeof(P));
+  P.g = g;
+  P.nslabs = nslab;
+  P.flags = h->flags;
+  P.timeout_ns = (unsigned long long)h->timeout_ms * 1000000ull;
+  P.status = s0.ctrl->status;
+  int begin = 0;
+  for (int k = 0; k < nslab; ++k) {
+    Slab &s = h->slabs[idx[k]];
+    JbSlab &d = P.s[k];
+    const int count = per + (k < total_ctas % nslab ? 1 : 0);
+    d.buf[0] = s.buf[0]; d.buf[1] = s.buf[1];
+    d.peer_top[0] = s.peer_top[0]; d.peer_top[1] = s.peer_top[1];
+    d.peer_bot[0] = s.peer_bot[0]; d.peer_bot[1] = s.peer_bot[1];
+    d.flag_in_top = &s.ctrl->flag_in[0];
+    d.flag_in_bot = &s.ctrl->flag_in[1];
+    d.flag_out_top = s.flag_out_top;
+    d.flag_out_bot = s.flag_out_bot;
+    d.side_ctr = s.ctrl->side_ctr;
+    d.barrier = &s.ctrl->barrier;
+    d.chunk = s.chunk;
+    d.cta_begin = begin;
+    d.cta_count = count;
+    d.slab_id = s.id;
+    begin += count;
+    const bool top = persist && s.has_top, bot = persist && s.has_bot;
+    const int64_t lo = top ? 2 : 1, hi = bot ? s.chunk - 1 : s.chunk;
+    const int64_t inner = hi - lo + 1;
+    int nt, nb, ni;
+    if (count < (top ? 1 : 0) + (bot ? 1 : 0) + (inner > 0 ? 1 : 0)) return JACOBI_ENOCOOP;
+    jbplan::tb_split(count, inner, top, bot, g.units, (int)h->boundary_ctas, &nt, &nb, &ni);
+    d.n_top = nt;
+    d.n_bot = nb;
+    const bool lockstep = h->schedule == 1 || (h->schedule < 0 && h->dim == 3);
+    d.k_planes = lockstep ? jbplan::lockstep_k(g.units, ni, inner) : 0;
+    s.desc = d;
+    s.grid = count;
+    s.smem = L.smem;
+  }
+  return JACOBI_OK;
+}
+
+int read_status(Slab &s) {
+  int st[2] = {0, 0};
+  CK(cudaSetDevice(s.device));
+  CK(cudaMemcpy(st, s.ctrl->status, sizeof(st), cudaMemcpyDeviceToHost));
+  return st[0] ? st[0] : JACOBI_OK;
+}
+
+// Launch groups of this context: one launch per device slab, or one for all (virtual).
+std::vector<std::vector<int>> launch_groups(jacobi_ctx *h) {
+  std::vector<std::vector<int>> groups;
+  if (h->kind == KIND_VIRTUAL) {
+    std::vector<int> all;
+    for (int i = 0; i < (int)h->slabs.size(); ++i) all.push_back(i);
+    groups.push_back(all);
+  } else {
+    for (int i = 0; i < (int)h->slabs.size(); ++i) groups.push_back({i});
+  }
+  return groups;
+}
+
+int run_cpufree(jacobi_ctx *h, int64_t iters) {
+  const bool nocomp = h->flags & JACOBI_FLAG_NO_COMPUTE;
+  auto groups = launch_groups(h);
+  std::vector<LaunchPlan> plans(groups.size());
+  for (size_t i = 0; i < groups.size(); ++i) {
+    int rc = plan_launch(h, groups[i], true, nocomp, plans[i]);
+    if (rc) return rc;
+    plans[i].P.t0 = h->t;
+    plans[i].P.iters = iters;
+  }
+  // Reset per-run counters (barrier, side counters, status); flags are monotonic across runs.
+  for (auto &L : plans) {
+    CK(cudaSetDevice(L.device));
+    for (int k : L.slab_idx) {
+      Slab &s = h->slabs[k];
+      CK(cudaMemsetAsync(&s.ctrl->barrier, 0,
+                         sizeof(s.ctrl->barrier) + sizeof(s.ctrl->side_ctr) + sizeof(s.ctrl->status),
+                         L.stream));
+    }
+  }
+  // One host thread launches every GPU's persistent kernel back to back (co-residency across
+  // GPUs only needs every kernel to start; the device watchdog bounds any wait).
+  for (auto &L : plans) {
+    CK(cudaSetDevice(L.device));
+    Slab &s0 = h->slabs[L.slab_idx[0]];
+    CK(cudaEventRecord(s0.ev0, L.stream));
+    CK(jbk::launch_sweep(L.P, nocomp, true, L.grid, L.smem, L.stream));
+    CK(cudaEventRecord(s0.ev1, L.stream));
+  }
+  int rc_all = JACOBI_OK;
+  double mx = 0;
+  for (auto &L : plans) {
+    CK(cudaSetDevice(L.device));
+    Slab &s0 = h->slabs[L.slab_idx[0]];
+    CK(cudaEventSynchronize(s0.ev1));
+    float ms = 0;
+    CK(cudaEventElapsedTime(&ms, s0.ev0, s0.ev1));
+    for (int k : L.slab_idx) h->slabs[k].last_ms = ms;
+    mx = std::max(mx, (double)ms);
+    int rc = read_status(s0);
+    if (rc && !rc_all) rc_all = rc;
+  }
+  h->last_ms_max = mx;
+  if (rc_all) return rc_all;
+  h->t += iters;
+  return JACOBI_OK;
+}
+
+int ensure_nccl(jacobi_ctx *h) {
+  if (h->nccl_ready) return JACOBI_OK;
+  if (h->kind == KIND_VIRTUAL && h->total > 1) return JACOBI_EINVAL;  // NCCL: one rank per GPU
+  if (h->kind == KIND_DIST) return JACOBI_ESTATE;  // needs jacobi_nccl_init via the binding
+  if (!g_nccl.load()) return JACOBI_ENCCL;
+  std::vector<int> devs;
+  for (auto &s : h->slabs) devs.push_back(s.device);
+  std::vector<ncclComm_t> comms(devs.size());
+  if (g_nccl.CommInitAll(comms.data(), (int)devs.size(), devs.data()) != ncclSuccess) return JACOBI_ENCCL;
+  for (size_t i = 0; i < devs.size(); ++i) h->slabs[i].comm = comms[i];
+  h->nccl_ready = true;
+  return JACOBI_OK;
+}
+
+// CPU-controlled baseline (Listing 2.1a, "Baseline Copy", P:230 host barrier):
+// every iteration the host launches the discrete kernel on every GPU, then moves the edge planes
+// into the neighbours' halos (cudaMemcpyPeerAsync or NCCL send/recv), then synchronises every
+// GPU's stream before the next iteration (the OpenMP/MPI barrier of the reference code).
+int run_baseline(jacobi_ctx *h, int64_t iters, bool nccl) {
+  const bool nocomp = h->flags & JACOBI_FLAG_NO_COMPUTE;
+  if (nccl) {
+    int rc = ensure_nccl(h);
+    if (rc) return rc;
+  } else if (h->kind == KIND_DIST && h->total > 1) {
+    return JACOBI_EINVAL;  // memcpy baseline needs a host barrier across processes: use NCCL
+  }
+  const int n = (int)h->slabs.size();
+  std::vector<LaunchPlan> plans(n);
+  for (int i = 0; i < n; ++i) {
+    int rc = plan_launch(h, {i}, false, nocomp, plans[i]);
+    if (rc) return rc;
+    plans[i].P.iters = 1;
+  }
+  const int64_t pe = h->geom.plane_elems;
+  const size_t plane_bytes = (size_t)pe * sizeof(double);
+  for (int i = 0; i < n; ++i) {
+    CK(cudaSetDevice(h->slabs[i].device));
+    CK(cudaEventRecord(h->slabs[i].ev0, h->slabs[i].stream));
+  }
+  for (int64_t it = 0; it < iters; ++it) {
+    const int64_t tg = h->t + it;
+    const int nxt = (int)((tg + 1) & 1);
+    for (int i = 0; i < n; ++i) {  // ② launch the compute kernel on every GPU
+      Slab &s = h->slabs[i];
+      CK(cudaSetDevice(s.device));
+      if (!nocomp) {
+        plans[i].P.t0 = tg;
+        CK(jbk::launch_sweep(plans[i].P, false, false, plans[i].grid, plans[i].smem, s.stream));
+      }
+    }
+    if (!nccl) {  // ④ write_neighbors with host-issued peer copies
+      for (int i = 0; i < n; ++i) {
+        Slab &s = h->slabs[i];
+        CK(cudaSetDevice(s.device));
+        if (s.has_top)
+          CK(cudaMemcpyPeerAsync(s.peer_top[nxt], s.peer_top_dev, s.buf[nxt] + 1 * pe, s.device, plane_bytes,
+                                 s.stream));
+        if (s.has_bot)
+          CK(cudaMemcpyPeerAsync(s.peer_bot[nxt], s.peer_bot_dev, s.buf[nxt] + s.chunk * pe, s.device,
+                                 plane_bytes, s.stream));
+      }
+    } else {
+      if (g_nccl.GroupStart() != ncclSuccess) return JACOBI_ENCCL;
+      for (int i = 0; i < n; ++i) {
+        Slab &s = h->slabs[i];
+        const int me = s.id;
+        double *b = s.buf[nxt];
+        if (s.has_top) {
+          if (g_nccl.Send(b + 1 * pe, pe, ncclFloat64, me - 1, s.comm, s.stream) != ncclSuccess) return JACOBI_ENCCL;
+          if (g_nccl.Recv(b, pe, ncclFloat64, me - 1, s.comm, s.stream) != ncclSuccess) return JACOBI_ENCCL;
+        }
+        if (s.has_bot) {
+          if (g_nccl.Send(b + s.chunk * pe, pe, ncclFloat64, me + 1, s.comm, s.stream) != ncclSuccess)
+            return JACOBI_ENCCL;
+          if (g_nccl.Recv(b + (s.chunk + 1) * pe, pe, ncclFloat64, me + 1, s.comm, s.stream) != ncclSuccess)
+            return JACOBI_ENCCL;
+        }
+      }
+      if (g_nccl.GroupEnd() != ncclSuccess) return JACOBI_ENCCL;
+    }
+    for (int i = 0; i < n; ++i) {  // ⑤ host barrier: wait for every GPU
+      CK(cudaSetDevice(h->slabs[i].device));
+      CK(cudaStreamSynchronize(h->slabs[i].stream));
+    }
+  }
+  double mx = 0;
+  for (int i = 0; i < n; ++i) {
+    Slab &s = h->slabs[i];
+    CK(cudaSetDevice(s.device));
+    CK(cudaEventRecord(s.ev1, s.stream));
+    CK(cudaEventSynchronize(s.ev1));
+    float ms = 0;
+    CK(cudaEventElapsedTime(&ms, s.ev0, s.ev1));
+    s.last_ms = ms;
+    mx = std::max(mx, (double)ms);
+  }
+  h->last_ms_max = mx;
+  h->t += iters;
+  // Keep the CPU-Free protocol consistent: inbound flags hold the global iteration count.
+  for (auto &s : h->slabs) {
+    CK(cudaSetDevice(s.device));
+    CK(jbk::launch_flag_max(s.ctrl->flag_in, 2, (unsigned long long)h->t, s.stream));
+    CK(cudaStreamSynchronize(s.stream));
+  }
+  return JACOBI_OK;
+}
+
+}  // namespace
+
+// ======================================================================== C ABI
+extern "C" {
+
+int jacobi_create(int64_t nx, int64_t ny, int64_t nz, int stencil, int ngpus, jacobi_t *out) {
+  if (!out) return JACOBI_EINVAL;
+  *out = nullptr;
+  int rc = validate(nx, ny, nz, stencil, ngpus);
+  if (rc) return rc;
+  int ndev = 0;
+  if (cudaGetDeviceCount(&ndev) != cudaSuccess || ndev < ngpus) return JACOBI_ENODEV;
+  for (int g = 0; g + 1 < ngpus; ++g) {
+    int a = 0, b = 0;
+    cudaDeviceCanAccessPeer(&a, g, g + 1);
+    cudaDeviceCanAccessPeer(&b, g + 1, g);
+    if (!a || !b) return JACOBI_ENOPEER;
+  }
+  jacobi_ctx *h = new_ctx(nx, ny, nz, stencil, ngpus);
+  h->kind = KIND_SINGLE;
+  h->slabs.resize(ngpus);
+  for (int g = 0; g < ngpus; ++g) {
+    Slab &s = h->slabs[g];
+    s.device = g;
+    s.id = g;
+    jbplan::decompose(h->n_out, ngpus, g, &s.start, &s.chunk);
+    rc = alloc_slab(h, s);
+    if (rc) { jacobi_destroy(h); return rc; }
+  }
+  for (int g = 0; g < ngpus; ++g) {
+    cudaSetDevice(g);
+    for (int o : {g - 1, g + 1}) {
+      if (o < 0 || o >= ngpus) continue;
+      cudaError_t e = cudaDeviceEnablePeerAccess(o, 0);
+      if (e == cudaErrorPeerAccessAlreadyEnabled) cudaGetLastError();
+      else if (e != cudaSuccess) { jacobi_destroy(h); return JACOBI_ENOPEER; }
+    }
+  }
+  link_local(h);
+  *out = h;
+  return JACOBI_OK;
+}
+
+int jacobi_create_virtual(int64_t nx, int64_t ny, int64_t nz, int stencil, int nslabs, int device,
+                          jacobi_t *out) {
+  if (!out) return JACOBI_EINVAL;
+  *out = nullptr;
+  if (nslabs > JB_MAX_SLABS) return JACOBI_EINVAL;
+  int rc = validate(nx, ny, nz, stencil, nslabs);
+  if (rc) return rc;
+  int ndev = 0;
+  if (cudaGetDeviceCount(&ndev) != cudaSuccess || device < 0 || device >= ndev) return JACOBI_ENODEV;
+  jacobi_ctx *h = new_ctx(nx, ny, nz, stencil, nslabs);
+  h->kind = KIND_VIRTUAL;
+  h->slabs.resize(nslabs);
+  for (int g = 0; g < nslabs; ++g) {
+    Slab &s = h->slabs[g];
+    s.device = device;
+    s.id = g;
+    jbplan::decompose(h->n_out, nslabs, g, &s.start, &s.chunk);
+    rc = alloc_slab(h, s);
+    if (rc) { jacobi_destroy(h); return rc; }
+  }
+  link_local(h);
+  *out = h;
+  return JACOBI_OK;
+}
+
+int jacobi_create_rank(int64_t nx, int64_t ny, int64_t nz, int stencil, int world_size, int rank,
+                       int device, jacobi_t *out) {
+  if (!out) return JACOBI_EINVAL;
+  *out = nullptr;
+  if (rank < 0 || rank >= world_size) return JACOBI_EINVAL;
+  int rc = validate(nx, ny, nz, stencil, world_size);
+  if (rc) return rc;
+  int ndev = 0;
+  if (cudaGetDeviceCount(&ndev) != cudaSuccess || device < 0 || device >= ndev) return JACOBI_ENODEV;
+  jacobi_ctx *h = new_ctx(nx, ny, nz, stencil, world_size);
+  h->kind = KIND_DIST;
+  h->rank = rank;
+  h->slabs.resize(1);
+  Slab &s = h->slabs[0];
+  s.device = device;
+  s.id = rank;
+  jbplan::decompose(h->n_out, world_size, rank, &s.start, &s.chunk);
+  rc = alloc_slab(h, s);
+  if (rc) { jacobi_destroy(h); return rc; }
+  s.has_top = rank > 0;
+  s.has_bot = rank < world_size - 1;
+  h->peers_ready = world_size == 1;
+  *out = h;
+  return JACOBI_OK;
+}
+
+int jacobi_ipc_handle_bytes(void) { return (int)sizeof(IpcBlob); }
+
+int jacobi_get_ipc_handle(jacobi_t h, void *out) {
+  if (!h || !out || h->kind != KIND_DIST) return JACOBI_EINVAL;
+  Slab &s = h->slabs[0];
+  IpcBlob b;
+  std::memset(&b, 0, sizeof(b));
+  b.magic = kIpcMagic;
+  b.rank = h->rank;
+  b.chunk = s.chunk;
+  b.plane_elems = h->geom.plane_elems;
+  CK(cudaSetDevice(s.device));
+  CK(cudaIpcGetMemHandle(&b.buf[0], s.buf[0]));
+  CK(cudaIpcGetMemHandle(&b.buf[1], s.buf[1]));
+  CK(cudaIpcGetMemHandle(&b.ctrl, s.ctrl));
+  std::memcpy(out, &b, sizeof(b));
+  return JACOBI_OK;
+}
+
+int jacobi_open_peers(jacobi_t h, const void *top_blob, const void *bottom_blob) {
+  if (!h || h->kind != KIND_DIST) return JACOBI_EINVAL;
+  Slab &s = h->slabs[0];
+  if ((s.has_top && !top_blob) || (s.has_bot && !bottom_blob)) return JACOBI_EINVAL;
+  CK(cudaSetDevice(s.device));
+  const int64_t pe = h->geom.plane_elems;
+  auto open = [&](const void *blob, int expect_rank, double **bufs, JbCtrl **ctrl, int64_t *chunk) -> int {
+    IpcBlob b;
+    std::memcpy(&b, blob, sizeof(b));
+    if (b.magic != kIpcMagic || b.rank != expect_rank || b.plane_elems != pe) return JACOBI_EINVAL;
+    for (int p = 0; p < 2; ++p) {
+      void *ptr = nullptr;
+      CK(cudaIpcOpenMemHandle(&ptr, b.buf[p], cudaIpcMemLazyEnablePeerAccess));
+      s.ipc_opened.push_back(ptr);
+      bufs[p] = static_cast<double *>(ptr);
+    }
+    void *c = nullptr;
+    CK(cudaIpcOpenMemHandle(&c, b.ctrl, cudaIpcMemLazyEnablePeerAccess));
+    s.ipc_opened.push_back(c);
+    *ctrl = static_cast<JbCtrl *>(c);
+    *chunk = b.chunk;
+    return JACOBI_OK;
+  };
+  if (s.has_top) {
+    double *bufs[2];
+    JbCtrl *ctrl;
+    int64_t chunk;
+    int rc = open(top_blob, h->rank - 1, bufs, &ctrl, &chunk);
+    if (rc) return rc;
+    for (int p = 0; p < 2; ++p) s.peer_top[p] = bufs[p] + (chunk + 1) * pe;
+    s.flag_out_top = &ctrl->flag_in[1];
+  }
+  if (s.has_bot) {
+    double *bufs[2];
+    JbCtrl *ctrl;
+    int64_t chunk;
+    int rc = open(bottom_blob, h->rank + 1, bufs, &ctrl, &chunk);
+    if (rc) return rc;
+    for (int p = 0; p < 2; ++p) s.peer_bot[p] = bufs[p];
+    s.flag_out_bot = &ctrl->flag_in[0];
+  }
+  h->peers_ready = true;
+  return JACOBI_OK;
+}
+
+int jacobi_nccl_unique_id(void *out128) {
+  if (!out128) return JACOBI_EINVAL;
+  if (!g_nccl.load()) return JACOBI_ENCCL;
+  ncclUniqueId id;
+  if (g_nccl.GetUniqueId(&id) != ncclSuccess) return JACOBI_ENCCL;
+  std::memcpy(out128, &id, sizeof(id));
+  return JACOBI_OK;
+}
+
+int jacobi_nccl_init(jacobi_t h, const void *id128) {
+  if (!h || !id128 || h->kind != KIND_DIST) return JACOBI_EINVAL;
+  if (!g_nccl.load()) return JACOBI_ENCCL;
+  Slab &s = h->slabs[0];
+  CK(cudaSetDevice(s.device));
+  ncclUniqueId id;
+  std::memcpy(&id, id128, sizeof(id));
+  if (g_nccl.CommInitRank(&s.comm, h->total, id, h->rank) != ncclSuccess) return JACOBI_ENCCL;
+  h->nccl_ready = true;
+  return JACOBI_OK;
+}
+
+int jacobi_run(jacobi_t h, int64_t iters) {
+  if (!h || iters < 0) return JACOBI_EINVAL;
+  if (!h->peers_ready) return JACOBI_ESTATE;
+  if (iters == 0) {
+    h->last_ms_max = 0;
+    return JACOBI_OK;
+  }
+  if (h->mode == JACOBI_MODE_CPUFREE) return run_cpufree(h, iters);
+  if (h->mode == JACOBI_MODE_BASELINE_MEMCPY) return run_baseline(h, iters, false);
+  if (h->mode == JACOBI_MODE_BASELINE_NCCL) return run_baseline(h, iters, true);
+  return JACOBI_EINVAL;
+}
+
+int jacobi_set_mode(jacobi_t h, int mode, int flags) {
+  if (!h) return JACOBI_EINVAL;
+  if (mode < JACOBI_MODE_CPUFREE || mode > JACOBI_MODE_BASELINE_NCCL) return JACOBI_EINVAL;
+  if (flags & ~(JACOBI_FLAG_NO_COMPUTE | JACOBI_FLAG_DROP_SIGNAL)) return JACOBI_EINVAL;
+  h->mode = mode;
+  h->flags = flags;
+  return JACOBI_OK;
+}
+
+static int64_t *param_slot(jacobi_t h, const char *name) {
+  if (!std::strcmp(name, "tile_x")) return &h->tile_x;
+  if (!std::strcmp(name, "tile_y")) return &h->tile_y;
+  if (!std::strcmp(name, "stages")) return &h->stages;
+  if (!std::strcmp(name, "boundary_ctas")) return &h->boundary_ctas;
+  if (!std::strcmp(name, "ctas")) return &h->ctas;
+  if (!std::strcmp(name, "schedule")) return &h->schedule;
+  if (!std::strcmp(name, "timeout_ms")) return &h->timeout_ms;
+  return nullptr;
+}
+
+int jacobi_set_param(jacobi_t h, const char *name, int64_t value) {
+  if (!h || !name) return JACOBI_EINVAL;
+  int64_t *p = param_slot(h, name);
+  if (!p) return JACOBI_EINVAL;
+  if (!std::strcmp(name, "timeout_ms")) value = value < 0 ? 20000 : value;
+  if (!std::strcmp(name, "tile_x") && value > 4096) return JACOBI_EINVAL;
+  if (!std::strcmp(name, "tile_y") && value > 30) return JACOBI_EINVAL;
+  *p = value;
+  return JACOBI_OK;
+}
+
+int jacobi_get_param(jacobi_t h, const char *name, int64_t *value) {
+  if (!h || !name || !value) return JACOBI_EINVAL;
+  int64_t *p = param_slot(h, name);
+  if (!p) return JACOBI_EINVAL;
+  *value = *p;
+  return JACOBI_OK;
+}
+
+int jacobi_scatter(jacobi_t h, const double *in) {
+  if (!h || !in) return JACOBI_EINVAL;
+  const int64_t pe = h->geom.plane_elems, pitch = h->geom.pitch;
+  const int64_t rows_per_plane = h->dim == 2 ? 1 : h->ny;
+  for (auto &s : h->slabs) {
+    CK(cudaSetDevice(s.device));
+    const double *src = in + (s.start - 1) * rows_per_plane * h->nx;
+    // All copies on the slab's stream, then a stream sync: a device-to-device cudaMemcpy is
+    // asynchronous w.r.t. the host and would race with the next launch on this stream.
+    CK(cudaMemcpy2DAsync(s.buf[0] + 3, pitch * sizeof(double), src, h->nx * sizeof(double),
+                         h->nx * sizeof(double), (s.chunk + 2) * rows_per_plane, cudaMemcpyHostToDevice,
+                         s.stream));
+    CK(cudaMemcpyAsync(s.buf[1], s.buf[0], (size_t)(s.chunk + 2) * pe * sizeof(double),
+                       cudaMemcpyDeviceToDevice, s.stream));
+  }
+  for (auto &s : h->slabs) {
+    CK(cudaSetDevice(s.device));
+    CK(cudaStreamSynchronize(s.stream));
+  }
+  return JACOBI_OK;
+}
+
+int jacobi_gather(jacobi_t h, double *out) {
+  if (!h || !out) return JACOBI_EINVAL;
+  const int64_t pe = h->geom.plane_elems, pitch = h->geom.pitch;
+  const int64_t rpp = h->dim == 2 ? 1 : h->ny;
+  const int cur = (int)(h->t & 1);
+  const size_t w = h->nx * sizeof(double), dp = pitch * sizeof(double);
+  for (auto &s : h->slabs) {
+    CK(cudaSetDevice(s.device));
+    CK(cudaMemcpy2DAsync(out + s.start * rpp * h->nx, w, s.buf[cur] + pe + 3, dp, w, s.chunk * rpp,
+                         cudaMemcpyDeviceToHost, s.stream));
+    if (s.id == 0)
+      CK(cudaMemcpy2DAsync(out, w, s.buf[cur] + 3, dp, w, rpp, cudaMemcpyDeviceToHost, s.stream));
+    if (s.id == h->total - 1)
+      CK(cudaMemcpy2DAsync(out + (h->n_out - 1) * rpp * h->nx, w, s.buf[cur] + (s.chunk + 1) * pe + 3, dp, w,
+                           rpp, cudaMemcpyDeviceToHost, s.stream));
+  }
+  for (auto &s : h->slabs) {
+    CK(cudaSetDevice(s.device));
+    CK(cudaStreamSynchronize(s.stream));
+  }
+  return JACOBI_OK;
+}
+
+int jacobi_last_time(jacobi_t h, double *ms_max, double *ms_per_slab) {
+  if (!h) return JACOBI_EINVAL;
+  if (ms_max) *ms_max = h->last_ms_max;
+  if (ms_per_slab)
+    for (size_t i = 0; i < h->slabs.size(); ++i) ms_per_slab[i] = h->slabs[i].last_ms;
+  return JACOBI_OK;
+}
+
+int jacobi_iterations(jacobi_t h, int64_t *t) {
+  if (!h || !t) return JACOBI_EINVAL;
+  *t = h->t;
+  return JACOBI_OK;
+}
+
+int jacobi_num_slabs(jacobi_t h, int *local, int *total) {
+  if (!h) return JACOBI_EINVAL;
+  if (local) *local = (int)h->slabs.size();
+  if (total) *total = h->total;
+  return JACOBI_OK;
+}
+
+int jacobi_describe(jacobi_t h, int i, int64_t *o) {
+  if (!h || !o || i < 0 || i >= (int)h->slabs.size()) return JACOBI_EINVAL;
+  Slab &s = h->slabs[i];
+  // Plan the CPU-free launch now so the description is current.
+  std::vector<LaunchPlan> plans;
+  for (auto &grp : launch_groups(h)) {
+    if (std::find(grp.begin(), grp.end(), i) == grp.end()) continue;
+    LaunchPlan L;
+    int rc = plan_launch(h, grp, true, h->flags & JACOBI_FLAG_NO_COMPUTE, L);
+    if (rc) return rc;
+    o[0] = s.start; o[1] = s.chunk; o[2] = L.P.g.pitch; o[3] = L.P.g.plane_elems;
+    o[4] = L.P.g.tx; o[5] = L.P.g.ty; o[6] = L.P.g.units_x; o[7] = L.P.g.units_y;
+    o[8] = L.P.g.stages; o[9] = s.desc.n_top; o[10] = s.desc.n_bot;
+    o[11] = s.desc.cta_count - s.desc.n_top - s.desc.n_bot; o[12] = s.desc.cta_count;
+    o[13] = s.desc.k_planes; o[14] = (int64_t)L.smem; o[15] = s.device;
+  }
+  return JACOBI_OK;
+}
+
+int jacobi_destroy(jacobi_t h) {
+  if (!h) return JACOBI_OK;
+  for (auto &s : h->slabs) {
+    if (s.device >= 0) cudaSetDevice(s.device);
+    if (s.stream) cudaStreamSynchronize(s.stream);
+  }
+  for (auto &s : h->slabs) free_slab(s);
+  delete h;
+  return JACOBI_OK;
+}
+
+}  // extern "C"

@@ -1,0 +1,218 @@
+"""GPU parity: the CUDA path (through the C ABI) vs the CPU oracle, element by element.
+
+Bar (BASELINE.json north_star): bit-exact fp64 — the kernel uses the oracle's
+operation order with contraction disabled — and the P-slab result bit-identical to P = 1.
+Shapes span several tiles with ragged tails in x, y and the outer axis; slab counts include
+remainders and the minimum chunk of 2 planes; modes cover CPU-Free, the memcpy baseline and
+NCCL (P = 1), and the no-compute / watchdog paths.
+"""
+import numpy as np
+import pytest
+
+import oracle
+import paper_conf_sc_baydamirlibu24_b200 as jb
+from jacobi_inputs import SEED_BENCH, integer_field, nv_field, u12
+
+pytestmark = pytest.mark.gpu
+
+
+def bits_equal(a, b):
+    return np.array_equal(np.asarray(a).view(np.uint64), np.asarray(b).view(np.uint64))
+
+
+def assert_bitwise(got, exp, what=""):
+    if not bits_equal(got, exp):
+        d = np.abs(got - exp)
+        idx = np.unravel_index(np.argmax(d), d.shape)
+        n = np.count_nonzero(got.view(np.uint64) != exp.view(np.uint64))
+        raise AssertionError(f"{what}: {n} cells differ, max |diff| {d.max()} at {idx}")
+
+
+def run_gpu(field, iters, virtual=0, mode=jb.MODE_CPUFREE, params=None, flags=0):
+    with jb.Jacobi(field.shape, virtual=virtual) as j:
+        for k, v in (params or {}).items():
+            j.set_param(k, v)
+        j.set_mode(mode, flags)
+        j.scatter(field)
+        j.run(iters)
+        return j.gather()
+
+
+# ---------------------------------------------------------------- 1 GPU
+def test_device_init_is_u12():
+    for shape in [(256, 256), (9, 37, 41)]:
+        with jb.Jacobi(shape) as j:
+            assert_bitwise(j.gather(), u12(shape, SEED_BENCH), "device U12 init")
+
+
+def test_c1_256sq_1000_iters_vs_oracle():
+    """BASELINE config C1: 2D 256x256, 1000 iterations, 1 GPU vs CPU oracle."""
+    f = u12((256, 256), SEED_BENCH)
+    with jb.Jacobi((256, 256)) as j:  # create initialises U12 on the device
+        j.run(1000)
+        got = j.gather()
+    assert_bitwise(got, oracle.jacobi(f, 1000, 8), "C1")
+
+
+@pytest.mark.parametrize("shape", [(3, 3), (4, 5), (37, 1500), (70, 2051), (300, 130)])
+@pytest.mark.parametrize("iters", [1, 2, 7])
+def test_2d_shapes(shape, iters):
+    f = u12(shape, 1)
+    exp = oracle.jacobi(f, iters)
+    assert_bitwise(run_gpu(f, iters), exp, f"2D {shape}")
+    assert_bitwise(run_gpu(f, iters, params={"tile_x": 64}), exp, f"2D {shape} tx64")
+
+
+@pytest.mark.parametrize("shape", [(3, 3, 3), (5, 4, 9), (13, 30, 70), (20, 61, 130), (9, 17, 600)])
+@pytest.mark.parametrize("iters", [1, 4])
+def test_3d_shapes(shape, iters):
+    f = u12(shape, 2)
+    exp = oracle.jacobi(f, iters)
+    assert_bitwise(run_gpu(f, iters), exp, f"3D {shape}")
+    assert_bitwise(run_gpu(f, iters, params={"tile_y": 3, "tile_x": 16}), exp, f"3D {shape} ty3")
+
+
+@pytest.mark.parametrize("sched", [0, 1])
+@pytest.mark.parametrize("stages", [4, 7])
+def test_schedules_and_ring_depths(sched, stages):
+    for shape in [(130, 333), (11, 40, 50)]:
+        f = u12(shape, 3)
+        exp = oracle.jacobi(f, 5)
+        got = run_gpu(f, 5, params={"schedule": sched, "stages": stages, "ctas": 5})
+        assert_bitwise(got, exp, f"{shape} sched={sched} stages={stages}")
+
+
+# ---------------------------------------------------------------- virtual slabs (multi-GPU protocol)
+@pytest.mark.parametrize("P", [2, 3, 4, 5, 8])
+def test_virtual_2d(P):
+    shape = (2 * P + 2 + 3, 777)  # chunk 2 for some slabs, remainder 3
+    f = u12(shape, 1)
+    for iters in (1, 6, 33):
+        assert_bitwise(run_gpu(f, iters, virtual=P), oracle.jacobi(f, iters), f"virtual P={P} it={iters}")
+
+
+@pytest.mark.parametrize("P", [2, 3, 8])
+def test_virtual_3d(P):
+    shape = (3 * P + 2 + 1, 21, 45)
+    f = u12(shape, 2)
+    for iters in (1, 9):
+        assert_bitwise(run_gpu(f, iters, virtual=P), oracle.jacobi(f, iters), f"virtual3d P={P}")
+
+
+def test_virtual_many_boundary_ctas():
+    f = u12((40, 4100), 3)
+    exp = oracle.jacobi(f, 11)
+    for bc in (1, 2, 4):
+        got = run_gpu(f, 11, virtual=4, params={"boundary_ctas": bc, "tile_x": 128})
+        assert_bitwise(got, exp, f"boundary_ctas={bc}")
+
+
+def test_virtual_c5_latency_shapes_long():
+    """C5 shapes (3D 128^3, 2D 1024^2) at P = 8 slabs, 100 iterations, vs P = 1 and the oracle."""
+    for shape in [(128, 128, 128), (1024, 1024)]:
+        f = u12(shape, SEED_BENCH)
+        exp = oracle.jacobi(f, 100, 8)
+        assert_bitwise(run_gpu(f, 100, virtual=8), exp, f"C5 {shape} P=8")
+        assert_bitwise(run_gpu(f, 100), exp, f"C5 {shape} P=1")
+
+
+# ---------------------------------------------------------------- baselines
+@pytest.mark.parametrize("P", [1, 2, 4])
+def test_baseline_memcpy_virtual(P):
+    f = u12((4 * P + 5, 300), 1)
+    exp = oracle.jacobi(f, 13)
+    assert_bitwise(run_gpu(f, 13, virtual=P, mode=jb.MODE_BASELINE_MEMCPY), exp, f"memcpy P={P}")
+    g = u12((3 * P + 3, 12, 33), 2)
+    assert_bitwise(run_gpu(g, 5, virtual=P, mode=jb.MODE_BASELINE_MEMCPY), oracle.jacobi(g, 5), "memcpy 3d")
+
+
+def test_baseline_nccl_single_gpu():
+    f = u12((65, 300), 1)
+    assert_bitwise(run_gpu(f, 9, mode=jb.MODE_BASELINE_NCCL), oracle.jacobi(f, 9), "nccl P=1")
+
+
+def test_mode_switching_and_run_splitting():
+    f = u12((50, 310), 2)
+    exp = oracle.jacobi(f, 20)
+    with jb.Jacobi(f.shape, virtual=3) as j:
+        j.scatter(f)
+        j.run(3)
+        j.set_mode(jb.MODE_BASELINE_MEMCPY).run(4)
+        j.set_mode(jb.MODE_CPUFREE).run(0).run(5)
+        j.set_mode(jb.MODE_BASELINE_MEMCPY).run(1)
+        j.set_mode(jb.MODE_CPUFREE).run(7)
+        assert j.iterations == 20
+        assert_bitwise(j.gather(), exp, "mixed modes")
+
+
+# ---------------------------------------------------------------- invariants through the C ABI
+def test_harmonic_and_constant_fields_stationary():
+    y, x = np.mgrid[0:40, 0:70].astype(np.float64)
+    for f in (3 + 2 * x - 5 * y, x * x - y * y, x * y, np.full((40, 70), np.pi)):
+        assert_bitwise(run_gpu(f, 101, virtual=3), f, "2D stationary")
+    z, y, x = np.mgrid[0:12, 0:13, 0:30].astype(np.float64)
+    for f in (1 + x + 2 * y - 3 * z, x * x + y * y - 2 * z * z, x * y + y * z + z * x):
+        assert_bitwise(run_gpu(f, 51, virtual=2), f, "3D stationary")
+
+
+def test_exact_integer_rational_field():
+    f = integer_field((33, 70), 5)
+    assert_bitwise(run_gpu(f, 20, virtual=2), oracle.jacobi(f, 20), "integer field")
+
+
+def test_subnormals_not_flushed():
+    f = nv_field((34, 2400))
+    exp = oracle.jacobi(f, 1000, 8)
+    got = run_gpu(f, 1000)
+    assert np.count_nonzero((exp != 0) & (np.abs(exp) < np.finfo(np.float64).tiny)) > 0
+    assert_bitwise(got, exp, "subnormals")
+
+
+def test_gather_scatter_roundtrip_and_run_zero():
+    f = u12((7, 19, 23), 9)
+    with jb.Jacobi(f.shape, virtual=2) as j:
+        j.scatter(f)
+        j.run(0)
+        assert_bitwise(j.gather(), f, "roundtrip")
+
+
+def test_no_compute_mode_moves_halos_only():
+    f = u12((20, 64), 4)
+    with jb.Jacobi(f.shape, virtual=2) as j:
+        j.scatter(f)
+        j.set_mode(jb.MODE_CPUFREE, jb.FLAG_NO_COMPUTE).run(3)
+        g = j.gather()
+    # owned planes untouched (no arithmetic), only halos (not gathered) change
+    assert_bitwise(g, f, "no-compute leaves owned planes")
+
+
+# ---------------------------------------------------------------- errors
+def test_errors():
+    with pytest.raises(jb.JacobiError) as e:
+        jb.Jacobi((2, 10))
+    assert e.value.code == jb.JACOBI_EINVAL
+    with pytest.raises(jb.JacobiError) as e:
+        jb.Jacobi((5, 10), virtual=2)  # chunk 1.5 < 2
+    assert e.value.code == jb.JACOBI_EINVAL
+    with pytest.raises(jb.JacobiError) as e:
+        jb.Jacobi((1000, 64), ngpus=64)
+    assert e.value.code == jb.JACOBI_ENODEV
+    with jb.Jacobi((10, 10)) as j:
+        with pytest.raises(jb.JacobiError):
+            j.set_mode(7)
+        with pytest.raises(jb.JacobiError):
+            j.run(-1)
+        with pytest.raises(jb.JacobiError):
+            j.set_param("nope", 1)
+
+
+def test_watchdog_timeout_without_hang():
+    with jb.Jacobi((40, 200), virtual=2) as j:
+        j.set_param("timeout_ms", 300)
+        j.set_mode(jb.MODE_CPUFREE, jb.FLAG_DROP_SIGNAL)
+        with pytest.raises(jb.JacobiError) as e:
+            j.run(10)
+        assert e.value.code == jb.JACOBI_ETIMEOUT
+    # the device is still healthy afterwards
+    f = u12((40, 200), 1)
+    assert_bitwise(run_gpu(f, 3, virtual=2), oracle.jacobi(f, 3), "after timeout")

@@ -1,0 +1,164 @@
+"""CPU-only tests of the C-ABI library: it loads, exports every symbol include/jacobi.h
+declares, and its host-only planning logic (slab decomposition P:350, TB split P:398-404,
+HBM geometry) is correct.  No kernel is launched here."""
+import ctypes
+import os
+import subprocess
+
+import numpy as np
+import pytest
+
+import paper_conf_sc_baydamirlibu24_b200 as jb
+
+
+@pytest.fixture(scope="module", autouse=True)
+def built():
+    from paper_conf_sc_baydamirlibu24_b200 import build as b
+    b.build()
+
+
+def test_library_exports_every_header_symbol():
+    names = jb.header_functions()
+    assert len(names) == len(jb._SIGS) == 24
+    L = ctypes.CDLL(jb.LIB_PATH)
+    missing = [n for n in names if not hasattr(L, n)]
+    assert not missing, missing
+    # and the binding mirrors every one of them
+    for n in names:
+        assert n in jb._SIGS, n
+
+
+def test_library_is_sm100a_only():
+    out = subprocess.run(["/usr/local/cuda/bin/cuobjdump", "--list-elf", jb.LIB_PATH],
+                         capture_output=True, text=True).stdout
+    assert "sm_100a" in out
+    for bad in ("sm_80", "sm_90", "sm_103"):
+        assert bad not in out
+
+
+def test_sass_uses_bulk_copy_and_no_fma():
+    sass = subprocess.run(["/usr/local/cuda/bin/cuobjdump", "-sass", jb.LIB_PATH],
+                          capture_output=True, text=True).stdout
+    assert "UBLKCP" in sass, "persistent kernel must stream planes with cp.async.bulk (TMA)"
+    # fp64 fused multiply-add would break the oracle's operation order
+    assert "DFMA" not in sass
+
+
+def test_strerror_and_version():
+    assert jb.strerror(0) == "ok"
+    assert "timeout" in jb.strerror(jb.JACOBI_ETIMEOUT)
+    assert jb.jacobi_version() >= 100
+
+
+@pytest.mark.parametrize("n_out", [3, 4, 5, 17, 258, 16384, 514])
+@pytest.mark.parametrize("P", [1, 2, 3, 4, 7, 8])
+def test_decompose(n_out, P):
+    inner = n_out - 2
+    q, r = divmod(inner, P)
+    nxt = 1
+    total = 0
+    for g in range(P):
+        s, c = jb.jacobi_decompose(n_out, P, g)
+        assert s == nxt
+        assert c == q + (1 if g < r else 0)
+        nxt = s + c
+        total += c
+    assert total == inner and nxt == n_out - 1
+
+
+def test_decompose_rejects():
+    with pytest.raises(jb.JacobiError):
+        jb.jacobi_decompose(2, 1, 0)
+    with pytest.raises(jb.JacobiError):
+        jb.jacobi_decompose(10, 2, 2)
+
+
+@pytest.mark.parametrize("ctas", [4, 18, 37, 74, 148])
+@pytest.mark.parametrize("chunk", [2, 3, 16, 64, 255, 2048])
+@pytest.mark.parametrize("sides", [(0, 0), (1, 0), (0, 1), (1, 1)])
+def test_tb_split(ctas, chunk, sides):
+    top, bot = sides
+    units = 16
+    lo, hi = (2 if top else 1), (chunk - 1 if bot else chunk)
+    inner = hi - lo + 1
+    try:
+        nt, nb, ni = jb.jacobi_tb_split(ctas, chunk, top, bot, units)
+    except jb.JacobiError:
+        assert ctas < top + bot + (inner > 0)
+        return
+    assert nt + nb + ni == ctas
+    assert (nt > 0) == bool(top) and (nb > 0) == bool(bot)
+    if top and bot:
+        assert nt == nb
+    assert nt <= units and nb <= units
+    if inner > 0:
+        assert ni >= 1
+    if not top and not bot:
+        assert ni == ctas
+    # the reconstructed P:400 formula: boundary share grows as the slab thins
+    if top and bot and inner > 0 and ctas >= 37:
+        thin = jb.jacobi_tb_split(ctas, 4, 1, 1, units)[0]
+        thick = jb.jacobi_tb_split(ctas, 2048, 1, 1, units)[0]
+        assert thin >= thick
+
+
+def test_tb_split_override():
+    assert jb.jacobi_tb_split(148, 100, 1, 1, 16, 3) == (3, 3, 142)
+
+
+@pytest.mark.parametrize("nx", [3, 4, 5, 6, 7, 130, 256, 511, 512, 1024, 16384])
+def test_geometry_alignment(nx):
+    for st, ny, nz in ((5, 9, 1), (7, 9, 5)):
+        g = jb.jacobi_geometry(nx, ny, nz, st)
+        pitch = g["pitch"]
+        assert pitch % 4 == 0 and pitch >= nx + 3
+        tx = g["tile_x"]
+        assert tx & (tx - 1) == 0 and tx >= 8
+        assert g["units_x"] == -(-(nx - 2) // tx)
+        for ux in range(g["units_x"]):
+            x0 = 1 + ux * tx
+            assert (x0 + 3) % 2 == 0          # first output cell 16-byte aligned
+            xs = 2 + ux * tx
+            xe = min(xs + tx + 4, pitch)
+            assert xs % 2 == 0 and (xe - xs) % 2 == 0  # bulk copy: 16 B aligned, multiple of 16 B
+            assert xs <= x0 - 1 + 3 and min(x0 + tx, nx - 1) + 3 < xe  # covers x0-1 .. last+1
+        if st == 5:
+            assert g["plane_elems"] == pitch and g["stage_rows"] == 1
+        else:
+            assert g["plane_elems"] == ny * pitch and g["stage_rows"] == g["tile_y"] + 2
+
+
+def test_geometry_rejects():
+    with pytest.raises(jb.JacobiError):
+        jb.jacobi_geometry(2, 9, 1, 5)
+    with pytest.raises(jb.JacobiError):
+        jb.jacobi_geometry(9, 9, 3, 5)
+    with pytest.raises(jb.JacobiError):
+        jb.jacobi_geometry(9, 9, 1, 7)
+
+
+def test_create_without_gpu_is_loud():
+    """On a box without a CUDA device the product path must fail, never fall back."""
+    import torch
+    if torch.cuda.is_available():
+        pytest.skip("GPU present")
+    with pytest.raises(jb.JacobiError) as e:
+        jb.Jacobi((10, 10))
+    assert e.value.code == jb.JACOBI_ENODEV
+
+
+def test_binding_rejects_bad_arrays():
+    with pytest.raises(ValueError):
+        jb._host_ptr(np.zeros(10, dtype=np.float32), 10, False)
+    with pytest.raises(ValueError):
+        jb._host_ptr(np.zeros(9), 10, False)
+
+
+def test_product_package_does_not_import_oracle():
+    pkg = os.path.dirname(jb.__file__)
+    for root, _, files in os.walk(pkg):
+        for f in files:
+            if f.endswith((".py", ".cu", ".cpp", ".h")):
+                src = open(os.path.join(root, f)).read()
+                assert "import oracle" not in src and "from oracle" not in src, f
+                assert "jacobi_oracle" not in src, f
