@@ -105,8 +105,11 @@ int jacobi_nccl_init(jacobi_t h, const void *id128);
 int jacobi_run(jacobi_t h, int64_t iters);
 int jacobi_set_mode(jacobi_t h, int mode, int flags);
 /* Tuning knobs (none changes results): "tile_x", "tile_y", "stages", "boundary_ctas",
- * "ctas" (persistent grid size per slab group, 0 = all co-resident), "schedule"
- * (-1 auto, 0 linear, 1 lockstep), "timeout_ms" (watchdog, default 20000).  -1 = default. */
+ * "ctas" (persistent grid size per slab group, 0 = all co-resident), "schedule" (interior
+ * work distribution: -1 auto = 2, 0 static linear, 1 static lockstep, 2 dynamic guided
+ * self-scheduling), "min_block" (smallest dynamic block, planes, default 8), "dyn_help"
+ * (1: boundary blocks join the dynamic interior after signalling), "timeout_ms" (watchdog,
+ * default 20000).  Unknown names return JACOBI_EINVAL. */
 int jacobi_set_param(jacobi_t h, const char *name, int64_t value);
 int jacobi_get_param(jacobi_t h, const char *name, int64_t *value);
 

@@ -8,6 +8,7 @@
 #define JB_NC (JB_NCW * 32)     // consumer threads per CTA
 #define JB_THREADS (JB_NC + 32) // + one producer warp (bulk-copy issue)
 #define JB_MAX_STAGES 32
+#define JB_RQ 4                 // run-descriptor queue depth (producer -> consumers)
 #define JB_SMEM_DEFAULT 232448  // B200 opt-in dynamic shared memory per block (227 KB)
 
 // Grid geometry in HBM and the tile shape of the march.
@@ -43,8 +44,17 @@ struct JbSlab {
   int64_t chunk;
   int32_t cta_begin, cta_count;
   int32_t n_top, n_bot;              // boundary CTAs per side (0: no neighbour on that side)
-  int32_t k_planes;                  // lockstep plane ranges for the interior (0: linear schedule)
+  int32_t k_planes;                  // static lockstep plane ranges for the interior (0: linear)
   int32_t slab_id;                   // global slab index g
+  // Dynamic (guided self-scheduling) interior work, used when dyn_min_blk > 0: items are
+  // (plane block, unit) pairs claimed from work_ctr[t & 1] in block-major order; block k has
+  // max(dyn_min_blk, ceil(rem * units / (2 * dyn_n))) planes (rem = planes not yet blocked).
+  unsigned int *work_ctr;            // local [2], one per iteration parity
+  int32_t dyn_min_blk;
+  int32_t dyn_n;
+  int32_t dyn_help;                  // boundary CTAs join the interior after signalling
+  int32_t pad1;
+  int64_t dyn_items;                 // units * number of blocks
 };
 
 struct JbParams {
@@ -56,6 +66,7 @@ struct JbParams {
   int64_t iters;
   unsigned long long timeout_ns;
   int *status;      // [0] error code (0 ok), [1] abort flag
+  unsigned long long *trace;  // debug (JACOBI_TRACE): per-iteration CTA work-end timestamps, or null
 };
 
 // Per-slab control block in device memory (one allocation, IPC-exportable).
@@ -64,7 +75,8 @@ struct JbCtrl {
   unsigned long long barrier;
   unsigned int side_ctr[2];
   int status[2];
-  unsigned long long pad[26];      // 256 B total
+  unsigned int work[2];            // dynamic-schedule claim counters per iteration parity
+  unsigned long long pad[25];      // 256 B total
 };
 
 // ---- host-side planning (plan.cpp) -----------------------------------------------------
@@ -78,6 +90,9 @@ void tb_split(int ctas, int64_t inner_planes, int has_top, int has_bot, int64_t 
               int override_per_side, int *n_top, int *n_bot, int *n_int);
 // Choose ty (3D) maximising the lockstep utilisation of `n_int` interior CTAs.
 int choose_ty(int64_t ny, int units_x, int n_int, int smem_bytes, int ws);
+int tallest_ty(int64_t ny, int smem_bytes, int ws);
 int lockstep_k(int units, int n_int, int64_t inner_planes);
+// Number of plane blocks of the guided dynamic schedule (see JbSlab::dyn_min_blk).
+int64_t dyn_blocks(int64_t npl, int units, int n, int min_blk);
 size_t smem_bytes(const JbGeom &g);
 }  // namespace jbplan

@@ -208,19 +208,39 @@ __device__ Sched make_sched(const JbGeom &g, const JbSlab &S, int role, int ridx
   return s;
 }
 
-// Ring position q -> slot / parity.
+// Position in the shared-memory ring: slot and the parity of the current use of that slot.
+struct RingPos {
+  uint32_t slot, phase;
+  __device__ __forceinline__ void advance(uint32_t S) {
+    if (++slot == S) {
+      slot = 0;
+      phase ^= 1u;
+    }
+  }
+};
+
 struct Ring {
   uint64_t *full, *empty;
   double *stages;
-  int S;
-  __device__ __forceinline__ int slot(uint32_t q) const { return (int)(q % (uint32_t)S); }
-  __device__ __forceinline__ uint32_t parity(uint32_t q) const { return (q / (uint32_t)S) & 1u; }
+  uint32_t S;
+  int stage_doubles;
+  __device__ __forceinline__ double *stage(const RingPos &p) const {
+    return stages + (size_t)p.slot * stage_doubles;
+  }
+  __device__ __forceinline__ void wait_full(const RingPos &p) const { mbar_wait(&full[p.slot], p.phase); }
+  // Consumer warp releases a stage: all lanes are done reading it (syncwarp), one lane arrives.
+  __device__ __forceinline__ void release(const RingPos &p, int lane) const {
+    __syncwarp();
+    if (lane == 0) mbar_arrive(&empty[p.slot]);
+  }
 };
 
 // ---------------------------------------------------------------- producer
 // Load planes pf..pl of tile `unit` from `cur` into consecutive ring stages starting at q.
+// A stage holds the tile's rows (1 in 2D; ty + 2 in 3D incl. the y halo rows), each row the
+// x window [x0-2, x0+tx+2) of 16-byte aligned doubles, one cp.async.bulk per row.
 __device__ __forceinline__ void produce_planes(const JbGeom &g, const double *cur, int32_t unit,
-                                               int64_t pf, int64_t pl, uint32_t &q, const Ring &R,
+                                               int64_t pf, int64_t pl, RingPos &q, const Ring &R,
                                                int lane) {
   const int ux = unit % g.units_x, uy = unit / g.units_x;
   const int64_t xs = 2 + (int64_t)ux * g.tx;
@@ -233,86 +253,271 @@ __device__ __forceinline__ void produce_planes(const JbGeom &g, const double *cu
     const int64_t yb = min(ya + 1 + g.ty, g.ny - 1);
     nrows = (int)(yb - ya + 1);
   }
-  for (int64_t p = pf; p <= pl; ++p, ++q) {
-    const int s = R.slot(q);
+  const double *src = cur + pf * g.plane_elems + xs + ya * g.pitch + (int64_t)lane * g.pitch;
+  for (int64_t p = pf; p <= pl; ++p) {
     if (lane == 0) {
-      if (q >= (uint32_t)R.S) mbar_wait(&R.empty[s], R.parity(q) ^ 1u);
-      mbar_expect_tx(&R.full[s], row_bytes * (uint32_t)nrows);
+      // First pass: waiting on the parity of the (virtual) preceding phase returns at once.
+      mbar_wait(&R.empty[q.slot], q.phase ^ 1u);
+      mbar_expect_tx(&R.full[q.slot], row_bytes * (uint32_t)nrows);
     }
     __syncwarp();
-    if (lane < nrows) {
-      const double *src = cur + p * g.plane_elems + xs + (g.dim == 3 ? (ya + lane) * g.pitch : 0);
-      double *dst = R.stages + (size_t)s * g.stage_doubles + (size_t)lane * g.ws;
-      bulk_g2s(dst, src, row_bytes, &R.full[s]);
-    }
+    if (lane < nrows) bulk_g2s(R.stage(q) + (size_t)lane * g.ws, src, row_bytes, &R.full[q.slot]);
+    src += g.plane_elems;
+    q.advance(R.S);
   }
 }
 
 // ---------------------------------------------------------------- consumers
 __device__ __forceinline__ double2 lds2(const double *p) { return *reinterpret_cast<const double2 *>(p); }
 
-template <int DIM, bool NOCOMP>
-__device__ __forceinline__ void compute_plane(const JbGeom &g, int32_t unit, int64_t p, const double *sm,
-                                              const double *sc, const double *sp, double *nxt,
-                                              double *remote, int ctid) {
-  const int ux = unit % g.units_x, uy = unit / g.units_x;
-  const int64_t x0 = 1 + (int64_t)ux * g.tx;
-  const int vx = (int)min((int64_t)g.tx, g.nx - 1 - x0);  // valid cells in x
-  int64_t y0 = 0;
-  int vy = 1;
-  if (DIM == 3) {
-    y0 = 1 + (int64_t)uy * g.ty;
-    vy = (int)min((int64_t)g.ty, g.ny - 1 - y0);
-  }
-  const int sh = g.txp_shift;
-  const int txp_mask = (1 << sh) - 1;
-  const int total = vy << sh;
-  double *dst_plane = nxt ? nxt + p * g.plane_elems : nullptr;
-  for (int k = ctid; k < total; k += JB_NC) {
-    const int r = k >> sh, kk = k & txp_mask;
-    if (2 * kk >= vx) continue;
-    const int j = 2 + 2 * kk;
-    const int row = (DIM == 3) ? (r + 1) * g.ws : 0;
-    const double *c = sc + row;
-    double o0, o1;
-    if (NOCOMP) {
-      const double2 cc = lds2(c + j);
-      o0 = cc.x;
-      o1 = cc.y;
-    } else if (DIM == 2) {
-      const double2 cc = lds2(c + j);
-      const double w = c[j - 1], e = c[j + 2];
-      const double2 n = lds2(sp + j);  // y+1
-      const double2 s = lds2(sm + j);  // y-1
-      o0 = 0.25 * (((cc.y + w) + n.x) + s.x);
-      o1 = 0.25 * (((e + cc.x) + n.y) + s.y);
-    } else {
-      const double2 cc = lds2(c + j);
-      const double w = c[j - 1], e = c[j + 2];
-      const double2 n = lds2(c + g.ws + j);  // y+1
-      const double2 s = lds2(c - g.ws + j);  // y-1
-      const double2 u = lds2(sp + row + j);  // z+1
-      const double2 d = lds2(sm + row + j);  // z-1
-      o0 = kC6 * (((((cc.y + w) + n.x) + s.x) + u.x) + d.x);
-      o1 = kC6 * (((((e + cc.x) + n.y) + s.y) + u.y) + d.y);
-    }
-    const int64_t off = (DIM == 3 ? (y0 + r) * g.pitch : 0) + 3 + x0 + 2 * kk;
-    const bool pair = (2 * kk + 1) < vx;
-    if (dst_plane) {
-      if (pair) *reinterpret_cast<double2 *>(dst_plane + off) = make_double2(o0, o1);
-      else dst_plane[off] = o0;
-    }
-    if (remote) {
-      if (pair) *reinterpret_cast<double2 *>(remote + off) = make_double2(o0, o1);
-      else remote[off] = o0;
-    }
-  }
+__device__ __forceinline__ void store_pair(double *p, double o0, double o1, bool pair) {
+  if (pair) *reinterpret_cast<double2 *>(p) = make_double2(o0, o1);
+  else *p = o0;
 }
 
-__device__ __forceinline__ void release_stage(const Ring &R, uint32_t q, int lane) {
-  __syncwarp();
-  if (lane == 0) mbar_arrive(&R.empty[R.slot(q)]);
+// 2D: march one x strip of tx cells over planes (= rows) p0..p1.  Thread ctid owns the
+// cell pairs kk = ctid + i*NC (i < PPT), contiguous across lanes (conflict-free 16-byte LDS,
+// coalesced 16-byte STG).  Rows y-1 / y are carried in registers along the march, so each
+// plane costs one 16-byte LDS + two 8-byte LDS (x-1, x+2) per pair.
+template <int PPT, bool NOCOMP>
+__device__ __forceinline__ void consume_run_2d(const JbGeom &g, const Ring &R, RingPos &q, const Run &run,
+                                               double *nxt, double *remote, int ctid, int lane) {
+  const int64_t x0 = 1 + (int64_t)run.unit * g.tx;
+  const int vx = (int)min((int64_t)g.tx, g.nx - 1 - x0);
+  const int txp = g.tx >> 1;
+  // pair i of this thread: kk = ctid + i*NC, smem column j0 + 2*i*NC, global column col + 2*i*NC
+  const int j0 = 2 + 2 * ctid;
+  unsigned in_tile = 0, ok = 0, full = 0;
+#pragma unroll
+  for (int i = 0; i < PPT; ++i) {
+    const int kk = ctid + i * JB_NC;
+    in_tile |= (kk < txp ? 1u : 0u) << i;
+    ok |= (kk < txp && 2 * kk < vx ? 1u : 0u) << i;
+    full |= (2 * kk + 1 < vx ? 1u : 0u) << i;
+  }
+  const int64_t col = 3 + x0 + 2 * ctid;
+  const int64_t L = run.p1 - run.p0 + 1;
+  if (NOCOMP) {
+    for (int64_t p = 0; p < L; ++p) {
+      R.wait_full(q);
+      const double *sc = R.stage(q) + j0;
+#pragma unroll
+      for (int i = 0; i < PPT; ++i)
+        if ((ok >> i & 1u) && remote) {
+          const double2 v = lds2(sc + 2 * i * JB_NC);
+          store_pair(remote + col + 2 * i * JB_NC, v.x, v.y, full >> i & 1u);
+        }
+      R.release(q, lane);
+      q.advance(R.S);
+    }
+    return;
+  }
+  RingPos pm = q, pc = q;
+  pc.advance(R.S);
+  RingPos pp = pc;
+  pp.advance(R.S);
+  R.wait_full(pm);
+  R.wait_full(pc);
+  double2 S[PPT], C[PPT];
+#pragma unroll
+  for (int i = 0; i < PPT; ++i)
+    if (in_tile >> i & 1u) {
+      S[i] = lds2(R.stage(pm) + j0 + 2 * i * JB_NC);
+      C[i] = lds2(R.stage(pc) + j0 + 2 * i * JB_NC);
+    }
+  double *dst = nxt + run.p0 * g.plane_elems + col;
+  double *rem = remote ? remote + col : nullptr;
+  const int64_t pe = g.plane_elems;
+  for (int64_t p = 0; p < L; ++p) {
+    R.wait_full(pp);
+    const double *sc = R.stage(pc) + j0, *sn = R.stage(pp) + j0;
+#pragma unroll
+    for (int i = 0; i < PPT; ++i)
+      if (in_tile >> i & 1u) {
+        const double2 N = lds2(sn + 2 * i * JB_NC);
+        const double W = sc[2 * i * JB_NC - 1], E = sc[2 * i * JB_NC + 2];
+        // oracle order: ((x+1) + (x-1)) + (y+1) + (y-1), then * 0.25
+        const double o0 = 0.25 * (((C[i].y + W) + N.x) + S[i].x);
+        const double o1 = 0.25 * (((E + C[i].x) + N.y) + S[i].y);
+        if (ok >> i & 1u) {
+          store_pair(dst + 2 * i * JB_NC, o0, o1, full >> i & 1u);
+          if (rem) store_pair(rem + 2 * i * JB_NC, o0, o1, full >> i & 1u);
+        }
+        S[i] = C[i];
+        C[i] = N;
+      }
+    R.release(pm, lane);
+    pm = pc;
+    pc = pp;
+    pp.advance(R.S);
+    dst += pe;
+  }
+  R.release(pm, lane);
+  R.release(pc, lane);
+  q = pp;
 }
+
+// 3D: march one (ty rows x tx cells) tile over z planes p0..p1.  Thread ctid owns the x pair
+// kk = ctid % (tx/2) in a contiguous block of rows; along y it carries rows y-1 / y in
+// registers, so each cell row costs LDS: 16 B (y+1) + 8 B + 8 B (x-1, x+2) + 16 B (z+1) +
+// 16 B (z-1) per pair.
+template <bool NOCOMP>
+__device__ __forceinline__ void consume_run_3d(const JbGeom &g, const Ring &R, RingPos &q, const Run &run,
+                                               double *nxt, double *remote, int ctid, int lane) {
+  const int ux = run.unit % g.units_x, uy = run.unit / g.units_x;
+  const int64_t x0 = 1 + (int64_t)ux * g.tx;
+  const int vx = (int)min((int64_t)g.tx, g.nx - 1 - x0);
+  const int64_t y0 = 1 + (int64_t)uy * g.ty;
+  const int vy = (int)min((int64_t)g.ty, g.ny - 1 - y0);
+  const int txp = g.tx >> 1;
+  const int G = JB_NC / txp;  // row groups
+  const int kk = ctid & (txp - 1), rg = ctid / txp;
+  const int rpt = (g.ty + G - 1) / G;
+  const int rb = rg * rpt, re = min(rb + rpt, vy);
+  const int j = 2 + 2 * kk;
+  const bool ok = 2 * kk < vx, full = 2 * kk + 1 < vx;
+  const int ws = g.ws;
+  const int64_t col = (y0 + rb) * g.pitch + 3 + x0 + 2 * kk;
+  const int64_t L = run.p1 - run.p0 + 1;
+  const int srow = (rb + 1) * ws + j;  // stage offset of (row rb, pair kk) center
+  if (NOCOMP) {
+    for (int64_t p = 0; p < L; ++p) {
+      R.wait_full(q);
+      if (remote && ok) {
+        const double *c = R.stage(q) + srow;
+        double *o = remote + col;
+        for (int r = rb; r < re; ++r, c += ws, o += g.pitch) {
+          const double2 v = lds2(c);
+          store_pair(o, v.x, v.y, full);
+        }
+      }
+      R.release(q, lane);
+      q.advance(R.S);
+    }
+    return;
+  }
+  RingPos pm = q, pc = q;
+  pc.advance(R.S);
+  RingPos pp = pc;
+  pp.advance(R.S);
+  R.wait_full(pm);
+  R.wait_full(pc);
+  double *dst = nxt + run.p0 * g.plane_elems + col;
+  double *rem = remote ? remote + col : nullptr;
+  for (int64_t p = 0; p < L; ++p) {
+    R.wait_full(pp);
+    if (rb < re) {
+      const double *c = R.stage(pc) + srow;
+      const double *u = R.stage(pp) + srow;
+      const double *d = R.stage(pm) + srow;
+      double2 S = lds2(c - ws), C = lds2(c);
+      double *o = dst, *ro = rem;
+#pragma unroll 2
+      for (int r = rb; r < re; ++r) {
+        const double2 N = lds2(c + ws);
+        const double w = c[-1], e = c[2];
+        const double2 U = lds2(u), D = lds2(d);
+        // oracle order: x+1, x-1, y+1, y-1, z+1, z-1, then * fl(1/6)
+        const double o0 = kC6 * (((((C.y + w) + N.x) + S.x) + U.x) + D.x);
+        const double o1 = kC6 * (((((e + C.x) + N.y) + S.y) + U.y) + D.y);
+        if (ok) {
+          store_pair(o, o0, o1, full);
+          if (ro) store_pair(ro, o0, o1, full);
+        }
+        S = C;
+        C = N;
+        c += ws;
+        u += ws;
+        d += ws;
+        o += g.pitch;
+        if (ro) ro += g.pitch;
+      }
+    }
+    R.release(pm, lane);
+    pm = pc;
+    pc = pp;
+    pp.advance(R.S);
+    dst += g.plane_elems;
+  }
+  R.release(pm, lane);
+  R.release(pc, lane);
+  q = pp;
+}
+
+template <int DIM, bool NOCOMP>
+__device__ __forceinline__ void consume_run(const JbGeom &g, const Ring &R, RingPos &q, const Run &run,
+                                            double *nxt, double *remote, int ctid, int lane) {
+  if (DIM == 3) {
+    consume_run_3d<NOCOMP>(g, R, q, run, nxt, remote, ctid, lane);
+    return;
+  }
+  const int ppt = g.tx / (2 * JB_NC);
+  if (ppt >= 4) consume_run_2d<4, NOCOMP>(g, R, q, run, nxt, remote, ctid, lane);
+  else if (ppt == 2) consume_run_2d<2, NOCOMP>(g, R, q, run, nxt, remote, ctid, lane);
+  else consume_run_2d<1, NOCOMP>(g, R, q, run, nxt, remote, ctid, lane);
+}
+
+// ---------------------------------------------------------------- run-descriptor queue
+// The producer warp decides the work (static runs, then dynamically claimed interior items) and
+// hands each run to the consumer warps through a JB_RQ-deep queue of descriptors in shared
+// memory, guarded by its own full/empty mbarriers.
+enum { RUN_WORK = 0, RUN_SIGNAL = 1, RUN_END = 2 };
+struct RunDesc {
+  int32_t kind;
+  int32_t unit;
+  int64_t p0, p1;
+};
+struct Queue {
+  uint64_t *full, *empty;
+  RunDesc *desc;
+};
+
+__device__ __forceinline__ void publish(const Queue &Q, RingPos &qp, int kind, const Run &r, int lane) {
+  if (lane == 0) {
+    mbar_wait(&Q.empty[qp.slot], qp.phase ^ 1u);
+    RunDesc d;
+    d.kind = kind;
+    d.unit = r.unit;
+    d.p0 = r.p0;
+    d.p1 = r.p1;
+    Q.desc[qp.slot] = d;
+    mbar_arrive(&Q.full[qp.slot]);  // release: the descriptor is visible to the waiters
+  }
+  qp.advance(JB_RQ);
+}
+
+__device__ __forceinline__ RunDesc fetch(const Queue &Q, RingPos &qc, int lane) {
+  mbar_wait(&Q.full[qc.slot], qc.phase);
+  const RunDesc d = Q.desc[qc.slot];
+  __syncwarp();
+  if (lane == 0) mbar_arrive(&Q.empty[qc.slot]);
+  qc.advance(JB_RQ);
+  return d;
+}
+
+// Guided self-scheduling blocks: block k covers `size` planes starting at `start`.
+struct DynWalk {
+  int64_t idx, start, size, left;
+  int64_t units, n2, min_blk;
+  __device__ __forceinline__ int64_t next_size() const {
+    int64_t sz = (left * units + n2 - 1) / n2;
+    sz = max(sz, min_blk);
+    return min(sz, left);
+  }
+  __device__ __forceinline__ void init(int64_t lo, int64_t npl) {
+    idx = 0;
+    start = lo;
+    left = npl;
+    size = next_size();
+    left -= size;
+  }
+  __device__ __forceinline__ void advance() {
+    start += size;
+    size = next_size();
+    left -= size;
+    ++idx;
+  }
+};
 
 // ---------------------------------------------------------------- the kernel
 template <int DIM, bool NOCOMP, bool PERSIST>
@@ -321,10 +526,16 @@ __global__ void __launch_bounds__(JB_THREADS, 1) jb_sweep(const __grid_constant_
   __shared__ int s_abort;
   const JbGeom &g = P.g;
   Ring R;
-  R.S = g.stages;
+  R.S = (uint32_t)g.stages;
+  R.stage_doubles = g.stage_doubles;
   R.full = reinterpret_cast<uint64_t *>(smem);
   R.empty = R.full + R.S;
-  R.stages = reinterpret_cast<double *>(smem + ((2 * R.S * 8 + 127) & ~127));
+  Queue Q;
+  Q.full = R.empty + R.S;
+  Q.empty = Q.full + JB_RQ;
+  Q.desc = reinterpret_cast<RunDesc *>(Q.empty + JB_RQ);
+  const uint32_t hdr = 2 * R.S * 8 + 2 * JB_RQ * 8 + JB_RQ * 32;
+  R.stages = reinterpret_cast<double *>(smem + ((hdr + 127) & ~127u));
 
   int si = 0;
   while (si + 1 < P.nslabs && (int)blockIdx.x >= P.s[si + 1].cta_begin) ++si;
@@ -343,19 +554,31 @@ __global__ void __launch_bounds__(JB_THREADS, 1) jb_sweep(const __grid_constant_
   const int ctid = threadIdx.x;  // consumer thread id (valid when !producer)
 
   if (threadIdx.x == 0) {
-    for (int i = 0; i < R.S; ++i) {
+    for (uint32_t i = 0; i < R.S; ++i) {
       mbar_init(&R.full[i], 1);
       mbar_init(&R.empty[i], JB_NCW);
+    }
+    for (int i = 0; i < JB_RQ; ++i) {
+      mbar_init(&Q.full[i], 1);
+      mbar_init(&Q.empty[i], JB_NCW);
     }
     fence_mbar_init();
     s_abort = 0;
   }
   __syncthreads();
 
-  const Sched sched0 = make_sched(g, SL, role, ridx, rcount);
+  const bool dyn = !NOCOMP && SL.dyn_min_blk > 0 && SL.dyn_items > 0 &&
+                   (role == ROLE_INT || SL.dyn_help);
+  // With the dynamic schedule the interior has no static runs.
+  const Sched sched0 = (role == ROLE_INT && SL.dyn_min_blk > 0 && !NOCOMP)
+                           ? Sched{0, 0, 0, 0, 0, 0, 0, 0, 0}
+                           : make_sched(g, SL, role, ridx, rcount);
   const bool drop_signal = (P.flags & JACOBI_FLAG_DROP_SIGNAL) && SL.slab_id == 0;
   const int side = role == ROLE_TOP ? 0 : 1;
-  uint32_t q = 0;  // ring position (producer and consumers advance it identically)
+  const int64_t lo = SL.n_top ? 2 : 1;
+  const int64_t npl = (SL.n_bot ? SL.chunk - 1 : SL.chunk) - lo + 1;
+  RingPos q = {0u, 0u};   // data ring: producer and consumers advance identical copies
+  RingPos rq = {0u, 0u};  // run queue
 
   for (int64_t t = 0; t < P.iters; ++t) {
     const int64_t tg = P.t0 + t;
@@ -365,12 +588,12 @@ __global__ void __launch_bounds__(JB_THREADS, 1) jb_sweep(const __grid_constant_
     if (role == ROLE_TOP) remote = SL.peer_top[(tg + 1) & 1];
     if (role == ROLE_BOT) remote = SL.peer_bot[(tg + 1) & 1];
     const bool active = !(NOCOMP && role == ROLE_INT);
-    Sched sched = sched0;
-    Run run;
 
     if (producer) {
       if (lane == 0) {
         fence_proxy_async_global();
+        // The claim counter of the next iteration is idle now (last used in iteration t-1).
+        if (c == 0 && SL.work_ctr) SL.work_ctr[(tg + 1) & 1] = 0u;
         // wait until the neighbour committed the halo of the previous time step.
         if (PERSIST && role != ROLE_INT) {
           const unsigned long long *f = role == ROLE_TOP ? SL.flag_in_top : SL.flag_in_bot;
@@ -379,58 +602,68 @@ __global__ void __launch_bounds__(JB_THREADS, 1) jb_sweep(const __grid_constant_
         }
       }
       __syncwarp();
+      Sched sched = sched0;
+      Run run;
       if (active) {
         while (sched.next(run)) {
+          publish(Q, rq, RUN_WORK, run, lane);
           if (NOCOMP) produce_planes(g, cur, run.unit, run.p0, run.p1, q, R, lane);
           else produce_planes(g, cur, run.unit, run.p0 - 1, run.p1 + 1, q, R, lane);
         }
       }
-    } else {
-      if (active) {
-        while (sched.next(run)) {
-          const int64_t L = run.p1 - run.p0 + 1;
-          if (NOCOMP) {
-            for (int64_t i = 0; i < L; ++i, ++q) {
-              mbar_wait(&R.full[R.slot(q)], R.parity(q));
-              const double *sc = R.stages + (size_t)R.slot(q) * g.stage_doubles;
-              compute_plane<DIM, true>(g, run.unit, run.p0 + i, sc, sc, sc, nullptr, remote, ctid);
-              release_stage(R, q, lane);
-            }
-            continue;
-          }
-          mbar_wait(&R.full[R.slot(q)], R.parity(q));
-          mbar_wait(&R.full[R.slot(q + 1)], R.parity(q + 1));
-          for (int64_t i = 0; i < L; ++i) {
-            const uint32_t qm = q + (uint32_t)i, qc = qm + 1, qp = qm + 2;
-            mbar_wait(&R.full[R.slot(qp)], R.parity(qp));
-            const double *sm = R.stages + (size_t)R.slot(qm) * g.stage_doubles;
-            const double *sc = R.stages + (size_t)R.slot(qc) * g.stage_doubles;
-            const double *sp = R.stages + (size_t)R.slot(qp) * g.stage_doubles;
-            compute_plane<DIM, false>(g, run.unit, run.p0 + i, sm, sc, sp, nxt, remote, ctid);
-            release_stage(R, qm, lane);
-          }
-          release_stage(R, q + (uint32_t)L, lane);
-          release_stage(R, q + (uint32_t)L + 1, lane);
-          q += (uint32_t)L + 2;
+      if (PERSIST && role != ROLE_INT) publish(Q, rq, RUN_SIGNAL, run, lane);
+      if (dyn) {
+        DynWalk wk;
+        wk.units = g.units;
+        wk.n2 = 2 * (int64_t)SL.dyn_n;
+        wk.min_blk = SL.dyn_min_blk;
+        wk.init(lo, npl);
+        unsigned int *ctr = SL.work_ctr + (tg & 1);
+        while (true) {
+          unsigned int cl = 0;
+          if (lane == 0) cl = atomicAdd(ctr, 1u);
+          cl = __shfl_sync(0xffffffffu, cl, 0);
+          if ((int64_t)cl >= SL.dyn_items) break;
+          const int64_t b = cl / g.units;
+          while (wk.idx < b) wk.advance();
+          run.unit = (int32_t)(cl - b * g.units);
+          run.p0 = wk.start;
+          run.p1 = wk.start + wk.size - 1;
+          publish(Q, rq, RUN_WORK, run, lane);
+          produce_planes(g, cur, run.unit, run.p0 - 1, run.p1 + 1, q, R, lane);
         }
+      }
+      publish(Q, rq, RUN_END, run, lane);
+    } else {
+      while (true) {
+        const RunDesc d = fetch(Q, rq, lane);
+        if (d.kind == RUN_END) break;
+        if (d.kind == RUN_SIGNAL) {
+          // P:364-365 / P:394: signal the neighbour that the halo of iteration tg+1 is in place.
+          named_bar_consumers();
+          if (ctid == 0 && !drop_signal) {
+            fence_acq_rel_sys();
+            const unsigned int old = atom_acq_rel_gpu_add(&SL.side_ctr[side], 1u);
+            if (old == (unsigned int)(rcount * (t + 1) - 1)) {
+              fence_acq_rel_sys();
+              st_release_sys(role == ROLE_TOP ? SL.flag_out_top : SL.flag_out_bot,
+                             (unsigned long long)(tg + 1));
+            }
+          }
+          remote = nullptr;  // later (interior) runs stay local
+          continue;
+        }
+        Run run;
+        run.unit = d.unit;
+        run.p0 = d.p0;
+        run.p1 = d.p1;
+        consume_run<DIM, NOCOMP>(g, R, q, run, nxt, remote, ctid, lane);
       }
       // Our generic-proxy stores must be ordered before later bulk (async-proxy) reads.
       fence_proxy_async_global();
-      // P:364-365 / P:394: signal the neighbour that the halo of iteration tg+1 is in place.
-      if (PERSIST && role != ROLE_INT) {
-        named_bar_consumers();
-        if (ctid == 0 && !drop_signal) {
-          fence_acq_rel_sys();
-          const unsigned int old = atom_acq_rel_gpu_add(&SL.side_ctr[side], 1u);
-          if (old == (unsigned int)(rcount * (t + 1) - 1)) {
-            fence_acq_rel_sys();
-            st_release_sys(role == ROLE_TOP ? SL.flag_out_top : SL.flag_out_bot,
-                           (unsigned long long)(tg + 1));
-          }
-        }
-      }
     }
     if (!PERSIST) break;
+    if (P.trace && t < 8 && threadIdx.x == 0) P.trace[t * gridDim.x + blockIdx.x] = globaltimer();
 
     // Device-side grid barrier of this slab's CTAs (P:372 grid.sync()).
     __syncthreads();

@@ -27,7 +27,7 @@ void decompose(int64_t n_out, int nslabs, int slab, int64_t *start, int64_t *chu
 }
 
 size_t smem_bytes(const JbGeom &g) {
-  size_t bar = (size_t)2 * g.stages * 8;
+  size_t bar = (size_t)2 * g.stages * 8 + (size_t)2 * JB_RQ * 8 + (size_t)JB_RQ * 32;
   bar = (bar + 127) / 128 * 128;
   return bar + (size_t)g.stages * g.stage_doubles * 8;
 }
@@ -39,9 +39,12 @@ int geometry(int64_t nx, int64_t ny, int64_t nz, int dim, int tile_x, int tile_y
   g->pitch = round_up(nx + 3, 4);
   g->plane_elems = dim == 2 ? g->pitch : ny * g->pitch;
   const int64_t ix = nx - 2;
-  int64_t tx = tile_x > 0 ? pow2ceil(tile_x) : std::min<int64_t>(dim == 2 ? 1024 : 512, pow2ceil(ix));
+  // 2D: up to 4 cell pairs per consumer thread (tx <= 8*JB_NC); 3D: one x pair per thread and
+  // row group (tx <= 2*JB_NC).
+  const int64_t tx_max = dim == 2 ? 8 * JB_NC : 2 * JB_NC;
+  int64_t tx = tile_x > 0 ? pow2ceil(tile_x) : std::min<int64_t>(tx_max, pow2ceil(ix));
   tx = std::max<int64_t>(tx, 8);
-  if (tx > 4096) return -1;
+  if (tx > tx_max) return -1;
   g->tx = (int)tx;
   int sh = 0;
   while ((int64_t(1) << sh) < tx / 2) ++sh;
@@ -61,7 +64,7 @@ int geometry(int64_t nx, int64_t ny, int64_t nz, int dim, int tile_x, int tile_y
   g->units = g->units_x * g->units_y;
   g->stage_doubles = g->rh * g->ws;
   const size_t stage_b = (size_t)g->stage_doubles * 8;
-  int s = (int)((smem - 256) / (stage_b + 16));
+  int s = (int)((smem - 512) / (stage_b + 16));
   s = std::min(s, JB_MAX_STAGES);
   if (stages_req > 0) s = std::min(s, stages_req);
   if (s < 4) return -1;  // need p-1, p, p+1 resident + one in flight
@@ -99,6 +102,29 @@ int lockstep_k(int units, int n_int, int64_t inner) {
   int64_t k = n_int / units;
   k = std::min<int64_t>(k, inner);
   return (int)std::max<int64_t>(k, 1);
+}
+
+int64_t dyn_blocks(int64_t npl, int units, int n, int min_blk) {
+  int64_t rem = npl, nb = 0;
+  while (rem > 0) {
+    int64_t s = (rem * units + 2 * (int64_t)n - 1) / (2 * (int64_t)n);
+    s = std::max<int64_t>(s, min_blk);
+    s = std::min(s, rem);
+    rem -= s;
+    ++nb;
+  }
+  return nb;
+}
+
+int tallest_ty(int64_t ny, int smem, int ws) {
+  int best = 1;
+  for (int ty = 1; ty <= 12; ++ty) {
+    if (ty > std::max<int64_t>(ny - 2, 1)) break;
+    const size_t stage_b = (size_t)(ty + 2) * ws * 8;
+    if ((size_t)(smem - 512) / (stage_b + 16) < 5) break;
+    best = ty;
+  }
+  return best;
 }
 
 int choose_ty(int64_t ny, int units_x, int n_int, int smem, int ws) {

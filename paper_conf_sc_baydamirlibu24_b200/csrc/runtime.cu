@@ -10,6 +10,7 @@
 #include <algorithm>
 #include <cstdio>
 #include <cstdlib>
+#include <cstddef>
 #include <cstring>
 #include <string>
 #include <vector>
@@ -117,6 +118,7 @@ struct jacobi_ctx {
   int64_t t = 0;
   int mode = JACOBI_MODE_CPUFREE, flags = 0;
   int64_t tile_x = -1, tile_y = -1, stages = -1, boundary_ctas = -1, ctas = -1, schedule = -1;
+  int64_t min_block = 8, dyn_help = 1;
   int64_t timeout_ms = 20000;
   bool peers_ready = false;
   bool nccl_ready = false;
@@ -236,7 +238,10 @@ int plan_launch(jacobi_ctx *h, const std::vector<int> &idx, bool persist, bool n
   if (h->ctas > 0) total_ctas = (int)std::min<int64_t>(h->ctas * nslab, sms);
   const int per = total_ctas / nslab;
   if (h->dim == 3 && h->tile_y <= 0) {
-    int ty = jbplan::choose_ty(h->ny, g.units_x, per - (h->total > 1 ? 2 : 0), smem_optin, g.ws);
+    // Static lockstep: pick ty for utilisation; dynamic: the tallest tile that keeps a >= 5-deep
+    // ring (fewest y-halo rows per row).
+    int ty = h->schedule == 1 ? jbplan::choose_ty(h->ny, g.units_x, per - (h->total > 1 ? 2 : 0), smem_optin, g.ws)
+                              : jbplan::tallest_ty(h->ny, smem_optin, g.ws);
     if (jbplan::geometry(h->nx, h->ny, h->nz, h->dim, (int)h->tile_x, ty, smem_optin, (int)h->stages, &g))
       return JACOBI_EINVAL;
   }
@@ -281,13 +286,29 @@ int plan_launch(jacobi_ctx *h, const std::vector<int> &idx, bool persist, bool n
     jbplan::tb_split(count, inner, top, bot, g.units, (int)h->boundary_ctas, &nt, &nb, &ni);
     d.n_top = nt;
     d.n_bot = nb;
-    const bool lockstep = h->schedule == 1 || (h->schedule < 0 && h->dim == 3);
+    const bool dynamic = h->schedule == 2 || h->schedule < 0;
+    const bool lockstep = h->schedule == 1;
     d.k_planes = lockstep ? jbplan::lockstep_k(g.units, ni, inner) : 0;
+    d.work_ctr = s.ctrl->work;
+    if (dynamic && inner > 0) {
+      // Guided self-scheduling over every CTA of the slab (boundary CTAs join after signalling).
+      d.dyn_min_blk = (int)std::max<int64_t>(1, h->min_block);
+      d.dyn_help = (h->dyn_help != 0) ? 1 : 0;
+      d.dyn_n = d.dyn_help ? count : ni;
+      d.dyn_items = (int64_t)g.units * jbplan::dyn_blocks(inner, g.units, d.dyn_n, d.dyn_min_blk);
+    }
     s.desc = d;
     s.grid = count;
     s.smem = L.smem;
   }
   return JACOBI_OK;
+}
+
+// Zero the per-run counters of a slab: barrier, side counters, status, claim counters.
+cudaError_t reset_run_counters(Slab &s, cudaStream_t st) {
+  static_assert(offsetof(JbCtrl, work) + sizeof(JbCtrl::work) - offsetof(JbCtrl, barrier) == 32,
+                "JbCtrl per-run counters must be contiguous");
+  return cudaMemsetAsync(&s.ctrl->barrier, 0, 32, st);
 }
 
 int read_status(Slab &s) {
@@ -325,10 +346,16 @@ int run_cpufree(jacobi_ctx *h, int64_t iters) {
     CK(cudaSetDevice(L.device));
     for (int k : L.slab_idx) {
       Slab &s = h->slabs[k];
-      CK(cudaMemsetAsync(&s.ctrl->barrier, 0,
-                         sizeof(s.ctrl->barrier) + sizeof(s.ctrl->side_ctr) + sizeof(s.ctrl->status),
-                         L.stream));
+      CK(reset_run_counters(s, L.stream));
     }
+  }
+  // Debug: JACOBI_TRACE=1 records when each CTA finished its work in the first 8 iterations.
+  unsigned long long *trace = nullptr;
+  const bool tracing = getenv("JACOBI_TRACE") && plans.size() == 1;
+  if (tracing) {
+    CK(cudaMalloc(&trace, 8 * plans[0].grid * sizeof(unsigned long long)));
+    CK(cudaMemset(trace, 0, 8 * plans[0].grid * sizeof(unsigned long long)));
+    plans[0].P.trace = trace;
   }
   // One host thread launches every GPU's persistent kernel back to back (co-residency across
   // GPUs only needs every kernel to start; the device watchdog bounds any wait).
@@ -353,6 +380,28 @@ int run_cpufree(jacobi_ctx *h, int64_t iters) {
     if (rc && !rc_all) rc_all = rc;
   }
   h->last_ms_max = mx;
+  if (tracing) {
+    const int n = plans[0].grid;
+    std::vector<unsigned long long> tr(8 * n);
+    CK(cudaMemcpy(tr.data(), trace, tr.size() * 8, cudaMemcpyDeviceToHost));
+    cudaFree(trace);
+    for (int it = 1; it < 8 && it < iters; ++it) {
+      std::vector<double> d;
+      unsigned long long t0 = ~0ull;
+      for (int c = 0; c < n; ++c) t0 = std::min(t0, tr[(it - 1) * n + c]);
+      for (int c = 0; c < n; ++c) d.push_back((tr[it * n + c] - t0) / 1e3);
+      std::vector<double> s = d;
+      std::sort(s.begin(), s.end());
+      fprintf(stderr, "[trace] it %d work-end us after prev barrier: min %.1f med %.1f max %.1f | slowest ctas:",
+              it, s[0], s[n / 2], s[n - 1]);
+      for (int k = 0; k < 4; ++k) {
+        int arg = (int)(std::max_element(d.begin(), d.end()) - d.begin());
+        fprintf(stderr, " %d(%.1f)", arg, d[arg]);
+        d[arg] = -1;
+      }
+      fprintf(stderr, "\n");
+    }
+  }
   if (rc_all) return rc_all;
   h->t += iters;
   return JACOBI_OK;
@@ -395,6 +444,7 @@ int run_baseline(jacobi_ctx *h, int64_t iters, bool nccl) {
   const size_t plane_bytes = (size_t)pe * sizeof(double);
   for (int i = 0; i < n; ++i) {
     CK(cudaSetDevice(h->slabs[i].device));
+    CK(reset_run_counters(h->slabs[i], h->slabs[i].stream));
     CK(cudaEventRecord(h->slabs[i].ev0, h->slabs[i].stream));
   }
   for (int64_t it = 0; it < iters; ++it) {
@@ -674,6 +724,8 @@ static int64_t *param_slot(jacobi_t h, const char *name) {
   if (!std::strcmp(name, "ctas")) return &h->ctas;
   if (!std::strcmp(name, "schedule")) return &h->schedule;
   if (!std::strcmp(name, "timeout_ms")) return &h->timeout_ms;
+  if (!std::strcmp(name, "min_block")) return &h->min_block;
+  if (!std::strcmp(name, "dyn_help")) return &h->dyn_help;
   return nullptr;
 }
 

@@ -72,7 +72,7 @@ def test_3d_shapes(shape, iters):
     assert_bitwise(run_gpu(f, iters, params={"tile_y": 3, "tile_x": 16}), exp, f"3D {shape} ty3")
 
 
-@pytest.mark.parametrize("sched", [0, 1])
+@pytest.mark.parametrize("sched", [0, 1, 2])
 @pytest.mark.parametrize("stages", [4, 7])
 def test_schedules_and_ring_depths(sched, stages):
     for shape in [(130, 333), (11, 40, 50)]:
@@ -105,6 +105,15 @@ def test_virtual_many_boundary_ctas():
     for bc in (1, 2, 4):
         got = run_gpu(f, 11, virtual=4, params={"boundary_ctas": bc, "tile_x": 128})
         assert_bitwise(got, exp, f"boundary_ctas={bc}")
+
+
+@pytest.mark.parametrize("min_block,help_", [(1, 1), (3, 0), (64, 1)])
+def test_dynamic_schedule_knobs(min_block, help_):
+    for shape, P in [((70, 1030), 3), ((23, 40, 130), 2), ((300, 77), 1)]:
+        f = u12(shape, 4)
+        exp = oracle.jacobi(f, 7)
+        got = run_gpu(f, 7, virtual=P, params={"schedule": 2, "min_block": min_block, "dyn_help": help_})
+        assert_bitwise(got, exp, f"{shape} P={P} min_block={min_block} help={help_}")
 
 
 def test_virtual_c5_latency_shapes_long():
