@@ -1,0 +1,87 @@
+#!/usr/bin/env python
+"""bench_latency.py — the communication-bound latency sweep of BASELINE.json configs[4] (C5):
+3D 128^3 and 2D 1024^2, CPU-Free persistent kernel vs the CPU-controlled baseline (one kernel
+launch per iteration + cudaMemcpyPeerAsync halo copies + host synchronisation), with
+and without compute (the "no compute" runs of P:238-241), at P = 2/4/8 slabs.
+
+On a 1-GPU box the P slabs are VIRTUAL (jacobi_create_virtual: P slab groups of thread blocks
+on one device running the complete flag/halo protocol; the baseline launches P kernels and
+2(P-1) peer copies per iteration on the same device).  This measures the orchestration cost
+(launch + host sync vs device flags + grid barrier) that the paper's claim is about; it does
+not exercise NVLink.  Per-iteration time = (T(2N) - T(N)) / N, cancelling launch skew.
+
+    python bench_latency.py [--iters N] [--out profiles/latency.json]
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import sys
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+if ROOT not in sys.path:
+    sys.path.insert(0, ROOT)
+
+import paper_conf_sc_baydamirlibu24_b200 as jb  # noqa: E402
+
+SHAPES = {"C5a 3D 128^3": (128, 128, 128), "C5b 2D 1024^2": (1, 1024, 1024)}
+MODES = {"cpufree": jb.MODE_CPUFREE, "baseline_memcpy": jb.MODE_BASELINE_MEMCPY}
+
+
+def per_iter_us(j: jb.Jacobi, n: int, reps: int = 3) -> float:
+    best = None
+    for _ in range(reps):
+        j.run(n)
+        t1 = j.last_time_ms()
+        j.run(2 * n)
+        t2 = j.last_time_ms()
+        v = (t2 - t1) * 1e3 / n
+        best = v if best is None else min(best, v)
+    return best
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--iters", type=int, default=500)
+    ap.add_argument("--slabs", default="1,2,4,8")
+    ap.add_argument("--out", default="")
+    args = ap.parse_args()
+    rows = []
+    for name, shape in SHAPES.items():
+        for P in [int(p) for p in args.slabs.split(",")]:
+            with jb.Jacobi(shape, virtual=P) if P > 1 else jb.Jacobi(shape) as j:
+                for mname, mode in MODES.items():
+                    for nocomp in (False, True):
+                        j.set_mode(mode, jb.FLAG_NO_COMPUTE if nocomp else 0)
+                        j.run(50)  # warm-up
+                        us = per_iter_us(j, args.iters)
+                        row = {"config": name, "slabs": P, "virtual": P > 1, "mode": mname,
+                               "no_compute": nocomp, "us_per_iter": round(us, 3)}
+                        if not nocomp:
+                            cells = (shape[2] - 2) * (shape[1] - 2) * (shape[0] - 2 if shape[0] > 1 else 1)
+                            row["gcells_per_s"] = round(cells / us / 1e3, 2)
+                        rows.append(row)
+                        print(json.dumps(row), flush=True)
+    # CPU-Free vs baseline: time reduction % per config / P / compute
+    summary = []
+    for r in rows:
+        if r["mode"] != "cpufree":
+            continue
+        b = next(x for x in rows if x["mode"] == "baseline_memcpy" and x["config"] == r["config"]
+                 and x["slabs"] == r["slabs"] and x["no_compute"] == r["no_compute"])
+        summary.append({"config": r["config"], "slabs": r["slabs"], "no_compute": r["no_compute"],
+                        "cpufree_us": r["us_per_iter"], "baseline_us": b["us_per_iter"],
+                        "reduction_pct": round(100 * (b["us_per_iter"] - r["us_per_iter"]) / b["us_per_iter"], 1),
+                        "ratio": round(b["us_per_iter"] / r["us_per_iter"], 2)})
+    for s in summary:
+        print(json.dumps({"summary": s}), flush=True)
+    if args.out:
+        with open(args.out, "w") as f:
+            json.dump({"rows": rows, "summary": summary,
+                       "note": "virtual slabs on one B200 (see module docstring); paper's 58.8% (8xA100) is context only"},
+                      f, indent=1)
+
+
+if __name__ == "__main__":
+    main()

@@ -640,15 +640,16 @@ __global__ void __launch_bounds__(JB_THREADS, 1) jb_sweep(const __grid_constant_
         if (d.kind == RUN_END) break;
         if (d.kind == RUN_SIGNAL) {
           // P:364-365 / P:394: signal the neighbour that the halo of iteration tg+1 is in place.
+          // bar.sync orders every consumer thread's peer stores before thread 0 (CTA scope);
+          // the sys-scope fence publishes them system-wide before the local counter update; the
+          // last boundary CTA of this side then sets the flag with a sys-scope release store.
           named_bar_consumers();
           if (ctid == 0 && !drop_signal) {
             fence_acq_rel_sys();
             const unsigned int old = atom_acq_rel_gpu_add(&SL.side_ctr[side], 1u);
-            if (old == (unsigned int)(rcount * (t + 1) - 1)) {
-              fence_acq_rel_sys();
+            if (old == (unsigned int)(rcount * (t + 1) - 1))
               st_release_sys(role == ROLE_TOP ? SL.flag_out_top : SL.flag_out_bot,
                              (unsigned long long)(tg + 1));
-            }
           }
           remote = nullptr;  // later (interior) runs stay local
           continue;

@@ -283,10 +283,16 @@ int plan_launch(jacobi_ctx *h, const std::vector<int> &idx, bool persist, bool n
     const int64_t inner = hi - lo + 1;
     int nt, nb, ni;
     if (count < (top ? 1 : 0) + (bot ? 1 : 0) + (inner > 0 ? 1 : 0)) return JACOBI_ENOCOOP;
-    jbplan::tb_split(count, inner, top, bot, g.units, (int)h->boundary_ctas, &nt, &nb, &ni);
+    const bool dynamic = h->schedule == 2 || h->schedule < 0;
+    int override_ps = (int)h->boundary_ctas;
+    if (override_ps <= 0 && dynamic && h->dyn_help && inner > 0 && (top || bot)) {
+      // Boundary CTAs join the dynamic interior after signalling, so give every boundary unit
+      // its own CTA (shortest halo critical path), up to a quarter of the grid per side.
+      override_ps = (int)std::max<int64_t>(1, std::min<int64_t>(g.units, count / 4));
+    }
+    jbplan::tb_split(count, inner, top, bot, g.units, override_ps, &nt, &nb, &ni);
     d.n_top = nt;
     d.n_bot = nb;
-    const bool dynamic = h->schedule == 2 || h->schedule < 0;
     const bool lockstep = h->schedule == 1;
     d.k_planes = lockstep ? jbplan::lockstep_k(g.units, ni, inner) : 0;
     d.work_ctr = s.ctrl->work;

@@ -1,0 +1,101 @@
+"""GPU parity at BASELINE.json's full sizes, in the launch configuration bench.py times.
+
+* C2 (2D 16384^2): 3 iterations compared cell-for-cell with the (OpenMP) oracle; 1000
+  iterations compared on sampled sub-domains the oracle can compute exactly: after k sweeps a
+  cell depends only on cells within distance k, so the oracle run on a box whose artificial
+  faces are > k cells away reproduces those cells bit for bit (light-cone sampling).
+* C3 (3D 512^3): 5 iterations cell-for-cell; 1000 iterations P = 8 virtual slabs bit-identical
+  to P = 1 and to the CPU-controlled baseline (decomposition invariance).
+* C4 (weak scaling, P = 2 shape 1024x512x512): P = 2 slabs == P = 1.
+"""
+import os
+
+import numpy as np
+import pytest
+
+import oracle
+import paper_conf_sc_baydamirlibu24_b200 as jb
+from jacobi_inputs import SEED_BENCH, u12
+
+pytestmark = pytest.mark.gpu
+THREADS = os.cpu_count() or 1
+
+
+def bits_equal(a, b):
+    return np.array_equal(np.asarray(a).view(np.uint64), np.asarray(b).view(np.uint64))
+
+
+def run(shape, iters, virtual=0, mode=jb.MODE_CPUFREE, field=None):
+    with jb.Jacobi(shape, virtual=virtual) as j:
+        j.set_mode(mode)
+        if field is not None:
+            j.scatter(field)
+        j.run(iters)
+        return j.gather()
+
+
+def cone_box_check(got, f, iters, corner):
+    """Compare `got` with the oracle on the box of size 2*iters+3 at `corner` (one of the domain
+    corners, so two faces per axis are real Dirichlet faces) on the cells whose distance to every
+    artificial face exceeds `iters`."""
+    k = iters
+    sl, ex = [], []
+    for ax, c in enumerate(corner):
+        n = f.shape[ax]
+        w = min(n, 2 * k + 3)
+        if c == 0:
+            lo, hi = 0, w
+            exact = slice(0, w - (k + 1)) if w < n else slice(0, w)
+        else:
+            lo, hi = n - w, n
+            exact = slice(k + 1, w) if w < n else slice(0, w)
+        sl.append(slice(lo, hi))
+        ex.append(exact)
+    box = np.ascontiguousarray(f[tuple(sl)])
+    ref = oracle.jacobi(box, iters, THREADS)
+    g = got[tuple(sl)]
+    assert bits_equal(g[tuple(ex)], ref[tuple(ex)]), f"cone sample at {corner} differs"
+    return ref[tuple(ex)].size
+
+
+@pytest.fixture(scope="module")
+def c2_field():
+    return u12((16384, 16384), SEED_BENCH)
+
+
+def test_c2_full_grid_3_iters(c2_field):
+    got = run((16384, 16384), 3)  # device-side U12 init == c2_field
+    exp = oracle.jacobi(c2_field, 3, THREADS)
+    assert bits_equal(got, exp)
+
+
+def test_c2_1000_iters_cone_samples(c2_field):
+    got = run((16384, 16384), 1000)
+    n = 0
+    for corner in [(0, 0), (16383, 16383), (0, 16383)]:
+        n += cone_box_check(got, c2_field, 1000, corner)
+    assert n > 3 * 1000 * 1000
+    # and the slab decomposition does not change a bit at full length
+    assert bits_equal(run((16384, 16384), 1000, virtual=8), got)
+
+
+def test_c3_full_grid_5_iters():
+    f = u12((512, 512, 512), SEED_BENCH)
+    got = run((512, 512, 512), 5)
+    assert bits_equal(got, oracle.jacobi(f, 5, THREADS))
+
+
+def test_c3_1000_iters_decomposition_and_baseline():
+    shape = (512, 512, 512)
+    ref = run(shape, 1000)
+    assert bits_equal(run(shape, 1000, virtual=8), ref)
+    assert bits_equal(run(shape, 1000, virtual=4, mode=jb.MODE_BASELINE_MEMCPY), ref)
+    # sanity: the field actually evolved and kept the maximum principle
+    f = u12((4, 4, 4), SEED_BENCH)  # any U12 values are in [1, 2)
+    assert ref.min() >= 1.0 and ref.max() < 2.0 and f.min() >= 1.0
+
+
+def test_c4_weak_p2_shape():
+    shape = (1024, 512, 512)
+    ref = run(shape, 50)
+    assert bits_equal(run(shape, 50, virtual=2), ref)
