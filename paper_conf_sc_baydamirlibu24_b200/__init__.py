@@ -320,20 +320,35 @@ class Jacobi:
             pass
 
 
-def exchange_peers(j: Jacobi, group=None, nccl: bool = True) -> None:
-    """Dist mode plumbing: all-gather every rank's IPC blob over torch.distributed, attach the
-    neighbours, and (optionally) set up the NCCL communicator of the baseline."""
+def exchange_blobs(blob: bytes, group=None):
+    """All-gather one opaque blob per rank over torch.distributed; return (top, bottom): the
+    blobs of ranks rank-1 and rank+1 (None at the ends of the slab chain)."""
     import torch.distributed as dist
 
-    blob = jacobi_get_ipc_handle(j.h)
     world = dist.get_world_size(group)
     rank = dist.get_rank(group)
     blobs = [None] * world
     dist.all_gather_object(blobs, blob, group=group)
     top = blobs[rank - 1] if rank > 0 else None
     bot = blobs[rank + 1] if rank < world - 1 else None
+    return top, bot
+
+
+def broadcast_blob(blob_on_rank0, group=None):
+    import torch.distributed as dist
+
+    obj = [blob_on_rank0]
+    dist.broadcast_object_list(obj, src=0, group=group)
+    return obj[0]
+
+
+def exchange_peers(j: Jacobi, group=None, nccl: bool = True) -> None:
+    """Dist mode plumbing: all-gather every rank's IPC blob over torch.distributed, attach the
+    neighbours, and (optionally) set up the NCCL communicator of the baseline."""
+    import torch.distributed as dist
+
+    top, bot = exchange_blobs(jacobi_get_ipc_handle(j.h), group)
     jacobi_open_peers(j.h, top, bot)
     if nccl:
-        uid = [jacobi_nccl_unique_id() if rank == 0 else None]
-        dist.broadcast_object_list(uid, src=0, group=group)
-        jacobi_nccl_init(j.h, uid[0])
+        uid = broadcast_blob(jacobi_nccl_unique_id() if dist.get_rank(group) == 0 else None, group)
+        jacobi_nccl_init(j.h, uid)
