@@ -29,16 +29,17 @@ SHAPES = {"C5a 3D 128^3": (128, 128, 128), "C5b 2D 1024^2": (1, 1024, 1024)}
 MODES = {"cpufree": jb.MODE_CPUFREE, "baseline_memcpy": jb.MODE_BASELINE_MEMCPY}
 
 
-def per_iter_us(j: jb.Jacobi, n: int, reps: int = 3) -> float:
-    best = None
+def per_iter_us(j: jb.Jacobi, n: int, reps: int = 5) -> float:
+    """Median over `reps` of (T(2n) - T(n)) / n: cancels the fixed launch/teardown cost."""
+    vals = []
     for _ in range(reps):
         j.run(n)
         t1 = j.last_time_ms()
         j.run(2 * n)
         t2 = j.last_time_ms()
-        v = (t2 - t1) * 1e3 / n
-        best = v if best is None else min(best, v)
-    return best
+        vals.append((t2 - t1) * 1e3 / n)
+    vals.sort()
+    return vals[len(vals) // 2]
 
 
 def main():
