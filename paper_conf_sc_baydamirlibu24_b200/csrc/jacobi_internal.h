@@ -49,11 +49,15 @@ struct JbSlab {
   // Dynamic (guided self-scheduling) interior work, used when dyn_min_blk > 0: items are
   // (plane block, unit) pairs claimed from work_ctr[t & 1] in block-major order; block k has
   // max(dyn_min_blk, ceil(rem * units / (2 * dyn_n))) planes (rem = planes not yet blocked).
+  // Item c -> block b = c / units, unit u = c % units; planes lo + dyn_table[b] ..
+  // lo + dyn_table[b+1] - 1 (host-built table).  Interior CTA i starts with item i (no claim);
+  // further items are dyn_first + atomicAdd(work_ctr[t & 1], 1).
   unsigned int *work_ctr;            // local [2], one per iteration parity
+  const int32_t *dyn_table;          // device, nblocks + 1 entries
   int32_t dyn_min_blk;
   int32_t dyn_n;
   int32_t dyn_help;                  // boundary CTAs join the interior after signalling
-  int32_t pad1;
+  int32_t dyn_first;                 // items handed out statically (one per interior CTA)
   int64_t dyn_items;                 // units * number of blocks
 };
 
@@ -93,6 +97,6 @@ int choose_ty(int64_t ny, int units_x, int n_int, int smem_bytes, int ws);
 int tallest_ty(int64_t ny, int smem_bytes, int ws);
 int lockstep_k(int units, int n_int, int64_t inner_planes);
 // Number of plane blocks of the guided dynamic schedule (see JbSlab::dyn_min_blk).
-int64_t dyn_blocks(int64_t npl, int units, int n, int min_blk);
+int64_t dyn_blocks(int64_t npl, int units, int n, int min_blk, int32_t *table = nullptr);
 size_t smem_bytes(const JbGeom &g);
 }  // namespace jbplan

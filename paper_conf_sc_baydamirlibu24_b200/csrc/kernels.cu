@@ -495,30 +495,6 @@ __device__ __forceinline__ RunDesc fetch(const Queue &Q, RingPos &qc, int lane) 
   return d;
 }
 
-// Guided self-scheduling blocks: block k covers `size` planes starting at `start`.
-struct DynWalk {
-  int64_t idx, start, size, left;
-  int64_t units, n2, min_blk;
-  __device__ __forceinline__ int64_t next_size() const {
-    int64_t sz = (left * units + n2 - 1) / n2;
-    sz = max(sz, min_blk);
-    return min(sz, left);
-  }
-  __device__ __forceinline__ void init(int64_t lo, int64_t npl) {
-    idx = 0;
-    start = lo;
-    left = npl;
-    size = next_size();
-    left -= size;
-  }
-  __device__ __forceinline__ void advance() {
-    start += size;
-    size = next_size();
-    left -= size;
-    ++idx;
-  }
-};
-
 // ---------------------------------------------------------------- the kernel
 template <int DIM, bool NOCOMP, bool PERSIST>
 __global__ void __launch_bounds__(JB_THREADS, 1) jb_sweep(const __grid_constant__ JbParams P) {
@@ -576,7 +552,6 @@ __global__ void __launch_bounds__(JB_THREADS, 1) jb_sweep(const __grid_constant_
   const bool drop_signal = (P.flags & JACOBI_FLAG_DROP_SIGNAL) && SL.slab_id == 0;
   const int side = role == ROLE_TOP ? 0 : 1;
   const int64_t lo = SL.n_top ? 2 : 1;
-  const int64_t npl = (SL.n_bot ? SL.chunk - 1 : SL.chunk) - lo + 1;
   RingPos q = {0u, 0u};   // data ring: producer and consumers advance identical copies
   RingPos rq = {0u, 0u};  // run queue
 
@@ -613,24 +588,30 @@ __global__ void __launch_bounds__(JB_THREADS, 1) jb_sweep(const __grid_constant_
       }
       if (PERSIST && role != ROLE_INT) publish(Q, rq, RUN_SIGNAL, run, lane);
       if (dyn) {
-        DynWalk wk;
-        wk.units = g.units;
-        wk.n2 = 2 * (int64_t)SL.dyn_n;
-        wk.min_blk = SL.dyn_min_blk;
-        wk.init(lo, npl);
+        // Guided self-scheduling (block-major items, host-built block table).  Interior CTA
+        // i's first item is item i; every further item is claimed with one atomicAdd, issued
+        // before the previous item's loads so its latency overlaps them.
         unsigned int *ctr = SL.work_ctr + (tg & 1);
-        while (true) {
-          unsigned int cl = 0;
-          if (lane == 0) cl = atomicAdd(ctr, 1u);
-          cl = __shfl_sync(0xffffffffu, cl, 0);
-          if ((int64_t)cl >= SL.dyn_items) break;
-          const int64_t b = cl / g.units;
-          while (wk.idx < b) wk.advance();
-          run.unit = (int32_t)(cl - b * g.units);
-          run.p0 = wk.start;
-          run.p1 = wk.start + wk.size - 1;
+        int64_t item = (role == ROLE_INT && ridx < SL.dyn_first) ? ridx : -1;
+        unsigned int claim = 0;
+        if (item < 0) {
+          if (lane == 0) claim = atomicAdd(ctr, 1u);
+          item = SL.dyn_first + (int64_t)__shfl_sync(0xffffffffu, claim, 0);
+        }
+        while (item < SL.dyn_items) {
+          const int64_t b = item / g.units;
+          run.unit = (int32_t)(item - b * g.units);
+          run.p0 = lo + SL.dyn_table[b];
+          run.p1 = lo + SL.dyn_table[b + 1] - 1;
+          // Claim the next item now if this one fits in the ring (its loads are issued at once,
+          // so the atomic's latency hides behind them); for a long item claim only after its
+          // loads are issued, or the claim would reserve work long before it is needed.
+          const bool early = run.p1 - run.p0 + 3 <= (int64_t)R.S;
+          if (early && lane == 0) claim = atomicAdd(ctr, 1u);
           publish(Q, rq, RUN_WORK, run, lane);
           produce_planes(g, cur, run.unit, run.p0 - 1, run.p1 + 1, q, R, lane);
+          if (!early && lane == 0) claim = atomicAdd(ctr, 1u);
+          item = SL.dyn_first + (int64_t)__shfl_sync(0xffffffffu, claim, 0);
         }
       }
       publish(Q, rq, RUN_END, run, lane);

@@ -104,15 +104,21 @@ int lockstep_k(int units, int n_int, int64_t inner) {
   return (int)std::max<int64_t>(k, 1);
 }
 
-int64_t dyn_blocks(int64_t npl, int units, int n, int min_blk) {
+int64_t dyn_blocks(int64_t npl, int units, int n, int min_blk, int32_t *table) {
+  // Guided self-scheduling: each block hands every unit rem/(f*n) of the remaining work.  When a
+  // CTA's share is small (< 4 minimum blocks) use f = 1 so the first round covers everything
+  // (latency-bound grids); otherwise f = 2 (half the work in the first round, shrinking tail).
+  const int64_t f = (npl * units < 4 * (int64_t)min_blk * n) ? 1 : 2;
   int64_t rem = npl, nb = 0;
   while (rem > 0) {
-    int64_t s = (rem * units + 2 * (int64_t)n - 1) / (2 * (int64_t)n);
+    if (table) table[nb] = (int32_t)(npl - rem);
+    int64_t s = (rem * units + f * (int64_t)n - 1) / (f * (int64_t)n);
     s = std::max<int64_t>(s, min_blk);
     s = std::min(s, rem);
     rem -= s;
     ++nb;
   }
+  if (table) table[nb] = (int32_t)npl;
   return nb;
 }
 

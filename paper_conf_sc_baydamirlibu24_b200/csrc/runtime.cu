@@ -104,6 +104,8 @@ struct Slab {
   ncclComm_t comm = nullptr;
   double last_ms = 0;
   JbSlab desc{};  // last launch descriptor (for jacobi_describe)
+  int32_t *dyn_table = nullptr;  // guided-schedule block table (device)
+  int64_t dyn_key[4] = {0, 0, 0, 0};
   int grid = 0;
   size_t smem = 0;
 };
@@ -176,6 +178,7 @@ void free_slab(Slab &s) {
   if (s.buf[0]) cudaFree(s.buf[0]);
   if (s.buf[1]) cudaFree(s.buf[1]);
   if (s.ctrl) cudaFree(s.ctrl);
+  if (s.dyn_table) cudaFree(s.dyn_table);
   if (s.ev0) cudaEventDestroy(s.ev0);
   if (s.ev1) cudaEventDestroy(s.ev1);
   if (s.stream) cudaStreamDestroy(s.stream);
@@ -204,6 +207,20 @@ void link_local(jacobi_ctx *h) {
     }
   }
   h->peers_ready = true;
+}
+
+// Device copy of the guided-schedule block table of a slab (rebuilt when its key changes).
+int upload_table(Slab &s, int64_t npl, int units, int n, int min_blk, int64_t nb) {
+  const int64_t key[4] = {npl, units, n, min_blk};
+  if (s.dyn_table && std::memcmp(key, s.dyn_key, sizeof(key)) == 0) return JACOBI_OK;
+  std::vector<int32_t> tab(nb + 1);
+  jbplan::dyn_blocks(npl, units, n, min_blk, tab.data());
+  if (s.dyn_table) cudaFree(s.dyn_table);
+  s.dyn_table = nullptr;
+  CK(cudaMalloc(&s.dyn_table, tab.size() * sizeof(int32_t)));
+  CK(cudaMemcpy(s.dyn_table, tab.data(), tab.size() * sizeof(int32_t), cudaMemcpyHostToDevice));
+  std::memcpy(s.dyn_key, key, sizeof(key));
+  return JACOBI_OK;
 }
 
 struct LaunchPlan {
@@ -301,7 +318,12 @@ int plan_launch(jacobi_ctx *h, const std::vector<int> &idx, bool persist, bool n
       d.dyn_min_blk = (int)std::max<int64_t>(1, h->min_block);
       d.dyn_help = (h->dyn_help != 0) ? 1 : 0;
       d.dyn_n = d.dyn_help ? count : ni;
-      d.dyn_items = (int64_t)g.units * jbplan::dyn_blocks(inner, g.units, d.dyn_n, d.dyn_min_blk);
+      const int64_t nb = jbplan::dyn_blocks(inner, g.units, d.dyn_n, d.dyn_min_blk);
+      d.dyn_items = (int64_t)g.units * nb;
+      d.dyn_first = (int)std::min<int64_t>(ni, d.dyn_items);
+      int rc = upload_table(s, inner, g.units, d.dyn_n, d.dyn_min_blk, nb);
+      if (rc) return rc;
+      d.dyn_table = s.dyn_table;
     }
     s.desc = d;
     s.grid = count;
