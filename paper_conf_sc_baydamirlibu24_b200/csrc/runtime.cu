@@ -255,10 +255,14 @@ int plan_launch(jacobi_ctx *h, const std::vector<int> &idx, bool persist, bool n
   if (h->ctas > 0) total_ctas = (int)std::min<int64_t>(h->ctas * nslab, sms);
   const int per = total_ctas / nslab;
   if (h->dim == 3 && h->tile_y <= 0) {
-    // Static lockstep: pick ty for utilisation; dynamic: the tallest tile that keeps a >= 5-deep
-    // ring (fewest y-halo rows per row).
-    int ty = h->schedule == 1 ? jbplan::choose_ty(h->ny, g.units_x, per - (h->total > 1 ? 2 : 0), smem_optin, g.ws)
-                              : jbplan::tallest_ty(h->ny, smem_optin, g.ws);
+    // Pick ty so that the tile count divides the CTA count well: a whole number of plane blocks
+    // per scheduling round keeps neighbouring tiles on the same planes, so their y-halo rows
+    // are L2 hits (measured C3: ty=7 -> 73 tiles, 2 per round of 148 CTAs, 0.97 of copy BW).
+    // Small (latency-bound) slabs prefer the tallest tile: fewer, larger items.
+    const int64_t planes_per_cta = (h->ny - 2) * (h->n_out - 2) / std::max<int64_t>(1, h->total) / per;
+    const bool small = planes_per_cta < 64 * 8;  // (rows x planes) per CTA below 64 planes of ty=8 tiles
+    int ty = (h->schedule == 0 || small) ? jbplan::tallest_ty(h->ny, smem_optin, g.ws)
+                                         : jbplan::choose_ty(h->ny, g.units_x, per, smem_optin, g.ws);
     if (jbplan::geometry(h->nx, h->ny, h->nz, h->dim, (int)h->tile_x, ty, smem_optin, (int)h->stages, &g))
       return JACOBI_EINVAL;
   }
