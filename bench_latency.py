@@ -26,7 +26,9 @@ if ROOT not in sys.path:
 import paper_conf_sc_baydamirlibu24_b200 as jb  # noqa: E402
 
 SHAPES = {"C5a 3D 128^3": (128, 128, 128), "C5b 2D 1024^2": (1, 1024, 1024)}
-MODES = {"cpufree": jb.MODE_CPUFREE, "baseline_memcpy": jb.MODE_BASELINE_MEMCPY}
+MODES = {"cpufree": jb.MODE_CPUFREE, "baseline_memcpy": jb.MODE_BASELINE_MEMCPY,
+         "baseline_overlap": jb.MODE_BASELINE_OVERLAP, "baseline_p2p": jb.MODE_BASELINE_P2P,
+         "baseline_graph": jb.MODE_BASELINE_GRAPH}
 
 
 def per_iter_us(j: jb.Jacobi, n: int, reps: int = 5) -> float:
@@ -64,17 +66,21 @@ def main():
                             row["gcells_per_s"] = round(cells / us / 1e3, 2)
                         rows.append(row)
                         print(json.dumps(row), flush=True)
-    # CPU-Free vs baseline: time reduction % per config / P / compute
+    # CPU-Free vs each baseline: time reduction % per config / P / compute
     summary = []
     for r in rows:
         if r["mode"] != "cpufree":
             continue
-        b = next(x for x in rows if x["mode"] == "baseline_memcpy" and x["config"] == r["config"]
-                 and x["slabs"] == r["slabs"] and x["no_compute"] == r["no_compute"])
-        summary.append({"config": r["config"], "slabs": r["slabs"], "no_compute": r["no_compute"],
-                        "cpufree_us": r["us_per_iter"], "baseline_us": b["us_per_iter"],
-                        "reduction_pct": round(100 * (b["us_per_iter"] - r["us_per_iter"]) / b["us_per_iter"], 1),
-                        "ratio": round(b["us_per_iter"] / r["us_per_iter"], 2)})
+        for bname in MODES:
+            if bname == "cpufree":
+                continue
+            b = next(x for x in rows if x["mode"] == bname and x["config"] == r["config"]
+                     and x["slabs"] == r["slabs"] and x["no_compute"] == r["no_compute"])
+            summary.append({"config": r["config"], "slabs": r["slabs"], "no_compute": r["no_compute"],
+                            "baseline": bname, "cpufree_us": r["us_per_iter"], "baseline_us": b["us_per_iter"],
+                            "reduction_pct": (round(100 * (b["us_per_iter"] - r["us_per_iter"]) / b["us_per_iter"], 1)
+                                              if b["us_per_iter"] > 0 else None),
+                            "ratio": round(b["us_per_iter"] / r["us_per_iter"], 2) if r["us_per_iter"] > 0 else None})
     for s in summary:
         print(json.dumps({"summary": s}), flush=True)
     if args.out:

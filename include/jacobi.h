@@ -13,9 +13,9 @@
  *   the edge plane, store it straight into the neighbour GPU's halo over NVLink and raise the
  *   neighbour's flag (Listing 4.1), interior thread blocks stream
  *   the bulk, and a device-side grid barrier ends the iteration.
- *   The CPU-controlled comparison modes launch one kernel per iteration and move halos with
- *   cudaMemcpyPeerAsync or NCCL send/recv, with a host synchronisation per iteration
- *   (Listing 2.1a).
+ *   The CPU-controlled comparison modes launch kernels every iteration and move halos with
+ *   cudaMemcpyPeerAsync, NCCL send/recv or in-kernel peer stores, with a host synchronisation
+ *   per iteration (Listing 2.1a), or replay the loop as a CUDA graph.
  *
  * Numerics (readings R1-R4): IEEE fp64, per interior cell
  *   2D: new = 0.25 * (((u[x+1] + u[x-1]) + u[y+1]) + u[y-1])
@@ -58,6 +58,12 @@ extern "C" {
 #define JACOBI_MODE_CPUFREE          0  /* persistent TB-specialised kernel, device-side flags (default) */
 #define JACOBI_MODE_BASELINE_MEMCPY  1  /* per-iteration kernel + cudaMemcpyPeerAsync + host sync */
 #define JACOBI_MODE_BASELINE_NCCL    2  /* per-iteration kernel + ncclSend/ncclRecv + host sync */
+#define JACOBI_MODE_BASELINE_OVERLAP 3  /* boundary kernel + copies on a comm stream, interior kernel
+                                           on the compute stream, host sync ("Overlap") */
+#define JACOBI_MODE_BASELINE_P2P     4  /* per-iteration kernel whose boundary blocks store into the
+                                           peers' halos (GPU-initiated data, host sync) */
+#define JACOBI_MODE_BASELINE_GRAPH   5  /* the MEMCPY loop captured once into a CUDA graph with
+                                           cross-GPU event edges, one host launch per run */
 
 /* ---- flags for jacobi_set_mode --------------------------------------------------------- */
 #define JACOBI_FLAG_NO_COMPUTE   1  /* measurement only: skip the stencil

@@ -32,6 +32,9 @@ JACOBI_ESTATE = -9
 MODE_CPUFREE = 0
 MODE_BASELINE_MEMCPY = 1
 MODE_BASELINE_NCCL = 2
+MODE_BASELINE_OVERLAP = 3
+MODE_BASELINE_P2P = 4
+MODE_BASELINE_GRAPH = 5
 FLAG_NO_COMPUTE = 1
 FLAG_DROP_SIGNAL = 2
 

@@ -9,6 +9,7 @@
 #define JB_THREADS (JB_NC + 32) // + one producer warp (bulk-copy issue)
 #define JB_MAX_STAGES 32
 #define JB_RQ 4                 // run-descriptor queue depth (producer -> consumers)
+#define JB_MAXK 32              // max boundary CTAs per side (one inbound flag slot each)
 #define JB_SMEM_DEFAULT 232448  // B200 opt-in dynamic shared memory per block (227 KB)
 
 // Grid geometry in HBM and the tile shape of the march.
@@ -35,10 +36,14 @@ struct JbSlab {
   double *buf[2];                 // local slab, planes 0..chunk+1 (0 and chunk+1 are halos)
   double *peer_top[2];            // top neighbour's plane chunk_top+1 (its bottom halo), per parity
   double *peer_bot[2];            // bottom neighbour's plane 0 (its top halo), per parity
-  unsigned long long *flag_in_top;   // local; set by the top neighbour to the iteration whose halo it delivered
-  unsigned long long *flag_in_bot;   // local; set by the bottom neighbour
+  // Flags: one u64 slot per boundary CTA of the sending side, in the RECEIVER's memory.
+  // Sender CTA j of a side sets slot j to the iteration whose halo it delivered (t+1) with one
+  // sys-scope release store; the receiver waits until slots 0..k_in-1 all reach t.
+  unsigned long long *flag_in_top;   // local [JB_MAXK]; written by the top neighbour's bottom CTAs
+  unsigned long long *flag_in_bot;   // local [JB_MAXK]; written by the bottom neighbour's top CTAs
   unsigned long long *flag_out_top;  // = top neighbour's flag_in_bot
   unsigned long long *flag_out_bot;  // = bottom neighbour's flag_in_top
+  int32_t k_in_top, k_in_bot;        // boundary CTA counts of the neighbours facing this slab
   unsigned int *side_ctr;            // local [2]: boundary CTAs done per side (reset each run)
   unsigned long long *barrier;       // local grid-barrier counter (reset each run)
   int64_t chunk;
@@ -59,6 +64,8 @@ struct JbSlab {
   int32_t dyn_help;                  // boundary CTAs join the interior after signalling
   int32_t dyn_first;                 // items handed out statically (one per interior CTA)
   int64_t dyn_items;                 // units * number of blocks
+  int32_t excl_top, excl_bot;        // interior excludes plane 1 / chunk although n_top/n_bot == 0
+                                     // (the inner kernel of the Copy-Overlap baseline)
 };
 
 struct JbParams {
@@ -75,12 +82,12 @@ struct JbParams {
 
 // Per-slab control block in device memory (one allocation, IPC-exportable).
 struct JbCtrl {
-  unsigned long long flag_in[2];   // [0] top, [1] bottom
+  unsigned long long flag_in[2][JB_MAXK];  // [0] from the top neighbour, [1] from the bottom one
   unsigned long long barrier;
   unsigned int side_ctr[2];
   int status[2];
   unsigned int work[2];            // dynamic-schedule claim counters per iteration parity
-  unsigned long long pad[25];      // 256 B total
+  unsigned long long pad[28];
 };
 
 // ---- host-side planning (plan.cpp) -----------------------------------------------------

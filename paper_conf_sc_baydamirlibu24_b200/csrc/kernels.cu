@@ -73,7 +73,6 @@ __device__ __forceinline__ void fence_proxy_async_global() {
 __device__ __forceinline__ void fence_mbar_init() {
   asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
 }
-__device__ __forceinline__ void fence_acq_rel_sys() { asm volatile("fence.acq_rel.sys;" ::: "memory"); }
 __device__ __forceinline__ unsigned long long ld_acquire_sys(const unsigned long long *p) {
   unsigned long long v;
   asm volatile("ld.acquire.sys.global.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
@@ -89,11 +88,6 @@ __device__ __forceinline__ void st_release_sys(unsigned long long *p, unsigned l
 }
 __device__ __forceinline__ void red_release_gpu_add(unsigned long long *p, unsigned long long v) {
   asm volatile("red.release.gpu.global.add.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
-}
-__device__ __forceinline__ unsigned int atom_acq_rel_gpu_add(unsigned int *p, unsigned int v) {
-  unsigned int old;
-  asm volatile("atom.acq_rel.gpu.global.add.u32 %0, [%1], %2;" : "=r"(old) : "l"(p), "r"(v) : "memory");
-  return old;
 }
 __device__ __forceinline__ unsigned long long globaltimer() {
   unsigned long long t;
@@ -122,6 +116,31 @@ __device__ bool wait_geq(const unsigned long long *p, unsigned long long target,
         atomicExch(P.status + 1, 1);
         return false;
       }
+    }
+  }
+}
+
+// Warp-cooperative wait until flag slots 0..k-1 all reach `target` (lane i polls slot i).
+__device__ bool wait_slots(const unsigned long long *slots, int k, unsigned long long target, const JbParams &P,
+                           int lane) {
+  const unsigned long long t_start = globaltimer();
+  uint32_t n = 0;
+  volatile int *abort_flag = P.status + 1;
+  while (true) {
+    const bool ok = lane >= k || ld_acquire_sys(slots + lane) >= target;
+    if (__all_sync(0xffffffffu, ok)) return true;
+    if ((++n & 127u) == 0) {
+      int stop = 0;
+      if (lane == 0) {
+        if (*abort_flag) {
+          stop = 1;
+        } else if (globaltimer() - t_start > P.timeout_ns) {
+          atomicCAS(P.status, 0, JACOBI_ETIMEOUT);
+          atomicExch(P.status + 1, 1);
+          stop = 1;
+        }
+      }
+      if (__shfl_sync(0xffffffffu, stop, 0)) return false;
     }
   }
 }
@@ -183,8 +202,8 @@ __device__ Sched make_sched(const JbGeom &g, const JbSlab &S, int role, int ridx
     s.plane = role == ROLE_TOP ? 1 : S.chunk;
     return s;
   }
-  const int64_t lo = S.n_top ? 2 : 1;
-  const int64_t hi = S.n_bot ? S.chunk - 1 : S.chunk;
+  const int64_t lo = (S.n_top || S.excl_top) ? 2 : 1;
+  const int64_t hi = (S.n_bot || S.excl_bot) ? S.chunk - 1 : S.chunk;
   const int64_t npl = hi - lo + 1;
   if (npl <= 0 || rcount <= 0) return s;
   if (S.k_planes > 0) {
@@ -236,33 +255,49 @@ struct Ring {
 };
 
 // ---------------------------------------------------------------- producer
+// Where one tile's stage comes from: the rows of tile `unit` (1 in 2D; ty + 2 in 3D incl. the y
+// halo rows), each row the x window [x0-2, x0+tx+2) of 16-byte aligned doubles, one
+// cp.async.bulk per row (one row per producer lane).
+struct TileSrc {
+  const double *base;  // cur + xs + ya*pitch + lane*pitch (plane 0)
+  uint32_t row_bytes;
+  int nrows;
+  __device__ __forceinline__ TileSrc(const JbGeom &g, const double *cur, int32_t unit, int lane) {
+    const int ux = unit % g.units_x, uy = unit / g.units_x;
+    const int64_t xs = 2 + (int64_t)ux * g.tx;
+    const int64_t xe = min(xs + g.tx + 4, g.pitch);
+    row_bytes = (uint32_t)((xe - xs) * 8);
+    int64_t ya = 0;
+    nrows = 1;
+    if (g.dim == 3) {
+      ya = (int64_t)uy * g.ty;  // = y0 - 1
+      const int64_t yb = min(ya + 1 + g.ty, g.ny - 1);
+      nrows = (int)(yb - ya + 1);
+    }
+    base = cur + xs + ya * g.pitch + (int64_t)lane * g.pitch;
+  }
+};
+
+// Load plane p of a tile into ring position `at` (acquire the stage, arm its full barrier, copy).
+__device__ __forceinline__ void produce_stage(const JbGeom &g, const TileSrc &T, int64_t p, const RingPos &at,
+                                              const Ring &R, int lane) {
+  if (lane == 0) {
+    // First pass: waiting on the parity of the (virtual) preceding phase returns at once.
+    mbar_wait(&R.empty[at.slot], at.phase ^ 1u);
+    mbar_expect_tx(&R.full[at.slot], T.row_bytes * (uint32_t)T.nrows);
+  }
+  __syncwarp();
+  if (lane < T.nrows)
+    bulk_g2s(R.stage(at) + (size_t)lane * g.ws, T.base + p * g.plane_elems, T.row_bytes, &R.full[at.slot]);
+}
+
 // Load planes pf..pl of tile `unit` from `cur` into consecutive ring stages starting at q.
-// A stage holds the tile's rows (1 in 2D; ty + 2 in 3D incl. the y halo rows), each row the
-// x window [x0-2, x0+tx+2) of 16-byte aligned doubles, one cp.async.bulk per row.
 __device__ __forceinline__ void produce_planes(const JbGeom &g, const double *cur, int32_t unit,
                                                int64_t pf, int64_t pl, RingPos &q, const Ring &R,
                                                int lane) {
-  const int ux = unit % g.units_x, uy = unit / g.units_x;
-  const int64_t xs = 2 + (int64_t)ux * g.tx;
-  const int64_t xe = min(xs + g.tx + 4, g.pitch);
-  const uint32_t row_bytes = (uint32_t)((xe - xs) * 8);
-  int64_t ya = 0;
-  int nrows = 1;
-  if (g.dim == 3) {
-    ya = (int64_t)uy * g.ty;  // = y0 - 1
-    const int64_t yb = min(ya + 1 + g.ty, g.ny - 1);
-    nrows = (int)(yb - ya + 1);
-  }
-  const double *src = cur + pf * g.plane_elems + xs + ya * g.pitch + (int64_t)lane * g.pitch;
+  const TileSrc T(g, cur, unit, lane);
   for (int64_t p = pf; p <= pl; ++p) {
-    if (lane == 0) {
-      // First pass: waiting on the parity of the (virtual) preceding phase returns at once.
-      mbar_wait(&R.empty[q.slot], q.phase ^ 1u);
-      mbar_expect_tx(&R.full[q.slot], row_bytes * (uint32_t)nrows);
-    }
-    __syncwarp();
-    if (lane < nrows) bulk_g2s(R.stage(q) + (size_t)lane * g.ws, src, row_bytes, &R.full[q.slot]);
-    src += g.plane_elems;
+    produce_stage(g, T, p, q, R, lane);
     q.advance(R.S);
   }
 }
@@ -550,8 +585,7 @@ __global__ void __launch_bounds__(JB_THREADS, 1) jb_sweep(const __grid_constant_
                            ? Sched{0, 0, 0, 0, 0, 0, 0, 0, 0}
                            : make_sched(g, SL, role, ridx, rcount);
   const bool drop_signal = (P.flags & JACOBI_FLAG_DROP_SIGNAL) && SL.slab_id == 0;
-  const int side = role == ROLE_TOP ? 0 : 1;
-  const int64_t lo = SL.n_top ? 2 : 1;
+  const int64_t lo = (SL.n_top || SL.excl_top) ? 2 : 1;
   RingPos q = {0u, 0u};   // data ring: producer and consumers advance identical copies
   RingPos rq = {0u, 0u};  // run queue
 
@@ -569,24 +603,59 @@ __global__ void __launch_bounds__(JB_THREADS, 1) jb_sweep(const __grid_constant_
         fence_proxy_async_global();
         // The claim counter of the next iteration is idle now (last used in iteration t-1).
         if (c == 0 && SL.work_ctr) SL.work_ctr[(tg + 1) & 1] = 0u;
-        // wait until the neighbour committed the halo of the previous time step.
-        if (PERSIST && role != ROLE_INT) {
-          const unsigned long long *f = role == ROLE_TOP ? SL.flag_in_top : SL.flag_in_bot;
-          wait_geq<true>(f, (unsigned long long)tg, P);
-          fence_proxy_async_global();
-        }
       }
-      __syncwarp();
+      // boundary blocks wait until the neighbour committed the halo of the previous time
+      // step.  With compute, the two owned planes of the first boundary tile are already in
+      // flight while we wait; only the halo plane's load waits for the flag.
+      bool waited = !(PERSIST && role != ROLE_INT);
+      auto wait_flag = [&]() {
+        if (!waited) {
+          if (role == ROLE_TOP) wait_slots(SL.flag_in_top, SL.k_in_top, (unsigned long long)tg, P, lane);
+          else wait_slots(SL.flag_in_bot, SL.k_in_bot, (unsigned long long)tg, P, lane);
+          if (lane == 0) fence_proxy_async_global();
+          __syncwarp();
+          waited = true;
+        }
+      };
       Sched sched = sched0;
       Run run;
       if (active) {
         while (sched.next(run)) {
-          publish(Q, rq, RUN_WORK, run, lane);
-          if (NOCOMP) produce_planes(g, cur, run.unit, run.p0, run.p1, q, R, lane);
-          else produce_planes(g, cur, run.unit, run.p0 - 1, run.p1 + 1, q, R, lane);
+          if (NOCOMP) {
+            wait_flag();  // remote stores of this run must follow the neighbour's signal
+            publish(Q, rq, RUN_WORK, run, lane);
+            produce_planes(g, cur, run.unit, run.p0, run.p1, q, R, lane);
+          } else if (role != ROLE_INT) {
+            // boundary tile (one plane): halo is p-1 (top) or p+1 (bottom)
+            publish(Q, rq, RUN_WORK, run, lane);
+            const TileSrc T(g, cur, run.unit, lane);
+            RingPos q1 = q, q2 = q;
+            q1.advance(R.S);
+            q2 = q1;
+            q2.advance(R.S);
+            const int64_t p = run.p0;
+            if (role == ROLE_TOP) {
+              produce_stage(g, T, p, q1, R, lane);
+              produce_stage(g, T, p + 1, q2, R, lane);
+              wait_flag();
+              produce_stage(g, T, p - 1, q, R, lane);
+            } else {
+              produce_stage(g, T, p - 1, q, R, lane);
+              produce_stage(g, T, p, q1, R, lane);
+              wait_flag();
+              produce_stage(g, T, p + 1, q2, R, lane);
+            }
+            q = q2;
+            q.advance(R.S);
+          } else {
+            publish(Q, rq, RUN_WORK, run, lane);
+            produce_planes(g, cur, run.unit, run.p0 - 1, run.p1 + 1, q, R, lane);
+          }
         }
       }
-      if (PERSIST && role != ROLE_INT) publish(Q, rq, RUN_SIGNAL, run, lane);
+      wait_flag();  // (boundary CTA without units this iteration still keeps the protocol)
+      // Boundary runs done: signal (CPU-Free) and, in every mode, stop peer stores.
+      if (role != ROLE_INT) publish(Q, rq, RUN_SIGNAL, run, lane);
       if (dyn) {
         // Guided self-scheduling (block-major items, host-built block table).  Interior CTA
         // i's first item is item i; every further item is claimed with one atomicAdd, issued
@@ -621,16 +690,12 @@ __global__ void __launch_bounds__(JB_THREADS, 1) jb_sweep(const __grid_constant_
         if (d.kind == RUN_END) break;
         if (d.kind == RUN_SIGNAL) {
           // P:364-365 / P:394: signal the neighbour that the halo of iteration tg+1 is in place.
-          // bar.sync orders every consumer thread's peer stores before thread 0 (CTA scope);
-          // the sys-scope fence publishes them system-wide before the local counter update; the
-          // last boundary CTA of this side then sets the flag with a sys-scope release store.
-          named_bar_consumers();
-          if (ctid == 0 && !drop_signal) {
-            fence_acq_rel_sys();
-            const unsigned int old = atom_acq_rel_gpu_add(&SL.side_ctr[side], 1u);
-            if (old == (unsigned int)(rcount * (t + 1) - 1))
-              st_release_sys(role == ROLE_TOP ? SL.flag_out_top : SL.flag_out_bot,
-                             (unsigned long long)(tg + 1));
+          if (PERSIST) named_bar_consumers();
+          // bar.sync makes every consumer thread's peer stores precede thread 0 (CTA scope);
+          // its sys-scope release store into this CTA's slot publishes them to the neighbour.
+          if (PERSIST && ctid == 0 && !drop_signal) {
+            unsigned long long *fo = role == ROLE_TOP ? SL.flag_out_top : SL.flag_out_bot;
+            st_release_sys(fo + ridx, (unsigned long long)(tg + 1));
           }
           remote = nullptr;  // later (interior) runs stay local
           continue;
@@ -660,9 +725,9 @@ __global__ void __launch_bounds__(JB_THREADS, 1) jb_sweep(const __grid_constant_
 
   // End of run: wait for the neighbour's last halo so no remote store is still in flight into
   // this GPU's buffers when the kernel (and the host's view of the run) completes.
-  if (PERSIST && producer && lane == 0 && role != ROLE_INT && P.iters > 0) {
-    const unsigned long long *f = role == ROLE_TOP ? SL.flag_in_top : SL.flag_in_bot;
-    wait_geq<true>(f, (unsigned long long)(P.t0 + P.iters), P);
+  if (PERSIST && producer && role != ROLE_INT && P.iters > 0) {
+    if (role == ROLE_TOP) wait_slots(SL.flag_in_top, SL.k_in_top, (unsigned long long)(P.t0 + P.iters), P, lane);
+    else wait_slots(SL.flag_in_bot, SL.k_in_bot, (unsigned long long)(P.t0 + P.iters), P, lane);
   }
 }
 
@@ -701,7 +766,7 @@ __global__ void jb_init_u12(double *b0, double *b1, int64_t nplanes, JbGeom g, i
 }
 
 __global__ void jb_flag_max(unsigned long long *flags, int n, unsigned long long v) {
-  if (threadIdx.x < n) atomicMax(flags + threadIdx.x, v);
+  for (int i = threadIdx.x; i < n; i += blockDim.x) atomicMax(flags + i, v);
 }
 
 template <int DIM, bool NOCOMP, bool PERSIST>
@@ -748,7 +813,7 @@ cudaError_t launch_init(double *b0, double *b1, int64_t nplanes, const JbGeom &g
 }
 
 cudaError_t launch_flag_max(unsigned long long *flags, int n, unsigned long long v, cudaStream_t st) {
-  jb_flag_max<<<1, 32, 0, st>>>(flags, n, v);
+  jb_flag_max<<<1, 64, 0, st>>>(flags, n, v);
   return cudaGetLastError();
 }
 

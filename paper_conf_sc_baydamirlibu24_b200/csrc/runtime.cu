@@ -78,6 +78,8 @@ NcclApi g_nccl;
 struct IpcBlob {
   uint32_t magic;
   int32_t rank;
+  int32_t sms;  // SM count of the rank's GPU: the CPU-Free role split must match across ranks
+  int32_t pad;
   int64_t chunk;
   int64_t plane_elems;
   cudaIpcMemHandle_t buf[2];
@@ -94,7 +96,9 @@ struct Slab {
   double *buf[2] = {nullptr, nullptr};
   JbCtrl *ctrl = nullptr;
   cudaStream_t stream = nullptr;
+  cudaStream_t stream2 = nullptr;  // comm stream of the Copy-Overlap baseline
   cudaEvent_t ev0 = nullptr, ev1 = nullptr;
+  cudaEvent_t ev_sync = nullptr, ev_copy = nullptr;  // baseline stream / graph dependencies
   bool has_top = false, has_bot = false;
   double *peer_top[2] = {nullptr, nullptr};
   double *peer_bot[2] = {nullptr, nullptr};
@@ -125,6 +129,10 @@ struct jacobi_ctx {
   bool peers_ready = false;
   bool nccl_ready = false;
   double last_ms_max = 0;
+  cudaGraphExec_t graph_exec = nullptr;  // cached GRAPH-baseline executable
+  int64_t graph_iters = -1;
+  int graph_parity = -1;
+  int64_t graph_gen = -1, plan_gen = 0;  // plan_gen bumps on every set_mode / set_param
   JbGeom geom{};  // layout geometry (pitch, plane_elems) fixed at create
 };
 
@@ -162,8 +170,11 @@ int alloc_slab(jacobi_ctx *h, Slab &s) {
   CK(cudaMalloc(&s.ctrl, sizeof(JbCtrl)));
   CK(cudaMemset(s.ctrl, 0, sizeof(JbCtrl)));
   CK(cudaStreamCreateWithFlags(&s.stream, cudaStreamNonBlocking));
+  CK(cudaStreamCreateWithFlags(&s.stream2, cudaStreamNonBlocking));
   CK(cudaEventCreate(&s.ev0));
   CK(cudaEventCreate(&s.ev1));
+  CK(cudaEventCreateWithFlags(&s.ev_sync, cudaEventDisableTiming));
+  CK(cudaEventCreateWithFlags(&s.ev_copy, cudaEventDisableTiming));
   // Deterministic U12 initial field, both buffers, padding = 0.
   CK(jbk::launch_init(s.buf[0], s.buf[1], s.chunk + 2, h->geom, s.start - 1, kSeedBench, s.stream));
   CK(cudaStreamSynchronize(s.stream));
@@ -181,6 +192,9 @@ void free_slab(Slab &s) {
   if (s.dyn_table) cudaFree(s.dyn_table);
   if (s.ev0) cudaEventDestroy(s.ev0);
   if (s.ev1) cudaEventDestroy(s.ev1);
+  if (s.ev_sync) cudaEventDestroy(s.ev_sync);
+  if (s.ev_copy) cudaEventDestroy(s.ev_copy);
+  if (s.stream2) cudaStreamDestroy(s.stream2);
   if (s.stream) cudaStreamDestroy(s.stream);
   s = Slab();
 }
@@ -196,13 +210,13 @@ void link_local(jacobi_ctx *h) {
     if (s.has_top) {
       Slab &o = h->slabs[i - 1];
       for (int p = 0; p < 2; ++p) s.peer_top[p] = o.buf[p] + (o.chunk + 1) * pe;
-      s.flag_out_top = &o.ctrl->flag_in[1];
+      s.flag_out_top = &o.ctrl->flag_in[1][0];
       s.peer_top_dev = o.device;
     }
     if (s.has_bot) {
       Slab &o = h->slabs[i + 1];
       for (int p = 0; p < 2; ++p) s.peer_bot[p] = o.buf[p];
-      s.flag_out_bot = &o.ctrl->flag_in[0];
+      s.flag_out_bot = &o.ctrl->flag_in[0][0];
       s.peer_bot_dev = o.device;
     }
   }
@@ -223,6 +237,50 @@ int upload_table(Slab &s, int64_t npl, int units, int n, int min_blk, int64_t nb
   return JACOBI_OK;
 }
 
+// CTAs of one launch on a GPU with `sms` SMs (all slabs of a virtual group share it).
+int launch_ctas(const jacobi_ctx *h, int sms) {
+  int total = sms;
+  const int nslab = h->kind == KIND_VIRTUAL ? h->total : 1;
+  if (h->ctas > 0) total = (int)std::min<int64_t>(h->ctas * nslab, sms);
+  return total;
+}
+
+// CTAs of slab `id` in its CPU-Free launch.
+int slab_ctas(const jacobi_ctx *h, int id, int sms) {
+  const int total = launch_ctas(h, sms);
+  if (h->kind != KIND_VIRTUAL) return total;
+  return total / h->total + (id < total % h->total ? 1 : 0);
+}
+
+// Boundary / interior split of a slab's CTAs (reconstructed P:398-404; R11).
+void split_roles(const jacobi_ctx *h, int count, int64_t inner, bool top, bool bot, int units, int *nt,
+                 int *nb, int *ni) {
+  const bool dynamic = h->schedule == 2 || h->schedule < 0;
+  int override_ps = (int)h->boundary_ctas;
+  if (override_ps <= 0 && dynamic && h->dyn_help && inner > 0 && (top || bot)) {
+    // Boundary CTAs join the dynamic interior after signalling, so give every boundary unit its
+    // own CTA (shortest halo critical path), up to a quarter of the grid per side.
+    override_ps = (int)std::max<int64_t>(1, std::min<int64_t>(units, count / 4));
+  }
+  override_ps = std::min(override_ps, JB_MAXK);
+  jbplan::tb_split(count, inner, top, bot, units, override_ps, nt, nb, ni);
+  *nt = std::min(*nt, JB_MAXK);
+  *nb = std::min(*nb, JB_MAXK);
+  *ni = count - *nt - *nb;
+}
+
+// The CPU-Free split of slab `id` as that slab computes it (same inputs, same function).
+void neighbour_roles(const jacobi_ctx *h, int id, int sms, int units, int *nt_out, int *nb_out) {
+  int64_t start, chunk;
+  jbplan::decompose(h->n_out, h->total, id, &start, &chunk);
+  const bool top = id > 0, bot = id < h->total - 1;
+  const int64_t inner = (bot ? chunk - 1 : chunk) - (top ? 2 : 1) + 1;
+  int nt, nb, ni;
+  split_roles(h, slab_ctas(h, id, sms), inner, top, bot, units, &nt, &nb, &ni);
+  if (nt_out) *nt_out = nt;
+  if (nb_out) *nb_out = nb;
+}
+
 struct LaunchPlan {
   JbParams P;
   int grid = 0;
@@ -234,7 +292,18 @@ struct LaunchPlan {
 
 // Plan one launch on one device over the local slabs `idx` (1 slab per GPU, or all slabs in
 // virtual mode).  persist=false plans the discrete baseline kernel (no boundary roles).
-int plan_launch(jacobi_ctx *h, const std::vector<int> &idx, bool persist, bool nocomp, LaunchPlan &L) {
+// What a launch computes (CPU-Free persistent kernel or one of the discrete baseline kernels).
+enum LaunchKind {
+  LK_PERSIST = 0,  // CPU-Free: roles, peer stores, flags, grid barrier, all iterations
+  LK_ALL,          // discrete: every plane 1..chunk, no roles (Copy / NCCL / graph baselines)
+  LK_P2P,          // discrete: boundary roles store edge planes straight into the peers' halos
+  LK_INNER,        // discrete: planes 2..chunk-1 only (Copy-Overlap compute kernel)
+  LK_EDGES,        // discrete: planes 1 and chunk only, no peer stores (Copy-Overlap comm kernel)
+};
+
+int plan_launch(jacobi_ctx *h, const std::vector<int> &idx, LaunchKind lk, bool nocomp, LaunchPlan &L,
+                int grid_override = 0) {
+  const bool persist = lk == LK_PERSIST;
   Slab &s0 = h->slabs[idx[0]];
   L.device = s0.device;
   L.stream = s0.stream;
@@ -251,8 +320,8 @@ int plan_launch(jacobi_ctx *h, const std::vector<int> &idx, bool persist, bool n
                        (int)h->stages, &g))
     return JACOBI_EINVAL;
   const int nslab = (int)idx.size();
-  int total_ctas = sms;  // one CTA per SM (occupancy verified below)
-  if (h->ctas > 0) total_ctas = (int)std::min<int64_t>(h->ctas * nslab, sms);
+  int total_ctas = launch_ctas(h, sms);  // one CTA per SM (occupancy verified below)
+  if (grid_override > 0) total_ctas = std::min(grid_override, sms);
   const int per = total_ctas / nslab;
   if (h->dim == 3 && h->tile_y <= 0) {
     // Pick ty so that the tile count divides the CTA count well: a whole number of plane blocks
@@ -288,8 +357,8 @@ int plan_launch(jacobi_ctx *h, const std::vector<int> &idx, bool persist, bool n
     d.buf[0] = s.buf[0]; d.buf[1] = s.buf[1];
     d.peer_top[0] = s.peer_top[0]; d.peer_top[1] = s.peer_top[1];
     d.peer_bot[0] = s.peer_bot[0]; d.peer_bot[1] = s.peer_bot[1];
-    d.flag_in_top = &s.ctrl->flag_in[0];
-    d.flag_in_bot = &s.ctrl->flag_in[1];
+    d.flag_in_top = &s.ctrl->flag_in[0][0];
+    d.flag_in_bot = &s.ctrl->flag_in[1][0];
     d.flag_out_top = s.flag_out_top;
     d.flag_out_bot = s.flag_out_bot;
     d.side_ctr = s.ctrl->side_ctr;
@@ -299,21 +368,42 @@ int plan_launch(jacobi_ctx *h, const std::vector<int> &idx, bool persist, bool n
     d.cta_count = count;
     d.slab_id = s.id;
     begin += count;
-    const bool top = persist && s.has_top, bot = persist && s.has_bot;
-    const int64_t lo = top ? 2 : 1, hi = bot ? s.chunk - 1 : s.chunk;
+    const bool roles = lk == LK_PERSIST || lk == LK_P2P || lk == LK_EDGES;
+    const bool top = roles && s.has_top, bot = roles && s.has_bot;
+    if (lk == LK_EDGES) {  // boundary planes only: CTAs split between the sides, no interior
+      d.peer_top[0] = d.peer_top[1] = d.peer_bot[0] = d.peer_bot[1] = nullptr;
+      const int sides = (top ? 1 : 0) + (bot ? 1 : 0);
+      d.n_top = top ? std::max(1, count / std::max(sides, 1)) : 0;
+      d.n_bot = bot ? count - d.n_top : 0;
+      d.cta_count = d.n_top + d.n_bot;
+      d.work_ctr = s.ctrl->work;
+      s.desc = d;
+      s.grid = d.cta_count;
+      s.smem = L.smem;
+      continue;
+    }
+    if (lk == LK_INNER) {
+      d.excl_top = s.has_top ? 1 : 0;
+      d.excl_bot = s.has_bot ? 1 : 0;
+    }
+    const int64_t lo = (top || d.excl_top) ? 2 : 1, hi = (bot || d.excl_bot) ? s.chunk - 1 : s.chunk;
     const int64_t inner = hi - lo + 1;
     int nt, nb, ni;
     if (count < (top ? 1 : 0) + (bot ? 1 : 0) + (inner > 0 ? 1 : 0)) return JACOBI_ENOCOOP;
     const bool dynamic = h->schedule == 2 || h->schedule < 0;
-    int override_ps = (int)h->boundary_ctas;
-    if (override_ps <= 0 && dynamic && h->dyn_help && inner > 0 && (top || bot)) {
-      // Boundary CTAs join the dynamic interior after signalling, so give every boundary unit
-      // its own CTA (shortest halo critical path), up to a quarter of the grid per side.
-      override_ps = (int)std::max<int64_t>(1, std::min<int64_t>(g.units, count / 4));
-    }
-    jbplan::tb_split(count, inner, top, bot, g.units, override_ps, &nt, &nb, &ni);
+    split_roles(h, count, inner, top, bot, g.units, &nt, &nb, &ni);
     d.n_top = nt;
     d.n_bot = nb;
+    if (persist) {
+      // The facing boundary-CTA counts of the neighbours (how many flag slots to wait for) are
+      // recomputed here with the neighbours' own chunk and CTA count: the split is deterministic.
+      int kt = 0, kb = 0;
+      if (s.has_top) neighbour_roles(h, s.id - 1, sms, g.units, nullptr, &kt);
+      if (s.has_bot) neighbour_roles(h, s.id + 1, sms, g.units, &kb, nullptr);
+      d.k_in_top = kt;
+      d.k_in_bot = kb;
+      if (kt > JB_MAXK || kb > JB_MAXK || nt > JB_MAXK || nb > JB_MAXK) return JACOBI_EINVAL;
+    }
     const bool lockstep = h->schedule == 1;
     d.k_planes = lockstep ? jbplan::lockstep_k(g.units, ni, inner) : 0;
     d.work_ctr = s.ctrl->work;
@@ -322,10 +412,10 @@ int plan_launch(jacobi_ctx *h, const std::vector<int> &idx, bool persist, bool n
       d.dyn_min_blk = (int)std::max<int64_t>(1, h->min_block);
       d.dyn_help = (h->dyn_help != 0) ? 1 : 0;
       d.dyn_n = d.dyn_help ? count : ni;
-      const int64_t nb = jbplan::dyn_blocks(inner, g.units, d.dyn_n, d.dyn_min_blk);
-      d.dyn_items = (int64_t)g.units * nb;
+      const int64_t nblk = jbplan::dyn_blocks(inner, g.units, d.dyn_n, d.dyn_min_blk);
+      d.dyn_items = (int64_t)g.units * nblk;
       d.dyn_first = (int)std::min<int64_t>(ni, d.dyn_items);
-      int rc = upload_table(s, inner, g.units, d.dyn_n, d.dyn_min_blk, nb);
+      int rc = upload_table(s, inner, g.units, d.dyn_n, d.dyn_min_blk, nblk);
       if (rc) return rc;
       d.dyn_table = s.dyn_table;
     }
@@ -368,17 +458,20 @@ int run_cpufree(jacobi_ctx *h, int64_t iters) {
   auto groups = launch_groups(h);
   std::vector<LaunchPlan> plans(groups.size());
   for (size_t i = 0; i < groups.size(); ++i) {
-    int rc = plan_launch(h, groups[i], true, nocomp, plans[i]);
+    int rc = plan_launch(h, groups[i], LK_PERSIST, nocomp, plans[i]);
     if (rc) return rc;
     plans[i].P.t0 = h->t;
     plans[i].P.iters = iters;
   }
-  // Reset per-run counters (barrier, side counters, status); flags are monotonic across runs.
+  // Reset per-run counters (barrier, status, claim counters).  Flags are monotonic across runs:
+  // raise every inbound slot to the current iteration (atomicMax: a neighbour that already
+  // signalled this run is kept), so slots unused by an earlier split never hold stale values.
   for (auto &L : plans) {
     CK(cudaSetDevice(L.device));
     for (int k : L.slab_idx) {
       Slab &s = h->slabs[k];
       CK(reset_run_counters(s, L.stream));
+      CK(jbk::launch_flag_max(&s.ctrl->flag_in[0][0], 2 * JB_MAXK, (unsigned long long)h->t, L.stream));
     }
   }
   // Debug: JACOBI_TRACE=1 records when each CTA finished its work in the first 8 iterations.
@@ -453,81 +546,32 @@ int ensure_nccl(jacobi_ctx *h) {
   return JACOBI_OK;
 }
 
-// CPU-controlled baseline (Listing 2.1a, "Baseline Copy", P:230 host barrier):
-// every iteration the host launches the discrete kernel on every GPU, then moves the edge planes
-// into the neighbours' halos (cudaMemcpyPeerAsync or NCCL send/recv), then synchronises every
-// GPU's stream before the next iteration (the OpenMP/MPI barrier of the reference code).
-int run_baseline(jacobi_ctx *h, int64_t iters, bool nccl) {
-  const bool nocomp = h->flags & JACOBI_FLAG_NO_COMPUTE;
-  if (nccl) {
-    int rc = ensure_nccl(h);
-    if (rc) return rc;
-  } else if (h->kind == KIND_DIST && h->total > 1) {
-    return JACOBI_EINVAL;  // memcpy baseline needs a host barrier across processes: use NCCL
+// CPU-controlled baselines (Listing 2.1a).
+// Every iteration the host launches discrete kernels on every GPU, moves the edge planes into
+// the neighbours' halos, and synchronises every GPU before the next iteration (the
+// OpenMP/MPI barrier of the reference code):
+//   COPY    : kernel over all planes, then cudaMemcpyPeerAsync of the edge planes
+//   NCCL    : kernel, then ncclSend/ncclRecv of the edge planes (grouped)
+//   OVERLAP : boundary planes on a comm stream (few CTAs) + memcpy, interior planes concurrently
+//             on the compute stream ("Baseline Overlap")
+//   P2P     : one kernel whose boundary CTAs store the edge planes into the peers' halos
+//   GRAPH   : the COPY loop captured once into a CUDA graph (all iterations, cross-GPU event
+//             dependencies instead of host barriers) and replayed with one launch — the strongest
+//             CPU-controlled variant (not in the paper).
+enum BaseKind { BK_COPY, BK_NCCL, BK_OVERLAP, BK_P2P, BK_GRAPH };
+
+int time_begin(jacobi_ctx *h) {
+  for (auto &s : h->slabs) {
+    CK(cudaSetDevice(s.device));
+    CK(reset_run_counters(s, s.stream));
+    CK(cudaEventRecord(s.ev0, s.stream));
   }
-  const int n = (int)h->slabs.size();
-  std::vector<LaunchPlan> plans(n);
-  for (int i = 0; i < n; ++i) {
-    int rc = plan_launch(h, {i}, false, nocomp, plans[i]);
-    if (rc) return rc;
-    plans[i].P.iters = 1;
-  }
-  const int64_t pe = h->geom.plane_elems;
-  const size_t plane_bytes = (size_t)pe * sizeof(double);
-  for (int i = 0; i < n; ++i) {
-    CK(cudaSetDevice(h->slabs[i].device));
-    CK(reset_run_counters(h->slabs[i], h->slabs[i].stream));
-    CK(cudaEventRecord(h->slabs[i].ev0, h->slabs[i].stream));
-  }
-  for (int64_t it = 0; it < iters; ++it) {
-    const int64_t tg = h->t + it;
-    const int nxt = (int)((tg + 1) & 1);
-    for (int i = 0; i < n; ++i) {  // ② launch the compute kernel on every GPU
-      Slab &s = h->slabs[i];
-      CK(cudaSetDevice(s.device));
-      if (!nocomp) {
-        plans[i].P.t0 = tg;
-        CK(jbk::launch_sweep(plans[i].P, false, false, plans[i].grid, plans[i].smem, s.stream));
-      }
-    }
-    if (!nccl) {  // ④ write_neighbors with host-issued peer copies
-      for (int i = 0; i < n; ++i) {
-        Slab &s = h->slabs[i];
-        CK(cudaSetDevice(s.device));
-        if (s.has_top)
-          CK(cudaMemcpyPeerAsync(s.peer_top[nxt], s.peer_top_dev, s.buf[nxt] + 1 * pe, s.device, plane_bytes,
-                                 s.stream));
-        if (s.has_bot)
-          CK(cudaMemcpyPeerAsync(s.peer_bot[nxt], s.peer_bot_dev, s.buf[nxt] + s.chunk * pe, s.device,
-                                 plane_bytes, s.stream));
-      }
-    } else {
-      if (g_nccl.GroupStart() != ncclSuccess) return JACOBI_ENCCL;
-      for (int i = 0; i < n; ++i) {
-        Slab &s = h->slabs[i];
-        const int me = s.id;
-        double *b = s.buf[nxt];
-        if (s.has_top) {
-          if (g_nccl.Send(b + 1 * pe, pe, ncclFloat64, me - 1, s.comm, s.stream) != ncclSuccess) return JACOBI_ENCCL;
-          if (g_nccl.Recv(b, pe, ncclFloat64, me - 1, s.comm, s.stream) != ncclSuccess) return JACOBI_ENCCL;
-        }
-        if (s.has_bot) {
-          if (g_nccl.Send(b + s.chunk * pe, pe, ncclFloat64, me + 1, s.comm, s.stream) != ncclSuccess)
-            return JACOBI_ENCCL;
-          if (g_nccl.Recv(b + (s.chunk + 1) * pe, pe, ncclFloat64, me + 1, s.comm, s.stream) != ncclSuccess)
-            return JACOBI_ENCCL;
-        }
-      }
-      if (g_nccl.GroupEnd() != ncclSuccess) return JACOBI_ENCCL;
-    }
-    for (int i = 0; i < n; ++i) {  // ⑤ host barrier: wait for every GPU
-      CK(cudaSetDevice(h->slabs[i].device));
-      CK(cudaStreamSynchronize(h->slabs[i].stream));
-    }
-  }
+  return JACOBI_OK;
+}
+
+int time_end(jacobi_ctx *h, int64_t iters) {
   double mx = 0;
-  for (int i = 0; i < n; ++i) {
-    Slab &s = h->slabs[i];
+  for (auto &s : h->slabs) {
     CK(cudaSetDevice(s.device));
     CK(cudaEventRecord(s.ev1, s.stream));
     CK(cudaEventSynchronize(s.ev1));
@@ -541,10 +585,190 @@ int run_baseline(jacobi_ctx *h, int64_t iters, bool nccl) {
   // Keep the CPU-Free protocol consistent: inbound flags hold the global iteration count.
   for (auto &s : h->slabs) {
     CK(cudaSetDevice(s.device));
-    CK(jbk::launch_flag_max(s.ctrl->flag_in, 2, (unsigned long long)h->t, s.stream));
+    CK(jbk::launch_flag_max(&s.ctrl->flag_in[0][0], 2 * JB_MAXK, (unsigned long long)h->t, s.stream));
     CK(cudaStreamSynchronize(s.stream));
   }
   return JACOBI_OK;
+}
+
+// Host-issued peer copies of slab s's edge planes of buffer `nxt` into its neighbours' halos.
+// (Inside a graph capture the UVA form cudaMemcpyAsync(cudaMemcpyDefault) is used: it is the
+// capturable equivalent of cudaMemcpyPeerAsync once peer access is enabled.)
+int copy_edges(jacobi_ctx *h, Slab &s, int nxt, cudaStream_t st, bool capturing = false) {
+  const int64_t pe = h->geom.plane_elems;
+  const size_t bytes = (size_t)pe * sizeof(double);
+  if (capturing) {
+    if (s.has_top) CK(cudaMemcpyAsync(s.peer_top[nxt], s.buf[nxt] + 1 * pe, bytes, cudaMemcpyDefault, st));
+    if (s.has_bot) CK(cudaMemcpyAsync(s.peer_bot[nxt], s.buf[nxt] + s.chunk * pe, bytes, cudaMemcpyDefault, st));
+    return JACOBI_OK;
+  }
+  if (s.has_top)
+    CK(cudaMemcpyPeerAsync(s.peer_top[nxt], s.peer_top_dev, s.buf[nxt] + 1 * pe, s.device, bytes, st));
+  if (s.has_bot)
+    CK(cudaMemcpyPeerAsync(s.peer_bot[nxt], s.peer_bot_dev, s.buf[nxt] + s.chunk * pe, s.device, bytes, st));
+  return JACOBI_OK;
+}
+
+int nccl_edges(jacobi_ctx *h, int nxt) {
+  const int64_t pe = h->geom.plane_elems;
+  if (g_nccl.GroupStart() != ncclSuccess) return JACOBI_ENCCL;
+  for (auto &s : h->slabs) {
+    const int me = s.id;
+    double *b = s.buf[nxt];
+    if (s.has_top) {
+      if (g_nccl.Send(b + 1 * pe, pe, ncclFloat64, me - 1, s.comm, s.stream) != ncclSuccess) return JACOBI_ENCCL;
+      if (g_nccl.Recv(b, pe, ncclFloat64, me - 1, s.comm, s.stream) != ncclSuccess) return JACOBI_ENCCL;
+    }
+    if (s.has_bot) {
+      if (g_nccl.Send(b + s.chunk * pe, pe, ncclFloat64, me + 1, s.comm, s.stream) != ncclSuccess)
+        return JACOBI_ENCCL;
+      if (g_nccl.Recv(b + (s.chunk + 1) * pe, pe, ncclFloat64, me + 1, s.comm, s.stream) != ncclSuccess)
+        return JACOBI_ENCCL;
+    }
+  }
+  if (g_nccl.GroupEnd() != ncclSuccess) return JACOBI_ENCCL;
+  return JACOBI_OK;
+}
+
+int run_graph(jacobi_ctx *h, int64_t iters, bool nocomp, std::vector<LaunchPlan> &plans);
+
+int run_baseline(jacobi_ctx *h, int64_t iters, BaseKind kind) {
+  const bool nocomp = h->flags & JACOBI_FLAG_NO_COMPUTE;
+  if (kind == BK_NCCL) {
+    int rc = ensure_nccl(h);
+    if (rc) return rc;
+  } else if (h->kind == KIND_DIST && h->total > 1) {
+    return JACOBI_EINVAL;  // host-synchronised peer baselines need one process: use NCCL
+  }
+  const int n = (int)h->slabs.size();
+  std::vector<LaunchPlan> plans(n), edges(n);
+  for (int i = 0; i < n; ++i) {
+    Slab &s = h->slabs[i];
+    int rc;
+    if (kind == BK_P2P) {
+      rc = plan_launch(h, {i}, LK_P2P, nocomp, plans[i]);
+    } else if (kind == BK_OVERLAP && (s.has_top || s.has_bot)) {
+      int sms = 0;
+      CK(cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, s.device));
+      const int ne = std::max(2, std::min(sms / 8, 32));  // boundary CTAs on the comm stream
+      rc = plan_launch(h, {i}, LK_EDGES, nocomp, edges[i], ne);
+      if (!rc) rc = plan_launch(h, {i}, LK_INNER, nocomp, plans[i], sms - edges[i].grid);
+    } else {
+      rc = plan_launch(h, {i}, LK_ALL, nocomp, plans[i]);
+    }
+    if (rc) return rc;
+    plans[i].P.iters = 1;
+    edges[i].P.iters = 1;
+  }
+  if (kind == BK_GRAPH) return run_graph(h, iters, nocomp, plans);
+  int rc = time_begin(h);
+  if (rc) return rc;
+  const bool launch_kernels = !nocomp || kind == BK_P2P;  // P2P no-compute still moves halos in-kernel
+  for (int64_t it = 0; it < iters; ++it) {
+    const int64_t tg = h->t + it;
+    const int nxt = (int)((tg + 1) & 1);
+    for (int i = 0; i < n; ++i) {  // ② launch the kernel(s) on every GPU
+      Slab &s = h->slabs[i];
+      CK(cudaSetDevice(s.device));
+      if (kind == BK_OVERLAP && edges[i].grid > 0) {
+        // comm stream: boundary planes first, then the peer copies; compute stream: interior
+        if (!nocomp) {
+          edges[i].P.t0 = tg;
+          CK(jbk::launch_sweep(edges[i].P, false, false, edges[i].grid, edges[i].smem, s.stream2));
+          plans[i].P.t0 = tg;
+          CK(jbk::launch_sweep(plans[i].P, false, false, plans[i].grid, plans[i].smem, s.stream));
+        }
+        rc = copy_edges(h, s, nxt, s.stream2);
+        if (rc) return rc;
+        continue;
+      }
+      if (launch_kernels) {
+        plans[i].P.t0 = tg;
+        CK(jbk::launch_sweep(plans[i].P, nocomp, false, plans[i].grid, plans[i].smem, s.stream));
+      }
+    }
+    if (kind == BK_COPY) {  // ④ write_neighbors with host-issued peer copies
+      for (auto &s : h->slabs) {
+        CK(cudaSetDevice(s.device));
+        rc = copy_edges(h, s, nxt, s.stream);
+        if (rc) return rc;
+      }
+    } else if (kind == BK_NCCL) {
+      rc = nccl_edges(h, nxt);
+      if (rc) return rc;
+    }
+    for (auto &s : h->slabs) {  // ⑤ sync streams, host barrier: wait for every GPU
+      CK(cudaSetDevice(s.device));
+      CK(cudaStreamSynchronize(s.stream2));
+      CK(cudaStreamSynchronize(s.stream));
+    }
+  }
+  return time_end(h, iters);
+}
+
+// GRAPH baseline: capture `iters` iterations of (kernel; peer copies) for every slab into one
+// graph.  Slab g's kernel of iteration t+1 waits (graph edge) for the copies of its neighbours
+// at iteration t; its copies follow its own kernel.  The instantiated graph is cached per
+// (iters, parity of t, plan generation).
+int run_graph(jacobi_ctx *h, int64_t iters, bool nocomp, std::vector<LaunchPlan> &plans) {
+  const int n = (int)h->slabs.size();
+  const int parity = (int)(h->t & 1);
+  if (!h->graph_exec || h->graph_iters != iters || h->graph_parity != parity || h->graph_gen != h->plan_gen) {
+    if (h->graph_exec) cudaGraphExecDestroy(h->graph_exec);
+    h->graph_exec = nullptr;
+    Slab &m = h->slabs[0];
+    CK(cudaSetDevice(m.device));
+    CK(cudaStreamBeginCapture(m.stream, cudaStreamCaptureModeRelaxed));
+    CK(cudaEventRecord(m.ev_sync, m.stream));
+    for (int i = 1; i < n; ++i) {  // fork every other slab's stream into the capture
+      CK(cudaSetDevice(h->slabs[i].device));
+      CK(cudaStreamWaitEvent(h->slabs[i].stream, m.ev_sync, 0));
+    }
+    for (int64_t it = 0; it < iters; ++it) {
+      const int64_t tg = h->t + it;
+      const int nxt = (int)((tg + 1) & 1);
+      for (int i = 0; i < n; ++i) {
+        Slab &s = h->slabs[i];
+        CK(cudaSetDevice(s.device));
+        if (it > 0) {  // halos of this iteration were written by the neighbours' copies
+          if (s.has_top) CK(cudaStreamWaitEvent(s.stream, h->slabs[i - 1].ev_copy, 0));
+          if (s.has_bot) CK(cudaStreamWaitEvent(s.stream, h->slabs[i + 1].ev_copy, 0));
+        }
+        if (!nocomp) {
+          plans[i].P.t0 = tg;
+          CK(jbk::launch_sweep(plans[i].P, false, false, plans[i].grid, plans[i].smem, s.stream));
+        }
+      }
+      for (int i = 0; i < n; ++i) {
+        Slab &s = h->slabs[i];
+        CK(cudaSetDevice(s.device));
+        int rc = copy_edges(h, s, nxt, s.stream, true);
+        if (rc) {
+          cudaGraph_t g;
+          cudaStreamEndCapture(m.stream, &g);
+          return rc;
+        }
+        CK(cudaEventRecord(s.ev_copy, s.stream));
+      }
+    }
+    CK(cudaSetDevice(m.device));
+    for (int i = 1; i < n; ++i) CK(cudaStreamWaitEvent(m.stream, h->slabs[i].ev_copy, 0));  // join
+    cudaGraph_t graph;
+    CK(cudaStreamEndCapture(m.stream, &graph));
+    cudaError_t e = cudaGraphInstantiate(&h->graph_exec, graph, 0);
+    cudaGraphDestroy(graph);
+    CK(e);
+    h->graph_iters = iters;
+    h->graph_parity = parity;
+    h->graph_gen = h->plan_gen;
+  }
+  int rc = time_begin(h);
+  if (rc) return rc;
+  Slab &m = h->slabs[0];
+  CK(cudaSetDevice(m.device));
+  CK(cudaGraphLaunch(h->graph_exec, m.stream));
+  CK(cudaStreamSynchronize(m.stream));
+  return time_end(h, iters);
 }
 
 }  // namespace
@@ -652,6 +876,7 @@ int jacobi_get_ipc_handle(jacobi_t h, void *out) {
   b.rank = h->rank;
   b.chunk = s.chunk;
   b.plane_elems = h->geom.plane_elems;
+  CK(cudaDeviceGetAttribute(&b.sms, cudaDevAttrMultiProcessorCount, s.device));
   CK(cudaSetDevice(s.device));
   CK(cudaIpcGetMemHandle(&b.buf[0], s.buf[0]));
   CK(cudaIpcGetMemHandle(&b.buf[1], s.buf[1]));
@@ -669,7 +894,9 @@ int jacobi_open_peers(jacobi_t h, const void *top_blob, const void *bottom_blob)
   auto open = [&](const void *blob, int expect_rank, double **bufs, JbCtrl **ctrl, int64_t *chunk) -> int {
     IpcBlob b;
     std::memcpy(&b, blob, sizeof(b));
-    if (b.magic != kIpcMagic || b.rank != expect_rank || b.plane_elems != pe) return JACOBI_EINVAL;
+    int sms = 0;
+    CK(cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, s.device));
+    if (b.magic != kIpcMagic || b.rank != expect_rank || b.plane_elems != pe || b.sms != sms) return JACOBI_EINVAL;
     for (int p = 0; p < 2; ++p) {
       void *ptr = nullptr;
       CK(cudaIpcOpenMemHandle(&ptr, b.buf[p], cudaIpcMemLazyEnablePeerAccess));
@@ -690,7 +917,7 @@ int jacobi_open_peers(jacobi_t h, const void *top_blob, const void *bottom_blob)
     int rc = open(top_blob, h->rank - 1, bufs, &ctrl, &chunk);
     if (rc) return rc;
     for (int p = 0; p < 2; ++p) s.peer_top[p] = bufs[p] + (chunk + 1) * pe;
-    s.flag_out_top = &ctrl->flag_in[1];
+    s.flag_out_top = &ctrl->flag_in[1][0];
   }
   if (s.has_bot) {
     double *bufs[2];
@@ -699,7 +926,7 @@ int jacobi_open_peers(jacobi_t h, const void *top_blob, const void *bottom_blob)
     int rc = open(bottom_blob, h->rank + 1, bufs, &ctrl, &chunk);
     if (rc) return rc;
     for (int p = 0; p < 2; ++p) s.peer_bot[p] = bufs[p];
-    s.flag_out_bot = &ctrl->flag_in[0];
+    s.flag_out_bot = &ctrl->flag_in[0][0];
   }
   h->peers_ready = true;
   return JACOBI_OK;
@@ -734,16 +961,20 @@ int jacobi_run(jacobi_t h, int64_t iters) {
     return JACOBI_OK;
   }
   if (h->mode == JACOBI_MODE_CPUFREE) return run_cpufree(h, iters);
-  if (h->mode == JACOBI_MODE_BASELINE_MEMCPY) return run_baseline(h, iters, false);
-  if (h->mode == JACOBI_MODE_BASELINE_NCCL) return run_baseline(h, iters, true);
+  if (h->mode == JACOBI_MODE_BASELINE_MEMCPY) return run_baseline(h, iters, BK_COPY);
+  if (h->mode == JACOBI_MODE_BASELINE_NCCL) return run_baseline(h, iters, BK_NCCL);
+  if (h->mode == JACOBI_MODE_BASELINE_OVERLAP) return run_baseline(h, iters, BK_OVERLAP);
+  if (h->mode == JACOBI_MODE_BASELINE_P2P) return run_baseline(h, iters, BK_P2P);
+  if (h->mode == JACOBI_MODE_BASELINE_GRAPH) return run_baseline(h, iters, BK_GRAPH);
   return JACOBI_EINVAL;
 }
 
 int jacobi_set_mode(jacobi_t h, int mode, int flags) {
   if (!h) return JACOBI_EINVAL;
-  if (mode < JACOBI_MODE_CPUFREE || mode > JACOBI_MODE_BASELINE_NCCL) return JACOBI_EINVAL;
+  if (mode < JACOBI_MODE_CPUFREE || mode > JACOBI_MODE_BASELINE_GRAPH) return JACOBI_EINVAL;
   if (flags & ~(JACOBI_FLAG_NO_COMPUTE | JACOBI_FLAG_DROP_SIGNAL)) return JACOBI_EINVAL;
   h->mode = mode;
+  h->plan_gen++;
   h->flags = flags;
   return JACOBI_OK;
 }
@@ -769,6 +1000,7 @@ int jacobi_set_param(jacobi_t h, const char *name, int64_t value) {
   if (!std::strcmp(name, "tile_x") && value > 4096) return JACOBI_EINVAL;
   if (!std::strcmp(name, "tile_y") && value > 30) return JACOBI_EINVAL;
   *p = value;
+  h->plan_gen++;
   return JACOBI_OK;
 }
 
@@ -854,7 +1086,7 @@ int jacobi_describe(jacobi_t h, int i, int64_t *o) {
   for (auto &grp : launch_groups(h)) {
     if (std::find(grp.begin(), grp.end(), i) == grp.end()) continue;
     LaunchPlan L;
-    int rc = plan_launch(h, grp, true, h->flags & JACOBI_FLAG_NO_COMPUTE, L);
+    int rc = plan_launch(h, grp, LK_PERSIST, h->flags & JACOBI_FLAG_NO_COMPUTE, L);
     if (rc) return rc;
     o[0] = s.start; o[1] = s.chunk; o[2] = L.P.g.pitch; o[3] = L.P.g.plane_elems;
     o[4] = L.P.g.tx; o[5] = L.P.g.ty; o[6] = L.P.g.units_x; o[7] = L.P.g.units_y;
@@ -872,6 +1104,7 @@ int jacobi_destroy(jacobi_t h) {
     if (s.stream) cudaStreamSynchronize(s.stream);
   }
   for (auto &s : h->slabs) free_slab(s);
+  if (h->graph_exec) cudaGraphExecDestroy(h->graph_exec);
   delete h;
   return JACOBI_OK;
 }

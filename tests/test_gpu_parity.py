@@ -135,6 +135,29 @@ def test_baseline_memcpy_virtual(P):
     assert_bitwise(run_gpu(g, 5, virtual=P, mode=jb.MODE_BASELINE_MEMCPY), oracle.jacobi(g, 5), "memcpy 3d")
 
 
+@pytest.mark.parametrize("mode", ["MODE_BASELINE_OVERLAP", "MODE_BASELINE_P2P", "MODE_BASELINE_GRAPH"])
+@pytest.mark.parametrize("P", [1, 2, 4])
+def test_baselines_n1(mode, P):
+    """SURVEY §8(f) N1 baselines (Copy-Overlap, P2P, CUDA graph) are bit-identical too."""
+    m = getattr(jb, mode)
+    f = u12((4 * P + 7, 520), 1)
+    assert_bitwise(run_gpu(f, 11, virtual=P, mode=m), oracle.jacobi(f, 11), f"{mode} P={P}")
+    g = u12((3 * P + 4, 13, 70), 2)
+    assert_bitwise(run_gpu(g, 6, virtual=P, mode=m), oracle.jacobi(g, 6), f"{mode} 3d P={P}")
+
+
+def test_graph_baseline_cache_and_mixing():
+    f = u12((30, 200), 3)
+    with jb.Jacobi(f.shape, virtual=3) as j:
+        j.scatter(f)
+        j.set_mode(jb.MODE_BASELINE_GRAPH)
+        j.run(4).run(4).run(5)           # cached graph reused for equal (iters, parity)
+        j.set_mode(jb.MODE_CPUFREE).run(3)
+        j.set_mode(jb.MODE_BASELINE_P2P).run(2)
+        j.set_mode(jb.MODE_BASELINE_OVERLAP).run(2)
+        assert_bitwise(j.gather(), oracle.jacobi(f, 20), "graph cache + mixing")
+
+
 def test_baseline_nccl_single_gpu():
     f = u12((65, 300), 1)
     assert_bitwise(run_gpu(f, 9, mode=jb.MODE_BASELINE_NCCL), oracle.jacobi(f, 9), "nccl P=1")
