@@ -301,6 +301,22 @@ def main():
         j.set_mode(jb.MODE_CPUFREE)
         line["cpu_controlled"] = base
 
+        # ---- per-iteration halo latency (no-compute runs): CPU-Free vs NCCL baseline
+        if world > 1:
+            halo = {}
+            for name, mode in (("cpufree", jb.MODE_CPUFREE), ("baseline_nccl", jb.MODE_BASELINE_NCCL)):
+                j.set_mode(mode, jb.FLAG_NO_COMPUTE)
+                j.run(100)
+                j.run(200)
+                t1 = max_over_ranks(j.last_time_ms())
+                j.run(400)
+                t2 = max_over_ranks(j.last_time_ms())
+                halo[name] = 1e3 * (t2 - t1) / 200
+            j.set_mode(jb.MODE_CPUFREE)
+            line["halo_us"] = halo
+        else:
+            line["halo_us"] = None  # one slab: no halo; see bench_latency.py (virtual slabs)
+
         # ---- e2e through the C ABI with pinned host buffers (scatter + run + gather per step)
         from jacobi_inputs import u12_flat
         nz, ny, nx = shape

@@ -114,8 +114,13 @@ int jacobi_set_mode(jacobi_t h, int mode, int flags);
  * "ctas" (persistent grid size per slab group, 0 = all co-resident), "schedule" (interior
  * work distribution: -1 auto = 2, 0 static linear, 1 static lockstep, 2 dynamic guided
  * self-scheduling), "min_block" (smallest dynamic block, planes, default 8), "dyn_help"
- * (1: boundary blocks join the dynamic interior after signalling), "timeout_ms" (watchdog,
- * default 20000).  Unknown names return JACOBI_EINVAL. */
+ * (1: boundary blocks join the dynamic interior after signalling), "resident" (CPU-Free runs
+ * with compute keep each slab on chip — PERKS-style, P:335-337, P:406-408 — when it fits in the
+ * shared memory/registers of its CTAs: -1 auto (default), 0 never, 1 always (EINVAL if it does
+ * not fit)), "block_sync" (resident kernel: 0 = default, device-wide grid barrier per iteration
+ * as in P:372; 1 = each block waits only for its face-sharing neighbour blocks' flags),
+ * "timeout_ms" (watchdog, default 20000).  Read-only: "last_resident" (1 if the last
+ * CPU-Free run used the resident kernel).  Unknown names return JACOBI_EINVAL. */
 int jacobi_set_param(jacobi_t h, const char *name, int64_t value);
 int jacobi_get_param(jacobi_t h, const char *name, int64_t *value);
 

@@ -10,6 +10,9 @@
 #define JB_MAX_STAGES 32
 #define JB_RQ 4                 // run-descriptor queue depth (producer -> consumers)
 #define JB_MAXK 32              // max boundary CTAs per side (one inbound flag slot each)
+#define JB_RNT 512              // threads per CTA of the resident (on-chip) kernel
+#define JB_MAX_BLOCKS 1024      // per-slab block flags of the resident kernel
+#define JB_RCPP_MAX 8           // max cell pairs per thread held in registers by the resident kernel
 #define JB_SMEM_DEFAULT 232448  // B200 opt-in dynamic shared memory per block (227 KB)
 
 // Grid geometry in HBM and the tile shape of the march.
@@ -29,7 +32,7 @@ struct JbGeom {
   int32_t units_x, units_y, units;
   int32_t stages;       // ring depth
   int32_t stage_doubles;// rh * ws
-  int32_t pad0;
+  int32_t res_rs;       // resident kernel: smem row stride in doubles (x at column x + 1)
 };
 
 struct JbSlab {
@@ -66,6 +69,10 @@ struct JbSlab {
   int64_t dyn_items;                 // units * number of blocks
   int32_t excl_top, excl_bot;        // interior excludes plane 1 / chunk although n_top/n_bot == 0
                                      // (the inner kernel of the Copy-Overlap baseline)
+  int32_t res_nbz, res_nby;          // resident kernel: the slab's (outer x y) block grid
+  int32_t res_relaxed;               // resident kernel: 1 = neighbour-block flags instead of the grid barrier
+  int32_t pad2;
+  unsigned long long *blk_flags;     // resident kernel: per-block "faces of iteration v are stored" flags
 };
 
 struct JbParams {
@@ -105,5 +112,12 @@ int tallest_ty(int64_t ny, int smem_bytes, int ws);
 int lockstep_k(int units, int n_int, int64_t inner_planes);
 // Number of plane blocks of the guided dynamic schedule (see JbSlab::dyn_min_blk).
 int64_t dyn_blocks(int64_t npl, int units, int n, int min_blk, int32_t *table = nullptr);
+// Resident (on-chip) tiling of a slab of `chunk` planes over at most `count` CTAs: nbz x nby
+// blocks whose rows (+ halo ring) fit in `smem` bytes and whose cell pairs fit in JB_RNT threads x
+// JB_RCPP_MAX registers.  Returns 0 and fills the outputs, or -1 if the slab does not fit.
+int resident_tiling(int64_t nx, int64_t ny, int dim, int64_t chunk, int count, int smem, int *nbz, int *nby,
+                    int *cpp, size_t *smem_used);
+// Even split of n items into k parts: part i has n/k (+1 for the first n%k) items starting at start.
+void even_split(int64_t n, int k, int i, int64_t *start, int64_t *len);
 size_t smem_bytes(const JbGeom &g);
 }  // namespace jbplan

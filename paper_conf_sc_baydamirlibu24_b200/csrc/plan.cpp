@@ -122,6 +122,43 @@ int64_t dyn_blocks(int64_t npl, int units, int n, int min_blk, int32_t *table) {
   return nb;
 }
 
+void even_split(int64_t n, int k, int i, int64_t *start, int64_t *len) {
+  const int64_t q = n / k, r = n % k;
+  *len = q + (i < r ? 1 : 0);
+  *start = (int64_t)i * q + std::min<int64_t>(i, r);
+}
+
+int resident_tiling(int64_t nx, int64_t ny, int dim, int64_t chunk, int count, int smem, int *nbz_out,
+                    int *nby_out, int *cpp_out, size_t *smem_used) {
+  const int64_t rs = round_up(nx + 1, 2);
+  const int64_t ppr = (nx - 1) / 2;  // cell pairs per row covering x = 1 .. nx-2
+  const int64_t rows_y = dim == 3 ? ny - 2 : 1;
+  double best = -1;
+  for (int nbz = 1; nbz <= std::min<int64_t>(chunk, count); ++nbz) {
+    int nby = dim == 3 ? (int)std::min<int64_t>({(int64_t)(count / nbz), rows_y, (int64_t)JB_MAXK}) : 1;
+    if (nby < 1) continue;
+    const int64_t zb = (chunk + nbz - 1) / nbz, yb = (rows_y + nby - 1) / nby;
+    const int64_t rows = (zb + 2) * (dim == 3 ? yb + 2 : 1);
+    const size_t sm = (size_t)rows * rs * 8;
+    if (sm > (size_t)smem) continue;
+    const int64_t pairs = zb * yb * ppr;
+    const int64_t cpp = (pairs + JB_RNT - 1) / JB_RNT;
+    if (cpp > JB_RCPP_MAX) continue;
+    // cost: cells per block (compute + write-back) plus its halo ring rows (L2 refresh)
+    const double cost = (double)zb * yb * (nx - 2) + 2.0 * (zb + (dim == 3 ? yb : 0)) * nx;
+    if (best < 0 || cost < best) {
+      best = cost;
+      *nbz_out = nbz;
+      *nby_out = nby;
+      int c = 1;
+      while (c < cpp) c <<= 1;
+      *cpp_out = c;
+      *smem_used = sm;
+    }
+  }
+  return best < 0 ? -1 : 0;
+}
+
 int tallest_ty(int64_t ny, int smem, int ws) {
   int best = 1;
   for (int ty = 1; ty <= 12; ++ty) {

@@ -26,6 +26,8 @@ cudaError_t launch_sweep(const JbParams &p, bool nocomp, bool persist, int grid,
 cudaError_t launch_init(double *b0, double *b1, int64_t nplanes, const JbGeom &g, int64_t z_first,
                         unsigned long long seed, cudaStream_t st);
 cudaError_t launch_flag_max(unsigned long long *flags, int n, unsigned long long v, cudaStream_t st);
+cudaError_t prepare_resident(int dim, int cpp, size_t smem, int *blocks_per_sm);
+cudaError_t launch_resident(const JbParams &p, int cpp, int grid, size_t smem, cudaStream_t st);
 }  // namespace jbk
 
 namespace {
@@ -109,6 +111,7 @@ struct Slab {
   double last_ms = 0;
   JbSlab desc{};  // last launch descriptor (for jacobi_describe)
   int32_t *dyn_table = nullptr;  // guided-schedule block table (device)
+  unsigned long long *blk_flags = nullptr;  // resident kernel: per-block flags (device)
   int64_t dyn_key[4] = {0, 0, 0, 0};
   int grid = 0;
   size_t smem = 0;
@@ -125,6 +128,9 @@ struct jacobi_ctx {
   int mode = JACOBI_MODE_CPUFREE, flags = 0;
   int64_t tile_x = -1, tile_y = -1, stages = -1, boundary_ctas = -1, ctas = -1, schedule = -1;
   int64_t min_block = 8, dyn_help = 1;
+  int64_t resident = -1;       // on-chip resident kernel: -1 auto (when the slab fits), 0 off, 1 on
+  int64_t block_sync = 0;      // resident kernel: 0 grid barrier, 1 neighbour-block flags
+  int64_t last_resident = 0;   // read-only: whether the last CPU-Free run used it
   int64_t timeout_ms = 20000;
   bool peers_ready = false;
   bool nccl_ready = false;
@@ -190,6 +196,7 @@ void free_slab(Slab &s) {
   if (s.buf[1]) cudaFree(s.buf[1]);
   if (s.ctrl) cudaFree(s.ctrl);
   if (s.dyn_table) cudaFree(s.dyn_table);
+  if (s.blk_flags) cudaFree(s.blk_flags);
   if (s.ev0) cudaEventDestroy(s.ev0);
   if (s.ev1) cudaEventDestroy(s.ev1);
   if (s.ev_sync) cudaEventDestroy(s.ev_sync);
@@ -284,6 +291,7 @@ void neighbour_roles(const jacobi_ctx *h, int id, int sms, int units, int *nt_ou
 struct LaunchPlan {
   JbParams P;
   int grid = 0;
+  int cpp = 0;  // resident kernel: cell pairs per thread
   size_t smem = 0;
   int device = 0;
   cudaStream_t stream = nullptr;
@@ -453,13 +461,102 @@ std::vector<std::vector<int>> launch_groups(jacobi_ctx *h) {
   return groups;
 }
 
+// Plan a resident (on-chip) launch over the slabs `idx` of one device.
+// Returns JACOBI_OK, or JACOBI_EINVAL when some slab does not fit on chip.
+int plan_resident(jacobi_ctx *h, const std::vector<int> &idx, LaunchPlan &L) {
+  Slab &s0 = h->slabs[idx[0]];
+  L.device = s0.device;
+  L.stream = s0.stream;
+  L.slab_idx = idx;
+  CK(cudaSetDevice(s0.device));
+  int sms = 0, smem_optin = 0;
+  CK(cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, s0.device));
+  CK(cudaDeviceGetAttribute(&smem_optin, cudaDevAttrMaxSharedMemoryPerBlockOptin, s0.device));
+  smem_optin = std::min(smem_optin, JB_SMEM_DEFAULT) - 1024;
+  JbParams &P = L.P;
+  std::memset(&P, 0, sizeof(P));
+  if (jbplan::geometry(h->nx, h->ny, h->nz, h->dim, 8, 1, JB_SMEM_DEFAULT, 0, &P.g)) return JACOBI_EINVAL;
+  P.g.res_rs = (int)((h->nx + 2) / 2 * 2);  // round_up(nx + 1, 2)
+  if ((h->slabs[idx[0]].chunk + 3) * P.g.plane_elems >= ((int64_t)1 << 31)) return JACOBI_EINVAL;
+  P.nslabs = (int)idx.size();
+  P.flags = h->flags;
+  P.timeout_ns = (unsigned long long)h->timeout_ms * 1000000ull;
+  P.status = s0.ctrl->status;
+  auto tiling = [&](int id, int *nbz, int *nby, int *cpp, size_t *sm) {
+    int64_t st, ch;
+    jbplan::decompose(h->n_out, h->total, id, &st, &ch);
+    return jbplan::resident_tiling(h->nx, h->ny, h->dim, ch, slab_ctas(h, id, sms), smem_optin, nbz, nby, cpp, sm);
+  };
+  int cpp_max = 1, begin = 0;
+  size_t smem = 0;
+  for (size_t k = 0; k < idx.size(); ++k) {
+    Slab &s = h->slabs[idx[k]];
+    JbSlab &d = P.s[k];
+    int nbz, nby, cpp;
+    size_t sm;
+    if (tiling(s.id, &nbz, &nby, &cpp, &sm)) return JACOBI_EINVAL;
+    cpp_max = std::max(cpp_max, cpp);
+    smem = std::max(smem, sm);
+    d.buf[0] = s.buf[0]; d.buf[1] = s.buf[1];
+    d.peer_top[0] = s.peer_top[0]; d.peer_top[1] = s.peer_top[1];
+    d.peer_bot[0] = s.peer_bot[0]; d.peer_bot[1] = s.peer_bot[1];
+    d.flag_in_top = &s.ctrl->flag_in[0][0];
+    d.flag_in_bot = &s.ctrl->flag_in[1][0];
+    d.flag_out_top = s.flag_out_top;
+    d.flag_out_bot = s.flag_out_bot;
+    d.barrier = &s.ctrl->barrier;
+    d.chunk = s.chunk;
+    d.slab_id = s.id;
+    d.res_nbz = nbz;
+    d.res_nby = nby;
+    d.res_relaxed = h->block_sync == 0 ? 0 : 1;
+    if (d.res_relaxed) {
+      if (nbz * nby > JB_MAX_BLOCKS) return JACOBI_EINVAL;
+      if (!s.blk_flags) {
+        CK(cudaMalloc(&s.blk_flags, JB_MAX_BLOCKS * sizeof(unsigned long long)));
+        CK(cudaMemset(s.blk_flags, 0, JB_MAX_BLOCKS * sizeof(unsigned long long)));
+      }
+      d.blk_flags = s.blk_flags;
+    }
+    d.cta_begin = begin;
+    d.cta_count = nbz * nby;
+    begin += d.cta_count;
+    // facing boundary blocks of the neighbours = their nby (one flag slot per boundary block)
+    int nz2, ny2, c2;
+    size_t sm2;
+    d.k_in_top = (s.has_top && !tiling(s.id - 1, &nz2, &ny2, &c2, &sm2)) ? ny2 : 0;
+    d.k_in_bot = (s.has_bot && !tiling(s.id + 1, &nz2, &ny2, &c2, &sm2)) ? ny2 : 0;
+    if ((s.has_top && d.k_in_top == 0) || (s.has_bot && d.k_in_bot == 0)) return JACOBI_EINVAL;
+    s.desc = d;
+    s.grid = d.cta_count;
+    s.smem = smem;
+  }
+  int occ = 0;
+  CK(jbk::prepare_resident(h->dim, cpp_max, smem, &occ));
+  if (occ < 1 || begin > sms * occ) return JACOBI_EINVAL;
+  L.grid = begin;
+  L.smem = smem;
+  L.cpp = cpp_max;
+  return JACOBI_OK;
+}
+
 int run_cpufree(jacobi_ctx *h, int64_t iters) {
   const bool nocomp = h->flags & JACOBI_FLAG_NO_COMPUTE;
   auto groups = launch_groups(h);
   std::vector<LaunchPlan> plans(groups.size());
+  // Resident (on-chip) kernel when every slab fits (auto) or when forced.
+  bool resident = !nocomp && h->resident != 0;
+  if (resident) {
+    for (size_t i = 0; i < groups.size() && resident; ++i)
+      if (plan_resident(h, groups[i], plans[i]) != JACOBI_OK) resident = false;
+    if (!resident && h->resident == 1) return JACOBI_EINVAL;
+  }
+  h->last_resident = resident ? 1 : 0;
   for (size_t i = 0; i < groups.size(); ++i) {
-    int rc = plan_launch(h, groups[i], LK_PERSIST, nocomp, plans[i]);
-    if (rc) return rc;
+    if (!resident) {
+      int rc = plan_launch(h, groups[i], LK_PERSIST, nocomp, plans[i]);
+      if (rc) return rc;
+    }
     plans[i].P.t0 = h->t;
     plans[i].P.iters = iters;
   }
@@ -472,6 +569,7 @@ int run_cpufree(jacobi_ctx *h, int64_t iters) {
       Slab &s = h->slabs[k];
       CK(reset_run_counters(s, L.stream));
       CK(jbk::launch_flag_max(&s.ctrl->flag_in[0][0], 2 * JB_MAXK, (unsigned long long)h->t, L.stream));
+      if (s.blk_flags) CK(jbk::launch_flag_max(s.blk_flags, JB_MAX_BLOCKS, (unsigned long long)h->t, L.stream));
     }
   }
   // Debug: JACOBI_TRACE=1 records when each CTA finished its work in the first 8 iterations.
@@ -488,7 +586,8 @@ int run_cpufree(jacobi_ctx *h, int64_t iters) {
     CK(cudaSetDevice(L.device));
     Slab &s0 = h->slabs[L.slab_idx[0]];
     CK(cudaEventRecord(s0.ev0, L.stream));
-    CK(jbk::launch_sweep(L.P, nocomp, true, L.grid, L.smem, L.stream));
+    if (resident) CK(jbk::launch_resident(L.P, L.cpp, L.grid, L.smem, L.stream));
+    else CK(jbk::launch_sweep(L.P, nocomp, true, L.grid, L.smem, L.stream));
     CK(cudaEventRecord(s0.ev1, L.stream));
   }
   int rc_all = JACOBI_OK;
@@ -989,11 +1088,15 @@ static int64_t *param_slot(jacobi_t h, const char *name) {
   if (!std::strcmp(name, "timeout_ms")) return &h->timeout_ms;
   if (!std::strcmp(name, "min_block")) return &h->min_block;
   if (!std::strcmp(name, "dyn_help")) return &h->dyn_help;
+  if (!std::strcmp(name, "resident")) return &h->resident;
+  if (!std::strcmp(name, "block_sync")) return &h->block_sync;
+  if (!std::strcmp(name, "last_resident")) return &h->last_resident;
   return nullptr;
 }
 
 int jacobi_set_param(jacobi_t h, const char *name, int64_t value) {
   if (!h || !name) return JACOBI_EINVAL;
+  if (!std::strcmp(name, "last_resident")) return JACOBI_EINVAL;  // read-only
   int64_t *p = param_slot(h, name);
   if (!p) return JACOBI_EINVAL;
   if (!std::strcmp(name, "timeout_ms")) value = value < 0 ? 20000 : value;

@@ -29,8 +29,11 @@ def assert_bitwise(got, exp, what=""):
 
 
 def run_gpu(field, iters, virtual=0, mode=jb.MODE_CPUFREE, params=None, flags=0):
+    """Run through the C ABI.  Unless `params` says otherwise the streaming kernel is forced
+    (resident=0), so these shapes exercise it; the resident kernel has its own tests below."""
+    params = {"resident": 0, **(params or {})}
     with jb.Jacobi(field.shape, virtual=virtual) as j:
-        for k, v in (params or {}).items():
+        for k, v in params.items():
             j.set_param(k, v)
         j.set_mode(mode, flags)
         j.scatter(field)
@@ -248,3 +251,56 @@ def test_watchdog_timeout_without_hang():
     # the device is still healthy afterwards
     f = u12((40, 200), 1)
     assert_bitwise(run_gpu(f, 3, virtual=2), oracle.jacobi(f, 3), "after timeout")
+
+
+# ---------------------------------------------------------------- resident (on-chip) kernel, N2
+@pytest.mark.parametrize("shape", [(3, 3), (9, 70), (300, 131), (1024, 1024), (5, 4, 9), (13, 30, 70),
+                                   (20, 61, 130), (40, 40, 40)])
+@pytest.mark.parametrize("P", [1, 2, 3])
+@pytest.mark.parametrize("sync", [0, 1])
+def test_resident_vs_oracle(shape, P, sync):
+    n_out = shape[0]
+    if P > 1 and (n_out - 2) // P < 2:
+        pytest.skip("slab too thin")
+    f = u12(shape, 5)
+    for iters in (1, 2, 9):
+        with jb.Jacobi(shape, virtual=P) if P > 1 else jb.Jacobi(shape) as j:
+            j.set_param("resident", 1)
+            j.set_param("block_sync", sync)
+            j.scatter(f)
+            j.run(iters)
+            assert jb.jacobi_get_param(j.h, "last_resident") == 1
+            assert_bitwise(j.gather(), oracle.jacobi(f, iters), f"resident {shape} P={P} it={iters}")
+
+
+def test_resident_auto_mixing_and_splitting():
+    f = u12((66, 400), 6)
+    exp = oracle.jacobi(f, 30)
+    with jb.Jacobi(f.shape, virtual=4) as j:
+        j.scatter(f)
+        j.run(5)                                              # auto -> resident (fits)
+        assert jb.jacobi_get_param(j.h, "last_resident") == 1
+        j.set_param("resident", 0).run(6)                     # streaming
+        j.set_mode(jb.MODE_BASELINE_MEMCPY).run(4)
+        j.set_mode(jb.MODE_CPUFREE).set_param("resident", 1).run(7).run(8)
+        assert j.iterations == 30
+        assert_bitwise(j.gather(), exp, "resident mixed")
+
+
+def test_resident_rejects_when_too_big():
+    with jb.Jacobi((1024, 4096)) as j:  # 32 MB slab: does not fit on chip
+        j.set_param("resident", 1)
+        with pytest.raises(jb.JacobiError):
+            j.run(1)
+        j.set_param("resident", -1).run(1)
+        assert jb.jacobi_get_param(j.h, "last_resident") == 0
+
+
+def test_resident_watchdog():
+    with jb.Jacobi((40, 200), virtual=2) as j:
+        j.set_param("timeout_ms", 300)
+        j.set_param("resident", 1)
+        j.set_mode(jb.MODE_CPUFREE, jb.FLAG_DROP_SIGNAL)
+        with pytest.raises(jb.JacobiError) as e:
+            j.run(10)
+        assert e.value.code == jb.JACOBI_ETIMEOUT
