@@ -15,7 +15,7 @@ import re
 import numpy as np
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(_HERE, "libjacobi_b200.so")
+LIB_PATH = os.environ.get("JACOBI_LIB") or os.path.join(_HERE, "libjacobi_b200.so")  # env: A/B measurement aid
 HEADER_PATH = os.path.join(os.path.dirname(_HERE), "include", "jacobi.h")
 
 JACOBI_OK = 0
