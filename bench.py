@@ -205,6 +205,8 @@ def main():
     import torch
     import paper_conf_sc_baydamirlibu24_b200 as jb
 
+    torch.cuda.set_device(local)
+    jb.use_torch_allocator()  # PyTorch owns the device memory of the slabs (north star)
     if world > 1:
         import torch.distributed as dist
         dist.init_process_group("gloo")

@@ -36,6 +36,7 @@
 #ifndef JACOBI_B200_H
 #define JACOBI_B200_H
 
+#include <stddef.h>
 #include <stdint.h>
 
 #ifdef __cplusplus
@@ -104,6 +105,19 @@ int jacobi_open_peers(jacobi_t h, const void *top_blob, const void *bottom_blob)
  * jacobi_nccl_init (collective).  libnccl.so.2 is loaded with dlopen on first use. */
 int jacobi_nccl_unique_id(void *out128);
 int jacobi_nccl_init(jacobi_t h, const void *id128);
+
+/* ---- device memory ------------------------------------------------------------------------
+ * The two field buffers and the control block of every slab are obtained from an allocator:
+ * cudaMalloc/cudaFree by default, or the caller's (e.g. PyTorch's caching allocator, installed by
+ * the Python binding's use_torch_allocator(); the north star's "PyTorch used for device memory").
+ * alloc(bytes, device, user) must return device memory on `device`, 16-byte aligned, or NULL;
+ * free(ptr, device, user) releases it.  Captured by each handle at creation; pass NULL, NULL to
+ * restore cudaMalloc.  Returns JACOBI_EINVAL if exactly one of the two is NULL. */
+typedef void *(*jacobi_alloc_fn)(size_t bytes, int device, void *user);
+typedef void (*jacobi_free_fn)(void *ptr, int device, void *user);
+int jacobi_set_allocator(jacobi_alloc_fn alloc, jacobi_free_fn free_fn, void *user);
+/* Bytes of ONE field buffer of slab `slab` (of `nslabs`) for this grid (host-only helper). */
+int jacobi_slab_bytes(int64_t nx, int64_t ny, int64_t nz, int stencil, int nslabs, int slab, int64_t *bytes);
 
 /* ---- running ----------------------------------------------------------------------------- */
 /* Advance the field by `iters` Jacobi iterations in the current mode.  Continues from the

@@ -66,7 +66,12 @@ _SIGS = {
     "jacobi_tb_split": ([_c.c_int, _i64, _c.c_int, _c.c_int, _i64, _c.c_int, _c.POINTER(_c.c_int)], _c.c_int),
     "jacobi_geometry": ([_i64, _i64, _i64, _c.c_int, _c.c_int, _c.c_int, _c.POINTER(_i64)], _c.c_int),
     "jacobi_version": ([], _c.c_int),
+    "jacobi_set_allocator": ([_p, _p, _p], _c.c_int),
+    "jacobi_slab_bytes": ([_i64, _i64, _i64, _c.c_int, _c.c_int, _c.c_int, _c.POINTER(_i64)], _c.c_int),
 }
+
+ALLOC_FN = _c.CFUNCTYPE(_c.c_void_p, _c.c_size_t, _c.c_int, _c.c_void_p)
+FREE_FN = _c.CFUNCTYPE(None, _c.c_void_p, _c.c_int, _c.c_void_p)
 
 _lib = None
 
@@ -248,6 +253,47 @@ def jacobi_geometry(nx, ny, nz, stencil, tile_x=0, tile_y=0) -> dict:
 
 def jacobi_version() -> int:
     return lib().jacobi_version()
+
+
+def jacobi_slab_bytes(nx, ny, nz, stencil, nslabs, slab) -> int:
+    b = _i64()
+    _check(lib().jacobi_slab_bytes(nx, ny, nz, stencil, nslabs, slab, _c.byref(b)), "jacobi_slab_bytes")
+    return b.value
+
+
+def jacobi_set_allocator(alloc_fn, free_fn, user=None) -> None:
+    """Install C-callable alloc/free callbacks (ctypes ALLOC_FN / FREE_FN) or (None, None)."""
+    _check(lib().jacobi_set_allocator(_c.cast(alloc_fn, _p) if alloc_fn else None,
+                                      _c.cast(free_fn, _p) if free_fn else None, user), "jacobi_set_allocator")
+
+
+_torch_blocks: dict = {}
+_torch_cbs = None
+
+
+def use_torch_allocator(enable: bool = True) -> None:
+    """Let PyTorch own the device memory of handles created from now on: the library's slab
+    buffers and control blocks become torch tensors from the CUDA caching allocator (kept alive
+    here until the library frees them)."""
+    global _torch_cbs
+    if not enable:
+        jacobi_set_allocator(None, None)
+        return
+    import torch
+
+    def _alloc(nbytes, device, _user):
+        try:
+            t = torch.empty(int(nbytes), dtype=torch.uint8, device=f"cuda:{device}")
+        except Exception:
+            return None
+        _torch_blocks[t.data_ptr()] = t
+        return t.data_ptr()
+
+    def _free(ptr, _device, _user):
+        _torch_blocks.pop(ptr, None)
+
+    _torch_cbs = (ALLOC_FN(_alloc), FREE_FN(_free))  # keep the thunks alive
+    jacobi_set_allocator(*_torch_cbs)
 
 
 # ---------------------------------------------------------------- convenience wrapper

@@ -76,6 +76,33 @@ struct NcclApi {
 };
 NcclApi g_nccl;
 
+// Device-memory allocator for the slab buffers and control blocks (jacobi_set_allocator):
+// cudaMalloc by default, or a caller-supplied one (the Python binding installs PyTorch's caching
+// allocator so that PyTorch owns the device memory, as the north star asks).
+struct Allocator {
+  jacobi_alloc_fn alloc = nullptr;
+  jacobi_free_fn free = nullptr;
+  void *user = nullptr;
+};
+Allocator g_alloc;
+
+// cuMemGetAddressRange through the runtime's driver entry point (no libcuda link needed): the
+// base of the allocation containing `p`, so IPC handles of sub-allocations carry their offset.
+typedef int (*PFN_getAddressRange)(unsigned long long *, size_t *, unsigned long long);
+size_t alloc_offset(const void *p) {
+  static PFN_getAddressRange fn = nullptr;
+  if (!fn) {
+    void *f = nullptr;
+    cudaDriverEntryPointQueryResult q;
+    if (cudaGetDriverEntryPoint("cuMemGetAddressRange", &f, cudaEnableDefault, &q) != cudaSuccess || !f) return 0;
+    fn = reinterpret_cast<PFN_getAddressRange>(f);
+  }
+  unsigned long long base = 0;
+  size_t size = 0;
+  if (fn(&base, &size, (unsigned long long)p) != 0) return 0;
+  return (size_t)((unsigned long long)p - base);
+}
+
 // ---------------------------------------------------------------- IPC blob (dist mode)
 struct IpcBlob {
   uint32_t magic;
@@ -86,6 +113,7 @@ struct IpcBlob {
   int64_t plane_elems;
   cudaIpcMemHandle_t buf[2];
   cudaIpcMemHandle_t ctrl;
+  uint64_t off[3];  // offsets of buf[0], buf[1], ctrl inside their allocations (caller allocators)
 };
 constexpr uint32_t kIpcMagic = 0x4A43424Bu;
 
@@ -140,6 +168,7 @@ struct jacobi_ctx {
   int graph_parity = -1;
   int64_t graph_gen = -1, plan_gen = 0;  // plan_gen bumps on every set_mode / set_param
   JbGeom geom{};  // layout geometry (pitch, plane_elems) fixed at create
+  Allocator alloc;  // allocator of buffers / control blocks (captured at create)
 };
 
 namespace {
@@ -161,6 +190,7 @@ jacobi_ctx *new_ctx(int64_t nx, int64_t ny, int64_t nz, int stencil, int total) 
   h->dim = stencil == 5 ? 2 : 3;
   h->n_out = h->dim == 2 ? ny : nz;
   h->total = total;
+  h->alloc = g_alloc;
   JbGeom g;
   // Layout only depends on pitch / plane_elems; tile parameters are re-planned per launch.
   jbplan::geometry(nx, ny, nz, h->dim, 8, 1, JB_SMEM_DEFAULT, 0, &g);
@@ -171,9 +201,19 @@ jacobi_ctx *new_ctx(int64_t nx, int64_t ny, int64_t nz, int stencil, int total) 
 int alloc_slab(jacobi_ctx *h, Slab &s) {
   CK(cudaSetDevice(s.device));
   const size_t bytes = (size_t)slab_elems(h, s) * sizeof(double);
-  CK(cudaMalloc(&s.buf[0], bytes));
-  CK(cudaMalloc(&s.buf[1], bytes));
-  CK(cudaMalloc(&s.ctrl, sizeof(JbCtrl)));
+  if (h->alloc.alloc) {
+    s.buf[0] = static_cast<double *>(h->alloc.alloc(bytes, s.device, h->alloc.user));
+    s.buf[1] = static_cast<double *>(h->alloc.alloc(bytes, s.device, h->alloc.user));
+    s.ctrl = static_cast<JbCtrl *>(h->alloc.alloc(sizeof(JbCtrl), s.device, h->alloc.user));
+    if (!s.buf[0] || !s.buf[1] || !s.ctrl) return JACOBI_ENOMEM;
+    CK(cudaSetDevice(s.device));  // the callback may have switched devices
+    for (const void *p : {(const void *)s.buf[0], (const void *)s.buf[1], (const void *)s.ctrl})
+      if ((uintptr_t)p % 16) return JACOBI_EINVAL;  // bulk copies and 16-byte stores need alignment
+  } else {
+    CK(cudaMalloc(&s.buf[0], bytes));
+    CK(cudaMalloc(&s.buf[1], bytes));
+    CK(cudaMalloc(&s.ctrl, sizeof(JbCtrl)));
+  }
   CK(cudaMemset(s.ctrl, 0, sizeof(JbCtrl)));
   CK(cudaStreamCreateWithFlags(&s.stream, cudaStreamNonBlocking));
   CK(cudaStreamCreateWithFlags(&s.stream2, cudaStreamNonBlocking));
@@ -187,14 +227,16 @@ int alloc_slab(jacobi_ctx *h, Slab &s) {
   return JACOBI_OK;
 }
 
-void free_slab(Slab &s) {
+void free_slab(Slab &s, const Allocator &a) {
   cudaSetDevice(s.device);
   if (s.comm && g_nccl.CommDestroy) g_nccl.CommDestroy(s.comm);
   for (void *p : s.ipc_opened) cudaIpcCloseMemHandle(p);
   s.ipc_opened.clear();
-  if (s.buf[0]) cudaFree(s.buf[0]);
-  if (s.buf[1]) cudaFree(s.buf[1]);
-  if (s.ctrl) cudaFree(s.ctrl);
+  for (void *p : {(void *)s.buf[0], (void *)s.buf[1], (void *)s.ctrl}) {
+    if (!p) continue;
+    if (a.free) a.free(p, s.device, a.user);
+    else if (!a.alloc) cudaFree(p);
+  }
   if (s.dyn_table) cudaFree(s.dyn_table);
   if (s.blk_flags) cudaFree(s.blk_flags);
   if (s.ev0) cudaEventDestroy(s.ev0);
@@ -964,6 +1006,26 @@ int jacobi_create_rank(int64_t nx, int64_t ny, int64_t nz, int stencil, int worl
   return JACOBI_OK;
 }
 
+int jacobi_set_allocator(jacobi_alloc_fn alloc, jacobi_free_fn free_fn, void *user) {
+  if ((alloc == nullptr) != (free_fn == nullptr)) return JACOBI_EINVAL;
+  g_alloc.alloc = alloc;
+  g_alloc.free = free_fn;
+  g_alloc.user = user;
+  return JACOBI_OK;
+}
+
+int jacobi_slab_bytes(int64_t nx, int64_t ny, int64_t nz, int stencil, int nslabs, int slab, int64_t *bytes) {
+  if (!bytes || slab < 0 || slab >= nslabs) return JACOBI_EINVAL;
+  int rc = validate(nx, ny, nz, stencil, nslabs);
+  if (rc) return rc;
+  JbGeom g;
+  if (jbplan::geometry(nx, ny, nz, stencil == 5 ? 2 : 3, 8, 1, JB_SMEM_DEFAULT, 0, &g)) return JACOBI_EINVAL;
+  int64_t start, chunk;
+  jbplan::decompose(stencil == 5 ? ny : nz, nslabs, slab, &start, &chunk);
+  *bytes = (chunk + 2) * g.plane_elems * (int64_t)sizeof(double);
+  return JACOBI_OK;
+}
+
 int jacobi_ipc_handle_bytes(void) { return (int)sizeof(IpcBlob); }
 
 int jacobi_get_ipc_handle(jacobi_t h, void *out) {
@@ -980,6 +1042,9 @@ int jacobi_get_ipc_handle(jacobi_t h, void *out) {
   CK(cudaIpcGetMemHandle(&b.buf[0], s.buf[0]));
   CK(cudaIpcGetMemHandle(&b.buf[1], s.buf[1]));
   CK(cudaIpcGetMemHandle(&b.ctrl, s.ctrl));
+  b.off[0] = alloc_offset(s.buf[0]);
+  b.off[1] = alloc_offset(s.buf[1]);
+  b.off[2] = alloc_offset(s.ctrl);
   std::memcpy(out, &b, sizeof(b));
   return JACOBI_OK;
 }
@@ -1000,12 +1065,12 @@ int jacobi_open_peers(jacobi_t h, const void *top_blob, const void *bottom_blob)
       void *ptr = nullptr;
       CK(cudaIpcOpenMemHandle(&ptr, b.buf[p], cudaIpcMemLazyEnablePeerAccess));
       s.ipc_opened.push_back(ptr);
-      bufs[p] = static_cast<double *>(ptr);
+      bufs[p] = reinterpret_cast<double *>(static_cast<char *>(ptr) + b.off[p]);
     }
     void *c = nullptr;
     CK(cudaIpcOpenMemHandle(&c, b.ctrl, cudaIpcMemLazyEnablePeerAccess));
     s.ipc_opened.push_back(c);
-    *ctrl = static_cast<JbCtrl *>(c);
+    *ctrl = reinterpret_cast<JbCtrl *>(static_cast<char *>(c) + b.off[2]);
     *chunk = b.chunk;
     return JACOBI_OK;
   };
@@ -1206,7 +1271,7 @@ int jacobi_destroy(jacobi_t h) {
     if (s.device >= 0) cudaSetDevice(s.device);
     if (s.stream) cudaStreamSynchronize(s.stream);
   }
-  for (auto &s : h->slabs) free_slab(s);
+  for (auto &s : h->slabs) free_slab(s, h->alloc);
   if (h->graph_exec) cudaGraphExecDestroy(h->graph_exec);
   delete h;
   return JACOBI_OK;

@@ -21,7 +21,7 @@ def _free_port():
     return p
 
 
-def _worker(rank, world, port, shape, iters, q):
+def _worker(rank, world, port, shape, iters, q, torch_alloc=False):
     try:
         os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
         import torch.distributed as dist
@@ -29,6 +29,8 @@ def _worker(rank, world, port, shape, iters, q):
         import paper_conf_sc_baydamirlibu24_b200 as jb
         from jacobi_inputs import u12
         f = u12(shape, 7)
+        if torch_alloc:  # IPC of sub-allocations of PyTorch's caching allocator (offsets in the blob)
+            jb.use_torch_allocator()
         j = jb.Jacobi(shape, dist=(rank, world), device=0)
         j.set_param("timeout_ms", 60000)
         jb.exchange_peers(j, nccl=False)
@@ -45,15 +47,17 @@ def _worker(rank, world, port, shape, iters, q):
         q.put((rank, None, repr(e)))
 
 
-@pytest.mark.parametrize("shape,iters", [((40, 96), 5), ((11, 12, 40), 3)])
-def test_two_ranks_one_gpu_ipc(shape, iters):
+@pytest.mark.parametrize("shape,iters,torch_alloc", [((40, 96), 5, False), ((11, 12, 40), 3, False),
+                                                     ((40, 96), 4, True)])
+def test_two_ranks_one_gpu_ipc(shape, iters, torch_alloc):
     import oracle
     from jacobi_inputs import u12
     ctx = mp.get_context("spawn")
     q = ctx.Queue()
     port = _free_port()
     world = 2
-    procs = [ctx.Process(target=_worker, args=(r, world, port, shape, iters, q)) for r in range(world)]
+    procs = [ctx.Process(target=_worker, args=(r, world, port, shape, iters, q, torch_alloc))
+             for r in range(world)]
     for p in procs:
         p.start()
     res = {}

@@ -304,3 +304,22 @@ def test_resident_watchdog():
         with pytest.raises(jb.JacobiError) as e:
             j.run(10)
         assert e.value.code == jb.JACOBI_ETIMEOUT
+
+
+def test_torch_allocator_owns_device_memory():
+    """With use_torch_allocator() the slab buffers are PyTorch tensors; results are unchanged."""
+    import torch
+    f = u12((70, 300), 8)
+    exp = oracle.jacobi(f, 9)
+    before = torch.cuda.memory_allocated(0)
+    jb.use_torch_allocator()
+    try:
+        with jb.Jacobi(f.shape, virtual=3) as j:
+            assert torch.cuda.memory_allocated(0) > before  # our buffers live in torch's allocator
+            j.scatter(f)
+            j.run(4)
+            j.set_param("resident", 0).run(5)
+            assert_bitwise(j.gather(), exp, "torch allocator")
+    finally:
+        jb.use_torch_allocator(False)
+    assert torch.cuda.memory_allocated(0) == before

@@ -19,7 +19,7 @@ def built():
 
 def test_library_exports_every_header_symbol():
     names = jb.header_functions()
-    assert len(names) == len(jb._SIGS) == 24
+    assert len(names) == len(jb._SIGS) == 26
     L = ctypes.CDLL(jb.LIB_PATH)
     missing = [n for n in names if not hasattr(L, n)]
     assert not missing, missing
@@ -162,3 +162,21 @@ def test_product_package_does_not_import_oracle():
                 src = open(os.path.join(root, f)).read()
                 assert "import oracle" not in src and "from oracle" not in src, f
                 assert "jacobi_oracle" not in src, f
+
+
+def test_slab_bytes_matches_layout():
+    g = jb.jacobi_geometry(1000, 64, 1, 5)
+    total = 0
+    for slab in range(3):
+        s, c = jb.jacobi_decompose(64, 3, slab)
+        b = jb.jacobi_slab_bytes(1000, 64, 1, 5, 3, slab)
+        assert b == (c + 2) * g["plane_elems"] * 8
+        total += c
+    assert total == 62
+
+
+def test_set_allocator_rejects_half():
+    cb = jb.ALLOC_FN(lambda n, d, u: None)
+    with pytest.raises(jb.JacobiError):
+        jb.jacobi_set_allocator(cb, None)
+    jb.jacobi_set_allocator(None, None)
