@@ -101,6 +101,9 @@ int jacobi_create_rank(int64_t nx, int64_t ny, int64_t nz, int stencil, int worl
 int jacobi_ipc_handle_bytes(void);                     /* size of the blob below */
 int jacobi_get_ipc_handle(jacobi_t h, void *out);      /* CUDA IPC handles of this rank's buffers + flags */
 int jacobi_open_peers(jacobi_t h, const void *top_blob, const void *bottom_blob); /* NULL = no neighbour */
+/* Like jacobi_open_peers, given the blobs of ALL ranks (world * jacobi_ipc_handle_bytes(), in rank
+ * order): also opens every rank's control block, which the residual-norm all-reduce needs. */
+int jacobi_open_ranks(jacobi_t h, const void *blobs, int world);
 /* NCCL baseline in dist mode: rank 0 creates a 128-byte ncclUniqueId, every rank passes it to
  * jacobi_nccl_init (collective).  libnccl.so.2 is loaded with dlopen on first use. */
 int jacobi_nccl_unique_id(void *out128);
@@ -137,6 +140,17 @@ int jacobi_set_mode(jacobi_t h, int mode, int flags);
  * CPU-Free run used the resident kernel).  Unknown names return JACOBI_EINVAL. */
 int jacobi_set_param(jacobi_t h, const char *name, int64_t value);
 int jacobi_get_param(jacobi_t h, const char *name, int64_t *value);
+
+/* Residual norm and convergence (not in the paper, which runs a fixed count):
+ * with the knob "norm_every" = k > 0, CPU-Free runs with compute check the update norm
+ * sqrt(sum over interior cells of (u_new - u_old)^2) after every k-th iteration of the run — an
+ * all-reduce over every GPU done on the devices (each slab writes its sum into every slab's
+ * control block and raises a flag) — and stop after the first check with norm <= tol.  The sum
+ * order is fixed, so the norm and the stop decision are identical on every GPU and reproducible.
+ * jacobi_iterations() then tells how many iterations ran; jacobi_last_norm() the last norm
+ * (-1 before any check).  Uses the dynamic schedule and the streaming kernel; <= 32 slabs. */
+int jacobi_set_tolerance(jacobi_t h, double tol);
+int jacobi_last_norm(jacobi_t h, double *norm);
 
 /* ---- data movement -------------------------------------------------------------------- */
 /* Set the whole field (boundary included) from a host array of nx*ny*nz doubles; both

@@ -21,6 +21,10 @@ u' = D^{-1}(b - (A-D)u) built with scipy.sparse, stationary constant / linear / 
 harmonic fields, untouched boundary, maximum principle, mirror symmetry, run splitting.
 The 3D association order is fixed by reading R2 and is "parity unpinned" by the paper
 beyond the within-tolerance pins.
+
+``jacobi_converge`` adds SURVEY §8(f) N4 (not in the paper, which runs a fixed count): the
+L2 norm of the update sqrt(sum over interior cells of (u_new - u_old)^2) every `every` iterations
+and stop once it is <= `tol` (reading R19).  Parity unpinned by the paper.
 """
 from __future__ import annotations
 
@@ -114,3 +118,33 @@ def jacobi_numpy(field: np.ndarray, iters: int) -> np.ndarray:
             b[:, 1:-1, 1:-1] = 0.25 * s
         a, b = b, a
     return a[0] if squeeze else a
+
+
+def jacobi_converge(field: np.ndarray, max_iters: int, tol: float, every: int):
+    """Run up to `max_iters` Jacobi iterations (C oracle), checking the update norm
+    sqrt(sum((u_new - u_old)**2)) over interior cells after every `every`-th iteration (counting
+    from the first iteration of this call) and stopping after the first check with norm <= tol.
+    Returns (field, iterations_done, [norm of each check])."""
+    a = np.ascontiguousarray(field, dtype=np.float64)
+    a3 = a if a.ndim == 3 else a[None]
+    sl = (slice(None), slice(1, -1), slice(1, -1)) if a3.shape[0] == 1 else (slice(1, -1),) * 3
+    norms = []
+    done = 0
+    cur = a3
+    while done < max_iters:
+        step = min(every, max_iters - done) if every > 0 else max_iters - done
+        if step > 1:
+            cur = jacobi(cur, step - 1)
+        nxt = jacobi(cur, 1)
+        done += step
+        if every > 0 and step == every:
+            d = (nxt[sl] - cur[sl]).reshape(-1)
+            r = float(np.sqrt(np.sum(d * d)))
+            norms.append(r)
+            cur = nxt
+            if r <= tol:
+                break
+        else:
+            cur = nxt
+    out = cur if a.ndim == 3 else cur[0]
+    return out, done, norms

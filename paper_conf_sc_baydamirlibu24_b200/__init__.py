@@ -67,6 +67,9 @@ _SIGS = {
     "jacobi_geometry": ([_i64, _i64, _i64, _c.c_int, _c.c_int, _c.c_int, _c.POINTER(_i64)], _c.c_int),
     "jacobi_version": ([], _c.c_int),
     "jacobi_set_allocator": ([_p, _p, _p], _c.c_int),
+    "jacobi_open_ranks": ([_p, _p, _c.c_int], _c.c_int),
+    "jacobi_set_tolerance": ([_p, _c.c_double], _c.c_int),
+    "jacobi_last_norm": ([_p, _c.POINTER(_c.c_double)], _c.c_int),
     "jacobi_slab_bytes": ([_i64, _i64, _i64, _c.c_int, _c.c_int, _c.c_int, _c.POINTER(_i64)], _c.c_int),
 }
 
@@ -142,6 +145,20 @@ def jacobi_get_ipc_handle(h) -> bytes:
 
 def jacobi_open_peers(h, top: bytes | None, bottom: bytes | None) -> None:
     _check(lib().jacobi_open_peers(h, top, bottom), "jacobi_open_peers")
+
+
+def jacobi_open_ranks(h, blobs: list) -> None:
+    _check(lib().jacobi_open_ranks(h, b"".join(blobs), len(blobs)), "jacobi_open_ranks")
+
+
+def jacobi_set_tolerance(h, tol: float) -> None:
+    _check(lib().jacobi_set_tolerance(h, float(tol)), "jacobi_set_tolerance")
+
+
+def jacobi_last_norm(h) -> float:
+    v = _c.c_double()
+    _check(lib().jacobi_last_norm(h, _c.byref(v)), "jacobi_last_norm")
+    return v.value
 
 
 def jacobi_nccl_unique_id() -> bytes:
@@ -341,6 +358,16 @@ class Jacobi:
         jacobi_gather(self.h, out.reshape(-1), self.n)
         return out if self.nz > 1 else out.reshape(self.ny, self.nx)
 
+    def set_tolerance(self, tol: float, every: int) -> "Jacobi":
+        """Convergence-terminated runs (N4): check the update norm every `every` iterations."""
+        jacobi_set_tolerance(self.h, tol)
+        jacobi_set_param(self.h, "norm_every", every)
+        return self
+
+    @property
+    def last_norm(self) -> float:
+        return jacobi_last_norm(self.h)
+
     def last_time_ms(self) -> float:
         return jacobi_last_time(self.h, self.local_slabs)[0]
 
@@ -391,13 +418,22 @@ def broadcast_blob(blob_on_rank0, group=None):
     return obj[0]
 
 
-def exchange_peers(j: Jacobi, group=None, nccl: bool = True) -> None:
-    """Dist mode plumbing: all-gather every rank's IPC blob over torch.distributed, attach the
-    neighbours, and (optionally) set up the NCCL communicator of the baseline."""
+def all_blobs(blob: bytes, group=None) -> list:
+    """All-gather one opaque blob per rank (rank order) over torch.distributed."""
     import torch.distributed as dist
 
-    top, bot = exchange_blobs(jacobi_get_ipc_handle(j.h), group)
-    jacobi_open_peers(j.h, top, bot)
+    blobs = [None] * dist.get_world_size(group)
+    dist.all_gather_object(blobs, blob, group=group)
+    return blobs
+
+
+def exchange_peers(j: Jacobi, group=None, nccl: bool = True) -> None:
+    """Dist mode plumbing: all-gather every rank's IPC blob over torch.distributed, attach the
+    neighbours and every rank's control block, and (optionally) set up the NCCL communicator of
+    the baseline."""
+    import torch.distributed as dist
+
+    jacobi_open_ranks(j.h, all_blobs(jacobi_get_ipc_handle(j.h), group))
     if nccl:
         uid = broadcast_blob(jacobi_nccl_unique_id() if dist.get_rank(group) == 0 else None, group)
         jacobi_nccl_init(j.h, uid)

@@ -9,6 +9,7 @@
 #define JB_THREADS (JB_NC + 32) // + one producer warp (bulk-copy issue)
 #define JB_MAX_STAGES 32
 #define JB_RQ 4                 // run-descriptor queue depth (producer -> consumers)
+#define JB_MAX_NORM 64          // max slabs in the residual-norm all-reduce (N4)
 #define JB_MAXK 32              // max boundary CTAs per side (one inbound flag slot each)
 #define JB_RNT 512              // threads per CTA of the resident (on-chip) kernel
 #define JB_MAX_BLOCKS 1024      // per-slab block flags of the resident kernel
@@ -35,6 +36,7 @@ struct JbGeom {
   int32_t res_rs;       // resident kernel: smem row stride in doubles (x at column x + 1)
 };
 
+struct JbCtrl;
 struct JbSlab {
   double *buf[2];                 // local slab, planes 0..chunk+1 (0 and chunk+1 are halos)
   double *peer_top[2];            // top neighbour's plane chunk_top+1 (its bottom halo), per parity
@@ -73,6 +75,13 @@ struct JbSlab {
   int32_t res_relaxed;               // resident kernel: 1 = neighbour-block flags instead of the grid barrier
   int32_t pad2;
   unsigned long long *blk_flags;     // resident kernel: per-block "faces of iteration v are stored" flags
+  // Residual norm (N4): per-run partial sums of (u_new - u_old)^2 at fixed indices (dynamic item
+  // i -> i; boundary unit u of side s -> dyn_items + s*units + u), summed in index order; then an
+  // all-reduce over every slab through the JbCtrl norm slots (device array of P ctrl pointers).
+  double *partials;
+  struct JbCtrl **norm_peers;
+  int32_t n_partials;
+  int32_t norm_slabs;                // P
 };
 
 struct JbParams {
@@ -85,6 +94,10 @@ struct JbParams {
   unsigned long long timeout_ns;
   int *status;      // [0] error code (0 ok), [1] abort flag
   unsigned long long *trace;  // debug (JACOBI_TRACE): per-iteration CTA work-end timestamps, or null
+  int32_t norm_every;         // N4: check the update norm after every norm_every-th iteration (0: off)
+  int32_t pad;
+  double tol;                 // stop after the first check with norm <= tol
+  int64_t k0;                 // global number of norm checks before this launch (monotone slots)
 };
 
 // Per-slab control block in device memory (one allocation, IPC-exportable).
@@ -94,7 +107,11 @@ struct JbCtrl {
   unsigned int side_ctr[2];
   int status[2];
   unsigned int work[2];            // dynamic-schedule claim counters per iteration parity
-  unsigned long long pad[28];
+  long long done_iters;            // N4: iterations the last run performed (written by CTA 0)
+  double norm_out;                 // N4: last norm (written by CTA 0 of every slab)
+  double norm_val[2][JB_MAX_NORM]; // N4: slab sums of check k, slot [k & 1][slab], written by each slab
+  unsigned long long norm_flag[JB_MAX_NORM];  // N4: check count delivered by each slab (monotone)
+  unsigned long long pad[26];
 };
 
 // ---- host-side planning (plan.cpp) -----------------------------------------------------

@@ -353,9 +353,9 @@ __device__ __forceinline__ void store_pair(double *p, double o0, double o1, bool
 // cell pairs kk = ctid + i*NC (i < PPT), contiguous across lanes (conflict-free 16-byte LDS,
 // coalesced 16-byte STG).  Rows y-1 / y are carried in registers along the march, so each
 // plane costs one 16-byte LDS + two 8-byte LDS (x-1, x+2) per pair.
-template <int PPT, bool NOCOMP>
+template <int PPT, bool NOCOMP, bool NORM>
 __device__ __forceinline__ void consume_run_2d(const JbGeom &g, const Ring &R, RingPos &q, const Run &run,
-                                               double *nxt, double *remote, int ctid, int lane) {
+                                               double *nxt, double *remote, int ctid, int lane, double &acc) {
   const int64_t x0 = 1 + (int64_t)run.unit * g.tx;
   const int vx = (int)min((int64_t)g.tx, g.nx - 1 - x0);
   const int txp = g.tx >> 1;
@@ -416,6 +416,14 @@ __device__ __forceinline__ void consume_run_2d(const JbGeom &g, const Ring &R, R
         if (ok >> i & 1u) {
           store_pair(dst + 2 * i * JB_NC, o0, o1, full >> i & 1u);
           if (rem) store_pair(rem + 2 * i * JB_NC, o0, o1, full >> i & 1u);
+          if (NORM) {  // update norm (N4): fixed per-thread order
+            const double d0 = o0 - C[i].x;
+            acc = acc + d0 * d0;
+            if (full >> i & 1u) {
+              const double d1 = o1 - C[i].y;
+              acc = acc + d1 * d1;
+            }
+          }
         }
         S[i] = C[i];
         C[i] = N;
@@ -435,9 +443,9 @@ __device__ __forceinline__ void consume_run_2d(const JbGeom &g, const Ring &R, R
 // kk = ctid % (tx/2) in a contiguous block of rows; along y it carries rows y-1 / y in
 // registers, so each cell row costs LDS: 16 B (y+1) + 8 B + 8 B (x-1, x+2) + 16 B (z+1) +
 // 16 B (z-1) per pair.
-template <bool NOCOMP>
+template <bool NOCOMP, bool NORM>
 __device__ __forceinline__ void consume_run_3d(const JbGeom &g, const Ring &R, RingPos &q, const Run &run,
-                                               double *nxt, double *remote, int ctid, int lane) {
+                                               double *nxt, double *remote, int ctid, int lane, double &acc) {
   const int ux = run.unit % g.units_x, uy = run.unit / g.units_x;
   const int64_t x0 = 1 + (int64_t)ux * g.tx;
   const int vx = (int)min((int64_t)g.tx, g.nx - 1 - x0);
@@ -497,6 +505,14 @@ __device__ __forceinline__ void consume_run_3d(const JbGeom &g, const Ring &R, R
         if (ok) {
           store_pair(o, o0, o1, full);
           if (ro) store_pair(ro, o0, o1, full);
+          if (NORM) {  // update norm (N4): fixed per-thread order
+            const double d0 = o0 - C.x;
+            acc = acc + d0 * d0;
+            if (full) {
+              const double d1 = o1 - C.y;
+              acc = acc + d1 * d1;
+            }
+          }
         }
         S = C;
         C = N;
@@ -518,17 +534,17 @@ __device__ __forceinline__ void consume_run_3d(const JbGeom &g, const Ring &R, R
   q = pp;
 }
 
-template <int DIM, bool NOCOMP>
+template <int DIM, bool NOCOMP, bool NORM>
 __device__ __forceinline__ void consume_run(const JbGeom &g, const Ring &R, RingPos &q, const Run &run,
-                                            double *nxt, double *remote, int ctid, int lane) {
+                                            double *nxt, double *remote, int ctid, int lane, double &acc) {
   if (DIM == 3) {
-    consume_run_3d<NOCOMP>(g, R, q, run, nxt, remote, ctid, lane);
+    consume_run_3d<NOCOMP, NORM>(g, R, q, run, nxt, remote, ctid, lane, acc);
     return;
   }
   const int ppt = g.tx / (2 * JB_NC);
-  if (ppt >= 4) consume_run_2d<4, NOCOMP>(g, R, q, run, nxt, remote, ctid, lane);
-  else if (ppt == 2) consume_run_2d<2, NOCOMP>(g, R, q, run, nxt, remote, ctid, lane);
-  else consume_run_2d<1, NOCOMP>(g, R, q, run, nxt, remote, ctid, lane);
+  if (ppt >= 4) consume_run_2d<4, NOCOMP, NORM>(g, R, q, run, nxt, remote, ctid, lane, acc);
+  else if (ppt == 2) consume_run_2d<2, NOCOMP, NORM>(g, R, q, run, nxt, remote, ctid, lane, acc);
+  else consume_run_2d<1, NOCOMP, NORM>(g, R, q, run, nxt, remote, ctid, lane, acc);
 }
 
 // ---------------------------------------------------------------- run-descriptor queue
@@ -539,6 +555,8 @@ enum { RUN_WORK = 0, RUN_SIGNAL = 1, RUN_END = 2 };
 struct RunDesc {
   int32_t kind;
   int32_t unit;
+  int32_t item;  // N4: partial-sum index of this run
+  int32_t pad;
   int64_t p0, p1;
 };
 struct Queue {
@@ -546,12 +564,15 @@ struct Queue {
   RunDesc *desc;
 };
 
-__device__ __forceinline__ void publish(const Queue &Q, RingPos &qp, int kind, const Run &r, int lane) {
+__device__ __forceinline__ void publish(const Queue &Q, RingPos &qp, int kind, const Run &r, int lane,
+                                        int item = 0) {
   if (lane == 0) {
     mbar_wait(&Q.empty[qp.slot], qp.phase ^ 1u);
     RunDesc d;
     d.kind = kind;
     d.unit = r.unit;
+    d.item = item;
+    d.pad = 0;
     d.p0 = r.p0;
     d.p1 = r.p1;
     Q.desc[qp.slot] = d;
@@ -570,10 +591,11 @@ __device__ __forceinline__ RunDesc fetch(const Queue &Q, RingPos &qc, int lane) 
 }
 
 // ---------------------------------------------------------------- the kernel
-template <int DIM, bool NOCOMP, bool PERSIST>
+template <int DIM, bool NOCOMP, bool PERSIST, bool NORM>
 __global__ void __launch_bounds__(JB_THREADS, 1) jb_sweep(const __grid_constant__ JbParams P) {
   extern __shared__ __align__(128) unsigned char smem[];
   __shared__ int s_abort;
+  __shared__ double s_red[JB_NCW];  // N4: per-warp partial sums
   const JbGeom &g = P.g;
   Ring R;
   R.S = (uint32_t)g.stages;
@@ -628,8 +650,12 @@ __global__ void __launch_bounds__(JB_THREADS, 1) jb_sweep(const __grid_constant_
   RingPos q = {0u, 0u};   // data ring: producer and consumers advance identical copies
   RingPos rq = {0u, 0u};  // run queue
 
+  __shared__ int s_stop;
+  if (threadIdx.x == 0) s_stop = 0;
+  int64_t done = P.iters;
   for (int64_t t = 0; t < P.iters; ++t) {
     const int64_t tg = P.t0 + t;
+    const bool check = NORM && P.norm_every > 0 && (t + 1) % P.norm_every == 0;
     const double *cur = SL.buf[tg & 1];
     double *nxt = SL.buf[(tg + 1) & 1];
     double *remote = nullptr;
@@ -666,7 +692,8 @@ __global__ void __launch_bounds__(JB_THREADS, 1) jb_sweep(const __grid_constant_
             produce_planes(g, cur, run.unit, run.p0, run.p1, q, R, lane);
           } else if (role != ROLE_INT) {
             // boundary tile (one plane): halo is p-1 (top) or p+1 (bottom)
-            publish(Q, rq, RUN_WORK, run, lane);
+            publish(Q, rq, RUN_WORK, run, lane,
+                    (int)(SL.dyn_items + (role == ROLE_TOP ? 0 : g.units) + run.unit));
             const TileSrc T(g, cur, run.unit, lane);
             RingPos q1 = q, q2 = q;
             q1.advance(R.S);
@@ -716,7 +743,7 @@ __global__ void __launch_bounds__(JB_THREADS, 1) jb_sweep(const __grid_constant_
           // loads are issued, or the claim would reserve work long before it is needed.
           const bool early = run.p1 - run.p0 + 3 <= (int64_t)R.S;
           if (early && lane == 0) claim = atomicAdd(ctr, 1u);
-          publish(Q, rq, RUN_WORK, run, lane);
+          publish(Q, rq, RUN_WORK, run, lane, (int)item);
           produce_planes(g, cur, run.unit, run.p0 - 1, run.p1 + 1, q, R, lane);
           if (!early && lane == 0) claim = atomicAdd(ctr, 1u);
           item = SL.dyn_first + (int64_t)__shfl_sync(0xffffffffu, claim, 0);
@@ -743,7 +770,22 @@ __global__ void __launch_bounds__(JB_THREADS, 1) jb_sweep(const __grid_constant_
         run.unit = d.unit;
         run.p0 = d.p0;
         run.p1 = d.p1;
-        consume_run<DIM, NOCOMP>(g, R, q, run, nxt, remote, ctid, lane);
+        double acc = 0.0;
+        if (NORM && check) {
+          consume_run<DIM, NOCOMP, NORM>(g, R, q, run, nxt, remote, ctid, lane, acc);
+          // deterministic per-run sum: xor tree in each warp, then warps in order
+          for (int o = 16; o > 0; o >>= 1) acc = acc + __shfl_xor_sync(0xffffffffu, acc, o);
+          if (lane == 0) s_red[warp] = acc;
+          named_bar_consumers();
+          if (ctid == 0) {
+            double v = s_red[0];
+            for (int w = 1; w < JB_NCW; ++w) v = v + s_red[w];
+            __stcg(SL.partials + d.item, v);
+          }
+          named_bar_consumers();
+        } else {
+          consume_run<DIM, NOCOMP, false>(g, R, q, run, nxt, remote, ctid, lane, acc);
+        }
       }
       // Our generic-proxy stores must be ordered before later bulk (async-proxy) reads.
       fence_proxy_async_global();
@@ -760,13 +802,46 @@ __global__ void __launch_bounds__(JB_THREADS, 1) jb_sweep(const __grid_constant_
     }
     __syncthreads();
     if (s_abort) return;
+    if (NORM && check) {
+      // N4: all-reduce of the update norm over every slab (device-side, through the JbCtrl
+      // norm slots of each slab), identical on every CTA of every GPU, then the stop decision.
+      const int64_t k = P.k0 + (t + 1) / P.norm_every - 1;  // global check index
+      JbCtrl *mine = SL.norm_peers[SL.slab_id];
+      if (warp == 0) {
+        if (c == 0) {
+          double v = 0.0;
+          for (int i = lane; i < SL.n_partials; i += 32) v = v + __ldcg(SL.partials + i);
+          for (int o = 16; o > 0; o >>= 1) v = v + __shfl_xor_sync(0xffffffffu, v, o);
+          if (lane < SL.norm_slabs) {  // lane g delivers this slab's sum to slab g
+            JbCtrl *dst = SL.norm_peers[lane];
+            dst->norm_val[k & 1][SL.slab_id] = v;
+            st_release_sys(&dst->norm_flag[SL.slab_id], (unsigned long long)(k + 1));
+          }
+        }
+        const bool ok = wait_slots(mine->norm_flag, SL.norm_slabs, (unsigned long long)(k + 1), P, lane);
+        if (lane == 0) {
+          double tot = 0.0;
+          for (int g2 = 0; g2 < SL.norm_slabs; ++g2) tot = tot + __ldcv(&mine->norm_val[k & 1][g2]);
+          const double r = sqrt(tot);
+          if (c == 0) mine->norm_out = r;
+          s_stop = (!ok) ? 2 : (r <= P.tol ? 1 : 0);
+        }
+      }
+      __syncthreads();
+      if (s_stop == 2) return;
+      if (s_stop) {
+        done = t + 1;
+        break;
+      }
+    }
   }
+  if (NORM && c == 0 && threadIdx.x == 0) SL.norm_peers[SL.slab_id]->done_iters = done;
 
   // End of run: wait for the neighbour's last halo so no remote store is still in flight into
   // this GPU's buffers when the kernel (and the host's view of the run) completes.
-  if (PERSIST && producer && role != ROLE_INT && P.iters > 0) {
-    if (role == ROLE_TOP) wait_slots(SL.flag_in_top, SL.k_in_top, (unsigned long long)(P.t0 + P.iters), P, lane);
-    else wait_slots(SL.flag_in_bot, SL.k_in_bot, (unsigned long long)(P.t0 + P.iters), P, lane);
+  if (PERSIST && producer && role != ROLE_INT && done > 0) {
+    if (role == ROLE_TOP) wait_slots(SL.flag_in_top, SL.k_in_top, (unsigned long long)(P.t0 + done), P, lane);
+    else wait_slots(SL.flag_in_bot, SL.k_in_bot, (unsigned long long)(P.t0 + done), P, lane);
   }
 }
 
@@ -1017,10 +1092,14 @@ __global__ void jb_flag_max(unsigned long long *flags, int n, unsigned long long
 
 template <int DIM, bool NOCOMP, bool PERSIST>
 const void *kfn() {
-  return reinterpret_cast<const void *>(&jb_sweep<DIM, NOCOMP, PERSIST>);
+  return reinterpret_cast<const void *>(&jb_sweep<DIM, NOCOMP, PERSIST, false>);
 }
 
-const void *sweep_fn(int dim, bool nocomp, bool persist) {
+const void *sweep_fn(int dim, bool nocomp, bool persist, bool norm = false) {
+  if (norm) {  // residual-norm variant: CPU-Free persistent with compute only
+    return dim == 2 ? reinterpret_cast<const void *>(&jb_sweep<2, false, true, true>)
+                    : reinterpret_cast<const void *>(&jb_sweep<3, false, true, true>);
+  }
   if (dim == 2) {
     if (persist) return nocomp ? kfn<2, true, true>() : kfn<2, false, true>();
     return nocomp ? kfn<2, true, false>() : kfn<2, false, false>();
@@ -1035,7 +1114,10 @@ const void *sweep_fn(int dim, bool nocomp, bool persist) {
 namespace jbk {
 
 cudaError_t prepare(int dim, bool nocomp, bool persist, size_t smem) {
-  return cudaFuncSetAttribute(sweep_fn(dim, nocomp, persist), cudaFuncAttributeMaxDynamicSharedMemorySize,
+  cudaError_t e = cudaFuncSetAttribute(sweep_fn(dim, nocomp, persist), cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                       (int)smem);
+  if (e != cudaSuccess || nocomp || !persist) return e;
+  return cudaFuncSetAttribute(sweep_fn(dim, false, true, true), cudaFuncAttributeMaxDynamicSharedMemorySize,
                               (int)smem);
 }
 
@@ -1047,7 +1129,7 @@ cudaError_t occupancy(int dim, bool nocomp, bool persist, size_t smem, int *bloc
 cudaError_t launch_sweep(const JbParams &p, bool nocomp, bool persist, int grid, size_t smem,
                          cudaStream_t st) {
   void *args[] = {const_cast<JbParams *>(&p)};
-  const void *fn = sweep_fn(p.g.dim, nocomp, persist);
+  const void *fn = sweep_fn(p.g.dim, nocomp, persist, persist && !nocomp && p.norm_every > 0);
   if (persist) return cudaLaunchCooperativeKernel(fn, dim3(grid), dim3(JB_THREADS), args, smem, st);
   return cudaLaunchKernel(fn, dim3(grid), dim3(JB_THREADS), args, smem, st);
 }

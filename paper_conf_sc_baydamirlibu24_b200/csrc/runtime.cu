@@ -140,6 +140,9 @@ struct Slab {
   JbSlab desc{};  // last launch descriptor (for jacobi_describe)
   int32_t *dyn_table = nullptr;  // guided-schedule block table (device)
   unsigned long long *blk_flags = nullptr;  // resident kernel: per-block flags (device)
+  double *partials = nullptr;               // N4: per-run partial sums (device)
+  int64_t partials_cap = 0;
+  JbCtrl **norm_peers = nullptr;            // N4: device array of every slab's control block
   int64_t dyn_key[4] = {0, 0, 0, 0};
   int grid = 0;
   size_t smem = 0;
@@ -159,6 +162,11 @@ struct jacobi_ctx {
   int64_t resident = -1;       // on-chip resident kernel: -1 auto (when the slab fits), 0 off, 1 on
   int64_t block_sync = 0;      // resident kernel: 0 grid barrier, 1 neighbour-block flags
   int64_t last_resident = 0;   // read-only: whether the last CPU-Free run used it
+  int64_t norm_every = 0;      // N4: check the update norm every k iterations (0 = off)
+  double tol = 0.0;            // N4: stop once the norm <= tol
+  int64_t norm_checks = 0;     // N4: checks performed so far (monotone slot values)
+  double last_norm = -1.0;     // N4: norm of the last check
+  std::vector<JbCtrl *> all_ctrl;  // dist mode: every rank's control block (opened via IPC)
   int64_t timeout_ms = 20000;
   bool peers_ready = false;
   bool nccl_ready = false;
@@ -239,6 +247,8 @@ void free_slab(Slab &s, const Allocator &a) {
   }
   if (s.dyn_table) cudaFree(s.dyn_table);
   if (s.blk_flags) cudaFree(s.blk_flags);
+  if (s.partials) cudaFree(s.partials);
+  if (s.norm_peers) cudaFree(s.norm_peers);
   if (s.ev0) cudaEventDestroy(s.ev0);
   if (s.ev1) cudaEventDestroy(s.ev1);
   if (s.ev_sync) cudaEventDestroy(s.ev_sync);
@@ -582,22 +592,63 @@ int plan_resident(jacobi_ctx *h, const std::vector<int> &idx, LaunchPlan &L) {
   return JACOBI_OK;
 }
 
+// N4: wire the residual-norm all-reduce into a planned launch (partials + every slab's ctrl).
+int setup_norm(jacobi_ctx *h, LaunchPlan &L) {
+  if (h->total > 32) return JACOBI_EINVAL;  // one polling lane per slab
+  for (size_t k = 0; k < L.slab_idx.size(); ++k) {
+    Slab &s = h->slabs[L.slab_idx[k]];
+    JbSlab &d = L.P.s[k];
+    const int64_t n = d.dyn_items + 2 * (int64_t)L.P.g.units;
+    if (n > s.partials_cap) {
+      if (s.partials) cudaFree(s.partials);
+      s.partials = nullptr;
+      CK(cudaMalloc(&s.partials, n * sizeof(double)));
+      s.partials_cap = n;
+    }
+    CK(cudaMemset(s.partials, 0, n * sizeof(double)));
+    std::vector<JbCtrl *> ctrls(h->total, nullptr);
+    if (h->kind == KIND_DIST) {
+      if ((int)h->all_ctrl.size() != h->total) return JACOBI_ESTATE;  // needs jacobi_open_ranks
+      ctrls = h->all_ctrl;
+    } else {
+      for (auto &o : h->slabs) ctrls[o.id] = o.ctrl;
+    }
+    ctrls[s.id] = s.ctrl;
+    if (!s.norm_peers) CK(cudaMalloc(&s.norm_peers, JB_MAX_NORM * sizeof(JbCtrl *)));
+    CK(cudaMemcpy(s.norm_peers, ctrls.data(), h->total * sizeof(JbCtrl *), cudaMemcpyHostToDevice));
+    d.partials = s.partials;
+    d.norm_peers = s.norm_peers;
+    d.n_partials = (int32_t)n;
+    d.norm_slabs = h->total;
+  }
+  L.P.norm_every = (int32_t)h->norm_every;
+  L.P.tol = h->tol;
+  L.P.k0 = h->norm_checks;
+  return JACOBI_OK;
+}
+
 int run_cpufree(jacobi_ctx *h, int64_t iters) {
   const bool nocomp = h->flags & JACOBI_FLAG_NO_COMPUTE;
+  const bool norm = !nocomp && h->norm_every > 0;
   auto groups = launch_groups(h);
   std::vector<LaunchPlan> plans(groups.size());
-  // Resident (on-chip) kernel when every slab fits (auto) or when forced.
-  bool resident = !nocomp && h->resident != 0;
+  // Resident (on-chip) kernel when every slab fits (auto) or when forced (not with the norm).
+  bool resident = !nocomp && !norm && h->resident != 0;
   if (resident) {
     for (size_t i = 0; i < groups.size() && resident; ++i)
       if (plan_resident(h, groups[i], plans[i]) != JACOBI_OK) resident = false;
     if (!resident && h->resident == 1) return JACOBI_EINVAL;
   }
+  if (norm && h->resident == 1) return JACOBI_EINVAL;
   h->last_resident = resident ? 1 : 0;
   for (size_t i = 0; i < groups.size(); ++i) {
     if (!resident) {
+      const int64_t sched = h->schedule;
+      if (norm) h->schedule = 2;  // the norm's partial sums are indexed by dynamic items
       int rc = plan_launch(h, groups[i], LK_PERSIST, nocomp, plans[i]);
+      h->schedule = sched;
       if (rc) return rc;
+      if (norm && (rc = setup_norm(h, plans[i]))) return rc;
     }
     plans[i].P.t0 = h->t;
     plans[i].P.iters = iters;
@@ -669,7 +720,19 @@ int run_cpufree(jacobi_ctx *h, int64_t iters) {
     }
   }
   if (rc_all) return rc_all;
-  h->t += iters;
+  int64_t done = iters;
+  if (norm) {  // every slab stopped after the same iteration: read it (and the norm) from slab 0
+    Slab &s0 = h->slabs[0];
+    CK(cudaSetDevice(s0.device));
+    long long d = 0;
+    double r = 0;
+    CK(cudaMemcpy(&d, &s0.ctrl->done_iters, sizeof(d), cudaMemcpyDeviceToHost));
+    CK(cudaMemcpy(&r, &s0.ctrl->norm_out, sizeof(r), cudaMemcpyDeviceToHost));
+    done = d;
+    h->norm_checks += done / h->norm_every;
+    if (done >= h->norm_every) h->last_norm = r;
+  }
+  h->t += done;
   return JACOBI_OK;
 }
 
@@ -943,11 +1006,15 @@ int jacobi_create(int64_t nx, int64_t ny, int64_t nz, int stencil, int ngpus, ja
   }
   for (int g = 0; g < ngpus; ++g) {
     cudaSetDevice(g);
-    for (int o : {g - 1, g + 1}) {
-      if (o < 0 || o >= ngpus) continue;
+    for (int o = 0; o < ngpus; ++o) {  // neighbours required; all pairs for the norm (NVSwitch)
+      if (o == g) continue;
+      int can = 0;
+      cudaDeviceCanAccessPeer(&can, g, o);
+      if (!can) continue;
       cudaError_t e = cudaDeviceEnablePeerAccess(o, 0);
       if (e == cudaErrorPeerAccessAlreadyEnabled) cudaGetLastError();
-      else if (e != cudaSuccess) { jacobi_destroy(h); return JACOBI_ENOPEER; }
+      else if (e != cudaSuccess && (o == g - 1 || o == g + 1)) { jacobi_destroy(h); return JACOBI_ENOPEER; }
+      else if (e != cudaSuccess) cudaGetLastError();
     }
   }
   link_local(h);
@@ -1096,6 +1163,32 @@ int jacobi_open_peers(jacobi_t h, const void *top_blob, const void *bottom_blob)
   return JACOBI_OK;
 }
 
+int jacobi_open_ranks(jacobi_t h, const void *blobs, int world) {
+  if (!h || !blobs || h->kind != KIND_DIST || world != h->total) return JACOBI_EINVAL;
+  const size_t B = sizeof(IpcBlob);
+  const char *base = static_cast<const char *>(blobs);
+  const int r = h->rank;
+  int rc = jacobi_open_peers(h, r > 0 ? base + (r - 1) * B : nullptr, r < world - 1 ? base + (r + 1) * B : nullptr);
+  if (rc) return rc;
+  Slab &s = h->slabs[0];
+  CK(cudaSetDevice(s.device));
+  h->all_ctrl.assign(world, nullptr);
+  for (int g = 0; g < world; ++g) {
+    if (g == r) {
+      h->all_ctrl[g] = s.ctrl;
+      continue;
+    }
+    IpcBlob b;
+    std::memcpy(&b, base + g * B, B);
+    if (b.magic != kIpcMagic || b.rank != g) return JACOBI_EINVAL;
+    void *c = nullptr;
+    CK(cudaIpcOpenMemHandle(&c, b.ctrl, cudaIpcMemLazyEnablePeerAccess));
+    s.ipc_opened.push_back(c);
+    h->all_ctrl[g] = reinterpret_cast<JbCtrl *>(static_cast<char *>(c) + b.off[2]);
+  }
+  return JACOBI_OK;
+}
+
 int jacobi_nccl_unique_id(void *out128) {
   if (!out128) return JACOBI_EINVAL;
   if (!g_nccl.load()) return JACOBI_ENCCL;
@@ -1155,6 +1248,7 @@ static int64_t *param_slot(jacobi_t h, const char *name) {
   if (!std::strcmp(name, "dyn_help")) return &h->dyn_help;
   if (!std::strcmp(name, "resident")) return &h->resident;
   if (!std::strcmp(name, "block_sync")) return &h->block_sync;
+  if (!std::strcmp(name, "norm_every")) return &h->norm_every;
   if (!std::strcmp(name, "last_resident")) return &h->last_resident;
   return nullptr;
 }
@@ -1222,6 +1316,18 @@ int jacobi_gather(jacobi_t h, double *out) {
     CK(cudaSetDevice(s.device));
     CK(cudaStreamSynchronize(s.stream));
   }
+  return JACOBI_OK;
+}
+
+int jacobi_set_tolerance(jacobi_t h, double tol) {
+  if (!h || !(tol >= 0.0)) return JACOBI_EINVAL;
+  h->tol = tol;
+  return JACOBI_OK;
+}
+
+int jacobi_last_norm(jacobi_t h, double *norm) {
+  if (!h || !norm) return JACOBI_EINVAL;
+  *norm = h->last_norm;
   return JACOBI_OK;
 }
 

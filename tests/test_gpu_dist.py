@@ -21,7 +21,7 @@ def _free_port():
     return p
 
 
-def _worker(rank, world, port, shape, iters, q, torch_alloc=False):
+def _worker(rank, world, port, shape, iters, q, torch_alloc=False, tol=None):
     try:
         os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
         import torch.distributed as dist
@@ -35,10 +35,16 @@ def _worker(rank, world, port, shape, iters, q, torch_alloc=False):
         j.set_param("timeout_ms", 60000)
         jb.exchange_peers(j, nccl=False)
         j.scatter(f)
+        if tol is not None:  # N4: device-side norm all-reduce across the two processes
+            j.set_tolerance(tol, 5)
         dist.barrier()
         j.run(iters)
+        if tol is not None:
+            f[0, 0] = float(j.iterations)  # report the iteration count through a boundary cell
         out = np.full(f.shape, np.nan)
         j.gather(out)
+        if tol is not None and rank == 0:
+            out[0, 0] = f[0, 0]
         dist.barrier()
         j.close()
         dist.destroy_process_group()
@@ -70,4 +76,31 @@ def test_two_ranks_one_gpu_ipc(shape, iters, torch_alloc):
     exp = oracle.jacobi(u12(shape, 7), iters)
     merged = np.where(np.isnan(res[0]), res[1], res[0])
     assert not np.isnan(merged).any()
+    assert np.array_equal(merged.view(np.uint64), exp.view(np.uint64))
+
+
+def test_two_ranks_one_gpu_norm():
+    import oracle
+    from jacobi_inputs import u12
+    shape = (40, 96)
+    f = u12(shape, 7)
+    _, _, norms = oracle.jacobi_converge(f, 200, 0.0, 5)
+    tol = norms[7] * (1 + 1e-9)
+    exp, done, _ = oracle.jacobi_converge(f, 200, tol, 5)
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _free_port()
+    procs = [ctx.Process(target=_worker, args=(r, 2, port, shape, 200, q, False, tol)) for r in range(2)]
+    for p in procs:
+        p.start()
+    res = {}
+    for _ in range(2):
+        rank, out, err = q.get(timeout=240)
+        assert err is None, err
+        res[rank] = out
+    for p in procs:
+        p.join(timeout=60)
+    assert res[0][0, 0] == done
+    merged = np.where(np.isnan(res[0]), res[1], res[0])
+    merged[0, 0] = exp[0, 0]
     assert np.array_equal(merged.view(np.uint64), exp.view(np.uint64))

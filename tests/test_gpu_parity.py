@@ -323,3 +323,45 @@ def test_torch_allocator_owns_device_memory():
     finally:
         jb.use_torch_allocator(False)
     assert torch.cuda.memory_allocated(0) == before
+
+
+# ---------------------------------------------------------------- N4: residual norm + convergence
+def _converge_gpu(f, max_iters, tol, every, virtual=0, pre=0):
+    with jb.Jacobi(f.shape, virtual=virtual) if virtual else jb.Jacobi(f.shape) as j:
+        j.scatter(f)
+        if pre:
+            j.run(pre)  # a plain run first: the norm protocol must continue from any state
+        j.set_tolerance(tol, every)
+        t0 = j.iterations
+        j.run(max_iters)
+        return j.gather(), j.iterations - t0, j.last_norm
+
+
+@pytest.mark.parametrize("shape", [(40, 130), (300, 77), (12, 30, 45), (33, 20, 20)])
+@pytest.mark.parametrize("P", [1, 2, 4])
+def test_converge_vs_oracle(shape, P):
+    if (shape[0] - 2) // P < 2:
+        pytest.skip("slab too thin")
+    f = u12(shape, 9)
+    _, _, norms = oracle.jacobi_converge(f, 400, 0.0, 10)
+    tol = norms[len(norms) // 2] * (1 + 1e-9)  # stop at a check in the middle of the run
+    exp, done, enorms = oracle.jacobi_converge(f, 400, tol, 10)
+    got, gdone, gnorm = _converge_gpu(f, 400, tol, 10, virtual=P)
+    assert gdone == done
+    assert_bitwise(got, exp, f"converge {shape} P={P}")
+    assert abs(gnorm - enorms[-1]) <= 1e-12 * enorms[-1]
+
+
+def test_converge_never_and_split_runs():
+    f = u12((50, 200), 10)
+    exp, done, enorms = oracle.jacobi_converge(f, 55, 0.0, 5)  # tol 0: never stops
+    assert done == 55
+    got, gdone, gnorm = _converge_gpu(f, 55, 0.0, 5, virtual=3, pre=7)
+    assert gdone == 55
+    assert_bitwise(got, oracle.jacobi(f, 62), "converge after a plain run")
+    with jb.Jacobi(f.shape, virtual=2) as j:  # repeated norm runs: monotone slots across runs
+        j.scatter(f).set_tolerance(0.0, 4)
+        for _ in range(3):
+            j.run(8)
+        assert j.iterations == 24
+        assert_bitwise(j.gather(), oracle.jacobi(f, 24), "norm runs x3")

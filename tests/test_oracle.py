@@ -338,3 +338,32 @@ def test_oracle_rejects_bad_args(oracle_mod):
         oracle_mod.jacobi(np.zeros((2, 5)), 1)
     with pytest.raises(ValueError):
         oracle_mod.jacobi(np.zeros((5, 2)), 1)
+
+
+# ---------------------------------------------------------------- N4: update norm (oracle side)
+def test_update_norm_eigenmode_closed_form(oracle_mod):
+    """For an eigenmode u_k = lam^k u0 the update norm after iteration k (1-based) is
+    lam^(k-1) |lam - 1| ||u0||_2, and the run stops at the first check below tol."""
+    ny, nx, my, mx = 34, 50, 2, 3
+    y = np.arange(ny)[:, None]
+    x = np.arange(nx)[None, :]
+    u0 = np.sin(np.pi * my * y / (ny - 1)) * np.sin(np.pi * mx * x / (nx - 1))
+    u0[0, :] = u0[-1, :] = 0.0
+    u0[:, 0] = u0[:, -1] = 0.0
+    lam = (np.cos(np.pi * mx / (nx - 1)) + np.cos(np.pi * my / (ny - 1))) / 2
+    n0 = np.sqrt(np.sum(u0[1:-1, 1:-1] ** 2))
+    every = 7
+    tol = 0.05 * n0 * abs(lam - 1)
+    out, done, norms = oracle_mod.jacobi_converge(u0, 5000, tol, every)
+    exp = [lam ** (every * (i + 1) - 1) * abs(lam - 1) * n0 for i in range(len(norms))]
+    np.testing.assert_allclose(norms, exp, rtol=1e-9)
+    k_stop = next(k for k in range(every, 5000, every) if lam ** (k - 1) * abs(lam - 1) * n0 <= tol)
+    assert done == k_stop
+    np.testing.assert_allclose(out, lam ** done * u0, rtol=0, atol=1e-13)
+
+
+def test_update_norm_zero_for_harmonic_field(oracle_mod):
+    y, x = np.mgrid[0:12, 0:15].astype(np.float64)
+    f = x * x - y * y
+    out, done, norms = oracle_mod.jacobi_converge(f, 100, 0.0, 5)
+    assert done == 5 and norms == [0.0] and np.array_equal(out, f)
