@@ -188,6 +188,8 @@ def main():
     ap.add_argument("--no-extras", action="store_true", help="skip e2e / cpu_baseline / baselines")
     ap.add_argument("--virtual", type=int, default=0, help="(measurement aid) P slabs on one GPU")
     ap.add_argument("--param", action="append", default=[], help="tuning knob name=value (jacobi_set_param)")
+    ap.add_argument("--transport", default="ipc", choices=["ipc", "nvshmem"],
+                    help="N>1: CUDA IPC peer stores (default) or the NVSHMEM variant (N3)")
     args = ap.parse_args()
     args.warmup = max(args.warmup, 3) if args.impl == "ours" else args.warmup
 
@@ -206,13 +208,19 @@ def main():
     import paper_conf_sc_baydamirlibu24_b200 as jb
 
     torch.cuda.set_device(local)
-    jb.use_torch_allocator()  # PyTorch owns the device memory of the slabs (north star)
-    if world > 1:
+    if world > 1 and args.transport == "nvshmem":
+        import torch.distributed as dist
+        dist.init_process_group("gloo")
+        j = jb.create_nvshmem(shape, device=local)  # symmetric heap owns the slabs
+        args.no_extras = True  # CPU-controlled baselines / e2e use the IPC build
+    elif world > 1:
+        jb.use_torch_allocator()  # PyTorch owns the device memory of the slabs (north star)
         import torch.distributed as dist
         dist.init_process_group("gloo")
         j = jb.Jacobi(shape, dist=(rank, world), device=local)
         jb.exchange_peers(j, nccl=True)
     else:
+        jb.use_torch_allocator()
         dist = None
         j = jb.Jacobi(shape, virtual=args.virtual) if args.virtual else jb.Jacobi(shape, ngpus=1)
     torch.cuda.set_device(local)
@@ -270,6 +278,7 @@ def main():
 
     line = {
         "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
+        "transport": args.transport if world > 1 else "none",
         "warmup": args.warmup, "ms_per_step": dev_ms / args.steps, "higher_is_better": True,
         "scaling": cfg["scaling"], "vs_baseline": None, "dtype": "f64",
         "data": "synthetic (U12 seed 0x5C24, initialised on the device)",
@@ -368,6 +377,8 @@ def main():
     if rank == 0:
         print(json.dumps(line), flush=True)
     j.close()
+    if args.transport == "nvshmem" and world > 1:
+        jb.nvshmem_finalize()
     if dist is not None:
         dist.barrier()
         dist.destroy_process_group()

@@ -122,6 +122,20 @@ int jacobi_set_allocator(jacobi_alloc_fn alloc, jacobi_free_fn free_fn, void *us
 /* Bytes of ONE field buffer of slab `slab` (of `nslabs`) for this grid (host-only helper). */
 int jacobi_slab_bytes(int64_t nx, int64_t ny, int64_t nz, int stencil, int nslabs, int slab, int64_t *bytes);
 
+/* ---- NVSHMEM variant — exported ONLY by libjacobi_b200_nvshmem.so --------
+ * Same library built with -DJB_NVSHMEM: one PE per process; the slab buffers and control blocks
+ * live on the NVSHMEM symmetric heap and the CPU-Free kernel's boundary blocks deliver halos with
+ * nvshmemx_putmem_signal_nbi_warp / nvshmem signals (the paper's own layer) instead
+ * of raw peer stores.  Rank 0 calls jacobi_nvshmem_uid(); every rank passes that id (any
+ * transport) to jacobi_create_nvshmem (collective, once per process; NVSHMEM_SYMMETRIC_SIZE is
+ * set from the grid if unset).  jacobi_destroy is collective for these handles; call
+ * jacobi_nvshmem_finalize() before process exit.  Baseline modes are not available here. */
+int jacobi_nvshmem_uid_bytes(void);
+int jacobi_nvshmem_uid(void *out);
+int jacobi_create_nvshmem(int64_t nx, int64_t ny, int64_t nz, int stencil, const void *uid, int world_size,
+                          int rank, int device, jacobi_t *out);
+int jacobi_nvshmem_finalize(void);
+
 /* ---- running ----------------------------------------------------------------------------- */
 /* Advance the field by `iters` Jacobi iterations in the current mode.  Continues from the
  * current state: run(a); run(b) == run(a+b) bitwise.  run(0) is a no-op.  Blocks until done. */

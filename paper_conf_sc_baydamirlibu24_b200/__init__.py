@@ -16,6 +16,7 @@ import numpy as np
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
 LIB_PATH = os.environ.get("JACOBI_LIB") or os.path.join(_HERE, "libjacobi_b200.so")  # env: A/B measurement aid
+NVSHMEM_LIB_PATH = os.path.join(_HERE, "libjacobi_b200_nvshmem.so")
 HEADER_PATH = os.path.join(os.path.dirname(_HERE), "include", "jacobi.h")
 
 JACOBI_OK = 0
@@ -72,6 +73,14 @@ _SIGS = {
     "jacobi_last_norm": ([_p, _c.POINTER(_c.c_double)], _c.c_int),
     "jacobi_slab_bytes": ([_i64, _i64, _i64, _c.c_int, _c.c_int, _c.c_int, _c.POINTER(_i64)], _c.c_int),
 }
+# exported only by the NVSHMEM variant (libjacobi_b200_nvshmem.so)
+_SIGS_NVSHMEM = {
+    "jacobi_nvshmem_uid_bytes": ([], _c.c_int),
+    "jacobi_nvshmem_uid": ([_p], _c.c_int),
+    "jacobi_create_nvshmem": ([_i64, _i64, _i64, _c.c_int, _p, _c.c_int, _c.c_int, _c.c_int, _c.POINTER(_p)],
+                              _c.c_int),
+    "jacobi_nvshmem_finalize": ([], _c.c_int),
+}
 
 ALLOC_FN = _c.CFUNCTYPE(_c.c_void_p, _c.c_size_t, _c.c_int, _c.c_void_p)
 FREE_FN = _c.CFUNCTYPE(None, _c.c_void_p, _c.c_int, _c.c_void_p)
@@ -92,7 +101,8 @@ def lib() -> ctypes.CDLL:
         if not os.path.exists(LIB_PATH):
             raise RuntimeError(f"CUDA extension missing: {LIB_PATH} (run __graft_entry__.build())")
         L = ctypes.CDLL(LIB_PATH)
-        for name, (args, res) in _SIGS.items():
+        sigs = dict(_SIGS, **(_SIGS_NVSHMEM if LIB_PATH == NVSHMEM_LIB_PATH else {}))
+        for name, (args, res) in sigs.items():
             fn = getattr(L, name)
             fn.argtypes = args
             fn.restype = res
@@ -100,11 +110,24 @@ def lib() -> ctypes.CDLL:
     return _lib
 
 
-def header_functions() -> list[str]:
-    """Names of every function declared in include/jacobi.h."""
+def use_nvshmem() -> None:
+    """Switch this process to the NVSHMEM variant of the library (N3).  Must be called before the
+    library is first used; every call of this module then goes through that library."""
+    global LIB_PATH
+    if _lib is not None and LIB_PATH != NVSHMEM_LIB_PATH:
+        raise RuntimeError("use_nvshmem() must precede the first use of the library")
+    if not os.path.exists(NVSHMEM_LIB_PATH):
+        raise RuntimeError(f"NVSHMEM variant missing: {NVSHMEM_LIB_PATH}")
+    LIB_PATH = NVSHMEM_LIB_PATH
+
+
+def header_functions(nvshmem: bool = False) -> list[str]:
+    """Names of the functions declared in include/jacobi.h: those of the main library, or (with
+    nvshmem=True) those exported only by the NVSHMEM variant."""
     with open(HEADER_PATH) as f:
         src = f.read()
-    return re.findall(r"^\s*(?:int|const char \*)\s*(jacobi_\w+)\s*\(", src, flags=re.M)
+    names = re.findall(r"^\s*(?:int|const char \*)\s*(jacobi_\w+)\s*\(", src, flags=re.M)
+    return [n for n in names if (n in _SIGS_NVSHMEM) == nvshmem]
 
 
 def strerror(code: int) -> str:
@@ -317,7 +340,7 @@ def use_torch_allocator(enable: bool = True) -> None:
 class Jacobi:
     """One handle of the library.  shape = (nz, ny, nx) or (ny, nx) including the boundary."""
 
-    def __init__(self, shape, ngpus: int = 1, virtual: int = 0, device: int = 0, dist=None):
+    def _init_shape(self, shape):
         shape = tuple(int(s) for s in shape)
         if len(shape) == 2:
             shape = (1,) + shape
@@ -326,6 +349,10 @@ class Jacobi:
         self.nx, self.ny, self.nz = nx, ny, nz
         self.stencil = 5 if nz == 1 else 7
         self.n = nx * ny * nz
+
+    def __init__(self, shape, ngpus: int = 1, virtual: int = 0, device: int = 0, dist=None):
+        self._init_shape(shape)
+        nz, ny, nx = self.shape
         if dist is not None:
             rank, world = dist
             self.h = jacobi_create_rank(nx, ny, nz, self.stencil, world, rank, device)
@@ -394,6 +421,32 @@ class Jacobi:
             self.close()
         except Exception:
             pass
+
+
+def create_nvshmem(shape, group=None, device: int = 0) -> "Jacobi":
+    """N3: one NVSHMEM PE per rank of `group` (torch.distributed carries the unique id)."""
+    import torch.distributed as dist
+
+    use_nvshmem()
+    rank, world = dist.get_rank(group), dist.get_world_size(group)
+    uid = None
+    if rank == 0:
+        buf = _c.create_string_buffer(lib().jacobi_nvshmem_uid_bytes())
+        _check(lib().jacobi_nvshmem_uid(buf), "jacobi_nvshmem_uid")
+        uid = buf.raw
+    uid = broadcast_blob(uid, group)
+    j = Jacobi.__new__(Jacobi)
+    j._init_shape(shape)
+    h = _p()
+    _check(lib().jacobi_create_nvshmem(j.nx, j.ny, j.nz, j.stencil, uid, world, rank, device, _c.byref(h)),
+           "jacobi_create_nvshmem")
+    j.h = h.value
+    j.local_slabs, j.total_slabs = jacobi_num_slabs(j.h)
+    return j
+
+
+def nvshmem_finalize() -> None:
+    lib().jacobi_nvshmem_finalize()
 
 
 def exchange_blobs(blob: bytes, group=None):

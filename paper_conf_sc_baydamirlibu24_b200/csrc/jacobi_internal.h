@@ -82,6 +82,11 @@ struct JbSlab {
   struct JbCtrl **norm_peers;
   int32_t n_partials;
   int32_t norm_slabs;                // P
+  // NVSHMEM variant (N3, libjacobi_b200_nvshmem.so only): peer_top/peer_bot and flag_out_* are
+  // symmetric-heap addresses, written with nvshmemx_putmem(_signal)_nbi_warp to these PEs.
+  int32_t use_shm;
+  int32_t shm_pe_top, shm_pe_bot;
+  int32_t pad3;
 };
 
 struct JbParams {

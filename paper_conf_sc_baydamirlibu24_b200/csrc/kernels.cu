@@ -23,6 +23,10 @@
 
 #include "../../include/jacobi.h"
 #include "jacobi_internal.h"
+#ifdef JB_NVSHMEM
+#include <nvshmem.h>
+#include <nvshmemx.h>
+#endif
 
 namespace {
 
@@ -590,6 +594,51 @@ __device__ __forceinline__ RunDesc fetch(const Queue &Q, RingPos &qc, int lane) 
   return d;
 }
 
+#ifdef JB_NVSHMEM
+// N3 — the paper's own communication layer: after a boundary CTA computed its edge
+// tiles, one warp sends them into the neighbour PE's halo with nvshmemx_putmem_nbi_warp, row by
+// row, and the last row with nvshmemx_putmem_signal_nbi_warp, which sets this CTA's flag slot on
+// the neighbour to t+1 once the data is there (nvshmem_fence orders the earlier rows before it).
+// (NO_COMPUTE: the owned edge plane of the current buffer is sent as-is.)
+template <int DIM, bool NOCOMP>
+__device__ void shm_put_boundary(const JbGeom &g, const JbSlab &SL, int role, int ridx, int rcount,
+                                 const double *cur, double *nxt, int64_t tg, bool drop_signal) {
+  const Sched sc = make_sched(g, SL, role, ridx, rcount);
+  const int pe = role == ROLE_TOP ? SL.shm_pe_top : SL.shm_pe_bot;
+  double *dst_plane = role == ROLE_TOP ? SL.peer_top[(tg + 1) & 1] : SL.peer_bot[(tg + 1) & 1];
+  uint64_t *sig = reinterpret_cast<uint64_t *>((role == ROLE_TOP ? SL.flag_out_top : SL.flag_out_bot) + ridx);
+  const double *src_plane = (NOCOMP ? cur : nxt) + sc.plane * g.plane_elems;
+  int rows_left = 0;
+  for (int u = sc.ub; u < sc.ue; ++u) {
+    const int uy = u / g.units_x;
+    const int64_t y0 = 1 + (int64_t)uy * g.ty;
+    rows_left += DIM == 3 ? (int)min((int64_t)g.ty, g.ny - 1 - y0) : 1;
+  }
+  bool signalled = false;
+  for (int u = sc.ub; u < sc.ue; ++u) {
+    const int ux = u % g.units_x, uy = u / g.units_x;
+    const int64_t x0 = 1 + (int64_t)ux * g.tx;
+    const int64_t vx = min((int64_t)g.tx, g.nx - 1 - x0);
+    const int64_t y0 = DIM == 3 ? 1 + (int64_t)uy * g.ty : 0;
+    const int vy = DIM == 3 ? (int)min((int64_t)g.ty, g.ny - 1 - y0) : 1;
+    for (int r = 0; r < vy; ++r) {
+      const int64_t off = (DIM == 3 ? (y0 + r) * g.pitch : 0) + 3 + x0;
+      if (--rows_left > 0 || drop_signal) {
+        nvshmemx_putmem_nbi_warp(dst_plane + off, src_plane + off, vx * sizeof(double), pe);
+      } else {
+        nvshmem_fence();
+        nvshmemx_putmem_signal_nbi_warp(dst_plane + off, src_plane + off, vx * sizeof(double), sig,
+                                        (uint64_t)(tg + 1), NVSHMEM_SIGNAL_SET, pe);
+        signalled = true;
+      }
+    }
+  }
+  if (!signalled && !drop_signal && (threadIdx.x & 31) == 0)
+    nvshmemx_signal_op(sig, (uint64_t)(tg + 1), NVSHMEM_SIGNAL_SET, pe);
+  nvshmem_quiet();  // the source planes may be overwritten two iterations later
+}
+#endif
+
 // ---------------------------------------------------------------- the kernel
 template <int DIM, bool NOCOMP, bool PERSIST, bool NORM>
 __global__ void __launch_bounds__(JB_THREADS, 1) jb_sweep(const __grid_constant__ JbParams P) {
@@ -658,9 +707,9 @@ __global__ void __launch_bounds__(JB_THREADS, 1) jb_sweep(const __grid_constant_
     const bool check = NORM && P.norm_every > 0 && (t + 1) % P.norm_every == 0;
     const double *cur = SL.buf[tg & 1];
     double *nxt = SL.buf[(tg + 1) & 1];
-    double *remote = nullptr;
-    if (role == ROLE_TOP) remote = SL.peer_top[(tg + 1) & 1];
-    if (role == ROLE_BOT) remote = SL.peer_bot[(tg + 1) & 1];
+    double *remote = nullptr;  // peer stores (UVA / IPC); the NVSHMEM variant puts after the run
+    if (role == ROLE_TOP && !SL.use_shm) remote = SL.peer_top[(tg + 1) & 1];
+    if (role == ROLE_BOT && !SL.use_shm) remote = SL.peer_bot[(tg + 1) & 1];
     const bool active = !(NOCOMP && role == ROLE_INT);
 
     if (producer) {
@@ -759,6 +808,13 @@ __global__ void __launch_bounds__(JB_THREADS, 1) jb_sweep(const __grid_constant_
           if (PERSIST) named_bar_consumers();
           // bar.sync makes every consumer thread's peer stores precede thread 0 (CTA scope);
           // its sys-scope release store into this CTA's slot publishes them to the neighbour.
+#ifdef JB_NVSHMEM
+          if (PERSIST && SL.use_shm) {
+            if (warp == 0) shm_put_boundary<DIM, NOCOMP>(g, SL, role, ridx, rcount, cur, nxt, tg, drop_signal);
+            remote = nullptr;
+            continue;
+          }
+#endif
           if (PERSIST && ctid == 0 && !drop_signal) {
             unsigned long long *fo = role == ROLE_TOP ? SL.flag_out_top : SL.flag_out_bot;
             st_release_sys(fo + ridx, (unsigned long long)(tg + 1));

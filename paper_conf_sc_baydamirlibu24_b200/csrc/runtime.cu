@@ -17,6 +17,10 @@
 
 #include "../../include/jacobi.h"
 #include "jacobi_internal.h"
+#ifdef JB_NVSHMEM
+#include <nvshmem.h>
+#include <nvshmemx.h>
+#endif
 
 namespace jbk {
 cudaError_t prepare(int dim, bool nocomp, bool persist, size_t smem);
@@ -33,7 +37,7 @@ cudaError_t launch_resident(const JbParams &p, int cpp, int grid, size_t smem, c
 namespace {
 
 constexpr unsigned long long kSeedBench = 0x5C24ull;
-enum Kind { KIND_SINGLE = 0, KIND_VIRTUAL = 1, KIND_DIST = 2 };
+enum Kind { KIND_SINGLE = 0, KIND_VIRTUAL = 1, KIND_DIST = 2, KIND_SHMEM = 3 };
 
 int cuda_err(cudaError_t e) {
   if (e == cudaSuccess) return JACOBI_OK;
@@ -134,6 +138,7 @@ struct Slab {
   double *peer_bot[2] = {nullptr, nullptr};
   unsigned long long *flag_out_top = nullptr, *flag_out_bot = nullptr;
   int peer_top_dev = -1, peer_bot_dev = -1;
+  int shm_pe_top = -1, shm_pe_bot = -1;  // NVSHMEM variant: neighbour PEs
   std::vector<void *> ipc_opened;
   ncclComm_t comm = nullptr;
   double last_ms = 0;
@@ -208,7 +213,12 @@ jacobi_ctx *new_ctx(int64_t nx, int64_t ny, int64_t nz, int stencil, int total) 
 
 int alloc_slab(jacobi_ctx *h, Slab &s) {
   CK(cudaSetDevice(s.device));
-  const size_t bytes = (size_t)slab_elems(h, s) * sizeof(double);
+  size_t bytes = (size_t)slab_elems(h, s) * sizeof(double);
+  if (h->kind == KIND_SHMEM) {  // symmetric heap: every PE allocates the largest slab
+    int64_t st, chunk_max;
+    jbplan::decompose(h->n_out, h->total, 0, &st, &chunk_max);
+    bytes = (size_t)(chunk_max + 2) * h->geom.plane_elems * sizeof(double);
+  }
   if (h->alloc.alloc) {
     s.buf[0] = static_cast<double *>(h->alloc.alloc(bytes, s.device, h->alloc.user));
     s.buf[1] = static_cast<double *>(h->alloc.alloc(bytes, s.device, h->alloc.user));
@@ -427,6 +437,9 @@ int plan_launch(jacobi_ctx *h, const std::vector<int> &idx, LaunchKind lk, bool 
     d.cta_begin = begin;
     d.cta_count = count;
     d.slab_id = s.id;
+    d.use_shm = h->kind == KIND_SHMEM ? 1 : 0;
+    d.shm_pe_top = s.shm_pe_top;
+    d.shm_pe_bot = s.shm_pe_bot;
     begin += count;
     const bool roles = lk == LK_PERSIST || lk == LK_P2P || lk == LK_EDGES;
     const bool top = roles && s.has_top, bot = roles && s.has_bot;
@@ -607,7 +620,7 @@ int setup_norm(jacobi_ctx *h, LaunchPlan &L) {
     }
     CK(cudaMemset(s.partials, 0, n * sizeof(double)));
     std::vector<JbCtrl *> ctrls(h->total, nullptr);
-    if (h->kind == KIND_DIST) {
+    if (h->kind == KIND_DIST || h->kind == KIND_SHMEM) {
       if ((int)h->all_ctrl.size() != h->total) return JACOBI_ESTATE;  // needs jacobi_open_ranks
       ctrls = h->all_ctrl;
     } else {
@@ -633,7 +646,7 @@ int run_cpufree(jacobi_ctx *h, int64_t iters) {
   auto groups = launch_groups(h);
   std::vector<LaunchPlan> plans(groups.size());
   // Resident (on-chip) kernel when every slab fits (auto) or when forced (not with the norm).
-  bool resident = !nocomp && !norm && h->resident != 0;
+  bool resident = !nocomp && !norm && h->resident != 0 && h->kind != KIND_SHMEM;
   if (resident) {
     for (size_t i = 0; i < groups.size() && resident; ++i)
       if (plan_resident(h, groups[i], plans[i]) != JACOBI_OK) resident = false;
@@ -740,6 +753,7 @@ int ensure_nccl(jacobi_ctx *h) {
   if (h->nccl_ready) return JACOBI_OK;
   if (h->kind == KIND_VIRTUAL && h->total > 1) return JACOBI_EINVAL;  // NCCL: one rank per GPU
   if (h->kind == KIND_DIST) return JACOBI_ESTATE;  // needs jacobi_nccl_init via the binding
+  if (h->kind == KIND_SHMEM) return JACOBI_EINVAL;
   if (!g_nccl.load()) return JACOBI_ENCCL;
   std::vector<int> devs;
   for (auto &s : h->slabs) devs.push_back(s.device);
@@ -841,7 +855,7 @@ int run_baseline(jacobi_ctx *h, int64_t iters, BaseKind kind) {
   if (kind == BK_NCCL) {
     int rc = ensure_nccl(h);
     if (rc) return rc;
-  } else if (h->kind == KIND_DIST && h->total > 1) {
+  } else if ((h->kind == KIND_DIST || h->kind == KIND_SHMEM) && h->total > 1) {
     return JACOBI_EINVAL;  // host-synchronised peer baselines need one process: use NCCL
   }
   const int n = (int)h->slabs.size();
@@ -1189,6 +1203,98 @@ int jacobi_open_ranks(jacobi_t h, const void *blobs, int world) {
   return JACOBI_OK;
 }
 
+#ifdef JB_NVSHMEM
+namespace {
+bool g_shm_init = false;
+void *shm_alloc(size_t bytes, int, void *) { return nvshmem_malloc(bytes); }
+void shm_free(void *p, int, void *) { nvshmem_free(p); }
+}  // namespace
+
+int jacobi_nvshmem_uid_bytes(void) { return (int)sizeof(nvshmemx_uniqueid_t); }
+
+int jacobi_nvshmem_uid(void *out) {
+  if (!out) return JACOBI_EINVAL;
+  nvshmemx_uniqueid_t uid = NVSHMEMX_UNIQUEID_INITIALIZER;
+  if (nvshmemx_get_uniqueid(&uid) != 0) return JACOBI_ECUDA;
+  std::memcpy(out, &uid, sizeof(uid));
+  return JACOBI_OK;
+}
+
+// N3: one PE per process, bootstrapped from a unique id (created by rank 0, shared by the caller),
+// slab buffers and control blocks on the NVSHMEM symmetric heap; halos are delivered with
+// nvshmemx_putmem_signal_nbi_warp by the boundary CTAs of the CPU-Free kernel.
+// Collective: every rank creates (and later destroys) its handle in the same order.
+int jacobi_create_nvshmem(int64_t nx, int64_t ny, int64_t nz, int stencil, const void *uid, int world_size,
+                          int rank, int device, jacobi_t *out) {
+  if (!out || !uid || rank < 0 || rank >= world_size || world_size > 32) return JACOBI_EINVAL;
+  *out = nullptr;
+  int rc = validate(nx, ny, nz, stencil, world_size);
+  if (rc) return rc;
+  CK(cudaSetDevice(device));
+  if (!g_shm_init) {
+    if (!getenv("NVSHMEM_SYMMETRIC_SIZE")) {  // room for two field buffers + control block
+      JbGeom g;
+      jbplan::geometry(nx, ny, nz, stencil == 5 ? 2 : 3, 8, 1, JB_SMEM_DEFAULT, 0, &g);
+      int64_t st, chunk_max;
+      jbplan::decompose(stencil == 5 ? ny : nz, world_size, 0, &st, &chunk_max);
+      const int64_t need = 2 * (chunk_max + 2) * g.plane_elems * 8 + (64 << 20);
+      const int64_t sz = std::max<int64_t>(need + need / 4, (int64_t)1 << 30);
+      setenv("NVSHMEM_SYMMETRIC_SIZE", std::to_string(sz).c_str(), 0);
+    }
+    nvshmemx_uniqueid_t id;
+    std::memcpy(&id, uid, sizeof(id));
+    nvshmemx_init_attr_t attr = NVSHMEMX_INIT_ATTR_INITIALIZER;
+    nvshmemx_set_attr_uniqueid_args(rank, world_size, &id, &attr);
+    if (nvshmemx_init_attr(NVSHMEMX_INIT_WITH_UNIQUEID, &attr) != 0) return JACOBI_ECUDA;
+    g_shm_init = true;
+  }
+  if (nvshmem_my_pe() != rank || nvshmem_n_pes() != world_size) return JACOBI_ESTATE;
+  jacobi_ctx *h = new_ctx(nx, ny, nz, stencil, world_size);
+  h->kind = KIND_SHMEM;
+  h->rank = rank;
+  h->alloc.alloc = shm_alloc;
+  h->alloc.free = shm_free;
+  h->alloc.user = nullptr;
+  h->slabs.resize(1);
+  Slab &s = h->slabs[0];
+  s.device = device;
+  s.id = rank;
+  jbplan::decompose(h->n_out, world_size, rank, &s.start, &s.chunk);
+  rc = alloc_slab(h, s);
+  if (rc) { delete h; return rc; }
+  const int64_t pe = h->geom.plane_elems;
+  s.has_top = rank > 0;
+  s.has_bot = rank < world_size - 1;
+  if (s.has_top) {  // symmetric addresses of the neighbour's bottom halo plane and flag slots
+    int64_t st, ct;
+    jbplan::decompose(h->n_out, world_size, rank - 1, &st, &ct);
+    for (int p = 0; p < 2; ++p) s.peer_top[p] = s.buf[p] + (ct + 1) * pe;
+    s.flag_out_top = &s.ctrl->flag_in[1][0];
+    s.shm_pe_top = rank - 1;
+  }
+  if (s.has_bot) {
+    for (int p = 0; p < 2; ++p) s.peer_bot[p] = s.buf[p];
+    s.flag_out_bot = &s.ctrl->flag_in[0][0];
+    s.shm_pe_bot = rank + 1;
+  }
+  h->all_ctrl.assign(world_size, nullptr);  // raw NVLink pointers for the norm all-reduce (N4)
+  for (int g = 0; g < world_size; ++g)
+    h->all_ctrl[g] = static_cast<JbCtrl *>(nvshmem_ptr(s.ctrl, g));
+  for (int g = 0; g < world_size; ++g)
+    if (!h->all_ctrl[g]) h->all_ctrl.clear();
+  h->peers_ready = true;
+  nvshmem_barrier_all();
+  *out = h;
+  return JACOBI_OK;
+}
+
+int jacobi_nvshmem_finalize(void) {
+  if (g_shm_init) nvshmem_finalize();
+  g_shm_init = false;
+  return JACOBI_OK;
+}
+#endif
+
 int jacobi_nccl_unique_id(void *out128) {
   if (!out128) return JACOBI_EINVAL;
   if (!g_nccl.load()) return JACOBI_ENCCL;
@@ -1377,6 +1483,9 @@ int jacobi_destroy(jacobi_t h) {
     if (s.device >= 0) cudaSetDevice(s.device);
     if (s.stream) cudaStreamSynchronize(s.stream);
   }
+#ifdef JB_NVSHMEM
+  if (h->kind == KIND_SHMEM) nvshmem_barrier_all();  // collective: no PE still reads our heap
+#endif
   for (auto &s : h->slabs) free_slab(s, h->alloc);
   if (h->graph_exec) cudaGraphExecDestroy(h->graph_exec);
   delete h;

@@ -28,6 +28,19 @@ def test_library_exports_every_header_symbol():
         assert n in jb._SIGS, n
 
 
+def test_nvshmem_variant_exports_everything():
+    """libjacobi_b200_nvshmem.so (N3) exports the whole ABI plus the NVSHMEM entry points.
+    (nm, not dlopen: it links libcuda, which a GPU-less box does not have.)"""
+    from paper_conf_sc_baydamirlibu24_b200 import build as b
+    if b.nvshmem_home() is None:
+        pytest.skip("no NVSHMEM wheel")
+    out = subprocess.run(["nm", "-D", "--defined-only", jb.NVSHMEM_LIB_PATH], capture_output=True, text=True).stdout
+    syms = {line.split()[-1] for line in out.splitlines() if line.strip()}
+    want = jb.header_functions() + jb.header_functions(nvshmem=True)
+    assert len(jb.header_functions(nvshmem=True)) == 4
+    assert not [n for n in want if n not in syms]
+
+
 def test_library_is_sm100a_only():
     out = subprocess.run(["/usr/local/cuda/bin/cuobjdump", "--list-elf", jb.LIB_PATH],
                          capture_output=True, text=True).stdout
