@@ -114,6 +114,11 @@ class ClockSampler:
                 "samples": len(sm)}
 
 
+def torch_device_count() -> int:
+    import torch
+    return torch.cuda.device_count()
+
+
 def dist_env():
     world = int(os.environ.get("WORLD_SIZE", "1"))
     rank = int(os.environ.get("RANK", "0"))
@@ -194,6 +199,8 @@ def main():
     args.warmup = max(args.warmup, 3) if args.impl == "ours" else args.warmup
 
     world, rank, local = dist_env()
+    ndev = torch_device_count()
+    local = local % max(ndev, 1)  # (more ranks than GPUs only in functional tests: time-sliced)
     cfg = dict(CONFIGS[args.config])
     if args.iters:
         cfg["iters"] = args.iters
@@ -218,7 +225,12 @@ def main():
         import torch.distributed as dist
         dist.init_process_group("gloo")
         j = jb.Jacobi(shape, dist=(rank, world), device=local)
-        jb.exchange_peers(j, nccl=True)
+        jb.exchange_peers(j, nccl=False)
+        try:  # NCCL comm of the CPU-controlled baseline (needs one GPU per rank)
+            uid = jb.broadcast_blob(jb.jacobi_nccl_unique_id() if rank == 0 else None)
+            jb.jacobi_nccl_init(j.h, uid)
+        except jb.JacobiError as e:
+            print(f"[bench] NCCL baseline unavailable: {e}", file=sys.stderr)
     else:
         jb.use_torch_allocator()
         dist = None
@@ -285,7 +297,8 @@ def main():
         "config": {"workload": cfg["workload"], "shape_zyx": list(shape), "iters": iters,
                    "parallelism": f"slab{world}" + (f" (virtual {args.virtual} slabs)" if args.virtual else ""),
                    "l2": ("inputs larger than L2" if 8 * cells > L2_BYTES else "L2-resident (latency config)"),
-                   "tile": {k: desc[k] for k in ("tile_x", "tile_y", "stages", "ctas", "n_top", "n_bot", "k_planes")}},
+                   "tile": {k: desc[k] for k in ("tile_x", "tile_y", "stages", "ctas", "n_top", "n_bot", "k_planes")},
+                   "kernel": "resident" if jb.jacobi_get_param(j.h, "last_resident") else "streaming"},
         "gpu_launches": args.steps * world,
         "wall_ms_per_step": 1e3 * t_wall / args.steps,
         "ms_per_iter": dev_ms / args.steps / iters,
@@ -316,13 +329,16 @@ def main():
         if world > 1:
             halo = {}
             for name, mode in (("cpufree", jb.MODE_CPUFREE), ("baseline_nccl", jb.MODE_BASELINE_NCCL)):
-                j.set_mode(mode, jb.FLAG_NO_COMPUTE)
-                j.run(100)
-                j.run(200)
-                t1 = max_over_ranks(j.last_time_ms())
-                j.run(400)
-                t2 = max_over_ranks(j.last_time_ms())
-                halo[name] = 1e3 * (t2 - t1) / 200
+                try:
+                    j.set_mode(mode, jb.FLAG_NO_COMPUTE)
+                    j.run(100)
+                    j.run(200)
+                    t1 = max_over_ranks(j.last_time_ms())
+                    j.run(400)
+                    t2 = max_over_ranks(j.last_time_ms())
+                    halo[name] = 1e3 * (t2 - t1) / 200
+                except jb.JacobiError as e:
+                    halo[name] = {"error": str(e)}
             j.set_mode(jb.MODE_CPUFREE)
             line["halo_us"] = halo
         else:
