@@ -65,6 +65,9 @@ extern "C" {
                                            peers' halos (GPU-initiated data, host sync) */
 #define JACOBI_MODE_BASELINE_GRAPH   5  /* the MEMCPY loop captured once into a CUDA graph with
                                            cross-GPU event edges, one host launch per run */
+#define JACOBI_MODE_BASELINE_NVSHMEM 6  /* NVSHMEM variant only: per iteration a discrete kernel whose
+                                           boundary blocks put halos with NVSHMEM, then a dedicated
+                                           neighbour-sync kernel; no host barrier */
 
 /* ---- flags for jacobi_set_mode --------------------------------------------------------- */
 #define JACOBI_FLAG_NO_COMPUTE   1  /* measurement only: skip the stencil

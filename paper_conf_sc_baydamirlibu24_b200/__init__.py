@@ -36,6 +36,7 @@ MODE_BASELINE_NCCL = 2
 MODE_BASELINE_OVERLAP = 3
 MODE_BASELINE_P2P = 4
 MODE_BASELINE_GRAPH = 5
+MODE_BASELINE_NVSHMEM = 6
 FLAG_NO_COMPUTE = 1
 FLAG_DROP_SIGNAL = 2
 

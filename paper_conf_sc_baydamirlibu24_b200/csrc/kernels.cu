@@ -805,11 +805,11 @@ __global__ void __launch_bounds__(JB_THREADS, 1) jb_sweep(const __grid_constant_
         if (d.kind == RUN_END) break;
         if (d.kind == RUN_SIGNAL) {
           // P:364-365 / P:394: signal the neighbour that the halo of iteration tg+1 is in place.
-          if (PERSIST) named_bar_consumers();
+          if (PERSIST || SL.use_shm) named_bar_consumers();
           // bar.sync makes every consumer thread's peer stores precede thread 0 (CTA scope);
           // its sys-scope release store into this CTA's slot publishes them to the neighbour.
 #ifdef JB_NVSHMEM
-          if (PERSIST && SL.use_shm) {
+          if (SL.use_shm) {  // CPU-Free (persistent) and the "Baseline NVSHMEM" discrete kernel
             if (warp == 0) shm_put_boundary<DIM, NOCOMP>(g, SL, role, ridx, rcount, cur, nxt, tg, drop_signal);
             remote = nullptr;
             continue;
@@ -1142,6 +1142,15 @@ __global__ void jb_init_u12(double *b0, double *b1, int64_t nplanes, JbGeom g, i
   }
 }
 
+// "Baseline NVSHMEM": the dedicated kernel, launched by the host every iteration after
+// the compute kernel, that waits until both neighbours delivered this iteration's halos.
+__global__ void jb_neighbour_wait(const __grid_constant__ JbParams P, unsigned long long target) {
+  const JbSlab &S = P.s[0];
+  const int lane = threadIdx.x & 31;
+  if (S.k_in_top > 0) wait_slots(S.flag_in_top, S.k_in_top, target, P, lane);
+  if (S.k_in_bot > 0) wait_slots(S.flag_in_bot, S.k_in_bot, target, P, lane);
+}
+
 __global__ void jb_flag_max(unsigned long long *flags, int n, unsigned long long v) {
   for (int i = threadIdx.x; i < n; i += blockDim.x) atomicMax(flags + i, v);
 }
@@ -1216,6 +1225,11 @@ cudaError_t launch_resident(const JbParams &p, int cpp, int grid, size_t smem, c
 cudaError_t launch_init(double *b0, double *b1, int64_t nplanes, const JbGeom &g, int64_t z_first,
                         unsigned long long seed, cudaStream_t st) {
   jb_init_u12<<<1184, 256, 0, st>>>(b0, b1, nplanes, g, z_first, seed);
+  return cudaGetLastError();
+}
+
+cudaError_t launch_neighbour_wait(const JbParams &p, unsigned long long target, cudaStream_t st) {
+  jb_neighbour_wait<<<1, 32, 0, st>>>(p, target);
   return cudaGetLastError();
 }
 

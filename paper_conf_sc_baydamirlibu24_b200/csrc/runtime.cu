@@ -32,6 +32,7 @@ cudaError_t launch_init(double *b0, double *b1, int64_t nplanes, const JbGeom &g
 cudaError_t launch_flag_max(unsigned long long *flags, int n, unsigned long long v, cudaStream_t st);
 cudaError_t prepare_resident(int dim, int cpp, size_t smem, int *blocks_per_sm);
 cudaError_t launch_resident(const JbParams &p, int cpp, int grid, size_t smem, cudaStream_t st);
+cudaError_t launch_neighbour_wait(const JbParams &p, unsigned long long target, cudaStream_t st);
 }  // namespace jbk
 
 namespace {
@@ -467,7 +468,7 @@ int plan_launch(jacobi_ctx *h, const std::vector<int> &idx, LaunchKind lk, bool 
     split_roles(h, count, inner, top, bot, g.units, &nt, &nb, &ni);
     d.n_top = nt;
     d.n_bot = nb;
-    if (persist) {
+    if (persist || lk == LK_P2P) {
       // The facing boundary-CTA counts of the neighbours (how many flag slots to wait for) are
       // recomputed here with the neighbours' own chunk and CTA count: the split is deterministic.
       int kt = 0, kb = 0;
@@ -776,7 +777,7 @@ int ensure_nccl(jacobi_ctx *h) {
 //   GRAPH   : the COPY loop captured once into a CUDA graph (all iterations, cross-GPU event
 //             dependencies instead of host barriers) and replayed with one launch — the strongest
 //             CPU-controlled variant (not in the paper).
-enum BaseKind { BK_COPY, BK_NCCL, BK_OVERLAP, BK_P2P, BK_GRAPH };
+enum BaseKind { BK_COPY, BK_NCCL, BK_OVERLAP, BK_P2P, BK_GRAPH, BK_SHMEM };
 
 int time_begin(jacobi_ctx *h) {
   for (auto &s : h->slabs) {
@@ -855,6 +856,8 @@ int run_baseline(jacobi_ctx *h, int64_t iters, BaseKind kind) {
   if (kind == BK_NCCL) {
     int rc = ensure_nccl(h);
     if (rc) return rc;
+  } else if (kind == BK_SHMEM) {
+    if (h->kind != KIND_SHMEM) return JACOBI_EINVAL;  // needs the NVSHMEM variant's handles
   } else if ((h->kind == KIND_DIST || h->kind == KIND_SHMEM) && h->total > 1) {
     return JACOBI_EINVAL;  // host-synchronised peer baselines need one process: use NCCL
   }
@@ -863,7 +866,7 @@ int run_baseline(jacobi_ctx *h, int64_t iters, BaseKind kind) {
   for (int i = 0; i < n; ++i) {
     Slab &s = h->slabs[i];
     int rc;
-    if (kind == BK_P2P) {
+    if (kind == BK_P2P || kind == BK_SHMEM) {
       rc = plan_launch(h, {i}, LK_P2P, nocomp, plans[i]);
     } else if (kind == BK_OVERLAP && (s.has_top || s.has_bot)) {
       int sms = 0;
@@ -881,7 +884,8 @@ int run_baseline(jacobi_ctx *h, int64_t iters, BaseKind kind) {
   if (kind == BK_GRAPH) return run_graph(h, iters, nocomp, plans);
   int rc = time_begin(h);
   if (rc) return rc;
-  const bool launch_kernels = !nocomp || kind == BK_P2P;  // P2P no-compute still moves halos in-kernel
+  // P2P / NVSHMEM no-compute still move halos in-kernel
+  const bool launch_kernels = !nocomp || kind == BK_P2P || kind == BK_SHMEM;
   for (int64_t it = 0; it < iters; ++it) {
     const int64_t tg = h->t + it;
     const int nxt = (int)((tg + 1) & 1);
@@ -914,6 +918,15 @@ int run_baseline(jacobi_ctx *h, int64_t iters, BaseKind kind) {
     } else if (kind == BK_NCCL) {
       rc = nccl_edges(h, nxt);
       if (rc) return rc;
+    } else if (kind == BK_SHMEM) {
+      // the second per-iteration kernel waits for the neighbours' signals; no host
+      // barrier — the next iteration's kernel is ordered behind it on the stream.
+      for (int i = 0; i < n; ++i) {
+        Slab &s = h->slabs[i];
+        CK(cudaSetDevice(s.device));
+        CK(jbk::launch_neighbour_wait(plans[i].P, (unsigned long long)(tg + 1), s.stream));
+      }
+      continue;
     }
     for (auto &s : h->slabs) {  // ⑤ sync streams, host barrier: wait for every GPU
       CK(cudaSetDevice(s.device));
@@ -1329,12 +1342,13 @@ int jacobi_run(jacobi_t h, int64_t iters) {
   if (h->mode == JACOBI_MODE_BASELINE_OVERLAP) return run_baseline(h, iters, BK_OVERLAP);
   if (h->mode == JACOBI_MODE_BASELINE_P2P) return run_baseline(h, iters, BK_P2P);
   if (h->mode == JACOBI_MODE_BASELINE_GRAPH) return run_baseline(h, iters, BK_GRAPH);
+  if (h->mode == JACOBI_MODE_BASELINE_NVSHMEM) return run_baseline(h, iters, BK_SHMEM);
   return JACOBI_EINVAL;
 }
 
 int jacobi_set_mode(jacobi_t h, int mode, int flags) {
   if (!h) return JACOBI_EINVAL;
-  if (mode < JACOBI_MODE_CPUFREE || mode > JACOBI_MODE_BASELINE_GRAPH) return JACOBI_EINVAL;
+  if (mode < JACOBI_MODE_CPUFREE || mode > JACOBI_MODE_BASELINE_NVSHMEM) return JACOBI_EINVAL;
   if (flags & ~(JACOBI_FLAG_NO_COMPUTE | JACOBI_FLAG_DROP_SIGNAL)) return JACOBI_EINVAL;
   h->mode = mode;
   h->plan_gen++;

@@ -32,9 +32,12 @@ def _worker(rank, world, port, shape, iters, tol, q):
         outs = []
         j = jb.create_nvshmem(shape)
         j.set_param("timeout_ms", 60000)
-        for mode_tol in (None, tol):
+        for mode_tol in (None, tol, "baseline"):
             j.scatter(f)
-            if mode_tol is not None:
+            if mode_tol == "baseline":  # P:531 "Baseline NVSHMEM": discrete kernels + sync kernel
+                j.set_tolerance(0.0, 0)
+                j.set_mode(jb.MODE_BASELINE_NVSHMEM)
+            elif mode_tol is not None:
                 j.set_tolerance(mode_tol, 5)
             t0 = j.iterations
             dist.barrier()
@@ -77,7 +80,7 @@ def test_nvshmem_two_pes(shape):
         res[rank] = outs
     for p in procs:
         p.join(timeout=60)
-    for k, (exp, n_exp) in enumerate([(exp_plain, iters), (exp_conv, done)]):
+    for k, (exp, n_exp) in enumerate([(exp_plain, iters), (exp_conv, done), (exp_plain, iters)]):
         a, na = res[0][k]
         bb, nb = res[1][k]
         assert na == nb == n_exp
