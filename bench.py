@@ -307,6 +307,29 @@ def main():
     }
 
     if not args.no_extras:
+        # ---- this box's own copy bandwidth (same method as MEASURED_PEAKS.json: torch copy_ of
+        #      1 Gi bf16 elements, read + write bytes, best of 10), for context beside `roofline`
+        try:
+            a = torch.empty(1 << 30, dtype=torch.bfloat16, device=f"cuda:{local}")
+            b = torch.empty_like(a)
+            e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            best = None
+            for _ in range(10):
+                e0.record()
+                b.copy_(a)
+                e1.record()
+                e1.synchronize()
+                ms = e0.elapsed_time(e1)
+                best = ms if best is None else min(best, ms)
+            box_copy = 2 * a.numel() * a.element_size() / (best / 1e3) / 1e9
+            line["roofline"]["box_copy_gbs"] = box_copy
+            line["roofline"]["frac_of_box_copy"] = line["roofline"]["achieved"] / box_copy
+            del a, b
+            torch.cuda.empty_cache()
+        except Exception as e:  # never fail the bench line for a context number
+            line["roofline"]["box_copy_gbs"] = None
+            print(f"[bench] box copy measurement failed: {e}", file=sys.stderr)
+
         # ---- CPU-controlled baselines (per-iteration launch + copy/NCCL + host sync), short run
         base = {}
         b_iters = min(iters, 200)
