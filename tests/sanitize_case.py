@@ -1,0 +1,25 @@
+"""Tiny runs of every kernel family for compute-sanitizer (tests/test_gpu_sanitizer.py)."""
+import os
+import sys
+
+sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+import numpy as np  # noqa: E402
+
+import oracle  # noqa: E402
+import paper_conf_sc_baydamirlibu24_b200 as jb  # noqa: E402
+from jacobi_inputs import u12  # noqa: E402
+
+ok = True
+for shape, P in [((20, 70), 2), ((8, 9, 33), 2), ((30, 40), 1)]:
+    f = u12(shape, 3)
+    for params, mode in [({"resident": 0}, jb.MODE_CPUFREE), ({"resident": 1}, jb.MODE_CPUFREE),
+                         ({}, jb.MODE_BASELINE_MEMCPY), ({}, jb.MODE_BASELINE_P2P),
+                         ({"resident": 0, "norm_every": 2}, jb.MODE_CPUFREE)]:
+        with jb.Jacobi(shape, virtual=P) if P > 1 else jb.Jacobi(shape) as j:
+            for k, v in params.items():
+                j.set_param(k, v)
+            j.set_mode(mode)
+            j.scatter(f)
+            j.run(3)
+            ok &= bool(np.array_equal(j.gather(), oracle.jacobi(f, 3)))
+print("SANITIZE_CASE_OK" if ok else "SANITIZE_CASE_MISMATCH")
