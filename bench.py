@@ -283,10 +283,13 @@ def main():
     alg_bytes = 16 * local_cells * iters  # read once + write once per cell-update
     achieved = alg_bytes / (launch_ms / 1e3) / 1e9
     traffic, _ = ncu_traffic(args.config, iters)
+    dimk = 2 if shape[0] == 1 else 3
+    kname = (f"jb_resident<{dimk},*> (persistent CPU-Free kernel, on-chip resident)"
+             if jb.jacobi_get_param(j.h, "last_resident") else
+             f"jb_sweep<{dimk},false,true,false> (persistent CPU-Free kernel, streaming)")
     roofline = {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
                 "frac": achieved / peak, "traffic": traffic, "peak_kind": peak_kind,
-                "kernel": f"jb_sweep<{2 if shape[0] == 1 else 3},false,true> (persistent CPU-Free kernel)",
-                "alg_bytes_per_launch": alg_bytes}
+                "kernel": kname, "alg_bytes_per_launch": alg_bytes}
 
     line = {
         "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
