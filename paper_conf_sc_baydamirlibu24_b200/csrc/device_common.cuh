@@ -1,0 +1,209 @@
+// device_common.cuh — PTX helpers, waits, ring positions and small device utilities shared by
+// the kernels of libjacobi_b200 (sweep.cu, resident.cu, util.cu).  Internal linkage per TU.
+#pragma once
+#include <cuda_runtime.h>
+#include <stdint.h>
+
+#include "../../include/jacobi.h"
+#include "jacobi_internal.h"
+#ifdef JB_NVSHMEM
+#include <nvshmem.h>
+#include <nvshmemx.h>
+#endif
+
+namespace {
+
+constexpr double kC6 = 0x1.5555555555555p-3;  // fl(1/6), reading R3
+constexpr unsigned long long kGolden = 0x9E3779B97F4A7C15ull;
+
+enum Role { ROLE_INT = 0, ROLE_TOP = 1, ROLE_BOT = 2 };
+
+// Same even split as jbplan::even_split (host): part i of n items over k parts.
+__device__ __forceinline__ void jbplan_even_split(int64_t n, int k, int i, int64_t *start, int64_t *len) {
+  const int64_t q = n / k, r = n % k;
+  *len = q + (i < r ? 1 : 0);
+  *start = (int64_t)i * q + min((int64_t)i, r);
+}
+
+// ---------------------------------------------------------------- PTX helpers
+__device__ __forceinline__ uint32_t sptr(const void *p) {
+  return static_cast<uint32_t>(__cvta_generic_to_shared(p));
+}
+__device__ __forceinline__ void mbar_init(uint64_t *b, uint32_t count) {
+  asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(sptr(b)), "r"(count) : "memory");
+}
+__device__ __forceinline__ void mbar_expect_tx(uint64_t *b, uint32_t bytes) {
+  asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(sptr(b)), "r"(bytes)
+               : "memory");
+}
+__device__ __forceinline__ void mbar_arrive(uint64_t *b) {
+  asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(sptr(b)) : "memory");
+}
+__device__ __forceinline__ bool mbar_try_wait(uint64_t *b, uint32_t parity) {
+  uint32_t ok;
+  asm volatile(
+      "{\n .reg .pred p;\n mbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2;\n"
+      " selp.u32 %0, 1, 0, p;\n}\n"
+      : "=r"(ok)
+      : "r"(sptr(b)), "r"(parity)
+      : "memory");
+  return ok != 0;
+}
+__device__ __forceinline__ void mbar_wait(uint64_t *b, uint32_t parity) {
+  while (!mbar_try_wait(b, parity)) {
+  }
+}
+// 1D bulk copy global -> shared (TMA engine), completion counted in bytes on an mbarrier.
+__device__ __forceinline__ void bulk_g2s(void *dst, const void *src, uint32_t bytes, uint64_t *bar) {
+  asm volatile(
+      "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(
+          sptr(dst)),
+      "l"(src), "r"(bytes), "r"(sptr(bar))
+      : "memory");
+}
+__device__ __forceinline__ void fence_proxy_async_global() {
+  asm volatile("fence.proxy.async.global;" ::: "memory");
+}
+__device__ __forceinline__ void fence_mbar_init() {
+  asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+}
+__device__ __forceinline__ unsigned long long ld_acquire_sys(const unsigned long long *p) {
+  unsigned long long v;
+  asm volatile("ld.acquire.sys.global.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
+  return v;
+}
+__device__ __forceinline__ unsigned long long ld_acquire_gpu(const unsigned long long *p) {
+  unsigned long long v;
+  asm volatile("ld.acquire.gpu.global.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
+  return v;
+}
+__device__ __forceinline__ void st_release_gpu(unsigned long long *p, unsigned long long v) {
+  asm volatile("st.release.gpu.global.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
+}
+__device__ __forceinline__ void st_release_sys(unsigned long long *p, unsigned long long v) {
+  asm volatile("st.release.sys.global.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
+}
+__device__ __forceinline__ void red_release_gpu_add(unsigned long long *p, unsigned long long v) {
+  asm volatile("red.release.gpu.global.add.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
+}
+__device__ __forceinline__ unsigned long long globaltimer() {
+  unsigned long long t;
+  asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+  return t;
+}
+__device__ __forceinline__ void named_bar_consumers() {
+  asm volatile("bar.sync 1, %0;" ::"r"(JB_NC) : "memory");
+}
+
+// Spin until *p >= target (acquire at sys or gpu scope).  Watchdog: after timeout_ns set
+// status = ETIMEOUT and the abort flag; also gives up once another CTA raised abort.
+template <bool SYS>
+__device__ bool wait_geq(const unsigned long long *p, unsigned long long target, const JbParams &P) {
+  auto ld = [&]() { return SYS ? ld_acquire_sys(p) : ld_acquire_gpu(p); };
+  if (ld() >= target) return true;
+  const unsigned long long t_start = globaltimer();
+  uint32_t n = 0;
+  volatile int *abort_flag = P.status + 1;
+  while (true) {
+    if (ld() >= target) return true;
+    if ((++n & 127u) == 0) {
+      if (*abort_flag) return false;
+      if (globaltimer() - t_start > P.timeout_ns) {
+        atomicCAS(P.status, 0, JACOBI_ETIMEOUT);
+        atomicExch(P.status + 1, 1);
+        return false;
+      }
+    }
+  }
+}
+
+// Warp-cooperative wait until flag slots 0..k-1 all reach `target` (lane i polls slot i).
+__device__ bool wait_slots(const unsigned long long *slots, int k, unsigned long long target, const JbParams &P,
+                           int lane) {
+  const unsigned long long t_start = globaltimer();
+  uint32_t n = 0;
+  volatile int *abort_flag = P.status + 1;
+  while (true) {
+    const bool ok = lane >= k || ld_acquire_sys(slots + lane) >= target;
+    if (__all_sync(0xffffffffu, ok)) return true;
+    if ((++n & 127u) == 0) {
+      int stop = 0;
+      if (lane == 0) {
+        if (*abort_flag) {
+          stop = 1;
+        } else if (globaltimer() - t_start > P.timeout_ns) {
+          atomicCAS(P.status, 0, JACOBI_ETIMEOUT);
+          atomicExch(P.status + 1, 1);
+          stop = 1;
+        }
+      }
+      if (__shfl_sync(0xffffffffu, stop, 0)) return false;
+    }
+  }
+}
+
+// Wait until flags[idx[i]] >= target for i < n (n <= 32; lane i polls entry i), gpu scope.
+__device__ bool wait_slots_idx(const unsigned long long *flags, const int *idx, int n, unsigned long long target,
+                               const JbParams &P, int lane) {
+  const unsigned long long *mine = nullptr;
+#pragma unroll
+  for (int i = 0; i < 4; ++i)
+    if (i == lane && i < n) mine = flags + idx[i];
+  const unsigned long long t_start = globaltimer();
+  uint32_t cnt = 0;
+  volatile int *abort_flag = P.status + 1;
+  while (true) {
+    const bool ok = mine == nullptr || ld_acquire_gpu(mine) >= target;
+    if (__all_sync(0xffffffffu, ok)) return true;
+    if ((++cnt & 127u) == 0) {
+      int stop = 0;
+      if (lane == 0) {
+        if (*abort_flag) {
+          stop = 1;
+        } else if (globaltimer() - t_start > P.timeout_ns) {
+          atomicCAS(P.status, 0, JACOBI_ETIMEOUT);
+          atomicExch(P.status + 1, 1);
+          stop = 1;
+        }
+      }
+      if (__shfl_sync(0xffffffffu, stop, 0)) return false;
+    }
+  }
+}
+
+// Position in the shared-memory ring: slot and the parity of the current use of that slot.
+struct RingPos {
+  uint32_t slot, phase;
+  __device__ __forceinline__ void advance(uint32_t S) {
+    if (++slot == S) {
+      slot = 0;
+      phase ^= 1u;
+    }
+  }
+};
+
+struct Ring {
+  uint64_t *full, *empty;
+  double *stages;
+  uint32_t S;
+  int stage_doubles;
+  __device__ __forceinline__ double *stage(const RingPos &p) const {
+    return stages + (size_t)p.slot * stage_doubles;
+  }
+  __device__ __forceinline__ void wait_full(const RingPos &p) const { mbar_wait(&full[p.slot], p.phase); }
+  // Consumer warp releases a stage: all lanes are done reading it (syncwarp), one lane arrives.
+  __device__ __forceinline__ void release(const RingPos &p, int lane) const {
+    __syncwarp();
+    if (lane == 0) mbar_arrive(&empty[p.slot]);
+  }
+};
+
+// ---------------------------------------------------------------- small load/store helpers
+__device__ __forceinline__ double2 lds2(const double *p) { return *reinterpret_cast<const double2 *>(p); }
+
+__device__ __forceinline__ void store_pair(double *p, double o0, double o1, bool pair) {
+  if (pair) *reinterpret_cast<double2 *>(p) = make_double2(o0, o1);
+  else *p = o0;
+}
+
+}  // namespace

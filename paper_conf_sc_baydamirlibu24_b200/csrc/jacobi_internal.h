@@ -1,5 +1,5 @@
 // jacobi_internal.h — structures shared by the host runtime (runtime.cu, plan.cpp) and the
-// device kernels (kernels.cu).  Product code only; nothing here is shared with oracle/.
+// device kernels (sweep.cu, resident.cu, util.cu).  Product code only; nothing here is shared with oracle/.
 #pragma once
 #include <stdint.h>
 

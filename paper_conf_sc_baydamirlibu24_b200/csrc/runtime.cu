@@ -2,7 +2,8 @@
 //
 // Owns devices, slabs (HBM buffers + control blocks), peer mappings (UVA peer access in one
 // process, CUDA IPC across processes), launches, timing, and the CPU-controlled baselines.
-// All device work is done by the kernels in kernels.cu; the host only orchestrates.
+// All device work is done by the kernels in sweep.cu / resident.cu / util.cu; the host only
+// orchestrates.
 #include <cuda_runtime.h>
 #include <dlfcn.h>
 #include <nccl.h>

@@ -1,4 +1,4 @@
-// kernels.cu — sm_100a device code of the CPU-Free Jacobi library.
+// sweep.cu — the streaming CPU-Free kernel and the discrete baseline kernels (sm_100a).
 //
 // jb_sweep<DIM, NOCOMP, PERSIST> is the whole hot path:
 //   PERSIST = true : the CPU-Free persistent kernel of PAPER.md Listing 4.1.  The time
@@ -18,175 +18,9 @@
 // completing on mbarriers, and 8 consumer warps march the tile along the outer axis (2.5D), so
 // every cell is read from HBM once and written once per iteration (16 B/cell).  Arithmetic is
 // fp64 in the oracle's order, compiled with -fmad=false (no contraction).
-#include <cuda_runtime.h>
-#include <stdint.h>
-
-#include "../../include/jacobi.h"
-#include "jacobi_internal.h"
-#ifdef JB_NVSHMEM
-#include <nvshmem.h>
-#include <nvshmemx.h>
-#endif
+#include "device_common.cuh"
 
 namespace {
-
-constexpr double kC6 = 0x1.5555555555555p-3;  // fl(1/6), reading R3
-constexpr unsigned long long kGolden = 0x9E3779B97F4A7C15ull;
-
-enum Role { ROLE_INT = 0, ROLE_TOP = 1, ROLE_BOT = 2 };
-
-// Same even split as jbplan::even_split (host): part i of n items over k parts.
-__device__ __forceinline__ void jbplan_even_split(int64_t n, int k, int i, int64_t *start, int64_t *len) {
-  const int64_t q = n / k, r = n % k;
-  *len = q + (i < r ? 1 : 0);
-  *start = (int64_t)i * q + min((int64_t)i, r);
-}
-
-// ---------------------------------------------------------------- PTX helpers
-__device__ __forceinline__ uint32_t sptr(const void *p) {
-  return static_cast<uint32_t>(__cvta_generic_to_shared(p));
-}
-__device__ __forceinline__ void mbar_init(uint64_t *b, uint32_t count) {
-  asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(sptr(b)), "r"(count) : "memory");
-}
-__device__ __forceinline__ void mbar_expect_tx(uint64_t *b, uint32_t bytes) {
-  asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(sptr(b)), "r"(bytes)
-               : "memory");
-}
-__device__ __forceinline__ void mbar_arrive(uint64_t *b) {
-  asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(sptr(b)) : "memory");
-}
-__device__ __forceinline__ bool mbar_try_wait(uint64_t *b, uint32_t parity) {
-  uint32_t ok;
-  asm volatile(
-      "{\n .reg .pred p;\n mbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2;\n"
-      " selp.u32 %0, 1, 0, p;\n}\n"
-      : "=r"(ok)
-      : "r"(sptr(b)), "r"(parity)
-      : "memory");
-  return ok != 0;
-}
-__device__ __forceinline__ void mbar_wait(uint64_t *b, uint32_t parity) {
-  while (!mbar_try_wait(b, parity)) {
-  }
-}
-// 1D bulk copy global -> shared (TMA engine), completion counted in bytes on an mbarrier.
-__device__ __forceinline__ void bulk_g2s(void *dst, const void *src, uint32_t bytes, uint64_t *bar) {
-  asm volatile(
-      "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(
-          sptr(dst)),
-      "l"(src), "r"(bytes), "r"(sptr(bar))
-      : "memory");
-}
-__device__ __forceinline__ void fence_proxy_async_global() {
-  asm volatile("fence.proxy.async.global;" ::: "memory");
-}
-__device__ __forceinline__ void fence_mbar_init() {
-  asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
-}
-__device__ __forceinline__ unsigned long long ld_acquire_sys(const unsigned long long *p) {
-  unsigned long long v;
-  asm volatile("ld.acquire.sys.global.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
-  return v;
-}
-__device__ __forceinline__ unsigned long long ld_acquire_gpu(const unsigned long long *p) {
-  unsigned long long v;
-  asm volatile("ld.acquire.gpu.global.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
-  return v;
-}
-__device__ __forceinline__ void st_release_gpu(unsigned long long *p, unsigned long long v) {
-  asm volatile("st.release.gpu.global.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
-}
-__device__ __forceinline__ void st_release_sys(unsigned long long *p, unsigned long long v) {
-  asm volatile("st.release.sys.global.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
-}
-__device__ __forceinline__ void red_release_gpu_add(unsigned long long *p, unsigned long long v) {
-  asm volatile("red.release.gpu.global.add.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
-}
-__device__ __forceinline__ unsigned long long globaltimer() {
-  unsigned long long t;
-  asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
-  return t;
-}
-__device__ __forceinline__ void named_bar_consumers() {
-  asm volatile("bar.sync 1, %0;" ::"r"(JB_NC) : "memory");
-}
-
-// Spin until *p >= target (acquire at sys or gpu scope).  Watchdog: after timeout_ns set
-// status = ETIMEOUT and the abort flag; also gives up once another CTA raised abort.
-template <bool SYS>
-__device__ bool wait_geq(const unsigned long long *p, unsigned long long target, const JbParams &P) {
-  auto ld = [&]() { return SYS ? ld_acquire_sys(p) : ld_acquire_gpu(p); };
-  if (ld() >= target) return true;
-  const unsigned long long t_start = globaltimer();
-  uint32_t n = 0;
-  volatile int *abort_flag = P.status + 1;
-  while (true) {
-    if (ld() >= target) return true;
-    if ((++n & 127u) == 0) {
-      if (*abort_flag) return false;
-      if (globaltimer() - t_start > P.timeout_ns) {
-        atomicCAS(P.status, 0, JACOBI_ETIMEOUT);
-        atomicExch(P.status + 1, 1);
-        return false;
-      }
-    }
-  }
-}
-
-// Warp-cooperative wait until flag slots 0..k-1 all reach `target` (lane i polls slot i).
-__device__ bool wait_slots(const unsigned long long *slots, int k, unsigned long long target, const JbParams &P,
-                           int lane) {
-  const unsigned long long t_start = globaltimer();
-  uint32_t n = 0;
-  volatile int *abort_flag = P.status + 1;
-  while (true) {
-    const bool ok = lane >= k || ld_acquire_sys(slots + lane) >= target;
-    if (__all_sync(0xffffffffu, ok)) return true;
-    if ((++n & 127u) == 0) {
-      int stop = 0;
-      if (lane == 0) {
-        if (*abort_flag) {
-          stop = 1;
-        } else if (globaltimer() - t_start > P.timeout_ns) {
-          atomicCAS(P.status, 0, JACOBI_ETIMEOUT);
-          atomicExch(P.status + 1, 1);
-          stop = 1;
-        }
-      }
-      if (__shfl_sync(0xffffffffu, stop, 0)) return false;
-    }
-  }
-}
-
-// Wait until flags[idx[i]] >= target for i < n (n <= 32; lane i polls entry i), gpu scope.
-__device__ bool wait_slots_idx(const unsigned long long *flags, const int *idx, int n, unsigned long long target,
-                               const JbParams &P, int lane) {
-  const unsigned long long *mine = nullptr;
-#pragma unroll
-  for (int i = 0; i < 4; ++i)
-    if (i == lane && i < n) mine = flags + idx[i];
-  const unsigned long long t_start = globaltimer();
-  uint32_t cnt = 0;
-  volatile int *abort_flag = P.status + 1;
-  while (true) {
-    const bool ok = mine == nullptr || ld_acquire_gpu(mine) >= target;
-    if (__all_sync(0xffffffffu, ok)) return true;
-    if ((++cnt & 127u) == 0) {
-      int stop = 0;
-      if (lane == 0) {
-        if (*abort_flag) {
-          stop = 1;
-        } else if (globaltimer() - t_start > P.timeout_ns) {
-          atomicCAS(P.status, 0, JACOBI_ETIMEOUT);
-          atomicExch(P.status + 1, 1);
-          stop = 1;
-        }
-      }
-      if (__shfl_sync(0xffffffffu, stop, 0)) return false;
-    }
-  }
-}
 
 // ---------------------------------------------------------------- work schedule
 struct Run {
@@ -270,33 +104,6 @@ __device__ Sched make_sched(const JbGeom &g, const JbSlab &S, int role, int ridx
   return s;
 }
 
-// Position in the shared-memory ring: slot and the parity of the current use of that slot.
-struct RingPos {
-  uint32_t slot, phase;
-  __device__ __forceinline__ void advance(uint32_t S) {
-    if (++slot == S) {
-      slot = 0;
-      phase ^= 1u;
-    }
-  }
-};
-
-struct Ring {
-  uint64_t *full, *empty;
-  double *stages;
-  uint32_t S;
-  int stage_doubles;
-  __device__ __forceinline__ double *stage(const RingPos &p) const {
-    return stages + (size_t)p.slot * stage_doubles;
-  }
-  __device__ __forceinline__ void wait_full(const RingPos &p) const { mbar_wait(&full[p.slot], p.phase); }
-  // Consumer warp releases a stage: all lanes are done reading it (syncwarp), one lane arrives.
-  __device__ __forceinline__ void release(const RingPos &p, int lane) const {
-    __syncwarp();
-    if (lane == 0) mbar_arrive(&empty[p.slot]);
-  }
-};
-
 // ---------------------------------------------------------------- producer
 // Where one tile's stage comes from: the rows of tile `unit` (1 in 2D; ty + 2 in 3D incl. the y
 // halo rows), each row the x window [x0-2, x0+tx+2) of 16-byte aligned doubles, one
@@ -346,12 +153,6 @@ __device__ __forceinline__ void produce_planes(const JbGeom &g, const double *cu
 }
 
 // ---------------------------------------------------------------- consumers
-__device__ __forceinline__ double2 lds2(const double *p) { return *reinterpret_cast<const double2 *>(p); }
-
-__device__ __forceinline__ void store_pair(double *p, double o0, double o1, bool pair) {
-  if (pair) *reinterpret_cast<double2 *>(p) = make_double2(o0, o1);
-  else *p = o0;
-}
 
 // 2D: march one x strip of tx cells over planes (= rows) p0..p1.  Thread ctid owns the
 // cell pairs kk = ctid + i*NC (i < PPT), contiguous across lanes (conflict-free 16-byte LDS,
@@ -901,247 +702,6 @@ __global__ void __launch_bounds__(JB_THREADS, 1) jb_sweep(const __grid_constant_
   }
 }
 
-// ---------------------------------------------------------------- resident (on-chip) kernel
-// SURVEY §8(f) N2, after PERKS: for slabs small enough to live in
-// the shared memory of their CTAs, each CTA keeps one (outer-plane x row) block of the slab — plus
-// a one-row halo ring — in shared memory for the whole run.  Per iteration it (1) refreshes only
-// the halo ring from L2 (its neighbour blocks' faces; the slab's outer halo after the neighbour
-// GPU's flag), (2) computes every owned cell into registers, (3) writes them back to shared memory
-// and stores only its faces to the next global buffer — plus, for blocks on the slab's edge
-// plane, into the neighbour GPU's halo followed by one sys-scope release of its flag slot
-// — and (4) joins the slab's grid barrier.  The full block is written to
-// global memory in the last iteration, so buffers are consistent between runs and modes.
-// Same fp64 operation order as the oracle.
-template <int DIM, int CPP>
-__global__ void __launch_bounds__(JB_RNT, 1) jb_resident(const __grid_constant__ JbParams P) {
-  extern __shared__ __align__(16) double tile[];
-  __shared__ int s_abort;
-  const JbGeom &g = P.g;
-  int si = 0;
-  while (si + 1 < P.nslabs && (int)blockIdx.x >= P.s[si + 1].cta_begin) ++si;
-  const JbSlab &SL = P.s[si];
-  const int c = (int)blockIdx.x - SL.cta_begin;
-  const int nby = SL.res_nby;
-  const int bz = c / nby, by = c - bz * nby;
-  int pz0, zb, y0 = 0, yb = 1;  // 32-bit: resident slabs are < 2^31 elements (host-checked)
-  {
-    int64_t a, b;
-    jbplan_even_split(SL.chunk, SL.res_nbz, bz, &a, &b);
-    pz0 = (int)a + 1;  // owned planes pz0 .. pz0+zb-1 (slab planes are 1-based)
-    zb = (int)b;
-    if (DIM == 3) {
-      jbplan_even_split(g.ny - 2, nby, by, &a, &b);
-      y0 = (int)a + 1;
-      yb = (int)b;
-    }
-  }
-  const int rs = g.res_rs;
-  const int YR = DIM == 3 ? yb + 2 : 1;  // smem rows per plane (incl. y halo rows)
-  const int pe = (int)g.plane_elems, pitch = (int)g.pitch;
-  const int nx = (int)g.nx;
-  const int ppr = (nx - 1) / 2;               // pairs per row: x = 1+2j, 2+2j
-  const int tid = threadIdx.x;
-  const bool has_top = SL.flag_out_top != nullptr, has_bot = SL.flag_out_bot != nullptr;
-  const bool top_blk = has_top && bz == 0, bot_blk = has_bot && bz == SL.res_nbz - 1;
-  // smem row of (lz, ly), lz in [-1, zb], ly in [-1, yb] (ly ignored in 2D)
-  auto srow = [&](int lz, int ly) { return ((lz + 1) * YR + (DIM == 3 ? ly + 1 : 0)) * rs; };
-  // global element offset of (plane pz0+lz, row y0+ly, x) in a slab buffer
-  auto goff = [&](int lz, int ly, int x) {
-    return (pz0 + lz) * pe + (DIM == 3 ? (y0 + ly) * pitch : 0) + 3 + x;
-  };
-
-  // ---- this thread's cell pairs (fixed for the run)
-  int soff[CPP];
-  int gofs[CPP];  // element offsets inside the slab buffer (host checks the slab is < 2^31 elements)
-  unsigned valid = 0, full = 0, face = 0, top_face = 0, bot_face = 0;
-  const int nrows = zb * yb;
-#pragma unroll
-  for (int i = 0; i < CPP; ++i) {
-    const int k = tid + i * JB_RNT;
-    const int r = k / ppr, j = k - r * ppr;
-    const int lz = DIM == 3 ? r / yb : r, ly = DIM == 3 ? r - lz * yb : 0;
-    const int x = 1 + 2 * j;
-    soff[i] = srow(lz, ly) + x + 1;
-    gofs[i] = (int)goff(lz, ly, x);
-    if (r < nrows) {
-      valid |= 1u << i;
-      if (x + 1 <= nx - 2) full |= 1u << i;
-      const bool f = lz == 0 || lz == zb - 1 || (DIM == 3 && (ly == 0 || ly == yb - 1));
-      if (f) face |= 1u << i;
-      if (top_blk && lz == 0) top_face |= 1u << i;
-      if (bot_blk && lz == zb - 1) bot_face |= 1u << i;
-    }
-  }
-  if (tid == 0) s_abort = 0;
-  // neighbour blocks (face-sharing) for the relaxed synchronisation
-  const bool relaxed = SL.res_relaxed != 0;
-  int nbr[4], n_nbr = 0;
-  if (bz > 0) nbr[n_nbr++] = c - nby;
-  if (bz < SL.res_nbz - 1) nbr[n_nbr++] = c + nby;
-  if (DIM == 3 && by > 0) nbr[n_nbr++] = c - 1;
-  if (DIM == 3 && by < nby - 1) nbr[n_nbr++] = c + 1;
-
-  // ---- whole block + ring (incl. the x boundary cells) at run start: flattened over all threads
-  auto load_all = [&](const double *src) {
-    const int nrow = (zb + 2) * YR;
-    for (int k = tid; k < nrow * nx; k += JB_RNT) {
-      const int rr = k / nx, x = k - rr * nx;
-      const int lz = rr / YR - 1, ly = DIM == 3 ? rr % YR - 1 : 0;
-      tile[srow(lz, ly) + 1 + x] = __ldcg(src + goff(lz, ly, x));
-    }
-  };
-  // ---- halo ring only (interior x), one 16-byte pair per thread per step: ring row rr is
-  //      2D: lz = -1, zb;  3D: (lz = -1 | zb, ly = 0..yb-1) then (ly = -1 | yb, lz = 0..zb-1)
-  const int ring_rows = DIM == 3 ? 2 * yb + 2 * zb : 2;
-  auto load_ring = [&](const double *src) {
-    for (int k = tid; k < ring_rows * ppr; k += JB_RNT) {
-      const int rr = k / ppr, q = k - rr * ppr;
-      int lz, ly;
-      if (DIM == 2) {
-        lz = rr == 0 ? -1 : zb;
-        ly = 0;
-      } else if (rr < 2 * yb) {
-        lz = rr < yb ? -1 : zb;
-        ly = rr < yb ? rr : rr - yb;
-      } else {
-        const int r2 = rr - 2 * yb;
-        ly = r2 < zb ? -1 : yb;
-        lz = r2 < zb ? r2 : r2 - zb;
-      }
-      const int x = 1 + 2 * q;
-      const double *gp = src + goff(lz, ly, x);
-      double *sp = tile + srow(lz, ly) + 1 + x;
-      if (x + 1 <= nx - 2) *reinterpret_cast<double2 *>(sp) = __ldcg(reinterpret_cast<const double2 *>(gp));
-      else *sp = __ldcg(gp);
-    }
-  };
-
-  for (int64_t t = 0; t < P.iters; ++t) {
-    const int64_t tg = P.t0 + t;
-    const double *cur = SL.buf[tg & 1];
-    double *nxt = SL.buf[(tg + 1) & 1];
-    // (1) halo: wait for the neighbour GPU's edge plane (and, with relaxed sync, for the
-    //     neighbour blocks' faces of the previous iteration), then refresh the ring from L2
-    if (t > 0 && (top_blk || bot_blk || relaxed)) {
-      if (tid < 32) {
-        bool ok = true;
-        if (top_blk) ok &= wait_slots(SL.flag_in_top, SL.k_in_top, (unsigned long long)tg, P, tid);
-        if (bot_blk) ok &= wait_slots(SL.flag_in_bot, SL.k_in_bot, (unsigned long long)tg, P, tid);
-        if (relaxed) ok &= wait_slots_idx(SL.blk_flags, nbr, n_nbr, (unsigned long long)tg, P, tid);
-        if (tid == 0 && !ok) s_abort = 1;
-      }
-      __syncthreads();
-      if (s_abort) return;
-    }
-    if (t == 0) load_all(cur);
-    else load_ring(cur);
-    __syncthreads();
-    // (2) compute every owned pair into registers (oracle order)
-    double2 v[CPP];
-#pragma unroll
-    for (int i = 0; i < CPP; ++i) {
-      if (valid >> i & 1u) {
-        const double *cc = tile + soff[i];
-        const double2 C = lds2(cc);
-        const double w = cc[-1], e = cc[2];
-        if (DIM == 2) {
-          const double2 N = lds2(cc + rs), S = lds2(cc - rs);  // y+1 / y-1 = next / previous plane
-          v[i].x = 0.25 * (((C.y + w) + N.x) + S.x);
-          v[i].y = 0.25 * (((e + C.x) + N.y) + S.y);
-        } else {
-          const double2 N = lds2(cc + rs), S = lds2(cc - rs);            // y+1, y-1
-          const double2 U = lds2(cc + YR * rs), D = lds2(cc - YR * rs);  // z+1, z-1
-          v[i].x = kC6 * (((((C.y + w) + N.x) + S.x) + U.x) + D.x);
-          v[i].y = kC6 * (((((e + C.x) + N.y) + S.y) + U.y) + D.y);
-        }
-      }
-    }
-    __syncthreads();
-    // (3) write back; faces (all cells in the last iteration) to the next buffer; edge-plane
-    //     cells also into the neighbour GPU's halo
-    const bool last = t == P.iters - 1;
-    double *rt = top_blk ? SL.peer_top[(tg + 1) & 1] : nullptr;
-    double *rb = bot_blk ? SL.peer_bot[(tg + 1) & 1] : nullptr;
-#pragma unroll
-    for (int i = 0; i < CPP; ++i) {
-      if (valid >> i & 1u) {
-        const bool fl = full >> i & 1u;
-        double *sp = tile + soff[i];
-        if (fl) *reinterpret_cast<double2 *>(sp) = v[i];
-        else sp[0] = v[i].x;
-        if (last || (face >> i & 1u)) {
-          double *gp = nxt + gofs[i];
-          if (fl) __stcg(reinterpret_cast<double2 *>(gp), v[i]);
-          else __stcg(gp, v[i].x);
-        }
-        // the peer halo plane has the same in-plane layout: drop this block's plane offset
-        if (top_face >> i & 1u) store_pair(rt + (gofs[i] - pz0 * pe), v[i].x, v[i].y, fl);
-        if (bot_face >> i & 1u) store_pair(rb + (gofs[i] - (pz0 + zb - 1) * pe), v[i].x, v[i].y, fl);
-      }
-    }
-    if (top_blk || bot_blk) {
-      __syncthreads();  // every thread's peer stores precede thread 0's release (CTA scope)
-      if (tid == 0 && !((P.flags & JACOBI_FLAG_DROP_SIGNAL) && SL.slab_id == 0)) {
-        if (top_blk) st_release_sys(SL.flag_out_top + by, (unsigned long long)(tg + 1));
-        if (bot_blk) st_release_sys(SL.flag_out_bot + by, (unsigned long long)(tg + 1));
-      }
-    }
-    // (4) grid barrier of the slab, or with relaxed sync only a release of this block's
-    //     flag: its neighbours wait for it before reading its faces (and nobody else needs to)
-    __syncthreads();
-    if (relaxed) {
-      if (tid == 0) st_release_gpu(SL.blk_flags + c, (unsigned long long)(tg + 1));
-      continue;
-    }
-    if (tid == 0) {
-      red_release_gpu_add(SL.barrier, 1ull);
-      const bool ok = wait_geq<false>(SL.barrier, (unsigned long long)SL.cta_count * (t + 1), P);
-      s_abort = (!ok || *(volatile int *)(P.status + 1)) ? 1 : 0;
-    }
-    __syncthreads();
-    if (s_abort) return;
-  }
-  // End of run: the neighbours' last halo planes have landed before the kernel completes.
-  if (tid < 32 && P.iters > 0) {
-    if (top_blk) wait_slots(SL.flag_in_top, SL.k_in_top, (unsigned long long)(P.t0 + P.iters), P, tid);
-    if (bot_blk) wait_slots(SL.flag_in_bot, SL.k_in_bot, (unsigned long long)(P.t0 + P.iters), P, tid);
-  }
-}
-
-// ---------------------------------------------------------------- init / utility kernels
-__device__ __forceinline__ double u12_value(unsigned long long idx, unsigned long long seed) {
-  unsigned long long z = seed + (idx + 1ull) * kGolden;
-  z = (z ^ (z >> 30)) * 0xBF58476D1CE4E5B9ull;
-  z = (z ^ (z >> 27)) * 0x94D049BB133111EBull;
-  z = z ^ (z >> 31);
-  return __longlong_as_double((long long)(0x3FF0000000000000ull | (z >> 12)));
-}
-
-// Fill planes 0..nplanes-1 of a slab whose plane 0 is global outer index z_first with U12.
-__global__ void jb_init_u12(double *b0, double *b1, int64_t nplanes, JbGeom g, int64_t z_first,
-                            unsigned long long seed) {
-  const int64_t n = nplanes * g.plane_elems;
-  for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n;
-       i += (int64_t)gridDim.x * blockDim.x) {
-    const int64_t p = i / g.plane_elems, rem = i - p * g.plane_elems;
-    int64_t y, pos, idx = -1;
-    if (g.dim == 2) {
-      y = z_first + p;
-      pos = rem;
-      const int64_t x = pos - 3;
-      if (x >= 0 && x < g.nx) idx = y * g.nx + x;
-    } else {
-      y = rem / g.pitch;
-      pos = rem - y * g.pitch;
-      const int64_t x = pos - 3;
-      if (x >= 0 && x < g.nx) idx = ((z_first + p) * g.ny + y) * g.nx + x;
-    }
-    const double v = idx >= 0 ? u12_value((unsigned long long)idx, seed) : 0.0;
-    b0[i] = v;
-    if (b1) b1[i] = v;
-  }
-}
-
 // "Baseline NVSHMEM": the dedicated kernel, launched by the host every iteration after
 // the compute kernel, that waits until both neighbours delivered this iteration's halos.
 __global__ void jb_neighbour_wait(const __grid_constant__ JbParams P, unsigned long long target) {
@@ -1149,10 +709,6 @@ __global__ void jb_neighbour_wait(const __grid_constant__ JbParams P, unsigned l
   const int lane = threadIdx.x & 31;
   if (S.k_in_top > 0) wait_slots(S.flag_in_top, S.k_in_top, target, P, lane);
   if (S.k_in_bot > 0) wait_slots(S.flag_in_bot, S.k_in_bot, target, P, lane);
-}
-
-__global__ void jb_flag_max(unsigned long long *flags, int n, unsigned long long v) {
-  for (int i = threadIdx.x; i < n; i += blockDim.x) atomicMax(flags + i, v);
 }
 
 template <int DIM, bool NOCOMP, bool PERSIST>
@@ -1199,42 +755,8 @@ cudaError_t launch_sweep(const JbParams &p, bool nocomp, bool persist, int grid,
   return cudaLaunchKernel(fn, dim3(grid), dim3(JB_THREADS), args, smem, st);
 }
 
-const void *resident_fn(int dim, int cpp) {
-#define JB_RES(D, C) reinterpret_cast<const void *>(&jb_resident<D, C>)
-  if (dim == 2) {
-    switch (cpp) { case 1: return JB_RES(2, 1); case 2: return JB_RES(2, 2); case 4: return JB_RES(2, 4);
-                   default: return JB_RES(2, 8); }
-  }
-  switch (cpp) { case 1: return JB_RES(3, 1); case 2: return JB_RES(3, 2); case 4: return JB_RES(3, 4);
-                 default: return JB_RES(3, 8); }
-#undef JB_RES
-}
-
-cudaError_t prepare_resident(int dim, int cpp, size_t smem, int *blocks_per_sm) {
-  const void *fn = resident_fn(dim, cpp);
-  cudaError_t e = cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-  if (e != cudaSuccess) return e;
-  return cudaOccupancyMaxActiveBlocksPerMultiprocessor(blocks_per_sm, fn, JB_RNT, smem);
-}
-
-cudaError_t launch_resident(const JbParams &p, int cpp, int grid, size_t smem, cudaStream_t st) {
-  void *args[] = {const_cast<JbParams *>(&p)};
-  return cudaLaunchCooperativeKernel(resident_fn(p.g.dim, cpp), dim3(grid), dim3(JB_RNT), args, smem, st);
-}
-
-cudaError_t launch_init(double *b0, double *b1, int64_t nplanes, const JbGeom &g, int64_t z_first,
-                        unsigned long long seed, cudaStream_t st) {
-  jb_init_u12<<<1184, 256, 0, st>>>(b0, b1, nplanes, g, z_first, seed);
-  return cudaGetLastError();
-}
-
 cudaError_t launch_neighbour_wait(const JbParams &p, unsigned long long target, cudaStream_t st) {
   jb_neighbour_wait<<<1, 32, 0, st>>>(p, target);
-  return cudaGetLastError();
-}
-
-cudaError_t launch_flag_max(unsigned long long *flags, int n, unsigned long long v, cudaStream_t st) {
-  jb_flag_max<<<1, 64, 0, st>>>(flags, n, v);
   return cudaGetLastError();
 }
 
