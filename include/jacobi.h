@@ -186,6 +186,10 @@ int jacobi_num_slabs(jacobi_t h, int *local, int *total);
 /* Plan of local slab `i`: out[0..15] = start, chunk, pitch, plane_elems, tile_x, tile_y,
  * units_x, units_y, stages, n_top, n_bot, n_interior, ctas, k_planes, smem_bytes, device. */
 int jacobi_describe(jacobi_t h, int i, int64_t *out16);
+/* Raw copy of local slab i's buffer `parity` (0/1) in its HBM layout ((chunk+2)
+ * planes of plane_elems doubles, halos included) into a caller array of
+ * (chunk+2)*plane_elems doubles — for tests of the halo protocol. */
+int jacobi_read_slab(jacobi_t h, int i, int parity, double *out);
 const char *jacobi_strerror(int code);
 int jacobi_destroy(jacobi_t h);                         /* NULL-safe */
 

@@ -73,6 +73,7 @@ _SIGS = {
     "jacobi_set_tolerance": ([_p, _c.c_double], _c.c_int),
     "jacobi_last_norm": ([_p, _c.POINTER(_c.c_double)], _c.c_int),
     "jacobi_slab_bytes": ([_i64, _i64, _i64, _c.c_int, _c.c_int, _c.c_int, _c.POINTER(_i64)], _c.c_int),
+    "jacobi_read_slab": ([_p, _c.c_int, _c.c_int, _p], _c.c_int),
 }
 # exported only by the NVSHMEM variant (libjacobi_b200_nvshmem.so)
 _SIGS_NVSHMEM = {
@@ -402,6 +403,16 @@ class Jacobi:
     @property
     def iterations(self) -> int:
         return jacobi_iterations(self.h)
+
+    def read_slab(self, i: int, parity: int) -> np.ndarray:
+        """Raw slab buffer (chunk+2 planes incl. halos) as (planes, [ny,] pitch)."""
+        d = self.describe(i)
+        planes = d["chunk"] + 2
+        out = np.empty(planes * d["plane_elems"], dtype=np.float64)
+        _check(lib().jacobi_read_slab(self.h, i, parity, out.ctypes.data), "jacobi_read_slab")
+        if self.nz > 1:
+            return out.reshape(planes, self.ny, d["pitch"])
+        return out.reshape(planes, d["pitch"])
 
     def describe(self, i: int = 0) -> dict:
         return jacobi_describe(self.h, i)

@@ -1452,6 +1452,14 @@ int jacobi_last_norm(jacobi_t h, double *norm) {
   return JACOBI_OK;
 }
 
+int jacobi_read_slab(jacobi_t h, int i, int parity, double *out) {
+  if (!h || !out || i < 0 || i >= (int)h->slabs.size() || (parity != 0 && parity != 1)) return JACOBI_EINVAL;
+  Slab &s = h->slabs[i];
+  CK(cudaSetDevice(s.device));
+  CK(cudaMemcpy(out, s.buf[parity], (size_t)slab_elems(h, s) * sizeof(double), cudaMemcpyDeviceToHost));
+  return JACOBI_OK;
+}
+
 int jacobi_last_time(jacobi_t h, double *ms_max, double *ms_per_slab) {
   if (!h) return JACOBI_EINVAL;
   if (ms_max) *ms_max = h->last_ms_max;

@@ -514,11 +514,11 @@ __global__ void __launch_bounds__(JB_THREADS, 1) jb_sweep(const __grid_constant_
     const bool active = !(NOCOMP && role == ROLE_INT);
 
     if (producer) {
-      if (lane == 0) {
-        fence_proxy_async_global();
-        // The claim counter of the next iteration is idle now (last used in iteration t-1).
-        if (c == 0 && SL.work_ctr) SL.work_ctr[(tg + 1) & 1] = 0u;
-      }
+      // Every lane that issues bulk copies orders them after the grid barrier's acquire (and the
+      // generic-proxy stores it covers) with its own proxy fence.
+      fence_proxy_async_global();
+      // The claim counter of the next iteration is idle now (last used in iteration t-1).
+      if (lane == 0 && c == 0 && SL.work_ctr) SL.work_ctr[(tg + 1) & 1] = 0u;
       // boundary blocks wait until the neighbour committed the halo of the previous time
       // step.  With compute, the two owned planes of the first boundary tile are already in
       // flight while we wait; only the halo plane's load waits for the flag.
@@ -527,8 +527,8 @@ __global__ void __launch_bounds__(JB_THREADS, 1) jb_sweep(const __grid_constant_
         if (!waited) {
           if (role == ROLE_TOP) wait_slots(SL.flag_in_top, SL.k_in_top, (unsigned long long)tg, P, lane);
           else wait_slots(SL.flag_in_bot, SL.k_in_bot, (unsigned long long)tg, P, lane);
-          if (lane == 0) fence_proxy_async_global();
           __syncwarp();
+          fence_proxy_async_global();  // every copying lane: halo rows written by the neighbour
           waited = true;
         }
       };

@@ -211,6 +211,26 @@ def test_gather_scatter_roundtrip_and_run_zero():
         assert_bitwise(j.gather(), f, "roundtrip")
 
 
+@pytest.mark.parametrize("shape", [(20, 64), (11, 9, 40)])
+def test_no_compute_halo_slots_hold_neighbour_edges(shape):
+    """after a no-compute run each slab's halo planes hold the neighbour's edge
+    planes (P:550-552 measurement mode still moves every halo byte)."""
+    f = u12(shape, 4)
+    P = 3
+    with jb.Jacobi(shape, virtual=P) as j:
+        j.scatter(f)
+        j.set_param("resident", 0)
+        j.set_mode(jb.MODE_CPUFREE, jb.FLAG_NO_COMPUTE).run(3)
+        par = j.iterations & 1
+        slabs = [j.read_slab(i, par) for i in range(P)]
+        chunks = [j.describe(i)["chunk"] for i in range(P)]
+    for g in range(P):
+        if g > 0:      # my top halo (plane 0) == top neighbour's last owned plane
+            assert np.array_equal(slabs[g][0], slabs[g - 1][chunks[g - 1]])
+        if g < P - 1:  # my bottom halo == bottom neighbour's first owned plane
+            assert np.array_equal(slabs[g][chunks[g] + 1], slabs[g + 1][1])
+
+
 def test_no_compute_mode_moves_halos_only():
     f = u12((20, 64), 4)
     with jb.Jacobi(f.shape, virtual=2) as j:
