@@ -1,0 +1,51 @@
+"""Write tests/golden/*.json — every stored value computed by oracle/ only (never the CUDA path).
+
+PAPER.md prints no numeric results and no worked example (its figures are images), so
+these fixtures are oracle regression anchors: SHA-256 digests of the bit patterns of oracle runs on
+the BASELINE.json workloads' small configs, plus a few sampled cell values for readability.
+Run:  python tests/golden/make_golden.py
+"""
+import hashlib
+import json
+import os
+import sys
+
+HERE = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, os.path.dirname(os.path.dirname(HERE)))
+
+import numpy as np  # noqa: E402
+
+import oracle  # noqa: E402
+from jacobi_inputs import SEED_BENCH, u12  # noqa: E402
+
+CASES = {
+    # name: (shape (z, y, x) or (y, x), iterations) — C1 of BASELINE.json and small 3D/2D anchors
+    "c1_2d_256x256_u12_5c24_1000it": ((256, 256), 1000),
+    "3d_34x30x40_u12_5c24_200it": ((34, 30, 40), 200),
+    "2d_66x1030_u12_5c24_77it": ((66, 1030), 77),
+}
+
+
+def digest(a: np.ndarray) -> str:
+    return hashlib.sha256(np.ascontiguousarray(a, dtype=np.float64).tobytes()).hexdigest()
+
+
+def compute(shape, iters):
+    return oracle.jacobi(u12(shape, SEED_BENCH), iters, os.cpu_count() or 1)
+
+
+def main():
+    out = {}
+    for name, (shape, iters) in CASES.items():
+        r = compute(shape, iters)
+        mid = tuple(s // 2 for s in shape)
+        out[name] = {"shape": list(shape), "iters": iters, "seed": SEED_BENCH, "sha256": digest(r),
+                     "center_value": float(r[mid]), "mean": float(r.mean()),
+                     "generator": "tests/golden/make_golden.py (oracle.jacobi, C oracle)"}
+    with open(os.path.join(HERE, "oracle_digests.json"), "w") as f:
+        json.dump(out, f, indent=1)
+    print(json.dumps(out, indent=1))
+
+
+if __name__ == "__main__":
+    main()

@@ -367,3 +367,18 @@ def test_update_norm_zero_for_harmonic_field(oracle_mod):
     f = x * x - y * y
     out, done, norms = oracle_mod.jacobi_converge(f, 100, 0.0, 5)
     assert done == 5 and norms == [0.0] and np.array_equal(out, f)
+
+
+def test_golden_digests(oracle_mod):
+    """Regression pin: the oracle still reproduces the committed digests (tests/golden)."""
+    import json
+    import os
+    import sys
+    here = os.path.join(os.path.dirname(__file__), "golden")
+    sys.path.insert(0, here)
+    import make_golden
+    with open(os.path.join(here, "oracle_digests.json")) as f:
+        gold = json.load(f)
+    for name, g in gold.items():
+        r = make_golden.compute(tuple(g["shape"]), g["iters"])
+        assert make_golden.digest(r) == g["sha256"], name
