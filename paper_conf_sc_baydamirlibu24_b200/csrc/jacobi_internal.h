@@ -34,6 +34,9 @@ struct JbGeom {
   int32_t stages;       // ring depth
   int32_t stage_doubles;// rh * ws
   int32_t res_rs;       // resident kernel: smem row stride in doubles (x at column x + 1)
+  int32_t l2hint;       // streaming loads: 1 = L2 evict_first for rows read once, evict_last for
+                        // 3D y-halo rows (read again by the neighbouring tile)
+  int32_t pad1;
 };
 
 struct JbCtrl;

@@ -168,6 +168,7 @@ struct jacobi_ctx {
   int64_t min_block = 8, dyn_help = 1;
   int64_t resident = -1;       // on-chip resident kernel: -1 auto (when the slab fits), 0 off, 1 on
   int64_t block_sync = 0;      // resident kernel: 0 grid barrier, 1 neighbour-block flags
+  int64_t l2hint = -1;         // streaming loads with L2 eviction hints (-1 default = off)
   int64_t last_resident = 0;   // read-only: whether the last CPU-Free run used it
   int64_t norm_every = 0;      // N4: check the update norm every k iterations (0 = off)
   double tol = 0.0;            // N4: stop once the norm <= tol
@@ -407,6 +408,7 @@ int plan_launch(jacobi_ctx *h, const std::vector<int> &idx, LaunchKind lk, bool 
     if (jbplan::geometry(h->nx, h->ny, h->nz, h->dim, (int)h->tile_x, ty, smem_optin, (int)h->stages, &g))
       return JACOBI_EINVAL;
   }
+  g.l2hint = (int32_t)(h->l2hint < 0 ? 0 : h->l2hint);
   L.smem = jbplan::smem_bytes(g);
   CK(jbk::prepare(h->dim, nocomp, persist, L.smem));
   int occ = 0;
@@ -1370,6 +1372,7 @@ static int64_t *param_slot(jacobi_t h, const char *name) {
   if (!std::strcmp(name, "resident")) return &h->resident;
   if (!std::strcmp(name, "block_sync")) return &h->block_sync;
   if (!std::strcmp(name, "norm_every")) return &h->norm_every;
+  if (!std::strcmp(name, "l2hint")) return &h->l2hint;
   if (!std::strcmp(name, "last_resident")) return &h->last_resident;
   return nullptr;
 }

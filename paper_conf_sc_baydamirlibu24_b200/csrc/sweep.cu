@@ -137,8 +137,15 @@ __device__ __forceinline__ void produce_stage(const JbGeom &g, const TileSrc &T,
     mbar_expect_tx(&R.full[at.slot], T.row_bytes * (uint32_t)T.nrows);
   }
   __syncwarp();
-  if (lane < T.nrows)
-    bulk_g2s(R.stage(at) + (size_t)lane * g.ws, T.base + p * g.plane_elems, T.row_bytes, &R.full[at.slot]);
+  if (lane < T.nrows) {
+    double *dst = R.stage(at) + (size_t)lane * g.ws;
+    const double *src = T.base + p * g.plane_elems;
+    if (g.l2hint)  // y-halo rows (first/last of a 3D stage) are read again by the neighbour tile
+      bulk_g2s_hint(dst, src, T.row_bytes, &R.full[at.slot],
+                    l2_policy(g.dim == 3 && (lane == 0 || lane == T.nrows - 1)));
+    else
+      bulk_g2s(dst, src, T.row_bytes, &R.full[at.slot]);
+  }
 }
 
 // Load planes pf..pl of tile `unit` from `cur` into consecutive ring stages starting at q.
