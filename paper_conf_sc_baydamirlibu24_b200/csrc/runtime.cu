@@ -1,194 +1,10 @@
-// runtime.cu — host runtime behind the C ABI in include/jacobi.h.
-//
-// Owns devices, slabs (HBM buffers + control blocks), peer mappings (UVA peer access in one
-// process, CUDA IPC across processes), launches, timing, and the CPU-controlled baselines.
-// All device work is done by the kernels in sweep.cu / resident.cu / util.cu; the host only
-// orchestrates.
-#include <cuda_runtime.h>
-#include <dlfcn.h>
-#include <nccl.h>
+// runtime.cu — host runtime behind the C ABI in include/jacobi.h: slabs (HBM buffers + control
+// blocks), planning (tiles, block split, schedules), the CPU-Free run, data movement.  The
+// CPU-controlled baselines live in baselines.cu, multi-process plumbing in multiproc.cu.  All
+// device work is done by the kernels in sweep.cu / resident.cu / util.cu.
+#include "runtime_internal.h"
 
-#include <algorithm>
-#include <cstdio>
-#include <cstdlib>
-#include <cstddef>
-#include <cstring>
-#include <string>
-#include <vector>
-
-#include "../../include/jacobi.h"
-#include "jacobi_internal.h"
-#ifdef JB_NVSHMEM
-#include <nvshmem.h>
-#include <nvshmemx.h>
-#endif
-
-namespace jbk {
-cudaError_t prepare(int dim, bool nocomp, bool persist, size_t smem);
-cudaError_t occupancy(int dim, bool nocomp, bool persist, size_t smem, int *blocks_per_sm);
-cudaError_t launch_sweep(const JbParams &p, bool nocomp, bool persist, int grid, size_t smem,
-                         cudaStream_t st);
-cudaError_t launch_init(double *b0, double *b1, int64_t nplanes, const JbGeom &g, int64_t z_first,
-                        unsigned long long seed, cudaStream_t st);
-cudaError_t launch_flag_max(unsigned long long *flags, int n, unsigned long long v, cudaStream_t st);
-cudaError_t prepare_resident(int dim, int cpp, size_t smem, int *blocks_per_sm);
-cudaError_t launch_resident(const JbParams &p, int cpp, int grid, size_t smem, cudaStream_t st);
-cudaError_t launch_neighbour_wait(const JbParams &p, unsigned long long target, cudaStream_t st);
-}  // namespace jbk
-
-namespace {
-
-constexpr unsigned long long kSeedBench = 0x5C24ull;
-enum Kind { KIND_SINGLE = 0, KIND_VIRTUAL = 1, KIND_DIST = 2, KIND_SHMEM = 3 };
-
-int cuda_err(cudaError_t e) {
-  if (e == cudaSuccess) return JACOBI_OK;
-  if (e == cudaErrorMemoryAllocation) return JACOBI_ENOMEM;
-  if (e == cudaErrorCooperativeLaunchTooLarge) return JACOBI_ENOCOOP;
-  if (getenv("JACOBI_DEBUG")) fprintf(stderr, "[jacobi] CUDA error: %s\n", cudaGetErrorString(e));
-  return JACOBI_ECUDA;
-}
-#define CK(x)                                  \
-  do {                                         \
-    int _rc = cuda_err(x);                     \
-    if (_rc != JACOBI_OK) return _rc;          \
-  } while (0)
-
-// ---------------------------------------------------------------- NCCL (dlopen'ed on demand)
-struct NcclApi {
-  void *lib = nullptr;
-  ncclResult_t (*GetUniqueId)(ncclUniqueId *) = nullptr;
-  ncclResult_t (*CommInitRank)(ncclComm_t *, int, ncclUniqueId, int) = nullptr;
-  ncclResult_t (*CommInitAll)(ncclComm_t *, int, const int *) = nullptr;
-  ncclResult_t (*CommDestroy)(ncclComm_t) = nullptr;
-  ncclResult_t (*Send)(const void *, size_t, ncclDataType_t, int, ncclComm_t, cudaStream_t) = nullptr;
-  ncclResult_t (*Recv)(void *, size_t, ncclDataType_t, int, ncclComm_t, cudaStream_t) = nullptr;
-  ncclResult_t (*GroupStart)() = nullptr;
-  ncclResult_t (*GroupEnd)() = nullptr;
-  bool load() {
-    if (lib) return true;
-    const char *names[] = {"libnccl.so.2", "libnccl.so"};
-    for (const char *n : names) {
-      lib = dlopen(n, RTLD_NOW | RTLD_GLOBAL);
-      if (lib) break;
-    }
-    if (!lib) return false;
-#define LD(f) f = reinterpret_cast<decltype(f)>(dlsym(lib, "nccl" #f))
-    LD(GetUniqueId); LD(CommInitRank); LD(CommInitAll); LD(CommDestroy);
-    LD(Send); LD(Recv); LD(GroupStart); LD(GroupEnd);
-#undef LD
-    return GetUniqueId && CommInitRank && CommInitAll && CommDestroy && Send && Recv && GroupStart && GroupEnd;
-  }
-};
-NcclApi g_nccl;
-
-// Device-memory allocator for the slab buffers and control blocks (jacobi_set_allocator):
-// cudaMalloc by default, or a caller-supplied one (the Python binding installs PyTorch's caching
-// allocator so that PyTorch owns the device memory, as the north star asks).
-struct Allocator {
-  jacobi_alloc_fn alloc = nullptr;
-  jacobi_free_fn free = nullptr;
-  void *user = nullptr;
-};
-Allocator g_alloc;
-
-// cuMemGetAddressRange through the runtime's driver entry point (no libcuda link needed): the
-// base of the allocation containing `p`, so IPC handles of sub-allocations carry their offset.
-typedef int (*PFN_getAddressRange)(unsigned long long *, size_t *, unsigned long long);
-size_t alloc_offset(const void *p) {
-  static PFN_getAddressRange fn = nullptr;
-  if (!fn) {
-    void *f = nullptr;
-    cudaDriverEntryPointQueryResult q;
-    if (cudaGetDriverEntryPoint("cuMemGetAddressRange", &f, cudaEnableDefault, &q) != cudaSuccess || !f) return 0;
-    fn = reinterpret_cast<PFN_getAddressRange>(f);
-  }
-  unsigned long long base = 0;
-  size_t size = 0;
-  if (fn(&base, &size, (unsigned long long)p) != 0) return 0;
-  return (size_t)((unsigned long long)p - base);
-}
-
-// ---------------------------------------------------------------- IPC blob (dist mode)
-struct IpcBlob {
-  uint32_t magic;
-  int32_t rank;
-  int32_t sms;  // SM count of the rank's GPU: the CPU-Free role split must match across ranks
-  int32_t pad;
-  int64_t chunk;
-  int64_t plane_elems;
-  cudaIpcMemHandle_t buf[2];
-  cudaIpcMemHandle_t ctrl;
-  uint64_t off[3];  // offsets of buf[0], buf[1], ctrl inside their allocations (caller allocators)
-};
-constexpr uint32_t kIpcMagic = 0x4A43424Bu;
-
-}  // namespace
-
-struct Slab {
-  int device = 0;
-  int id = 0;  // global slab index
-  int64_t start = 0, chunk = 0;
-  double *buf[2] = {nullptr, nullptr};
-  JbCtrl *ctrl = nullptr;
-  cudaStream_t stream = nullptr;
-  cudaStream_t stream2 = nullptr;  // comm stream of the Copy-Overlap baseline
-  cudaEvent_t ev0 = nullptr, ev1 = nullptr;
-  cudaEvent_t ev_sync = nullptr, ev_copy = nullptr;  // baseline stream / graph dependencies
-  bool has_top = false, has_bot = false;
-  double *peer_top[2] = {nullptr, nullptr};
-  double *peer_bot[2] = {nullptr, nullptr};
-  unsigned long long *flag_out_top = nullptr, *flag_out_bot = nullptr;
-  int peer_top_dev = -1, peer_bot_dev = -1;
-  int shm_pe_top = -1, shm_pe_bot = -1;  // NVSHMEM variant: neighbour PEs
-  std::vector<void *> ipc_opened;
-  ncclComm_t comm = nullptr;
-  double last_ms = 0;
-  JbSlab desc{};  // last launch descriptor (for jacobi_describe)
-  int32_t *dyn_table = nullptr;  // guided-schedule block table (device)
-  unsigned long long *blk_flags = nullptr;  // resident kernel: per-block flags (device)
-  double *partials = nullptr;               // N4: per-run partial sums (device)
-  int64_t partials_cap = 0;
-  JbCtrl **norm_peers = nullptr;            // N4: device array of every slab's control block
-  int64_t dyn_key[4] = {0, 0, 0, 0};
-  int grid = 0;
-  size_t smem = 0;
-};
-
-struct jacobi_ctx {
-  int kind = KIND_SINGLE;
-  int64_t nx = 0, ny = 0, nz = 0, n_out = 0;
-  int stencil = 5, dim = 2;
-  int total = 1;  // total slabs P
-  int rank = 0;
-  std::vector<Slab> slabs;
-  int64_t t = 0;
-  int mode = JACOBI_MODE_CPUFREE, flags = 0;
-  int64_t tile_x = -1, tile_y = -1, stages = -1, boundary_ctas = -1, ctas = -1, schedule = -1;
-  int64_t min_block = 8, dyn_help = 1;
-  int64_t resident = -1;       // on-chip resident kernel: -1 auto (when the slab fits), 0 off, 1 on
-  int64_t block_sync = 0;      // resident kernel: 0 grid barrier, 1 neighbour-block flags
-  int64_t l2hint = -1;         // streaming loads with L2 eviction hints (-1 default = off)
-  int64_t last_resident = 0;   // read-only: whether the last CPU-Free run used it
-  int64_t norm_every = 0;      // N4: check the update norm every k iterations (0 = off)
-  double tol = 0.0;            // N4: stop once the norm <= tol
-  int64_t norm_checks = 0;     // N4: checks performed so far (monotone slot values)
-  double last_norm = -1.0;     // N4: norm of the last check
-  std::vector<JbCtrl *> all_ctrl;  // dist mode: every rank's control block (opened via IPC)
-  int64_t timeout_ms = 20000;
-  bool peers_ready = false;
-  bool nccl_ready = false;
-  double last_ms_max = 0;
-  cudaGraphExec_t graph_exec = nullptr;  // cached GRAPH-baseline executable
-  int64_t graph_iters = -1;
-  int graph_parity = -1;
-  int64_t graph_gen = -1, plan_gen = 0;  // plan_gen bumps on every set_mode / set_param
-  JbGeom geom{};  // layout geometry (pitch, plane_elems) fixed at create
-  Allocator alloc;  // allocator of buffers / control blocks (captured at create)
-};
-
-namespace {
-
+namespace jbrt {
 int64_t slab_elems(const jacobi_ctx *h, const Slab &s) { return (s.chunk + 2) * h->geom.plane_elems; }
 
 int validate(int64_t nx, int64_t ny, int64_t nz, int stencil, int nslabs) {
@@ -353,29 +169,14 @@ void neighbour_roles(const jacobi_ctx *h, int id, int sms, int units, int *nt_ou
   if (nb_out) *nb_out = nb;
 }
 
-struct LaunchPlan {
-  JbParams P;
-  int grid = 0;
-  int cpp = 0;  // resident kernel: cell pairs per thread
-  size_t smem = 0;
-  int device = 0;
-  cudaStream_t stream = nullptr;
-  std::vector<int> slab_idx;
-};
+
 
 // Plan one launch on one device over the local slabs `idx` (1 slab per GPU, or all slabs in
 // virtual mode).  persist=false plans the discrete baseline kernel (no boundary roles).
-// What a launch computes (CPU-Free persistent kernel or one of the discrete baseline kernels).
-enum LaunchKind {
-  LK_PERSIST = 0,  // CPU-Free: roles, peer stores, flags, grid barrier, all iterations
-  LK_ALL,          // discrete: every plane 1..chunk, no roles (Copy / NCCL / graph baselines)
-  LK_P2P,          // discrete: boundary roles store edge planes straight into the peers' halos
-  LK_INNER,        // discrete: planes 2..chunk-1 only (Copy-Overlap compute kernel)
-  LK_EDGES,        // discrete: planes 1 and chunk only, no peer stores (Copy-Overlap comm kernel)
-};
+
 
 int plan_launch(jacobi_ctx *h, const std::vector<int> &idx, LaunchKind lk, bool nocomp, LaunchPlan &L,
-                int grid_override = 0) {
+                int grid_override) {
   const bool persist = lk == LK_PERSIST;
   Slab &s0 = h->slabs[idx[0]];
   L.device = s0.device;
@@ -752,264 +553,9 @@ int run_cpufree(jacobi_ctx *h, int64_t iters) {
   h->t += done;
   return JACOBI_OK;
 }
+}  // namespace jbrt
 
-int ensure_nccl(jacobi_ctx *h) {
-  if (h->nccl_ready) return JACOBI_OK;
-  if (h->kind == KIND_VIRTUAL && h->total > 1) return JACOBI_EINVAL;  // NCCL: one rank per GPU
-  if (h->kind == KIND_DIST) return JACOBI_ESTATE;  // needs jacobi_nccl_init via the binding
-  if (h->kind == KIND_SHMEM) return JACOBI_EINVAL;
-  if (!g_nccl.load()) return JACOBI_ENCCL;
-  std::vector<int> devs;
-  for (auto &s : h->slabs) devs.push_back(s.device);
-  std::vector<ncclComm_t> comms(devs.size());
-  if (g_nccl.CommInitAll(comms.data(), (int)devs.size(), devs.data()) != ncclSuccess) return JACOBI_ENCCL;
-  for (size_t i = 0; i < devs.size(); ++i) h->slabs[i].comm = comms[i];
-  h->nccl_ready = true;
-  return JACOBI_OK;
-}
-
-// CPU-controlled baselines (Listing 2.1a).
-// Every iteration the host launches discrete kernels on every GPU, moves the edge planes into
-// the neighbours' halos, and synchronises every GPU before the next iteration (the
-// OpenMP/MPI barrier of the reference code):
-//   COPY    : kernel over all planes, then cudaMemcpyPeerAsync of the edge planes
-//   NCCL    : kernel, then ncclSend/ncclRecv of the edge planes (grouped)
-//   OVERLAP : boundary planes on a comm stream (few CTAs) + memcpy, interior planes concurrently
-//             on the compute stream ("Baseline Overlap")
-//   P2P     : one kernel whose boundary CTAs store the edge planes into the peers' halos
-//   GRAPH   : the COPY loop captured once into a CUDA graph (all iterations, cross-GPU event
-//             dependencies instead of host barriers) and replayed with one launch — the strongest
-//             CPU-controlled variant (not in the paper).
-enum BaseKind { BK_COPY, BK_NCCL, BK_OVERLAP, BK_P2P, BK_GRAPH, BK_SHMEM };
-
-int time_begin(jacobi_ctx *h) {
-  for (auto &s : h->slabs) {
-    CK(cudaSetDevice(s.device));
-    CK(reset_run_counters(s, s.stream));
-    CK(cudaEventRecord(s.ev0, s.stream));
-  }
-  return JACOBI_OK;
-}
-
-int time_end(jacobi_ctx *h, int64_t iters) {
-  double mx = 0;
-  for (auto &s : h->slabs) {
-    CK(cudaSetDevice(s.device));
-    CK(cudaEventRecord(s.ev1, s.stream));
-    CK(cudaEventSynchronize(s.ev1));
-    float ms = 0;
-    CK(cudaEventElapsedTime(&ms, s.ev0, s.ev1));
-    s.last_ms = ms;
-    mx = std::max(mx, (double)ms);
-  }
-  h->last_ms_max = mx;
-  h->t += iters;
-  // Keep the CPU-Free protocol consistent: inbound flags hold the global iteration count.
-  for (auto &s : h->slabs) {
-    CK(cudaSetDevice(s.device));
-    CK(jbk::launch_flag_max(&s.ctrl->flag_in[0][0], 2 * JB_MAXK, (unsigned long long)h->t, s.stream));
-    CK(cudaStreamSynchronize(s.stream));
-  }
-  return JACOBI_OK;
-}
-
-// Host-issued peer copies of slab s's edge planes of buffer `nxt` into its neighbours' halos.
-// (Inside a graph capture the UVA form cudaMemcpyAsync(cudaMemcpyDefault) is used: it is the
-// capturable equivalent of cudaMemcpyPeerAsync once peer access is enabled.)
-int copy_edges(jacobi_ctx *h, Slab &s, int nxt, cudaStream_t st, bool capturing = false) {
-  const int64_t pe = h->geom.plane_elems;
-  const size_t bytes = (size_t)pe * sizeof(double);
-  if (capturing) {
-    if (s.has_top) CK(cudaMemcpyAsync(s.peer_top[nxt], s.buf[nxt] + 1 * pe, bytes, cudaMemcpyDefault, st));
-    if (s.has_bot) CK(cudaMemcpyAsync(s.peer_bot[nxt], s.buf[nxt] + s.chunk * pe, bytes, cudaMemcpyDefault, st));
-    return JACOBI_OK;
-  }
-  if (s.has_top)
-    CK(cudaMemcpyPeerAsync(s.peer_top[nxt], s.peer_top_dev, s.buf[nxt] + 1 * pe, s.device, bytes, st));
-  if (s.has_bot)
-    CK(cudaMemcpyPeerAsync(s.peer_bot[nxt], s.peer_bot_dev, s.buf[nxt] + s.chunk * pe, s.device, bytes, st));
-  return JACOBI_OK;
-}
-
-int nccl_edges(jacobi_ctx *h, int nxt) {
-  const int64_t pe = h->geom.plane_elems;
-  if (g_nccl.GroupStart() != ncclSuccess) return JACOBI_ENCCL;
-  for (auto &s : h->slabs) {
-    const int me = s.id;
-    double *b = s.buf[nxt];
-    if (s.has_top) {
-      if (g_nccl.Send(b + 1 * pe, pe, ncclFloat64, me - 1, s.comm, s.stream) != ncclSuccess) return JACOBI_ENCCL;
-      if (g_nccl.Recv(b, pe, ncclFloat64, me - 1, s.comm, s.stream) != ncclSuccess) return JACOBI_ENCCL;
-    }
-    if (s.has_bot) {
-      if (g_nccl.Send(b + s.chunk * pe, pe, ncclFloat64, me + 1, s.comm, s.stream) != ncclSuccess)
-        return JACOBI_ENCCL;
-      if (g_nccl.Recv(b + (s.chunk + 1) * pe, pe, ncclFloat64, me + 1, s.comm, s.stream) != ncclSuccess)
-        return JACOBI_ENCCL;
-    }
-  }
-  if (g_nccl.GroupEnd() != ncclSuccess) return JACOBI_ENCCL;
-  return JACOBI_OK;
-}
-
-int run_graph(jacobi_ctx *h, int64_t iters, bool nocomp, std::vector<LaunchPlan> &plans);
-
-int run_baseline(jacobi_ctx *h, int64_t iters, BaseKind kind) {
-  const bool nocomp = h->flags & JACOBI_FLAG_NO_COMPUTE;
-  if (kind == BK_NCCL) {
-    int rc = ensure_nccl(h);
-    if (rc) return rc;
-  } else if (kind == BK_SHMEM) {
-    if (h->kind != KIND_SHMEM) return JACOBI_EINVAL;  // needs the NVSHMEM variant's handles
-  } else if ((h->kind == KIND_DIST || h->kind == KIND_SHMEM) && h->total > 1) {
-    return JACOBI_EINVAL;  // host-synchronised peer baselines need one process: use NCCL
-  }
-  const int n = (int)h->slabs.size();
-  std::vector<LaunchPlan> plans(n), edges(n);
-  for (int i = 0; i < n; ++i) {
-    Slab &s = h->slabs[i];
-    int rc;
-    if (kind == BK_P2P || kind == BK_SHMEM) {
-      rc = plan_launch(h, {i}, LK_P2P, nocomp, plans[i]);
-    } else if (kind == BK_OVERLAP && (s.has_top || s.has_bot)) {
-      int sms = 0;
-      CK(cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, s.device));
-      const int ne = std::max(2, std::min(sms / 8, 32));  // boundary CTAs on the comm stream
-      rc = plan_launch(h, {i}, LK_EDGES, nocomp, edges[i], ne);
-      if (!rc) rc = plan_launch(h, {i}, LK_INNER, nocomp, plans[i], sms - edges[i].grid);
-    } else {
-      rc = plan_launch(h, {i}, LK_ALL, nocomp, plans[i]);
-    }
-    if (rc) return rc;
-    plans[i].P.iters = 1;
-    edges[i].P.iters = 1;
-  }
-  if (kind == BK_GRAPH) return run_graph(h, iters, nocomp, plans);
-  int rc = time_begin(h);
-  if (rc) return rc;
-  // P2P / NVSHMEM no-compute still move halos in-kernel
-  const bool launch_kernels = !nocomp || kind == BK_P2P || kind == BK_SHMEM;
-  for (int64_t it = 0; it < iters; ++it) {
-    const int64_t tg = h->t + it;
-    const int nxt = (int)((tg + 1) & 1);
-    for (int i = 0; i < n; ++i) {  // ② launch the kernel(s) on every GPU
-      Slab &s = h->slabs[i];
-      CK(cudaSetDevice(s.device));
-      if (kind == BK_OVERLAP && edges[i].grid > 0) {
-        // comm stream: boundary planes first, then the peer copies; compute stream: interior
-        if (!nocomp) {
-          edges[i].P.t0 = tg;
-          CK(jbk::launch_sweep(edges[i].P, false, false, edges[i].grid, edges[i].smem, s.stream2));
-          plans[i].P.t0 = tg;
-          CK(jbk::launch_sweep(plans[i].P, false, false, plans[i].grid, plans[i].smem, s.stream));
-        }
-        rc = copy_edges(h, s, nxt, s.stream2);
-        if (rc) return rc;
-        continue;
-      }
-      if (launch_kernels) {
-        plans[i].P.t0 = tg;
-        CK(jbk::launch_sweep(plans[i].P, nocomp, false, plans[i].grid, plans[i].smem, s.stream));
-      }
-    }
-    if (kind == BK_COPY) {  // ④ write_neighbors with host-issued peer copies
-      for (auto &s : h->slabs) {
-        CK(cudaSetDevice(s.device));
-        rc = copy_edges(h, s, nxt, s.stream);
-        if (rc) return rc;
-      }
-    } else if (kind == BK_NCCL) {
-      rc = nccl_edges(h, nxt);
-      if (rc) return rc;
-    } else if (kind == BK_SHMEM) {
-      // the second per-iteration kernel waits for the neighbours' signals; no host
-      // barrier — the next iteration's kernel is ordered behind it on the stream.
-      for (int i = 0; i < n; ++i) {
-        Slab &s = h->slabs[i];
-        CK(cudaSetDevice(s.device));
-        CK(jbk::launch_neighbour_wait(plans[i].P, (unsigned long long)(tg + 1), s.stream));
-      }
-      continue;
-    }
-    for (auto &s : h->slabs) {  // ⑤ sync streams, host barrier: wait for every GPU
-      CK(cudaSetDevice(s.device));
-      CK(cudaStreamSynchronize(s.stream2));
-      CK(cudaStreamSynchronize(s.stream));
-    }
-  }
-  return time_end(h, iters);
-}
-
-// GRAPH baseline: capture `iters` iterations of (kernel; peer copies) for every slab into one
-// graph.  Slab g's kernel of iteration t+1 waits (graph edge) for the copies of its neighbours
-// at iteration t; its copies follow its own kernel.  The instantiated graph is cached per
-// (iters, parity of t, plan generation).
-int run_graph(jacobi_ctx *h, int64_t iters, bool nocomp, std::vector<LaunchPlan> &plans) {
-  const int n = (int)h->slabs.size();
-  const int parity = (int)(h->t & 1);
-  if (!h->graph_exec || h->graph_iters != iters || h->graph_parity != parity || h->graph_gen != h->plan_gen) {
-    if (h->graph_exec) cudaGraphExecDestroy(h->graph_exec);
-    h->graph_exec = nullptr;
-    Slab &m = h->slabs[0];
-    CK(cudaSetDevice(m.device));
-    CK(cudaStreamBeginCapture(m.stream, cudaStreamCaptureModeRelaxed));
-    CK(cudaEventRecord(m.ev_sync, m.stream));
-    for (int i = 1; i < n; ++i) {  // fork every other slab's stream into the capture
-      CK(cudaSetDevice(h->slabs[i].device));
-      CK(cudaStreamWaitEvent(h->slabs[i].stream, m.ev_sync, 0));
-    }
-    for (int64_t it = 0; it < iters; ++it) {
-      const int64_t tg = h->t + it;
-      const int nxt = (int)((tg + 1) & 1);
-      for (int i = 0; i < n; ++i) {
-        Slab &s = h->slabs[i];
-        CK(cudaSetDevice(s.device));
-        if (it > 0) {  // halos of this iteration were written by the neighbours' copies
-          if (s.has_top) CK(cudaStreamWaitEvent(s.stream, h->slabs[i - 1].ev_copy, 0));
-          if (s.has_bot) CK(cudaStreamWaitEvent(s.stream, h->slabs[i + 1].ev_copy, 0));
-        }
-        if (!nocomp) {
-          plans[i].P.t0 = tg;
-          CK(jbk::launch_sweep(plans[i].P, false, false, plans[i].grid, plans[i].smem, s.stream));
-        }
-      }
-      for (int i = 0; i < n; ++i) {
-        Slab &s = h->slabs[i];
-        CK(cudaSetDevice(s.device));
-        int rc = copy_edges(h, s, nxt, s.stream, true);
-        if (rc) {
-          cudaGraph_t g;
-          cudaStreamEndCapture(m.stream, &g);
-          return rc;
-        }
-        CK(cudaEventRecord(s.ev_copy, s.stream));
-      }
-    }
-    CK(cudaSetDevice(m.device));
-    for (int i = 1; i < n; ++i) CK(cudaStreamWaitEvent(m.stream, h->slabs[i].ev_copy, 0));  // join
-    cudaGraph_t graph;
-    CK(cudaStreamEndCapture(m.stream, &graph));
-    cudaError_t e = cudaGraphInstantiate(&h->graph_exec, graph, 0);
-    cudaGraphDestroy(graph);
-    CK(e);
-    h->graph_iters = iters;
-    h->graph_parity = parity;
-    h->graph_gen = h->plan_gen;
-  }
-  int rc = time_begin(h);
-  if (rc) return rc;
-  Slab &m = h->slabs[0];
-  CK(cudaSetDevice(m.device));
-  CK(cudaGraphLaunch(h->graph_exec, m.stream));
-  CK(cudaStreamSynchronize(m.stream));
-  return time_end(h, iters);
-}
-
-}  // namespace
-
-// ======================================================================== C ABI
 extern "C" {
-
 int jacobi_create(int64_t nx, int64_t ny, int64_t nz, int stencil, int ngpus, jacobi_t *out) {
   if (!out) return JACOBI_EINVAL;
   *out = nullptr;
@@ -1077,260 +623,7 @@ int jacobi_create_virtual(int64_t nx, int64_t ny, int64_t nz, int stencil, int n
   return JACOBI_OK;
 }
 
-int jacobi_create_rank(int64_t nx, int64_t ny, int64_t nz, int stencil, int world_size, int rank,
-                       int device, jacobi_t *out) {
-  if (!out) return JACOBI_EINVAL;
-  *out = nullptr;
-  if (rank < 0 || rank >= world_size) return JACOBI_EINVAL;
-  int rc = validate(nx, ny, nz, stencil, world_size);
-  if (rc) return rc;
-  int ndev = 0;
-  if (cudaGetDeviceCount(&ndev) != cudaSuccess || device < 0 || device >= ndev) return JACOBI_ENODEV;
-  jacobi_ctx *h = new_ctx(nx, ny, nz, stencil, world_size);
-  h->kind = KIND_DIST;
-  h->rank = rank;
-  h->slabs.resize(1);
-  Slab &s = h->slabs[0];
-  s.device = device;
-  s.id = rank;
-  jbplan::decompose(h->n_out, world_size, rank, &s.start, &s.chunk);
-  rc = alloc_slab(h, s);
-  if (rc) { jacobi_destroy(h); return rc; }
-  s.has_top = rank > 0;
-  s.has_bot = rank < world_size - 1;
-  h->peers_ready = world_size == 1;
-  *out = h;
-  return JACOBI_OK;
-}
 
-int jacobi_set_allocator(jacobi_alloc_fn alloc, jacobi_free_fn free_fn, void *user) {
-  if ((alloc == nullptr) != (free_fn == nullptr)) return JACOBI_EINVAL;
-  g_alloc.alloc = alloc;
-  g_alloc.free = free_fn;
-  g_alloc.user = user;
-  return JACOBI_OK;
-}
-
-int jacobi_slab_bytes(int64_t nx, int64_t ny, int64_t nz, int stencil, int nslabs, int slab, int64_t *bytes) {
-  if (!bytes || slab < 0 || slab >= nslabs) return JACOBI_EINVAL;
-  int rc = validate(nx, ny, nz, stencil, nslabs);
-  if (rc) return rc;
-  JbGeom g;
-  if (jbplan::geometry(nx, ny, nz, stencil == 5 ? 2 : 3, 8, 1, JB_SMEM_DEFAULT, 0, &g)) return JACOBI_EINVAL;
-  int64_t start, chunk;
-  jbplan::decompose(stencil == 5 ? ny : nz, nslabs, slab, &start, &chunk);
-  *bytes = (chunk + 2) * g.plane_elems * (int64_t)sizeof(double);
-  return JACOBI_OK;
-}
-
-int jacobi_ipc_handle_bytes(void) { return (int)sizeof(IpcBlob); }
-
-int jacobi_get_ipc_handle(jacobi_t h, void *out) {
-  if (!h || !out || h->kind != KIND_DIST) return JACOBI_EINVAL;
-  Slab &s = h->slabs[0];
-  IpcBlob b;
-  std::memset(&b, 0, sizeof(b));
-  b.magic = kIpcMagic;
-  b.rank = h->rank;
-  b.chunk = s.chunk;
-  b.plane_elems = h->geom.plane_elems;
-  CK(cudaDeviceGetAttribute(&b.sms, cudaDevAttrMultiProcessorCount, s.device));
-  CK(cudaSetDevice(s.device));
-  CK(cudaIpcGetMemHandle(&b.buf[0], s.buf[0]));
-  CK(cudaIpcGetMemHandle(&b.buf[1], s.buf[1]));
-  CK(cudaIpcGetMemHandle(&b.ctrl, s.ctrl));
-  b.off[0] = alloc_offset(s.buf[0]);
-  b.off[1] = alloc_offset(s.buf[1]);
-  b.off[2] = alloc_offset(s.ctrl);
-  std::memcpy(out, &b, sizeof(b));
-  return JACOBI_OK;
-}
-
-int jacobi_open_peers(jacobi_t h, const void *top_blob, const void *bottom_blob) {
-  if (!h || h->kind != KIND_DIST) return JACOBI_EINVAL;
-  Slab &s = h->slabs[0];
-  if ((s.has_top && !top_blob) || (s.has_bot && !bottom_blob)) return JACOBI_EINVAL;
-  CK(cudaSetDevice(s.device));
-  const int64_t pe = h->geom.plane_elems;
-  auto open = [&](const void *blob, int expect_rank, double **bufs, JbCtrl **ctrl, int64_t *chunk) -> int {
-    IpcBlob b;
-    std::memcpy(&b, blob, sizeof(b));
-    int sms = 0;
-    CK(cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, s.device));
-    if (b.magic != kIpcMagic || b.rank != expect_rank || b.plane_elems != pe || b.sms != sms) return JACOBI_EINVAL;
-    for (int p = 0; p < 2; ++p) {
-      void *ptr = nullptr;
-      CK(cudaIpcOpenMemHandle(&ptr, b.buf[p], cudaIpcMemLazyEnablePeerAccess));
-      s.ipc_opened.push_back(ptr);
-      bufs[p] = reinterpret_cast<double *>(static_cast<char *>(ptr) + b.off[p]);
-    }
-    void *c = nullptr;
-    CK(cudaIpcOpenMemHandle(&c, b.ctrl, cudaIpcMemLazyEnablePeerAccess));
-    s.ipc_opened.push_back(c);
-    *ctrl = reinterpret_cast<JbCtrl *>(static_cast<char *>(c) + b.off[2]);
-    *chunk = b.chunk;
-    return JACOBI_OK;
-  };
-  if (s.has_top) {
-    double *bufs[2];
-    JbCtrl *ctrl;
-    int64_t chunk;
-    int rc = open(top_blob, h->rank - 1, bufs, &ctrl, &chunk);
-    if (rc) return rc;
-    for (int p = 0; p < 2; ++p) s.peer_top[p] = bufs[p] + (chunk + 1) * pe;
-    s.flag_out_top = &ctrl->flag_in[1][0];
-  }
-  if (s.has_bot) {
-    double *bufs[2];
-    JbCtrl *ctrl;
-    int64_t chunk;
-    int rc = open(bottom_blob, h->rank + 1, bufs, &ctrl, &chunk);
-    if (rc) return rc;
-    for (int p = 0; p < 2; ++p) s.peer_bot[p] = bufs[p];
-    s.flag_out_bot = &ctrl->flag_in[0][0];
-  }
-  h->peers_ready = true;
-  return JACOBI_OK;
-}
-
-int jacobi_open_ranks(jacobi_t h, const void *blobs, int world) {
-  if (!h || !blobs || h->kind != KIND_DIST || world != h->total) return JACOBI_EINVAL;
-  const size_t B = sizeof(IpcBlob);
-  const char *base = static_cast<const char *>(blobs);
-  const int r = h->rank;
-  int rc = jacobi_open_peers(h, r > 0 ? base + (r - 1) * B : nullptr, r < world - 1 ? base + (r + 1) * B : nullptr);
-  if (rc) return rc;
-  Slab &s = h->slabs[0];
-  CK(cudaSetDevice(s.device));
-  h->all_ctrl.assign(world, nullptr);
-  for (int g = 0; g < world; ++g) {
-    if (g == r) {
-      h->all_ctrl[g] = s.ctrl;
-      continue;
-    }
-    IpcBlob b;
-    std::memcpy(&b, base + g * B, B);
-    if (b.magic != kIpcMagic || b.rank != g) return JACOBI_EINVAL;
-    void *c = nullptr;
-    CK(cudaIpcOpenMemHandle(&c, b.ctrl, cudaIpcMemLazyEnablePeerAccess));
-    s.ipc_opened.push_back(c);
-    h->all_ctrl[g] = reinterpret_cast<JbCtrl *>(static_cast<char *>(c) + b.off[2]);
-  }
-  return JACOBI_OK;
-}
-
-#ifdef JB_NVSHMEM
-namespace {
-bool g_shm_init = false;
-void *shm_alloc(size_t bytes, int, void *) { return nvshmem_malloc(bytes); }
-void shm_free(void *p, int, void *) { nvshmem_free(p); }
-}  // namespace
-
-int jacobi_nvshmem_uid_bytes(void) { return (int)sizeof(nvshmemx_uniqueid_t); }
-
-int jacobi_nvshmem_uid(void *out) {
-  if (!out) return JACOBI_EINVAL;
-  nvshmemx_uniqueid_t uid = NVSHMEMX_UNIQUEID_INITIALIZER;
-  if (nvshmemx_get_uniqueid(&uid) != 0) return JACOBI_ECUDA;
-  std::memcpy(out, &uid, sizeof(uid));
-  return JACOBI_OK;
-}
-
-// N3: one PE per process, bootstrapped from a unique id (created by rank 0, shared by the caller),
-// slab buffers and control blocks on the NVSHMEM symmetric heap; halos are delivered with
-// nvshmemx_putmem_signal_nbi_warp by the boundary CTAs of the CPU-Free kernel.
-// Collective: every rank creates (and later destroys) its handle in the same order.
-int jacobi_create_nvshmem(int64_t nx, int64_t ny, int64_t nz, int stencil, const void *uid, int world_size,
-                          int rank, int device, jacobi_t *out) {
-  if (!out || !uid || rank < 0 || rank >= world_size || world_size > 32) return JACOBI_EINVAL;
-  *out = nullptr;
-  int rc = validate(nx, ny, nz, stencil, world_size);
-  if (rc) return rc;
-  CK(cudaSetDevice(device));
-  if (!g_shm_init) {
-    if (!getenv("NVSHMEM_SYMMETRIC_SIZE")) {  // room for two field buffers + control block
-      JbGeom g;
-      jbplan::geometry(nx, ny, nz, stencil == 5 ? 2 : 3, 8, 1, JB_SMEM_DEFAULT, 0, &g);
-      int64_t st, chunk_max;
-      jbplan::decompose(stencil == 5 ? ny : nz, world_size, 0, &st, &chunk_max);
-      const int64_t need = 2 * (chunk_max + 2) * g.plane_elems * 8 + (64 << 20);
-      const int64_t sz = std::max<int64_t>(need + need / 4, (int64_t)1 << 30);
-      setenv("NVSHMEM_SYMMETRIC_SIZE", std::to_string(sz).c_str(), 0);
-    }
-    nvshmemx_uniqueid_t id;
-    std::memcpy(&id, uid, sizeof(id));
-    nvshmemx_init_attr_t attr = NVSHMEMX_INIT_ATTR_INITIALIZER;
-    nvshmemx_set_attr_uniqueid_args(rank, world_size, &id, &attr);
-    if (nvshmemx_init_attr(NVSHMEMX_INIT_WITH_UNIQUEID, &attr) != 0) return JACOBI_ECUDA;
-    g_shm_init = true;
-  }
-  if (nvshmem_my_pe() != rank || nvshmem_n_pes() != world_size) return JACOBI_ESTATE;
-  jacobi_ctx *h = new_ctx(nx, ny, nz, stencil, world_size);
-  h->kind = KIND_SHMEM;
-  h->rank = rank;
-  h->alloc.alloc = shm_alloc;
-  h->alloc.free = shm_free;
-  h->alloc.user = nullptr;
-  h->slabs.resize(1);
-  Slab &s = h->slabs[0];
-  s.device = device;
-  s.id = rank;
-  jbplan::decompose(h->n_out, world_size, rank, &s.start, &s.chunk);
-  rc = alloc_slab(h, s);
-  if (rc) { delete h; return rc; }
-  const int64_t pe = h->geom.plane_elems;
-  s.has_top = rank > 0;
-  s.has_bot = rank < world_size - 1;
-  if (s.has_top) {  // symmetric addresses of the neighbour's bottom halo plane and flag slots
-    int64_t st, ct;
-    jbplan::decompose(h->n_out, world_size, rank - 1, &st, &ct);
-    for (int p = 0; p < 2; ++p) s.peer_top[p] = s.buf[p] + (ct + 1) * pe;
-    s.flag_out_top = &s.ctrl->flag_in[1][0];
-    s.shm_pe_top = rank - 1;
-  }
-  if (s.has_bot) {
-    for (int p = 0; p < 2; ++p) s.peer_bot[p] = s.buf[p];
-    s.flag_out_bot = &s.ctrl->flag_in[0][0];
-    s.shm_pe_bot = rank + 1;
-  }
-  h->all_ctrl.assign(world_size, nullptr);  // raw NVLink pointers for the norm all-reduce (N4)
-  for (int g = 0; g < world_size; ++g)
-    h->all_ctrl[g] = static_cast<JbCtrl *>(nvshmem_ptr(s.ctrl, g));
-  for (int g = 0; g < world_size; ++g)
-    if (!h->all_ctrl[g]) h->all_ctrl.clear();
-  h->peers_ready = true;
-  nvshmem_barrier_all();
-  *out = h;
-  return JACOBI_OK;
-}
-
-int jacobi_nvshmem_finalize(void) {
-  if (g_shm_init) nvshmem_finalize();
-  g_shm_init = false;
-  return JACOBI_OK;
-}
-#endif
-
-int jacobi_nccl_unique_id(void *out128) {
-  if (!out128) return JACOBI_EINVAL;
-  if (!g_nccl.load()) return JACOBI_ENCCL;
-  ncclUniqueId id;
-  if (g_nccl.GetUniqueId(&id) != ncclSuccess) return JACOBI_ENCCL;
-  std::memcpy(out128, &id, sizeof(id));
-  return JACOBI_OK;
-}
-
-int jacobi_nccl_init(jacobi_t h, const void *id128) {
-  if (!h || !id128 || h->kind != KIND_DIST) return JACOBI_EINVAL;
-  if (!g_nccl.load()) return JACOBI_ENCCL;
-  Slab &s = h->slabs[0];
-  CK(cudaSetDevice(s.device));
-  ncclUniqueId id;
-  std::memcpy(&id, id128, sizeof(id));
-  if (g_nccl.CommInitRank(&s.comm, h->total, id, h->rank) != ncclSuccess) return JACOBI_ENCCL;
-  h->nccl_ready = true;
-  return JACOBI_OK;
-}
 
 int jacobi_run(jacobi_t h, int64_t iters) {
   if (!h || iters < 0) return JACOBI_EINVAL;
@@ -1517,5 +810,4 @@ int jacobi_destroy(jacobi_t h) {
   delete h;
   return JACOBI_OK;
 }
-
 }  // extern "C"
