@@ -277,19 +277,30 @@ def main():
     dev_ms = max_over_ranks(dev_ms_local)
     value = cells * iters * args.steps / (dev_ms / 1e3) / 1e9
 
-    # ---- roofline of the dominant (only) kernel: the persistent sweep
+    # ---- roofline of the dominant kernel.  Per cell-update it moves 16 B (read once + write
+    #      once) when it runs one iteration per pass over HBM, 16/K B when the
+    #      temporally blocked kernel runs K iterations per pass.
     peak, peak_kind = measured_hbm()
     launch_ms = dev_ms_local / args.steps
-    alg_bytes = 16 * local_cells * iters  # read once + write once per cell-update
+    tb_iters = jb.jacobi_get_param(j.h, "last_tblock")
+    tb_k = 2
+    alg_bytes = local_cells * (16 * (iters - tb_iters) + 16 // tb_k * tb_iters)
     achieved = alg_bytes / (launch_ms / 1e3) / 1e9
-    traffic, _ = ncu_traffic(args.config, iters)
     dimk = 2 if shape[0] == 1 else 3
-    kname = (f"jb_resident<{dimk},*> (persistent CPU-Free kernel, on-chip resident)"
-             if jb.jacobi_get_param(j.h, "last_resident") else
-             f"jb_sweep<{dimk},false,true,false> (persistent CPU-Free kernel, streaming)")
+    if tb_iters:
+        kname = f"jb_tblock2d<8,*> (persistent CPU-Free kernel, {tb_k} iterations per HBM pass)"
+        kkind = "tblock"
+    elif jb.jacobi_get_param(j.h, "last_resident"):
+        kname = f"jb_resident<{dimk},*> (persistent CPU-Free kernel, on-chip resident)"
+        kkind = "resident"
+    else:
+        kname = f"jb_sweep<{dimk},false,true,false> (persistent CPU-Free kernel, streaming)"
+        kkind = "streaming"
+    traffic, _ = ncu_traffic(args.config + ("_tblock" if tb_iters else ""), iters)
     roofline = {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
                 "frac": achieved / peak, "traffic": traffic, "peak_kind": peak_kind,
-                "kernel": kname, "alg_bytes_per_launch": alg_bytes}
+                "kernel": kname, "alg_bytes_per_launch": alg_bytes,
+                "alg_bytes_per_cell_update": alg_bytes / (local_cells * iters)}
 
     line = {
         "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
@@ -301,8 +312,8 @@ def main():
                    "parallelism": f"slab{world}" + (f" (virtual {args.virtual} slabs)" if args.virtual else ""),
                    "l2": ("inputs larger than L2" if 8 * cells > L2_BYTES else "L2-resident (latency config)"),
                    "tile": {k: desc[k] for k in ("tile_x", "tile_y", "stages", "ctas", "n_top", "n_bot", "k_planes")},
-                   "kernel": "resident" if jb.jacobi_get_param(j.h, "last_resident") else "streaming"},
-        "gpu_launches": args.steps * world,
+                   "kernel": kkind},
+        "gpu_launches": args.steps * world * (2 if 0 < tb_iters < iters else 1),
         "wall_ms_per_step": 1e3 * t_wall / args.steps,
         "ms_per_iter": dev_ms / args.steps / iters,
         "roofline": roofline,
@@ -332,6 +343,23 @@ def main():
         except Exception as e:  # never fail the bench line for a context number
             line["roofline"]["box_copy_gbs"] = None
             print(f"[bench] box copy measurement failed: {e}", file=sys.stderr)
+
+        # ---- the per-iteration CPU-Free kernel (one iteration per HBM pass, the paper's Listing
+        #      4.1 structure) on the same workload, for comparison with the time-blocked one
+        if tb_iters:
+            j.set_param("tblock", 0)
+            j.run(iters)
+            ms1 = []
+            for _ in range(args.steps):
+                j.run(iters)
+                ms1.append(j.last_time_ms())
+            j.set_param("tblock", -1)
+            ms1 = max_over_ranks(sum(ms1))
+            v1 = cells * iters * args.steps / (ms1 / 1e3) / 1e9
+            a1 = 16 * local_cells * iters / (ms1 / args.steps / 1e3) / 1e9
+            line["per_iteration_kernel"] = {"value": v1, "unit": UNIT, "kernel": "jb_sweep (streaming)",
+                                            "achieved_gbs": a1, "frac": a1 / peak,
+                                            "alg_bytes_per_cell_update": 16}
 
         # ---- CPU-controlled baselines (per-iteration launch + copy/NCCL + host sync), short run
         base = {}

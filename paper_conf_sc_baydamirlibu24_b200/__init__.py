@@ -376,6 +376,9 @@ class Jacobi:
         jacobi_set_param(self.h, name, value)
         return self
 
+    def get_param(self, name: str) -> int:
+        return jacobi_get_param(self.h, name)
+
     def scatter(self, field: np.ndarray) -> "Jacobi":
         a = np.ascontiguousarray(field, dtype=np.float64)
         jacobi_scatter(self.h, a.reshape(-1), self.n)

@@ -195,7 +195,7 @@ int plan_launch(jacobi_ctx *h, const std::vector<int> &idx, LaunchKind lk, bool 
     return JACOBI_EINVAL;
   const int nslab = (int)idx.size();
   int total_ctas = launch_ctas(h, sms);  // one CTA per SM (occupancy verified below)
-  if (grid_override > 0) total_ctas = std::min(grid_override, sms);
+  if (grid_override > 0) total_ctas = std::min(grid_override, lk == LK_PERSIST ? 2 * sms : sms);
   const int per = total_ctas / nslab;
   if (h->dim == 3 && h->tile_y <= 0) {
     // Pick ty so that the tile count divides the CTA count well: a whole number of plane blocks
@@ -445,7 +445,7 @@ int setup_norm(jacobi_ctx *h, LaunchPlan &L) {
   return JACOBI_OK;
 }
 
-int run_cpufree(jacobi_ctx *h, int64_t iters) {
+int run_cpufree_k1(jacobi_ctx *h, int64_t iters) {
   const bool nocomp = h->flags & JACOBI_FLAG_NO_COMPUTE;
   const bool norm = !nocomp && h->norm_every > 0;
   auto groups = launch_groups(h);
@@ -551,6 +551,95 @@ int run_cpufree(jacobi_ctx *h, int64_t iters) {
     if (done >= h->norm_every) h->last_norm = r;
   }
   h->t += done;
+  return JACOBI_OK;
+}
+
+// Temporally blocked CPU-Free launch (tblock.cu) of `iters` (a multiple of
+// 2K) iterations on a single slab without neighbours: the guided dynamic schedule of
+// plan_launch, with the ring shortened to leave room for the level-1 row ring.
+int run_tblock(jacobi_ctx *h, int64_t iters) {
+  LaunchPlan L;
+  const int64_t sched = h->schedule, minb = h->min_block;
+  h->schedule = 2;
+  h->min_block = std::max<int64_t>(1, h->tb_min_block);
+  int sms = 0;
+  CK(cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, h->slabs[0].device));
+  const int per_sm = h->tb_ctas >= 2 ? 2 : 1;
+  int rc = plan_launch(h, {0}, LK_PERSIST, false, L, per_sm == 2 ? launch_ctas(h, sms) * 2 : 0);
+  h->schedule = sched;
+  h->min_block = minb;
+  if (rc) return rc;
+  JbGeom &g = L.P.g;
+  int smem_optin = 0;
+  CK(cudaDeviceGetAttribute(&smem_optin, cudaDevAttrMaxSharedMemoryPerBlockOptin, L.device));
+  smem_optin = std::min(smem_optin, JB_SMEM_DEFAULT) - 1024;
+  if (per_sm == 2) {  // two CTAs share the SM's shared memory (1 KB reserved per CTA + static)
+    int smem_sm = 0;
+    CK(cudaDeviceGetAttribute(&smem_sm, cudaDevAttrMaxSharedMemoryPerMultiprocessor, L.device));
+    smem_optin = std::min(smem_optin, smem_sm / 2 - 1024 - 512);
+  }
+  while (g.stages > 3 && jbk::tblock_smem(g) > (size_t)smem_optin) --g.stages;
+  if (jbk::tblock_smem(g) > (size_t)smem_optin) return JACOBI_EINVAL;
+  L.smem = jbk::tblock_smem(g);
+  int occ = 0;
+  CK(jbk::prepare_tblock(g, per_sm, L.smem, &occ));
+  if (occ < per_sm) {
+    if (getenv("JACOBI_DEBUG")) fprintf(stderr, "[jacobi] tblock: occupancy %d < %d (smem %zu)\n", occ, per_sm, L.smem);
+    return JACOBI_ENOCOOP;
+  }
+  Slab &s = h->slabs[0];
+  s.smem = L.smem;
+  L.P.t0 = h->t;
+  L.P.iters = iters;
+  CK(reset_run_counters(s, L.stream));
+  CK(cudaEventRecord(s.ev0, L.stream));
+  CK(jbk::launch_tblock(L.P, per_sm, L.grid, L.smem, L.stream));
+  CK(cudaEventRecord(s.ev1, L.stream));
+  CK(cudaEventSynchronize(s.ev1));
+  float ms = 0;
+  CK(cudaEventElapsedTime(&ms, s.ev0, s.ev1));
+  s.last_ms = ms;
+  h->last_ms_max = ms;
+  rc = read_status(s);
+  if (rc) return rc;
+  h->t += iters;
+  return JACOBI_OK;
+}
+
+// CPU-Free run: the temporally blocked kernel for as many whole pairs of time blocks as fit when
+// the run is eligible (one slab without neighbours, 2D, compute, no norm, not on-chip resident),
+// the per-iteration kernels (streaming / resident) for the rest.  Device times add up.
+int run_cpufree(jacobi_ctx *h, int64_t iters) {
+  h->last_tblock = 0;
+  h->last_resident = 0;
+  const bool nocomp = h->flags & JACOBI_FLAG_NO_COMPUTE;
+  const bool eligible = h->tblock != 0 && !nocomp && h->norm_every <= 0 && h->dim == 2 && h->total == 1 &&
+                        h->slabs.size() == 1 && (h->kind == KIND_SINGLE || h->kind == KIND_DIST);
+  if (h->tblock == 1 && !eligible) return JACOBI_EINVAL;
+  int64_t tb_iters = 0;
+  if (eligible) {
+    const int64_t step = 2 * jbk::tblock_k();  // even block count: the result stays in buf[t & 1]
+    tb_iters = iters / step * step;
+    if (h->tblock < 0 && h->resident != 0) {
+      // auto: slabs that fit on chip run the resident kernel (faster for those small grids)
+      LaunchPlan R;
+      if (plan_resident(h, {0}, R) == JACOBI_OK) tb_iters = 0;
+    }
+  }
+  double ms = 0;
+  if (tb_iters > 0) {
+    int rc = run_tblock(h, tb_iters);
+    if (rc) return rc;
+    ms = h->last_ms_max;
+    h->last_tblock = tb_iters;
+  }
+  if (iters - tb_iters > 0) {
+    int rc = run_cpufree_k1(h, iters - tb_iters);
+    if (rc) return rc;
+    ms += h->last_ms_max;
+  }
+  h->last_ms_max = ms;
+  for (auto &s : h->slabs) s.last_ms = ms;
   return JACOBI_OK;
 }
 }  // namespace jbrt
@@ -667,12 +756,16 @@ static int64_t *param_slot(jacobi_t h, const char *name) {
   if (!std::strcmp(name, "norm_every")) return &h->norm_every;
   if (!std::strcmp(name, "l2hint")) return &h->l2hint;
   if (!std::strcmp(name, "last_resident")) return &h->last_resident;
+  if (!std::strcmp(name, "tblock")) return &h->tblock;
+  if (!std::strcmp(name, "tb_min_block")) return &h->tb_min_block;
+  if (!std::strcmp(name, "tb_ctas")) return &h->tb_ctas;
+  if (!std::strcmp(name, "last_tblock")) return &h->last_tblock;
   return nullptr;
 }
 
 int jacobi_set_param(jacobi_t h, const char *name, int64_t value) {
   if (!h || !name) return JACOBI_EINVAL;
-  if (!std::strcmp(name, "last_resident")) return JACOBI_EINVAL;  // read-only
+  if (!std::strcmp(name, "last_resident") || !std::strcmp(name, "last_tblock")) return JACOBI_EINVAL;  // read-only
   int64_t *p = param_slot(h, name);
   if (!p) return JACOBI_EINVAL;
   if (!std::strcmp(name, "timeout_ms")) value = value < 0 ? 20000 : value;

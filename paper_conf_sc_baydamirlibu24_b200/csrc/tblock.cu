@@ -1,0 +1,358 @@
+// tblock.cu — temporally blocked CPU-Free sweep: K = 2 Jacobi iterations per pass
+// over HBM, for a slab without neighbours (P = 1, both outer halos are the Dirichlet planes).
+//
+// The method is unchanged — every cell is updated every iteration with the oracle's fp64 order
+// (-fmad=false), each iteration reads only the previous time step, Dirichlet cells are
+// never written — only the schedule of the updates differs: a work item (plane block
+// [a, b] x x-strip) streams the time-t planes a-2 .. b+2 of its strip from HBM through the same
+// TMA bulk-copy ring as jb_sweep, computes time t+1 for planes a-1 .. b+1 in registers (x
+// neighbours by warp shuffles), and from those time t+2 for planes a .. b, columns
+// x0 .. x0+tx-1, which it stores into the other buffer.  The intermediate time level never
+// touches HBM, so the algorithmic traffic per cell-update is 16 B / K = 8 B instead of 16 B
+// (overlapped tiling: the t+1 values of the 2 extra planes of each item and of one extra column
+// at each end of each warp's segment are recomputed, < 2 % extra arithmetic at C2).
+// The persistent structure of the paper is kept: one cooperative launch for the whole run, a
+// device-side grid barrier between time blocks, no host involvement.
+//
+// Buffers: time block j of a launch reads buf[(t0 + j) & 1] and writes buf[(t0 + j + 1) & 1]
+// (out of place — neighbouring strips still read the time-t columns of this strip); the host
+// runs an even number of blocks, so the result lands in buf[(t0 + 2 nb) & 1] as in every other
+// path (R10).
+#include "device_common.cuh"
+
+namespace {
+
+constexpr int TB_K = 2;  // iterations per time block
+
+enum { TB_WORK = 0, TB_END = 1 };
+struct TbDesc {
+  int32_t kind;
+  int32_t unit;
+  int64_t a, b;  // output planes a..b of this item (time t+2)
+  int64_t pad;
+};
+
+// Position `off` stages after p in the ring.
+__device__ __forceinline__ RingPos ring_add(RingPos p, uint32_t off, uint32_t S) {
+  const uint32_t s = p.slot + off;
+  const uint32_t wraps = s / S;
+  return RingPos{s - wraps * S, p.phase ^ (wraps & 1u)};
+}
+
+// Per-warp geometry of one item.
+struct TbSeg {
+  int j0;                // stage index of pair i = 0 (stage s <-> column x0 - 2 + s)
+  unsigned in_tile, ok, full, first, last;
+  int sx;                // stage index of this lane's extra level-1 cell (segment ends)
+  bool ex_in;            // that extra cell is an interior column
+  bool fast;             // every pair of the segment is interior: no per-pair masks
+};
+
+// Level 1 (t+1) of this lane's pairs and extra cell on the row whose level-0 stages are
+// sm (row-1), sc (row), sn (row+1); rows outside 1..C keep level 0 (rowin = false).
+template <int PPT, bool FAST>
+__device__ __forceinline__ void tb_level1(const TbSeg &L, const double *sm, const double *sc, const double *sn,
+                                          bool rowin, double2 *V, double &ex) {
+#pragma unroll
+  for (int i = 0; i < PPT; ++i) {
+    const int j = L.j0 + 64 * i;
+    if (FAST || (L.in_tile >> i & 1u)) {
+      const double2 S0 = lds2(sm + j), C0 = lds2(sc + j), N0 = lds2(sn + j);
+      const double W = sc[j - 1], E = sc[j + 2];
+      // oracle order: ((x+1) + (x-1)) + (y+1) + (y-1), then * 0.25
+      const double l0 = 0.25 * (((C0.y + W) + N0.x) + S0.x);
+      const double l1 = 0.25 * (((E + C0.x) + N0.y) + S0.y);
+      V[i].x = (rowin && (FAST || (L.ok >> i & 1u))) ? l0 : C0.x;  // Dirichlet cells keep level 0
+      V[i].y = (rowin && (FAST || (L.full >> i & 1u))) ? l1 : C0.y;
+    }
+  }
+  const int x = L.sx;
+  const double e = 0.25 * (((sc[x + 1] + sc[x - 1]) + sn[x]) + sm[x]);
+  ex = (rowin && L.ex_in) ? e : sc[x];
+}
+
+// Level 2 (t+2) of the middle level-1 row C1 (rows S1, C1, N1), stored at o.  x neighbours by
+// rotations: lane l gets lane l-1's .y (W) and lane l+1's .x (E); lane 0 / lane 31 take the
+// wrapped value of the previous / next pair, the segment's end pairs the extra cells.
+template <int PPT, bool FAST>
+__device__ __forceinline__ void tb_level2(const TbSeg &L, const double2 *S1, const double2 *C1, const double2 *N1,
+                                          double exl, double exr, int lane, double *o) {
+  double rw_prev = 0.0;
+  double re_next = __shfl_sync(0xffffffffu, C1[0].x, (lane + 1) & 31);
+#pragma unroll
+  for (int i = 0; i < PPT; ++i) {
+    const double rw = __shfl_sync(0xffffffffu, C1[i].y, (lane + 31) & 31);
+    const double re = re_next;
+    if (i + 1 < PPT) re_next = __shfl_sync(0xffffffffu, C1[i + 1].x, (lane + 1) & 31);
+    const double W = (L.first >> i & 1u) ? exl : (lane == 0 ? rw_prev : rw);
+    const double E = (L.last >> i & 1u) ? exr : (lane == 31 ? re_next : re);
+    const double o0 = 0.25 * (((C1[i].y + W) + N1[i].x) + S1[i].x);
+    const double o1 = 0.25 * (((E + C1[i].x) + N1[i].y) + S1[i].y);
+    if (FAST) *reinterpret_cast<double2 *>(o + 64 * i) = make_double2(o0, o1);
+    else if (L.ok >> i & 1u) store_pair(o + 64 * i, o0, o1, L.full >> i & 1u);
+    rw_prev = rw;
+  }
+}
+
+// One item: level-0 rows r0..r1 of strip `unit` sit in consecutive ring stages from q.
+//   level 1 (t+1): rows q1 = a-1 .. b+1 (Dirichlet rows / columns keep level 0)
+//   level 2 (t+2): rows a .. b, columns x0 .. x0+tx-1  -> out
+// Warp w owns the contiguous cell pairs kk = w*32*PPT + i*32 + lane (i < PPT): conflict-free
+// 16-byte stage loads, coalesced 16-byte stores.  Level-1 x neighbours inside the segment come
+// from neighbouring lanes by shuffles; at the segment's ends the warp computes one extra
+// level-1 cell from the level-0 stage (overlapped by one cell per side), so warps never wait
+// for each other: no CTA barrier, each warp marches at its own pace.
+template <int PPT, bool FAST>
+__device__ __forceinline__ void tb2_march(const TbSeg &L, const Ring &R, RingPos q, int64_t a, int64_t b,
+                                          int64_t C, int64_t r0, int64_t r1, double *dst, int64_t pe, int lane) {
+  double2 S1[PPT], C1[PPT], N1[PPT];
+  double exl_c, exl_n, exr_c, exr_n, ex;
+  // Level-1 row q1 reads level-0 rows max(q1-1, r0), q1, min(q1+1, r1): ring positions pm, pc,
+  // pn, advanced by one stage per row (row a-2 exists iff r0 = a-2).
+  RingPos pc = ring_add(q, (uint32_t)(a - 1 - r0), R.S);
+  RingPos pm = a - 2 >= r0 ? q : pc;
+  R.wait_full(pm);
+  R.wait_full(pc);
+  auto row = [&](int64_t q1, double2 *out) {
+    RingPos pn = pc;
+    if (q1 + 1 <= r1) pn.advance(R.S);
+    R.wait_full(pn);
+    tb_level1<PPT, FAST>(L, R.stage(pm), R.stage(pc), R.stage(pn), q1 >= 1 && q1 <= C, out, ex);
+    if (q1 - 1 >= r0) R.release(pm, lane);  // row q1-1 is no longer needed
+    pm = pc;
+    pc = pn;
+  };
+  // prologue: level-1 rows a-1 and a; extras: lane 0 holds the left one, lane 1 the right one
+  row(a - 1, C1);
+  exl_c = __shfl_sync(0xffffffffu, ex, 0);
+  exr_c = __shfl_sync(0xffffffffu, ex, 1);
+  row(a, N1);
+  exl_n = __shfl_sync(0xffffffffu, ex, 0);
+  exr_n = __shfl_sync(0xffffffffu, ex, 1);
+  double *o = dst + a * pe;
+  for (int64_t q1 = a + 1; q1 <= b + 1; ++q1) {
+#pragma unroll
+    for (int i = 0; i < PPT; ++i) S1[i] = C1[i];
+#pragma unroll
+    for (int i = 0; i < PPT; ++i) C1[i] = N1[i];
+    exl_c = exl_n;
+    exr_c = exr_n;
+    row(q1, N1);
+    exl_n = __shfl_sync(0xffffffffu, ex, 0);
+    exr_n = __shfl_sync(0xffffffffu, ex, 1);
+    tb_level2<PPT, FAST>(L, S1, C1, N1, exl_c, exr_c, lane, o);
+    o += pe;
+  }
+  // rows b+1 .. r1 were not released by the march
+  RingPos pr = ring_add(q, (uint32_t)(b + 1 - r0), R.S);
+  for (int64_t p = b + 1; p <= r1; ++p) {
+    R.release(pr, lane);
+    pr.advance(R.S);
+  }
+}
+
+template <int PPT>
+__device__ __forceinline__ void tb2_item(const JbGeom &g, const Ring &R, RingPos &q, int unit, int64_t a,
+                                         int64_t b, int64_t C, double *out, int warp, int lane) {
+  const int64_t x0 = 1 + (int64_t)unit * g.tx;
+  const int vx = (int)min((int64_t)g.tx, g.nx - 1 - x0);  // interior columns of this strip
+  const int txp = g.tx >> 1;
+  const int seg_b = warp * 32 * PPT;             // first pair of this warp's segment
+  const int seg_e = min(seg_b + 32 * PPT, txp);  // one past its last pair
+  const int64_t r0 = max(a - 2, (int64_t)0), r1 = min(b + 2, C + 1);
+  const RingPos q0 = q;
+  q = ring_add(q, (uint32_t)(r1 - r0 + 1), R.S);
+  if (seg_b >= seg_e) {  // no pairs in this strip for this warp: only return the stages
+    for (int64_t p = r0; p <= r1; ++p) {
+      const RingPos pp = ring_add(q0, (uint32_t)(p - r0), R.S);
+      R.wait_full(pp);
+      R.release(pp, lane);
+    }
+    return;
+  }
+  TbSeg L;
+  L.j0 = 2 + 2 * (seg_b + lane);
+  L.in_tile = L.ok = L.full = L.first = L.last = 0;
+#pragma unroll
+  for (int i = 0; i < PPT; ++i) {
+    const int kk = seg_b + i * 32 + lane;
+    L.in_tile |= (kk < seg_e ? 1u : 0u) << i;
+    L.ok |= (kk < seg_e && 2 * kk < vx ? 1u : 0u) << i;
+    L.full |= (kk < seg_e && 2 * kk + 1 < vx ? 1u : 0u) << i;
+    L.first |= (kk == seg_b ? 1u : 0u) << i;
+    L.last |= (kk == seg_e - 1 ? 1u : 0u) << i;
+  }
+  // extra level-1 cells: lane 1 computes the right one (column x0 + 2 seg_e), every other lane
+  // the left one (x0 + 2 seg_b - 1); level 2 takes them from lanes 0 and 1.
+  L.sx = lane == 1 ? 2 * seg_e + 2 : 2 * seg_b + 1;
+  const int64_t cx = x0 - 2 + L.sx;
+  L.ex_in = cx >= 1 && cx <= g.nx - 2;
+  const bool fast = seg_e - seg_b == 32 * PPT && 2 * seg_e <= vx;
+  double *dst = out + 3 + x0 + 2 * (seg_b + lane);
+  if (fast) tb2_march<PPT, true>(L, R, q0, a, b, C, r0, r1, dst, g.plane_elems, lane);
+  else tb2_march<PPT, false>(L, R, q0, a, b, C, r0, r1, dst, g.plane_elems, lane);
+}
+
+template <int NCW, int PPT>
+__device__ __forceinline__ void tb_body(const JbParams &P) {
+  extern __shared__ __align__(128) unsigned char smem[];
+  __shared__ int s_abort;
+  const JbGeom &g = P.g;
+  const JbSlab &SL = P.s[0];
+  Ring R;
+  R.S = (uint32_t)g.stages;
+  R.stage_doubles = g.stage_doubles;
+  R.full = reinterpret_cast<uint64_t *>(smem);
+  R.empty = R.full + R.S;
+  uint64_t *qfull = R.empty + R.S;
+  uint64_t *qempty = qfull + JB_RQ;
+  TbDesc *desc = reinterpret_cast<TbDesc *>(qempty + JB_RQ);
+  const uint32_t hdr = 2 * R.S * 8 + 2 * JB_RQ * 8 + JB_RQ * (uint32_t)sizeof(TbDesc);
+  R.stages = reinterpret_cast<double *>(smem + ((hdr + 127) & ~127u));
+
+  const int c = (int)blockIdx.x;
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const bool producer = warp == NCW;
+  if (threadIdx.x == 0) {
+    for (uint32_t i = 0; i < R.S; ++i) {
+      mbar_init(&R.full[i], 1);
+      mbar_init(&R.empty[i], NCW);
+    }
+    for (int i = 0; i < JB_RQ; ++i) {
+      mbar_init(&qfull[i], 1);
+      mbar_init(&qempty[i], NCW);
+    }
+    fence_mbar_init();
+    s_abort = 0;
+  }
+  __syncthreads();
+
+  const int64_t C = SL.chunk;
+  const int64_t nblocks = P.iters / TB_K;
+  RingPos q = {0u, 0u}, rq = {0u, 0u};
+  for (int64_t j = 0; j < nblocks; ++j) {
+    const double *cur = SL.buf[(P.t0 + j) & 1];
+    double *nxt = SL.buf[(P.t0 + j + 1) & 1];
+    if (producer) {
+      fence_proxy_async_global();
+      if (lane == 0 && c == 0) SL.work_ctr[(j + 1) & 1] = 0u;  // idle since block j-1
+      // Guided self-scheduling over (plane block, strip) items, as jb_sweep.
+      unsigned int *ctr = SL.work_ctr + (j & 1);
+      int64_t item = c < SL.dyn_first ? c : -1;
+      unsigned int claim = 0;
+      if (item < 0) {
+        if (lane == 0) claim = atomicAdd(ctr, 1u);
+        item = SL.dyn_first + (int64_t)__shfl_sync(0xffffffffu, claim, 0);
+      }
+      while (item < SL.dyn_items) {
+        const int64_t blk = item / g.units;
+        const int32_t unit = (int32_t)(item - blk * g.units);
+        const int64_t a = 1 + SL.dyn_table[blk], b = SL.dyn_table[blk + 1];
+        const int64_t r0 = max(a - 2, (int64_t)0), r1 = min(b + 2, C + 1);
+        const bool early = r1 - r0 + 1 <= (int64_t)R.S;
+        if (early && lane == 0) claim = atomicAdd(ctr, 1u);
+        if (lane == 0) {
+          mbar_wait(&qempty[rq.slot], rq.phase ^ 1u);
+          TbDesc d;
+          d.kind = TB_WORK;
+          d.unit = unit;
+          d.a = a;
+          d.b = b;
+          d.pad = 0;
+          desc[rq.slot] = d;
+          mbar_arrive(&qfull[rq.slot]);
+          // level-0 rows r0..r1 of the strip: one bulk copy of the x window [x0-2, x0+tx+2)
+          const int64_t xs = 2 + (int64_t)unit * g.tx;
+          const int64_t xe = min(xs + g.tx + 4, g.pitch);
+          const uint32_t bytes = (uint32_t)((xe - xs) * 8);
+          const double *src = cur + xs;
+          for (int64_t p = r0; p <= r1; ++p) {
+            mbar_wait(&R.empty[q.slot], q.phase ^ 1u);
+            mbar_expect_tx(&R.full[q.slot], bytes);
+            bulk_g2s(R.stage(q), src + p * g.plane_elems, bytes, &R.full[q.slot]);
+            q.advance(R.S);
+          }
+        } else {
+          for (int64_t p = r0; p <= r1; ++p) q.advance(R.S);
+        }
+        rq.advance(JB_RQ);
+        if (!early && lane == 0) claim = atomicAdd(ctr, 1u);
+        item = SL.dyn_first + (int64_t)__shfl_sync(0xffffffffu, claim, 0);
+      }
+      if (lane == 0) {
+        mbar_wait(&qempty[rq.slot], rq.phase ^ 1u);
+        desc[rq.slot].kind = TB_END;
+        mbar_arrive(&qfull[rq.slot]);
+      }
+      rq.advance(JB_RQ);
+    } else {
+      while (true) {
+        mbar_wait(&qfull[rq.slot], rq.phase);
+        const TbDesc d = desc[rq.slot];
+        __syncwarp();
+        if (lane == 0) mbar_arrive(&qempty[rq.slot]);
+        rq.advance(JB_RQ);
+        if (d.kind == TB_END) break;
+        tb2_item<PPT>(g, R, q, d.unit, d.a, d.b, C, nxt, warp, lane);
+      }
+      fence_proxy_async_global();  // generic-proxy stores before the next block's bulk reads
+    }
+    // Device-side grid barrier between time blocks.
+    __syncthreads();
+    if (threadIdx.x == 0) {
+      red_release_gpu_add(SL.barrier, 1ull);
+      const bool okb = wait_geq<false>(SL.barrier, (unsigned long long)SL.cta_count * (j + 1), P);
+      s_abort = (!okb || *(volatile int *)(P.status + 1)) ? 1 : 0;
+    }
+    __syncthreads();
+    if (s_abort) return;
+  }
+}
+
+// One CTA per SM (up to 224 registers per thread) or two (96: 2 x 9 warps fit the register file
+// only at <= 96 registers, given the 4-warp allocation granularity).
+template <int PPT>
+__global__ void __launch_bounds__(JB_NC + 32, 1) jb_tblock2d(const __grid_constant__ JbParams P) {
+  tb_body<JB_NCW, PPT>(P);
+}
+template <int PPT>
+__global__ void __maxnreg__(96) jb_tblock2d_x2(const __grid_constant__ JbParams P) {
+  tb_body<JB_NCW, PPT>(P);
+}
+
+const void *tblock_fn(int ppt, int per_sm) {
+#define JB_TB(K, p) reinterpret_cast<const void *>(&K<p>)
+  if (per_sm >= 2) return ppt >= 4 ? JB_TB(jb_tblock2d_x2, 4) : ppt == 2 ? JB_TB(jb_tblock2d_x2, 2) : JB_TB(jb_tblock2d_x2, 1);
+  return ppt >= 4 ? JB_TB(jb_tblock2d, 4) : ppt == 2 ? JB_TB(jb_tblock2d, 2) : JB_TB(jb_tblock2d, 1);
+#undef JB_TB
+}
+
+}  // namespace
+
+namespace jbk {
+
+int tblock_k() { return TB_K; }
+int tblock_threads() { return JB_NC + 32; }
+
+// Dynamic shared memory of the temporally blocked kernel: header + ring stages.
+size_t tblock_smem(const JbGeom &g) {
+  const size_t hdr = (size_t)2 * g.stages * 8 + (size_t)2 * JB_RQ * 8 + (size_t)JB_RQ * sizeof(TbDesc);
+  return (hdr + 127) / 128 * 128 + (size_t)g.stages * g.stage_doubles * 8;
+}
+
+cudaError_t prepare_tblock(const JbGeom &g, int per_sm, size_t smem, int *blocks_per_sm) {
+  const void *fn = tblock_fn(g.tx / (2 * JB_NC), per_sm);
+  cudaError_t e = cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+  if (e != cudaSuccess) return e;
+  e = cudaFuncSetAttribute(fn, cudaFuncAttributePreferredSharedMemoryCarveout, (int)cudaSharedmemCarveoutMaxShared);
+  if (e != cudaSuccess) return e;
+  return cudaOccupancyMaxActiveBlocksPerMultiprocessor(blocks_per_sm, fn, JB_NC + 32, smem);
+}
+
+cudaError_t launch_tblock(const JbParams &p, int per_sm, int grid, size_t smem, cudaStream_t st) {
+  void *args[] = {const_cast<JbParams *>(&p)};
+  return cudaLaunchCooperativeKernel(tblock_fn(p.g.tx / (2 * JB_NC), per_sm), dim3(grid), dim3(JB_NC + 32), args, smem,
+                                     st);
+}
+
+}  // namespace jbk

@@ -29,9 +29,10 @@ def assert_bitwise(got, exp, what=""):
 
 
 def run_gpu(field, iters, virtual=0, mode=jb.MODE_CPUFREE, params=None, flags=0):
-    """Run through the C ABI.  Unless `params` says otherwise the streaming kernel is forced
-    (resident=0), so these shapes exercise it; the resident kernel has its own tests below."""
-    params = {"resident": 0, **(params or {})}
+    """Run through the C ABI.  Unless `params` says otherwise the per-iteration streaming kernel
+    is forced (resident=0, tblock=0), so these shapes exercise it; the resident and the
+    temporally blocked kernels have their own tests (below, test_gpu_tblock.py)."""
+    params = {"resident": 0, "tblock": 0, **(params or {})}
     with jb.Jacobi(field.shape, virtual=virtual) as j:
         for k, v in params.items():
             j.set_param(k, v)

@@ -1,0 +1,144 @@
+"""GPU parity of the temporally blocked CPU-Free kernel (tblock.cu): two Jacobi
+iterations per pass over HBM for a slab without neighbours.  It reorders WHEN cells are
+updated, never HOW (oracle operation order, -fmad=false), so the bar is bit-exact equality with
+the oracle — over ragged strips, tiny and single-plane blocks, the Dirichlet rows/columns that
+the intermediate level must keep, odd iteration counts (the remainder runs per-iteration) and
+run splitting / mixing with the other kernels and modes."""
+import numpy as np
+import pytest
+
+import oracle
+import paper_conf_sc_baydamirlibu24_b200 as jb
+from jacobi_inputs import SEED_BENCH, integer_field, nv_field, u12
+
+pytestmark = pytest.mark.gpu
+
+
+def assert_bitwise(got, exp, what=""):
+    if not np.array_equal(np.asarray(got).view(np.uint64), np.asarray(exp).view(np.uint64)):
+        d = np.abs(got - exp)
+        idx = np.unravel_index(np.argmax(d), d.shape)
+        n = np.count_nonzero(got.view(np.uint64) != exp.view(np.uint64))
+        raise AssertionError(f"{what}: {n} cells differ, max |diff| {d.max()} at {idx}")
+
+
+def run_tb(field, iters, params=None, runs=None):
+    """Force the temporally blocked kernel (tblock=1, resident off); returns (field, last_tblock)."""
+    params = {"tblock": 1, "resident": 0, **(params or {})}
+    with jb.Jacobi(field.shape) as j:
+        for k, v in params.items():
+            j.set_param(k, v)
+        j.scatter(field)
+        for n in (runs or [iters]):
+            j.run(n)
+        return j.gather(), j.get_param("last_tblock")
+
+
+@pytest.mark.parametrize("shape", [(3, 3), (3, 40), (4, 5), (6, 9), (37, 1500), (70, 2051), (300, 130),
+                                   (1000, 37), (17, 4100)])
+@pytest.mark.parametrize("iters", [4, 5, 12, 29])
+def test_tblock_shapes(shape, iters):
+    f = u12(shape, 1)
+    exp = oracle.jacobi(f, iters)
+    got, tb = run_tb(f, iters)
+    assert tb == iters // 4 * 4
+    assert_bitwise(got, exp, f"tblock {shape} it{iters}")
+
+
+@pytest.mark.parametrize("tile_x,min_block", [(8, 1), (16, 2), (64, 1), (256, 3), (1024, 16), (2048, 5)])
+@pytest.mark.parametrize("ctas", [1, 2])
+def test_tblock_tiles_and_blocks(tile_x, min_block, ctas):
+    """Many strips (ragged last strip, strips narrower than a warp), single-plane blocks, one or
+    two CTAs per SM."""
+    shape = (133, 2100)
+    f = u12(shape, 2)
+    got, _ = run_tb(f, 8, {"tile_x": tile_x, "tb_min_block": min_block, "tb_ctas": ctas})
+    assert_bitwise(got, oracle.jacobi(f, 8), f"tx{tile_x} mb{min_block}")
+
+
+@pytest.mark.parametrize("stages", [4, 5, 9])
+def test_tblock_ring_depths(stages):
+    f = u12((400, 700), 3)
+    got, _ = run_tb(f, 16, {"stages": stages, "tb_min_block": 40})
+    assert_bitwise(got, oracle.jacobi(f, 16), f"stages {stages}")
+
+
+def test_tblock_run_splitting_and_mixing():
+    """run(a); run(b) == run(a+b) across the time-blocked, per-iteration, resident and baseline
+    kernels (the buffer parity convention is shared)."""
+    f = u12((90, 300), 4)
+    exp = oracle.jacobi(f, 31)
+    got, _ = run_tb(f, 31, runs=[4, 1, 8, 3, 5, 6, 4])
+    assert_bitwise(got, exp, "split")
+    with jb.Jacobi(f.shape) as j:
+        j.set_param("resident", 0)
+        j.scatter(f)
+        j.run(6)                                  # auto: 4 time-blocked + 2 per-iteration
+        assert j.get_param("last_tblock") == 4
+        j.set_mode(jb.MODE_BASELINE_MEMCPY)
+        j.run(3)
+        j.set_mode(jb.MODE_CPUFREE)
+        j.set_param("resident", 1)
+        j.run(5)                                  # resident kernel
+        j.set_param("resident", 0)
+        j.run(17)                                 # 16 time-blocked + 1
+        assert_bitwise(j.gather(), exp, "mixed")
+
+
+def test_tblock_invariants_and_special_fields():
+    y, x = np.mgrid[0:41, 0:77].astype(np.float64)
+    for h in (3 + 2 * x - 5 * y, x * x - y * y, x * y, np.full((41, 77), np.pi)):
+        got, _ = run_tb(np.ascontiguousarray(h), 24)
+        assert_bitwise(got, h, "harmonic field stationary")
+    f = integer_field((50, 60), 5)
+    got, _ = run_tb(f, 12)
+    assert_bitwise(got, oracle.jacobi(f, 12), "integer field")
+    f = nv_field((34, 2400))
+    got, _ = run_tb(f, 1000)
+    exp = oracle.jacobi(f, 1000)
+    assert np.count_nonzero((exp != 0) & (np.abs(exp) < np.finfo(np.float64).tiny)) > 0
+    assert_bitwise(got, exp, "subnormals")
+
+
+def test_tblock_auto_selection_and_errors():
+    f = u12((64, 96), 1)
+    with jb.Jacobi(f.shape) as j:  # fits on chip: auto keeps the resident kernel
+        j.scatter(f)
+        j.run(8)
+        assert j.get_param("last_tblock") == 0 and j.get_param("last_resident") == 1
+        j.set_param("tblock", 0)
+        j.set_param("resident", 0)
+        j.run(8)
+        assert j.get_param("last_tblock") == 0
+        with pytest.raises(jb.JacobiError):
+            j.set_param("last_tblock", 1)
+    with jb.Jacobi((64, 96), virtual=2) as j:  # slabs with neighbours: not eligible
+        j.set_param("tblock", 1)
+        with pytest.raises(jb.JacobiError):
+            j.run(4)
+        j.set_param("tblock", -1)
+        j.run(4)
+        assert j.get_param("last_tblock") == 0
+    with jb.Jacobi((6, 8, 10)) as j:  # 3D: per-iteration kernels
+        j.set_param("tblock", 1)
+        with pytest.raises(jb.JacobiError):
+            j.run(4)
+
+
+def test_tblock_watchdog_state_is_clean():
+    """A run after a time-blocked run on the same handle starts from consistent counters."""
+    f = u12((200, 5000), 6)
+    got, _ = run_tb(f, 40, runs=[20, 20])
+    assert_bitwise(got, oracle.jacobi(f, 40), "two runs")
+
+
+def test_c2_full_grid_8_iters_time_blocked():
+    """C2 at full size in the bench's launch configuration (auto selects the time-blocked
+    kernel), cell for cell against the OpenMP oracle."""
+    import os
+    with jb.Jacobi((16384, 16384)) as j:
+        j.run(8)
+        assert j.get_param("last_tblock") == 8
+        got = j.gather()
+    exp = oracle.jacobi(u12((16384, 16384), SEED_BENCH), 8, os.cpu_count() or 1)
+    assert_bitwise(got, exp, "C2 8 iterations")
