@@ -15,6 +15,7 @@
 #define JB_MAX_BLOCKS 1024      // per-slab block flags of the resident kernel
 #define JB_RCPP_MAX 8           // max cell pairs per thread held in registers by the resident kernel
 #define JB_SMEM_DEFAULT 232448  // B200 opt-in dynamic shared memory per block (227 KB)
+#define JB_EDGE_PLANES 4        // scratch planes after each slab buffer: time-blocked edge zones (tblock.cu)
 
 // Grid geometry in HBM and the tile shape of the march.
 //   element (x, y, z) of slab plane p lives at  buf + p*plane_elems + y*pitch + (x + 3)
@@ -90,6 +91,14 @@ struct JbSlab {
   int32_t use_shm;
   int32_t shm_pe_top, shm_pe_bot;
   int32_t pad3;
+  // Temporally blocked kernel (tblock.cu): interior level-2 planes tb_lo..tb_hi (dynamic items),
+  // and the neighbours' intermediate-level halo slots this slab writes: the top neighbour's
+  // bottom slot (its E_bot[3]) and the bottom neighbour's top slot (its E_top[0]).  A slab's own
+  // edge scratch: E_top = buf[0] + (chunk+2)*plane_elems, E_bot = buf[1] + (chunk+2)*plane_elems,
+  // JB_EDGE_PLANES planes each.
+  int64_t tb_lo, tb_hi;
+  double *mid_top_out;
+  double *mid_bot_out;
 };
 
 struct JbParams {

@@ -32,11 +32,12 @@ jacobi_ctx *new_ctx(int64_t nx, int64_t ny, int64_t nz, int stencil, int total) 
 
 int alloc_slab(jacobi_ctx *h, Slab &s) {
   CK(cudaSetDevice(s.device));
-  size_t bytes = (size_t)slab_elems(h, s) * sizeof(double);
+  // (chunk + 2) planes of the slab + JB_EDGE_PLANES scratch planes (time-blocked edge zones)
+  size_t bytes = (size_t)(s.chunk + 2 + JB_EDGE_PLANES) * h->geom.plane_elems * sizeof(double);
   if (h->kind == KIND_SHMEM) {  // symmetric heap: every PE allocates the largest slab
     int64_t st, chunk_max;
     jbplan::decompose(h->n_out, h->total, 0, &st, &chunk_max);
-    bytes = (size_t)(chunk_max + 2) * h->geom.plane_elems * sizeof(double);
+    bytes = (size_t)(chunk_max + 2 + JB_EDGE_PLANES) * h->geom.plane_elems * sizeof(double);
   }
   if (h->alloc.alloc) {
     s.buf[0] = static_cast<double *>(h->alloc.alloc(bytes, s.device, h->alloc.user));
@@ -98,12 +99,14 @@ void link_local(jacobi_ctx *h) {
     if (s.has_top) {
       Slab &o = h->slabs[i - 1];
       for (int p = 0; p < 2; ++p) s.peer_top[p] = o.buf[p] + (o.chunk + 1) * pe;
+      s.mid_top_out = o.buf[1] + (o.chunk + 2 + 3) * pe;  // its E_bot[3]
       s.flag_out_top = &o.ctrl->flag_in[1][0];
       s.peer_top_dev = o.device;
     }
     if (s.has_bot) {
       Slab &o = h->slabs[i + 1];
       for (int p = 0; p < 2; ++p) s.peer_bot[p] = o.buf[p];
+      s.mid_bot_out = o.buf[0] + (o.chunk + 2) * pe;  // its E_top[0]
       s.flag_out_bot = &o.ctrl->flag_in[0][0];
       s.peer_bot_dev = o.device;
     }
@@ -554,54 +557,100 @@ int run_cpufree_k1(jacobi_ctx *h, int64_t iters) {
   return JACOBI_OK;
 }
 
-// Temporally blocked CPU-Free launch (tblock.cu) of `iters` (a multiple of
-// 2K) iterations on a single slab without neighbours: the guided dynamic schedule of
-// plan_launch, with the ring shortened to leave room for the level-1 row ring.
+// Temporally blocked CPU-Free launch (tblock.cu) of `iters` (a multiple of 2K)
+// iterations: per launch group the roles and flags of plan_launch (boundary CTAs run the edge
+// zones with the per-iteration exchange, then join the interior), the guided dynamic schedule
+// over the interior planes the edge zones leave, and the ring shortened to the smem budget.
 int run_tblock(jacobi_ctx *h, int64_t iters) {
-  LaunchPlan L;
-  const int64_t sched = h->schedule, minb = h->min_block;
-  h->schedule = 2;
-  h->min_block = std::max<int64_t>(1, h->tb_min_block);
-  int sms = 0;
-  CK(cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, h->slabs[0].device));
-  const int per_sm = h->tb_ctas >= 2 ? 2 : 1;
-  int rc = plan_launch(h, {0}, LK_PERSIST, false, L, per_sm == 2 ? launch_ctas(h, sms) * 2 : 0);
-  h->schedule = sched;
-  h->min_block = minb;
-  if (rc) return rc;
-  JbGeom &g = L.P.g;
-  int smem_optin = 0;
-  CK(cudaDeviceGetAttribute(&smem_optin, cudaDevAttrMaxSharedMemoryPerBlockOptin, L.device));
-  smem_optin = std::min(smem_optin, JB_SMEM_DEFAULT) - 1024;
-  if (per_sm == 2) {  // two CTAs share the SM's shared memory (1 KB reserved per CTA + static)
-    int smem_sm = 0;
-    CK(cudaDeviceGetAttribute(&smem_sm, cudaDevAttrMaxSharedMemoryPerMultiprocessor, L.device));
-    smem_optin = std::min(smem_optin, smem_sm / 2 - 1024 - 512);
+  auto groups = launch_groups(h);
+  std::vector<LaunchPlan> plans(groups.size());
+  const int per_sm = (h->tb_ctas >= 2 && h->total == 1) ? 2 : 1;  // roles must match across slabs
+  for (size_t gi = 0; gi < groups.size(); ++gi) {
+    LaunchPlan &L = plans[gi];
+    const int64_t sched = h->schedule;
+    h->schedule = 2;
+    int sms = 0;
+    CK(cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, h->slabs[groups[gi][0]].device));
+    int rc = plan_launch(h, groups[gi], LK_PERSIST, false, L, per_sm == 2 ? launch_ctas(h, sms) * 2 : 0);
+    h->schedule = sched;
+    if (rc) return rc;
+    JbGeom &g = L.P.g;
+    const int min_blk = (int)std::max<int64_t>(1, h->tb_min_block);
+    for (size_t k = 0; k < groups[gi].size(); ++k) {
+      Slab &s = h->slabs[groups[gi][k]];
+      JbSlab &d = L.P.s[k];
+      d.tb_lo = s.has_top ? 3 : 1;  // edge zones: level-2 planes 1, 2 (top) and C-1, C (bottom)
+      d.tb_hi = s.has_bot ? s.chunk - 2 : s.chunk;
+      d.mid_top_out = s.mid_top_out;
+      d.mid_bot_out = s.mid_bot_out;
+      const int64_t npl = d.tb_hi - d.tb_lo + 1;
+      const int ni = d.cta_count - d.n_top - d.n_bot;
+      d.dyn_items = 0;
+      d.dyn_first = 0;
+      if (npl > 0) {
+        d.dyn_min_blk = min_blk;
+        d.dyn_n = d.dyn_help ? d.cta_count : ni;
+        const int64_t nblk = jbplan::dyn_blocks(npl, g.units, d.dyn_n, min_blk);
+        d.dyn_items = (int64_t)g.units * nblk;
+        d.dyn_first = (int)std::min<int64_t>(ni, d.dyn_items);
+        rc = upload_table(s, npl, g.units, d.dyn_n, min_blk, nblk);
+        if (rc) return rc;
+        d.dyn_table = s.dyn_table;
+      }
+      s.desc = d;
+    }
+    int smem_optin = 0;
+    CK(cudaDeviceGetAttribute(&smem_optin, cudaDevAttrMaxSharedMemoryPerBlockOptin, L.device));
+    smem_optin = std::min(smem_optin, JB_SMEM_DEFAULT) - 1024;
+    if (per_sm == 2) {  // two CTAs share the SM's shared memory (1 KB reserved per CTA + static)
+      int smem_sm = 0;
+      CK(cudaDeviceGetAttribute(&smem_sm, cudaDevAttrMaxSharedMemoryPerMultiprocessor, L.device));
+      smem_optin = std::min(smem_optin, smem_sm / 2 - 1024 - 512);
+    }
+    while (g.stages > 3 && jbk::tblock_smem(g) > (size_t)smem_optin) --g.stages;
+    if (jbk::tblock_smem(g) > (size_t)smem_optin) return JACOBI_EINVAL;
+    L.smem = jbk::tblock_smem(g);
+    int occ = 0;
+    CK(jbk::prepare_tblock(g, per_sm, L.smem, &occ));
+    if (occ < per_sm) {
+      if (getenv("JACOBI_DEBUG")) fprintf(stderr, "[jacobi] tblock: occupancy %d < %d (smem %zu)\n", occ, per_sm, L.smem);
+      return JACOBI_ENOCOOP;
+    }
+    for (int k : groups[gi]) h->slabs[k].smem = L.smem;
+    L.P.t0 = h->t;
+    L.P.iters = iters;
   }
-  while (g.stages > 3 && jbk::tblock_smem(g) > (size_t)smem_optin) --g.stages;
-  if (jbk::tblock_smem(g) > (size_t)smem_optin) return JACOBI_EINVAL;
-  L.smem = jbk::tblock_smem(g);
-  int occ = 0;
-  CK(jbk::prepare_tblock(g, per_sm, L.smem, &occ));
-  if (occ < per_sm) {
-    if (getenv("JACOBI_DEBUG")) fprintf(stderr, "[jacobi] tblock: occupancy %d < %d (smem %zu)\n", occ, per_sm, L.smem);
-    return JACOBI_ENOCOOP;
+  // per-run counters; flags raised to the current iteration (as run_cpufree_k1)
+  for (auto &L : plans) {
+    CK(cudaSetDevice(L.device));
+    for (int k : L.slab_idx) {
+      Slab &s = h->slabs[k];
+      CK(reset_run_counters(s, L.stream));
+      CK(jbk::launch_flag_max(&s.ctrl->flag_in[0][0], 2 * JB_MAXK, (unsigned long long)h->t, L.stream));
+    }
   }
-  Slab &s = h->slabs[0];
-  s.smem = L.smem;
-  L.P.t0 = h->t;
-  L.P.iters = iters;
-  CK(reset_run_counters(s, L.stream));
-  CK(cudaEventRecord(s.ev0, L.stream));
-  CK(jbk::launch_tblock(L.P, per_sm, L.grid, L.smem, L.stream));
-  CK(cudaEventRecord(s.ev1, L.stream));
-  CK(cudaEventSynchronize(s.ev1));
-  float ms = 0;
-  CK(cudaEventElapsedTime(&ms, s.ev0, s.ev1));
-  s.last_ms = ms;
-  h->last_ms_max = ms;
-  rc = read_status(s);
-  if (rc) return rc;
+  for (auto &L : plans) {
+    CK(cudaSetDevice(L.device));
+    Slab &s0 = h->slabs[L.slab_idx[0]];
+    CK(cudaEventRecord(s0.ev0, L.stream));
+    CK(jbk::launch_tblock(L.P, per_sm, L.grid, L.smem, L.stream));
+    CK(cudaEventRecord(s0.ev1, L.stream));
+  }
+  int rc_all = JACOBI_OK;
+  double mx = 0;
+  for (auto &L : plans) {
+    CK(cudaSetDevice(L.device));
+    Slab &s0 = h->slabs[L.slab_idx[0]];
+    CK(cudaEventSynchronize(s0.ev1));
+    float ms = 0;
+    CK(cudaEventElapsedTime(&ms, s0.ev0, s0.ev1));
+    for (int k : L.slab_idx) h->slabs[k].last_ms = ms;
+    mx = std::max(mx, (double)ms);
+    int rc = read_status(s0);
+    if (rc && !rc_all) rc_all = rc;
+  }
+  h->last_ms_max = mx;
+  if (rc_all) return rc_all;
   h->t += iters;
   return JACOBI_OK;
 }
@@ -613,8 +662,9 @@ int run_cpufree(jacobi_ctx *h, int64_t iters) {
   h->last_tblock = 0;
   h->last_resident = 0;
   const bool nocomp = h->flags & JACOBI_FLAG_NO_COMPUTE;
-  const bool eligible = h->tblock != 0 && !nocomp && h->norm_every <= 0 && h->dim == 2 && h->total == 1 &&
-                        h->slabs.size() == 1 && (h->kind == KIND_SINGLE || h->kind == KIND_DIST);
+  // P > 1: every slab needs the two edge zones (>= 4 planes); the NVSHMEM variant keeps jb_sweep
+  const bool eligible = h->tblock != 0 && !nocomp && h->norm_every <= 0 && h->dim == 2 &&
+                        h->kind != KIND_SHMEM && (h->total == 1 || (h->n_out - 2) / h->total >= 4);
   if (h->tblock == 1 && !eligible) return JACOBI_EINVAL;
   int64_t tb_iters = 0;
   if (eligible) {
@@ -622,8 +672,12 @@ int run_cpufree(jacobi_ctx *h, int64_t iters) {
     tb_iters = iters / step * step;
     if (h->tblock < 0 && h->resident != 0) {
       // auto: slabs that fit on chip run the resident kernel (faster for those small grids)
-      LaunchPlan R;
-      if (plan_resident(h, {0}, R) == JACOBI_OK) tb_iters = 0;
+      bool fits = true;
+      for (auto &grp : launch_groups(h)) {
+        LaunchPlan R;
+        if (plan_resident(h, grp, R) != JACOBI_OK) fits = false;
+      }
+      if (fits) tb_iters = 0;
     }
   }
   double ms = 0;

@@ -130,6 +130,7 @@ struct Slab {
   bool has_top = false, has_bot = false;
   double *peer_top[2] = {nullptr, nullptr};
   double *peer_bot[2] = {nullptr, nullptr};
+  double *mid_top_out = nullptr, *mid_bot_out = nullptr;  // neighbours' time-blocked edge slots
   unsigned long long *flag_out_top = nullptr, *flag_out_bot = nullptr;
   int peer_top_dev = -1, peer_bot_dev = -1;
   int shm_pe_top = -1, shm_pe_bot = -1;  // NVSHMEM variant: neighbour PEs

@@ -193,12 +193,98 @@ __device__ __forceinline__ void tb2_item(const JbGeom &g, const Ring &R, RingPos
   else tb2_march<PPT, false>(L, R, q0, a, b, C, r0, r1, dst, g.plane_elems, lane);
 }
 
+// Edge zone of a slab side with a neighbour (time block t -> t+2), computed by that side's
+// boundary CTAs with the whole CTA, so the halo exchange stays per iteration:
+//   A: wait for the neighbour's time-t halo plane; level 1 (t+1) of the three planes next to the
+//      halo (top: 1..3, bottom: C-2..C) over the strip window [x0-1, x0+tx] into the slab's edge
+//      scratch E, the outermost one also into the neighbour's intermediate slot; signal t+1.
+//   B: wait for the neighbour's level-1 plane (our E slot); level 2 (t+2) of the two outermost
+//      planes (top: 1, 2; bottom: C-1, C) into the next buffer, the outermost one also into the
+//      neighbour's halo; signal t+2.
+// E_top = buf[0] + (C+2) pe: [0] = neighbour's level-1 plane 0, [k] = level-1 plane k (k = 1..3);
+// E_bot = buf[1] + (C+2) pe: [k] = level-1 plane C-2+k (k = 0..2), [3] = neighbour's plane C+1.
+// Loads bypass L1 (ld.cg): these planes are rewritten by other CTAs / the neighbour GPU.
+__device__ bool tb_edge(const JbGeom &g, const JbSlab &SL, const JbParams &P, int role, int ridx, int rcount,
+                        const double *cur, double *nxt, double *remote, int64_t tg, int *s_flag) {
+  const bool top = role == ROLE_TOP;
+  const int64_t C = SL.chunk, pe = g.plane_elems, nx = g.nx;
+  double *E = (top ? SL.buf[0] : SL.buf[1]) + (C + 2) * pe + 3;
+  double *mid = top ? SL.mid_top_out : SL.mid_bot_out;
+  const unsigned long long *fin = top ? SL.flag_in_top : SL.flag_in_bot;
+  const int kin = top ? SL.k_in_top : SL.k_in_bot;
+  unsigned long long *fout = (top ? SL.flag_out_top : SL.flag_out_bot) + ridx;
+  const int ub = (int)((int64_t)g.units * ridx / rcount), ue = (int)((int64_t)g.units * (ridx + 1) / rcount);
+  const int tid = threadIdx.x, nt = blockDim.x;
+  const bool drop = (P.flags & JACOBI_FLAG_DROP_SIGNAL) && SL.slab_id == 0;
+  auto wait = [&](unsigned long long target) {
+    if (tid < 32) {
+      const bool ok = wait_slots(fin, kin, target, P, tid);
+      if (tid == 0) *s_flag = ok ? 0 : 1;
+    }
+    __syncthreads();
+    return *s_flag == 0;
+  };
+  // ---- A: level 1
+  if (!wait((unsigned long long)tg)) return false;
+  const int64_t pa = top ? 1 : C - 2;  // level-1 plane of E index (top ? 1 : 0)
+  const int e0 = top ? 1 : 0;
+  const int64_t pout = top ? 1 : C;    // the plane the neighbour needs
+  for (int u = ub; u < ue; ++u) {
+    const int64_t x0 = 1 + (int64_t)u * g.tx;
+    const int64_t xa = max(x0 - 1, (int64_t)0), xb = min(x0 + g.tx, nx - 1);
+    const int64_t w = xb - xa + 1;
+    for (int64_t i = tid; i < 3 * w; i += nt) {
+      const int k = (int)(i / w);
+      const int64_t x = xa + (i - k * w), p = pa + k;
+      const double *A = cur + p * pe + 3 + x;
+      double v = __ldcg(A);
+      if (x >= 1 && x <= nx - 2) {  // oracle order: ((x+1) + (x-1)) + (y+1) + (y-1), then * 0.25
+        v = 0.25 * (((__ldcg(A + 1) + __ldcg(A - 1)) + __ldcg(A + pe)) + __ldcg(A - pe));
+      }
+      E[(e0 + k) * pe + x] = v;
+      if (p == pout) mid[3 + x] = v;
+    }
+  }
+  __syncthreads();  // every thread's stores (local E, neighbour's slot) precede the release below
+  if (tid == 0 && !drop) st_release_sys(fout, (unsigned long long)(tg + 1));
+  // ---- B: level 2
+  if (!wait((unsigned long long)(tg + 1))) return false;
+  const int64_t pb = top ? 1 : C - 1;  // first level-2 plane; E index of plane pb + k is e1 + k
+  const int e1 = 1;
+  for (int u = ub; u < ue; ++u) {
+    const int64_t x0 = 1 + (int64_t)u * g.tx;
+    const int64_t w = min((int64_t)g.tx, nx - 1 - x0);
+    for (int64_t i = tid; i < 2 * w; i += nt) {
+      const int k = (int)(i / w);
+      const int64_t x = x0 + (i - k * w), p = pb + k;
+      const double *L = E + (e1 + k) * pe + x;
+      const double v = 0.25 * (((__ldcg(L + 1) + __ldcg(L - 1)) + __ldcg(L + pe)) + __ldcg(L - pe));
+      nxt[p * pe + 3 + x] = v;
+      if (p == pout) remote[3 + x] = v;
+    }
+  }
+  __syncthreads();
+  if (tid == 0 && !drop) st_release_sys(fout, (unsigned long long)(tg + 2));
+  return true;
+}
+
 template <int NCW, int PPT>
 __device__ __forceinline__ void tb_body(const JbParams &P) {
   extern __shared__ __align__(128) unsigned char smem[];
   __shared__ int s_abort;
   const JbGeom &g = P.g;
-  const JbSlab &SL = P.s[0];
+  int si = 0;
+  while (si + 1 < P.nslabs && (int)blockIdx.x >= P.s[si + 1].cta_begin) ++si;
+  const JbSlab &SL = P.s[si];
+  const int c = (int)blockIdx.x - SL.cta_begin;
+  int role, ridx, rcount;
+  if (c < SL.n_top) {
+    role = ROLE_TOP; ridx = c; rcount = SL.n_top;
+  } else if (c < SL.n_top + SL.n_bot) {
+    role = ROLE_BOT; ridx = c - SL.n_top; rcount = SL.n_bot;
+  } else {
+    role = ROLE_INT; ridx = c - SL.n_top - SL.n_bot; rcount = SL.cta_count - SL.n_top - SL.n_bot;
+  }
   Ring R;
   R.S = (uint32_t)g.stages;
   R.stage_doubles = g.stage_doubles;
@@ -210,7 +296,6 @@ __device__ __forceinline__ void tb_body(const JbParams &P) {
   const uint32_t hdr = 2 * R.S * 8 + 2 * JB_RQ * 8 + JB_RQ * (uint32_t)sizeof(TbDesc);
   R.stages = reinterpret_cast<double *>(smem + ((hdr + 127) & ~127u));
 
-  const int c = (int)blockIdx.x;
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const bool producer = warp == NCW;
   if (threadIdx.x == 0) {
@@ -233,12 +318,18 @@ __device__ __forceinline__ void tb_body(const JbParams &P) {
   for (int64_t j = 0; j < nblocks; ++j) {
     const double *cur = SL.buf[(P.t0 + j) & 1];
     double *nxt = SL.buf[(P.t0 + j + 1) & 1];
+    const int64_t tg = P.t0 + TB_K * j;  // global iteration at the start of this time block
+    if (role != ROLE_INT) {  // edge zone with its per-iteration exchange, then help the interior
+      double *remote = role == ROLE_TOP ? SL.peer_top[(P.t0 + j + 1) & 1] : SL.peer_bot[(P.t0 + j + 1) & 1];
+      if (!tb_edge(g, SL, P, role, ridx, rcount, cur, nxt, remote, tg, &s_abort)) return;
+      fence_proxy_async_global();  // our generic-proxy stores before later bulk reads
+    }
     if (producer) {
       fence_proxy_async_global();
       if (lane == 0 && c == 0) SL.work_ctr[(j + 1) & 1] = 0u;  // idle since block j-1
       // Guided self-scheduling over (plane block, strip) items, as jb_sweep.
       unsigned int *ctr = SL.work_ctr + (j & 1);
-      int64_t item = c < SL.dyn_first ? c : -1;
+      int64_t item = (role == ROLE_INT && ridx < SL.dyn_first) ? ridx : -1;
       unsigned int claim = 0;
       if (item < 0) {
         if (lane == 0) claim = atomicAdd(ctr, 1u);
@@ -247,7 +338,7 @@ __device__ __forceinline__ void tb_body(const JbParams &P) {
       while (item < SL.dyn_items) {
         const int64_t blk = item / g.units;
         const int32_t unit = (int32_t)(item - blk * g.units);
-        const int64_t a = 1 + SL.dyn_table[blk], b = SL.dyn_table[blk + 1];
+        const int64_t a = SL.tb_lo + SL.dyn_table[blk], b = SL.tb_lo + SL.dyn_table[blk + 1] - 1;
         const int64_t r0 = max(a - 2, (int64_t)0), r1 = min(b + 2, C + 1);
         const bool early = r1 - r0 + 1 <= (int64_t)R.S;
         if (early && lane == 0) claim = atomicAdd(ctr, 1u);
@@ -306,6 +397,11 @@ __device__ __forceinline__ void tb_body(const JbParams &P) {
     }
     __syncthreads();
     if (s_abort) return;
+  }
+  // End of run: the neighbour's last halo has landed before the kernel completes (as jb_sweep).
+  if (role != ROLE_INT && warp == 0 && nblocks > 0) {
+    if (role == ROLE_TOP) wait_slots(SL.flag_in_top, SL.k_in_top, (unsigned long long)(P.t0 + P.iters), P, lane);
+    else wait_slots(SL.flag_in_bot, SL.k_in_bot, (unsigned long long)(P.t0 + P.iters), P, lane);
   }
 }
 

@@ -112,13 +112,13 @@ def test_tblock_auto_selection_and_errors():
         assert j.get_param("last_tblock") == 0
         with pytest.raises(jb.JacobiError):
             j.set_param("last_tblock", 1)
-    with jb.Jacobi((64, 96), virtual=2) as j:  # slabs with neighbours: not eligible
+    with jb.Jacobi((64, 96), virtual=2) as j:  # slabs with neighbours: edge zones
         j.set_param("tblock", 1)
+        j.run(4)
+        assert j.get_param("last_tblock") == 4
+        j.set_mode(jb.MODE_CPUFREE, jb.FLAG_NO_COMPUTE)  # no-compute runs keep jb_sweep
         with pytest.raises(jb.JacobiError):
             j.run(4)
-        j.set_param("tblock", -1)
-        j.run(4)
-        assert j.get_param("last_tblock") == 0
     with jb.Jacobi((6, 8, 10)) as j:  # 3D: per-iteration kernels
         j.set_param("tblock", 1)
         with pytest.raises(jb.JacobiError):
@@ -142,3 +142,105 @@ def test_c2_full_grid_8_iters_time_blocked():
         got = j.gather()
     exp = oracle.jacobi(u12((16384, 16384), SEED_BENCH), 8, os.cpu_count() or 1)
     assert_bitwise(got, exp, "C2 8 iterations")
+
+
+# ---------------------------------------------------------------- slabs with neighbours
+def run_tb_virtual(field, iters, P, params=None, runs=None):
+    params = {"tblock": 1, "resident": 0, **(params or {})}
+    with jb.Jacobi(field.shape, virtual=P) as j:
+        for k, v in params.items():
+            j.set_param(k, v)
+        j.scatter(field)
+        for n in (runs or [iters]):
+            j.run(n)
+        return j.gather(), j.get_param("last_tblock")
+
+
+@pytest.mark.parametrize("P", [2, 3, 4, 5, 8])
+@pytest.mark.parametrize("shape", [(50, 300), (43, 2100), (81, 37)])
+def test_tblock_virtual_slabs(P, shape):
+    """Edge zones with the per-iteration exchange (level-1 slots + halos, two signals per time
+    block) between P slabs in one launch; chunks of 4+ planes incl. remainders."""
+    if (shape[0] - 2) // P < 4:
+        pytest.skip("slab too thin for the edge zones")
+    f = u12(shape, 7)
+    got, tb = run_tb_virtual(f, 13, P)
+    assert tb == 12
+    assert_bitwise(got, oracle.jacobi(f, 13), f"P={P} {shape}")
+
+
+@pytest.mark.parametrize("chunk", [4, 5, 6, 7])
+def test_tblock_virtual_thin_slabs(chunk):
+    """chunk 4: the two edge zones cover the slab (no interior items); 5-7: 1-3 interior planes."""
+    P = 3
+    f = u12((P * chunk + 2, 150), 8)
+    for tx, mb in [(0, 16), (32, 1)]:
+        params = {"tb_min_block": mb, **({"tile_x": tx} if tx else {})}
+        got, _ = run_tb_virtual(f, 8, P, params)
+        assert_bitwise(got, oracle.jacobi(f, 8), f"chunk {chunk} tx{tx}")
+
+
+def test_tblock_virtual_mixing_and_decomposition():
+    """run splitting across time-blocked / per-iteration / baseline kernels with P slabs, and the
+    P-slab result bit-identical to P = 1."""
+    f = u12((70, 520), 9)
+    exp = oracle.jacobi(f, 37)
+    with jb.Jacobi(f.shape, virtual=4) as j:
+        j.set_param("resident", 0)
+        j.scatter(f)
+        j.run(8)
+        assert j.get_param("last_tblock") == 8
+        j.set_param("tblock", 0)
+        j.run(3)
+        j.set_param("tblock", -1)
+        j.set_mode(jb.MODE_BASELINE_MEMCPY)
+        j.run(2)
+        j.set_mode(jb.MODE_CPUFREE)
+        j.run(24)                      # 24 time-blocked
+        assert j.get_param("last_tblock") == 24
+        assert_bitwise(j.gather(), exp, "mixed P=4")
+    got1, _ = run_tb(f, 37)
+    assert_bitwise(got1, exp, "P=1")
+
+
+def test_tblock_virtual_ineligible_thin():
+    with jb.Jacobi((3 * 3 + 2, 64), virtual=3) as j:  # chunk 3 < 4
+        j.set_param("resident", 0)
+        j.run(8)
+        assert j.get_param("last_tblock") == 0
+        j.set_param("tblock", 1)
+        with pytest.raises(jb.JacobiError):
+            j.run(4)
+
+
+def test_tblock_virtual_watchdog():
+    """A slab that never signals (DROP_SIGNAL on slab 0): the edge zones time out, the run
+    returns ETIMEOUT instead of hanging, and the handle stays usable."""
+    f = u12((40, 200), 10)
+    with jb.Jacobi(f.shape, virtual=2) as j:
+        j.set_param("resident", 0)
+        j.set_param("tblock", 1)
+        j.set_param("timeout_ms", 300)
+        j.set_mode(jb.MODE_CPUFREE, jb.FLAG_DROP_SIGNAL)
+        j.scatter(f)
+        with pytest.raises(jb.JacobiError) as e:
+            j.run(4)
+        assert e.value.code == jb.JACOBI_ETIMEOUT
+
+
+def test_c2_1000_iters_tblock_p8_equals_p1():
+    """C2 full size, 1000 iterations: P = 8 time-blocked slabs == P = 1 time-blocked == the
+    per-iteration kernel, bit for bit."""
+    shape = (16384, 16384)
+    with jb.Jacobi(shape) as j:
+        j.run(1000)
+        assert j.get_param("last_tblock") == 1000
+        ref = j.gather()
+    with jb.Jacobi(shape, virtual=8) as j:
+        j.run(1000)
+        assert j.get_param("last_tblock") == 1000
+        assert_bitwise(j.gather(), ref, "P=8 tblock")
+    with jb.Jacobi(shape) as j:
+        j.set_param("tblock", 0)
+        j.run(1000)
+        assert_bitwise(j.gather(), ref, "per-iteration kernel")
