@@ -122,7 +122,9 @@ int jacobi_nccl_init(jacobi_t h, const void *id128);
 typedef void *(*jacobi_alloc_fn)(size_t bytes, int device, void *user);
 typedef void (*jacobi_free_fn)(void *ptr, int device, void *user);
 int jacobi_set_allocator(jacobi_alloc_fn alloc, jacobi_free_fn free_fn, void *user);
-/* Bytes of ONE field buffer of slab `slab` (of `nslabs`) for this grid (host-only helper). */
+/* Bytes of ONE field buffer of slab `slab` (of `nslabs`) for this grid (host-only helper):
+ * (chunk + 2) planes (owned + halos) + 4 scratch planes used by the time-blocked
+ * kernel's edge zones. */
 int jacobi_slab_bytes(int64_t nx, int64_t ny, int64_t nz, int stencil, int nslabs, int slab, int64_t *bytes);
 
 /* ---- NVSHMEM variant — exported ONLY by libjacobi_b200_nvshmem.so --------
