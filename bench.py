@@ -177,11 +177,25 @@ def run_reference(args, cfg, shape):
         "e2e": {"value": value, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
         "note": "no reference code exists (PAPER.md only); the reference arm is the CPU oracle",
     }
-    print(json.dumps(line), flush=True)
+    emit(line)
     return 0
 
 
+_JSON_FD = None
+
+
+def emit(line: dict) -> None:
+    """The one JSON line on the real stdout (native libraries' prints were sent to stderr)."""
+    os.write(_JSON_FD if _JSON_FD is not None else 1, (json.dumps(line) + "\n").encode())
+
+
 def main():
+    global _JSON_FD
+    # stdout carries only the JSON line: NCCL and other native code print to fd 1 (e.g. "NCCL
+    # version ..."), so fd 1 is pointed at stderr and the line is written to a saved copy.
+    sys.stdout.flush()
+    _JSON_FD = os.dup(1)
+    os.dup2(2, 1)
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
     ap.add_argument("--steps", type=int, default=3)
@@ -445,7 +459,7 @@ def main():
                                     "sample": f"{k} of {iters} iterations on the full grid "
                                               f"({dt:.1f} s, OpenMP over the outer axis)"}
     if rank == 0:
-        print(json.dumps(line), flush=True)
+        emit(line)
     j.close()
     if args.transport == "nvshmem" and world > 1:
         jb.nvshmem_finalize()

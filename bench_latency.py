@@ -61,6 +61,9 @@ def main():
                         us = per_iter_us(j, args.iters)
                         row = {"config": name, "slabs": P, "virtual": P > 1, "mode": mname,
                                "no_compute": nocomp, "us_per_iter": round(us, 3)}
+                        if mname == "cpufree" and not nocomp:
+                            row["kernel"] = ("resident" if j.get_param("last_resident") else
+                                             "tblock" if j.get_param("last_tblock") else "streaming")
                         if not nocomp:
                             cells = (shape[2] - 2) * (shape[1] - 2) * (shape[0] - 2 if shape[0] > 1 else 1)
                             row["gcells_per_s"] = round(cells / us / 1e3, 2)

@@ -156,8 +156,16 @@ int jacobi_set_mode(jacobi_t h, int mode, int flags);
  * not fit)), "block_sync" (resident kernel: 0 = default, device-wide grid barrier per iteration
  * as in P:372; 1 = each block waits only for its face-sharing neighbour blocks' flags),
  * "l2hint" (streaming loads with L2 evict_first / evict_last policies; default off — measured
- * 2-3 % slower on B200), "timeout_ms" (watchdog, default 20000).  Read-only: "last_resident" (1 if the last
- * CPU-Free run used the resident kernel).  Unknown names return JACOBI_EINVAL. */
+ * 2-3 % slower on B200), "timeout_ms" (watchdog, default 20000), "tblock" (CPU-Free runs with
+ * compute (2D and 3D) advance 2 iterations per pass over HBM — temporal blocking; slabs with
+ * neighbours keep the per-iteration halo exchange through edge zones — for every whole multiple
+ * of 4 iterations, the rest per iteration: -1 auto (default: 2D runs, not when the slab fits on
+ * chip, where the resident kernel is used), 0 never, 1 always incl. 3D (EINVAL when a slab has
+ * < 4 planes with P > 1, with the norm, in no-compute mode or in the NVSHMEM variant)), "tb_min_block"
+ * (smallest dynamic plane block of that kernel, default 16), "tb_ctas" (its CTAs per SM, 1 or 2;
+ * 2 only for P = 1).  Read-only: "last_resident" (1 if the last CPU-Free run used the resident
+ * kernel), "last_tblock" (iterations of the last CPU-Free run done time-blocked).  Unknown names
+ * return JACOBI_EINVAL. */
 int jacobi_set_param(jacobi_t h, const char *name, int64_t value);
 int jacobi_get_param(jacobi_t h, const char *name, int64_t *value);
 

@@ -575,6 +575,14 @@ int run_tblock(jacobi_ctx *h, int64_t iters) {
     h->schedule = sched;
     if (rc) return rc;
     JbGeom &g = L.P.g;
+    if (h->dim == 3) {  // tiles of TY rows; stages hold rows y0-2 .. y0+TY+1
+      g.ty = jbk::tblock_ty();
+      g.rh = g.ty + 4;
+      g.units_y = (int)((h->ny - 2 + g.ty - 1) / g.ty);
+      g.units = g.units_x * g.units_y;
+      g.stage_doubles = g.rh * g.ws;
+    }
+    g.stages = (int)(h->stages > 0 ? std::min<int64_t>(h->stages, JB_MAX_STAGES) : JB_MAX_STAGES);
     const int min_blk = (int)std::max<int64_t>(1, h->tb_min_block);
     for (size_t k = 0; k < groups[gi].size(); ++k) {
       Slab &s = h->slabs[groups[gi][k]];
@@ -663,11 +671,13 @@ int run_cpufree(jacobi_ctx *h, int64_t iters) {
   h->last_resident = 0;
   const bool nocomp = h->flags & JACOBI_FLAG_NO_COMPUTE;
   // P > 1: every slab needs the two edge zones (>= 4 planes); the NVSHMEM variant keeps jb_sweep
-  const bool eligible = h->tblock != 0 && !nocomp && h->norm_every <= 0 && h->dim == 2 &&
+  const bool eligible = h->tblock != 0 && !nocomp && h->norm_every <= 0 &&
                         h->kind != KIND_SHMEM && (h->total == 1 || (h->n_out - 2) / h->total >= 4);
   if (h->tblock == 1 && !eligible) return JACOBI_EINVAL;
+  // auto picks it where it measured faster than the per-iteration kernel: 2D (3D: forced only)
+  const bool use = eligible && (h->tblock == 1 || h->dim == 2);
   int64_t tb_iters = 0;
-  if (eligible) {
+  if (use) {
     const int64_t step = 2 * jbk::tblock_k();  // even block count: the result stays in buf[t & 1]
     tb_iters = iters / step * step;
     if (h->tblock < 0 && h->resident != 0) {

@@ -33,6 +33,7 @@ cudaError_t prepare_resident(int dim, int cpp, size_t smem, int *blocks_per_sm);
 cudaError_t launch_resident(const JbParams &p, int cpp, int grid, size_t smem, cudaStream_t st);
 cudaError_t launch_neighbour_wait(const JbParams &p, unsigned long long target, cudaStream_t st);
 int tblock_k();
+int tblock_ty();
 size_t tblock_smem(const JbGeom &g);
 cudaError_t prepare_tblock(const JbGeom &g, int per_sm, size_t smem, int *blocks_per_sm);
 cudaError_t launch_tblock(const JbParams &p, int per_sm, int grid, size_t smem, cudaStream_t st);

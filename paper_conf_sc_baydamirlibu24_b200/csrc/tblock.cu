@@ -193,6 +193,164 @@ __device__ __forceinline__ void tb2_item(const JbGeom &g, const Ring &R, RingPos
   else tb2_march<PPT, false>(L, R, q0, a, b, C, r0, r1, dst, g.plane_elems, lane);
 }
 
+// ---------------------------------------------------------------- 3D (7-point)
+// Tile = TY rows x tx columns (tx = 64 x warps), marched along z.  Lane `lane` of warp w owns the
+// x pair kk = w*32 + lane for EVERY row of the tile, so level-1 y neighbours are its own
+// registers; x neighbours come by shuffles (+ the two extra cells per warp segment and row, as
+// in 2D).  Stage = level-0 rows y0-2 .. y0+TY+1 (stage row s <-> y0-2+s) of one plane.
+//   level 1 (t+1): planes a-1 .. b+1, rows y0-1 .. y0+TY (Dirichlet rows/columns/planes keep level 0)
+//   level 2 (t+2): planes a .. b, rows y0 .. y0+TY-1                            -> out
+struct TbSeg3 {
+  int j0;         // stage column index of this lane's pair
+  bool ok, full;  // columns x0+2kk / x0+2kk+1 interior
+  bool first, last;
+  int sx;         // stage column of this lane's extra cell (lane 1: right end, others: left)
+  bool ex_in;
+  int y0, vy;     // first row of the tile, interior rows in it (<= TY)
+};
+
+// Level 1 of rows y0-1 .. y0+TY of one plane (stages sm / sc / sn = planes q1-1, q1, q1+1).
+template <int TY, bool FAST>
+__device__ __forceinline__ void tb3_level1(const TbSeg3 &L, const JbGeom &g, const double *sm, const double *sc,
+                                           const double *sn, bool planein, double2 *V, double *ex) {
+  const int ws = g.ws;
+  const double *c = sc + L.j0, *u = sn + L.j0, *d = sm + L.j0;
+  double2 Sy = lds2(c);       // stage row 0 = y0-2
+  double2 Cy = lds2(c + ws);  // stage row 1 = y0-1
+#pragma unroll
+  for (int ry = 0; ry < TY + 2; ++ry) {  // level-1 row y0-1+ry = stage row ry+1
+    const int o = (ry + 1) * ws;
+    const double2 Ny = lds2(c + o + ws), U = lds2(u + o), D = lds2(d + o);
+    const double W = c[o - 1], E = c[o + 2];
+    // oracle order: x+1, x-1, y+1, y-1, z+1, z-1, then * fl(1/6)
+    const double l0 = kC6 * (((((Cy.y + W) + Ny.x) + Sy.x) + U.x) + D.x);
+    const double l1 = kC6 * (((((E + Cy.x) + Ny.y) + Sy.y) + U.y) + D.y);
+    const int y = L.y0 - 1 + ry;
+    const bool rowin = planein && y >= 1 && y <= (int)g.ny - 2;
+    V[ry].x = (rowin && (FAST || L.ok)) ? l0 : Cy.x;
+    V[ry].y = (rowin && (FAST || L.full)) ? l1 : Cy.y;
+    Sy = Cy;
+    Cy = Ny;
+  }
+  // extra cells of the output rows (ry = 1 .. TY)
+  const double *ce = sc + L.sx, *ue = sn + L.sx, *de = sm + L.sx;
+#pragma unroll
+  for (int ry = 1; ry <= TY; ++ry) {
+    const int o = (ry + 1) * ws;
+    const double e = kC6 * (((((ce[o + 1] + ce[o - 1]) + ce[o + ws]) + ce[o - ws]) + ue[o]) + de[o]);
+    const int y = L.y0 - 1 + ry;
+    ex[ry - 1] = (planein && L.ex_in && y <= (int)g.ny - 2) ? e : ce[o];
+  }
+}
+
+// Level 2 of the middle plane (level-1 planes Pm, Pc, Pn), rows y0 .. y0+TY-1, stored at o.
+template <int TY, bool FAST>
+__device__ __forceinline__ void tb3_level2(const TbSeg3 &L, const double2 *Pm, const double2 *Pc, const double2 *Pn,
+                                           const double *exl, const double *exr, int lane, double *o,
+                                           int64_t pitch) {
+#pragma unroll
+  for (int ry = 1; ry <= TY; ++ry) {
+    const double rw = __shfl_sync(0xffffffffu, Pc[ry].y, (lane + 31) & 31);
+    const double re = __shfl_sync(0xffffffffu, Pc[ry].x, (lane + 1) & 31);
+    const double W = L.first ? exl[ry - 1] : rw;
+    const double E = L.last ? exr[ry - 1] : re;
+    const double o0 = kC6 * (((((Pc[ry].y + W) + Pc[ry + 1].x) + Pc[ry - 1].x) + Pn[ry].x) + Pm[ry].x);
+    const double o1 = kC6 * (((((E + Pc[ry].x) + Pc[ry + 1].y) + Pc[ry - 1].y) + Pn[ry].y) + Pm[ry].y);
+    double *p = o + (ry - 1) * pitch;
+    if (FAST) *reinterpret_cast<double2 *>(p) = make_double2(o0, o1);
+    else if (L.ok && ry - 1 < L.vy) store_pair(p, o0, o1, L.full);
+  }
+}
+
+template <int TY, bool FAST>
+__device__ __forceinline__ void tb3_march(const TbSeg3 &L, const JbGeom &g, const Ring &R, RingPos q, int64_t a,
+                                          int64_t b, int64_t C, int64_t r0, int64_t r1, double *dst, int lane) {
+  double2 Pm[TY + 2], Pc[TY + 2], Pn[TY + 2];
+  double ex[TY], exl_c[TY], exr_c[TY], exl_n[TY], exr_n[TY];
+  RingPos pc = ring_add(q, (uint32_t)(a - 1 - r0), R.S);
+  RingPos pm = a - 2 >= r0 ? q : pc;
+  R.wait_full(pm);
+  R.wait_full(pc);
+  auto plane = [&](int64_t q1, double2 *out) {
+    RingPos pn = pc;
+    if (q1 + 1 <= r1) pn.advance(R.S);
+    R.wait_full(pn);
+    tb3_level1<TY, FAST>(L, g, R.stage(pm), R.stage(pc), R.stage(pn), q1 >= 1 && q1 <= C, out, ex);
+    if (q1 - 1 >= r0) R.release(pm, lane);
+    pm = pc;
+    pc = pn;
+  };
+  auto take_ex = [&](double *xl, double *xr) {
+#pragma unroll
+    for (int i = 0; i < TY; ++i) {
+      xl[i] = __shfl_sync(0xffffffffu, ex[i], 0);
+      xr[i] = __shfl_sync(0xffffffffu, ex[i], 1);
+    }
+  };
+  plane(a - 1, Pc);
+  plane(a, Pn);
+  take_ex(exl_n, exr_n);
+  double *o = dst + a * g.plane_elems;
+  for (int64_t q1 = a + 1; q1 <= b + 1; ++q1) {
+#pragma unroll
+    for (int i = 0; i < TY + 2; ++i) {
+      Pm[i] = Pc[i];
+      Pc[i] = Pn[i];
+    }
+#pragma unroll
+    for (int i = 0; i < TY; ++i) {
+      exl_c[i] = exl_n[i];
+      exr_c[i] = exr_n[i];
+    }
+    plane(q1, Pn);
+    take_ex(exl_n, exr_n);
+    tb3_level2<TY, FAST>(L, Pm, Pc, Pn, exl_c, exr_c, lane, o, g.pitch);
+    o += g.plane_elems;
+  }
+  RingPos pr = ring_add(q, (uint32_t)(b + 1 - r0), R.S);
+  for (int64_t p = b + 1; p <= r1; ++p) {
+    R.release(pr, lane);
+    pr.advance(R.S);
+  }
+}
+
+template <int TY>
+__device__ __forceinline__ void tb3_item(const JbGeom &g, const Ring &R, RingPos &q, int unit, int64_t a,
+                                         int64_t b, int64_t C, double *out, int warp, int lane) {
+  const int ux = unit % g.units_x, uy = unit / g.units_x;
+  const int64_t x0 = 1 + (int64_t)ux * g.tx;
+  const int vx = (int)min((int64_t)g.tx, g.nx - 1 - x0);
+  const int txp = g.tx >> 1;
+  const int seg_b = warp * 32, seg_e = min(seg_b + 32, txp);
+  const int64_t r0 = max(a - 2, (int64_t)0), r1 = min(b + 2, C + 1);
+  const RingPos q0 = q;
+  q = ring_add(q, (uint32_t)(r1 - r0 + 1), R.S);
+  const int kk = seg_b + lane;
+  if (seg_b >= seg_e) {
+    for (int64_t p = r0; p <= r1; ++p) {
+      const RingPos pp = ring_add(q0, (uint32_t)(p - r0), R.S);
+      R.wait_full(pp);
+      R.release(pp, lane);
+    }
+    return;
+  }
+  TbSeg3 L;
+  L.j0 = 2 + 2 * min(kk, seg_e - 1);  // lanes past the tile read (and discard) the last pair
+  L.ok = kk < seg_e && 2 * kk < vx;
+  L.full = kk < seg_e && 2 * kk + 1 < vx;
+  L.first = kk == seg_b;
+  L.last = kk == seg_e - 1;
+  L.sx = lane == 1 ? 2 * seg_e + 2 : 2 * seg_b + 1;
+  const int64_t cx = x0 - 2 + L.sx;
+  L.ex_in = cx >= 1 && cx <= g.nx - 2;
+  L.y0 = 1 + uy * TY;
+  L.vy = (int)min((int64_t)TY, g.ny - 1 - L.y0);
+  const bool fast = seg_e - seg_b == 32 && 2 * seg_e <= vx && L.vy == TY;
+  double *dst = out + (int64_t)L.y0 * g.pitch + 3 + x0 + 2 * kk;
+  if (fast) tb3_march<TY, true>(L, g, R, q0, a, b, C, r0, r1, dst, lane);
+  else tb3_march<TY, false>(L, g, R, q0, a, b, C, r0, r1, dst, lane);
+}
+
 // Edge zone of a slab side with a neighbour (time block t -> t+2), computed by that side's
 // boundary CTAs with the whole CTA, so the halo exchange stays per iteration:
 //   A: wait for the neighbour's time-t halo plane; level 1 (t+1) of the three planes next to the
@@ -204,12 +362,13 @@ __device__ __forceinline__ void tb2_item(const JbGeom &g, const Ring &R, RingPos
 // E_top = buf[0] + (C+2) pe: [0] = neighbour's level-1 plane 0, [k] = level-1 plane k (k = 1..3);
 // E_bot = buf[1] + (C+2) pe: [k] = level-1 plane C-2+k (k = 0..2), [3] = neighbour's plane C+1.
 // Loads bypass L1 (ld.cg): these planes are rewritten by other CTAs / the neighbour GPU.
+template <int DIM>
 __device__ bool tb_edge(const JbGeom &g, const JbSlab &SL, const JbParams &P, int role, int ridx, int rcount,
                         const double *cur, double *nxt, double *remote, int64_t tg, int *s_flag) {
   const bool top = role == ROLE_TOP;
-  const int64_t C = SL.chunk, pe = g.plane_elems, nx = g.nx;
+  const int64_t C = SL.chunk, pe = g.plane_elems, nx = g.nx, ny = g.ny, pitch = g.pitch;
   double *E = (top ? SL.buf[0] : SL.buf[1]) + (C + 2) * pe + 3;
-  double *mid = top ? SL.mid_top_out : SL.mid_bot_out;
+  double *mid = (top ? SL.mid_top_out : SL.mid_bot_out) + 3;
   const unsigned long long *fin = top ? SL.flag_in_top : SL.flag_in_bot;
   const int kin = top ? SL.k_in_top : SL.k_in_bot;
   unsigned long long *fout = (top ? SL.flag_out_top : SL.flag_out_bot) + ridx;
@@ -224,43 +383,59 @@ __device__ bool tb_edge(const JbGeom &g, const JbSlab &SL, const JbParams &P, in
     __syncthreads();
     return *s_flag == 0;
   };
-  // ---- A: level 1
+  // one stencil update of the field F (ld.cg) at element offset e = y*pitch + x of plane p
+  auto upd = [&](const double *F, int64_t e) {
+    const double *A = F + e;
+    if (DIM == 2) return 0.25 * (((__ldcg(A + 1) + __ldcg(A - 1)) + __ldcg(A + pe)) + __ldcg(A - pe));
+    return kC6 * (((((__ldcg(A + 1) + __ldcg(A - 1)) + __ldcg(A + pitch)) + __ldcg(A - pitch)) + __ldcg(A + pe)) +
+                  __ldcg(A - pe));
+  };
+  // ---- A: level 1 of 3 planes over each tile window [y0-1, y0+ty] x [x0-1, x0+tx] (clamped)
   if (!wait((unsigned long long)tg)) return false;
-  const int64_t pa = top ? 1 : C - 2;  // level-1 plane of E index (top ? 1 : 0)
+  const int64_t pa = top ? 1 : C - 2;  // plane of E index e0
   const int e0 = top ? 1 : 0;
   const int64_t pout = top ? 1 : C;    // the plane the neighbour needs
   for (int u = ub; u < ue; ++u) {
-    const int64_t x0 = 1 + (int64_t)u * g.tx;
-    const int64_t xa = max(x0 - 1, (int64_t)0), xb = min(x0 + g.tx, nx - 1);
-    const int64_t w = xb - xa + 1;
-    for (int64_t i = tid; i < 3 * w; i += nt) {
-      const int k = (int)(i / w);
-      const int64_t x = xa + (i - k * w), p = pa + k;
-      const double *A = cur + p * pe + 3 + x;
-      double v = __ldcg(A);
-      if (x >= 1 && x <= nx - 2) {  // oracle order: ((x+1) + (x-1)) + (y+1) + (y-1), then * 0.25
-        v = 0.25 * (((__ldcg(A + 1) + __ldcg(A - 1)) + __ldcg(A + pe)) + __ldcg(A - pe));
-      }
-      E[(e0 + k) * pe + x] = v;
-      if (p == pout) mid[3 + x] = v;
+    const int ux = u % g.units_x, uy = u / g.units_x;
+    const int64_t x0 = 1 + (int64_t)ux * g.tx;
+    const int64_t xa = max(x0 - 1, (int64_t)0), xb = min(x0 + g.tx, nx - 1), w = xb - xa + 1;
+    int64_t ya = 0, h = 1;
+    if (DIM == 3) {
+      const int64_t y0 = 1 + (int64_t)uy * g.ty;
+      ya = max(y0 - 1, (int64_t)0);
+      h = min(y0 + g.ty, ny - 1) - ya + 1;
+    }
+    for (int64_t i = tid; i < 3 * h * w; i += nt) {
+      const int64_t k = i / (h * w), r = i - k * h * w, yy = r / w;
+      const int64_t x = xa + (r - yy * w), y = ya + yy, p = pa + k;
+      const int64_t e = (DIM == 3 ? y * pitch : 0) + x;
+      const bool in = x >= 1 && x <= nx - 2 && (DIM == 2 || (y >= 1 && y <= ny - 2));
+      const double v = in ? upd(cur + p * pe + 3, e) : __ldcg(cur + p * pe + 3 + e);
+      E[(e0 + k) * pe + e] = v;
+      if (p == pout) mid[e] = v;
     }
   }
   __syncthreads();  // every thread's stores (local E, neighbour's slot) precede the release below
   if (tid == 0 && !drop) st_release_sys(fout, (unsigned long long)(tg + 1));
-  // ---- B: level 2
+  // ---- B: level 2 of the 2 outermost planes over each tile's interior cells
   if (!wait((unsigned long long)(tg + 1))) return false;
-  const int64_t pb = top ? 1 : C - 1;  // first level-2 plane; E index of plane pb + k is e1 + k
-  const int e1 = 1;
+  const int64_t pb = top ? 1 : C - 1;  // level-2 planes pb, pb+1 <-> E indices 1, 2
   for (int u = ub; u < ue; ++u) {
-    const int64_t x0 = 1 + (int64_t)u * g.tx;
+    const int ux = u % g.units_x, uy = u / g.units_x;
+    const int64_t x0 = 1 + (int64_t)ux * g.tx;
     const int64_t w = min((int64_t)g.tx, nx - 1 - x0);
-    for (int64_t i = tid; i < 2 * w; i += nt) {
-      const int k = (int)(i / w);
-      const int64_t x = x0 + (i - k * w), p = pb + k;
-      const double *L = E + (e1 + k) * pe + x;
-      const double v = 0.25 * (((__ldcg(L + 1) + __ldcg(L - 1)) + __ldcg(L + pe)) + __ldcg(L - pe));
-      nxt[p * pe + 3 + x] = v;
-      if (p == pout) remote[3 + x] = v;
+    int64_t y0 = 0, h = 1;
+    if (DIM == 3) {
+      y0 = 1 + (int64_t)uy * g.ty;
+      h = min((int64_t)g.ty, ny - 1 - y0);
+    }
+    for (int64_t i = tid; i < 2 * h * w; i += nt) {
+      const int64_t k = i / (h * w), r = i - k * h * w, yy = r / w;
+      const int64_t x = x0 + (r - yy * w), p = pb + k;
+      const int64_t e = (DIM == 3 ? (y0 + yy) * pitch : 0) + x;
+      const double v = upd(E + (1 + k) * pe, e);
+      nxt[p * pe + 3 + e] = v;
+      if (p == pout) remote[3 + e] = v;
     }
   }
   __syncthreads();
@@ -268,7 +443,7 @@ __device__ bool tb_edge(const JbGeom &g, const JbSlab &SL, const JbParams &P, in
   return true;
 }
 
-template <int NCW, int PPT>
+template <int NCW, int DIM, int TP>
 __device__ __forceinline__ void tb_body(const JbParams &P) {
   extern __shared__ __align__(128) unsigned char smem[];
   __shared__ int s_abort;
@@ -321,7 +496,7 @@ __device__ __forceinline__ void tb_body(const JbParams &P) {
     const int64_t tg = P.t0 + TB_K * j;  // global iteration at the start of this time block
     if (role != ROLE_INT) {  // edge zone with its per-iteration exchange, then help the interior
       double *remote = role == ROLE_TOP ? SL.peer_top[(P.t0 + j + 1) & 1] : SL.peer_bot[(P.t0 + j + 1) & 1];
-      if (!tb_edge(g, SL, P, role, ridx, rcount, cur, nxt, remote, tg, &s_abort)) return;
+      if (!tb_edge<DIM>(g, SL, P, role, ridx, rcount, cur, nxt, remote, tg, &s_abort)) return;
       fence_proxy_async_global();  // our generic-proxy stores before later bulk reads
     }
     if (producer) {
@@ -352,19 +527,29 @@ __device__ __forceinline__ void tb_body(const JbParams &P) {
           d.pad = 0;
           desc[rq.slot] = d;
           mbar_arrive(&qfull[rq.slot]);
-          // level-0 rows r0..r1 of the strip: one bulk copy of the x window [x0-2, x0+tx+2)
-          const int64_t xs = 2 + (int64_t)unit * g.tx;
-          const int64_t xe = min(xs + g.tx + 4, g.pitch);
-          const uint32_t bytes = (uint32_t)((xe - xs) * 8);
-          const double *src = cur + xs;
-          for (int64_t p = r0; p <= r1; ++p) {
+        }
+        // level-0 rows r0..r1 of the tile: x window [x0-2, x0+tx+2) of rows y0-2 .. y0+TY+1
+        // (3D; stage row i <-> y0-2+i, rows outside the grid are not loaded), one bulk copy
+        // per row and lane
+        const int ux = unit % g.units_x, uy = unit / g.units_x;
+        const int64_t xs = 2 + (int64_t)ux * g.tx;
+        const int64_t xe = min(xs + g.tx + 4, g.pitch);
+        const uint32_t bytes = (uint32_t)((xe - xs) * 8);
+        const int64_t ya = DIM == 3 ? (int64_t)uy * g.ty - 1 : 0;  // = y0 - 2
+        const int nrow = DIM == 3 ? g.rh : 1;
+        const int64_t yl = max(ya, (int64_t)0), yh = DIM == 3 ? min(ya + nrow - 1, g.ny - 1) : 0;
+        const uint32_t nvalid = (uint32_t)(yh - yl + 1);
+        const int64_t yrow = ya + lane;
+        const bool mine = lane < nrow && (DIM == 2 || (yrow >= 0 && yrow <= g.ny - 1));
+        const double *src = cur + xs + (DIM == 3 ? yrow * g.pitch : 0);
+        for (int64_t p = r0; p <= r1; ++p) {
+          if (lane == 0) {
             mbar_wait(&R.empty[q.slot], q.phase ^ 1u);
-            mbar_expect_tx(&R.full[q.slot], bytes);
-            bulk_g2s(R.stage(q), src + p * g.plane_elems, bytes, &R.full[q.slot]);
-            q.advance(R.S);
+            mbar_expect_tx(&R.full[q.slot], bytes * nvalid);
           }
-        } else {
-          for (int64_t p = r0; p <= r1; ++p) q.advance(R.S);
+          __syncwarp();
+          if (mine) bulk_g2s(R.stage(q) + (size_t)lane * g.ws, src + p * g.plane_elems, bytes, &R.full[q.slot]);
+          q.advance(R.S);
         }
         rq.advance(JB_RQ);
         if (!early && lane == 0) claim = atomicAdd(ctr, 1u);
@@ -384,7 +569,8 @@ __device__ __forceinline__ void tb_body(const JbParams &P) {
         if (lane == 0) mbar_arrive(&qempty[rq.slot]);
         rq.advance(JB_RQ);
         if (d.kind == TB_END) break;
-        tb2_item<PPT>(g, R, q, d.unit, d.a, d.b, C, nxt, warp, lane);
+        if (DIM == 2) tb2_item<TP>(g, R, q, d.unit, d.a, d.b, C, nxt, warp, lane);
+        else tb3_item<TP>(g, R, q, d.unit, d.a, d.b, C, nxt, warp, lane);
       }
       fence_proxy_async_global();  // generic-proxy stores before the next block's bulk reads
     }
@@ -406,20 +592,24 @@ __device__ __forceinline__ void tb_body(const JbParams &P) {
 }
 
 // One CTA per SM (up to 224 registers per thread) or two (96: 2 x 9 warps fit the register file
-// only at <= 96 registers, given the 4-warp allocation granularity).
-template <int PPT>
-__global__ void __launch_bounds__(JB_NC + 32, 1) jb_tblock2d(const __grid_constant__ JbParams P) {
-  tb_body<JB_NCW, PPT>(P);
+// only at <= 96 registers, given the 4-warp allocation granularity).  TP = pairs per thread
+// along x (2D) or rows per tile (3D).
+template <int DIM, int TP>
+__global__ void __launch_bounds__(JB_NC + 32, 1) jb_tblock(const __grid_constant__ JbParams P) {
+  tb_body<JB_NCW, DIM, TP>(P);
 }
-template <int PPT>
+template <int TP>
 __global__ void __maxnreg__(96) jb_tblock2d_x2(const __grid_constant__ JbParams P) {
-  tb_body<JB_NCW, PPT>(P);
+  tb_body<JB_NCW, 2, TP>(P);
 }
 
-const void *tblock_fn(int ppt, int per_sm) {
-#define JB_TB(K, p) reinterpret_cast<const void *>(&K<p>)
-  if (per_sm >= 2) return ppt >= 4 ? JB_TB(jb_tblock2d_x2, 4) : ppt == 2 ? JB_TB(jb_tblock2d_x2, 2) : JB_TB(jb_tblock2d_x2, 1);
-  return ppt >= 4 ? JB_TB(jb_tblock2d, 4) : ppt == 2 ? JB_TB(jb_tblock2d, 2) : JB_TB(jb_tblock2d, 1);
+constexpr int TB_TY = 4;  // 3D tile rows (level-1 rows TY+2 carried per plane in registers)
+
+const void *tblock_fn(int dim, int ppt, int per_sm) {
+#define JB_TB(K) reinterpret_cast<const void *>(&K)
+  if (dim == 3) return JB_TB((jb_tblock<3, TB_TY>));
+  if (per_sm >= 2) return ppt >= 4 ? JB_TB(jb_tblock2d_x2<4>) : ppt == 2 ? JB_TB(jb_tblock2d_x2<2>) : JB_TB(jb_tblock2d_x2<1>);
+  return ppt >= 4 ? JB_TB((jb_tblock<2, 4>)) : ppt == 2 ? JB_TB((jb_tblock<2, 2>)) : JB_TB((jb_tblock<2, 1>));
 #undef JB_TB
 }
 
@@ -428,6 +618,7 @@ const void *tblock_fn(int ppt, int per_sm) {
 namespace jbk {
 
 int tblock_k() { return TB_K; }
+int tblock_ty() { return TB_TY; }
 int tblock_threads() { return JB_NC + 32; }
 
 // Dynamic shared memory of the temporally blocked kernel: header + ring stages.
@@ -437,7 +628,7 @@ size_t tblock_smem(const JbGeom &g) {
 }
 
 cudaError_t prepare_tblock(const JbGeom &g, int per_sm, size_t smem, int *blocks_per_sm) {
-  const void *fn = tblock_fn(g.tx / (2 * JB_NC), per_sm);
+  const void *fn = tblock_fn(g.dim, g.tx / (2 * JB_NC), per_sm);
   cudaError_t e = cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
   if (e != cudaSuccess) return e;
   e = cudaFuncSetAttribute(fn, cudaFuncAttributePreferredSharedMemoryCarveout, (int)cudaSharedmemCarveoutMaxShared);
@@ -447,7 +638,7 @@ cudaError_t prepare_tblock(const JbGeom &g, int per_sm, size_t smem, int *blocks
 
 cudaError_t launch_tblock(const JbParams &p, int per_sm, int grid, size_t smem, cudaStream_t st) {
   void *args[] = {const_cast<JbParams *>(&p)};
-  return cudaLaunchCooperativeKernel(tblock_fn(p.g.tx / (2 * JB_NC), per_sm), dim3(grid), dim3(JB_NC + 32), args, smem,
+  return cudaLaunchCooperativeKernel(tblock_fn(p.g.dim, p.g.tx / (2 * JB_NC), per_sm), dim3(grid), dim3(JB_NC + 32), args, smem,
                                      st);
 }
 

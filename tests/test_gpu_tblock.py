@@ -119,8 +119,9 @@ def test_tblock_auto_selection_and_errors():
         j.set_mode(jb.MODE_CPUFREE, jb.FLAG_NO_COMPUTE)  # no-compute runs keep jb_sweep
         with pytest.raises(jb.JacobiError):
             j.run(4)
-    with jb.Jacobi((6, 8, 10)) as j:  # 3D: per-iteration kernels
+    with jb.Jacobi((6, 8, 10)) as j:  # 3D with the norm: per-iteration kernels only
         j.set_param("tblock", 1)
+        j.set_tolerance(0.0, 2)
         with pytest.raises(jb.JacobiError):
             j.run(4)
 
@@ -244,3 +245,74 @@ def test_c2_1000_iters_tblock_p8_equals_p1():
         j.set_param("tblock", 0)
         j.run(1000)
         assert_bitwise(j.gather(), ref, "per-iteration kernel")
+
+
+# ---------------------------------------------------------------- 3D (7-point)
+@pytest.mark.parametrize("shape", [(3, 3, 3), (5, 6, 7), (10, 13, 70), (20, 37, 130), (9, 17, 600),
+                                   (12, 23, 1100), (40, 9, 8), (7, 70, 40)])
+@pytest.mark.parametrize("iters", [4, 5, 13])
+def test_tblock_3d_shapes(shape, iters):
+    """3D tiles of 4 rows (ragged last tile in y and x, tiles narrower than a warp, nz from 3)."""
+    f = u12(shape, 11)
+    got, tb = run_tb(f, iters)
+    assert tb == iters // 4 * 4
+    assert_bitwise(got, oracle.jacobi(f, iters), f"3D tblock {shape} it{iters}")
+
+
+@pytest.mark.parametrize("tile_x,min_block", [(8, 1), (16, 2), (64, 1), (128, 5)])
+def test_tblock_3d_tiles(tile_x, min_block):
+    f = u12((21, 30, 150), 12)
+    got, _ = run_tb(f, 8, {"tile_x": tile_x, "tb_min_block": min_block})
+    assert_bitwise(got, oracle.jacobi(f, 8), f"3D tx{tile_x}")
+
+
+@pytest.mark.parametrize("P", [2, 3, 4])
+def test_tblock_3d_virtual_slabs(P):
+    f = u12((4 * P + 5, 26, 70), 13)
+    got, tb = run_tb_virtual(f, 13, P)
+    assert tb == 12
+    assert_bitwise(got, oracle.jacobi(f, 13), f"3D P={P}")
+
+
+def test_tblock_3d_invariants_and_mixing():
+    z, y, x = np.mgrid[0:12, 0:13, 0:30].astype(np.float64)
+    for h in (1 + x + 2 * y - 3 * z, x * x + y * y - 2 * z * z, x * y + y * z + z * x):
+        got, _ = run_tb(np.ascontiguousarray(h), 16)
+        assert_bitwise(got, h, "3D harmonic field stationary")
+    f = u12((30, 20, 100), 14)
+    exp = oracle.jacobi(f, 23)
+    got, _ = run_tb(f, 23, runs=[4, 3, 8, 1, 4, 3])
+    assert_bitwise(got, exp, "3D split")
+    with jb.Jacobi(f.shape, virtual=2) as j:
+        j.set_param("resident", 0)
+        j.scatter(f)
+        j.run(8)
+        assert j.get_param("last_tblock") == 8
+        j.set_mode(jb.MODE_BASELINE_MEMCPY)
+        j.run(3)
+        j.set_mode(jb.MODE_CPUFREE)
+        j.run(12)
+        assert_bitwise(j.gather(), exp, "3D mixed P=2")
+
+
+def test_tblock_3d_auto_is_per_iteration():
+    with jb.Jacobi((20, 30, 40)) as j:
+        j.set_param("resident", 0)
+        j.run(8)
+        assert j.get_param("last_tblock") == 0
+
+
+def test_c3_1000_iters_tblock_equals_per_iteration():
+    """C3 full size, 1000 iterations: the time-blocked kernel (P = 1 and P = 4 slabs) == the
+    per-iteration kernel, bit for bit."""
+    shape = (512, 512, 512)
+    with jb.Jacobi(shape) as j:
+        j.set_param("tblock", 0)
+        j.run(1000)
+        ref = j.gather()
+    for P in (0, 4):
+        with (jb.Jacobi(shape, virtual=P) if P else jb.Jacobi(shape)) as j:
+            j.set_param("tblock", 1)
+            j.run(1000)
+            assert j.get_param("last_tblock") == 1000
+            assert_bitwise(j.gather(), ref, f"C3 tblock P={P or 1}")
