@@ -285,6 +285,7 @@ def test_tblock_3d_invariants_and_mixing():
     assert_bitwise(got, exp, "3D split")
     with jb.Jacobi(f.shape, virtual=2) as j:
         j.set_param("resident", 0)
+        j.set_param("tblock", 1)
         j.scatter(f)
         j.run(8)
         assert j.get_param("last_tblock") == 8
