@@ -447,6 +447,7 @@ template <int NCW, int DIM, int TP>
 __device__ __forceinline__ void tb_body(const JbParams &P) {
   extern __shared__ __align__(128) unsigned char smem[];
   __shared__ int s_abort;
+  __shared__ int s_edge;  // the edge zones' wait result (own variable: s_abort is read after the barrier)
   const JbGeom &g = P.g;
   int si = 0;
   while (si + 1 < P.nslabs && (int)blockIdx.x >= P.s[si + 1].cta_begin) ++si;
@@ -496,7 +497,7 @@ __device__ __forceinline__ void tb_body(const JbParams &P) {
     const int64_t tg = P.t0 + TB_K * j;  // global iteration at the start of this time block
     if (role != ROLE_INT) {  // edge zone with its per-iteration exchange, then help the interior
       double *remote = role == ROLE_TOP ? SL.peer_top[(P.t0 + j + 1) & 1] : SL.peer_bot[(P.t0 + j + 1) & 1];
-      if (!tb_edge<DIM>(g, SL, P, role, ridx, rcount, cur, nxt, remote, tg, &s_abort)) return;
+      if (!tb_edge<DIM>(g, SL, P, role, ridx, rcount, cur, nxt, remote, tg, &s_edge)) return;
       fence_proxy_async_global();  // our generic-proxy stores before later bulk reads
     }
     if (producer) {

@@ -22,4 +22,13 @@ for shape, P in [((20, 70), 2), ((8, 9, 33), 2), ((30, 40), 1)]:
             j.scatter(f)
             j.run(3)
             ok &= bool(np.array_equal(j.gather(), oracle.jacobi(f, 3)))
+# time-blocked kernel (2D and 3D, with and without neighbours): TMA ring, shuffles, edge zones
+for shape, P in [((20, 70), 2), ((12, 9, 33), 2), ((30, 40), 1)]:
+    f = u12(shape, 4)
+    with jb.Jacobi(shape, virtual=P) if P > 1 else jb.Jacobi(shape) as j:
+        j.set_param("tblock", 1)
+        j.set_param("resident", 0)
+        j.scatter(f)
+        j.run(8)
+        ok &= bool(np.array_equal(j.gather(), oracle.jacobi(f, 8)))
 print("SANITIZE_CASE_OK" if ok else "SANITIZE_CASE_MISMATCH")

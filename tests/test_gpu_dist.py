@@ -21,7 +21,7 @@ def _free_port():
     return p
 
 
-def _worker(rank, world, port, shape, iters, q, torch_alloc=False, tol=None):
+def _worker(rank, world, port, shape, iters, q, torch_alloc=False, tol=None, params=None):
     try:
         os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
         import torch.distributed as dist
@@ -33,6 +33,8 @@ def _worker(rank, world, port, shape, iters, q, torch_alloc=False, tol=None):
             jb.use_torch_allocator()
         j = jb.Jacobi(shape, dist=(rank, world), device=0)
         j.set_param("timeout_ms", 60000)
+        for k, v in (params or {}).items():
+            j.set_param(k, v)
         jb.exchange_peers(j, nccl=False)
         j.scatter(f)
         if tol is not None:  # N4: device-side norm all-reduce across the two processes
@@ -53,16 +55,20 @@ def _worker(rank, world, port, shape, iters, q, torch_alloc=False, tol=None):
         q.put((rank, None, repr(e)))
 
 
-@pytest.mark.parametrize("shape,iters,torch_alloc", [((40, 96), 5, False), ((11, 12, 40), 3, False),
-                                                     ((40, 96), 4, True)])
-def test_two_ranks_one_gpu_ipc(shape, iters, torch_alloc):
+TB = {"tblock": 1, "resident": 0}  # the time-blocked kernel's edge zones across two processes
+
+
+@pytest.mark.parametrize("shape,iters,torch_alloc,params", [((40, 96), 5, False, None), ((11, 12, 40), 3, False, None),
+                                                            ((40, 96), 4, True, None), ((40, 96), 9, False, TB),
+                                                            ((40, 96), 8, True, TB), ((14, 12, 40), 9, False, TB)])
+def test_two_ranks_one_gpu_ipc(shape, iters, torch_alloc, params):
     import oracle
     from jacobi_inputs import u12
     ctx = mp.get_context("spawn")
     q = ctx.Queue()
     port = _free_port()
     world = 2
-    procs = [ctx.Process(target=_worker, args=(r, world, port, shape, iters, q, torch_alloc))
+    procs = [ctx.Process(target=_worker, args=(r, world, port, shape, iters, q, torch_alloc, None, params))
              for r in range(world)]
     for p in procs:
         p.start()
