@@ -18,6 +18,8 @@
 // (out of place — neighbouring strips still read the time-t columns of this strip); the host
 // runs an even number of blocks, so the result lands in buf[(t0 + 2 nb) & 1] as in every other
 // path (R10).
+#include <type_traits>
+
 #include "device_common.cuh"
 
 namespace {
@@ -50,9 +52,10 @@ struct TbSeg {
 
 // Level 1 (t+1) of this lane's pairs and extra cell on the row whose level-0 stages are
 // sm (row-1), sc (row), sn (row+1); rows outside 1..C keep level 0 (rowin = false).
-template <int PPT, bool FAST>
+template <int PPT, bool FAST, bool ROWIN>
 __device__ __forceinline__ void tb_level1(const TbSeg &L, const double *sm, const double *sc, const double *sn,
-                                          bool rowin, double2 *V, double &ex) {
+                                          bool rowin_rt, double2 *V, double &ex) {
+  const bool rowin = ROWIN || rowin_rt;
 #pragma unroll
   for (int i = 0; i < PPT; ++i) {
     const int j = L.j0 + 64 * i;
@@ -105,43 +108,65 @@ __device__ __forceinline__ void tb_level2(const TbSeg &L, const double2 *S1, con
 template <int PPT, bool FAST>
 __device__ __forceinline__ void tb2_march(const TbSeg &L, const Ring &R, RingPos q, int64_t a, int64_t b,
                                           int64_t C, int64_t r0, int64_t r1, double *dst, int64_t pe, int lane) {
-  double2 S1[PPT], C1[PPT], N1[PPT];
-  double exl_c, exl_n, exr_c, exr_n, ex;
+  // Level-1 rows live in three register sets X0, X1, X2 whose roles (y-1, y, y+1) rotate with
+  // the march; the loop is unrolled by three so the rotation is static (no register moves).
+  // Extras: lane 0 holds the left one, lane 1 the right one, one slot per set.
+  double2 X0[PPT], X1[PPT], X2[PPT];
+  double e0, e1, e2;
   // Level-1 row q1 reads level-0 rows max(q1-1, r0), q1, min(q1+1, r1): ring positions pm, pc,
   // pn, advanced by one stage per row (row a-2 exists iff r0 = a-2).
   RingPos pc = ring_add(q, (uint32_t)(a - 1 - r0), R.S);
   RingPos pm = a - 2 >= r0 ? q : pc;
   R.wait_full(pm);
   R.wait_full(pc);
-  auto row = [&](int64_t q1, double2 *out) {
+  // rows 1..C are interior (compile-time in the steady state); 0 and C+1 keep level 0
+  auto row = [&](auto rowin_ct, int64_t q1, double2 *out, double &e) {
     RingPos pn = pc;
     if (q1 + 1 <= r1) pn.advance(R.S);
     R.wait_full(pn);
-    tb_level1<PPT, FAST>(L, R.stage(pm), R.stage(pc), R.stage(pn), q1 >= 1 && q1 <= C, out, ex);
+    double ex;
+    tb_level1<PPT, FAST, decltype(rowin_ct)::value>(L, R.stage(pm), R.stage(pc), R.stage(pn),
+                                                    q1 >= 1 && q1 <= C, out, ex);
+    e = ex;
     if (q1 - 1 >= r0) R.release(pm, lane);  // row q1-1 is no longer needed
     pm = pc;
     pc = pn;
   };
-  // prologue: level-1 rows a-1 and a; extras: lane 0 holds the left one, lane 1 the right one
-  row(a - 1, C1);
-  exl_c = __shfl_sync(0xffffffffu, ex, 0);
-  exr_c = __shfl_sync(0xffffffffu, ex, 1);
-  row(a, N1);
-  exl_n = __shfl_sync(0xffffffffu, ex, 0);
-  exr_n = __shfl_sync(0xffffffffu, ex, 1);
+  using RT = std::integral_constant<bool, true>;
+  using RF = std::integral_constant<bool, false>;
   double *o = dst + a * pe;
-  for (int64_t q1 = a + 1; q1 <= b + 1; ++q1) {
-#pragma unroll
-    for (int i = 0; i < PPT; ++i) S1[i] = C1[i];
-#pragma unroll
-    for (int i = 0; i < PPT; ++i) C1[i] = N1[i];
-    exl_c = exl_n;
-    exr_c = exr_n;
-    row(q1, N1);
-    exl_n = __shfl_sync(0xffffffffu, ex, 0);
-    exr_n = __shfl_sync(0xffffffffu, ex, 1);
-    tb_level2<PPT, FAST>(L, S1, C1, N1, exl_c, exr_c, lane, o);
+  // level 2 of the middle row from (S, C, N); extras of the middle row: shuffles from lanes 0/1
+  auto lvl2 = [&](const double2 *S, const double2 *Cm, const double2 *N, double em) {
+    const double exl = __shfl_sync(0xffffffffu, em, 0), exr = __shfl_sync(0xffffffffu, em, 1);
+    tb_level2<PPT, FAST>(L, S, Cm, N, exl, exr, lane, o);
     o += pe;
+  };
+  row(RF{}, a - 1, X0, e0);  // may be the Dirichlet row 0
+  row(RT{}, a, X1, e1);      // a >= 1
+  const int64_t qe = min(b + 1, C);  // last interior level-1 row of the march
+  int64_t q1 = a + 1;
+  for (; q1 + 2 <= qe; q1 += 3) {
+    row(RT{}, q1, X2, e2);
+    lvl2(X0, X1, X2, e1);
+    row(RT{}, q1 + 1, X0, e0);
+    lvl2(X1, X2, X0, e2);
+    row(RT{}, q1 + 2, X1, e1);
+    lvl2(X2, X0, X1, e0);
+  }
+  // 0-2 interior rows left, then (b == C) the Dirichlet row C+1; the set roles continue the cycle
+  // (left <= 3)
+  const int64_t left = qe - q1 + 1 + (b + 1 > C ? 1 : 0);
+  if (left >= 1) {
+    if (q1 <= C) row(RT{}, q1, X2, e2); else row(RF{}, q1, X2, e2);
+    lvl2(X0, X1, X2, e1);
+  }
+  if (left >= 2) {
+    if (q1 + 1 <= C) row(RT{}, q1 + 1, X0, e0); else row(RF{}, q1 + 1, X0, e0);
+    lvl2(X1, X2, X0, e2);
+  }
+  if (left >= 3) {  // two interior rows + the Dirichlet row C+1
+    row(RF{}, q1 + 2, X1, e1);
+    lvl2(X2, X0, X1, e0);
   }
   // rows b+1 .. r1 were not released by the march
   RingPos pr = ring_add(q, (uint32_t)(b + 1 - r0), R.S);
