@@ -297,12 +297,12 @@ def main():
     peak, peak_kind = measured_hbm()
     launch_ms = dev_ms_local / args.steps
     tb_iters = jb.jacobi_get_param(j.h, "last_tblock")
-    tb_k = 2
-    alg_bytes = local_cells * (16 * (iters - tb_iters) + 16 // tb_k * tb_iters)
+    tb_k = max(jb.jacobi_get_param(j.h, "last_tb_k"), 1)
+    alg_bytes = round(local_cells * (16 * (iters - tb_iters) + 16 / tb_k * tb_iters))
     achieved = alg_bytes / (launch_ms / 1e3) / 1e9
     dimk = 2 if shape[0] == 1 else 3
     if tb_iters:
-        kname = f"jb_tblock2d<8,*> (persistent CPU-Free kernel, {tb_k} iterations per HBM pass)"
+        kname = f"jb_tblock<{dimk},{tb_k},*> (persistent CPU-Free kernel, {tb_k} iterations per HBM pass)"
         kkind = "tblock"
     elif jb.jacobi_get_param(j.h, "last_resident"):
         kname = f"jb_resident<{dimk},*> (persistent CPU-Free kernel, on-chip resident)"

@@ -15,7 +15,14 @@
 #define JB_MAX_BLOCKS 1024      // per-slab block flags of the resident kernel
 #define JB_RCPP_MAX 8           // max cell pairs per thread held in registers by the resident kernel
 #define JB_SMEM_DEFAULT 232448  // B200 opt-in dynamic shared memory per block (227 KB)
-#define JB_EDGE_PLANES 4        // scratch planes after each slab buffer: time-blocked edge zones (tblock.cu)
+#define JB_TB_KMAX2 5           // deepest time block of the 2D time-blocked kernel (tblock.cu)
+#define JB_TB_K2D 5             // its default depth (auto; measured fastest)
+
+// Scratch planes after each slab buffer for the time-blocked kernel's edge zones of depth K
+// (tblock.cu): K-1 slots for the neighbour's intermediate levels + the side's own level-m planes,
+// 2K-m of them for m = 1..K-1.  2D buffers carry enough for JB_TB_KMAX2, 3D ones for K = 2.
+static inline int64_t jb_edge_planes_k(int K) { return (K - 1) + (int64_t)(K - 1) * 2 * K - (int64_t)(K - 1) * K / 2; }
+static inline int64_t jb_edge_planes(int dim) { return jb_edge_planes_k(dim == 2 ? JB_TB_KMAX2 : 2); }
 
 // Grid geometry in HBM and the tile shape of the march.
 //   element (x, y, z) of slab plane p lives at  buf + p*plane_elems + y*pitch + (x + 3)
@@ -91,11 +98,11 @@ struct JbSlab {
   int32_t use_shm;
   int32_t shm_pe_top, shm_pe_bot;
   int32_t pad3;
-  // Temporally blocked kernel (tblock.cu): interior level-2 planes tb_lo..tb_hi (dynamic items),
-  // and the neighbours' intermediate-level halo slots this slab writes: the top neighbour's
-  // bottom slot (its E_bot[3]) and the bottom neighbour's top slot (its E_top[0]).  A slab's own
-  // edge scratch: E_top = buf[0] + (chunk+2)*plane_elems, E_bot = buf[1] + (chunk+2)*plane_elems,
-  // JB_EDGE_PLANES planes each.
+  // Temporally blocked kernel (tblock.cu): interior level-K planes tb_lo..tb_hi (dynamic items),
+  // and the neighbours' intermediate-level slots this slab writes: the top neighbour's bottom
+  // scratch (its E_bot) and the bottom neighbour's top scratch (its E_top); slot m-1 holds level m.
+  // A slab's own edge scratch: E_top = buf[0] + (chunk+2)*plane_elems, E_bot = buf[1] +
+  // (chunk+2)*plane_elems, jb_edge_planes(dim) planes each.
   int64_t tb_lo, tb_hi;
   double *mid_top_out;
   double *mid_bot_out;

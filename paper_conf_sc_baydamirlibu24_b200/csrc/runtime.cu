@@ -32,12 +32,12 @@ jacobi_ctx *new_ctx(int64_t nx, int64_t ny, int64_t nz, int stencil, int total) 
 
 int alloc_slab(jacobi_ctx *h, Slab &s) {
   CK(cudaSetDevice(s.device));
-  // (chunk + 2) planes of the slab + JB_EDGE_PLANES scratch planes (time-blocked edge zones)
-  size_t bytes = (size_t)(s.chunk + 2 + JB_EDGE_PLANES) * h->geom.plane_elems * sizeof(double);
+  // (chunk + 2) planes of the slab + jb_edge_planes(h->dim) scratch planes (time-blocked edge zones)
+  size_t bytes = (size_t)(s.chunk + 2 + jb_edge_planes(h->dim)) * h->geom.plane_elems * sizeof(double);
   if (h->kind == KIND_SHMEM) {  // symmetric heap: every PE allocates the largest slab
     int64_t st, chunk_max;
     jbplan::decompose(h->n_out, h->total, 0, &st, &chunk_max);
-    bytes = (size_t)(chunk_max + 2 + JB_EDGE_PLANES) * h->geom.plane_elems * sizeof(double);
+    bytes = (size_t)(chunk_max + 2 + jb_edge_planes(h->dim)) * h->geom.plane_elems * sizeof(double);
   }
   if (h->alloc.alloc) {
     s.buf[0] = static_cast<double *>(h->alloc.alloc(bytes, s.device, h->alloc.user));
@@ -99,14 +99,14 @@ void link_local(jacobi_ctx *h) {
     if (s.has_top) {
       Slab &o = h->slabs[i - 1];
       for (int p = 0; p < 2; ++p) s.peer_top[p] = o.buf[p] + (o.chunk + 1) * pe;
-      s.mid_top_out = o.buf[1] + (o.chunk + 2 + 3) * pe;  // its E_bot[3]
+      s.mid_top_out = o.buf[1] + (o.chunk + 2) * pe;  // its E_bot (slot 0)
       s.flag_out_top = &o.ctrl->flag_in[1][0];
       s.peer_top_dev = o.device;
     }
     if (s.has_bot) {
       Slab &o = h->slabs[i + 1];
       for (int p = 0; p < 2; ++p) s.peer_bot[p] = o.buf[p];
-      s.mid_bot_out = o.buf[0] + (o.chunk + 2) * pe;  // its E_top[0]
+      s.mid_bot_out = o.buf[0] + (o.chunk + 2) * pe;  // its E_top (slot 0)
       s.flag_out_bot = &o.ctrl->flag_in[0][0];
       s.peer_bot_dev = o.device;
     }
@@ -561,10 +561,26 @@ int run_cpufree_k1(jacobi_ctx *h, int64_t iters) {
 // iterations: per launch group the roles and flags of plan_launch (boundary CTAs run the edge
 // zones with the per-iteration exchange, then join the interior), the guided dynamic schedule
 // over the interior planes the edge zones leave, and the ring shortened to the smem budget.
-int run_tblock(jacobi_ctx *h, int64_t iters) {
+void tblock_choice(const jacobi_ctx *h, int *k_out, int *ppt_out) {
+  int k = h->tb_k >= 2 ? (int)std::min<int64_t>(h->tb_k, JB_TB_KMAX2) : (h->dim == 2 ? JB_TB_K2D : 2);
+  if (h->dim == 3) k = 2;
+  // every slab needs its edge zones (2K planes) when it has neighbours: shallower blocks otherwise
+  const int64_t chunk_min = (h->n_out - 2) / h->total;
+  auto fits = [&](int kk) { return h->total == 1 || chunk_min >= 2 * kk; };
+  while (k > 2 && !(fits(k) && jbk::tblock_ncw(h->dim, k, k == 5 ? 2 : 4, 1) > 0)) k -= (k == 3 ? 1 : 2);
+  int ppt = 4;
+  if (k == 5) ppt = 2;
+  if (h->tb_ppt > 0 && h->dim == 2 && jbk::tblock_ncw(2, k, (int)h->tb_ppt, 1) > 0) ppt = (int)h->tb_ppt;
+  if (!fits(k)) k = 0;
+  *k_out = k;
+  *ppt_out = ppt;
+}
+
+int run_tblock(jacobi_ctx *h, int64_t iters, int K, int ppt) {
   auto groups = launch_groups(h);
   std::vector<LaunchPlan> plans(groups.size());
-  const int per_sm = (h->tb_ctas >= 2 && h->total == 1) ? 2 : 1;  // roles must match across slabs
+  // roles must match across slabs; two CTAs per SM only for K = 2
+  const int per_sm = (h->tb_ctas >= 2 && h->total == 1 && K == 2) ? 2 : 1;
   for (size_t gi = 0; gi < groups.size(); ++gi) {
     LaunchPlan &L = plans[gi];
     const int64_t sched = h->schedule;
@@ -581,14 +597,23 @@ int run_tblock(jacobi_ctx *h, int64_t iters) {
       g.units_y = (int)((h->ny - 2 + g.ty - 1) / g.ty);
       g.units = g.units_x * g.units_y;
       g.stage_doubles = g.rh * g.ws;
+    } else if (K > 2) {  // odd K: JB_NCW warps x (64 ppt - 2(K-1)) output columns per strip
+      g.tx = jbk::tblock_ncw(2, K, ppt, 1) * (64 * ppt - 2 * (K - 1));
+      g.ws = g.tx + 2 * K + 2;
+      g.units_x = (int)((h->nx - 2 + g.tx - 1) / g.tx);
+      g.units_y = 1;
+      g.units = g.units_x;
+      g.stage_doubles = g.ws;
+    } else {  // K = 2: the strip of plan_launch (tile_x), ppt pairs per thread cover it
+      ppt = g.tx >= 4 * JB_NC * 2 ? 4 : g.tx >= 2 * JB_NC * 2 ? 2 : 1;
     }
     g.stages = (int)(h->stages > 0 ? std::min<int64_t>(h->stages, JB_MAX_STAGES) : JB_MAX_STAGES);
     const int min_blk = (int)std::max<int64_t>(1, h->tb_min_block);
     for (size_t k = 0; k < groups[gi].size(); ++k) {
       Slab &s = h->slabs[groups[gi][k]];
       JbSlab &d = L.P.s[k];
-      d.tb_lo = s.has_top ? 3 : 1;  // edge zones: level-2 planes 1, 2 (top) and C-1, C (bottom)
-      d.tb_hi = s.has_bot ? s.chunk - 2 : s.chunk;
+      d.tb_lo = s.has_top ? K + 1 : 1;  // edge zones: level-K planes 1..K (top), C-K+1..C (bottom)
+      d.tb_hi = s.has_bot ? s.chunk - K : s.chunk;
       d.mid_top_out = s.mid_top_out;
       d.mid_bot_out = s.mid_bot_out;
       const int64_t npl = d.tb_hi - d.tb_lo + 1;
@@ -619,7 +644,7 @@ int run_tblock(jacobi_ctx *h, int64_t iters) {
     if (jbk::tblock_smem(g) > (size_t)smem_optin) return JACOBI_EINVAL;
     L.smem = jbk::tblock_smem(g);
     int occ = 0;
-    CK(jbk::prepare_tblock(g, per_sm, L.smem, &occ));
+    CK(jbk::prepare_tblock(g, K, ppt, per_sm, L.smem, &occ));
     if (occ < per_sm) {
       if (getenv("JACOBI_DEBUG")) fprintf(stderr, "[jacobi] tblock: occupancy %d < %d (smem %zu)\n", occ, per_sm, L.smem);
       return JACOBI_ENOCOOP;
@@ -641,7 +666,7 @@ int run_tblock(jacobi_ctx *h, int64_t iters) {
     CK(cudaSetDevice(L.device));
     Slab &s0 = h->slabs[L.slab_idx[0]];
     CK(cudaEventRecord(s0.ev0, L.stream));
-    CK(jbk::launch_tblock(L.P, per_sm, L.grid, L.smem, L.stream));
+    CK(jbk::launch_tblock(L.P, K, ppt, per_sm, L.grid, L.smem, L.stream));
     CK(cudaEventRecord(s0.ev1, L.stream));
   }
   int rc_all = JACOBI_OK;
@@ -668,17 +693,20 @@ int run_tblock(jacobi_ctx *h, int64_t iters) {
 // the per-iteration kernels (streaming / resident) for the rest.  Device times add up.
 int run_cpufree(jacobi_ctx *h, int64_t iters) {
   h->last_tblock = 0;
+  h->last_tb_k = 0;
   h->last_resident = 0;
   const bool nocomp = h->flags & JACOBI_FLAG_NO_COMPUTE;
-  // P > 1: every slab needs the two edge zones (>= 4 planes); the NVSHMEM variant keeps jb_sweep
-  const bool eligible = h->tblock != 0 && !nocomp && h->norm_every <= 0 &&
-                        h->kind != KIND_SHMEM && (h->total == 1 || (h->n_out - 2) / h->total >= 4);
+  // P > 1: every slab needs the two edge zones (>= 2K planes); the NVSHMEM variant keeps jb_sweep
+  int K = 0, ppt = 0;
+  tblock_choice(h, &K, &ppt);
+  const bool eligible = h->tblock != 0 && !nocomp && h->norm_every <= 0 && h->kind != KIND_SHMEM && K >= 2;
   if (h->tblock == 1 && !eligible) return JACOBI_EINVAL;
   // auto picks it where it measured faster than the per-iteration kernel: 2D (3D: forced only)
   const bool use = eligible && (h->tblock == 1 || h->dim == 2);
   int64_t tb_iters = 0;
   if (use) {
-    const int64_t step = 2 * jbk::tblock_k();  // even block count: the result stays in buf[t & 1]
+    // odd K: any block count; K = 2: an even one (the result stays in buf[t & 1], R10)
+    const int64_t step = (K & 1) ? K : 2 * K;
     tb_iters = iters / step * step;
     if (h->tblock < 0 && h->resident != 0) {
       // auto: slabs that fit on chip run the resident kernel (faster for those small grids)
@@ -692,10 +720,11 @@ int run_cpufree(jacobi_ctx *h, int64_t iters) {
   }
   double ms = 0;
   if (tb_iters > 0) {
-    int rc = run_tblock(h, tb_iters);
+    int rc = run_tblock(h, tb_iters, K, ppt);
     if (rc) return rc;
     ms = h->last_ms_max;
     h->last_tblock = tb_iters;
+    h->last_tb_k = K;
   }
   if (iters - tb_iters > 0) {
     int rc = run_cpufree_k1(h, iters - tb_iters);
@@ -823,13 +852,17 @@ static int64_t *param_slot(jacobi_t h, const char *name) {
   if (!std::strcmp(name, "tblock")) return &h->tblock;
   if (!std::strcmp(name, "tb_min_block")) return &h->tb_min_block;
   if (!std::strcmp(name, "tb_ctas")) return &h->tb_ctas;
+  if (!std::strcmp(name, "tb_k")) return &h->tb_k;
+  if (!std::strcmp(name, "tb_ppt")) return &h->tb_ppt;
+  if (!std::strcmp(name, "last_tb_k")) return &h->last_tb_k;
   if (!std::strcmp(name, "last_tblock")) return &h->last_tblock;
   return nullptr;
 }
 
 int jacobi_set_param(jacobi_t h, const char *name, int64_t value) {
   if (!h || !name) return JACOBI_EINVAL;
-  if (!std::strcmp(name, "last_resident") || !std::strcmp(name, "last_tblock")) return JACOBI_EINVAL;  // read-only
+  if (!std::strcmp(name, "last_resident") || !std::strcmp(name, "last_tblock") || !std::strcmp(name, "last_tb_k"))
+    return JACOBI_EINVAL;  // read-only
   int64_t *p = param_slot(h, name);
   if (!p) return JACOBI_EINVAL;
   if (!std::strcmp(name, "timeout_ms")) value = value < 0 ? 20000 : value;

@@ -24,8 +24,6 @@
 
 namespace {
 
-constexpr int TB_K = 2;  // iterations per time block
-
 enum { TB_WORK = 0, TB_END = 1 };
 struct TbDesc {
   int32_t kind;
@@ -218,6 +216,167 @@ __device__ __forceinline__ void tb2_item(const JbGeom &g, const Ring &R, RingPos
   else tb2_march<PPT, false>(L, R, q0, a, b, C, r0, r1, dst, g.plane_elems, lane);
 }
 
+// ---------------------------------------------------------------- 2D, deeper time blocks (K odd)
+// K = 3, 5: levels 1 .. K of one item, no extra cells.  Warp w computes every level over the same
+// 64 PPT columns s_w .. s_w + 64 PPT - 1 (s_w = x0 + w WO - (K-1), WO = 64 PPT - 2 (K-1)): level
+// 1 from the level-0 stage (x neighbours from the stage), level k >= 2 from level k-1 in
+// registers (x neighbours by shuffles).  At the two ends of the segment a level loses one valid
+// column per side (the shuffle wraps around), so level K is valid on the middle WO columns, which
+// are this warp's outputs; neighbouring warps overlap by 2(K-1) columns, never communicate.  With
+// K odd both the level-1 loads (stage index 2 + 2 kk) and the level-K stores (column s_w + K-1,
+// odd x) stay 16-byte aligned.  Rows: the march takes one level-0 row R per step and computes
+// level k of row R-k for every k (a wavefront), so each level keeps three rows in registers;
+// register set m % 3 holds the row computed at step m (static rotation, unrolled by three).
+// Cells outside the interior (Dirichlet rows / columns, the garbage columns past the grid)
+// keep their previous level — the definition's untouched boundary — and never reach an
+// interior output.
+struct TbkLane {
+  int j0;                  // stage index of pair 0 of this lane
+  unsigned ok, full, st;   // per pair: cell x / x+1 interior; pair stored at level K
+};
+
+template <int PPT, bool FAST, bool STEADY>
+__device__ __forceinline__ void tbk_level1(const TbkLane &L, const double *sm, const double *sc, const double *sn,
+                                           bool rowin, double2 *V) {
+#pragma unroll
+  for (int i = 0; i < PPT; ++i) {
+    const int j = L.j0 + 64 * i;
+    const double2 S0 = lds2(sm + j), C0 = lds2(sc + j), N0 = lds2(sn + j);
+    const double W = sc[j - 1], E = sc[j + 2];
+    // oracle order: ((x+1) + (x-1)) + (y+1) + (y-1), then * 0.25
+    const double l0 = 0.25 * (((C0.y + W) + N0.x) + S0.x);
+    const double l1 = 0.25 * (((E + C0.x) + N0.y) + S0.y);
+    if (FAST && STEADY) {
+      V[i] = make_double2(l0, l1);
+    } else {
+      const bool r = STEADY || rowin;
+      V[i].x = (r && (FAST || (L.ok >> i & 1u))) ? l0 : C0.x;
+      V[i].y = (r && (FAST || (L.full >> i & 1u))) ? l1 : C0.y;
+    }
+  }
+}
+
+// Level k >= 2 of the middle row of (S, Cm, N) (level k-1).  Lane l takes lane l-1's .y (W) and
+// lane l+1's .x (E); lane 0 / 31 the wrapped value of the previous / next pair.  STORE: level K,
+// written to o (row pointer of this lane's pair 0) instead of V.
+template <int PPT, bool FAST, bool STEADY, bool STORE>
+__device__ __forceinline__ void tbk_levelk(const TbkLane &L, const double2 *S, const double2 *Cm, const double2 *N,
+                                           bool rowin, int lane, double2 *V, double *o) {
+  double rw_prev = Cm[0].x;  // lane 0, pair 0: outside the valid span (any finite value)
+  double re_next = __shfl_sync(0xffffffffu, Cm[0].x, (lane + 1) & 31);
+#pragma unroll
+  for (int i = 0; i < PPT; ++i) {
+    const double rw = __shfl_sync(0xffffffffu, Cm[i].y, (lane + 31) & 31);
+    const double re = re_next;
+    if (i + 1 < PPT) re_next = __shfl_sync(0xffffffffu, Cm[i + 1].x, (lane + 1) & 31);
+    const double W = lane == 0 ? rw_prev : rw;
+    const double E = lane == 31 ? re_next : re;
+    const double o0 = 0.25 * (((Cm[i].y + W) + N[i].x) + S[i].x);
+    const double o1 = 0.25 * (((E + Cm[i].x) + N[i].y) + S[i].y);
+    if (STORE) {
+      if (L.st >> i & 1u) {
+        if (FAST) *reinterpret_cast<double2 *>(o + 64 * i) = make_double2(o0, o1);
+        else store_pair(o + 64 * i, o0, o1, L.full >> i & 1u);
+      }
+    } else if (FAST && STEADY) {
+      V[i] = make_double2(o0, o1);
+    } else {
+      const bool r = STEADY || rowin;
+      V[i].x = (r && (FAST || (L.ok >> i & 1u))) ? o0 : Cm[i].x;
+      V[i].y = (r && (FAST || (L.full >> i & 1u))) ? o1 : Cm[i].y;
+    }
+    rw_prev = rw;
+  }
+}
+
+template <int K, int PPT, bool FAST>
+__device__ __forceinline__ void tbk_march(const TbkLane &L, const Ring &R, RingPos q, int64_t a, int64_t b,
+                                          int64_t C, int64_t r0, int64_t r1, double *dst, int64_t pe, int lane) {
+  double2 X[K - 1][3][PPT];  // X[k-1][m % 3]: level k of the row computed at step m
+  const int64_t Rs = a - K >= 0 ? r0 + 2 : r0 + 1;  // first step (r0 = 0 when a - K < 0)
+  const int64_t Re = b + K;                          // last step: level K of row b
+  // stage positions of level-0 rows R-2, R-1, R, clamped to r0 .. r1
+  RingPos pm = q, pc = Rs == r0 + 2 ? ring_add(q, 1u, R.S) : q, pn = pc;
+  if (Rs <= r1) pn = ring_add(q, (uint32_t)(Rs - r0), R.S);
+  R.wait_full(pm);
+  R.wait_full(pc);
+  // one step: level-0 row Rr enters; level k of row Rr-k for k = 1..K
+  auto step = [&](auto u_ct, auto steady_ct, int64_t Rr) {
+    constexpr int U = decltype(u_ct)::value;
+    constexpr bool ST = decltype(steady_ct)::value;
+    constexpr int Sx = (U + 1) % 3, Cx = (U + 2) % 3;
+    if (Rr <= r1) R.wait_full(pn);
+    tbk_level1<PPT, FAST, ST>(L, R.stage(pm), R.stage(pc), R.stage(pn), Rr - 1 >= 1 && Rr - 1 <= C, X[0][U]);
+    if (Rr - 2 >= r0 && Rr - 2 <= r1) R.release(pm, lane);  // row Rr-2 is no longer needed
+#pragma unroll
+    for (int k = 2; k < K; ++k)
+      tbk_levelk<PPT, FAST, ST, false>(L, X[k - 2][Sx], X[k - 2][Cx], X[k - 2][U], Rr - k >= 1 && Rr - k <= C, lane,
+                                       X[k - 1][U], nullptr);
+    if (Rr - K >= a)
+      tbk_levelk<PPT, FAST, ST, true>(L, X[K - 2][Sx], X[K - 2][Cx], X[K - 2][U], true, lane, nullptr,
+                                      dst + (Rr - K) * pe);
+    pm = pc;
+    pc = pn;
+    if (Rr + 1 <= r1) pn.advance(R.S);
+  };
+  using U0 = std::integral_constant<int, 0>;
+  using U1 = std::integral_constant<int, 1>;
+  using U2 = std::integral_constant<int, 2>;
+  using TT = std::integral_constant<bool, true>;
+  using TF = std::integral_constant<bool, false>;
+  int64_t Rr = Rs;
+  for (; Rr <= Re; Rr += 3) {
+    if (Rr >= K && Rr + 2 <= C + 1 && Rr + 2 <= Re) {  // every level's row interior: no row masks
+      step(U0{}, TT{}, Rr);
+      step(U1{}, TT{}, Rr + 1);
+      step(U2{}, TT{}, Rr + 2);
+    } else {
+      step(U0{}, TF{}, Rr);
+      if (Rr + 1 <= Re) step(U1{}, TF{}, Rr + 1);
+      if (Rr + 2 <= Re) step(U2{}, TF{}, Rr + 2);
+    }
+  }
+  // rows Re-1, Re (if they exist) were not released by the march: pm, pc after the last step
+  if (Re - 1 <= r1) R.release(pm, lane);
+  if (Re <= r1) R.release(pc, lane);
+}
+
+template <int K, int PPT>
+__device__ __forceinline__ void tbk_item(const JbGeom &g, const Ring &R, RingPos &q, int unit, int64_t a, int64_t b,
+                                         int64_t C, double *out, int warp, int lane) {
+  constexpr int WO = 64 * PPT - 2 * (K - 1);
+  const int64_t x0 = 1 + (int64_t)unit * g.tx;
+  const int64_t r0 = max(a - K, (int64_t)0), r1 = min(b + K, C + 1);
+  const RingPos q0 = q;
+  q = ring_add(q, (uint32_t)(r1 - r0 + 1), R.S);
+  const int64_t ow = x0 + (int64_t)warp * WO;  // first output column of this warp
+  if (ow > g.nx - 2) {  // no outputs in this strip for this warp: only return the stages
+    for (int64_t p = r0; p <= r1; ++p) {
+      const RingPos pp = ring_add(q0, (uint32_t)(p - r0), R.S);
+      R.wait_full(pp);
+      R.release(pp, lane);
+    }
+    return;
+  }
+  const int64_t sw = ow - (K - 1);
+  TbkLane L;
+  L.j0 = warp * WO + 2 + 2 * lane;
+  L.ok = L.full = L.st = 0;
+#pragma unroll
+  for (int i = 0; i < PPT; ++i) {
+    const int kk = 32 * i + lane;
+    const int64_t c = sw + 2 * kk;
+    const bool ok = c >= 1 && c <= g.nx - 2;
+    L.ok |= (ok ? 1u : 0u) << i;
+    L.full |= (ok && c + 1 <= g.nx - 2 ? 1u : 0u) << i;
+    L.st |= (ok && kk >= (K - 1) / 2 && kk < 32 * PPT - (K - 1) / 2 ? 1u : 0u) << i;
+  }
+  const bool fast = sw >= 1 && sw + 64 * PPT - 1 <= g.nx - 2;
+  double *dst = out + 3 + sw + 2 * lane;
+  if (fast) tbk_march<K, PPT, true>(L, R, q0, a, b, C, r0, r1, dst, g.plane_elems, lane);
+  else tbk_march<K, PPT, false>(L, R, q0, a, b, C, r0, r1, dst, g.plane_elems, lane);
+}
+
 // ---------------------------------------------------------------- 3D (7-point)
 // Tile = TY rows x tx columns (tx = 64 x warps), marched along z.  Lane `lane` of warp w owns the
 // x pair kk = w*32 + lane for EVERY row of the tile, so level-1 y neighbours are its own
@@ -376,18 +535,20 @@ __device__ __forceinline__ void tb3_item(const JbGeom &g, const Ring &R, RingPos
   else tb3_march<TY, false>(L, g, R, q0, a, b, C, r0, r1, dst, lane);
 }
 
-// Edge zone of a slab side with a neighbour (time block t -> t+2), computed by that side's
-// boundary CTAs with the whole CTA, so the halo exchange stays per iteration:
-//   A: wait for the neighbour's time-t halo plane; level 1 (t+1) of the three planes next to the
-//      halo (top: 1..3, bottom: C-2..C) over the strip window [x0-1, x0+tx] into the slab's edge
-//      scratch E, the outermost one also into the neighbour's intermediate slot; signal t+1.
-//   B: wait for the neighbour's level-1 plane (our E slot); level 2 (t+2) of the two outermost
-//      planes (top: 1, 2; bottom: C-1, C) into the next buffer, the outermost one also into the
-//      neighbour's halo; signal t+2.
-// E_top = buf[0] + (C+2) pe: [0] = neighbour's level-1 plane 0, [k] = level-1 plane k (k = 1..3);
-// E_bot = buf[1] + (C+2) pe: [k] = level-1 plane C-2+k (k = 0..2), [3] = neighbour's plane C+1.
+// Edge zone of a slab side with a neighbour (time block t -> t+K), computed by that side's
+// boundary CTAs with the whole CTA, so the halo exchange stays per iteration.
+// Phase m = 1..K: wait until the neighbour delivered its level m-1 plane (m = 1: the time-t halo
+// in `cur`; m >= 2: our slot m-1 in the scratch), then compute level m (t+m) of the planes next to
+// the halo — 2K-m of them for m < K over the strip window widened by K-m cells per side (the
+// next phase reads one cell further), the K output planes (tile cells only) for m = K — and store
+// the outermost plane also to the neighbour: its slot m (m < K) or its halo (m = K); signal t+m.
+// The interior items then cover level-K planes K+1 .. C-K, which need no halo.
+// Scratch E (per side, jb_edge_planes_k(K) planes; E_top after buf[0], E_bot after buf[1]):
+//   [m-1], m = 1..K-1           the neighbour's level-m plane (written by the neighbour)
+//   [lbase(m) + i], i < 2K-m    this side's level-m plane first(m) + i (top: 1 + i,
+//                               bottom: C-2K+m+1 + i)
 // Loads bypass L1 (ld.cg): these planes are rewritten by other CTAs / the neighbour GPU.
-template <int DIM>
+template <int DIM, int K>
 __device__ bool tb_edge(const JbGeom &g, const JbSlab &SL, const JbParams &P, int role, int ridx, int rcount,
                         const double *cur, double *nxt, double *remote, int64_t tg, int *s_flag) {
   const bool top = role == ROLE_TOP;
@@ -408,68 +569,79 @@ __device__ bool tb_edge(const JbGeom &g, const JbSlab &SL, const JbParams &P, in
     __syncthreads();
     return *s_flag == 0;
   };
-  // one stencil update of the field F (ld.cg) at element offset e = y*pitch + x of plane p
-  auto upd = [&](const double *F, int64_t e) {
-    const double *A = F + e;
-    if (DIM == 2) return 0.25 * (((__ldcg(A + 1) + __ldcg(A - 1)) + __ldcg(A + pe)) + __ldcg(A - pe));
-    return kC6 * (((((__ldcg(A + 1) + __ldcg(A - 1)) + __ldcg(A + pitch)) + __ldcg(A - pitch)) + __ldcg(A + pe)) +
-                  __ldcg(A - pe));
-  };
-  // ---- A: level 1 of 3 planes over each tile window [y0-1, y0+ty] x [x0-1, x0+tx] (clamped)
-  if (!wait((unsigned long long)tg)) return false;
-  const int64_t pa = top ? 1 : C - 2;  // plane of E index e0
-  const int e0 = top ? 1 : 0;
-  const int64_t pout = top ? 1 : C;    // the plane the neighbour needs
-  for (int u = ub; u < ue; ++u) {
-    const int ux = u % g.units_x, uy = u / g.units_x;
-    const int64_t x0 = 1 + (int64_t)ux * g.tx;
-    const int64_t xa = max(x0 - 1, (int64_t)0), xb = min(x0 + g.tx, nx - 1), w = xb - xa + 1;
-    int64_t ya = 0, h = 1;
-    if (DIM == 3) {
-      const int64_t y0 = 1 + (int64_t)uy * g.ty;
-      ya = max(y0 - 1, (int64_t)0);
-      h = min(y0 + g.ty, ny - 1) - ya + 1;
+  auto lbase = [](int m) { return (int64_t)(K - 1) + (int64_t)(m - 1) * 2 * K - (int64_t)(m - 1) * m / 2; };
+  const int64_t halo = top ? 0 : C + 1;
+  const int64_t pout = top ? 1 : C;  // the plane the neighbour needs
+#pragma unroll 1
+  for (int m = 1; m <= K; ++m) {
+    if (!wait((unsigned long long)(tg + m - 1))) return false;
+    const int64_t np = m < K ? 2 * K - m : K;        // level-m planes of this side
+    const int64_t pf = top ? 1 : C - np + 1;         // the first of them
+    const int64_t npv = 2 * K - (m - 1);             // level-(m-1) planes of this side (m >= 2)
+    const int64_t pfv = top ? 1 : C - npv + 1;
+    // level m-1 of plane p (element offset 3 of x = 0, row 0)
+    auto src = [&](int64_t p) -> const double * {
+      if (m == 1) return cur + p * pe + 3;
+      if (p == halo) return E + (int64_t)(m - 2) * pe;
+      return E + (lbase(m - 1) + (p - pfv)) * pe;
+    };
+    const int64_t mg = K - m;  // window margin
+    for (int u = ub; u < ue; ++u) {
+      const int ux = u % g.units_x, uy = u / g.units_x;
+      const int64_t x0 = 1 + (int64_t)ux * g.tx;
+      int64_t xa, xb, ya = 0, yb = 0;
+      if (m < K) {
+        xa = max(x0 - mg, (int64_t)0);
+        xb = min(x0 + g.tx - 1 + mg, nx - 1);
+      } else {
+        xa = x0;
+        xb = min(x0 + g.tx, nx - 1) - 1;
+      }
+      if (DIM == 3) {
+        const int64_t y0 = 1 + (int64_t)uy * g.ty;
+        if (m < K) {
+          ya = max(y0 - mg, (int64_t)0);
+          yb = min(y0 + g.ty - 1 + mg, ny - 1);
+        } else {
+          ya = y0;
+          yb = min(y0 + g.ty, ny - 1) - 1;
+        }
+      }
+      const int64_t w = xb - xa + 1, h = yb - ya + 1;
+      for (int64_t i = tid; i < np * h * w; i += nt) {
+        const int64_t k = i / (h * w), r = i - k * h * w, yy = r / w;
+        const int64_t x = xa + (r - yy * w), y = ya + yy, p = pf + k;
+        const int64_t e = (DIM == 3 ? y * pitch : 0) + x;
+        const bool in = x >= 1 && x <= nx - 2 && (DIM == 2 || (y >= 1 && y <= ny - 2));
+        const double *A = src(p) + e;
+        double v;
+        if (!in) {
+          v = __ldcg(A);
+        } else if (DIM == 2) {  // oracle order: x+1, x-1, y+1, y-1 (then z+1, z-1), then the scale
+          v = 0.25 * (((__ldcg(A + 1) + __ldcg(A - 1)) + __ldcg(src(p + 1) + e)) + __ldcg(src(p - 1) + e));
+        } else {
+          v = kC6 * (((((__ldcg(A + 1) + __ldcg(A - 1)) + __ldcg(A + pitch)) + __ldcg(A - pitch)) +
+                      __ldcg(src(p + 1) + e)) +
+                     __ldcg(src(p - 1) + e));
+        }
+        if (m < K) {
+          E[(lbase(m) + k) * pe + e] = v;
+          if (p == pout) mid[(int64_t)(m - 1) * pe + e] = v;
+        } else {
+          nxt[p * pe + 3 + e] = v;
+          if (p == pout) remote[3 + e] = v;
+        }
+      }
     }
-    for (int64_t i = tid; i < 3 * h * w; i += nt) {
-      const int64_t k = i / (h * w), r = i - k * h * w, yy = r / w;
-      const int64_t x = xa + (r - yy * w), y = ya + yy, p = pa + k;
-      const int64_t e = (DIM == 3 ? y * pitch : 0) + x;
-      const bool in = x >= 1 && x <= nx - 2 && (DIM == 2 || (y >= 1 && y <= ny - 2));
-      const double v = in ? upd(cur + p * pe + 3, e) : __ldcg(cur + p * pe + 3 + e);
-      E[(e0 + k) * pe + e] = v;
-      if (p == pout) mid[e] = v;
-    }
+    __syncthreads();  // every thread's stores (local, neighbour's) precede the release below
+    if (tid == 0 && !drop) st_release_sys(fout, (unsigned long long)(tg + m));
   }
-  __syncthreads();  // every thread's stores (local E, neighbour's slot) precede the release below
-  if (tid == 0 && !drop) st_release_sys(fout, (unsigned long long)(tg + 1));
-  // ---- B: level 2 of the 2 outermost planes over each tile's interior cells
-  if (!wait((unsigned long long)(tg + 1))) return false;
-  const int64_t pb = top ? 1 : C - 1;  // level-2 planes pb, pb+1 <-> E indices 1, 2
-  for (int u = ub; u < ue; ++u) {
-    const int ux = u % g.units_x, uy = u / g.units_x;
-    const int64_t x0 = 1 + (int64_t)ux * g.tx;
-    const int64_t w = min((int64_t)g.tx, nx - 1 - x0);
-    int64_t y0 = 0, h = 1;
-    if (DIM == 3) {
-      y0 = 1 + (int64_t)uy * g.ty;
-      h = min((int64_t)g.ty, ny - 1 - y0);
-    }
-    for (int64_t i = tid; i < 2 * h * w; i += nt) {
-      const int64_t k = i / (h * w), r = i - k * h * w, yy = r / w;
-      const int64_t x = x0 + (r - yy * w), p = pb + k;
-      const int64_t e = (DIM == 3 ? (y0 + yy) * pitch : 0) + x;
-      const double v = upd(E + (1 + k) * pe, e);
-      nxt[p * pe + 3 + e] = v;
-      if (p == pout) remote[3 + e] = v;
-    }
-  }
-  __syncthreads();
-  if (tid == 0 && !drop) st_release_sys(fout, (unsigned long long)(tg + 2));
   return true;
 }
 
-template <int NCW, int DIM, int TP>
+template <int NCW, int DIM, int K, int TP>
 __device__ __forceinline__ void tb_body(const JbParams &P) {
+  static_assert(K == 2 || (DIM == 2 && (K & 1)), "3D: K = 2; 2D: K = 2 or odd");
   extern __shared__ __align__(128) unsigned char smem[];
   __shared__ int s_abort;
   __shared__ int s_edge;  // the edge zones' wait result (own variable: s_abort is read after the barrier)
@@ -514,15 +686,15 @@ __device__ __forceinline__ void tb_body(const JbParams &P) {
   __syncthreads();
 
   const int64_t C = SL.chunk;
-  const int64_t nblocks = P.iters / TB_K;
+  const int64_t nblocks = P.iters / K;
   RingPos q = {0u, 0u}, rq = {0u, 0u};
   for (int64_t j = 0; j < nblocks; ++j) {
     const double *cur = SL.buf[(P.t0 + j) & 1];
     double *nxt = SL.buf[(P.t0 + j + 1) & 1];
-    const int64_t tg = P.t0 + TB_K * j;  // global iteration at the start of this time block
+    const int64_t tg = P.t0 + K * j;  // global iteration at the start of this time block
     if (role != ROLE_INT) {  // edge zone with its per-iteration exchange, then help the interior
       double *remote = role == ROLE_TOP ? SL.peer_top[(P.t0 + j + 1) & 1] : SL.peer_bot[(P.t0 + j + 1) & 1];
-      if (!tb_edge<DIM>(g, SL, P, role, ridx, rcount, cur, nxt, remote, tg, &s_edge)) return;
+      if (!tb_edge<DIM, K>(g, SL, P, role, ridx, rcount, cur, nxt, remote, tg, &s_edge)) return;
       fence_proxy_async_global();  // our generic-proxy stores before later bulk reads
     }
     if (producer) {
@@ -540,7 +712,7 @@ __device__ __forceinline__ void tb_body(const JbParams &P) {
         const int64_t blk = item / g.units;
         const int32_t unit = (int32_t)(item - blk * g.units);
         const int64_t a = SL.tb_lo + SL.dyn_table[blk], b = SL.tb_lo + SL.dyn_table[blk + 1] - 1;
-        const int64_t r0 = max(a - 2, (int64_t)0), r1 = min(b + 2, C + 1);
+        const int64_t r0 = max(a - K, (int64_t)0), r1 = min(b + K, C + 1);
         const bool early = r1 - r0 + 1 <= (int64_t)R.S;
         if (early && lane == 0) claim = atomicAdd(ctr, 1u);
         if (lane == 0) {
@@ -556,11 +728,14 @@ __device__ __forceinline__ void tb_body(const JbParams &P) {
         }
         // level-0 rows r0..r1 of the tile: x window [x0-2, x0+tx+2) of rows y0-2 .. y0+TY+1
         // (3D; stage row i <-> y0-2+i, rows outside the grid are not loaded), one bulk copy
-        // per row and lane
+        // per row and lane; 2D with K odd: columns x0-K-1 .. x0+tx+K (stage index 0 <-> x0-K-1;
+        // columns left of the row's padding are not loaded: they only feed Dirichlet cells)
         const int ux = unit % g.units_x, uy = unit / g.units_x;
-        const int64_t xs = 2 + (int64_t)ux * g.tx;
-        const int64_t xe = min(xs + g.tx + 4, g.pitch);
+        const int64_t xs_w = (DIM == 2 && K > 2) ? 3 - K + (int64_t)ux * g.tx : 2 + (int64_t)ux * g.tx;
+        const int64_t xs = max(xs_w, (int64_t)0);
+        const int64_t xe = min(xs_w + ((DIM == 2 && K > 2) ? g.tx + 2 * K + 2 : g.tx + 4), g.pitch);
         const uint32_t bytes = (uint32_t)((xe - xs) * 8);
+        const int64_t dso = xs - xs_w;  // stage offset of the first loaded column
         const int64_t ya = DIM == 3 ? (int64_t)uy * g.ty - 1 : 0;  // = y0 - 2
         const int nrow = DIM == 3 ? g.rh : 1;
         const int64_t yl = max(ya, (int64_t)0), yh = DIM == 3 ? min(ya + nrow - 1, g.ny - 1) : 0;
@@ -574,7 +749,7 @@ __device__ __forceinline__ void tb_body(const JbParams &P) {
             mbar_expect_tx(&R.full[q.slot], bytes * nvalid);
           }
           __syncwarp();
-          if (mine) bulk_g2s(R.stage(q) + (size_t)lane * g.ws, src + p * g.plane_elems, bytes, &R.full[q.slot]);
+          if (mine) bulk_g2s(R.stage(q) + (size_t)lane * g.ws + dso, src + p * g.plane_elems, bytes, &R.full[q.slot]);
           q.advance(R.S);
         }
         rq.advance(JB_RQ);
@@ -595,8 +770,9 @@ __device__ __forceinline__ void tb_body(const JbParams &P) {
         if (lane == 0) mbar_arrive(&qempty[rq.slot]);
         rq.advance(JB_RQ);
         if (d.kind == TB_END) break;
-        if (DIM == 2) tb2_item<TP>(g, R, q, d.unit, d.a, d.b, C, nxt, warp, lane);
-        else tb3_item<TP>(g, R, q, d.unit, d.a, d.b, C, nxt, warp, lane);
+        if constexpr (DIM == 3) tb3_item<TP>(g, R, q, d.unit, d.a, d.b, C, nxt, warp, lane);
+        else if constexpr (K == 2) tb2_item<TP>(g, R, q, d.unit, d.a, d.b, C, nxt, warp, lane);
+        else tbk_item<K, TP>(g, R, q, d.unit, d.a, d.b, C, nxt, warp, lane);
       }
       fence_proxy_async_global();  // generic-proxy stores before the next block's bulk reads
     }
@@ -618,24 +794,36 @@ __device__ __forceinline__ void tb_body(const JbParams &P) {
 }
 
 // One CTA per SM (up to 224 registers per thread) or two (96: 2 x 9 warps fit the register file
-// only at <= 96 registers, given the 4-warp allocation granularity).  TP = pairs per thread
-// along x (2D) or rows per tile (3D).
-template <int DIM, int TP>
-__global__ void __launch_bounds__(JB_NC + 32, 1) jb_tblock(const __grid_constant__ JbParams P) {
-  tb_body<JB_NCW, DIM, TP>(P);
+// only at <= 96 registers, given the 4-warp allocation granularity).  K = iterations per time
+// block; TP = pairs per thread along x (2D) or rows per tile (3D).
+template <int DIM, int K, int TP, int NCW = JB_NCW>
+__global__ void __launch_bounds__((NCW + 1) * 32, 1) jb_tblock(const __grid_constant__ JbParams P) {
+  tb_body<NCW, DIM, K, TP>(P);
 }
 template <int TP>
 __global__ void __maxnreg__(96) jb_tblock2d_x2(const __grid_constant__ JbParams P) {
-  tb_body<JB_NCW, 2, TP>(P);
+  tb_body<JB_NCW, 2, 2, TP>(P);
 }
 
 constexpr int TB_TY = 4;  // 3D tile rows (level-1 rows TY+2 carried per plane in registers)
 
-const void *tblock_fn(int dim, int ppt, int per_sm) {
-#define JB_TB(K) reinterpret_cast<const void *>(&K)
-  if (dim == 3) return JB_TB((jb_tblock<3, TB_TY>));
-  if (per_sm >= 2) return ppt >= 4 ? JB_TB(jb_tblock2d_x2<4>) : ppt == 2 ? JB_TB(jb_tblock2d_x2<2>) : JB_TB(jb_tblock2d_x2<1>);
-  return ppt >= 4 ? JB_TB((jb_tblock<2, 4>)) : ppt == 2 ? JB_TB((jb_tblock<2, 2>)) : JB_TB((jb_tblock<2, 1>));
+// Kernel for (dim, K, pairs per thread, CTAs per SM) and its consumer warp count; nullptr if not
+// instantiated.  Odd K holds 2(K-1) level rows per lane: with PPT = 4 (K = 3) or K = 5 the
+// kernel needs > 168 registers, i.e. 7 consumer warps (256 threads: up to 255 registers).
+const void *tblock_fn(int dim, int k, int ppt, int per_sm, int *ncw) {
+#define JB_TB(...) reinterpret_cast<const void *>(&__VA_ARGS__)
+  *ncw = JB_NCW;
+  if (dim == 3) return k == 2 ? JB_TB(jb_tblock<3, 2, TB_TY>) : nullptr;
+  if (k == 2) {
+    if (per_sm >= 2) return ppt >= 4 ? JB_TB(jb_tblock2d_x2<4>) : ppt == 2 ? JB_TB(jb_tblock2d_x2<2>) : JB_TB(jb_tblock2d_x2<1>);
+    return ppt >= 4 ? JB_TB(jb_tblock<2, 2, 4>) : ppt == 2 ? JB_TB(jb_tblock<2, 2, 2>) : JB_TB(jb_tblock<2, 2, 1>);
+  }
+  if (per_sm >= 2) return nullptr;
+  if (k == 3 && ppt == 2) return JB_TB(jb_tblock<2, 3, 2>);
+  *ncw = 7;
+  if (k == 3 && ppt == 4) return JB_TB(jb_tblock<2, 3, 4, 7>);
+  if (k == 5 && ppt == 2) return JB_TB(jb_tblock<2, 5, 2, 7>);
+  return nullptr;
 #undef JB_TB
 }
 
@@ -643,9 +831,12 @@ const void *tblock_fn(int dim, int ppt, int per_sm) {
 
 namespace jbk {
 
-int tblock_k() { return TB_K; }
 int tblock_ty() { return TB_TY; }
-int tblock_threads() { return JB_NC + 32; }
+// consumer warps of the kernel for (dim, k, ppt) with one CTA per SM; 0 if not instantiated
+int tblock_ncw(int dim, int k, int ppt, int per_sm) {
+  int ncw = 0;
+  return tblock_fn(dim, k, ppt, per_sm, &ncw) ? ncw : 0;
+}
 
 // Dynamic shared memory of the temporally blocked kernel: header + ring stages.
 size_t tblock_smem(const JbGeom &g) {
@@ -653,19 +844,23 @@ size_t tblock_smem(const JbGeom &g) {
   return (hdr + 127) / 128 * 128 + (size_t)g.stages * g.stage_doubles * 8;
 }
 
-cudaError_t prepare_tblock(const JbGeom &g, int per_sm, size_t smem, int *blocks_per_sm) {
-  const void *fn = tblock_fn(g.dim, g.tx / (2 * JB_NC), per_sm);
+cudaError_t prepare_tblock(const JbGeom &g, int k, int ppt, int per_sm, size_t smem, int *blocks_per_sm) {
+  int ncw = 0;
+  const void *fn = tblock_fn(g.dim, k, ppt, per_sm, &ncw);
+  if (!fn) return cudaErrorInvalidValue;
   cudaError_t e = cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
   if (e != cudaSuccess) return e;
   e = cudaFuncSetAttribute(fn, cudaFuncAttributePreferredSharedMemoryCarveout, (int)cudaSharedmemCarveoutMaxShared);
   if (e != cudaSuccess) return e;
-  return cudaOccupancyMaxActiveBlocksPerMultiprocessor(blocks_per_sm, fn, JB_NC + 32, smem);
+  return cudaOccupancyMaxActiveBlocksPerMultiprocessor(blocks_per_sm, fn, (ncw + 1) * 32, smem);
 }
 
-cudaError_t launch_tblock(const JbParams &p, int per_sm, int grid, size_t smem, cudaStream_t st) {
+cudaError_t launch_tblock(const JbParams &p, int k, int ppt, int per_sm, int grid, size_t smem, cudaStream_t st) {
   void *args[] = {const_cast<JbParams *>(&p)};
-  return cudaLaunchCooperativeKernel(tblock_fn(p.g.dim, p.g.tx / (2 * JB_NC), per_sm), dim3(grid), dim3(JB_NC + 32), args, smem,
-                                     st);
+  int ncw = 0;
+  const void *fn = tblock_fn(p.g.dim, k, ppt, per_sm, &ncw);
+  if (!fn) return cudaErrorInvalidValue;
+  return cudaLaunchCooperativeKernel(fn, dim3(grid), dim3((ncw + 1) * 32), args, smem, st);
 }
 
 }  // namespace jbk

@@ -1,6 +1,6 @@
 #!/bin/bash
 # Run on the GPU box (gpurun): launch list of the bench command + ncu --set full of the CPU-Free
-# kernels (20-iteration launches) for C2 (time-blocked), C2 per-iteration and C3, under gpurun_out/.
+# kernels (20-iteration launches) for C2 (time-blocked K=5 default, K=2), C2 per-iteration and C3, under gpurun_out/.
 set -x
 out=gpurun_out
 ncu --metrics gpu__time_duration.sum --clock-control none --csv --log-file $out/launches_c2.csv \
@@ -12,5 +12,6 @@ run_full() {  # name, kernel regex, bench args
   ncu -i $out/full_$1.ncu-rep --page details --csv > $out/full_$1_details.csv 2>/dev/null
 }
 run_full c2_tblock jb_tblock --config c2
+run_full c2_tblock_k2 jb_tblock --config c2 --param tb_k=2
 run_full c2 jb_sweep --config c2 --param tblock=0
 run_full c3 jb_sweep --config c3

@@ -1,9 +1,11 @@
-"""GPU parity of the temporally blocked CPU-Free kernel (tblock.cu): two Jacobi
-iterations per pass over HBM for a slab without neighbours.  It reorders WHEN cells are
-updated, never HOW (oracle operation order, -fmad=false), so the bar is bit-exact equality with
-the oracle — over ragged strips, tiny and single-plane blocks, the Dirichlet rows/columns that
-the intermediate level must keep, odd iteration counts (the remainder runs per-iteration) and
-run splitting / mixing with the other kernels and modes."""
+"""GPU parity of the temporally blocked CPU-Free kernel (tblock.cu): K Jacobi
+iterations per pass over HBM (2D: K = 2 with extra cells, K = 3 / 5 with overlapped warp
+segments; 3D: K = 2), edge zones keeping the per-iteration halo exchange between slabs.  It
+reorders WHEN cells are updated, never HOW (oracle operation order, -fmad=false), so the bar is
+bit-exact equality with the oracle — over ragged strips, tiny and single-plane blocks, the
+Dirichlet rows/columns that the intermediate levels must keep, iteration counts that are not a
+multiple of K (the remainder runs per-iteration) and run splitting / mixing with the other
+kernels and modes."""
 import numpy as np
 import pytest
 
@@ -12,6 +14,27 @@ import paper_conf_sc_baydamirlibu24_b200 as jb
 from jacobi_inputs import SEED_BENCH, integer_field, nv_field, u12
 
 pytestmark = pytest.mark.gpu
+
+# 2D variants (K, pairs per thread); the default (auto) is K = 5, ppt = 2
+KV = [(2, 4), (3, 2), (3, 4), (5, 2)]
+K_AUTO = 5
+
+
+def step(k):
+    """Iterations per whole time-blocked unit: K (odd), 2K (K = 2: even block count)."""
+    return k if k % 2 else 2 * k
+
+
+def tb_iters(iters, k):
+    return iters // step(k) * step(k)
+
+
+def k_fit(chunk, k=K_AUTO):
+    """Deepest supported K <= k whose edge zones (2K planes) fit a slab of `chunk` planes."""
+    for kk in (5, 3, 2):
+        if kk <= k and chunk >= 2 * kk:
+            return kk
+    return 0
 
 
 def assert_bitwise(got, exp, what=""):
@@ -22,9 +45,10 @@ def assert_bitwise(got, exp, what=""):
         raise AssertionError(f"{what}: {n} cells differ, max |diff| {d.max()} at {idx}")
 
 
-def run_tb(field, iters, params=None, runs=None):
-    """Force the temporally blocked kernel (tblock=1, resident off); returns (field, last_tblock)."""
-    params = {"tblock": 1, "resident": 0, **(params or {})}
+def run_tb(field, iters, params=None, runs=None, kv=None):
+    """Force the temporally blocked kernel (tblock=1, resident off), variant kv = (K, ppt) or
+    auto; returns (field, last_tblock)."""
+    params = {"tblock": 1, "resident": 0, **({"tb_k": kv[0], "tb_ppt": kv[1]} if kv else {}), **(params or {})}
     with jb.Jacobi(field.shape) as j:
         for k, v in params.items():
             j.set_param(k, v)
@@ -37,64 +61,83 @@ def run_tb(field, iters, params=None, runs=None):
 @pytest.mark.parametrize("shape", [(3, 3), (3, 40), (4, 5), (6, 9), (37, 1500), (70, 2051), (300, 130),
                                    (1000, 37), (17, 4100)])
 @pytest.mark.parametrize("iters", [4, 5, 12, 29])
-def test_tblock_shapes(shape, iters):
+@pytest.mark.parametrize("kv", KV)
+def test_tblock_shapes(shape, iters, kv):
     f = u12(shape, 1)
     exp = oracle.jacobi(f, iters)
-    got, tb = run_tb(f, iters)
-    assert tb == iters // 4 * 4
-    assert_bitwise(got, exp, f"tblock {shape} it{iters}")
+    got, tb = run_tb(f, iters, kv=kv)
+    assert tb == tb_iters(iters, kv[0])
+    assert_bitwise(got, exp, f"tblock K={kv} {shape} it{iters}")
 
 
 @pytest.mark.parametrize("tile_x,min_block", [(8, 1), (16, 2), (64, 1), (256, 3), (1024, 16), (2048, 5)])
 @pytest.mark.parametrize("ctas", [1, 2])
 def test_tblock_tiles_and_blocks(tile_x, min_block, ctas):
-    """Many strips (ragged last strip, strips narrower than a warp), single-plane blocks, one or
-    two CTAs per SM."""
+    """K = 2: many strips (ragged last strip, strips narrower than a warp), single-plane blocks,
+    one or two CTAs per SM."""
     shape = (133, 2100)
     f = u12(shape, 2)
-    got, _ = run_tb(f, 8, {"tile_x": tile_x, "tb_min_block": min_block, "tb_ctas": ctas})
+    got, _ = run_tb(f, 8, {"tile_x": tile_x, "tb_min_block": min_block, "tb_ctas": ctas}, kv=(2, 4))
     assert_bitwise(got, oracle.jacobi(f, 8), f"tx{tile_x} mb{min_block}")
 
 
+@pytest.mark.parametrize("min_block", [1, 2, 7, 16, 64])
+@pytest.mark.parametrize("kv", KV[1:])
+def test_tblock_odd_k_blocks_and_strips(kv, min_block):
+    """Odd K: single-plane and short blocks (the wavefront's warm-up and drain rows dominate),
+    several strips with a ragged last one and warps without outputs in it."""
+    for shape in [(133, 2100), (61, 4100), (40, 967)]:
+        f = u12(shape, 2)
+        got, _ = run_tb(f, 15, {"tb_min_block": min_block}, kv=kv)
+        assert_bitwise(got, oracle.jacobi(f, 15), f"K={kv} {shape} mb{min_block}")
+
+
 @pytest.mark.parametrize("stages", [4, 5, 9])
-def test_tblock_ring_depths(stages):
+@pytest.mark.parametrize("kv", KV)
+def test_tblock_ring_depths(stages, kv):
     f = u12((400, 700), 3)
-    got, _ = run_tb(f, 16, {"stages": stages, "tb_min_block": 40})
-    assert_bitwise(got, oracle.jacobi(f, 16), f"stages {stages}")
+    got, _ = run_tb(f, 30, {"stages": stages, "tb_min_block": 40}, kv=kv)
+    assert_bitwise(got, oracle.jacobi(f, 30), f"stages {stages}")
 
 
-def test_tblock_run_splitting_and_mixing():
+@pytest.mark.parametrize("kv", KV)
+def test_tblock_run_splitting_and_mixing(kv):
     """run(a); run(b) == run(a+b) across the time-blocked, per-iteration, resident and baseline
     kernels (the buffer parity convention is shared)."""
     f = u12((90, 300), 4)
     exp = oracle.jacobi(f, 31)
-    got, _ = run_tb(f, 31, runs=[4, 1, 8, 3, 5, 6, 4])
+    got, _ = run_tb(f, 31, runs=[4, 1, 8, 3, 5, 6, 4], kv=kv)
     assert_bitwise(got, exp, "split")
+    K = kv[0]
     with jb.Jacobi(f.shape) as j:
         j.set_param("resident", 0)
+        j.set_param("tb_k", K)
+        j.set_param("tb_ppt", kv[1])
         j.scatter(f)
-        j.run(6)                                  # auto: 4 time-blocked + 2 per-iteration
-        assert j.get_param("last_tblock") == 4
+        j.run(6)                                  # auto: time-blocked + per-iteration remainder
+        assert j.get_param("last_tblock") == tb_iters(6, K) and j.get_param("last_tb_k") == K
         j.set_mode(jb.MODE_BASELINE_MEMCPY)
         j.run(3)
         j.set_mode(jb.MODE_CPUFREE)
         j.set_param("resident", 1)
         j.run(5)                                  # resident kernel
         j.set_param("resident", 0)
-        j.run(17)                                 # 16 time-blocked + 1
+        j.run(17)
+        assert j.get_param("last_tblock") == tb_iters(17, K)
         assert_bitwise(j.gather(), exp, "mixed")
 
 
-def test_tblock_invariants_and_special_fields():
+@pytest.mark.parametrize("kv", KV)
+def test_tblock_invariants_and_special_fields(kv):
     y, x = np.mgrid[0:41, 0:77].astype(np.float64)
     for h in (3 + 2 * x - 5 * y, x * x - y * y, x * y, np.full((41, 77), np.pi)):
-        got, _ = run_tb(np.ascontiguousarray(h), 24)
+        got, _ = run_tb(np.ascontiguousarray(h), 30, kv=kv)
         assert_bitwise(got, h, "harmonic field stationary")
     f = integer_field((50, 60), 5)
-    got, _ = run_tb(f, 12)
-    assert_bitwise(got, oracle.jacobi(f, 12), "integer field")
+    got, _ = run_tb(f, 15, kv=kv)
+    assert_bitwise(got, oracle.jacobi(f, 15), "integer field")
     f = nv_field((34, 2400))
-    got, _ = run_tb(f, 1000)
+    got, _ = run_tb(f, 1000, kv=kv)
     exp = oracle.jacobi(f, 1000)
     assert np.count_nonzero((exp != 0) & (np.abs(exp) < np.finfo(np.float64).tiny)) > 0
     assert_bitwise(got, exp, "subnormals")
@@ -106,16 +149,27 @@ def test_tblock_auto_selection_and_errors():
         j.scatter(f)
         j.run(8)
         assert j.get_param("last_tblock") == 0 and j.get_param("last_resident") == 1
+        j.set_param("resident", 0)
+        j.run(8)                   # auto depth K = 5: 5 time-blocked + 3 per-iteration
+        assert j.get_param("last_tblock") == 5 and j.get_param("last_tb_k") == K_AUTO
+        for bad in (4, 7, 1):      # no kernel for that depth: auto falls back to the default
+            j.set_param("tb_k", bad)
+            j.run(5)
+            assert j.get_param("last_tb_k") in (2, 3, 5)
+        j.set_param("tb_k", -1)
+        j.set_param("resident", -1)
         j.set_param("tblock", 0)
         j.set_param("resident", 0)
         j.run(8)
         assert j.get_param("last_tblock") == 0
         with pytest.raises(jb.JacobiError):
             j.set_param("last_tblock", 1)
+        with pytest.raises(jb.JacobiError):
+            j.set_param("last_tb_k", 1)
     with jb.Jacobi((64, 96), virtual=2) as j:  # slabs with neighbours: edge zones
         j.set_param("tblock", 1)
-        j.run(4)
-        assert j.get_param("last_tblock") == 4
+        j.run(5)
+        assert j.get_param("last_tblock") == 5
         j.set_mode(jb.MODE_CPUFREE, jb.FLAG_NO_COMPUTE)  # no-compute runs keep jb_sweep
         with pytest.raises(jb.JacobiError):
             j.run(4)
@@ -131,6 +185,8 @@ def test_tblock_watchdog_state_is_clean():
     f = u12((200, 5000), 6)
     got, _ = run_tb(f, 40, runs=[20, 20])
     assert_bitwise(got, oracle.jacobi(f, 40), "two runs")
+    got, _ = run_tb(f, 40, runs=[20, 20], kv=(2, 4))
+    assert_bitwise(got, oracle.jacobi(f, 40), "two runs")
 
 
 def test_c2_full_grid_8_iters_time_blocked():
@@ -139,15 +195,21 @@ def test_c2_full_grid_8_iters_time_blocked():
     import os
     with jb.Jacobi((16384, 16384)) as j:
         j.run(8)
-        assert j.get_param("last_tblock") == 8
+        assert j.get_param("last_tblock") == 5 and j.get_param("last_tb_k") == K_AUTO
         got = j.gather()
     exp = oracle.jacobi(u12((16384, 16384), SEED_BENCH), 8, os.cpu_count() or 1)
     assert_bitwise(got, exp, "C2 8 iterations")
+    with jb.Jacobi((16384, 16384)) as j:
+        j.run(10)
+        assert j.get_param("last_tblock") == 10
+        got = j.gather()
+    exp = oracle.jacobi(exp, 2, os.cpu_count() or 1)
+    assert_bitwise(got, exp, "C2 10 iterations (two time blocks of 5)")
 
 
 # ---------------------------------------------------------------- slabs with neighbours
-def run_tb_virtual(field, iters, P, params=None, runs=None):
-    params = {"tblock": 1, "resident": 0, **(params or {})}
+def run_tb_virtual(field, iters, P, params=None, runs=None, kv=None):
+    params = {"tblock": 1, "resident": 0, **({"tb_k": kv[0], "tb_ppt": kv[1]} if kv else {}), **(params or {})}
     with jb.Jacobi(field.shape, virtual=P) as j:
         for k, v in params.items():
             j.set_param(k, v)
@@ -158,27 +220,40 @@ def run_tb_virtual(field, iters, P, params=None, runs=None):
 
 
 @pytest.mark.parametrize("P", [2, 3, 4, 5, 8])
-@pytest.mark.parametrize("shape", [(50, 300), (43, 2100), (81, 37)])
-def test_tblock_virtual_slabs(P, shape):
-    """Edge zones with the per-iteration exchange (level-1 slots + halos, two signals per time
-    block) between P slabs in one launch; chunks of 4+ planes incl. remainders."""
-    if (shape[0] - 2) // P < 4:
+@pytest.mark.parametrize("shape", [(50, 300), (43, 2100), (81, 37), (130, 1100)])
+@pytest.mark.parametrize("kv", KV)
+def test_tblock_virtual_slabs(P, shape, kv):
+    """Edge zones with the per-iteration exchange (K-1 intermediate-level slots + halos, K signals
+    per time block) between P slabs in one launch; chunks of 2K+ planes incl. remainders; the
+    runtime falls back to a shallower K when the slabs are too thin for the requested one."""
+    chunk = (shape[0] - 2) // P
+    K = k_fit(chunk, kv[0])
+    if K == 0:
         pytest.skip("slab too thin for the edge zones")
     f = u12(shape, 7)
-    got, tb = run_tb_virtual(f, 13, P)
-    assert tb == 12
-    assert_bitwise(got, oracle.jacobi(f, 13), f"P={P} {shape}")
+    with jb.Jacobi(f.shape, virtual=P) as j:
+        for n, v in {"tblock": 1, "resident": 0, "tb_k": kv[0], "tb_ppt": kv[1]}.items():
+            j.set_param(n, v)
+        j.scatter(f)
+        j.run(31)
+        assert j.get_param("last_tb_k") == K
+        assert j.get_param("last_tblock") == tb_iters(31, K)
+        assert_bitwise(j.gather(), oracle.jacobi(f, 31), f"P={P} {shape} K={kv}")
 
 
-@pytest.mark.parametrize("chunk", [4, 5, 6, 7])
-def test_tblock_virtual_thin_slabs(chunk):
-    """chunk 4: the two edge zones cover the slab (no interior items); 5-7: 1-3 interior planes."""
+@pytest.mark.parametrize("chunk", [4, 5, 6, 7, 10, 11, 13])
+@pytest.mark.parametrize("kv", KV)
+def test_tblock_virtual_thin_slabs(chunk, kv):
+    """chunk 2K: the two edge zones cover the slab (no interior items); 2K+1 ..: 1-3 interior
+    planes."""
     P = 3
+    if k_fit(chunk, kv[0]) == 0:
+        pytest.skip("slab too thin")
     f = u12((P * chunk + 2, 150), 8)
     for tx, mb in [(0, 16), (32, 1)]:
         params = {"tb_min_block": mb, **({"tile_x": tx} if tx else {})}
-        got, _ = run_tb_virtual(f, 8, P, params)
-        assert_bitwise(got, oracle.jacobi(f, 8), f"chunk {chunk} tx{tx}")
+        got, _ = run_tb_virtual(f, 15, P, params, kv=kv)
+        assert_bitwise(got, oracle.jacobi(f, 15), f"chunk {chunk} tx{tx}")
 
 
 def test_tblock_virtual_mixing_and_decomposition():
@@ -190,15 +265,15 @@ def test_tblock_virtual_mixing_and_decomposition():
         j.set_param("resident", 0)
         j.scatter(f)
         j.run(8)
-        assert j.get_param("last_tblock") == 8
+        assert j.get_param("last_tblock") == 5     # chunk 17: K = 5
         j.set_param("tblock", 0)
         j.run(3)
         j.set_param("tblock", -1)
         j.set_mode(jb.MODE_BASELINE_MEMCPY)
         j.run(2)
         j.set_mode(jb.MODE_CPUFREE)
-        j.run(24)                      # 24 time-blocked
-        assert j.get_param("last_tblock") == 24
+        j.run(24)                      # 20 time-blocked + 4
+        assert j.get_param("last_tblock") == 20
         assert_bitwise(j.gather(), exp, "mixed P=4")
     got1, _ = run_tb(f, 37)
     assert_bitwise(got1, exp, "P=1")
@@ -225,7 +300,7 @@ def test_tblock_virtual_watchdog():
         j.set_mode(jb.MODE_CPUFREE, jb.FLAG_DROP_SIGNAL)
         j.scatter(f)
         with pytest.raises(jb.JacobiError) as e:
-            j.run(4)
+            j.run(5)
         assert e.value.code == jb.JACOBI_ETIMEOUT
 
 

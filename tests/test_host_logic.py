@@ -191,10 +191,18 @@ def test_slab_bytes_matches_layout():
     for slab in range(3):
         s, c = jb.jacobi_decompose(64, 3, slab)
         b = jb.jacobi_slab_bytes(1000, 64, 1, 5, 3, slab)
-        # (chunk + 2) planes + 4 scratch planes for the time-blocked kernel's edge zones
-        assert b == (c + 2 + 4) * g["plane_elems"] * 8
+        # (chunk + 2) planes + the time-blocked kernel's edge-zone scratch: per side K-1 slots for
+        # the neighbour's intermediate levels + 2K-m own level-m planes (m < K), for 2D K <= 5: 34
+        kmax = 5
+        scratch = (kmax - 1) + sum(2 * kmax - m for m in range(1, kmax))
+        assert scratch == 34
+        assert b == (c + 2 + scratch) * g["plane_elems"] * 8
         total += c
     assert total == 62
+    # 3D keeps K = 2: 1 slot + 3 level-1 planes
+    g3 = jb.jacobi_geometry(40, 30, 64, 7)
+    s, c = jb.jacobi_decompose(64, 3, 1)
+    assert jb.jacobi_slab_bytes(40, 30, 64, 7, 3, 1) == (c + 2 + 4) * g3["plane_elems"] * 8
 
 
 def test_set_allocator_rejects_half():
