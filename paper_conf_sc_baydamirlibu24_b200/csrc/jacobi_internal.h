@@ -17,6 +17,8 @@
 #define JB_SMEM_DEFAULT 232448  // B200 opt-in dynamic shared memory per block (227 KB)
 #define JB_TB_KMAX2 5           // deepest time block of the 2D time-blocked kernel (tblock.cu)
 #define JB_TB_K2D 5             // its default depth (auto; measured fastest)
+#define JB_TB_PPT5 2            // default cell pairs per lane at K = 5
+#define JB_TB_LAG 1             // default wavefront lag of the odd-K march
 
 // Scratch planes after each slab buffer for the time-blocked kernel's edge zones of depth K
 // (tblock.cu): K-1 slots for the neighbour's intermediate levels + the side's own level-m planes,

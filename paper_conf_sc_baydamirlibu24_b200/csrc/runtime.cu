@@ -561,22 +561,26 @@ int run_cpufree_k1(jacobi_ctx *h, int64_t iters) {
 // iterations: per launch group the roles and flags of plan_launch (boundary CTAs run the edge
 // zones with the per-iteration exchange, then join the interior), the guided dynamic schedule
 // over the interior planes the edge zones leave, and the ring shortened to the smem budget.
-void tblock_choice(const jacobi_ctx *h, int *k_out, int *ppt_out) {
+void tblock_choice(const jacobi_ctx *h, int *k_out, int *ppt_out, int *lag_out) {
   int k = h->tb_k >= 2 ? (int)std::min<int64_t>(h->tb_k, JB_TB_KMAX2) : (h->dim == 2 ? JB_TB_K2D : 2);
   if (h->dim == 3) k = 2;
   // every slab needs its edge zones (2K planes) when it has neighbours: shallower blocks otherwise
   const int64_t chunk_min = (h->n_out - 2) / h->total;
   auto fits = [&](int kk) { return h->total == 1 || chunk_min >= 2 * kk; };
-  while (k > 2 && !(fits(k) && jbk::tblock_ncw(h->dim, k, k == 5 ? 2 : 4, 1) > 0)) k -= (k == 3 ? 1 : 2);
-  int ppt = 4;
-  if (k == 5) ppt = 2;
-  if (h->tb_ppt > 0 && h->dim == 2 && jbk::tblock_ncw(2, k, (int)h->tb_ppt, 1) > 0) ppt = (int)h->tb_ppt;
+  auto dflt_ppt = [](int kk) { return kk == 5 ? JB_TB_PPT5 : 4; };
+  while (k > 2 && !(fits(k) && jbk::tblock_ncw(h->dim, k, dflt_ppt(k), 1, 1) > 0)) k -= (k == 3 ? 1 : 2);
+  int ppt = dflt_ppt(k), lag = k > 2 ? JB_TB_LAG : 1;
+  if (h->tb_ppt > 0 && jbk::tblock_ncw(h->dim, k, (int)h->tb_ppt, lag, 1) > 0) ppt = (int)h->tb_ppt;
+  if (h->tb_lag > 0 && jbk::tblock_ncw(h->dim, k, ppt, (int)h->tb_lag, 1) > 0) lag = (int)h->tb_lag;
+  if (jbk::tblock_ncw(h->dim, k, ppt, lag, 1) == 0) lag = 1;
+  if (jbk::tblock_ncw(h->dim, k, ppt, lag, 1) == 0) ppt = dflt_ppt(k);
   if (!fits(k)) k = 0;
   *k_out = k;
   *ppt_out = ppt;
+  *lag_out = lag;
 }
 
-int run_tblock(jacobi_ctx *h, int64_t iters, int K, int ppt) {
+int run_tblock(jacobi_ctx *h, int64_t iters, int K, int ppt, int lag) {
   auto groups = launch_groups(h);
   std::vector<LaunchPlan> plans(groups.size());
   // roles must match across slabs; two CTAs per SM only for K = 2
@@ -598,7 +602,7 @@ int run_tblock(jacobi_ctx *h, int64_t iters, int K, int ppt) {
       g.units = g.units_x * g.units_y;
       g.stage_doubles = g.rh * g.ws;
     } else if (K > 2) {  // odd K: JB_NCW warps x (64 ppt - 2(K-1)) output columns per strip
-      g.tx = jbk::tblock_ncw(2, K, ppt, 1) * (64 * ppt - 2 * (K - 1));
+      g.tx = jbk::tblock_ncw(2, K, ppt, lag, 1) * (64 * ppt - 2 * (K - 1));
       g.ws = g.tx + 2 * K + 2;
       g.units_x = (int)((h->nx - 2 + g.tx - 1) / g.tx);
       g.units_y = 1;
@@ -644,7 +648,7 @@ int run_tblock(jacobi_ctx *h, int64_t iters, int K, int ppt) {
     if (jbk::tblock_smem(g) > (size_t)smem_optin) return JACOBI_EINVAL;
     L.smem = jbk::tblock_smem(g);
     int occ = 0;
-    CK(jbk::prepare_tblock(g, K, ppt, per_sm, L.smem, &occ));
+    CK(jbk::prepare_tblock(g, K, ppt, lag, per_sm, L.smem, &occ));
     if (occ < per_sm) {
       if (getenv("JACOBI_DEBUG")) fprintf(stderr, "[jacobi] tblock: occupancy %d < %d (smem %zu)\n", occ, per_sm, L.smem);
       return JACOBI_ENOCOOP;
@@ -666,7 +670,7 @@ int run_tblock(jacobi_ctx *h, int64_t iters, int K, int ppt) {
     CK(cudaSetDevice(L.device));
     Slab &s0 = h->slabs[L.slab_idx[0]];
     CK(cudaEventRecord(s0.ev0, L.stream));
-    CK(jbk::launch_tblock(L.P, K, ppt, per_sm, L.grid, L.smem, L.stream));
+    CK(jbk::launch_tblock(L.P, K, ppt, lag, per_sm, L.grid, L.smem, L.stream));
     CK(cudaEventRecord(s0.ev1, L.stream));
   }
   int rc_all = JACOBI_OK;
@@ -697,8 +701,8 @@ int run_cpufree(jacobi_ctx *h, int64_t iters) {
   h->last_resident = 0;
   const bool nocomp = h->flags & JACOBI_FLAG_NO_COMPUTE;
   // P > 1: every slab needs the two edge zones (>= 2K planes); the NVSHMEM variant keeps jb_sweep
-  int K = 0, ppt = 0;
-  tblock_choice(h, &K, &ppt);
+  int K = 0, ppt = 0, lag = 1;
+  tblock_choice(h, &K, &ppt, &lag);
   const bool eligible = h->tblock != 0 && !nocomp && h->norm_every <= 0 && h->kind != KIND_SHMEM && K >= 2;
   if (h->tblock == 1 && !eligible) return JACOBI_EINVAL;
   // auto picks it where it measured faster than the per-iteration kernel: 2D (3D: forced only)
@@ -720,7 +724,7 @@ int run_cpufree(jacobi_ctx *h, int64_t iters) {
   }
   double ms = 0;
   if (tb_iters > 0) {
-    int rc = run_tblock(h, tb_iters, K, ppt);
+    int rc = run_tblock(h, tb_iters, K, ppt, lag);
     if (rc) return rc;
     ms = h->last_ms_max;
     h->last_tblock = tb_iters;
@@ -854,6 +858,7 @@ static int64_t *param_slot(jacobi_t h, const char *name) {
   if (!std::strcmp(name, "tb_ctas")) return &h->tb_ctas;
   if (!std::strcmp(name, "tb_k")) return &h->tb_k;
   if (!std::strcmp(name, "tb_ppt")) return &h->tb_ppt;
+  if (!std::strcmp(name, "tb_lag")) return &h->tb_lag;
   if (!std::strcmp(name, "last_tb_k")) return &h->last_tb_k;
   if (!std::strcmp(name, "last_tblock")) return &h->last_tblock;
   return nullptr;

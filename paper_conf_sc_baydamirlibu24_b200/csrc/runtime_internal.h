@@ -33,10 +33,11 @@ cudaError_t prepare_resident(int dim, int cpp, size_t smem, int *blocks_per_sm);
 cudaError_t launch_resident(const JbParams &p, int cpp, int grid, size_t smem, cudaStream_t st);
 cudaError_t launch_neighbour_wait(const JbParams &p, unsigned long long target, cudaStream_t st);
 int tblock_ty();
-int tblock_ncw(int dim, int k, int ppt, int per_sm);
+int tblock_ncw(int dim, int k, int ppt, int lag, int per_sm);
 size_t tblock_smem(const JbGeom &g);
-cudaError_t prepare_tblock(const JbGeom &g, int k, int ppt, int per_sm, size_t smem, int *blocks_per_sm);
-cudaError_t launch_tblock(const JbParams &p, int k, int ppt, int per_sm, int grid, size_t smem, cudaStream_t st);
+cudaError_t prepare_tblock(const JbGeom &g, int k, int ppt, int lag, int per_sm, size_t smem, int *blocks_per_sm);
+cudaError_t launch_tblock(const JbParams &p, int k, int ppt, int lag, int per_sm, int grid, size_t smem,
+                          cudaStream_t st);
 }  // namespace jbk
 
 namespace jbrt {
@@ -170,6 +171,7 @@ struct jacobi_ctx {
   int64_t tb_ctas = 1;         // CTAs per SM of the temporally blocked kernel (1 or 2; K = 2 only)
   int64_t tb_k = -1;           // iterations per time block: -1 auto (2D: JB_TB_K2D, 3D: 2), 2D: 2, 3, 5
   int64_t tb_ppt = -1;         // 2D cell pairs per thread and level: -1 auto (4 for K <= 3, 2 for K = 5)
+  int64_t tb_lag = -1;         // 2D odd K: wavefront lag between levels (1 or 2; -1 auto)
   int64_t last_tb_k = 0;       // read-only: K of the last time-blocked run
   int64_t last_tblock = 0;     // read-only: iterations of the last CPU-Free run done time-blocked
   int64_t norm_every = 0;      // N4: check the update norm every k iterations (0 = off)
@@ -233,9 +235,9 @@ int plan_resident(jacobi_ctx *h, const std::vector<int> &idx, LaunchPlan &L);
 int setup_norm(jacobi_ctx *h, LaunchPlan &L);
 int run_cpufree(jacobi_ctx *h, int64_t iters);
 int run_cpufree_k1(jacobi_ctx *h, int64_t iters);
-int run_tblock(jacobi_ctx *h, int64_t iters, int k, int ppt);
+int run_tblock(jacobi_ctx *h, int64_t iters, int k, int ppt, int lag);
 // Time-block depth and pairs per thread the runtime would use for this handle (K = 0: none).
-void tblock_choice(const jacobi_ctx *h, int *k, int *ppt);
+void tblock_choice(const jacobi_ctx *h, int *k, int *ppt, int *lag);
 int ensure_nccl(jacobi_ctx *h);
 int time_begin(jacobi_ctx *h);
 int time_end(jacobi_ctx *h, int64_t iters);

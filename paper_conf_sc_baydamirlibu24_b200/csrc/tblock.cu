@@ -218,15 +218,15 @@ __device__ __forceinline__ void tb2_item(const JbGeom &g, const Ring &R, RingPos
 
 // ---------------------------------------------------------------- 2D, deeper time blocks (K odd)
 // K = 3, 5: levels 1 .. K of one item, no extra cells.  Warp w computes every level over the same
-// 64 PPT columns s_w .. s_w + 64 PPT - 1 (s_w = x0 + w WO - (K-1), WO = 64 PPT - 2 (K-1)): level
-// 1 from the level-0 stage (x neighbours from the stage), level k >= 2 from level k-1 in
-// registers (x neighbours by shuffles).  At the two ends of the segment a level loses one valid
-// column per side (the shuffle wraps around), so level K is valid on the middle WO columns, which
-// are this warp's outputs; neighbouring warps overlap by 2(K-1) columns, never communicate.  With
-// K odd both the level-1 loads (stage index 2 + 2 kk) and the level-K stores (column s_w + K-1,
-// odd x) stay 16-byte aligned.  Rows: the march takes one level-0 row R per step and computes
-// level k of row R-k for every k (a wavefront), so each level keeps three rows in registers;
-// register set m % 3 holds the row computed at step m (static rotation, unrolled by three).
+// 64 PPT columns s_w .. s_w + 64 PPT - 1 (s_w = x0 + w WO - (K-1), WO = 64 PPT - 2 (K-1)); lane l
+// owns the PPT contiguous cell pairs kk = l PPT + i.  Level 1 comes from the level-0 stage,
+// level k >= 2 from level k-1 in registers: x neighbours inside a lane are its own registers,
+// across lanes one shuffle per side and level.  At the two ends of the segment a level loses one
+// valid column per side (the shuffle wraps around), so level K is valid on the middle WO columns,
+// which are this warp's outputs; neighbouring warps overlap by 2(K-1) columns and never
+// communicate.  With K odd both the level-1 loads (stage index 2 + 2 kk) and the level-K
+// stores (column s_w + K-1, odd x) stay 16-byte aligned.  Rows: the march takes one level-0 row
+// per step and advances every level by one row (a wavefront, see tbk_march).
 // Cells outside the interior (Dirichlet rows / columns, the garbage columns past the grid)
 // keep their previous level — the definition's untouched boundary — and never reach an
 // interior output.
@@ -238,45 +238,59 @@ struct TbkLane {
 template <int PPT, bool FAST, bool STEADY>
 __device__ __forceinline__ void tbk_level1(const TbkLane &L, const double *sm, const double *sc, const double *sn,
                                            bool rowin, double2 *V) {
+  double2 S0[PPT], C0[PPT], N0[PPT];
 #pragma unroll
   for (int i = 0; i < PPT; ++i) {
-    const int j = L.j0 + 64 * i;
-    const double2 S0 = lds2(sm + j), C0 = lds2(sc + j), N0 = lds2(sn + j);
-    const double W = sc[j - 1], E = sc[j + 2];
+    S0[i] = lds2(sm + L.j0 + 2 * i);
+    C0[i] = lds2(sc + L.j0 + 2 * i);
+    N0[i] = lds2(sn + L.j0 + 2 * i);
+  }
+  const double Wl = sc[L.j0 - 1], Er = sc[L.j0 + 2 * PPT];
+#pragma unroll
+  for (int i = 0; i < PPT; ++i) {
+    const double W = i == 0 ? Wl : C0[i - 1].y;
+    const double E = i == PPT - 1 ? Er : C0[i + 1].x;
     // oracle order: ((x+1) + (x-1)) + (y+1) + (y-1), then * 0.25
-    const double l0 = 0.25 * (((C0.y + W) + N0.x) + S0.x);
-    const double l1 = 0.25 * (((E + C0.x) + N0.y) + S0.y);
+    const double l0 = 0.25 * (((C0[i].y + W) + N0[i].x) + S0[i].x);
+    const double l1 = 0.25 * (((E + C0[i].x) + N0[i].y) + S0[i].y);
     if (FAST && STEADY) {
       V[i] = make_double2(l0, l1);
     } else {
       const bool r = STEADY || rowin;
-      V[i].x = (r && (FAST || (L.ok >> i & 1u))) ? l0 : C0.x;
-      V[i].y = (r && (FAST || (L.full >> i & 1u))) ? l1 : C0.y;
+      V[i].x = (r && (FAST || (L.ok >> i & 1u))) ? l0 : C0[i].x;
+      V[i].y = (r && (FAST || (L.full >> i & 1u))) ? l1 : C0[i].y;
     }
   }
 }
 
-// Level k >= 2 of the middle row of (S, Cm, N) (level k-1).  Lane l takes lane l-1's .y (W) and
-// lane l+1's .x (E); lane 0 / 31 the wrapped value of the previous / next pair.  STORE: level K,
-// written to o (row pointer of this lane's pair 0) instead of V.
+// A double from lane src (two 32-bit shuffles, halves kept in place).
+__device__ __forceinline__ double shfl_d(double v, int src) {
+  double r;
+  asm("{\n .reg .b32 lo, hi;\n mov.b64 {lo, hi}, %1;\n shfl.sync.idx.b32 lo, lo, %2, 0x1f, -1;\n"
+      " shfl.sync.idx.b32 hi, hi, %2, 0x1f, -1;\n mov.b64 %0, {lo, hi};\n}"
+      : "=d"(r)
+      : "d"(v), "r"(src));
+  return r;
+}
+
+// Level k >= 2 of the middle row of (S, Cm, N) (level k-1): W of pair 0 from lane l-1's last
+// pair, E of the last pair from lane l+1's first (lane 0 / 31: wrapped, outside the valid span).
+// STORE: level K, written to o (this lane's pair 0 in the output row) instead of V.
 template <int PPT, bool FAST, bool STEADY, bool STORE>
 __device__ __forceinline__ void tbk_levelk(const TbkLane &L, const double2 *S, const double2 *Cm, const double2 *N,
                                            bool rowin, int lane, double2 *V, double *o) {
-  double rw_prev = Cm[0].x;  // lane 0, pair 0: outside the valid span (any finite value)
-  double re_next = __shfl_sync(0xffffffffu, Cm[0].x, (lane + 1) & 31);
+  const double Wl = shfl_d(Cm[PPT - 1].y, (lane + 31) & 31);
+  const double Er = shfl_d(Cm[0].x, (lane + 1) & 31);
 #pragma unroll
   for (int i = 0; i < PPT; ++i) {
-    const double rw = __shfl_sync(0xffffffffu, Cm[i].y, (lane + 31) & 31);
-    const double re = re_next;
-    if (i + 1 < PPT) re_next = __shfl_sync(0xffffffffu, Cm[i + 1].x, (lane + 1) & 31);
-    const double W = lane == 0 ? rw_prev : rw;
-    const double E = lane == 31 ? re_next : re;
+    const double W = i == 0 ? Wl : Cm[i - 1].y;
+    const double E = i == PPT - 1 ? Er : Cm[i + 1].x;
     const double o0 = 0.25 * (((Cm[i].y + W) + N[i].x) + S[i].x);
     const double o1 = 0.25 * (((E + Cm[i].x) + N[i].y) + S[i].y);
     if (STORE) {
       if (L.st >> i & 1u) {
-        if (FAST) *reinterpret_cast<double2 *>(o + 64 * i) = make_double2(o0, o1);
-        else store_pair(o + 64 * i, o0, o1, L.full >> i & 1u);
+        if (FAST) *reinterpret_cast<double2 *>(o + 2 * i) = make_double2(o0, o1);
+        else store_pair(o + 2 * i, o0, o1, L.full >> i & 1u);
       }
     } else if (FAST && STEADY) {
       V[i] = make_double2(o0, o1);
@@ -285,63 +299,87 @@ __device__ __forceinline__ void tbk_levelk(const TbkLane &L, const double2 *S, c
       V[i].x = (r && (FAST || (L.ok >> i & 1u))) ? o0 : Cm[i].x;
       V[i].y = (r && (FAST || (L.full >> i & 1u))) ? o1 : Cm[i].y;
     }
-    rw_prev = rw;
   }
 }
 
-template <int K, int PPT, bool FAST>
-__device__ __forceinline__ void tbk_march(const TbkLane &L, const Ring &R, RingPos q, int64_t a, int64_t b,
-                                          int64_t C, int64_t r0, int64_t r1, double *dst, int64_t pe, int lane) {
-  double2 X[K - 1][3][PPT];  // X[k-1][m % 3]: level k of the row computed at step m
-  const int64_t Rs = a - K >= 0 ? r0 + 2 : r0 + 1;  // first step (r0 = 0 when a - K < 0)
-  const int64_t Re = b + K;                          // last step: level K of row b
+// The wavefront: at step R (level-0 row R enters) level k computes row R - 1 - LAG (k-1), which
+// needs level k-1 rows up to R - LAG (k-1): computed LAG-1 steps earlier.  LAG = 1: the levels of
+// a step form one dependency chain, three rows per level in registers; LAG = 2: the K levels of a
+// step are independent (more instruction-level parallelism, four rows per level).  Set m % NS
+// of a level holds its row computed at step m (static rotation, the loop unrolled by NS).
+template <int K, int PPT, int LAG, bool FAST>
+__device__ __forceinline__ void tbk_march(const TbkLane &L, const Ring &R, RingPos q, int a, int b, int C, int r0,
+                                          int r1, double *dst, int64_t pe, int lane) {
+  constexpr int NS = LAG + 2;
+  double2 X[K - 1][NS][PPT];  // X[k-1][m % NS]: level k of the row computed at step m
+  const int Rs = a - K >= 0 ? r0 + 2 : r0 + 1;  // first step (r0 = 0 when a - K < 0)
+  const int Re = b + 1 + LAG * (K - 1);         // last step: level K of row b
+  // steady window: every level's row is needed and interior, level K is stored
+  const int Ws = a + 1 + LAG * (K - 1), We = min(b + K, C + 1);
+  double *o = dst + (int64_t)(Rs - 1 - LAG * (K - 1)) * pe;  // output row of step Rs (advanced per step)
   // stage positions of level-0 rows R-2, R-1, R, clamped to r0 .. r1
   RingPos pm = q, pc = Rs == r0 + 2 ? ring_add(q, 1u, R.S) : q, pn = pc;
   if (Rs <= r1) pn = ring_add(q, (uint32_t)(Rs - r0), R.S);
   R.wait_full(pm);
   R.wait_full(pc);
-  // one step: level-0 row Rr enters; level k of row Rr-k for k = 1..K
-  auto step = [&](auto u_ct, auto steady_ct, int64_t Rr) {
+  auto step = [&](auto u_ct, auto steady_ct, int Rr) {
     constexpr int U = decltype(u_ct)::value;
     constexpr bool ST = decltype(steady_ct)::value;
-    constexpr int Sx = (U + 1) % 3, Cx = (U + 2) % 3;
-    if (Rr <= r1) R.wait_full(pn);
-    tbk_level1<PPT, FAST, ST>(L, R.stage(pm), R.stage(pc), R.stage(pn), Rr - 1 >= 1 && Rr - 1 <= C, X[0][U]);
-    if (Rr - 2 >= r0 && Rr - 2 <= r1) R.release(pm, lane);  // row Rr-2 is no longer needed
+    // level k-1 rows r+1, r, r-1 were computed at steps m-(LAG-1), m-LAG, m-LAG-1
+    constexpr int SN = (U + NS - (LAG - 1)) % NS, SC = (U + NS - LAG) % NS, SS = (U + 2 * NS - LAG - 1) % NS;
+    // level k computes row Rr-1-LAG(k-1) if it lies in its range [a-(K-k), b+(K-k)] ∩ [0, C+1]
+    auto need = [&](int k, int r) { return r >= max(a - (K - k), 0) && r <= min(b + (K - k), C + 1); };
+    if (ST || Rr <= r1) R.wait_full(pn);
+    if (ST || need(1, Rr - 1))
+      tbk_level1<PPT, FAST, ST>(L, R.stage(pm), R.stage(pc), R.stage(pn), Rr - 1 >= 1 && Rr - 1 <= C, X[0][U]);
+    if (ST || (Rr - 2 >= r0 && Rr - 2 <= r1)) R.release(pm, lane);  // row Rr-2 is no longer needed
 #pragma unroll
-    for (int k = 2; k < K; ++k)
-      tbk_levelk<PPT, FAST, ST, false>(L, X[k - 2][Sx], X[k - 2][Cx], X[k - 2][U], Rr - k >= 1 && Rr - k <= C, lane,
-                                       X[k - 1][U], nullptr);
-    if (Rr - K >= a)
-      tbk_levelk<PPT, FAST, ST, true>(L, X[K - 2][Sx], X[K - 2][Cx], X[K - 2][U], true, lane, nullptr,
-                                      dst + (Rr - K) * pe);
+    for (int k = 2; k < K; ++k) {
+      const int r = Rr - 1 - LAG * (k - 1);
+      if (ST || need(k, r))
+        tbk_levelk<PPT, FAST, ST, false>(L, X[k - 2][SS], X[k - 2][SC], X[k - 2][SN], r >= 1 && r <= C, lane,
+                                         X[k - 1][U], nullptr);
+    }
+    const int ro = Rr - 1 - LAG * (K - 1);
+    if (ST || (ro >= a && ro <= b))
+      tbk_levelk<PPT, FAST, ST, true>(L, X[K - 2][SS], X[K - 2][SC], X[K - 2][SN], true, lane, nullptr, o);
+    o += pe;
     pm = pc;
     pc = pn;
-    if (Rr + 1 <= r1) pn.advance(R.S);
+    if (Rr + 1 <= r1) {  // branch-free ring advance
+      const uint32_t sl = pn.slot + 1u;
+      const bool wrap = sl == R.S;
+      pn.slot = wrap ? 0u : sl;
+      pn.phase ^= wrap ? 1u : 0u;
+    }
   };
-  using U0 = std::integral_constant<int, 0>;
-  using U1 = std::integral_constant<int, 1>;
-  using U2 = std::integral_constant<int, 2>;
   using TT = std::integral_constant<bool, true>;
   using TF = std::integral_constant<bool, false>;
-  int64_t Rr = Rs;
-  for (; Rr <= Re; Rr += 3) {
-    if (Rr >= K && Rr + 2 <= C + 1 && Rr + 2 <= Re) {  // every level's row interior: no row masks
-      step(U0{}, TT{}, Rr);
-      step(U1{}, TT{}, Rr + 1);
-      step(U2{}, TT{}, Rr + 2);
-    } else {
-      step(U0{}, TF{}, Rr);
-      if (Rr + 1 <= Re) step(U1{}, TF{}, Rr + 1);
-      if (Rr + 2 <= Re) step(U2{}, TF{}, Rr + 2);
+  auto group = [&](auto steady_ct, int Rr) {
+    constexpr bool ST = decltype(steady_ct)::value;
+    step(std::integral_constant<int, 0>{}, steady_ct, Rr);
+    if (ST || Rr + 1 <= Re) step(std::integral_constant<int, 1>{}, steady_ct, Rr + 1);
+    if (ST || Rr + 2 <= Re) step(std::integral_constant<int, 2>{}, steady_ct, Rr + 2);
+    if constexpr (NS == 4)
+      if (ST || Rr + 3 <= Re) step(std::integral_constant<int, 3 % NS>{}, steady_ct, Rr + 3);
+  };
+  // groups of NS steps: a masked prefix, the steady middle, a masked suffix
+  const int nsteady = Ws <= We ? (We - max(Ws, Rs) + 1) / NS : 0;  // whole steady groups
+  int Rr = Rs;
+  if (nsteady > 0) {
+    for (; Rr < Ws; Rr += NS) group(TF{}, Rr);  // the prefix keeps the group phase (set rotation)
+    if (Rr + NS - 1 <= We) {
+      const int Rend = Rr + ((We - Rr + 1) / NS) * NS;
+      for (; Rr < Rend; Rr += NS) group(TT{}, Rr);
     }
   }
+  for (; Rr <= Re; Rr += NS) group(TF{}, Rr);
   // rows Re-1, Re (if they exist) were not released by the march: pm, pc after the last step
   if (Re - 1 <= r1) R.release(pm, lane);
   if (Re <= r1) R.release(pc, lane);
 }
 
-template <int K, int PPT>
+template <int K, int PPT, int LAG>
 __device__ __forceinline__ void tbk_item(const JbGeom &g, const Ring &R, RingPos &q, int unit, int64_t a, int64_t b,
                                          int64_t C, double *out, int warp, int lane) {
   constexpr int WO = 64 * PPT - 2 * (K - 1);
@@ -360,11 +398,11 @@ __device__ __forceinline__ void tbk_item(const JbGeom &g, const Ring &R, RingPos
   }
   const int64_t sw = ow - (K - 1);
   TbkLane L;
-  L.j0 = warp * WO + 2 + 2 * lane;
+  L.j0 = warp * WO + 2 + 2 * PPT * lane;
   L.ok = L.full = L.st = 0;
 #pragma unroll
   for (int i = 0; i < PPT; ++i) {
-    const int kk = 32 * i + lane;
+    const int kk = PPT * lane + i;
     const int64_t c = sw + 2 * kk;
     const bool ok = c >= 1 && c <= g.nx - 2;
     L.ok |= (ok ? 1u : 0u) << i;
@@ -372,9 +410,9 @@ __device__ __forceinline__ void tbk_item(const JbGeom &g, const Ring &R, RingPos
     L.st |= (ok && kk >= (K - 1) / 2 && kk < 32 * PPT - (K - 1) / 2 ? 1u : 0u) << i;
   }
   const bool fast = sw >= 1 && sw + 64 * PPT - 1 <= g.nx - 2;
-  double *dst = out + 3 + sw + 2 * lane;
-  if (fast) tbk_march<K, PPT, true>(L, R, q0, a, b, C, r0, r1, dst, g.plane_elems, lane);
-  else tbk_march<K, PPT, false>(L, R, q0, a, b, C, r0, r1, dst, g.plane_elems, lane);
+  double *dst = out + 3 + sw + 2 * PPT * lane;
+  if (fast) tbk_march<K, PPT, LAG, true>(L, R, q0, (int)a, (int)b, (int)C, (int)r0, (int)r1, dst, g.plane_elems, lane);
+  else tbk_march<K, PPT, LAG, false>(L, R, q0, (int)a, (int)b, (int)C, (int)r0, (int)r1, dst, g.plane_elems, lane);
 }
 
 // ---------------------------------------------------------------- 3D (7-point)
@@ -639,7 +677,7 @@ __device__ bool tb_edge(const JbGeom &g, const JbSlab &SL, const JbParams &P, in
   return true;
 }
 
-template <int NCW, int DIM, int K, int TP>
+template <int NCW, int DIM, int K, int TP, int LAG>
 __device__ __forceinline__ void tb_body(const JbParams &P) {
   static_assert(K == 2 || (DIM == 2 && (K & 1)), "3D: K = 2; 2D: K = 2 or odd");
   extern __shared__ __align__(128) unsigned char smem[];
@@ -772,7 +810,7 @@ __device__ __forceinline__ void tb_body(const JbParams &P) {
         if (d.kind == TB_END) break;
         if constexpr (DIM == 3) tb3_item<TP>(g, R, q, d.unit, d.a, d.b, C, nxt, warp, lane);
         else if constexpr (K == 2) tb2_item<TP>(g, R, q, d.unit, d.a, d.b, C, nxt, warp, lane);
-        else tbk_item<K, TP>(g, R, q, d.unit, d.a, d.b, C, nxt, warp, lane);
+        else tbk_item<K, TP, LAG>(g, R, q, d.unit, d.a, d.b, C, nxt, warp, lane);
       }
       fence_proxy_async_global();  // generic-proxy stores before the next block's bulk reads
     }
@@ -796,21 +834,21 @@ __device__ __forceinline__ void tb_body(const JbParams &P) {
 // One CTA per SM (up to 224 registers per thread) or two (96: 2 x 9 warps fit the register file
 // only at <= 96 registers, given the 4-warp allocation granularity).  K = iterations per time
 // block; TP = pairs per thread along x (2D) or rows per tile (3D).
-template <int DIM, int K, int TP, int NCW = JB_NCW>
+template <int DIM, int K, int TP, int NCW = JB_NCW, int LAG = 1>
 __global__ void __launch_bounds__((NCW + 1) * 32, 1) jb_tblock(const __grid_constant__ JbParams P) {
-  tb_body<NCW, DIM, K, TP>(P);
+  tb_body<NCW, DIM, K, TP, LAG>(P);
 }
 template <int TP>
 __global__ void __maxnreg__(96) jb_tblock2d_x2(const __grid_constant__ JbParams P) {
-  tb_body<JB_NCW, 2, 2, TP>(P);
+  tb_body<JB_NCW, 2, 2, TP, 1>(P);
 }
 
 constexpr int TB_TY = 4;  // 3D tile rows (level-1 rows TY+2 carried per plane in registers)
 
-// Kernel for (dim, K, pairs per thread, CTAs per SM) and its consumer warp count; nullptr if not
-// instantiated.  Odd K holds 2(K-1) level rows per lane: with PPT = 4 (K = 3) or K = 5 the
-// kernel needs > 168 registers, i.e. 7 consumer warps (256 threads: up to 255 registers).
-const void *tblock_fn(int dim, int k, int ppt, int per_sm, int *ncw) {
+// Kernel for (dim, K, pairs per thread, wavefront lag, CTAs per SM) and its consumer warp count;
+// nullptr if not instantiated.  Odd K holds (LAG+2)(K-1) level rows per lane: beyond ~168
+// registers, i.e. 7 consumer warps (256 threads: up to 255 registers).
+const void *tblock_fn(int dim, int k, int ppt, int lag, int per_sm, int *ncw) {
 #define JB_TB(...) reinterpret_cast<const void *>(&__VA_ARGS__)
   *ncw = JB_NCW;
   if (dim == 3) return k == 2 ? JB_TB(jb_tblock<3, 2, TB_TY>) : nullptr;
@@ -819,8 +857,14 @@ const void *tblock_fn(int dim, int k, int ppt, int per_sm, int *ncw) {
     return ppt >= 4 ? JB_TB(jb_tblock<2, 2, 4>) : ppt == 2 ? JB_TB(jb_tblock<2, 2, 2>) : JB_TB(jb_tblock<2, 2, 1>);
   }
   if (per_sm >= 2) return nullptr;
-  if (k == 3 && ppt == 2) return JB_TB(jb_tblock<2, 3, 2>);
   *ncw = 7;
+  if (lag == 2) {
+    if (k == 3 && ppt == 2) return JB_TB(jb_tblock<2, 3, 2, 7, 2>);
+    if (k == 5 && ppt == 1) return JB_TB(jb_tblock<2, 5, 1, 7, 2>);
+    if (k == 5 && ppt == 2) return JB_TB(jb_tblock<2, 5, 2, 7, 2>);
+    return nullptr;
+  }
+  if (k == 3 && ppt == 2) return JB_TB(jb_tblock<2, 3, 2, 7>);
   if (k == 3 && ppt == 4) return JB_TB(jb_tblock<2, 3, 4, 7>);
   if (k == 5 && ppt == 2) return JB_TB(jb_tblock<2, 5, 2, 7>);
   return nullptr;
@@ -833,9 +877,9 @@ namespace jbk {
 
 int tblock_ty() { return TB_TY; }
 // consumer warps of the kernel for (dim, k, ppt) with one CTA per SM; 0 if not instantiated
-int tblock_ncw(int dim, int k, int ppt, int per_sm) {
+int tblock_ncw(int dim, int k, int ppt, int lag, int per_sm) {
   int ncw = 0;
-  return tblock_fn(dim, k, ppt, per_sm, &ncw) ? ncw : 0;
+  return tblock_fn(dim, k, ppt, lag, per_sm, &ncw) ? ncw : 0;
 }
 
 // Dynamic shared memory of the temporally blocked kernel: header + ring stages.
@@ -844,9 +888,9 @@ size_t tblock_smem(const JbGeom &g) {
   return (hdr + 127) / 128 * 128 + (size_t)g.stages * g.stage_doubles * 8;
 }
 
-cudaError_t prepare_tblock(const JbGeom &g, int k, int ppt, int per_sm, size_t smem, int *blocks_per_sm) {
+cudaError_t prepare_tblock(const JbGeom &g, int k, int ppt, int lag, int per_sm, size_t smem, int *blocks_per_sm) {
   int ncw = 0;
-  const void *fn = tblock_fn(g.dim, k, ppt, per_sm, &ncw);
+  const void *fn = tblock_fn(g.dim, k, ppt, lag, per_sm, &ncw);
   if (!fn) return cudaErrorInvalidValue;
   cudaError_t e = cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
   if (e != cudaSuccess) return e;
@@ -855,10 +899,11 @@ cudaError_t prepare_tblock(const JbGeom &g, int k, int ppt, int per_sm, size_t s
   return cudaOccupancyMaxActiveBlocksPerMultiprocessor(blocks_per_sm, fn, (ncw + 1) * 32, smem);
 }
 
-cudaError_t launch_tblock(const JbParams &p, int k, int ppt, int per_sm, int grid, size_t smem, cudaStream_t st) {
+cudaError_t launch_tblock(const JbParams &p, int k, int ppt, int lag, int per_sm, int grid, size_t smem,
+                          cudaStream_t st) {
   void *args[] = {const_cast<JbParams *>(&p)};
   int ncw = 0;
-  const void *fn = tblock_fn(p.g.dim, k, ppt, per_sm, &ncw);
+  const void *fn = tblock_fn(p.g.dim, k, ppt, lag, per_sm, &ncw);
   if (!fn) return cudaErrorInvalidValue;
   return cudaLaunchCooperativeKernel(fn, dim3(grid), dim3((ncw + 1) * 32), args, smem, st);
 }

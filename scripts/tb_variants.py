@@ -14,12 +14,12 @@ import oracle  # noqa: E402
 import paper_conf_sc_baydamirlibu24_b200 as jb  # noqa: E402
 from jacobi_inputs import u12  # noqa: E402
 
-VARIANTS = [(2, 4), (3, 2), (3, 4), (5, 2)]
+VARIANTS = [(2, 4, 1), (3, 2, 1), (3, 2, 2), (5, 2, 1)]
 
 
-def run(shape, iters, k, ppt, virtual=0, extra=None):
+def run(shape, iters, k, ppt, lag, virtual=0, extra=None):
     with jb.Jacobi(shape, virtual=virtual) as j:
-        for n, v in {"tblock": 1, "resident": 0, "tb_k": k, "tb_ppt": ppt, **(extra or {})}.items():
+        for n, v in {"tblock": 1, "resident": 0, "tb_k": k, "tb_ppt": ppt, "tb_lag": lag, **(extra or {})}.items():
             j.set_param(n, v)
         f = u12(shape, 3)
         j.scatter(f)
@@ -29,15 +29,15 @@ def run(shape, iters, k, ppt, virtual=0, extra=None):
 
 def check():
     bad = 0
-    for k, ppt in VARIANTS:
+    for k, ppt, lag in VARIANTS:
         for shape, iters, virtual in [((40, 3000), 15, 0), ((70, 2051), 11, 0), ((300, 130), 10, 0), ((5, 4100), 7, 0),
                                       ((3, 3), 5, 0), ((1000, 37), 20, 0), ((97, 1990), 15, 2), ((130, 2200), 30, 3),
                                       ((64, 1500), 20, 5)]:
-            f, got, kk, tb = run(shape, iters, k, ppt, virtual)
+            f, got, kk, tb = run(shape, iters, k, ppt, lag, virtual)
             exp = oracle.jacobi(f, iters)
             same = np.array_equal(got.view(np.uint64), exp.view(np.uint64))
             n = int(np.count_nonzero(got.view(np.uint64) != exp.view(np.uint64)))
-            print(f"K={k} ppt={ppt} {shape} it={iters} P={virtual or 1}: used K={kk} tb_iters={tb} "
+            print(f"K={k} ppt={ppt} lag={lag} {shape} it={iters} P={virtual or 1}: used K={kk} tb_iters={tb} "
                   f"{'OK' if same else f'MISMATCH {n} cells'}", flush=True)
             bad += not same
     return bad
@@ -46,10 +46,11 @@ def check():
 def timing(iters=200):
     shape = (16384, 16384)
     cells = (shape[0] - 2) * (shape[1] - 2)
-    for k, ppt in VARIANTS:
+    for k, ppt, lag in VARIANTS:
         for mb in (16, 32):
             with jb.Jacobi(shape) as j:
-                for n, v in {"tblock": 1, "resident": 0, "tb_k": k, "tb_ppt": ppt, "tb_min_block": mb}.items():
+                for n, v in {"tblock": 1, "resident": 0, "tb_k": k, "tb_ppt": ppt, "tb_lag": lag,
+                             "tb_min_block": mb}.items():
                     j.set_param(n, v)
                 j.run(iters)
                 ts = []
@@ -57,7 +58,7 @@ def timing(iters=200):
                     j.run(iters)
                     ts.append(j.last_time_ms())
                 t = min(ts)
-                print(f"C2 K={k} ppt={ppt} min_block={mb}: {cells * iters / t / 1e6:.1f} Gcell/s "
+                print(f"C2 K={k} ppt={ppt} lag={lag} min_block={mb}: {cells * iters / t / 1e6:.1f} Gcell/s "
                       f"({t / iters * 1e3:.1f} us/iter, K used {j.get_param('last_tb_k')})", flush=True)
 
 
