@@ -315,6 +315,21 @@ def main():
                 "frac": achieved / peak, "traffic": traffic, "peak_kind": peak_kind,
                 "kernel": kname, "alg_bytes_per_launch": alg_bytes,
                 "alg_bytes_per_cell_update": alg_bytes / (local_cells * iters)}
+    if tb_iters:
+        # K iterations per HBM pass move 16/K B per update, so HBM is no longer the only ceiling:
+        # (a) the bandwidth a one-iteration-per-pass kernel would need for the same throughput
+        #     (16 B per update; > the HBM peak means the time blocking beat the HBM roofline);
+        # (b) the fp64 pipe: 3 DADD + 1 DMUL (2D) / 5 + 1 (3D) per update, no FMA (oracle order),
+        #     64 fp64 lanes per SM per clock (B200 vector fp64 ~37 TFLOP/s; ncu's
+        #     sm__pipe_fp64_cycles_active agrees: DESIGN.md §5.8), 148 SMs at the max SM clock.
+        sm_mhz = (clk or {}).get("sm_max_mhz") or 1965.0
+        fp64_peak = 64 * 148 * sm_mhz * 1e6
+        ops = 4 if dimk == 2 else 6
+        roofline["equivalent_gbs_at_16B"] = 16 * local_cells * iters / (launch_ms / 1e3) / 1e9
+        roofline["equivalent_frac_at_16B"] = roofline["equivalent_gbs_at_16B"] / peak
+        roofline["fp64_pipe"] = {"achieved_ops": ops * local_cells * iters / (launch_ms / 1e3),
+                                 "peak_ops": fp64_peak, "frac": ops * local_cells * iters / (launch_ms / 1e3) / fp64_peak,
+                                 "ops_per_update": ops, "peak_basis": "64 fp64 lanes/SM/clk x 148 SMs x max SM clock (DESIGN.md 5.8)"}
 
     line = {
         "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,

@@ -123,8 +123,8 @@ typedef void *(*jacobi_alloc_fn)(size_t bytes, int device, void *user);
 typedef void (*jacobi_free_fn)(void *ptr, int device, void *user);
 int jacobi_set_allocator(jacobi_alloc_fn alloc, jacobi_free_fn free_fn, void *user);
 /* Bytes of ONE field buffer of slab `slab` (of `nslabs`) for this grid (host-only helper):
- * (chunk + 2) planes (owned + halos) + 4 scratch planes used by the time-blocked
- * kernel's edge zones. */
+ * (chunk + 2) planes (owned + halos) + the time-blocked kernel's edge-zone scratch
+ * (DESIGN.md §5.7-5.9): 34 planes in 2D (time blocks up to K = 5), 11 in 3D (K <= 3). */
 int jacobi_slab_bytes(int64_t nx, int64_t ny, int64_t nz, int stencil, int nslabs, int slab, int64_t *bytes);
 
 /* ---- NVSHMEM variant — exported ONLY by libjacobi_b200_nvshmem.so --------
@@ -157,15 +157,19 @@ int jacobi_set_mode(jacobi_t h, int mode, int flags);
  * as in P:372; 1 = each block waits only for its face-sharing neighbour blocks' flags),
  * "l2hint" (streaming loads with L2 evict_first / evict_last policies; default off — measured
  * 2-3 % slower on B200), "timeout_ms" (watchdog, default 20000), "tblock" (CPU-Free runs with
- * compute (2D and 3D) advance 2 iterations per pass over HBM — temporal blocking; slabs with
- * neighbours keep the per-iteration halo exchange through edge zones — for every whole multiple
- * of 4 iterations, the rest per iteration: -1 auto (default: 2D runs, not when the slab fits on
- * chip, where the resident kernel is used), 0 never, 1 always incl. 3D (EINVAL when a slab has
- * < 4 planes with P > 1, with the norm, in no-compute mode or in the NVSHMEM variant)), "tb_min_block"
- * (smallest dynamic plane block of that kernel, default 16), "tb_ctas" (its CTAs per SM, 1 or 2;
- * 2 only for P = 1).  Read-only: "last_resident" (1 if the last CPU-Free run used the resident
- * kernel), "last_tblock" (iterations of the last CPU-Free run done time-blocked).  Unknown names
- * return JACOBI_EINVAL. */
+ * compute advance K iterations per pass over HBM — temporal blocking; slabs
+ * with neighbours keep the per-iteration halo exchange through edge zones, which need 2K planes
+ * per slab — for every whole multiple of K iterations (2K for K = 2), the rest per iteration:
+ * -1 auto (default: 2D runs, not when the slab fits on chip, where the resident kernel is used),
+ * 0 never, 1 always incl. 3D (EINVAL when a slab has < 4 planes with P > 1, with the norm, in
+ * no-compute mode or in the NVSHMEM variant)), "tb_k" (iterations per time block: -1 auto = 5 in
+ * 2D, 2 in 3D; 2D accepts 2, 3, 5 — a deeper K than the slabs fit falls back to 3, then 2),
+ * "tb_ppt" (2D cell pairs per lane and level: K = 2: from tile_x; K = 3: 2 or 4; K = 5: 2),
+ * "tb_lag" (odd K: wavefront skew between levels, 1 default or 2), "tb_min_block" (smallest
+ * dynamic plane block of that kernel, default 16), "tb_ctas" (its CTAs per SM, 1 or 2; 2 only
+ * for K = 2 and P = 1).  Read-only: "last_resident" (1 if the last CPU-Free run used the resident
+ * kernel), "last_tblock" (iterations of the last CPU-Free run done time-blocked), "last_tb_k"
+ * (its K, 0 if none).  Unknown names return JACOBI_EINVAL. */
 int jacobi_set_param(jacobi_t h, const char *name, int64_t value);
 int jacobi_get_param(jacobi_t h, const char *name, int64_t *value);
 

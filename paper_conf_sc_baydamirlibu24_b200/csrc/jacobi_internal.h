@@ -19,12 +19,15 @@
 #define JB_TB_K2D 5             // its default depth (auto; measured fastest)
 #define JB_TB_PPT5 2            // default cell pairs per lane at K = 5
 #define JB_TB_LAG 1             // default wavefront lag of the odd-K march
+#define JB_TB_KMAX3 3           // deepest time block of the 3D time-blocked kernel
+#define JB_TB_K3D 2             // its default depth (auto)
+#define JB_TB_RPW3 4            // 3D odd K: default rows per warp
 
 // Scratch planes after each slab buffer for the time-blocked kernel's edge zones of depth K
 // (tblock.cu): K-1 slots for the neighbour's intermediate levels + the side's own level-m planes,
-// 2K-m of them for m = 1..K-1.  2D buffers carry enough for JB_TB_KMAX2, 3D ones for K = 2.
+// 2K-m of them for m = 1..K-1.  2D buffers carry enough for JB_TB_KMAX2, 3D ones for JB_TB_KMAX3.
 static inline int64_t jb_edge_planes_k(int K) { return (K - 1) + (int64_t)(K - 1) * 2 * K - (int64_t)(K - 1) * K / 2; }
-static inline int64_t jb_edge_planes(int dim) { return jb_edge_planes_k(dim == 2 ? JB_TB_KMAX2 : 2); }
+static inline int64_t jb_edge_planes(int dim) { return jb_edge_planes_k(dim == 2 ? JB_TB_KMAX2 : JB_TB_KMAX3); }
 
 // Grid geometry in HBM and the tile shape of the march.
 //   element (x, y, z) of slab plane p lives at  buf + p*plane_elems + y*pitch + (x + 3)
@@ -46,7 +49,7 @@ struct JbGeom {
   int32_t res_rs;       // resident kernel: smem row stride in doubles (x at column x + 1)
   int32_t l2hint;       // streaming loads: 1 = L2 evict_first for rows read once, evict_last for
                         // 3D y-halo rows (read again by the neighbouring tile)
-  int32_t pad1;
+  int32_t xch_doubles;  // time-blocked 3D kernel with K odd: shared-memory row exchange (doubles)
 };
 
 struct JbCtrl;

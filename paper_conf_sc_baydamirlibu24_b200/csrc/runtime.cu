@@ -561,23 +561,33 @@ int run_cpufree_k1(jacobi_ctx *h, int64_t iters) {
 // iterations: per launch group the roles and flags of plan_launch (boundary CTAs run the edge
 // zones with the per-iteration exchange, then join the interior), the guided dynamic schedule
 // over the interior planes the edge zones leave, and the ring shortened to the smem budget.
-void tblock_choice(const jacobi_ctx *h, int *k_out, int *ppt_out, int *lag_out) {
-  int k = h->tb_k >= 2 ? (int)std::min<int64_t>(h->tb_k, JB_TB_KMAX2) : (h->dim == 2 ? JB_TB_K2D : 2);
-  if (h->dim == 3) k = 2;
+// (K, pairs per lane, variant) of the time-blocked kernel for this handle; K = 0: none fits.
+// variant: 2D odd K = the wavefront lag (1, 2); 3D odd K = rows per warp of the tile.
+void tblock_choice(const jacobi_ctx *h, int *k_out, int *ppt_out, int *var_out) {
+  const int kmax = h->dim == 2 ? JB_TB_KMAX2 : JB_TB_KMAX3;
+  int k = h->tb_k >= 2 ? (int)std::min<int64_t>(h->tb_k, kmax) : (h->dim == 2 ? JB_TB_K2D : JB_TB_K3D);
   // every slab needs its edge zones (2K planes) when it has neighbours: shallower blocks otherwise
   const int64_t chunk_min = (h->n_out - 2) / h->total;
   auto fits = [&](int kk) { return h->total == 1 || chunk_min >= 2 * kk; };
-  auto dflt_ppt = [](int kk) { return kk == 5 ? JB_TB_PPT5 : 4; };
-  while (k > 2 && !(fits(k) && jbk::tblock_ncw(h->dim, k, dflt_ppt(k), 1, 1) > 0)) k -= (k == 3 ? 1 : 2);
-  int ppt = dflt_ppt(k), lag = k > 2 ? JB_TB_LAG : 1;
-  if (h->tb_ppt > 0 && jbk::tblock_ncw(h->dim, k, (int)h->tb_ppt, lag, 1) > 0) ppt = (int)h->tb_ppt;
-  if (h->tb_lag > 0 && jbk::tblock_ncw(h->dim, k, ppt, (int)h->tb_lag, 1) > 0) lag = (int)h->tb_lag;
-  if (jbk::tblock_ncw(h->dim, k, ppt, lag, 1) == 0) lag = 1;
-  if (jbk::tblock_ncw(h->dim, k, ppt, lag, 1) == 0) ppt = dflt_ppt(k);
+  auto dflt_ppt = [&](int kk) { return h->dim == 3 ? (kk == 2 ? 4 : 1) : kk == 5 ? JB_TB_PPT5 : 4; };
+  auto dflt_var = [&](int kk) { return kk == 2 ? 1 : h->dim == 3 ? JB_TB_RPW3 : JB_TB_LAG; };
+  while (k > 2 && !(fits(k) && jbk::tblock_ncw(h->dim, k, dflt_ppt(k), dflt_var(k), 1) > 0)) k -= (k == 3 ? 1 : 2);
+  int ppt = dflt_ppt(k), var = dflt_var(k);
+  const int64_t var_req = h->dim == 3 ? h->tb_rpw : h->tb_lag;
+  if (h->tb_ppt > 0 && jbk::tblock_ncw(h->dim, k, (int)h->tb_ppt, var, 1) > 0) ppt = (int)h->tb_ppt;
+  if (var_req > 0 && jbk::tblock_ncw(h->dim, k, ppt, (int)var_req, 1) > 0) var = (int)var_req;
+  if (h->tb_ppt > 0 && var_req > 0 && jbk::tblock_ncw(h->dim, k, (int)h->tb_ppt, (int)var_req, 1) > 0) {
+    ppt = (int)h->tb_ppt;
+    var = (int)var_req;
+  }
+  if (jbk::tblock_ncw(h->dim, k, ppt, var, 1) == 0) {
+    ppt = dflt_ppt(k);
+    var = dflt_var(k);
+  }
   if (!fits(k)) k = 0;
   *k_out = k;
   *ppt_out = ppt;
-  *lag_out = lag;
+  *var_out = var;
 }
 
 int run_tblock(jacobi_ctx *h, int64_t iters, int K, int ppt, int lag) {
@@ -595,7 +605,18 @@ int run_tblock(jacobi_ctx *h, int64_t iters, int K, int ppt, int lag) {
     h->schedule = sched;
     if (rc) return rc;
     JbGeom &g = L.P.g;
-    if (h->dim == 3) {  // tiles of TY rows; stages hold rows y0-2 .. y0+TY+1
+    if (h->dim == 3 && K > 2) {  // odd K: NCW warps x RPW rows x 64 ppt columns, outputs shrink by 2(K-1)
+      const int ncw = jbk::tblock_ncw(3, K, ppt, lag, 1), ty_all = ncw * lag;
+      g.tx = 64 * ppt - 2 * (K - 1);
+      g.ty = ty_all - 2 * (K - 1);
+      g.rh = ty_all + 2;
+      g.ws = 64 * ppt + 4;
+      g.units_x = (int)((h->nx - 2 + g.tx - 1) / g.tx);
+      g.units_y = (int)((h->ny - 2 + g.ty - 1) / g.ty);
+      g.units = g.units_x * g.units_y;
+      g.stage_doubles = g.rh * g.ws;
+      g.xch_doubles = (K - 1) * 2 * ncw * 2 * 64 * ppt;
+    } else if (h->dim == 3) {  // tiles of TY rows; stages hold rows y0-2 .. y0+TY+1
       g.ty = jbk::tblock_ty();
       g.rh = g.ty + 4;
       g.units_y = (int)((h->ny - 2 + g.ty - 1) / g.ty);
@@ -859,6 +880,7 @@ static int64_t *param_slot(jacobi_t h, const char *name) {
   if (!std::strcmp(name, "tb_k")) return &h->tb_k;
   if (!std::strcmp(name, "tb_ppt")) return &h->tb_ppt;
   if (!std::strcmp(name, "tb_lag")) return &h->tb_lag;
+  if (!std::strcmp(name, "tb_rpw")) return &h->tb_rpw;
   if (!std::strcmp(name, "last_tb_k")) return &h->last_tb_k;
   if (!std::strcmp(name, "last_tblock")) return &h->last_tblock;
   return nullptr;

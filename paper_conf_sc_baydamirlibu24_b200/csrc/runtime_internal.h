@@ -172,6 +172,7 @@ struct jacobi_ctx {
   int64_t tb_k = -1;           // iterations per time block: -1 auto (2D: JB_TB_K2D, 3D: 2), 2D: 2, 3, 5
   int64_t tb_ppt = -1;         // 2D cell pairs per thread and level: -1 auto (4 for K <= 3, 2 for K = 5)
   int64_t tb_lag = -1;         // 2D odd K: wavefront lag between levels (1 or 2; -1 auto)
+  int64_t tb_rpw = -1;         // 3D odd K: rows per warp of the tile (-1 auto)
   int64_t last_tb_k = 0;       // read-only: K of the last time-blocked run
   int64_t last_tblock = 0;     // read-only: iterations of the last CPU-Free run done time-blocked
   int64_t norm_every = 0;      // N4: check the update norm every k iterations (0 = off)

@@ -573,6 +573,229 @@ __device__ __forceinline__ void tb3_item(const JbGeom &g, const Ring &R, RingPos
   else tb3_march<TY, false>(L, g, R, q0, a, b, C, r0, r1, dst, lane);
 }
 
+// ---------------------------------------------------------------- 3D, deeper time blocks (K odd)
+// Tile = TY = NCW·RPW rows x TX = 64·PPT columns, computed at every level and marched along z.
+// Warp w owns the tile rows w·RPW .. w·RPW+RPW-1, lane l the contiguous pairs kk = l·PPT + i.
+// Neighbours of a level-(k-1) cell: x — own registers / one shuffle per side (as 2D); y — own
+// registers, except above the warp's first and below its last row: the neighbouring warps'
+// boundary rows, exchanged through shared memory (double-buffered by step parity, so ONE
+// consumer barrier per step orders them); z — the level's previous / next plane, in registers
+// (z wavefront with LAG = 1, three planes per level).  Every level loses one valid column and
+// row per side at the tile's edges (the tile's outermost warps / lanes have no neighbour data),
+// so level K is valid on the middle WO = TX - 2(K-1) columns and HO = TY - 2(K-1) rows: the
+// tile's outputs (g.tx = WO, g.ty = HO).  Level 1 reads the level-0 stage, which holds the
+// tile's rows plus one on each side, so it is valid everywhere.  K odd keeps 16-byte alignment.
+struct Tb3kLane {
+  int j0;                // stage column index of pair 0 of this lane (stage col 0 <-> s - 2)
+  unsigned ok, full, st; // per pair: x / x+1 interior, stored at level K
+  unsigned rok, rst;     // per row of the warp: interior row, stored at level K
+};
+
+template <int NCW>
+__device__ __forceinline__ void bar_consumers() {
+  asm volatile("bar.sync 1, %0;" ::"r"(NCW * 32) : "memory");
+}
+
+// Level 1 of the warp's RPW rows of the plane whose level-0 stages are zm (z-1), zc, zp (z+1).
+template <int PPT, int RPW, bool FAST, bool STEADY>
+__device__ __forceinline__ void tb3k_level1(const Tb3kLane &L, int sr0, int ws, const double *zm, const double *zc,
+                                            const double *zp, bool planein, double2 (*V)[PPT]) {
+  double2 Cr[RPW + 2][PPT];  // rows sr0-1 .. sr0+RPW of the centre plane
+#pragma unroll
+  for (int j = 0; j < RPW + 2; ++j)
+#pragma unroll
+    for (int i = 0; i < PPT; ++i) Cr[j][i] = lds2(zc + (sr0 - 1 + j) * ws + L.j0 + 2 * i);
+#pragma unroll
+  for (int j = 0; j < RPW; ++j) {
+    const int o = (sr0 + j) * ws + L.j0;
+    const double Wl = zc[o - 1], Er = zc[o + 2 * PPT];
+#pragma unroll
+    for (int i = 0; i < PPT; ++i) {
+      const double2 Up = lds2(zp + o + 2 * i), Dn = lds2(zm + o + 2 * i);
+      const double2 C = Cr[j + 1][i], N = Cr[j + 2][i], S = Cr[j][i];
+      const double W = i == 0 ? Wl : Cr[j + 1][i - 1].y;
+      const double E = i == PPT - 1 ? Er : Cr[j + 1][i + 1].x;
+      // oracle order: x+1, x-1, y+1, y-1, z+1, z-1, then * fl(1/6)
+      const double l0 = kC6 * (((((C.y + W) + N.x) + S.x) + Up.x) + Dn.x);
+      const double l1 = kC6 * (((((E + C.x) + N.y) + S.y) + Up.y) + Dn.y);
+      if (FAST && STEADY) {
+        V[j][i] = make_double2(l0, l1);
+      } else {
+        const bool r = (STEADY || planein) && (FAST || (L.rok >> j & 1u));
+        V[j][i].x = (r && (FAST || (L.ok >> i & 1u))) ? l0 : C.x;
+        V[j][i].y = (r && (FAST || (L.full >> i & 1u))) ? l1 : C.y;
+      }
+    }
+  }
+}
+
+// Level k >= 2 of the warp's rows of the centre plane Zc (level k-1 planes Zm, Zc, Zp); yT / yB:
+// the level-(k-1) rows just above / below the warp (other warps' boundary rows).  STORE: level
+// K, pair i of row j stored at o + j·pitch + 2i.
+template <int PPT, int RPW, bool FAST, bool STEADY, bool STORE>
+__device__ __forceinline__ void tb3k_levelk(const Tb3kLane &L, const double2 (*Zm)[PPT], const double2 (*Zc)[PPT],
+                                            const double2 (*Zp)[PPT], const double2 *yT, const double2 *yB,
+                                            bool planein, int lane, double2 (*V)[PPT], double *o, int64_t pitch) {
+#pragma unroll
+  for (int j = 0; j < RPW; ++j) {
+    const double Wl = shfl_d(Zc[j][PPT - 1].y, (lane + 31) & 31);
+    const double Er = shfl_d(Zc[j][0].x, (lane + 1) & 31);
+#pragma unroll
+    for (int i = 0; i < PPT; ++i) {
+      const double2 C = Zc[j][i];
+      const double2 N = j + 1 < RPW ? Zc[j + 1 < RPW ? j + 1 : j][i] : yB[i];
+      const double2 S = j > 0 ? Zc[j > 0 ? j - 1 : j][i] : yT[i];
+      const double W = i == 0 ? Wl : Zc[j][i > 0 ? i - 1 : 0].y;
+      const double E = i == PPT - 1 ? Er : Zc[j][i + 1 < PPT ? i + 1 : i].x;
+      const double2 Up = Zp[j][i], Dn = Zm[j][i];
+      const double o0 = kC6 * (((((C.y + W) + N.x) + S.x) + Up.x) + Dn.x);
+      const double o1 = kC6 * (((((E + C.x) + N.y) + S.y) + Up.y) + Dn.y);
+      if (STORE) {
+        if ((L.rst >> j & 1u) && (L.st >> i & 1u)) {
+          double *po = o + j * pitch + 2 * i;
+          if (FAST) *reinterpret_cast<double2 *>(po) = make_double2(o0, o1);
+          else store_pair(po, o0, o1, L.full >> i & 1u);
+        }
+      } else if (FAST && STEADY) {
+        V[j][i] = make_double2(o0, o1);
+      } else {
+        const bool r = (STEADY || planein) && (FAST || (L.rok >> j & 1u));
+        V[j][i].x = (r && (FAST || (L.ok >> i & 1u))) ? o0 : C.x;
+        V[j][i].y = (r && (FAST || (L.full >> i & 1u))) ? o1 : C.y;
+      }
+    }
+  }
+}
+
+template <int K, int PPT, int RPW, int NCW, bool FAST>
+__device__ __forceinline__ void tb3k_march(const Tb3kLane &L, const JbGeom &g, const Ring &R, RingPos q, int a,
+                                           int b, int C, int r0, int r1, double *dst, double *xch, int warp,
+                                           int lane) {
+  constexpr int NS = 3;
+  constexpr int TX = 64 * PPT;
+  double2 X[K - 1][NS][RPW][PPT];  // X[k-1][m % 3]: level k of the plane computed at step m
+  const int Rs = a - K >= 0 ? r0 + 2 : r0 + 1;
+  const int Re = b + K;
+  const int Ws = a + K, We = min(b + K, C + 1);
+  const int ws = g.ws, sr0 = warp * RPW + 1;
+  const int64_t pe = g.plane_elems, pitch = g.pitch;
+  double *o = dst + (int64_t)(Rs - K) * pe;
+  // exchange slots: [level k-1][parity][warp][0 = first row, 1 = last row][TX]
+  auto xrow = [&](int k1, int par, int w, int side) { return xch + ((((k1 * 2 + par) * NCW + w) * 2 + side) * TX); };
+  const int wu = warp > 0 ? warp - 1 : warp, wd = warp + 1 < NCW ? warp + 1 : warp;  // edge warps: any row
+  RingPos pm = q, pc = Rs == r0 + 2 ? ring_add(q, 1u, R.S) : q, pn = pc;
+  if (Rs <= r1) pn = ring_add(q, (uint32_t)(Rs - r0), R.S);
+  R.wait_full(pm);
+  R.wait_full(pc);
+  auto publish = [&](int k1, int par, const double2 (*V)[PPT]) {
+#pragma unroll
+    for (int i = 0; i < PPT; ++i) {
+      *reinterpret_cast<double2 *>(xrow(k1, par, warp, 0) + 2 * (lane * PPT + i)) = V[0][i];
+      *reinterpret_cast<double2 *>(xrow(k1, par, warp, 1) + 2 * (lane * PPT + i)) = V[RPW - 1][i];
+    }
+  };
+  auto step = [&](auto u_ct, auto steady_ct, int Rr) {
+    constexpr int U = decltype(u_ct)::value;
+    constexpr bool ST = decltype(steady_ct)::value;
+    constexpr int SN = U, SC = (U + NS - 1) % NS, SS = (U + NS - 2) % NS;
+    const int par = Rr & 1, prv = par ^ 1;
+    auto need = [&](int k, int r) { return r >= max(a - (K - k), 0) && r <= min(b + (K - k), C + 1); };
+    if (ST || Rr <= r1) R.wait_full(pn);
+    bar_consumers<NCW>();  // the previous step's exchange rows are visible; its reads are done
+    if (ST || need(1, Rr - 1)) {
+      tb3k_level1<PPT, RPW, FAST, ST>(L, sr0, ws, R.stage(pm), R.stage(pc), R.stage(pn), Rr - 1 >= 1 && Rr - 1 <= C,
+                                      X[0][U]);
+      publish(0, par, X[0][U]);
+    }
+    if (ST || (Rr - 2 >= r0 && Rr - 2 <= r1)) R.release(pm, lane);
+#pragma unroll
+    for (int k = 2; k <= K; ++k) {
+      const int r = Rr - k;
+      if (!(ST || need(k, r))) continue;
+      double2 yT[PPT], yB[PPT];
+#pragma unroll
+      for (int i = 0; i < PPT; ++i) {
+        yT[i] = lds2(xrow(k - 2, prv, wu, 1) + 2 * (lane * PPT + i));
+        yB[i] = lds2(xrow(k - 2, prv, wd, 0) + 2 * (lane * PPT + i));
+      }
+      if (k < K) {
+        tb3k_levelk<PPT, RPW, FAST, ST, false>(L, X[k - 2][SS], X[k - 2][SC], X[k - 2][SN], yT, yB,
+                                               r >= 1 && r <= C, lane, X[k - 1][U], nullptr, pitch);
+        publish(k - 1, par, X[k - 1][U]);
+      } else {
+        tb3k_levelk<PPT, RPW, FAST, ST, true>(L, X[k - 2][SS], X[k - 2][SC], X[k - 2][SN], yT, yB, true, lane,
+                                              nullptr, o, pitch);
+      }
+    }
+    o += pe;
+    pm = pc;
+    pc = pn;
+    if (Rr + 1 <= r1) {
+      const uint32_t sl = pn.slot + 1u;
+      const bool wrap = sl == R.S;
+      pn.slot = wrap ? 0u : sl;
+      pn.phase ^= wrap ? 1u : 0u;
+    }
+  };
+  using TT = std::integral_constant<bool, true>;
+  using TF = std::integral_constant<bool, false>;
+  auto group = [&](auto steady_ct, int Rr) {
+    constexpr bool ST = decltype(steady_ct)::value;
+    step(std::integral_constant<int, 0>{}, steady_ct, Rr);
+    if (ST || Rr + 1 <= Re) step(std::integral_constant<int, 1>{}, steady_ct, Rr + 1);
+    if (ST || Rr + 2 <= Re) step(std::integral_constant<int, 2>{}, steady_ct, Rr + 2);
+  };
+  int Rr = Rs;
+  if (Ws <= We) {
+    for (; Rr < Ws; Rr += NS) group(TF{}, Rr);
+    if (Rr + NS - 1 <= We) {
+      const int Rend = Rr + ((We - Rr + 1) / NS) * NS;
+      for (; Rr < Rend; Rr += NS) group(TT{}, Rr);
+    }
+  }
+  for (; Rr <= Re; Rr += NS) group(TF{}, Rr);
+  if (Re - 1 <= r1) R.release(pm, lane);
+  if (Re <= r1) R.release(pc, lane);
+}
+
+template <int K, int PPT, int RPW, int NCW>
+__device__ __forceinline__ void tb3k_item(const JbGeom &g, const Ring &R, RingPos &q, int unit, int64_t a, int64_t b,
+                                          int64_t C, double *out, double *xch, int warp, int lane) {
+  constexpr int TY = NCW * RPW;
+  const int ux = unit % g.units_x, uy = unit / g.units_x;
+  const int64_t x0 = 1 + (int64_t)ux * g.tx, y0 = 1 + (int64_t)uy * g.ty;
+  const int64_t sx = x0 - (K - 1), sy = y0 - (K - 1);  // first computed column / row of the tile
+  const int64_t r0 = max(a - K, (int64_t)0), r1 = min(b + K, C + 1);
+  const RingPos q0 = q;
+  q = ring_add(q, (uint32_t)(r1 - r0 + 1), R.S);
+  Tb3kLane L;
+  L.j0 = 2 + 2 * PPT * lane;
+  L.ok = L.full = L.st = L.rok = L.rst = 0;
+#pragma unroll
+  for (int i = 0; i < PPT; ++i) {
+    const int kk = PPT * lane + i;
+    const int64_t c = sx + 2 * kk;
+    const bool ok = c >= 1 && c <= g.nx - 2;
+    L.ok |= (ok ? 1u : 0u) << i;
+    L.full |= (ok && c + 1 <= g.nx - 2 ? 1u : 0u) << i;
+    L.st |= (ok && kk >= (K - 1) / 2 && kk < 32 * PPT - (K - 1) / 2 ? 1u : 0u) << i;
+  }
+#pragma unroll
+  for (int j = 0; j < RPW; ++j) {
+    const int t = warp * RPW + j;  // tile row
+    const int64_t y = sy + t;
+    const bool rok = y >= 1 && y <= g.ny - 2;
+    L.rok |= (rok ? 1u : 0u) << j;
+    L.rst |= (rok && t >= K - 1 && t <= TY - K ? 1u : 0u) << j;
+  }
+  const bool fast = sx >= 1 && sx + 64 * PPT - 1 <= g.nx - 2 && sy >= 1 && sy + TY - 1 <= g.ny - 2;
+  double *dst = out + (sy + (int64_t)warp * RPW) * g.pitch + 3 + sx + 2 * PPT * lane;
+  if (fast)
+    tb3k_march<K, PPT, RPW, NCW, true>(L, g, R, q0, (int)a, (int)b, (int)C, (int)r0, (int)r1, dst, xch, warp, lane);
+  else
+    tb3k_march<K, PPT, RPW, NCW, false>(L, g, R, q0, (int)a, (int)b, (int)C, (int)r0, (int)r1, dst, xch, warp, lane);
+}
+
 // Edge zone of a slab side with a neighbour (time block t -> t+K), computed by that side's
 // boundary CTAs with the whole CTA, so the halo exchange stays per iteration.
 // Phase m = 1..K: wait until the neighbour delivered its level m-1 plane (m = 1: the time-t halo
@@ -677,9 +900,9 @@ __device__ bool tb_edge(const JbGeom &g, const JbSlab &SL, const JbParams &P, in
   return true;
 }
 
-template <int NCW, int DIM, int K, int TP, int LAG>
+template <int NCW, int DIM, int K, int TP, int LAG, int RPW>
 __device__ __forceinline__ void tb_body(const JbParams &P) {
-  static_assert(K == 2 || (DIM == 2 && (K & 1)), "3D: K = 2; 2D: K = 2 or odd");
+  static_assert(K == 2 || (K & 1), "K = 2 or odd");
   extern __shared__ __align__(128) unsigned char smem[];
   __shared__ int s_abort;
   __shared__ int s_edge;  // the edge zones' wait result (own variable: s_abort is read after the barrier)
@@ -769,25 +992,29 @@ __device__ __forceinline__ void tb_body(const JbParams &P) {
         // per row and lane; 2D with K odd: columns x0-K-1 .. x0+tx+K (stage index 0 <-> x0-K-1;
         // columns left of the row's padding are not loaded: they only feed Dirichlet cells)
         const int ux = unit % g.units_x, uy = unit / g.units_x;
-        const int64_t xs_w = (DIM == 2 && K > 2) ? 3 - K + (int64_t)ux * g.tx : 2 + (int64_t)ux * g.tx;
+        const int64_t xs_w = K > 2 ? 3 - K + (int64_t)ux * g.tx : 2 + (int64_t)ux * g.tx;
         const int64_t xs = max(xs_w, (int64_t)0);
-        const int64_t xe = min(xs_w + ((DIM == 2 && K > 2) ? g.tx + 2 * K + 2 : g.tx + 4), g.pitch);
+        const int64_t xe = min(xs_w + (K > 2 ? g.tx + 2 * K + 2 : g.tx + 4), g.pitch);
         const uint32_t bytes = (uint32_t)((xe - xs) * 8);
         const int64_t dso = xs - xs_w;  // stage offset of the first loaded column
-        const int64_t ya = DIM == 3 ? (int64_t)uy * g.ty - 1 : 0;  // = y0 - 2
+        // 3D: stage row i <-> y0-2+i (K = 2) or y0-K+i (odd K: the tile's rows y0-(K-1) ..
+        // y0-(K-1)+TY-1 plus one on each side); lane i copies rows i, i+32, ...
+        const int64_t ya = DIM == 3 ? (K > 2 ? (int64_t)uy * g.ty + 1 - K : (int64_t)uy * g.ty - 1) : 0;
         const int nrow = DIM == 3 ? g.rh : 1;
         const int64_t yl = max(ya, (int64_t)0), yh = DIM == 3 ? min(ya + nrow - 1, g.ny - 1) : 0;
         const uint32_t nvalid = (uint32_t)(yh - yl + 1);
-        const int64_t yrow = ya + lane;
-        const bool mine = lane < nrow && (DIM == 2 || (yrow >= 0 && yrow <= g.ny - 1));
-        const double *src = cur + xs + (DIM == 3 ? yrow * g.pitch : 0);
         for (int64_t p = r0; p <= r1; ++p) {
           if (lane == 0) {
             mbar_wait(&R.empty[q.slot], q.phase ^ 1u);
             mbar_expect_tx(&R.full[q.slot], bytes * nvalid);
           }
           __syncwarp();
-          if (mine) bulk_g2s(R.stage(q) + (size_t)lane * g.ws + dso, src + p * g.plane_elems, bytes, &R.full[q.slot]);
+          for (int rr = lane; rr < nrow; rr += 32) {
+            const int64_t yrow = ya + rr;
+            if (DIM == 2 || (yrow >= 0 && yrow <= g.ny - 1))
+              bulk_g2s(R.stage(q) + (size_t)rr * g.ws + dso, cur + xs + (DIM == 3 ? yrow * g.pitch : 0) + p * g.plane_elems,
+                       bytes, &R.full[q.slot]);
+          }
           q.advance(R.S);
         }
         rq.advance(JB_RQ);
@@ -808,7 +1035,10 @@ __device__ __forceinline__ void tb_body(const JbParams &P) {
         if (lane == 0) mbar_arrive(&qempty[rq.slot]);
         rq.advance(JB_RQ);
         if (d.kind == TB_END) break;
-        if constexpr (DIM == 3) tb3_item<TP>(g, R, q, d.unit, d.a, d.b, C, nxt, warp, lane);
+        if constexpr (DIM == 3 && K > 2)
+          tb3k_item<K, TP, RPW, NCW>(g, R, q, d.unit, d.a, d.b, C, nxt, R.stages + (size_t)R.S * R.stage_doubles, warp,
+                                     lane);
+        else if constexpr (DIM == 3) tb3_item<TP>(g, R, q, d.unit, d.a, d.b, C, nxt, warp, lane);
         else if constexpr (K == 2) tb2_item<TP>(g, R, q, d.unit, d.a, d.b, C, nxt, warp, lane);
         else tbk_item<K, TP, LAG>(g, R, q, d.unit, d.a, d.b, C, nxt, warp, lane);
       }
@@ -834,13 +1064,13 @@ __device__ __forceinline__ void tb_body(const JbParams &P) {
 // One CTA per SM (up to 224 registers per thread) or two (96: 2 x 9 warps fit the register file
 // only at <= 96 registers, given the 4-warp allocation granularity).  K = iterations per time
 // block; TP = pairs per thread along x (2D) or rows per tile (3D).
-template <int DIM, int K, int TP, int NCW = JB_NCW, int LAG = 1>
+template <int DIM, int K, int TP, int NCW = JB_NCW, int LAG = 1, int RPW = 1>
 __global__ void __launch_bounds__((NCW + 1) * 32, 1) jb_tblock(const __grid_constant__ JbParams P) {
-  tb_body<NCW, DIM, K, TP, LAG>(P);
+  tb_body<NCW, DIM, K, TP, LAG, RPW>(P);
 }
 template <int TP>
 __global__ void __maxnreg__(96) jb_tblock2d_x2(const __grid_constant__ JbParams P) {
-  tb_body<JB_NCW, 2, 2, TP, 1>(P);
+  tb_body<JB_NCW, 2, 2, TP, 1, 1>(P);
 }
 
 constexpr int TB_TY = 4;  // 3D tile rows (level-1 rows TY+2 carried per plane in registers)
@@ -851,7 +1081,15 @@ constexpr int TB_TY = 4;  // 3D tile rows (level-1 rows TY+2 carried per plane i
 const void *tblock_fn(int dim, int k, int ppt, int lag, int per_sm, int *ncw) {
 #define JB_TB(...) reinterpret_cast<const void *>(&__VA_ARGS__)
   *ncw = JB_NCW;
-  if (dim == 3) return k == 2 ? JB_TB(jb_tblock<3, 2, TB_TY>) : nullptr;
+  if (dim == 3) {
+    if (k == 2) return JB_TB(jb_tblock<3, 2, TB_TY>);
+    // odd K: (K, PPT, RPW) -> NCW consumer warps x RPW rows per tile
+    if (k == 3 && ppt == 1 && lag == 4) return JB_TB(jb_tblock<3, 3, 1, 8, 1, 4>);
+    *ncw = 7;
+    if (k == 3 && ppt == 1 && lag == 5) return JB_TB(jb_tblock<3, 3, 1, 7, 1, 5>);
+    if (k == 3 && ppt == 2 && lag == 2) return JB_TB(jb_tblock<3, 3, 2, 7, 1, 2>);
+    return nullptr;
+  }
   if (k == 2) {
     if (per_sm >= 2) return ppt >= 4 ? JB_TB(jb_tblock2d_x2<4>) : ppt == 2 ? JB_TB(jb_tblock2d_x2<2>) : JB_TB(jb_tblock2d_x2<1>);
     return ppt >= 4 ? JB_TB(jb_tblock<2, 2, 4>) : ppt == 2 ? JB_TB(jb_tblock<2, 2, 2>) : JB_TB(jb_tblock<2, 2, 1>);
@@ -882,10 +1120,11 @@ int tblock_ncw(int dim, int k, int ppt, int lag, int per_sm) {
   return tblock_fn(dim, k, ppt, lag, per_sm, &ncw) ? ncw : 0;
 }
 
-// Dynamic shared memory of the temporally blocked kernel: header + ring stages.
+// Dynamic shared memory of the temporally blocked kernel: header + ring stages (+ the 3D
+// odd-K row exchange).
 size_t tblock_smem(const JbGeom &g) {
   const size_t hdr = (size_t)2 * g.stages * 8 + (size_t)2 * JB_RQ * 8 + (size_t)JB_RQ * sizeof(TbDesc);
-  return (hdr + 127) / 128 * 128 + (size_t)g.stages * g.stage_doubles * 8;
+  return (hdr + 127) / 128 * 128 + (size_t)g.stages * g.stage_doubles * 8 + (size_t)g.xch_doubles * 8;
 }
 
 cudaError_t prepare_tblock(const JbGeom &g, int k, int ppt, int lag, int per_sm, size_t smem, int *blocks_per_sm) {
