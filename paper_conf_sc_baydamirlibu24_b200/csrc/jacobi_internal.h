@@ -20,8 +20,8 @@
 #define JB_TB_PPT5 2            // default cell pairs per lane at K = 5
 #define JB_TB_LAG 1             // default wavefront lag of the odd-K march
 #define JB_TB_KMAX3 3           // deepest time block of the 3D time-blocked kernel
-#define JB_TB_K3D 2             // its default depth (auto)
-#define JB_TB_RPW3 4            // 3D odd K: default rows per warp
+#define JB_TB_K3D 3             // its default depth (auto; slabs without neighbours only)
+#define JB_TB_RPW3 2            // 3D odd K: default rows per warp (x 11 warps)
 
 // Scratch planes after each slab buffer for the time-blocked kernel's edge zones of depth K
 // (tblock.cu): K-1 slots for the neighbour's intermediate levels + the side's own level-m planes,
@@ -111,6 +111,7 @@ struct JbSlab {
   int64_t tb_lo, tb_hi;
   double *mid_top_out;
   double *mid_bot_out;
+  const void *tmap;                  // 3D odd-K time-blocked kernel: CUtensorMap[2] (buf[0], buf[1]) or null
 };
 
 struct JbParams {

@@ -79,6 +79,7 @@ void free_slab(Slab &s, const Allocator &a) {
   if (s.blk_flags) cudaFree(s.blk_flags);
   if (s.partials) cudaFree(s.partials);
   if (s.norm_peers) cudaFree(s.norm_peers);
+  if (s.tmap) cudaFree(s.tmap);
   if (s.ev0) cudaEventDestroy(s.ev0);
   if (s.ev1) cudaEventDestroy(s.ev1);
   if (s.ev_sync) cudaEventDestroy(s.ev_sync);
@@ -112,6 +113,44 @@ void link_local(jacobi_ctx *h) {
     }
   }
   h->peers_ready = true;
+}
+
+// Tensor maps (TMA descriptors) of a slab's two buffers, viewed as [planes][ny][pitch] fp64, box
+// = one plane's `rows` x `cols` window; out-of-bounds elements are zero-filled (they only feed
+// Dirichlet / discarded cells).  Encoded with the driver's cuTensorMapEncodeTiled (entry point
+// via the runtime, no -lcuda) and kept in device memory for the kernel.
+int slab_tensor_maps(jacobi_ctx *h, Slab &s, int cols, int rows) {
+  if (s.tmap && s.tmap_key[0] == cols && s.tmap_key[1] == rows) return JACOBI_OK;
+  using EncodeFn = CUresult (*)(CUtensorMap *, CUtensorMapDataType, cuuint32_t, void *, const cuuint64_t *,
+                                const cuuint64_t *, const cuuint32_t *, const cuuint32_t *, CUtensorMapInterleave,
+                                CUtensorMapSwizzle, CUtensorMapL2promotion, CUtensorMapFloatOOBfill);
+  static EncodeFn encode = nullptr;
+  if (!encode) {
+    void *fn = nullptr;
+    cudaDriverEntryPointQueryResult q;
+    CK(cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", &fn, cudaEnableDefault, &q));
+    if (!fn || q != cudaDriverEntryPointSuccess) return JACOBI_ECUDA;
+    encode = reinterpret_cast<EncodeFn>(fn);
+  }
+  const JbGeom &g = h->geom;
+  const int64_t planes = s.chunk + 2 + jb_edge_planes(h->dim);
+  CUtensorMap maps[2];
+  for (int b = 0; b < 2; ++b) {
+    const cuuint64_t dims[3] = {(cuuint64_t)g.pitch, (cuuint64_t)h->ny, (cuuint64_t)planes};
+    const cuuint64_t strides[2] = {(cuuint64_t)g.pitch * 8, (cuuint64_t)g.plane_elems * 8};
+    const cuuint32_t box[3] = {(cuuint32_t)cols, (cuuint32_t)rows, 1};
+    const cuuint32_t estr[3] = {1, 1, 1};
+    const CUresult r = encode(&maps[b], CU_TENSOR_MAP_DATA_TYPE_FLOAT64, 3, s.buf[b], dims, strides, box, estr,
+                              CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_NONE,
+                              CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+    if (r != CUDA_SUCCESS) return JACOBI_ECUDA;
+  }
+  CK(cudaSetDevice(s.device));
+  if (!s.tmap) CK(cudaMalloc(&s.tmap, sizeof(maps)));
+  CK(cudaMemcpy(s.tmap, maps, sizeof(maps), cudaMemcpyHostToDevice));
+  s.tmap_key[0] = cols;
+  s.tmap_key[1] = rows;
+  return JACOBI_OK;
 }
 
 // Device copy of the guided-schedule block table of a slab (rebuilt when its key changes).
@@ -614,7 +653,7 @@ int run_tblock(jacobi_ctx *h, int64_t iters, int K, int ppt, int lag) {
       g.units_x = (int)((h->nx - 2 + g.tx - 1) / g.tx);
       g.units_y = (int)((h->ny - 2 + g.ty - 1) / g.ty);
       g.units = g.units_x * g.units_y;
-      g.stage_doubles = g.rh * g.ws;
+      g.stage_doubles = (g.rh * g.ws + 15) / 16 * 16;  // TMA box destinations: 128-byte aligned
       g.xch_doubles = (K - 1) * 2 * ncw * 2 * 64 * ppt;
     } else if (h->dim == 3) {  // tiles of TY rows; stages hold rows y0-2 .. y0+TY+1
       g.ty = jbk::tblock_ty();
@@ -641,6 +680,12 @@ int run_tblock(jacobi_ctx *h, int64_t iters, int K, int ppt, int lag) {
       d.tb_hi = s.has_bot ? s.chunk - K : s.chunk;
       d.mid_top_out = s.mid_top_out;
       d.mid_bot_out = s.mid_bot_out;
+      d.tmap = nullptr;
+      if (h->dim == 3 && K > 2) {  // one TMA box copy per plane: the tile's rh rows x ws columns
+        rc = slab_tensor_maps(h, s, g.ws, g.rh);
+        if (rc) return rc;
+        d.tmap = s.tmap;
+      }
       const int64_t npl = d.tb_hi - d.tb_lo + 1;
       const int ni = d.cta_count - d.n_top - d.n_bot;
       d.dyn_items = 0;
@@ -726,8 +771,9 @@ int run_cpufree(jacobi_ctx *h, int64_t iters) {
   tblock_choice(h, &K, &ppt, &lag);
   const bool eligible = h->tblock != 0 && !nocomp && h->norm_every <= 0 && h->kind != KIND_SHMEM && K >= 2;
   if (h->tblock == 1 && !eligible) return JACOBI_EINVAL;
-  // auto picks it where it measured faster than the per-iteration kernel: 2D (3D: forced only)
-  const bool use = eligible && (h->tblock == 1 || h->dim == 2);
+  // auto picks it where it measured faster than the per-iteration kernel: 2D, and 3D slabs
+  // without neighbours (3D edge zones are whole planes: slower than per-iteration at P > 1)
+  const bool use = eligible && (h->tblock == 1 || h->dim == 2 || h->total == 1);
   int64_t tb_iters = 0;
   if (use) {
     // odd K: any block count; K = 2: an even one (the result stays in buf[t & 1], R10)

@@ -2,6 +2,7 @@
 // CPU-Free run and the C ABI), baselines.cu (CPU-controlled comparison modes) and multiproc.cu
 // (CUDA IPC, NCCL, NVSHMEM, device-memory allocators).  Product code only.
 #pragma once
+#include <cuda.h>
 #include <cuda_runtime.h>
 #include <dlfcn.h>
 #include <nccl.h>
@@ -146,6 +147,8 @@ struct Slab {
   int64_t partials_cap = 0;
   JbCtrl **norm_peers = nullptr;            // N4: device array of every slab's control block
   int64_t dyn_key[4] = {0, 0, 0, 0};
+  void *tmap = nullptr;       // time-blocked 3D kernel: two CUtensorMaps (buf[0], buf[1]) in device memory
+  int tmap_key[2] = {0, 0};   // their box (columns, rows)
   int grid = 0;
   size_t smem = 0;
 };
@@ -237,6 +240,8 @@ int setup_norm(jacobi_ctx *h, LaunchPlan &L);
 int run_cpufree(jacobi_ctx *h, int64_t iters);
 int run_cpufree_k1(jacobi_ctx *h, int64_t iters);
 int run_tblock(jacobi_ctx *h, int64_t iters, int k, int ppt, int lag);
+// Tensor maps of a slab's two buffers for TMA box loads of `cols` x `rows` elements (one plane).
+int slab_tensor_maps(jacobi_ctx *h, Slab &s, int cols, int rows);
 // Time-block depth and pairs per thread the runtime would use for this handle (K = 0: none).
 void tblock_choice(const jacobi_ctx *h, int *k, int *ppt, int *lag);
 int ensure_nccl(jacobi_ctx *h);

@@ -32,6 +32,15 @@ struct TbDesc {
   int64_t pad;
 };
 
+// TMA box copy (tensor map in global memory) of one plane window into shared memory.
+__device__ __forceinline__ void tma_box3(void *dst, const void *tmap, int c0, int c1, int c2, uint64_t *bar) {
+  asm volatile(
+      "cp.async.bulk.tensor.3d.shared::cluster.global.tile.mbarrier::complete_tx::bytes [%0], [%1, {%2, %3, %4}], "
+      "[%5];" ::"r"(sptr(dst)),
+      "l"(tmap), "r"(c0), "r"(c1), "r"(c2), "r"(sptr(bar))
+      : "memory");
+}
+
 // Position `off` stages after p in the ring.
 __device__ __forceinline__ RingPos ring_add(RingPos p, uint32_t off, uint32_t S) {
   const uint32_t s = p.slot + off;
@@ -1003,6 +1012,23 @@ __device__ __forceinline__ void tb_body(const JbParams &P) {
         const int nrow = DIM == 3 ? g.rh : 1;
         const int64_t yl = max(ya, (int64_t)0), yh = DIM == 3 ? min(ya + nrow - 1, g.ny - 1) : 0;
         const uint32_t nvalid = (uint32_t)(yh - yl + 1);
+        if (DIM == 3 && K > 2 && SL.tmap) {  // one TMA box per plane (zero fill outside the grid)
+          const void *tm = static_cast<const char *>(SL.tmap) + 128 * ((P.t0 + j) & 1);
+          const uint32_t box = (uint32_t)(nrow * g.ws * 8);
+          for (int64_t p = r0; p <= r1; ++p) {
+            if (lane == 0) {
+              mbar_wait(&R.empty[q.slot], q.phase ^ 1u);
+              mbar_expect_tx(&R.full[q.slot], box);
+              tma_box3(R.stage(q), tm, (int)xs_w, (int)ya, (int)p, &R.full[q.slot]);
+            }
+            q.advance(R.S);
+          }
+          __syncwarp();
+          rq.advance(JB_RQ);
+          if (!early && lane == 0) claim = atomicAdd(ctr, 1u);
+          item = SL.dyn_first + (int64_t)__shfl_sync(0xffffffffu, claim, 0);
+          continue;
+        }
         for (int64_t p = r0; p <= r1; ++p) {
           if (lane == 0) {
             mbar_wait(&R.empty[q.slot], q.phase ^ 1u);
@@ -1083,11 +1109,13 @@ const void *tblock_fn(int dim, int k, int ppt, int lag, int per_sm, int *ncw) {
   *ncw = JB_NCW;
   if (dim == 3) {
     if (k == 2) return JB_TB(jb_tblock<3, 2, TB_TY>);
-    // odd K: (K, PPT, RPW) -> NCW consumer warps x RPW rows per tile
-    if (k == 3 && ppt == 1 && lag == 4) return JB_TB(jb_tblock<3, 3, 1, 8, 1, 4>);
+    // odd K: (K, PPT, RPW = `lag`) -> NCW consumer warps x RPW rows per tile
+    if (k != 3) return nullptr;
+    *ncw = 11;
+    if (ppt == 1 && lag == 2) return JB_TB(jb_tblock<3, 3, 1, 11, 1, 2>);
     *ncw = 7;
-    if (k == 3 && ppt == 1 && lag == 5) return JB_TB(jb_tblock<3, 3, 1, 7, 1, 5>);
-    if (k == 3 && ppt == 2 && lag == 2) return JB_TB(jb_tblock<3, 3, 2, 7, 1, 2>);
+    if (ppt == 1 && lag == 3) return JB_TB(jb_tblock<3, 3, 1, 7, 1, 3>);
+    if (ppt == 2 && lag == 2) return JB_TB(jb_tblock<3, 3, 2, 7, 1, 2>);
     return nullptr;
   }
   if (k == 2) {

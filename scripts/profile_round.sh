@@ -1,6 +1,7 @@
 #!/bin/bash
 # Run on the GPU box (gpurun): launch list of the bench command + ncu --set full of the CPU-Free
-# kernels (20-iteration launches) for C2 (time-blocked K=5 default, K=2), C2 per-iteration and C3, under gpurun_out/.
+# kernels (20/21-iteration launches) for C2 (time-blocked K=5 default, K=2), C2 per-iteration, C3 per-iteration and
+# C3 time-blocked (K=3), under gpurun_out/.
 set -x
 out=gpurun_out
 ncu --metrics gpu__time_duration.sum --clock-control none --csv --log-file $out/launches_c2.csv \
@@ -14,4 +15,5 @@ run_full() {  # name, kernel regex, bench args
 run_full c2_tblock jb_tblock --config c2
 run_full c2_tblock_k2 jb_tblock --config c2 --param tb_k=2
 run_full c2 jb_sweep --config c2 --param tblock=0
-run_full c3 jb_sweep --config c3
+run_full c3 jb_sweep --config c3 --param tblock=0
+run_full c3_tblock jb_tblock --config c3 --iters 21

@@ -22,12 +22,17 @@ for shape, P in [((20, 70), 2), ((8, 9, 33), 2), ((30, 40), 1)]:
             j.scatter(f)
             j.run(3)
             ok &= bool(np.array_equal(j.gather(), oracle.jacobi(f, 3)))
-# time-blocked kernel (2D and 3D, with and without neighbours): TMA ring, shuffles, edge zones
-for shape, P in [((20, 70), 2), ((12, 9, 33), 2), ((30, 40), 1)]:
+# time-blocked kernel (2D K = 5 / 3 / 2, 3D K = 3 / 2, with and without neighbours): TMA ring
+# and TMA boxes, shuffles, the 3D shared-memory row exchange, edge zones
+for shape, P, prm in [((24, 70), 2, {}), ((20, 70), 2, {"tb_k": 2}), ((12, 9, 33), 2, {}),
+                      ((12, 9, 33), 1, {}), ((12, 9, 33), 1, {"tb_k": 2}), ((30, 40), 1, {}),
+                      ((30, 40), 1, {"tb_k": 3})]:
     f = u12(shape, 4)
     with jb.Jacobi(shape, virtual=P) if P > 1 else jb.Jacobi(shape) as j:
         j.set_param("tblock", 1)
         j.set_param("resident", 0)
+        for k, v in prm.items():
+            j.set_param(k, v)
         j.scatter(f)
         j.run(8)
         ok &= bool(np.array_equal(j.gather(), oracle.jacobi(f, 8)))

@@ -18,6 +18,8 @@ pytestmark = pytest.mark.gpu
 # 2D variants (K, pairs per thread); the default (auto) is K = 5, ppt = 2
 KV = [(2, 4), (3, 2), (3, 4), (5, 2)]
 K_AUTO = 5
+K3_AUTO = 3  # 3D default (slabs without neighbours)
+KV3 = [(2, 4, -1), (3, 1, 2), (3, 1, 3), (3, 2, 2)]  # 3D (K, ppt, rows per warp)
 
 
 def step(k):
@@ -326,44 +328,69 @@ def test_c2_1000_iters_tblock_p8_equals_p1():
 @pytest.mark.parametrize("shape", [(3, 3, 3), (5, 6, 7), (10, 13, 70), (20, 37, 130), (9, 17, 600),
                                    (12, 23, 1100), (40, 9, 8), (7, 70, 40)])
 @pytest.mark.parametrize("iters", [4, 5, 13])
-def test_tblock_3d_shapes(shape, iters):
-    """3D tiles of 4 rows (ragged last tile in y and x, tiles narrower than a warp, nz from 3)."""
+@pytest.mark.parametrize("kv", KV3)
+def test_tblock_3d_shapes(shape, iters, kv):
+    """3D: K = 2 (tiles of 4 rows, extra cells) and K = 3 (tiles of NCW x RPW rows with the
+    shared-memory row exchange, TMA box loads): ragged last tile in y and x, tiles narrower than
+    a warp, nz from 3."""
     f = u12(shape, 11)
-    got, tb = run_tb(f, iters)
-    assert tb == iters // 4 * 4
-    assert_bitwise(got, oracle.jacobi(f, iters), f"3D tblock {shape} it{iters}")
+    params = {"tb_rpw": kv[2]} if kv[2] > 0 else {}
+    got, tb = run_tb(f, iters, params, kv=kv[:2])
+    assert tb == tb_iters(iters, kv[0])
+    assert_bitwise(got, oracle.jacobi(f, iters), f"3D tblock K={kv} {shape} it{iters}")
 
 
 @pytest.mark.parametrize("tile_x,min_block", [(8, 1), (16, 2), (64, 1), (128, 5)])
 def test_tblock_3d_tiles(tile_x, min_block):
     f = u12((21, 30, 150), 12)
-    got, _ = run_tb(f, 8, {"tile_x": tile_x, "tb_min_block": min_block})
+    got, _ = run_tb(f, 8, {"tile_x": tile_x, "tb_min_block": min_block}, kv=(2, 4))
     assert_bitwise(got, oracle.jacobi(f, 8), f"3D tx{tile_x}")
 
 
+@pytest.mark.parametrize("min_block", [1, 3, 16])
+@pytest.mark.parametrize("kv", KV3[1:])
+def test_tblock_3d_odd_k_blocks(kv, min_block):
+    """3D K = 3: single-plane and short plane blocks, tiles with rows / columns past the grid."""
+    for shape in [(40, 61, 130), (25, 100, 70)]:
+        f = u12(shape, 12)
+        got, _ = run_tb(f, 9, {"tb_min_block": min_block, "tb_rpw": kv[2]}, kv=kv[:2])
+        assert_bitwise(got, oracle.jacobi(f, 9), f"3D K={kv} {shape} mb{min_block}")
+
+
 @pytest.mark.parametrize("P", [2, 3, 4])
-def test_tblock_3d_virtual_slabs(P):
-    f = u12((4 * P + 5, 26, 70), 13)
-    got, tb = run_tb_virtual(f, 13, P)
-    assert tb == 12
-    assert_bitwise(got, oracle.jacobi(f, 13), f"3D P={P}")
+@pytest.mark.parametrize("kv", KV3[:2])
+def test_tblock_3d_virtual_slabs(P, kv):
+    """3D edge zones (K phases over whole planes) between P slabs."""
+    f = u12((6 * P + 5, 26, 70), 13)
+    params = {"tb_rpw": kv[2]} if kv[2] > 0 else {}
+    with jb.Jacobi(f.shape, virtual=P) as j:
+        for n, v in {"tblock": 1, "resident": 0, "tb_k": kv[0], "tb_ppt": kv[1], **params}.items():
+            j.set_param(n, v)
+        j.scatter(f)
+        j.run(13)
+        K = j.get_param("last_tb_k")
+        assert K == kv[0]
+        assert j.get_param("last_tblock") == tb_iters(13, K)
+        assert_bitwise(j.gather(), oracle.jacobi(f, 13), f"3D P={P} K={kv}")
 
 
 def test_tblock_3d_invariants_and_mixing():
     z, y, x = np.mgrid[0:12, 0:13, 0:30].astype(np.float64)
     for h in (1 + x + 2 * y - 3 * z, x * x + y * y - 2 * z * z, x * y + y * z + z * x):
-        got, _ = run_tb(np.ascontiguousarray(h), 16)
+        got, _ = run_tb(np.ascontiguousarray(h), 18)
         assert_bitwise(got, h, "3D harmonic field stationary")
     f = u12((30, 20, 100), 14)
     exp = oracle.jacobi(f, 23)
     got, _ = run_tb(f, 23, runs=[4, 3, 8, 1, 4, 3])
     assert_bitwise(got, exp, "3D split")
+    got, _ = run_tb(f, 23, runs=[4, 3, 8, 1, 4, 3], kv=(2, 4))
+    assert_bitwise(got, exp, "3D split K=2")
     with jb.Jacobi(f.shape, virtual=2) as j:
         j.set_param("resident", 0)
         j.set_param("tblock", 1)
         j.scatter(f)
         j.run(8)
-        assert j.get_param("last_tblock") == 8
+        assert j.get_param("last_tblock") == 6 and j.get_param("last_tb_k") == 3  # chunk 14
         j.set_mode(jb.MODE_BASELINE_MEMCPY)
         j.run(3)
         j.set_mode(jb.MODE_CPUFREE)
@@ -371,8 +398,14 @@ def test_tblock_3d_invariants_and_mixing():
         assert_bitwise(j.gather(), exp, "3D mixed P=2")
 
 
-def test_tblock_3d_auto_is_per_iteration():
+def test_tblock_3d_auto_selection():
+    """3D auto: time-blocked K = 3 for a slab without neighbours, per-iteration with neighbours
+    (whole-plane edge zones measured slower there)."""
     with jb.Jacobi((20, 30, 40)) as j:
+        j.set_param("resident", 0)
+        j.run(8)
+        assert j.get_param("last_tblock") == 6 and j.get_param("last_tb_k") == K3_AUTO
+    with jb.Jacobi((20, 30, 40), virtual=2) as j:
         j.set_param("resident", 0)
         j.run(8)
         assert j.get_param("last_tblock") == 0
@@ -386,9 +419,11 @@ def test_c3_1000_iters_tblock_equals_per_iteration():
         j.set_param("tblock", 0)
         j.run(1000)
         ref = j.gather()
-    for P in (0, 4):
+    for P, k in ((0, 3), (0, 2), (4, 3)):
         with (jb.Jacobi(shape, virtual=P) if P else jb.Jacobi(shape)) as j:
             j.set_param("tblock", 1)
+            j.set_param("tb_k", k)
             j.run(1000)
-            assert j.get_param("last_tblock") == 1000
-            assert_bitwise(j.gather(), ref, f"C3 tblock P={P or 1}")
+            assert j.get_param("last_tb_k") == k
+            assert j.get_param("last_tblock") == tb_iters(1000, k)
+            assert_bitwise(j.gather(), ref, f"C3 tblock P={P or 1} K={k}")
