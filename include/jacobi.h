@@ -164,7 +164,9 @@ int jacobi_set_mode(jacobi_t h, int mode, int flags);
  * 0 never, 1 always incl. 3D (EINVAL when a slab has < 4 planes with P > 1, with the norm, in
  * no-compute mode or in the NVSHMEM variant)), "tb_k" (iterations per time block: -1 auto = 5 in
  * 2D, 2 in 3D; 2D accepts 2, 3, 5 — a deeper K than the slabs fit falls back to 3, then 2),
- * "tb_ppt" (2D cell pairs per lane and level: K = 2: from tile_x; K = 3: 2 or 4; K = 5: 2),
+ * "tb_ppt" (2D cell pairs per lane and level: K = 2: from tile_x; K = 3: 2 or 4; K = 5: 1 (default,
+ * 11 consumer warps) or 2 (7 warps); 3D K = 3: 1 (default) or 2), "tb_rpw" (3D K = 3: rows per
+ * warp, 2 (default, 11 warps) or 3 (7 warps)),
  * "tb_lag" (odd K: wavefront skew between levels, 1 default or 2), "tb_min_block" (smallest
  * dynamic plane block of that kernel, default 16), "tb_ctas" (its CTAs per SM, 1 or 2; 2 only
  * for K = 2 and P = 1).  Read-only: "last_resident" (1 if the last CPU-Free run used the resident

@@ -206,11 +206,12 @@ struct Ring {
     return stages + (size_t)p.slot * stage_doubles;
   }
   __device__ __forceinline__ void wait_full(const RingPos &p) const { mbar_wait(&full[p.slot], p.phase); }
-  // Consumer warp releases a stage: all lanes are done reading it (syncwarp), one lane arrives.
-  __device__ __forceinline__ void release(const RingPos &p, int lane) const {
-    __syncwarp();
-    if (lane == 0) mbar_arrive(&empty[p.slot]);
-  }
+  // A consumer warp releases a stage: every lane arrives after its own last read (the empty
+  // barrier counts consumer THREADS), so each reading thread orders its reads before the
+  // producer's next bulk copy into the slot itself (mbarrier release/acquire) — the canonical
+  // TMA-pipeline form, which compute-sanitizer's racecheck can follow (a __syncwarp + one
+  // lane's arrive is ordered by the PTX model too, but racecheck flags it once the ring wraps).
+  __device__ __forceinline__ void release(const RingPos &p, int /*lane*/) const { mbar_arrive(&empty[p.slot]); }
 };
 
 // ---------------------------------------------------------------- small load/store helpers

@@ -17,7 +17,7 @@
 #define JB_SMEM_DEFAULT 232448  // B200 opt-in dynamic shared memory per block (227 KB)
 #define JB_TB_KMAX2 5           // deepest time block of the 2D time-blocked kernel (tblock.cu)
 #define JB_TB_K2D 5             // its default depth (auto; measured fastest)
-#define JB_TB_PPT5 2            // default cell pairs per lane at K = 5
+#define JB_TB_PPT5 1            // default cell pairs per lane at K = 5 (x 11 consumer warps)
 #define JB_TB_LAG 1             // default wavefront lag of the odd-K march
 #define JB_TB_KMAX3 3           // deepest time block of the 3D time-blocked kernel
 #define JB_TB_K3D 3             // its default depth (auto; slabs without neighbours only)

@@ -485,7 +485,7 @@ __global__ void __launch_bounds__(JB_THREADS, 1) jb_sweep(const __grid_constant_
   if (threadIdx.x == 0) {
     for (uint32_t i = 0; i < R.S; ++i) {
       mbar_init(&R.full[i], 1);
-      mbar_init(&R.empty[i], JB_NCW);
+      mbar_init(&R.empty[i], JB_NC);  // one arrival per consumer thread (Ring::release)
     }
     for (int i = 0; i < JB_RQ; ++i) {
       mbar_init(&Q.full[i], 1);

@@ -944,7 +944,7 @@ __device__ __forceinline__ void tb_body(const JbParams &P) {
   if (threadIdx.x == 0) {
     for (uint32_t i = 0; i < R.S; ++i) {
       mbar_init(&R.full[i], 1);
-      mbar_init(&R.empty[i], NCW);
+      mbar_init(&R.empty[i], NCW * 32);  // one arrival per consumer thread (Ring::release)
     }
     for (int i = 0; i < JB_RQ; ++i) {
       mbar_init(&qfull[i], 1);
@@ -1123,6 +1123,8 @@ const void *tblock_fn(int dim, int k, int ppt, int lag, int per_sm, int *ncw) {
     return ppt >= 4 ? JB_TB(jb_tblock<2, 2, 4>) : ppt == 2 ? JB_TB(jb_tblock<2, 2, 2>) : JB_TB(jb_tblock<2, 2, 1>);
   }
   if (per_sm >= 2) return nullptr;
+  *ncw = 11;
+  if (k == 5 && ppt == 1 && lag == 1) return JB_TB(jb_tblock<2, 5, 1, 11, 1>);
   *ncw = 7;
   if (lag == 2) {
     if (k == 3 && ppt == 2) return JB_TB(jb_tblock<2, 3, 2, 7, 2>);

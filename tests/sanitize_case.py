@@ -23,10 +23,12 @@ for shape, P in [((20, 70), 2), ((8, 9, 33), 2), ((30, 40), 1)]:
             j.run(3)
             ok &= bool(np.array_equal(j.gather(), oracle.jacobi(f, 3)))
 # time-blocked kernel (2D K = 5 / 3 / 2, 3D K = 3 / 2, with and without neighbours): TMA ring
-# and TMA boxes, shuffles, the 3D shared-memory row exchange, edge zones
+# and TMA boxes, shuffles, the 3D shared-memory row exchange, edge zones; rings short enough to
+# wrap inside an item (stages=4, and K = 3 with 4 pairs per lane: 14 KB stages)
 for shape, P, prm in [((24, 70), 2, {}), ((20, 70), 2, {"tb_k": 2}), ((12, 9, 33), 2, {}),
                       ((12, 9, 33), 1, {}), ((12, 9, 33), 1, {"tb_k": 2}), ((30, 40), 1, {}),
-                      ((30, 40), 1, {"tb_k": 3})]:
+                      ((30, 40), 1, {"tb_k": 3}), ((30, 40), 1, {"tb_k": 5, "tb_ppt": 2}),
+                      ((30, 40), 1, {"stages": 4}), ((30, 40), 1, {"tb_k": 2, "stages": 4})]:
     f = u12(shape, 4)
     with jb.Jacobi(shape, virtual=P) if P > 1 else jb.Jacobi(shape) as j:
         j.set_param("tblock", 1)

@@ -15,8 +15,8 @@ from jacobi_inputs import SEED_BENCH, integer_field, nv_field, u12
 
 pytestmark = pytest.mark.gpu
 
-# 2D variants (K, pairs per thread); the default (auto) is K = 5, ppt = 2
-KV = [(2, 4), (3, 2), (3, 4), (5, 2)]
+# 2D variants (K, pairs per thread); the default (auto) is K = 5, ppt = 1 (11 consumer warps)
+KV = [(2, 4), (3, 2), (3, 4), (5, 2), (5, 1)]
 K_AUTO = 5
 K3_AUTO = 3  # 3D default (slabs without neighbours)
 KV3 = [(2, 4, -1), (3, 1, 2), (3, 1, 3), (3, 2, 2)]  # 3D (K, ppt, rows per warp)
