@@ -877,29 +877,29 @@ __device__ bool tb_edge(const JbGeom &g, const JbSlab &SL, const JbParams &P, in
           yb = min(y0 + g.ty, ny - 1) - 1;
         }
       }
-      const int64_t w = xb - xa + 1, h = yb - ya + 1;
-      for (int64_t i = tid; i < np * h * w; i += nt) {
-        const int64_t k = i / (h * w), r = i - k * h * w, yy = r / w;
-        const int64_t x = xa + (r - yy * w), y = ya + yy, p = pf + k;
-        const int64_t e = (DIM == 3 ? y * pitch : 0) + x;
-        const bool in = x >= 1 && x <= nx - 2 && (DIM == 2 || (y >= 1 && y <= ny - 2));
-        const double *A = src(p) + e;
-        double v;
-        if (!in) {
-          v = __ldcg(A);
-        } else if (DIM == 2) {  // oracle order: x+1, x-1, y+1, y-1 (then z+1, z-1), then the scale
-          v = 0.25 * (((__ldcg(A + 1) + __ldcg(A - 1)) + __ldcg(src(p + 1) + e)) + __ldcg(src(p - 1) + e));
-        } else {
-          v = kC6 * (((((__ldcg(A + 1) + __ldcg(A - 1)) + __ldcg(A + pitch)) + __ldcg(A - pitch)) +
-                      __ldcg(src(p + 1) + e)) +
-                     __ldcg(src(p - 1) + e));
-        }
-        if (m < K) {
-          E[(lbase(m) + k) * pe + e] = v;
-          if (p == pout) mid[(int64_t)(m - 1) * pe + e] = v;
-        } else {
-          nxt[p * pe + 3 + e] = v;
-          if (p == pout) remote[3 + e] = v;
+      const int w = (int)(xb - xa + 1), hw = (int)(yb - ya + 1) * w;
+      for (int64_t k = 0; k < np; ++k) {  // per plane: source / destination pointers hoisted
+        const int64_t p = pf + k;
+        const double *Sm = src(p - 1), *Sc = src(p), *Sp = src(p + 1);
+        double *D = m < K ? E + (lbase(m) + k) * pe : nxt + p * pe + 3;
+        double *D2 = p != pout ? nullptr : m < K ? mid + (int64_t)(m - 1) * pe : remote + 3;
+        for (int c = tid; c < hw; c += nt) {  // (row, column) of the window, 32-bit index math
+          const int yy = DIM == 3 ? c / w : 0, xx = c - yy * w;
+          const int64_t x = xa + xx, y = ya + yy;
+          const int64_t e = (DIM == 3 ? y * pitch : 0) + x;
+          const bool in = x >= 1 && x <= nx - 2 && (DIM == 2 || (y >= 1 && y <= ny - 2));
+          const double *A = Sc + e;
+          double v;
+          if (!in) {
+            v = __ldcg(A);
+          } else if (DIM == 2) {  // oracle order: x+1, x-1, y+1, y-1 (then z+1, z-1), then the scale
+            v = 0.25 * (((__ldcg(A + 1) + __ldcg(A - 1)) + __ldcg(Sp + e)) + __ldcg(Sm + e));
+          } else {
+            v = kC6 * (((((__ldcg(A + 1) + __ldcg(A - 1)) + __ldcg(A + pitch)) + __ldcg(A - pitch)) + __ldcg(Sp + e)) +
+                       __ldcg(Sm + e));
+          }
+          D[e] = v;
+          if (D2) D2[e] = v;
         }
       }
     }
