@@ -8,7 +8,7 @@ cases = [((24, 70), 2, {}), ((20, 70), 2, {"tb_k": 2}), ((12, 9, 33), 2, {}),
          ((12, 9, 33), 1, {}), ((12, 9, 33), 1, {"tb_k": 2}), ((30, 40), 1, {}), ((30, 40), 1, {"tb_k": 3}),
          ((30, 40), 1, {"tb_k": 5, "stages": 4}), ((30, 40), 1, {"tb_k": 2, "stages": 4}),
          ((30, 40), 1, {"tb_k": 3, "tb_ppt": 2, "stages": 4}), ((30, 40), 1, {"tb_k": 3, "tb_ppt": 4, "stages": 32}),
-         ((30, 600), 1, {"tb_k": 3, "tb_ppt": 4})]
+         ((30, 600), 1, {"tb_k": 3, "tb_ppt": 4}), ((30, 50, 140), 1, {}), ((26, 50, 140), 2, {"tb_k": 3})]
 shape, P, prm = cases[int(sys.argv[1])]
 f = u12(shape, 4)
 with jb.Jacobi(shape, virtual=P) if P > 1 else jb.Jacobi(shape) as j:

@@ -13,7 +13,7 @@ import oracle  # noqa: E402
 import paper_conf_sc_baydamirlibu24_b200 as jb  # noqa: E402
 from jacobi_inputs import u12  # noqa: E402
 
-VARIANTS = [(3, 1, 3), (3, 1, 2)]  # (K, ppt, rows per warp)
+VARIANTS = [(3, 1, 2), (3, 1, 3)]  # (K, ppt, rows per warp)
 
 
 def params(k, ppt, rpw):
