@@ -61,3 +61,51 @@ def test_random_cases(case):
         got = j.gather()
     exp = oracle.jacobi(f, iters)
     assert np.array_equal(got.view(np.uint64), exp.view(np.uint64)), case
+
+
+@st.composite
+def tblock_cases(draw):
+    """The time-blocked kernels: random extents, slab counts, depth K,
+    pairs per lane, wavefront lag / rows per warp, plane blocks, ring depths, iteration counts
+    (not multiples of K: the remainder runs per iteration)."""
+    three_d = draw(st.booleans())
+    P = draw(st.integers(1, 4))
+    n_out = draw(st.integers(3, 2 * P + 60))
+    if three_d:
+        shape = (n_out, draw(st.integers(3, 70)), draw(st.integers(3, 200)))
+        k, ppt = draw(st.sampled_from([(2, 4), (3, 1), (3, 2)]))
+        var = {"tb_rpw": draw(st.sampled_from([2, 3]))}
+    else:
+        shape = (n_out, draw(st.integers(3, 2500)))
+        k, ppt = draw(st.sampled_from([(2, 4), (3, 2), (3, 4), (5, 1), (5, 2)]))
+        var = {"tb_lag": draw(st.sampled_from([1, 2]))}
+    params = {"resident": 0, "tblock": 1, "tb_k": k, "tb_ppt": ppt, **var,
+              "tb_min_block": draw(st.sampled_from([1, 2, 5, 16, 40])),
+              "stages": draw(st.sampled_from([-1, 4, 6]))}
+    iters = draw(st.integers(1, 26))
+    seed = draw(st.integers(0, 2 ** 31))
+    return shape, P, params, iters, seed
+
+
+@settings(max_examples=120, deadline=None, derandomize=True,
+          suppress_health_check=[HealthCheck.too_slow, HealthCheck.data_too_large])
+@given(tblock_cases())
+def test_random_tblock_cases(case):
+    shape, P, params, iters, seed = case
+    if P > 1 and (shape[0] - 2) // P < 2:
+        return  # jacobi_create rejects slabs thinner than 2 planes
+    f = u12(shape, seed)
+    with jb.Jacobi(shape, virtual=P) if P > 1 else jb.Jacobi(shape) as j:
+        for k, v in params.items():
+            j.set_param(k, v)
+        j.scatter(f)
+        try:
+            j.run(iters)
+        except jb.JacobiError as e:
+            # forced with slabs too thin for even K = 2's edge zones: the only allowed refusal
+            assert P > 1 and (shape[0] - 2) // P < 4 and e.code == jb.JACOBI_EINVAL, (case, e)
+            return
+        got = j.gather()
+        kk = j.get_param("last_tb_k")
+    exp = oracle.jacobi(f, iters)
+    assert np.array_equal(got.view(np.uint64), exp.view(np.uint64)), (case, kk)
