@@ -41,6 +41,9 @@ __device__ __forceinline__ void tma_box3(void *dst, const void *tmap, int c0, in
       : "memory");
 }
 
+// The odd-K marches run towards row / plane 0 (shorter fp64 dependency chain, see tbk_march).
+constexpr bool TB_REV = true;
+
 // Position `off` stages after p in the ring.
 __device__ __forceinline__ RingPos ring_add(RingPos p, uint32_t off, uint32_t S) {
   const uint32_t s = p.slot + off;
@@ -316,7 +319,13 @@ __device__ __forceinline__ void tbk_levelk(const TbkLane &L, const double2 *S, c
 // a step form one dependency chain, three rows per level in registers; LAG = 2: the K levels of a
 // step are independent (more instruction-level parallelism, four rows per level).  Set m % NS
 // of a level holds its row computed at step m (static rotation, the loop unrolled by NS).
-template <int K, int PPT, int LAG, bool FAST>
+// REV: the march runs towards row 0 (the producer streams the rows in decreasing order; a, b,
+// r0, r1 are then mirrored row indices r' = C+1-r).  In the oracle order ((x+1 + x-1) + y+1) +
+// y-1, the row a level just computed is the NEWEST row of the march: marching up it is y+1
+// (three dependent fp64 operations after it: + y+1, + y-1, * 1/4), marching down it is y-1
+// (two: + y-1, * 1/4), so the dependency chain through the K levels of a step is ~25 % shorter
+// — same operations, same order, bit-identical results.
+template <int K, int PPT, int LAG, bool FAST, bool REV>
 __device__ __forceinline__ void tbk_march(const TbkLane &L, const Ring &R, RingPos q, int a, int b, int C, int r0,
                                           int r1, double *dst, int64_t pe, int lane) {
   constexpr int NS = LAG + 2;
@@ -325,7 +334,10 @@ __device__ __forceinline__ void tbk_march(const TbkLane &L, const Ring &R, RingP
   const int Re = b + 1 + LAG * (K - 1);         // last step: level K of row b
   // steady window: every level's row is needed and interior, level K is stored
   const int Ws = a + 1 + LAG * (K - 1), We = min(b + K, C + 1);
-  double *o = dst + (int64_t)(Rs - 1 - LAG * (K - 1)) * pe;  // output row of step Rs (advanced per step)
+  // output row of step Rs (advanced per step; REV: actual row C+1-r', moving down)
+  const int ro0 = Rs - 1 - LAG * (K - 1);
+  double *o = dst + (int64_t)(REV ? C + 1 - ro0 : ro0) * pe;
+  const int64_t ostep = REV ? -pe : pe;
   // stage positions of level-0 rows R-2, R-1, R, clamped to r0 .. r1
   RingPos pm = q, pc = Rs == r0 + 2 ? ring_add(q, 1u, R.S) : q, pn = pc;
   if (Rs <= r1) pn = ring_add(q, (uint32_t)(Rs - r0), R.S);
@@ -339,20 +351,23 @@ __device__ __forceinline__ void tbk_march(const TbkLane &L, const Ring &R, RingP
     // level k computes row Rr-1-LAG(k-1) if it lies in its range [a-(K-k), b+(K-k)] ∩ [0, C+1]
     auto need = [&](int k, int r) { return r >= max(a - (K - k), 0) && r <= min(b + (K - k), C + 1); };
     if (ST || Rr <= r1) R.wait_full(pn);
+    // (y-1, centre, y+1) rows: the march's older / newer neighbours, swapped when it runs down
     if (ST || need(1, Rr - 1))
-      tbk_level1<PPT, FAST, ST>(L, R.stage(pm), R.stage(pc), R.stage(pn), Rr - 1 >= 1 && Rr - 1 <= C, X[0][U]);
+      tbk_level1<PPT, FAST, ST>(L, R.stage(REV ? pn : pm), R.stage(pc), R.stage(REV ? pm : pn), Rr - 1 >= 1 && Rr - 1 <= C,
+                                X[0][U]);
     if (ST || (Rr - 2 >= r0 && Rr - 2 <= r1)) R.release(pm, lane);  // row Rr-2 is no longer needed
 #pragma unroll
     for (int k = 2; k < K; ++k) {
       const int r = Rr - 1 - LAG * (k - 1);
       if (ST || need(k, r))
-        tbk_levelk<PPT, FAST, ST, false>(L, X[k - 2][SS], X[k - 2][SC], X[k - 2][SN], r >= 1 && r <= C, lane,
-                                         X[k - 1][U], nullptr);
+        tbk_levelk<PPT, FAST, ST, false>(L, X[k - 2][REV ? SN : SS], X[k - 2][SC], X[k - 2][REV ? SS : SN],
+                                         r >= 1 && r <= C, lane, X[k - 1][U], nullptr);
     }
     const int ro = Rr - 1 - LAG * (K - 1);
     if (ST || (ro >= a && ro <= b))
-      tbk_levelk<PPT, FAST, ST, true>(L, X[K - 2][SS], X[K - 2][SC], X[K - 2][SN], true, lane, nullptr, o);
-    o += pe;
+      tbk_levelk<PPT, FAST, ST, true>(L, X[K - 2][REV ? SN : SS], X[K - 2][SC], X[K - 2][REV ? SS : SN], true, lane,
+                                      nullptr, o);
+    o += ostep;
     pm = pc;
     pc = pn;
     if (Rr + 1 <= r1) {  // branch-free ring advance
@@ -420,8 +435,11 @@ __device__ __forceinline__ void tbk_item(const JbGeom &g, const Ring &R, RingPos
   }
   const bool fast = sw >= 1 && sw + 64 * PPT - 1 <= g.nx - 2;
   double *dst = out + 3 + sw + 2 * PPT * lane;
-  if (fast) tbk_march<K, PPT, LAG, true>(L, R, q0, (int)a, (int)b, (int)C, (int)r0, (int)r1, dst, g.plane_elems, lane);
-  else tbk_march<K, PPT, LAG, false>(L, R, q0, (int)a, (int)b, (int)C, (int)r0, (int)r1, dst, g.plane_elems, lane);
+  // march downwards (TB_REV): rows in mirrored coordinates r' = C+1-r
+  const int ma = TB_REV ? (int)(C + 1 - b) : (int)a, mb = TB_REV ? (int)(C + 1 - a) : (int)b;
+  const int m0 = TB_REV ? (int)(C + 1 - r1) : (int)r0, m1 = TB_REV ? (int)(C + 1 - r0) : (int)r1;
+  if (fast) tbk_march<K, PPT, LAG, true, TB_REV>(L, R, q0, ma, mb, (int)C, m0, m1, dst, g.plane_elems, lane);
+  else tbk_march<K, PPT, LAG, false, TB_REV>(L, R, q0, ma, mb, (int)C, m0, m1, dst, g.plane_elems, lane);
 }
 
 // ---------------------------------------------------------------- 3D (7-point)
@@ -676,7 +694,10 @@ __device__ __forceinline__ void tb3k_levelk(const Tb3kLane &L, const double2 (*Z
   }
 }
 
-template <int K, int PPT, int RPW, int NCW, bool FAST>
+// REV (TB_REV): the z march runs towards plane 0 (a, b, r0, r1 in mirrored plane indices
+// p' = C+1-p), so the newest level plane is z-1, the last term of the oracle order: two instead
+// of three dependent fp64 operations per level on the step's critical path (see tbk_march).
+template <int K, int PPT, int RPW, int NCW, bool FAST, bool REV>
 __device__ __forceinline__ void tb3k_march(const Tb3kLane &L, const JbGeom &g, const Ring &R, RingPos q, int a,
                                            int b, int C, int r0, int r1, double *dst, double *xch, int warp,
                                            int lane) {
@@ -688,7 +709,8 @@ __device__ __forceinline__ void tb3k_march(const Tb3kLane &L, const JbGeom &g, c
   const int Ws = a + K, We = min(b + K, C + 1);
   const int ws = g.ws, sr0 = warp * RPW + 1;
   const int64_t pe = g.plane_elems, pitch = g.pitch;
-  double *o = dst + (int64_t)(Rs - K) * pe;
+  double *o = dst + (int64_t)(REV ? C + 1 - (Rs - K) : Rs - K) * pe;
+  const int64_t ostep = REV ? -pe : pe;
   // exchange slots: [level k-1][parity][warp][0 = first row, 1 = last row][TX]
   auto xrow = [&](int k1, int par, int w, int side) { return xch + ((((k1 * 2 + par) * NCW + w) * 2 + side) * TX); };
   const int wu = warp > 0 ? warp - 1 : warp, wd = warp + 1 < NCW ? warp + 1 : warp;  // edge warps: any row
@@ -712,7 +734,8 @@ __device__ __forceinline__ void tb3k_march(const Tb3kLane &L, const JbGeom &g, c
     if (ST || Rr <= r1) R.wait_full(pn);
     bar_consumers<NCW>();  // the previous step's exchange rows are visible; its reads are done
     if (ST || need(1, Rr - 1)) {
-      tb3k_level1<PPT, RPW, FAST, ST>(L, sr0, ws, R.stage(pm), R.stage(pc), R.stage(pn), Rr - 1 >= 1 && Rr - 1 <= C,
+      tb3k_level1<PPT, RPW, FAST, ST>(L, sr0, ws, R.stage(REV ? pn : pm), R.stage(pc), R.stage(REV ? pm : pn),
+                                      Rr - 1 >= 1 && Rr - 1 <= C,
                                       X[0][U]);
       publish(0, par, X[0][U]);
     }
@@ -728,15 +751,16 @@ __device__ __forceinline__ void tb3k_march(const Tb3kLane &L, const JbGeom &g, c
         yB[i] = lds2(xrow(k - 2, prv, wd, 0) + 2 * (lane * PPT + i));
       }
       if (k < K) {
-        tb3k_levelk<PPT, RPW, FAST, ST, false>(L, X[k - 2][SS], X[k - 2][SC], X[k - 2][SN], yT, yB,
+        tb3k_levelk<PPT, RPW, FAST, ST, false>(L, X[k - 2][REV ? SN : SS], X[k - 2][SC], X[k - 2][REV ? SS : SN], yT, yB,
                                                r >= 1 && r <= C, lane, X[k - 1][U], nullptr, pitch);
         publish(k - 1, par, X[k - 1][U]);
       } else {
-        tb3k_levelk<PPT, RPW, FAST, ST, true>(L, X[k - 2][SS], X[k - 2][SC], X[k - 2][SN], yT, yB, true, lane,
+        tb3k_levelk<PPT, RPW, FAST, ST, true>(L, X[k - 2][REV ? SN : SS], X[k - 2][SC], X[k - 2][REV ? SS : SN], yT, yB,
+                                              true, lane,
                                               nullptr, o, pitch);
       }
     }
-    o += pe;
+    o += ostep;
     pm = pc;
     pc = pn;
     if (Rr + 1 <= r1) {
@@ -799,10 +823,12 @@ __device__ __forceinline__ void tb3k_item(const JbGeom &g, const Ring &R, RingPo
   }
   const bool fast = sx >= 1 && sx + 64 * PPT - 1 <= g.nx - 2 && sy >= 1 && sy + TY - 1 <= g.ny - 2;
   double *dst = out + (sy + (int64_t)warp * RPW) * g.pitch + 3 + sx + 2 * PPT * lane;
+  const int ma = TB_REV ? (int)(C + 1 - b) : (int)a, mb = TB_REV ? (int)(C + 1 - a) : (int)b;
+  const int m0 = TB_REV ? (int)(C + 1 - r1) : (int)r0, m1 = TB_REV ? (int)(C + 1 - r0) : (int)r1;
   if (fast)
-    tb3k_march<K, PPT, RPW, NCW, true>(L, g, R, q0, (int)a, (int)b, (int)C, (int)r0, (int)r1, dst, xch, warp, lane);
+    tb3k_march<K, PPT, RPW, NCW, true, TB_REV>(L, g, R, q0, ma, mb, (int)C, m0, m1, dst, xch, warp, lane);
   else
-    tb3k_march<K, PPT, RPW, NCW, false>(L, g, R, q0, (int)a, (int)b, (int)C, (int)r0, (int)r1, dst, xch, warp, lane);
+    tb3k_march<K, PPT, RPW, NCW, false, TB_REV>(L, g, R, q0, ma, mb, (int)C, m0, m1, dst, xch, warp, lane);
 }
 
 // Edge zone of a slab side with a neighbour (time block t -> t+K), computed by that side's
@@ -1019,7 +1045,7 @@ __device__ __forceinline__ void tb_body(const JbParams &P) {
             if (lane == 0) {
               mbar_wait(&R.empty[q.slot], q.phase ^ 1u);
               mbar_expect_tx(&R.full[q.slot], box);
-              tma_box3(R.stage(q), tm, (int)xs_w, (int)ya, (int)p, &R.full[q.slot]);
+              tma_box3(R.stage(q), tm, (int)xs_w, (int)ya, (int)(TB_REV ? r0 + r1 - p : p), &R.full[q.slot]);
             }
             q.advance(R.S);
           }
@@ -1029,7 +1055,9 @@ __device__ __forceinline__ void tb_body(const JbParams &P) {
           item = SL.dyn_first + (int64_t)__shfl_sync(0xffffffffu, claim, 0);
           continue;
         }
-        for (int64_t p = r0; p <= r1; ++p) {
+        const bool down = K > 2 && TB_REV;  // the odd-K marches run towards row / plane 0
+        for (int64_t i = r0; i <= r1; ++i) {
+          const int64_t p = down ? r0 + r1 - i : i;
           if (lane == 0) {
             mbar_wait(&R.empty[q.slot], q.phase ^ 1u);
             mbar_expect_tx(&R.full[q.slot], bytes * nvalid);
