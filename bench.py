@@ -341,7 +341,11 @@ def main():
                    "parallelism": f"slab{world}" + (f" (virtual {args.virtual} slabs)" if args.virtual else ""),
                    "l2": ("inputs larger than L2" if 8 * cells > L2_BYTES else "L2-resident (latency config)"),
                    "tile": {k: desc[k] for k in ("tile_x", "tile_y", "stages", "ctas", "n_top", "n_bot", "k_planes")},
-                   "kernel": kkind},
+                   "kernel": kkind,
+                   **({"time_block": {"K": tb_k, "iters_time_blocked": tb_iters,
+                                      "note": "tile above is the per-iteration plan; the time-blocked "
+                                              "kernel's strips/tiles are in DESIGN.md 5.8-5.9"}}
+                      if tb_iters else {})},
         "gpu_launches": args.steps * world * (2 if 0 < tb_iters < iters else 1),
         "wall_ms_per_step": 1e3 * t_wall / args.steps,
         "ms_per_iter": dev_ms / args.steps / iters,
