@@ -14,7 +14,7 @@ import oracle  # noqa: E402
 import paper_conf_sc_baydamirlibu24_b200 as jb  # noqa: E402
 from jacobi_inputs import u12  # noqa: E402
 
-VARIANTS = [(5, 1, 1), (5, 2, 1), (3, 2, 1)]
+VARIANTS = [(5, 1, 1), (5, 1, 2), (3, 1, 2)]
 
 
 def run(shape, iters, k, ppt, lag, virtual=0, extra=None):
