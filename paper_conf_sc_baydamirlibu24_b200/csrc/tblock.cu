@@ -1,23 +1,25 @@
-// tblock.cu — temporally blocked CPU-Free sweep: K = 2 Jacobi iterations per pass
-// over HBM, for a slab without neighbours (P = 1, both outer halos are the Dirichlet planes).
+// tblock.cu — temporally blocked CPU-Free sweep: K Jacobi iterations per
+// pass over HBM — 2D: K = 2 (extra-cell scheme, §5.7), K = 3 / 5 (overlapped warp segments,
+// §5.8; default K = 5); 3D: K = 2 (§5.7), K = 3 (x/y-overlapped tiles with a shared-memory row
+// exchange and TMA box loads, §5.9; the default for slabs without neighbours).
 //
 // The method is unchanged — every cell is updated every iteration with the oracle's fp64 order
 // (-fmad=false), each iteration reads only the previous time step, Dirichlet cells are
 // never written — only the schedule of the updates differs: a work item (plane block
-// [a, b] x x-strip) streams the time-t planes a-2 .. b+2 of its strip from HBM through the same
-// TMA bulk-copy ring as jb_sweep, computes time t+1 for planes a-1 .. b+1 in registers (x
-// neighbours by warp shuffles), and from those time t+2 for planes a .. b, columns
-// x0 .. x0+tx-1, which it stores into the other buffer.  The intermediate time level never
-// touches HBM, so the algorithmic traffic per cell-update is 16 B / K = 8 B instead of 16 B
-// (overlapped tiling: the t+1 values of the 2 extra planes of each item and of one extra column
-// at each end of each warp's segment are recomputed, < 2 % extra arithmetic at C2).
-// The persistent structure of the paper is kept: one cooperative launch for the whole run, a
-// device-side grid barrier between time blocks, no host involvement.
+// [a, b] x strip / tile) streams the time-t planes a-K .. b+K of its strip from HBM through the
+// same TMA ring as jb_sweep, computes the intermediate levels t+1 .. t+K-1 in registers (x
+// neighbours by warp shuffles) and level t+K for planes a .. b, which it stores into the other
+// buffer.  The intermediate levels never touch HBM, so the algorithmic traffic per cell-update
+// is 16 B / K instead of 16 B (overlapped tiling: the values near a strip's / tile's edges are
+// recomputed by its neighbours).  Slabs with neighbours keep the paper's per-iteration halo
+// exchange through edge zones (K phases per time block, tb_edge).  The persistent structure of
+// the paper is kept: one cooperative launch for the whole run, a device-side grid barrier
+// between time blocks, no host involvement.
 //
 // Buffers: time block j of a launch reads buf[(t0 + j) & 1] and writes buf[(t0 + j + 1) & 1]
-// (out of place — neighbouring strips still read the time-t columns of this strip); the host
-// runs an even number of blocks, so the result lands in buf[(t0 + 2 nb) & 1] as in every other
-// path (R10).
+// (out of place — neighbouring strips still read the time-t columns of this strip); for K = 2
+// the host runs an even number of blocks, for odd K any number, so the result lands in
+// buf[(t0 + K nb) & 1] as in every other path (R10).
 #include <type_traits>
 
 #include "device_common.cuh"
