@@ -7,14 +7,23 @@ One "step" is one pass of the whole hot path over the BASELINE.json workload: on
 ``jacobi_run(iters)`` call — ONE persistent kernel per GPU running every iteration with the
 halo exchange, flags and grid barriers inside.  At N = 1 the
 workload is BASELINE.json configs[1] (C2: 2D 5-point 16384x16384 fp64, 1000 iterations).
-``value`` = interior cells x iterations x K / max-over-ranks device time (CUDA events on the
+``value`` = interior cells x iterations x steps / max-over-ranks device time (CUDA events on the
 launch stream around each launch), in Gcell-updates/s.  Inputs (2 GiB per buffer) are larger
 than the 126 MB L2, so no flush is needed between steps.
 
-Extra keys: ``roofline`` (the persistent kernel vs the measured HBM copy bandwidth),
-``cpu_baseline`` (the CPU oracle on this host's cores, bounded sample), ``e2e`` (the same
-metric through the C ABI with pinned host buffers: scatter + run + gather per step),
-``cpu_controlled`` (the per-iteration-launch baselines), ``clocks``.
+N GPUs: under torchrun (WORLD_SIZE > 1) one rank per GPU, slabs linked by CUDA IPC; without
+torchrun ``--gpus N`` drives N GPUs from one process (jacobi_create(ngpus=N): UVA peer stores
+after cudaDeviceEnablePeerAccess) and exits with an error (JACOBI_ENODEV) if fewer are visible.
+C2/C3 keep the grid (strong scaling), C4 grows it to 512x512x(512N) (weak scaling).
+
+Extra keys: ``roofline`` (the persistent kernel vs the measured HBM copy bandwidth, per GPU;
+µs/iteration for the L2-resident latency configs C1/C5), ``cpu_baseline`` (the CPU oracle on
+this host's cores, bounded sample), ``e2e`` (the same metric through the C ABI with pinned host
+buffers: scatter + run + gather per step), ``cpu_controlled`` (the per-iteration-launch
+baselines), ``clocks``; at N > 1 ``halo_us`` (per-iteration time of
+no-compute runs, CPU-Free vs the CPU-controlled baselines), ``halo_traffic`` (halo
+bytes per iteration and GB/s vs NVLink's 900 GB/s) and ``halo_spans_*`` (in-kernel %globaltimer
+wait -> flag -> signal spans of the boundary blocks, jacobi_halo_trace).
 
 ``--impl reference``: there is no reference implementation to install (PAPER.md only), so
 the reference arm is the CPU oracle timed on this host.
@@ -151,7 +160,27 @@ def ncu_traffic(config: str, iters: int):
         return None, None
 
 
-def run_reference(args, cfg, shape):
+def cpu_model() -> str:
+    try:
+        with open("/proc/cpuinfo") as f:
+            for line in f:
+                if line.startswith("model name"):
+                    return line.split(":", 1)[1].strip()
+    except OSError:
+        pass
+    return "unknown"
+
+
+def workload_config(cfg, shape, n_gpus, virtual=0):
+    """The `config` object of BOTH arms (same keys and values, so the driver can pair the lines):
+    what the workload is, never how an arm computes it."""
+    cells = interior_cells(shape)
+    return {"workload": cfg["workload"], "shape_zyx": list(shape), "iters": cfg["iters"],
+            "parallelism": f"slab{n_gpus}" + (f" (virtual {virtual} slabs)" if virtual else ""),
+            "l2": ("inputs larger than L2" if 8 * cells > L2_BYTES else "L2-resident (latency config)")}
+
+
+def run_reference(args, cfg, shape, n_gpus):
     world, rank, _ = dist_env()
     if rank != 0:
         return 0
@@ -168,14 +197,16 @@ def run_reference(args, cfg, shape):
     value = interior_cells(shape) * k_iter * args.steps / sum(secs) / 1e9
     sample = f"{k_iter} of {cfg['iters']} iterations of the full {cfg['workload'].split(':')[0]} grid per step"
     line = {
-        "impl": "reference", "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": args.gpus,
+        "impl": "reference", "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": n_gpus,
         "steps": args.steps, "warmup": args.warmup, "ms_per_step": 1e3 * sum(secs) / args.steps,
         "higher_is_better": True, "scaling": cfg["scaling"], "vs_baseline": None, "dtype": "f64",
         "data": "synthetic (U12 seed 0x5C24)",
-        "config": {"workload": cfg["workload"], "shape_zyx": list(shape), "iters": cfg["iters"]},
-        "cpu_baseline": {"value": value, "unit": UNIT, "cores": cores, "kind": "oracle", "sample": sample},
+        "config": workload_config(cfg, shape, n_gpus),
+        "cpu_baseline": {"value": value, "unit": UNIT, "cores": cores, "cpu_model": cpu_model(), "kind": "oracle",
+                         "sample": sample},
         "e2e": {"value": value, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
-        "note": "no reference code exists (PAPER.md only); the reference arm is the CPU oracle",
+        "note": "no reference code exists (PAPER.md only); the reference arm is the CPU oracle (plain C, "
+                "OpenMP over the outer axis) on this host's cores",
     }
     emit(line)
     return 0
@@ -189,6 +220,47 @@ def emit(line: dict) -> None:
     os.write(_JSON_FD if _JSON_FD is not None else 1, (json.dumps(line) + "\n").encode())
 
 
+def halo_latency(j, jb, modes, max_over_ranks, n=200):
+    """Per-iteration time of no-compute runs (halo copies, flags and barriers only),
+    (T(2n) - T(n)) / n to cancel the launch cost; µs.  Modes a handle does not support are
+    reported as errors (e.g. the host-copy baselines in one-process-per-GPU mode)."""
+    out = {}
+    for name, mode in modes:
+        try:
+            j.set_mode(mode, jb.FLAG_NO_COMPUTE)
+            j.run(n // 2)
+            j.run(n)
+            t1 = max_over_ranks(j.last_time_ms())
+            j.run(2 * n)
+            t2 = max_over_ranks(j.last_time_ms())
+            out[name] = 1e3 * (t2 - t1) / n
+        except jb.JacobiError as e:
+            out[name] = {"error": str(e)}
+    j.set_mode(jb.MODE_CPUFREE)
+    return out
+
+
+def traced_spans(j, jb, iters, n_trace, gather):
+    """In-kernel %globaltimer spans of the boundary blocks (wait -> flag -> signal) over one
+    CPU-Free run of the current workload; median over exchanges and slabs (skipping the first
+    few exchanges of the launch), max over ranks via `gather`."""
+    j.set_param("halo_trace", n_trace)
+    try:
+        j.run(iters)
+        spans = []
+        for i in range(j.local_slabs):
+            spans.append(jb.halo_spans(j.halo_trace(i, min(n_trace, iters)), skip=min(8, iters // 4)))
+    finally:
+        j.set_param("halo_trace", 0)
+    keys = ("wait_us", "put_us", "span_us", "period_us")
+    res = {}
+    for k in keys:
+        v = [sp[k] for sp in spans if sp[k] is not None]
+        res[k] = gather(max(v)) if v else None
+    res["exchanges_per_slab"] = spans[0]["exchanges"] if spans else 0
+    return res
+
+
 def main():
     global _JSON_FD
     # stdout carries only the JSON line: NCCL and other native code print to fd 1 (e.g. "NCCL
@@ -197,7 +269,9 @@ def main():
     _JSON_FD = os.dup(1)
     os.dup2(2, 1)
     ap = argparse.ArgumentParser()
-    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--gpus", type=int, default=1,
+                    help="GPUs: under torchrun one rank per GPU (WORLD_SIZE wins); without it one "
+                         "process drives N GPUs (jacobi_create(ngpus=N), UVA peer stores)")
     ap.add_argument("--steps", type=int, default=3)
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--config", default="c2", choices=sorted(CONFIGS))
@@ -205,6 +279,7 @@ def main():
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--ref-iters", type=int, default=2, help="oracle iterations per reference step")
     ap.add_argument("--no-extras", action="store_true", help="skip e2e / cpu_baseline / baselines")
+    ap.add_argument("--no-clocks", action="store_true", help="(diagnostic) no nvidia-smi sampling")
     ap.add_argument("--virtual", type=int, default=0, help="(measurement aid) P slabs on one GPU")
     ap.add_argument("--param", action="append", default=[], help="tuning knob name=value (jacobi_set_param)")
     ap.add_argument("--transport", default="ipc", choices=["ipc", "nvshmem"],
@@ -213,18 +288,29 @@ def main():
     args.warmup = max(args.warmup, 3) if args.impl == "ours" else args.warmup
 
     world, rank, local = dist_env()
-    ndev = torch_device_count()
-    local = local % max(ndev, 1)  # (more ranks than GPUs only in functional tests: time-sliced)
+    # N GPUs of the whole job: torchrun ranks, or --gpus in one process
+    n_gpus = world if world > 1 else max(args.gpus, 1)
+    single_multi = world == 1 and n_gpus > 1
     cfg = dict(CONFIGS[args.config])
     if args.iters:
         cfg["iters"] = args.iters
-    shape = cfg["shape"] or (512 * max(world, 1), 512, 512)
+    shape = cfg["shape"] or (512 * n_gpus, 512, 512)  # C4 weak scaling: 512 z planes per GPU (R15)
     iters = cfg["iters"]
 
     if args.impl == "reference":
-        return run_reference(args, cfg, shape)
+        return run_reference(args, cfg, shape, n_gpus)
 
-    import numpy as np
+    ndev = torch_device_count()
+    if single_multi and ndev < n_gpus:
+        # fail loudly (JACOBI_ENODEV): never measure fewer GPUs than asked for
+        print(f"[bench] --gpus {n_gpus} needs {n_gpus} visible GPUs, found {ndev} (JACOBI_ENODEV)", file=sys.stderr)
+        return 2
+    if world > 1 and ndev < 1:
+        print("[bench] no GPU visible to this rank (JACOBI_ENODEV)", file=sys.stderr)
+        return 2
+    local = local % max(ndev, 1)  # (more ranks than GPUs only in functional tests: time-sliced)
+
+    import numpy as np  # noqa: F401
     import torch
     import paper_conf_sc_baydamirlibu24_b200 as jb
 
@@ -248,7 +334,7 @@ def main():
     else:
         jb.use_torch_allocator()
         dist = None
-        j = jb.Jacobi(shape, virtual=args.virtual) if args.virtual else jb.Jacobi(shape, ngpus=1)
+        j = jb.Jacobi(shape, virtual=args.virtual) if args.virtual else jb.Jacobi(shape, ngpus=n_gpus)
     torch.cuda.set_device(local)
     for kv in args.param:
         k, v = kv.split("=")
@@ -265,90 +351,123 @@ def main():
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
         return float(t.item())
 
+    def sum_over_ranks(x: float) -> float:
+        if dist is None:
+            return x
+        t = torch.tensor([x], dtype=torch.float64)
+        dist.all_reduce(t, op=dist.ReduceOp.SUM)
+        return float(t.item())
+
+    def sync_all():
+        for d in range(ndev if single_multi else 0):
+            torch.cuda.synchronize(d)
+        torch.cuda.synchronize(local)
+
     cells = interior_cells(shape)
-    desc = j.describe(0)
-    local_cells = cells // (shape[0] - 2 if shape[0] > 1 else shape[1] - 2) * desc["chunk"] \
-        if world > 1 else cells
+    desc = j.describe(0)  # slab 0 owns the largest chunk (the first r slabs get one more plane)
+    per_plane = cells // (shape[0] - 2 if shape[0] > 1 else shape[1] - 2)
+    local_cells = per_plane * desc["chunk"] if n_gpus > 1 else cells  # cells of the busiest GPU
 
     # ---- warm-up + timed region (device time per launch from CUDA events on the launch stream)
     for _ in range(args.warmup):
         j.run(iters)
     barrier()
-    torch.cuda.synchronize()
-    clocks = ClockSampler(local) if rank == 0 else None
+    sync_all()
+    clocks = ClockSampler(local) if rank == 0 and not args.no_clocks else None
     if clocks:
         clocks.start()
     t_wall0 = time.perf_counter()
     step_ms = []
+    launches = 0
     for _ in range(args.steps):
         j.run(iters)
-        step_ms.append(j.last_time_ms())
-    torch.cuda.synchronize()
+        step_ms.append(j.last_time_ms())  # max over this process's GPUs
+        launches += j.get_param("last_launches")
+    sync_all()
     barrier()
     t_wall = time.perf_counter() - t_wall0
     clk = clocks.stop() if clocks else None
     dev_ms_local = sum(step_ms)
     dev_ms = max_over_ranks(dev_ms_local)
     value = cells * iters * args.steps / (dev_ms / 1e3) / 1e9
+    launches = int(sum_over_ranks(launches))
 
     # ---- roofline of the dominant kernel.  Per cell-update it moves 16 B (read once + write
     #      once) when it runs one iteration per pass over HBM, 16/K B when the
-    #      temporally blocked kernel runs K iterations per pass.
+    #      temporally blocked kernel runs K iterations per pass.  Per GPU: the
+    #      busiest GPU's cells over its launch time.
     peak, peak_kind = measured_hbm()
-    launch_ms = dev_ms_local / args.steps
+    launch_ms = dev_ms / args.steps
     tb_iters = jb.jacobi_get_param(j.h, "last_tblock")
     tb_k = max(jb.jacobi_get_param(j.h, "last_tb_k"), 1)
+    resident = bool(jb.jacobi_get_param(j.h, "last_resident"))
     alg_bytes = round(local_cells * (16 * (iters - tb_iters) + 16 / tb_k * tb_iters))
     achieved = alg_bytes / (launch_ms / 1e3) / 1e9
     dimk = 2 if shape[0] == 1 else 3
     if tb_iters:
         kname = f"jb_tblock<{dimk},{tb_k},*> (persistent CPU-Free kernel, {tb_k} iterations per HBM pass)"
         kkind = "tblock"
-    elif jb.jacobi_get_param(j.h, "last_resident"):
+    elif resident:
         kname = f"jb_resident<{dimk},*> (persistent CPU-Free kernel, on-chip resident)"
         kkind = "resident"
     else:
         kname = f"jb_sweep<{dimk},false,true,false> (persistent CPU-Free kernel, streaming)"
         kkind = "streaming"
-    traffic, _ = ncu_traffic(args.config + ("_tblock" if tb_iters else ""), iters)
-    roofline = {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
-                "frac": achieved / peak, "traffic": traffic, "peak_kind": peak_kind,
-                "kernel": kname, "alg_bytes_per_launch": alg_bytes,
-                "alg_bytes_per_cell_update": alg_bytes / (local_cells * iters)}
-    if tb_iters:
-        # K iterations per HBM pass move 16/K B per update, so HBM is no longer the only ceiling:
-        # (a) the bandwidth a one-iteration-per-pass kernel would need for the same throughput
-        #     (16 B per update; > the HBM peak means the time blocking beat the HBM roofline);
-        # (b) the fp64 pipe: 3 DADD + 1 DMUL (2D) / 5 + 1 (3D) per update, no FMA (oracle order),
-        #     64 fp64 lanes per SM per clock (B200 vector fp64 ~37 TFLOP/s; ncu's
-        #     sm__pipe_fp64_cycles_active agrees: DESIGN.md §5.8), 148 SMs at the max SM clock.
-        sm_mhz = (clk or {}).get("sm_max_mhz") or 1965.0
-        fp64_peak = 64 * 148 * sm_mhz * 1e6
-        ops = 4 if dimk == 2 else 6
-        roofline["equivalent_gbs_at_16B"] = 16 * local_cells * iters / (launch_ms / 1e3) / 1e9
-        roofline["equivalent_frac_at_16B"] = roofline["equivalent_gbs_at_16B"] / peak
-        roofline["fp64_pipe"] = {"achieved_ops": ops * local_cells * iters / (launch_ms / 1e3),
-                                 "peak_ops": fp64_peak, "frac": ops * local_cells * iters / (launch_ms / 1e3) / fp64_peak,
-                                 "ops_per_update": ops, "peak_basis": "64 fp64 lanes/SM/clk x 148 SMs x max SM clock (DESIGN.md 5.8)"}
+    l2_resident = 8 * cells <= L2_BYTES
+    us_per_iter = 1e3 * launch_ms / iters
+    if l2_resident:
+        # C1 / C5: the field lives in L2 (or on chip), so HBM is not the bound: latency per
+        # iteration (grid barrier + flag round trip) is the figure of merit
+        roofline = {"bound": "latency", "achieved": us_per_iter, "peak": None, "unit": "us/iteration",
+                    "frac": None, "traffic": None, "kernel": kname,
+                    "note": "L2-resident latency config: microseconds per iteration, not an HBM fraction"}
+    else:
+        traffic, _ = ncu_traffic(args.config + ("_tblock" if tb_iters else ""), iters)
+        roofline = {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
+                    "frac": achieved / peak, "traffic": traffic, "peak_kind": peak_kind,
+                    "kernel": kname, "alg_bytes_per_launch": alg_bytes,
+                    "alg_bytes_per_cell_update": alg_bytes / (local_cells * iters),
+                    "per_gpu": n_gpus > 1}
+        if tb_iters:
+            # K iterations per HBM pass move 16/K B per update, so HBM is no longer the only ceiling:
+            # (a) the bandwidth a one-iteration-per-pass kernel would need for the same throughput
+            #     (16 B per update; > the HBM peak means the time blocking beat the HBM roofline);
+            # (b) the fp64 pipe: 3 DADD + 1 DMUL (2D) / 5 + 1 (3D) per update, no FMA (oracle order),
+            #     64 fp64 lanes per SM per clock (B200 vector fp64 ~37 TFLOP/s; ncu's
+            #     sm__pipe_fp64_cycles_active agrees: DESIGN.md §5.8), 148 SMs at the max SM clock.
+            sm_mhz = (clk or {}).get("sm_max_mhz") or 1965.0
+            fp64_peak = 64 * 148 * sm_mhz * 1e6
+            ops = 4 if dimk == 2 else 6
+            roofline["equivalent_gbs_at_16B"] = 16 * local_cells * iters / (launch_ms / 1e3) / 1e9
+            roofline["equivalent_frac_at_16B"] = roofline["equivalent_gbs_at_16B"] / peak
+            roofline["fp64_pipe"] = {"achieved_ops": ops * local_cells * iters / (launch_ms / 1e3),
+                                     "peak_ops": fp64_peak,
+                                     "frac": ops * local_cells * iters / (launch_ms / 1e3) / fp64_peak,
+                                     "ops_per_update": ops,
+                                     "peak_basis": "64 fp64 lanes/SM/clk x 148 SMs x max SM clock (DESIGN.md 5.8)"}
 
+    transport = ("none" if n_gpus == 1 else
+                 "nvshmem" if (world > 1 and args.transport == "nvshmem") else
+                 "cuda-ipc peer stores (one process per GPU)" if world > 1 else
+                 "UVA peer stores (one process, cudaDeviceEnablePeerAccess)")
     line = {
-        "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
-        "transport": args.transport if world > 1 else "none",
+        "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": n_gpus, "steps": args.steps,
+        "transport": transport,
         "warmup": args.warmup, "ms_per_step": dev_ms / args.steps, "higher_is_better": True,
         "scaling": cfg["scaling"], "vs_baseline": None, "dtype": "f64",
         "data": "synthetic (U12 seed 0x5C24, initialised on the device)",
-        "config": {"workload": cfg["workload"], "shape_zyx": list(shape), "iters": iters,
-                   "parallelism": f"slab{world}" + (f" (virtual {args.virtual} slabs)" if args.virtual else ""),
-                   "l2": ("inputs larger than L2" if 8 * cells > L2_BYTES else "L2-resident (latency config)"),
-                   "tile": {k: desc[k] for k in ("tile_x", "tile_y", "stages", "ctas", "n_top", "n_bot", "k_planes")},
-                   "kernel": kkind,
-                   **({"time_block": {"K": tb_k, "iters_time_blocked": tb_iters,
-                                      "note": "tile above is the per-iteration plan; the time-blocked "
-                                              "kernel's strips/tiles are in DESIGN.md 5.8-5.9"}}
-                      if tb_iters else {})},
-        "gpu_launches": args.steps * world * (2 if 0 < tb_iters < iters else 1),
+        "config": workload_config(cfg, shape, n_gpus, args.virtual),
+        "kernel_config": {"kernel": kkind,
+                          "tile": {k: desc[k] for k in ("tile_x", "tile_y", "stages", "ctas", "n_top", "n_bot",
+                                                        "k_planes")},
+                          **({"time_block": {"K": tb_k, "iters_time_blocked": tb_iters,
+                                             "note": "tile above is the per-iteration plan; the time-blocked "
+                                                     "kernel's strips/tiles are in DESIGN.md 5.8-5.9"}}
+                             if tb_iters else {})},
+        "gpu_launches": launches,
         "wall_ms_per_step": 1e3 * t_wall / args.steps,
         "ms_per_iter": dev_ms / args.steps / iters,
+        "us_per_iter": us_per_iter,
         "roofline": roofline,
         "clocks": clk,
     }
@@ -369,12 +488,12 @@ def main():
                 ms = e0.elapsed_time(e1)
                 best = ms if best is None else min(best, ms)
             box_copy = 2 * a.numel() * a.element_size() / (best / 1e3) / 1e9
-            line["roofline"]["box_copy_gbs"] = box_copy
-            line["roofline"]["frac_of_box_copy"] = line["roofline"]["achieved"] / box_copy
+            if roofline["bound"] == "hbm":
+                line["roofline"]["box_copy_gbs"] = box_copy
+                line["roofline"]["frac_of_box_copy"] = line["roofline"]["achieved"] / box_copy
             del a, b
             torch.cuda.empty_cache()
         except Exception as e:  # never fail the bench line for a context number
-            line["roofline"]["box_copy_gbs"] = None
             print(f"[bench] box copy measurement failed: {e}", file=sys.stderr)
 
         # ---- the per-iteration CPU-Free kernel (one iteration per HBM pass, the paper's Listing
@@ -397,9 +516,13 @@ def main():
         # ---- CPU-controlled baselines (per-iteration launch + copy/NCCL + host sync), short run
         base = {}
         b_iters = min(iters, 200)
-        for name, mode in (("memcpy", jb.MODE_BASELINE_MEMCPY), ("nccl", jb.MODE_BASELINE_NCCL)):
+        bmodes = [("memcpy", jb.MODE_BASELINE_MEMCPY), ("nccl", jb.MODE_BASELINE_NCCL)]
+        if single_multi:
+            bmodes += [("overlap", jb.MODE_BASELINE_OVERLAP), ("p2p", jb.MODE_BASELINE_P2P),
+                       ("graph", jb.MODE_BASELINE_GRAPH)]
+        for name, mode in bmodes:
             if world > 1 and name == "memcpy":
-                continue
+                continue  # host peer copies need one process (dist mode: NCCL)
             try:
                 j.set_mode(mode)
                 j.run(b_iters)  # warm
@@ -412,22 +535,41 @@ def main():
         j.set_mode(jb.MODE_CPUFREE)
         line["cpu_controlled"] = base
 
-        # ---- per-iteration halo latency (no-compute runs): CPU-Free vs NCCL baseline
-        if world > 1:
-            halo = {}
-            for name, mode in (("cpufree", jb.MODE_CPUFREE), ("baseline_nccl", jb.MODE_BASELINE_NCCL)):
-                try:
-                    j.set_mode(mode, jb.FLAG_NO_COMPUTE)
-                    j.run(100)
-                    j.run(200)
-                    t1 = max_over_ranks(j.last_time_ms())
-                    j.run(400)
-                    t2 = max_over_ranks(j.last_time_ms())
-                    halo[name] = 1e3 * (t2 - t1) / 200
-                except jb.JacobiError as e:
-                    halo[name] = {"error": str(e)}
-            j.set_mode(jb.MODE_CPUFREE)
+        # ---- per-iteration halo latency (no-compute runs) and NVLink evidence at N > 1
+        if n_gpus > 1 or args.virtual > 1:
+            hmodes = [("cpufree", jb.MODE_CPUFREE), ("baseline_nccl", jb.MODE_BASELINE_NCCL)]
+            if world == 1:
+                hmodes += [("baseline_memcpy", jb.MODE_BASELINE_MEMCPY), ("baseline_graph", jb.MODE_BASELINE_GRAPH)]
+            halo = halo_latency(j, jb, hmodes, max_over_ranks)
+            nz, ny, nx = shape
+            plane_bytes = 8 * nx * (ny if nz > 1 else 1)  # one halo message = one outer plane
+            sides = 2 if n_gpus > 2 or args.virtual > 2 else 1  # interior GPUs send to both neighbours
+            msg = {"halo_bytes_per_iter_per_gpu_out": sides * plane_bytes,
+                   "halo_bytes_per_iter_per_gpu_in": sides * plane_bytes,
+                   "message_bytes": plane_bytes, "nvlink_peak_gbs_per_direction": 900.0}
+            if isinstance(halo.get("cpufree"), float) and halo["cpufree"] > 0:
+                gbs = sides * plane_bytes / (halo["cpufree"] * 1e-6) / 1e9
+                msg["achieved_gbs_per_direction_nocompute"] = gbs
+                msg["frac_of_nvlink"] = gbs / 900.0
+            if tb_iters == 0 and not resident:
+                # compute runs of the per-iteration kernel deliver one plane per side per iteration
+                gbs = sides * plane_bytes / (1e-3 * launch_ms / iters) / 1e9
+                msg["halo_gbs_during_compute_run"] = gbs
             line["halo_us"] = halo
+            line["halo_traffic"] = msg
+            if args.virtual > 1:
+                line["halo_traffic"]["note"] = "virtual slabs share one GPU: no NVLink traffic"
+            # in-kernel spans of the boundary blocks: the compute run of the timed kernel and a
+            # no-compute run (flag round trip + barrier only)
+            try:
+                n_tr = min(iters, 1024)
+                line["halo_spans_compute"] = traced_spans(j, jb, iters, n_tr, max_over_ranks)
+                j.set_mode(jb.MODE_CPUFREE, jb.FLAG_NO_COMPUTE)
+                line["halo_spans_nocompute"] = traced_spans(j, jb, 400, 400, max_over_ranks)
+                j.set_mode(jb.MODE_CPUFREE)
+            except jb.JacobiError as e:
+                line["halo_spans_compute"] = {"error": str(e)}
+                j.set_mode(jb.MODE_CPUFREE)
         else:
             line["halo_us"] = None  # one slab: no halo; see bench_latency.py (virtual slabs)
 
@@ -447,7 +589,10 @@ def main():
         h_in.numpy()[:] = u12_flat(lo * plane, (hi - lo) * plane, 0x5C24)
         base_in = h_in.data_ptr() - lo * plane * 8
         base_out = h_out.data_ptr() - lo * plane * 8
-        d2h = (chunk + (1 if start == 1 else 0) + (1 if start + chunk == n_out - 1 else 0)) * plane * 8
+        if world > 1:
+            d2h = (chunk + (1 if start == 1 else 0) + (1 if start + chunk == n_out - 1 else 0)) * plane * 8
+        else:
+            d2h = n_out * plane * 8
         jb.jacobi_scatter_ptr(j.h, base_in)
         j.run(iters)
         jb.jacobi_gather_ptr(j.h, base_out)
@@ -459,22 +604,21 @@ def main():
             jb.jacobi_gather_ptr(j.h, base_out)
         barrier()
         e2e_s = max_over_ranks(time.perf_counter() - t0)
-        h2d_total = max_over_ranks(float(nbytes)) if world == 1 else nbytes * world
-        d2h_total = float(d2h) if world == 1 else None
-        if world > 1:
-            d2h_total = max_over_ranks(float(d2h)) * world
+        h2d_total = sum_over_ranks(float(nbytes))
+        d2h_total = sum_over_ranks(float(d2h))
         line["e2e"] = {"value": cells * iters * args.steps / e2e_s / 1e9, "unit": UNIT,
                        "h2d_bytes_per_step": int(h2d_total), "d2h_bytes_per_step": int(d2h_total),
                        "ms_per_step": 1e3 * e2e_s / args.steps,
                        "path": "jacobi_scatter (pinned H2D) + jacobi_run + jacobi_gather (pinned D2H)"}
 
         # ---- CPU oracle on this host's cores (rank 0, N = 1 only), bounded sample
-        if rank == 0 and world == 1:
+        if rank == 0 and n_gpus == 1:
             field = h_in.numpy().reshape(shape if nz > 1 else shape[1:])
             v1, dt1, cores = oracle_sample(shape, 1, field=field)
             k = int(max(1, min(50, 10.0 / max(dt1, 1e-3))))
             v, dt, cores = oracle_sample(shape, k, field=field)
-            line["cpu_baseline"] = {"value": v, "unit": UNIT, "cores": cores, "kind": "oracle",
+            line["cpu_baseline"] = {"value": v, "unit": UNIT, "cores": cores, "cpu_model": cpu_model(),
+                                    "kind": "oracle",
                                     "sample": f"{k} of {iters} iterations on the full grid "
                                               f"({dt:.1f} s, OpenMP over the outer axis)"}
     if rank == 0:

@@ -142,9 +142,18 @@ int jacobi_create_nvshmem(int64_t nx, int64_t ny, int64_t nz, int stencil, const
 int jacobi_nvshmem_finalize(void);
 
 /* ---- running ----------------------------------------------------------------------------- */
-/* Advance the field by `iters` Jacobi iterations in the current mode.  Continues from the
- * current state: run(a); run(b) == run(a+b) bitwise.  run(0) is a no-op.  Blocks until done. */
+/* Advance the field by `iters` Jacobi iterations in the current mode (the fixed iteration count
+ * of P:355, Listing 4.1 "for (iter = 0; iter < iter_max; ...)").  CPU-Free mode: ONE persistent
+ * cooperative launch per GPU for all `iters` (§3.1.1, §4.1.1) — the only host
+ * action of the run; baseline modes: one host-driven launch + halo copy +
+ * host sync per iteration (Listing 2.1a).  Continues from the current state:
+ * run(a); run(b) == run(a+b) bitwise (every iteration reads only the previous time step).
+ * run(0) is a no-op.  iters < 0: JACOBI_EINVAL; peers not attached (dist mode): JACOBI_ESTATE;
+ * a neighbour that never signals: JACOBI_ETIMEOUT (watchdog, field undefined).  Blocks until done. */
 int jacobi_run(jacobi_t h, int64_t iters);
+/* Select how later runs are orchestrated (JACOBI_MODE_*, the paper's CPU-Free model vs the
+ * CPU-controlled baselines of P:528-531) and measurement flags (JACOBI_FLAG_*, the no-compute
+ * runs of P:550-552).  Unknown mode / flag bits: JACOBI_EINVAL.  Collective in dist mode. */
 int jacobi_set_mode(jacobi_t h, int mode, int flags);
 /* Tuning knobs (none changes results): "tile_x", "tile_y", "stages", "boundary_ctas",
  * "ctas" (persistent grid size per slab group, 0 = all co-resident), "schedule" (interior
@@ -163,7 +172,7 @@ int jacobi_set_mode(jacobi_t h, int mode, int flags);
  * -1 auto (default: 2D runs, not when the slab fits on chip, where the resident kernel is used),
  * 0 never, 1 always incl. 3D (EINVAL when a slab has < 4 planes with P > 1, with the norm, in
  * no-compute mode or in the NVSHMEM variant)), "tb_k" (iterations per time block: -1 auto = 5 in
- * 2D, 2 in 3D; 2D accepts 2, 3, 5 — a deeper K than the slabs fit falls back to 3, then 2),
+ * 2D, 3 in 3D; 2D accepts 2, 3, 5, 3D 2, 3 — a deeper K than the slabs fit falls back to 3, then 2),
  * "tb_ppt" (2D cell pairs per lane and level: K = 2: from tile_x; K = 3: 2 or 4; K = 5: 1 (default,
  * 11 consumer warps) or 2 (7 warps); 3D K = 3: 1 (default) or 2), "tb_rpw" (3D K = 3: rows per
  * warp, 2 (default, 11 warps) or 3 (7 warps)),
@@ -171,7 +180,9 @@ int jacobi_set_mode(jacobi_t h, int mode, int flags);
  * dynamic plane block of that kernel, default 16), "tb_ctas" (its CTAs per SM, 1 or 2; 2 only
  * for K = 2 and P = 1).  Read-only: "last_resident" (1 if the last CPU-Free run used the resident
  * kernel), "last_tblock" (iterations of the last CPU-Free run done time-blocked), "last_tb_k"
- * (its K, 0 if none).  Unknown names return JACOBI_EINVAL. */
+ * (its K, 0 if none), "last_launches" (kernels this process launched in the last jacobi_run, all
+ * GPUs).  Measurement: "halo_trace" (see jacobi_halo_trace; 0 = off, <= 2^20).
+ * Unknown names return JACOBI_EINVAL. */
 int jacobi_set_param(jacobi_t h, const char *name, int64_t value);
 int jacobi_get_param(jacobi_t h, const char *name, int64_t *value);
 
@@ -187,17 +198,38 @@ int jacobi_set_tolerance(jacobi_t h, double tol);
 int jacobi_last_norm(jacobi_t h, double *norm);
 
 /* ---- data movement -------------------------------------------------------------------- */
-/* Set the whole field (boundary included) from a host array of nx*ny*nz doubles; both
- * device buffers are written.  In dist mode only this rank's slab (+ its halos) is read. */
+/* Set the whole field (boundary included: the Dirichlet data of P:197 is whatever the caller's
+ * boundary cells hold) from a caller-owned host array `in` of nx*ny*nz doubles (layout above);
+ * both device buffers are written (R10), each slab receives its owned planes plus one
+ * halo plane per side.  In dist mode only this rank's slab (+ its halos) is read.
+ * `in` NULL: JACOBI_EINVAL.  Synchronous (returns after the copies completed). */
 int jacobi_scatter(jacobi_t h, const double *in);
-/* Write the current field into a host array of nx*ny*nz doubles.  In dist mode only this
- * rank's owned planes (and the global boundary planes it holds) are written. */
+/* Write the current field (buf[t & 1], the result of the last completed iteration) into a
+ * caller-owned host array `out` of nx*ny*nz doubles (layout above): every slab's owned planes, and
+ * the global boundary planes from the first / last slab.  In dist mode only this rank's owned
+ * planes (and the global boundary planes it holds) are written; the rest of `out` is untouched.
+ * `out` NULL: JACOBI_EINVAL.  Synchronous. */
 int jacobi_gather(jacobi_t h, double *out);
 
 /* ---- introspection ---------------------------------------------------------------------- */
-/* Device time of the last jacobi_run: max over GPUs and, if ms_per_slab != NULL, one entry
- * per local slab (CUDA events on each GPU's launch stream around the launch(es)). */
+/* Device time of the last jacobi_run (the quantity behind the paper's timing method, "minimum
+ * of 5 runs", and SURVEY §8(d)): max over this process's GPUs into *ms_max and, if
+ * ms_per_slab != NULL (caller array of one double per LOCAL slab), one entry per slab.  CUDA
+ * events on each GPU's launch stream around the launch(es) — the persistent kernel in CPU-Free
+ * mode, the whole host loop in the baseline modes (host overhead shows as GPU idle time).
+ * Multi-process: the caller takes the max over ranks.  h NULL: JACOBI_EINVAL. */
 int jacobi_last_time(jacobi_t h, double *ms_max, double *ms_per_slab);
+/* Halo-exchange trace of the last CPU-Free run (measurement of P:394's wait -> compute + put ->
+ * signal sequence and of the per-iteration halo latency): with the knob "halo_trace"
+ * = n > 0, the first boundary thread block of each side of every slab records %globaltimer (ns,
+ * per-GPU clock) for the first n exchanges of a run (one exchange = one iteration; the
+ * time-blocked kernel's K phases per block are K exchanges): [0] the wait for the neighbour's
+ * flag begins, [1] the flag was acquired, [2] this block's own signal was released.  Copies 2 x n
+ * x 3 uint64 into `out` (caller-owned): side 0 (top) exchanges 0..n-1, then side 1 (bottom); zero
+ * where nothing was recorded (no neighbour on that side, or the event did not happen — e.g. no
+ * wait before iteration 0 of the resident kernel).  n larger than the last traced run recorded:
+ * JACOBI_ESTATE; bad slab index / NULL: JACOBI_EINVAL. */
+int jacobi_halo_trace(jacobi_t h, int slab, uint64_t *out, int64_t n);
 int jacobi_iterations(jacobi_t h, int64_t *t);          /* global iteration counter */
 int jacobi_num_slabs(jacobi_t h, int *local, int *total);
 /* Plan of local slab `i`: out[0..15] = start, chunk, pitch, plane_elems, tile_x, tile_y,
@@ -207,8 +239,13 @@ int jacobi_describe(jacobi_t h, int i, int64_t *out16);
  * planes of plane_elems doubles, halos included) into a caller array of
  * (chunk+2)*plane_elems doubles — for tests of the halo protocol. */
 int jacobi_read_slab(jacobi_t h, int i, int parity, double *out);
+/* Static English text of a JACOBI_* code ("unknown error" otherwise); never NULL. */
 const char *jacobi_strerror(int code);
-int jacobi_destroy(jacobi_t h);                         /* NULL-safe */
+/* Release everything the handle owns: waits for its streams, frees the slab buffers, control
+ * blocks, peer / IPC mappings, NCCL communicators and cached graphs (the halos and
+ * flags of P:394 live in those buffers).  NULL-safe (returns JACOBI_OK); valid after any error.
+ * NVSHMEM handles: collective.  The handle must not be used afterwards. */
+int jacobi_destroy(jacobi_t h);
 
 /* ---- host-only helpers (no GPU needed) ---------------------------------------------------- */
 /* Slab decomposition of the interior outer indices 1..n_out-2 into nslabs chunks: with

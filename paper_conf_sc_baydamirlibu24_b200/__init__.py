@@ -74,6 +74,7 @@ _SIGS = {
     "jacobi_last_norm": ([_p, _c.POINTER(_c.c_double)], _c.c_int),
     "jacobi_slab_bytes": ([_i64, _i64, _i64, _c.c_int, _c.c_int, _c.c_int, _c.POINTER(_i64)], _c.c_int),
     "jacobi_read_slab": ([_p, _c.c_int, _c.c_int, _p], _c.c_int),
+    "jacobi_halo_trace": ([_p, _c.c_int, _p, _i64], _c.c_int),
 }
 # exported only by the NVSHMEM variant (libjacobi_b200_nvshmem.so)
 _SIGS_NVSHMEM = {
@@ -243,6 +244,39 @@ def jacobi_last_time(h, nslabs: int):
     per = (_c.c_double * max(nslabs, 1))()
     _check(lib().jacobi_last_time(h, _c.byref(mx), per), "jacobi_last_time")
     return mx.value, list(per)[:nslabs]
+
+
+def jacobi_halo_trace(h, slab: int, n: int) -> np.ndarray:
+    """Raw halo-exchange trace of the last CPU-Free run: uint64 array [2 sides][n exchanges][3]
+    (%globaltimer ns at wait begin / flag acquired / signal released; 0 = not recorded)."""
+    out = np.zeros((2, n, 3), dtype=np.uint64)
+    _check(lib().jacobi_halo_trace(h, int(slab), out.ctypes.data, int(n)), "jacobi_halo_trace")
+    return out
+
+
+def halo_spans(trace: np.ndarray, skip: int = 0) -> dict:
+    """Summary (median µs over exchanges >= skip, both sides) of a jacobi_halo_trace array:
+    wait = flag acquired - wait begin, put = signal - flag acquired (edge plane compute + peer
+    stores + release), span = signal - wait begin (the boundary block's whole exchange), period =
+    time between consecutive signals of a side (the per-iteration halo cadence)."""
+    t = trace.astype(np.int64)
+    out = {}
+    for key, (i, j) in {"wait_us": (0, 1), "put_us": (1, 2), "span_us": (0, 2)}.items():
+        v = []
+        for side in range(2):
+            a, b = t[side, skip:, i], t[side, skip:, j]
+            m = (a > 0) & (b > 0)
+            v.extend(((b[m] - a[m]) / 1e3).tolist())
+        out[key] = float(np.median(v)) if v else None
+    per = []
+    for side in range(2):
+        sg = t[side, skip:, 2]
+        sg = sg[sg > 0]
+        if len(sg) > 1:
+            per.extend((np.diff(sg) / 1e3).tolist())
+    out["period_us"] = float(np.median(per)) if per else None
+    out["exchanges"] = int(((t[:, skip:, 2] > 0)).sum())
+    return out
 
 
 def jacobi_iterations(h) -> int:
@@ -419,6 +453,9 @@ class Jacobi:
 
     def describe(self, i: int = 0) -> dict:
         return jacobi_describe(self.h, i)
+
+    def halo_trace(self, slab: int, n: int) -> np.ndarray:
+        return jacobi_halo_trace(self.h, slab, n)
 
     def close(self) -> None:
         if getattr(self, "h", None):

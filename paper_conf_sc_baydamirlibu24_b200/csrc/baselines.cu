@@ -59,6 +59,7 @@ int time_end(jacobi_ctx *h, int64_t iters) {
   for (auto &s : h->slabs) {
     CK(cudaSetDevice(s.device));
     CK(jbk::launch_flag_max(&s.ctrl->flag_in[0][0], 2 * JB_MAXK, (unsigned long long)h->t, s.stream));
+    ++h->last_launches;
     CK(cudaStreamSynchronize(s.stream));
   }
   return JACOBI_OK;
@@ -106,6 +107,7 @@ int nccl_edges(jacobi_ctx *h, int nxt) {
 int run_graph(jacobi_ctx *h, int64_t iters, bool nocomp, std::vector<LaunchPlan> &plans);
 
 int run_baseline(jacobi_ctx *h, int64_t iters, BaseKind kind) {
+  h->last_launches = 0;
   const bool nocomp = h->flags & JACOBI_FLAG_NO_COMPUTE;
   if (kind == BK_NCCL) {
     int rc = ensure_nccl(h);
@@ -151,8 +153,10 @@ int run_baseline(jacobi_ctx *h, int64_t iters, BaseKind kind) {
         if (!nocomp) {
           edges[i].P.t0 = tg;
           CK(jbk::launch_sweep(edges[i].P, false, false, edges[i].grid, edges[i].smem, s.stream2));
+          ++h->last_launches;
           plans[i].P.t0 = tg;
           CK(jbk::launch_sweep(plans[i].P, false, false, plans[i].grid, plans[i].smem, s.stream));
+          ++h->last_launches;
         }
         rc = copy_edges(h, s, nxt, s.stream2);
         if (rc) return rc;
@@ -161,6 +165,7 @@ int run_baseline(jacobi_ctx *h, int64_t iters, BaseKind kind) {
       if (launch_kernels) {
         plans[i].P.t0 = tg;
         CK(jbk::launch_sweep(plans[i].P, nocomp, false, plans[i].grid, plans[i].smem, s.stream));
+        ++h->last_launches;
       }
     }
     if (kind == BK_COPY) {  // ④ write_neighbors with host-issued peer copies
@@ -179,6 +184,7 @@ int run_baseline(jacobi_ctx *h, int64_t iters, BaseKind kind) {
         Slab &s = h->slabs[i];
         CK(cudaSetDevice(s.device));
         CK(jbk::launch_neighbour_wait(plans[i].P, (unsigned long long)(tg + 1), s.stream));
+        ++h->last_launches;
       }
       continue;
     }
@@ -252,6 +258,7 @@ int run_graph(jacobi_ctx *h, int64_t iters, bool nocomp, std::vector<LaunchPlan>
   Slab &m = h->slabs[0];
   CK(cudaSetDevice(m.device));
   CK(cudaGraphLaunch(h->graph_exec, m.stream));
+  h->last_launches += nocomp ? 0 : iters * n;  // the graph's kernel nodes
   CK(cudaStreamSynchronize(m.stream));
   return time_end(h, iters);
 }

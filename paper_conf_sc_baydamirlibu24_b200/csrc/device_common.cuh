@@ -186,6 +186,13 @@ __device__ bool wait_slots_idx(const unsigned long long *flags, const int *idx, 
   }
 }
 
+// Halo-exchange trace (measurement only, JbSlab::halo_trace): exchange e of side `side` (0 top,
+// 1 bottom), event `which` (0 wait begins, 1 neighbour's flag acquired, 2 own signal released).
+__device__ __forceinline__ void halo_mark(const JbSlab &SL, const JbParams &P, int side, int64_t e, int which) {
+  if (SL.halo_trace && e >= 0 && e < P.halo_trace_n)
+    SL.halo_trace[((int64_t)side * P.halo_trace_n + e) * 3 + which] = globaltimer();
+}
+
 // Position in the shared-memory ring: slot and the parity of the current use of that slot.
 struct RingPos {
   uint32_t slot, phase;

@@ -112,6 +112,10 @@ struct JbSlab {
   double *mid_top_out;
   double *mid_bot_out;
   const void *tmap;                  // 3D odd-K time-blocked kernel: CUtensorMap[2] (buf[0], buf[1]) or null
+  // Halo-exchange trace (measurement, param halo_trace = n > 0): for the first n exchanges of a run
+  // the first boundary CTA of each side records %globaltimer at wait begin / flag acquired /
+  // signal released: halo_trace[(side * n + e) * 3 + {0, 1, 2}], side 0 = top, 1 = bottom.
+  unsigned long long *halo_trace;
 };
 
 struct JbParams {
@@ -125,7 +129,7 @@ struct JbParams {
   int *status;      // [0] error code (0 ok), [1] abort flag
   unsigned long long *trace;  // debug (JACOBI_TRACE): per-iteration CTA work-end timestamps, or null
   int32_t norm_every;         // N4: check the update norm after every norm_every-th iteration (0: off)
-  int32_t pad;
+  int32_t halo_trace_n;       // exchanges recorded per side in JbSlab::halo_trace (0: off)
   double tol;                 // stop after the first check with norm <= tol
   int64_t k0;                 // global number of norm checks before this launch (monotone slots)
 };

@@ -125,12 +125,20 @@ __global__ void __launch_bounds__(JB_RNT, 1) jb_resident(const __grid_constant__
     // (1) halo: wait for the neighbour GPU's edge plane (and, with relaxed sync, for the
     //     neighbour blocks' faces of the previous iteration), then refresh the ring from L2
     if (t > 0 && (top_blk || bot_blk || relaxed)) {
+      if (tid == 0 && by == 0) {
+        if (top_blk) halo_mark(SL, P, 0, t, 0);
+        if (bot_blk) halo_mark(SL, P, 1, t, 0);
+      }
       if (tid < 32) {
         bool ok = true;
         if (top_blk) ok &= wait_slots(SL.flag_in_top, SL.k_in_top, (unsigned long long)tg, P, tid);
         if (bot_blk) ok &= wait_slots(SL.flag_in_bot, SL.k_in_bot, (unsigned long long)tg, P, tid);
         if (relaxed) ok &= wait_slots_idx(SL.blk_flags, nbr, n_nbr, (unsigned long long)tg, P, tid);
         if (tid == 0 && !ok) s_abort = 1;
+        if (tid == 0 && by == 0) {
+          if (top_blk) halo_mark(SL, P, 0, t, 1);
+          if (bot_blk) halo_mark(SL, P, 1, t, 1);
+        }
       }
       __syncthreads();
       if (s_abort) return;
@@ -186,6 +194,10 @@ __global__ void __launch_bounds__(JB_RNT, 1) jb_resident(const __grid_constant__
       if (tid == 0 && !((P.flags & JACOBI_FLAG_DROP_SIGNAL) && SL.slab_id == 0)) {
         if (top_blk) st_release_sys(SL.flag_out_top + by, (unsigned long long)(tg + 1));
         if (bot_blk) st_release_sys(SL.flag_out_bot + by, (unsigned long long)(tg + 1));
+        if (by == 0) {
+          if (top_blk) halo_mark(SL, P, 0, t, 2);
+          if (bot_blk) halo_mark(SL, P, 1, t, 2);
+        }
       }
     }
     // (4) grid barrier of the slab, or with relaxed sync only a release of this block's

@@ -75,11 +75,13 @@ void free_slab(Slab &s, const Allocator &a) {
     if (a.free) a.free(p, s.device, a.user);
     else if (!a.alloc) cudaFree(p);
   }
-  if (s.dyn_table) cudaFree(s.dyn_table);
+  for (auto &t : s.tabs)
+    if (t.ptr) cudaFree(t.ptr);
   if (s.blk_flags) cudaFree(s.blk_flags);
   if (s.partials) cudaFree(s.partials);
   if (s.norm_peers) cudaFree(s.norm_peers);
   if (s.tmap) cudaFree(s.tmap);
+  if (s.trace) cudaFree(s.trace);
   if (s.ev0) cudaEventDestroy(s.ev0);
   if (s.ev1) cudaEventDestroy(s.ev1);
   if (s.ev_sync) cudaEventDestroy(s.ev_sync);
@@ -153,17 +155,33 @@ int slab_tensor_maps(jacobi_ctx *h, Slab &s, int cols, int rows) {
   return JACOBI_OK;
 }
 
-// Device copy of the guided-schedule block table of a slab (rebuilt when its key changes).
+// Device copy of the guided-schedule block table of a slab.  Two cached entries (LRU): a
+// time-blocked run plans the per-iteration launch too, so the two tables alternate within every
+// jacobi_run; rebuilding them each time cost a cudaFree (an implicit device sync) + cudaMalloc
+// per run.  An evicted entry's allocation is reused when it is large enough.
 int upload_table(Slab &s, int64_t npl, int units, int n, int min_blk, int64_t nb) {
   const int64_t key[4] = {npl, units, n, min_blk};
-  if (s.dyn_table && std::memcmp(key, s.dyn_key, sizeof(key)) == 0) return JACOBI_OK;
+  ++s.tab_clock;
+  for (auto &t : s.tabs)
+    if (t.ptr && std::memcmp(key, t.key, sizeof(key)) == 0) {
+      t.used = s.tab_clock;
+      s.dyn_table = t.ptr;
+      return JACOBI_OK;
+    }
+  auto &t = s.tabs[0].used <= s.tabs[1].used ? s.tabs[0] : s.tabs[1];
   std::vector<int32_t> tab(nb + 1);
   jbplan::dyn_blocks(npl, units, n, min_blk, tab.data());
-  if (s.dyn_table) cudaFree(s.dyn_table);
-  s.dyn_table = nullptr;
-  CK(cudaMalloc(&s.dyn_table, tab.size() * sizeof(int32_t)));
-  CK(cudaMemcpy(s.dyn_table, tab.data(), tab.size() * sizeof(int32_t), cudaMemcpyHostToDevice));
-  std::memcpy(s.dyn_key, key, sizeof(key));
+  if (t.cap < nb + 1) {
+    if (t.ptr) cudaFree(t.ptr);
+    t.ptr = nullptr;
+    t.cap = 0;
+    CK(cudaMalloc(&t.ptr, tab.size() * sizeof(int32_t)));
+    t.cap = nb + 1;
+  }
+  CK(cudaMemcpy(t.ptr, tab.data(), tab.size() * sizeof(int32_t), cudaMemcpyHostToDevice));
+  std::memcpy(t.key, key, sizeof(key));
+  t.used = s.tab_clock;
+  s.dyn_table = t.ptr;
   return JACOBI_OK;
 }
 
@@ -452,9 +470,42 @@ int plan_resident(jacobi_ctx *h, const std::vector<int> &idx, LaunchPlan &L) {
   return JACOBI_OK;
 }
 
+// Whether EVERY slab of the run (all ids 0..total-1, not only this process's) fits the resident
+// kernel.  One process per GPU decides on its own, so the choice must be a deterministic function
+// of the global problem: a rank picking the resident kernel while its neighbour streams would
+// disagree on the flag slots and their meaning (per iteration vs per phase).  Same inputs as
+// plan_resident (decompose, resident_tiling with the slab's CTA count, the 2^31 element limit,
+// occupancy of the chosen variant); ranks run on equal GPUs (SM count checked in the IPC blob).
+bool resident_fits_all(jacobi_ctx *h) {
+  const int dev = h->slabs[0].device;
+  if (cudaSetDevice(dev) != cudaSuccess) return false;
+  int sms = 0, smem_optin = 0;
+  if (cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev) != cudaSuccess) return false;
+  if (cudaDeviceGetAttribute(&smem_optin, cudaDevAttrMaxSharedMemoryPerBlockOptin, dev) != cudaSuccess) return false;
+  smem_optin = std::min(smem_optin, JB_SMEM_DEFAULT) - 1024;
+  int64_t group_ctas = 0;
+  for (int id = 0; id < h->total; ++id) {
+    int64_t st, ch;
+    jbplan::decompose(h->n_out, h->total, id, &st, &ch);
+    if ((ch + 3) * h->geom.plane_elems >= ((int64_t)1 << 31)) return false;
+    int nbz, nby, cpp;
+    size_t sm;
+    if (jbplan::resident_tiling(h->nx, h->ny, h->dim, ch, slab_ctas(h, id, sms), smem_optin, &nbz, &nby, &cpp, &sm))
+      return false;
+    int occ = 0;
+    if (jbk::prepare_resident(h->dim, cpp, sm, &occ) != cudaSuccess || occ < 1) return false;
+    if (h->block_sync && nbz * nby > JB_MAX_BLOCKS) return false;
+    group_ctas = h->kind == KIND_VIRTUAL ? group_ctas + nbz * nby : nbz * nby;
+    if (group_ctas > (int64_t)sms * occ) return false;
+  }
+  return true;
+}
+
 // N4: wire the residual-norm all-reduce into a planned launch (partials + every slab's ctrl).
 int setup_norm(jacobi_ctx *h, LaunchPlan &L) {
   if (h->total > 32) return JACOBI_EINVAL;  // one polling lane per slab
+  // every slab stores its sum into every other slab's control block: all pairs must be mapped
+  if (h->kind == KIND_SINGLE && !h->all_peers) return JACOBI_ENOPEER;
   for (size_t k = 0; k < L.slab_idx.size(); ++k) {
     Slab &s = h->slabs[L.slab_idx[k]];
     JbSlab &d = L.P.s[k];
@@ -487,6 +538,30 @@ int setup_norm(jacobi_ctx *h, LaunchPlan &L) {
   return JACOBI_OK;
 }
 
+// Halo-exchange trace (param halo_trace = n): a zeroed per-slab buffer of 2 sides x n exchanges
+// x 3 timestamps, wired into a planned CPU-Free launch (streaming, resident or time-blocked).
+int setup_trace(jacobi_ctx *h, LaunchPlan &L) {
+  const int64_t n = h->halo_trace;
+  L.P.halo_trace_n = (int32_t)n;
+  for (size_t k = 0; k < L.slab_idx.size(); ++k) {
+    Slab &s = h->slabs[L.slab_idx[k]];
+    L.P.s[k].halo_trace = nullptr;
+    if (n <= 0) continue;
+    CK(cudaSetDevice(s.device));
+    if (s.trace_cap < n) {
+      if (s.trace) cudaFree(s.trace);
+      s.trace = nullptr;
+      s.trace_cap = 0;
+      CK(cudaMalloc(&s.trace, (size_t)n * 6 * sizeof(unsigned long long)));
+      s.trace_cap = n;
+    }
+    CK(cudaMemsetAsync(s.trace, 0, (size_t)n * 6 * sizeof(unsigned long long), L.stream));
+    s.trace_n = n;
+    L.P.s[k].halo_trace = s.trace;
+  }
+  return JACOBI_OK;
+}
+
 int run_cpufree_k1(jacobi_ctx *h, int64_t iters) {
   const bool nocomp = h->flags & JACOBI_FLAG_NO_COMPUTE;
   const bool norm = !nocomp && h->norm_every > 0;
@@ -494,6 +569,10 @@ int run_cpufree_k1(jacobi_ctx *h, int64_t iters) {
   std::vector<LaunchPlan> plans(groups.size());
   // Resident (on-chip) kernel when every slab fits (auto) or when forced (not with the norm).
   bool resident = !nocomp && !norm && h->resident != 0 && h->kind != KIND_SHMEM;
+  if (resident && !resident_fits_all(h)) {
+    if (h->resident == 1) return JACOBI_EINVAL;
+    resident = false;
+  }
   if (resident) {
     for (size_t i = 0; i < groups.size() && resident; ++i)
       if (plan_resident(h, groups[i], plans[i]) != JACOBI_OK) resident = false;
@@ -513,6 +592,10 @@ int run_cpufree_k1(jacobi_ctx *h, int64_t iters) {
     plans[i].P.t0 = h->t;
     plans[i].P.iters = iters;
   }
+  for (auto &L : plans) {
+    int rc = setup_trace(h, L);
+    if (rc) return rc;
+  }
   // Reset per-run counters (barrier, status, claim counters).  Flags are monotonic across runs:
   // raise every inbound slot to the current iteration (atomicMax: a neighbour that already
   // signalled this run is kept), so slots unused by an earlier split never hold stale values.
@@ -522,7 +605,11 @@ int run_cpufree_k1(jacobi_ctx *h, int64_t iters) {
       Slab &s = h->slabs[k];
       CK(reset_run_counters(s, L.stream));
       CK(jbk::launch_flag_max(&s.ctrl->flag_in[0][0], 2 * JB_MAXK, (unsigned long long)h->t, L.stream));
-      if (s.blk_flags) CK(jbk::launch_flag_max(s.blk_flags, JB_MAX_BLOCKS, (unsigned long long)h->t, L.stream));
+      ++h->last_launches;
+      if (s.blk_flags) {
+        CK(jbk::launch_flag_max(s.blk_flags, JB_MAX_BLOCKS, (unsigned long long)h->t, L.stream));
+        ++h->last_launches;
+      }
     }
   }
   // Debug: JACOBI_TRACE=1 records when each CTA finished its work in the first 8 iterations.
@@ -541,6 +628,7 @@ int run_cpufree_k1(jacobi_ctx *h, int64_t iters) {
     CK(cudaEventRecord(s0.ev0, L.stream));
     if (resident) CK(jbk::launch_resident(L.P, L.cpp, L.grid, L.smem, L.stream));
     else CK(jbk::launch_sweep(L.P, nocomp, true, L.grid, L.smem, L.stream));
+    ++h->last_launches;
     CK(cudaEventRecord(s0.ev1, L.stream));
   }
   int rc_all = JACOBI_OK;
@@ -723,6 +811,10 @@ int run_tblock(jacobi_ctx *h, int64_t iters, int K, int ppt, int lag) {
     L.P.t0 = h->t;
     L.P.iters = iters;
   }
+  for (auto &L : plans) {
+    int rc = setup_trace(h, L);
+    if (rc) return rc;
+  }
   // per-run counters; flags raised to the current iteration (as run_cpufree_k1)
   for (auto &L : plans) {
     CK(cudaSetDevice(L.device));
@@ -730,6 +822,7 @@ int run_tblock(jacobi_ctx *h, int64_t iters, int K, int ppt, int lag) {
       Slab &s = h->slabs[k];
       CK(reset_run_counters(s, L.stream));
       CK(jbk::launch_flag_max(&s.ctrl->flag_in[0][0], 2 * JB_MAXK, (unsigned long long)h->t, L.stream));
+      ++h->last_launches;
     }
   }
   for (auto &L : plans) {
@@ -737,6 +830,7 @@ int run_tblock(jacobi_ctx *h, int64_t iters, int K, int ppt, int lag) {
     Slab &s0 = h->slabs[L.slab_idx[0]];
     CK(cudaEventRecord(s0.ev0, L.stream));
     CK(jbk::launch_tblock(L.P, K, ppt, lag, per_sm, L.grid, L.smem, L.stream));
+    ++h->last_launches;
     CK(cudaEventRecord(s0.ev1, L.stream));
   }
   int rc_all = JACOBI_OK;
@@ -762,6 +856,7 @@ int run_tblock(jacobi_ctx *h, int64_t iters, int K, int ppt, int lag) {
 // the run is eligible (one slab without neighbours, 2D, compute, no norm, not on-chip resident),
 // the per-iteration kernels (streaming / resident) for the rest.  Device times add up.
 int run_cpufree(jacobi_ctx *h, int64_t iters) {
+  h->last_launches = 0;
   h->last_tblock = 0;
   h->last_tb_k = 0;
   h->last_resident = 0;
@@ -779,15 +874,9 @@ int run_cpufree(jacobi_ctx *h, int64_t iters) {
     // odd K: any block count; K = 2: an even one (the result stays in buf[t & 1], R10)
     const int64_t step = (K & 1) ? K : 2 * K;
     tb_iters = iters / step * step;
-    if (h->tblock < 0 && h->resident != 0) {
-      // auto: slabs that fit on chip run the resident kernel (faster for those small grids)
-      bool fits = true;
-      for (auto &grp : launch_groups(h)) {
-        LaunchPlan R;
-        if (plan_resident(h, grp, R) != JACOBI_OK) fits = false;
-      }
-      if (fits) tb_iters = 0;
-    }
+    // auto: slabs that fit on chip run the resident kernel (faster for those small grids);
+    // decided over every slab of the run so that all ranks take the same kernel
+    if (h->tblock < 0 && h->resident != 0 && resident_fits_all(h)) tb_iters = 0;
   }
   double ms = 0;
   if (tb_iters > 0) {
@@ -839,11 +928,14 @@ int jacobi_create(int64_t nx, int64_t ny, int64_t nz, int stencil, int ngpus, ja
       if (o == g) continue;
       int can = 0;
       cudaDeviceCanAccessPeer(&can, g, o);
-      if (!can) continue;
+      if (!can) {
+        h->all_peers = false;  // neighbours were checked above; only the norm needs this pair
+        continue;
+      }
       cudaError_t e = cudaDeviceEnablePeerAccess(o, 0);
       if (e == cudaErrorPeerAccessAlreadyEnabled) cudaGetLastError();
       else if (e != cudaSuccess && (o == g - 1 || o == g + 1)) { jacobi_destroy(h); return JACOBI_ENOPEER; }
-      else if (e != cudaSuccess) cudaGetLastError();
+      else if (e != cudaSuccess) { cudaGetLastError(); h->all_peers = false; }
     }
   }
   link_local(h);
@@ -929,18 +1021,22 @@ static int64_t *param_slot(jacobi_t h, const char *name) {
   if (!std::strcmp(name, "tb_rpw")) return &h->tb_rpw;
   if (!std::strcmp(name, "last_tb_k")) return &h->last_tb_k;
   if (!std::strcmp(name, "last_tblock")) return &h->last_tblock;
+  if (!std::strcmp(name, "halo_trace")) return &h->halo_trace;
+  if (!std::strcmp(name, "last_launches")) return &h->last_launches;
   return nullptr;
 }
 
 int jacobi_set_param(jacobi_t h, const char *name, int64_t value) {
   if (!h || !name) return JACOBI_EINVAL;
-  if (!std::strcmp(name, "last_resident") || !std::strcmp(name, "last_tblock") || !std::strcmp(name, "last_tb_k"))
+  if (!std::strcmp(name, "last_resident") || !std::strcmp(name, "last_tblock") || !std::strcmp(name, "last_tb_k") ||
+      !std::strcmp(name, "last_launches"))
     return JACOBI_EINVAL;  // read-only
   int64_t *p = param_slot(h, name);
   if (!p) return JACOBI_EINVAL;
   if (!std::strcmp(name, "timeout_ms")) value = value < 0 ? 20000 : value;
   if (!std::strcmp(name, "tile_x") && value > 4096) return JACOBI_EINVAL;
   if (!std::strcmp(name, "tile_y") && value > 30) return JACOBI_EINVAL;
+  if (!std::strcmp(name, "halo_trace") && (value < 0 || value > (1 << 20))) return JACOBI_EINVAL;
   *p = value;
   h->plan_gen++;
   return JACOBI_OK;
@@ -1024,6 +1120,19 @@ int jacobi_last_time(jacobi_t h, double *ms_max, double *ms_per_slab) {
   if (ms_max) *ms_max = h->last_ms_max;
   if (ms_per_slab)
     for (size_t i = 0; i < h->slabs.size(); ++i) ms_per_slab[i] = h->slabs[i].last_ms;
+  return JACOBI_OK;
+}
+
+int jacobi_halo_trace(jacobi_t h, int slab, uint64_t *out, int64_t n) {
+  if (!h || !out || slab < 0 || slab >= (int)h->slabs.size() || n < 0) return JACOBI_EINVAL;
+  Slab &s = h->slabs[slab];
+  if (n > s.trace_n || !s.trace) return JACOBI_ESTATE;  // no traced run of that length yet
+  CK(cudaSetDevice(s.device));
+  CK(cudaStreamSynchronize(s.stream));
+  // the last run laid the buffer out for trace_n exchanges per side: copy each side's first n
+  for (int side = 0; side < 2; ++side)
+    CK(cudaMemcpy(out + (size_t)side * n * 3, s.trace + (size_t)side * s.trace_n * 3, (size_t)n * 3 * 8,
+                  cudaMemcpyDeviceToHost));
   return JACOBI_OK;
 }
 

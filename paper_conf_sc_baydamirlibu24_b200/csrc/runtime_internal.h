@@ -141,12 +141,21 @@ struct Slab {
   ncclComm_t comm = nullptr;
   double last_ms = 0;
   JbSlab desc{};  // last launch descriptor (for jacobi_describe)
-  int32_t *dyn_table = nullptr;  // guided-schedule block table (device)
+  int32_t *dyn_table = nullptr;  // guided-schedule block table of the last plan (device; one of tabs)
+  struct DynTab {                // cached tables: the per-iteration and the time-blocked plan alternate
+    int32_t *ptr = nullptr;      // within one jacobi_run, so two entries keep both resident
+    int64_t cap = 0;             // entries allocated
+    int64_t key[4] = {0, 0, 0, 0};
+    uint64_t used = 0;           // LRU stamp
+  } tabs[2];
+  uint64_t tab_clock = 0;
   unsigned long long *blk_flags = nullptr;  // resident kernel: per-block flags (device)
   double *partials = nullptr;               // N4: per-run partial sums (device)
   int64_t partials_cap = 0;
   JbCtrl **norm_peers = nullptr;            // N4: device array of every slab's control block
-  int64_t dyn_key[4] = {0, 0, 0, 0};
+  unsigned long long *trace = nullptr;  // halo-exchange trace of the last CPU-Free run (device)
+  int64_t trace_cap = 0;                // its capacity (exchanges per side)
+  int64_t trace_n = 0;                  // exchanges per side recorded by the last run (its stride)
   void *tmap = nullptr;       // time-blocked 3D kernel: two CUtensorMaps (buf[0], buf[1]) in device memory
   int tmap_key[2] = {0, 0};   // their box (columns, rows)
   int grid = 0;
@@ -168,16 +177,19 @@ struct jacobi_ctx {
   int64_t block_sync = 0;      // resident kernel: 0 grid barrier, 1 neighbour-block flags
   int64_t l2hint = -1;         // streaming loads with L2 eviction hints (-1 default = off)
   int64_t last_resident = 0;   // read-only: whether the last CPU-Free run used it
-  int64_t tblock = -1;         // temporally blocked kernel (K iterations per HBM pass) for slabs
-                               // without neighbours: -1 auto (2D streaming runs), 0 never, 1 force
+  int64_t tblock = -1;         // temporally blocked kernel (K iterations per HBM pass): -1 auto
+                               // (2D always, edge zones between slabs; 3D see run_cpufree), 0 never, 1 force
   int64_t tb_min_block = 16;   // smallest dynamic plane block of the temporally blocked kernel
   int64_t tb_ctas = 1;         // CTAs per SM of the temporally blocked kernel (1 or 2; K = 2 only)
-  int64_t tb_k = -1;           // iterations per time block: -1 auto (2D: JB_TB_K2D, 3D: 2), 2D: 2, 3, 5
+  int64_t tb_k = -1;           // iterations per time block: -1 auto (2D: JB_TB_K2D = 5, 3D: JB_TB_K3D = 3); 2, 3, 5
   int64_t tb_ppt = -1;         // 2D cell pairs per thread and level: -1 auto (4 for K <= 3, 2 for K = 5)
   int64_t tb_lag = -1;         // 2D odd K: wavefront lag between levels (1 or 2; -1 auto)
   int64_t tb_rpw = -1;         // 3D odd K: rows per warp of the tile (-1 auto)
   int64_t last_tb_k = 0;       // read-only: K of the last time-blocked run
   int64_t last_tblock = 0;     // read-only: iterations of the last CPU-Free run done time-blocked
+  int64_t last_launches = 0;   // read-only: kernels this process launched in the last jacobi_run
+  int64_t halo_trace = 0;      // measurement: record the first n halo exchanges of each CPU-Free run
+                               // (%globaltimer wait begin / flag acquired / signal; jacobi_halo_trace)
   int64_t norm_every = 0;      // N4: check the update norm every k iterations (0 = off)
   double tol = 0.0;            // N4: stop once the norm <= tol
   int64_t norm_checks = 0;     // N4: checks performed so far (monotone slot values)
@@ -185,6 +197,7 @@ struct jacobi_ctx {
   std::vector<JbCtrl *> all_ctrl;  // dist mode: every rank's control block (opened via IPC)
   int64_t timeout_ms = 20000;
   bool peers_ready = false;
+  bool all_peers = true;   // single process: peer access enabled between EVERY pair of GPUs (norm all-reduce)
   bool nccl_ready = false;
   double last_ms_max = 0;
   cudaGraphExec_t graph_exec = nullptr;  // cached GRAPH-baseline executable
@@ -236,7 +249,9 @@ cudaError_t reset_run_counters(Slab &s, cudaStream_t st);
 int read_status(Slab &s);
 std::vector<std::vector<int>> launch_groups(jacobi_ctx *h);
 int plan_resident(jacobi_ctx *h, const std::vector<int> &idx, LaunchPlan &L);
+bool resident_fits_all(jacobi_ctx *h);
 int setup_norm(jacobi_ctx *h, LaunchPlan &L);
+int setup_trace(jacobi_ctx *h, LaunchPlan &L);
 int run_cpufree(jacobi_ctx *h, int64_t iters);
 int run_cpufree_k1(jacobi_ctx *h, int64_t iters);
 int run_tblock(jacobi_ctx *h, int64_t iters, int k, int ppt, int lag);

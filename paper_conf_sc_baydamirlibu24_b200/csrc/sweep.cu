@@ -532,8 +532,11 @@ __global__ void __launch_bounds__(JB_THREADS, 1) jb_sweep(const __grid_constant_
       bool waited = !(PERSIST && role != ROLE_INT);
       auto wait_flag = [&]() {
         if (!waited) {
+          const bool mark = PERSIST && lane == 0 && ridx == 0;
+          if (mark) halo_mark(SL, P, role == ROLE_BOT, t, 0);
           if (role == ROLE_TOP) wait_slots(SL.flag_in_top, SL.k_in_top, (unsigned long long)tg, P, lane);
           else wait_slots(SL.flag_in_bot, SL.k_in_bot, (unsigned long long)tg, P, lane);
+          if (mark) halo_mark(SL, P, role == ROLE_BOT, t, 1);
           __syncwarp();
           fence_proxy_async_global();  // every copying lane: halo rows written by the neighbour
           waited = true;
@@ -626,6 +629,7 @@ __global__ void __launch_bounds__(JB_THREADS, 1) jb_sweep(const __grid_constant_
           if (PERSIST && ctid == 0 && !drop_signal) {
             unsigned long long *fo = role == ROLE_TOP ? SL.flag_out_top : SL.flag_out_bot;
             st_release_sys(fo + ridx, (unsigned long long)(tg + 1));
+            if (ridx == 0) halo_mark(SL, P, role == ROLE_BOT, t, 2);
           }
           remote = nullptr;  // later (interior) runs stay local
           continue;

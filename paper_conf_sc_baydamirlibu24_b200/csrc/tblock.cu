@@ -859,10 +859,14 @@ __device__ bool tb_edge(const JbGeom &g, const JbSlab &SL, const JbParams &P, in
   const int ub = (int)((int64_t)g.units * ridx / rcount), ue = (int)((int64_t)g.units * (ridx + 1) / rcount);
   const int tid = threadIdx.x, nt = blockDim.x;
   const bool drop = (P.flags & JACOBI_FLAG_DROP_SIGNAL) && SL.slab_id == 0;
+  const int side = top ? 0 : 1;
+  const bool mark = ridx == 0 && tid == 0;
   auto wait = [&](unsigned long long target) {
     if (tid < 32) {
+      if (mark) halo_mark(SL, P, side, (int64_t)target - P.t0, 0);
       const bool ok = wait_slots(fin, kin, target, P, tid);
       if (tid == 0) *s_flag = ok ? 0 : 1;
+      if (mark) halo_mark(SL, P, side, (int64_t)target - P.t0, 1);
     }
     __syncthreads();
     return *s_flag == 0;
@@ -933,6 +937,7 @@ __device__ bool tb_edge(const JbGeom &g, const JbSlab &SL, const JbParams &P, in
     }
     __syncthreads();  // every thread's stores (local, neighbour's) precede the release below
     if (tid == 0 && !drop) st_release_sys(fout, (unsigned long long)(tg + m));
+    if (mark) halo_mark(SL, P, side, tg + m - 1 - P.t0, 2);
   }
   return true;
 }

@@ -19,7 +19,7 @@ def built():
 
 def test_library_exports_every_header_symbol():
     names = jb.header_functions()
-    assert len(names) == len(jb._SIGS) == 30
+    assert len(names) == len(jb._SIGS) == 31
     L = ctypes.CDLL(jb.LIB_PATH)
     missing = [n for n in names if not hasattr(L, n)]
     assert not missing, missing
