@@ -124,7 +124,8 @@ typedef void (*jacobi_free_fn)(void *ptr, int device, void *user);
 int jacobi_set_allocator(jacobi_alloc_fn alloc, jacobi_free_fn free_fn, void *user);
 /* Bytes of ONE field buffer of slab `slab` (of `nslabs`) for this grid (host-only helper):
  * (chunk + 2) planes (owned + halos) + the time-blocked kernel's edge-zone scratch
- * (DESIGN.md §5.7-5.9): 34 planes in 2D (time blocks up to K = 5), 11 in 3D (K <= 3). */
+ * (DESIGN.md §5.7-5.9): 34 planes in 2D (time blocks up to K = 5), 11 in 3D (K <= 3), + 8 doubles
+ * of read slack (the edge zones' 16-byte pair loads at the last grid column). */
 int jacobi_slab_bytes(int64_t nx, int64_t ny, int64_t nz, int stencil, int nslabs, int slab, int64_t *bytes);
 
 /* ---- NVSHMEM variant — exported ONLY by libjacobi_b200_nvshmem.so --------

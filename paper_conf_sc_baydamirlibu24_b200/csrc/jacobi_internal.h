@@ -28,6 +28,14 @@
 // 2K-m of them for m = 1..K-1.  2D buffers carry enough for JB_TB_KMAX2, 3D ones for JB_TB_KMAX3.
 static inline int64_t jb_edge_planes_k(int K) { return (K - 1) + (int64_t)(K - 1) * 2 * K - (int64_t)(K - 1) * K / 2; }
 static inline int64_t jb_edge_planes(int dim) { return jb_edge_planes_k(dim == 2 ? JB_TB_KMAX2 : JB_TB_KMAX3); }
+// Read slack after each field buffer (doubles): the vectorised edge zones load whole 16-byte cell
+// pairs and their x neighbours, which at the grid's last column reach up to two doubles past the
+// last row of the last scratch plane (the values are never used).
+#define JB_BUF_SLACK 8
+// Doubles of ONE field buffer of a slab with `chunk` owned planes.
+static inline int64_t jb_buf_doubles(int64_t chunk, int dim, int64_t plane_elems) {
+  return (chunk + 2 + jb_edge_planes(dim)) * plane_elems + JB_BUF_SLACK;
+}
 
 // Grid geometry in HBM and the tile shape of the march.
 //   element (x, y, z) of slab plane p lives at  buf + p*plane_elems + y*pitch + (x + 3)

@@ -64,7 +64,7 @@ int jacobi_slab_bytes(int64_t nx, int64_t ny, int64_t nz, int stencil, int nslab
   if (jbplan::geometry(nx, ny, nz, stencil == 5 ? 2 : 3, 8, 1, JB_SMEM_DEFAULT, 0, &g)) return JACOBI_EINVAL;
   int64_t start, chunk;
   jbplan::decompose(stencil == 5 ? ny : nz, nslabs, slab, &start, &chunk);
-  *bytes = (chunk + 2 + jb_edge_planes(g.dim)) * g.plane_elems * (int64_t)sizeof(double);
+  *bytes = jb_buf_doubles(chunk, g.dim, g.plane_elems) * (int64_t)sizeof(double);
   return JACOBI_OK;
 }
 
@@ -200,7 +200,7 @@ int jacobi_create_nvshmem(int64_t nx, int64_t ny, int64_t nz, int stencil, const
       jbplan::geometry(nx, ny, nz, stencil == 5 ? 2 : 3, 8, 1, JB_SMEM_DEFAULT, 0, &g);
       int64_t st, chunk_max;
       jbplan::decompose(stencil == 5 ? ny : nz, world_size, 0, &st, &chunk_max);
-      const int64_t need = 2 * (chunk_max + 2 + jb_edge_planes(g.dim)) * g.plane_elems * 8 + (64 << 20);
+      const int64_t need = 2 * jb_buf_doubles(chunk_max, g.dim, g.plane_elems) * 8 + (64 << 20);
       const int64_t sz = std::max<int64_t>(need + need / 4, (int64_t)1 << 30);
       setenv("NVSHMEM_SYMMETRIC_SIZE", std::to_string(sz).c_str(), 0);
     }

@@ -33,11 +33,11 @@ jacobi_ctx *new_ctx(int64_t nx, int64_t ny, int64_t nz, int stencil, int total) 
 int alloc_slab(jacobi_ctx *h, Slab &s) {
   CK(cudaSetDevice(s.device));
   // (chunk + 2) planes of the slab + jb_edge_planes(h->dim) scratch planes (time-blocked edge zones)
-  size_t bytes = (size_t)(s.chunk + 2 + jb_edge_planes(h->dim)) * h->geom.plane_elems * sizeof(double);
+  size_t bytes = (size_t)jb_buf_doubles(s.chunk, h->dim, h->geom.plane_elems) * sizeof(double);
   if (h->kind == KIND_SHMEM) {  // symmetric heap: every PE allocates the largest slab
     int64_t st, chunk_max;
     jbplan::decompose(h->n_out, h->total, 0, &st, &chunk_max);
-    bytes = (size_t)(chunk_max + 2 + jb_edge_planes(h->dim)) * h->geom.plane_elems * sizeof(double);
+    bytes = (size_t)jb_buf_doubles(chunk_max, h->dim, h->geom.plane_elems) * sizeof(double);
   }
   if (h->alloc.alloc) {
     s.buf[0] = static_cast<double *>(h->alloc.alloc(bytes, s.device, h->alloc.user));

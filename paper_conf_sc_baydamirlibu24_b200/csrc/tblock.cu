@@ -846,18 +846,113 @@ __device__ __forceinline__ void tb3k_item(const JbGeom &g, const Ring &R, RingPo
 //   [lbase(m) + i], i < 2K-m    this side's level-m plane first(m) + i (top: 1 + i,
 //                               bottom: C-2K+m+1 + i)
 // Loads bypass L1 (ld.cg): these planes are rewritten by other CTAs / the neighbour GPU.
+__device__ __forceinline__ double2 ldcg2(const double *p) { return __ldcg(reinterpret_cast<const double2 *>(p)); }
+
+// One phase, vectorised: a thread owns one 16-byte cell pair (x odd, x+1; 3D: of one row y) of the
+// window and marches it through the phase's NP planes, keeping the level-(m-1) pairs of the
+// march's three consecutive planes in registers (loaded once each, every load issued up front),
+// so a cell update costs 1.5 loads in 2D (pair + its two x neighbours per plane, the plane
+// neighbours are the march's registers) and 2.5 in 3D, and every store is a 16-byte store into
+// the local scratch / next buffer and, for the outermost plane, straight into the neighbour's
+// slot or halo.  Same oracle order; cells outside the interior keep level m-1.
+template <int DIM, int K, int M>
+__device__ __forceinline__ void tb_edge_phase(const JbGeom &g, bool top, int64_t C, const double *cur, double *E,
+                                              double *nxt, double *mid, double *remote, int ub, int ue) {
+  constexpr int NP = M < K ? 2 * K - M : K;  // level-M planes of this side
+  constexpr int NPV = 2 * K - (M - 1);       // level-(M-1) planes of this side (M >= 2)
+  constexpr int MG = K - M;                  // window margin
+  const int64_t pe = g.plane_elems, pitch = g.pitch;
+  const int nx = (int)g.nx, ny = (int)g.ny;
+  const int64_t pf = top ? 1 : C - NP + 1;  // first level-M plane
+  const int64_t pfv = top ? 1 : C - NPV + 1;
+  const int64_t halo = top ? 0 : C + 1;
+  auto lbase = [](int m) { return (int64_t)(K - 1) + (int64_t)(m - 1) * 2 * K - (int64_t)(m - 1) * m / 2; };
+  // level M-1 of plane p (element offset 3 of x = 0, row 0)
+  auto src = [&](int64_t p) -> const double * {
+    if (M == 1) return cur + p * pe + 3;
+    if (p == halo) return E + (int64_t)(M - 2) * pe;
+    return E + (lbase(M - 1) + (p - pfv)) * pe;
+  };
+  auto dst = [&](int k) -> double * { return M < K ? E + (lbase(M) + k) * pe : nxt + (pf + k) * pe + 3; };
+  double *d2 = M < K ? mid + (int64_t)(M - 1) * pe : remote + 3;  // the neighbour's slot / halo
+  const int kout = top ? 0 : NP - 1;                               // plane index of pout
+  for (int u = ub; u < ue; ++u) {
+    const int ux = u % g.units_x, uy = u / g.units_x;
+    const int x0 = 1 + ux * g.tx;
+    int xa, xb, ya = 0, yb = 0;
+    if (M < K) {
+      xa = max(x0 - MG, 0);
+      xb = min(x0 + g.tx - 1 + MG, nx - 1);
+    } else {
+      xa = x0;
+      xb = min(x0 + g.tx, nx - 1) - 1;
+    }
+    if (DIM == 3) {
+      const int y0 = 1 + uy * g.ty;
+      if (M < K) {
+        ya = max(y0 - MG, 0);
+        yb = min(y0 + g.ty - 1 + MG, ny - 1);
+      } else {
+        ya = y0;
+        yb = min(y0 + g.ty, ny - 1) - 1;
+      }
+    }
+    const int xp0 = (xa & 1) ? xa : xa - 1;  // first pair (x odd: 16-byte aligned)
+    const int npx = (xb - xp0) / 2 + 1;
+    const int items = npx * (yb - ya + 1);
+    for (int c = threadIdx.x; c < items; c += blockDim.x) {
+      const int ry = DIM == 3 ? c / npx : 0;
+      const int x = xp0 + 2 * (c - ry * npx), y = ya + ry;
+      const int64_t e = (DIM == 3 ? (int64_t)y * pitch : 0) + x;
+      const bool yin = DIM == 2 || (y >= 1 && y <= ny - 2);
+      const bool in0 = yin && x >= 1 && x <= nx - 2, in1 = yin && x + 1 <= nx - 2;
+      const bool st0 = x >= xa, st1 = x + 1 <= xb;
+      // y neighbours of the Dirichlet rows are never used: keep their loads inside the plane
+      const int64_t yn = (DIM == 3 && y < ny - 1) ? pitch : 0, ys = (DIM == 3 && y > 0) ? -pitch : 0;
+      double2 Cp[NP + 2];  // level M-1 pairs of planes pf-1 .. pf+NP
+#pragma unroll
+      for (int i = 0; i < NP + 2; ++i) Cp[i] = ldcg2(src(pf - 1 + i) + e);
+#pragma unroll
+      for (int k = 0; k < NP; ++k) {
+        const double *A = src(pf + k) + e;
+        const double W = __ldcg(A - 1), Ee = __ldcg(A + 2);
+        const double2 c0 = Cp[k + 1];
+        double v0, v1;
+        if (DIM == 2) {  // oracle order: x+1, x-1, y+1 (plane p+1), y-1 (plane p-1), then * 1/4
+          v0 = 0.25 * (((c0.y + W) + Cp[k + 2].x) + Cp[k].x);
+          v1 = 0.25 * (((Ee + c0.x) + Cp[k + 2].y) + Cp[k].y);
+        } else {  // x+1, x-1, y+1, y-1, z+1 (plane p+1), z-1 (plane p-1), then * fl(1/6)
+          const double2 N = ldcg2(A + yn), S = ldcg2(A + ys);
+          v0 = kC6 * (((((c0.y + W) + N.x) + S.x) + Cp[k + 2].x) + Cp[k].x);
+          v1 = kC6 * (((((Ee + c0.x) + N.y) + S.y) + Cp[k + 2].y) + Cp[k].y);
+        }
+        const double2 v = make_double2(in0 ? v0 : c0.x, in1 ? v1 : c0.y);
+        auto put = [&](double *d) {
+          if (st0 && st1) *reinterpret_cast<double2 *>(d) = v;
+          else if (st0) d[0] = v.x;
+          else if (st1) d[1] = v.y;
+        };
+        put(dst(k) + e);
+        if (k == kout) put(d2 + e);
+      }
+    }
+  }
+}
+
+// Not inlined: its fully unrolled phases would otherwise raise the register pressure of the
+// interior march they share the kernel with (measured: spills in the hot loop).
 template <int DIM, int K>
-__device__ bool tb_edge(const JbGeom &g, const JbSlab &SL, const JbParams &P, int role, int ridx, int rcount,
+__device__ __noinline__ bool tb_edge(const JbGeom &g, const JbSlab &SL, const JbParams &P, int role, int ridx, int rcount,
                         const double *cur, double *nxt, double *remote, int64_t tg, int *s_flag) {
   const bool top = role == ROLE_TOP;
-  const int64_t C = SL.chunk, pe = g.plane_elems, nx = g.nx, ny = g.ny, pitch = g.pitch;
+  const int64_t C = SL.chunk, pe = g.plane_elems;
   double *E = (top ? SL.buf[0] : SL.buf[1]) + (C + 2) * pe + 3;
   double *mid = (top ? SL.mid_top_out : SL.mid_bot_out) + 3;
   const unsigned long long *fin = top ? SL.flag_in_top : SL.flag_in_bot;
   const int kin = top ? SL.k_in_top : SL.k_in_bot;
   unsigned long long *fout = (top ? SL.flag_out_top : SL.flag_out_bot) + ridx;
   const int ub = (int)((int64_t)g.units * ridx / rcount), ue = (int)((int64_t)g.units * (ridx + 1) / rcount);
-  const int tid = threadIdx.x, nt = blockDim.x;
+  const int tid = threadIdx.x;
   const bool drop = (P.flags & JACOBI_FLAG_DROP_SIGNAL) && SL.slab_id == 0;
   const int side = top ? 0 : 1;
   const bool mark = ridx == 0 && tid == 0;
@@ -871,70 +966,15 @@ __device__ bool tb_edge(const JbGeom &g, const JbSlab &SL, const JbParams &P, in
     __syncthreads();
     return *s_flag == 0;
   };
-  auto lbase = [](int m) { return (int64_t)(K - 1) + (int64_t)(m - 1) * 2 * K - (int64_t)(m - 1) * m / 2; };
-  const int64_t halo = top ? 0 : C + 1;
-  const int64_t pout = top ? 1 : C;  // the plane the neighbour needs
-#pragma unroll 1
+#pragma unroll
   for (int m = 1; m <= K; ++m) {
     if (!wait((unsigned long long)(tg + m - 1))) return false;
-    const int64_t np = m < K ? 2 * K - m : K;        // level-m planes of this side
-    const int64_t pf = top ? 1 : C - np + 1;         // the first of them
-    const int64_t npv = 2 * K - (m - 1);             // level-(m-1) planes of this side (m >= 2)
-    const int64_t pfv = top ? 1 : C - npv + 1;
-    // level m-1 of plane p (element offset 3 of x = 0, row 0)
-    auto src = [&](int64_t p) -> const double * {
-      if (m == 1) return cur + p * pe + 3;
-      if (p == halo) return E + (int64_t)(m - 2) * pe;
-      return E + (lbase(m - 1) + (p - pfv)) * pe;
-    };
-    const int64_t mg = K - m;  // window margin
-    for (int u = ub; u < ue; ++u) {
-      const int ux = u % g.units_x, uy = u / g.units_x;
-      const int64_t x0 = 1 + (int64_t)ux * g.tx;
-      int64_t xa, xb, ya = 0, yb = 0;
-      if (m < K) {
-        xa = max(x0 - mg, (int64_t)0);
-        xb = min(x0 + g.tx - 1 + mg, nx - 1);
-      } else {
-        xa = x0;
-        xb = min(x0 + g.tx, nx - 1) - 1;
-      }
-      if (DIM == 3) {
-        const int64_t y0 = 1 + (int64_t)uy * g.ty;
-        if (m < K) {
-          ya = max(y0 - mg, (int64_t)0);
-          yb = min(y0 + g.ty - 1 + mg, ny - 1);
-        } else {
-          ya = y0;
-          yb = min(y0 + g.ty, ny - 1) - 1;
-        }
-      }
-      const int w = (int)(xb - xa + 1), hw = (int)(yb - ya + 1) * w;
-      for (int64_t k = 0; k < np; ++k) {  // per plane: source / destination pointers hoisted
-        const int64_t p = pf + k;
-        const double *Sm = src(p - 1), *Sc = src(p), *Sp = src(p + 1);
-        double *D = m < K ? E + (lbase(m) + k) * pe : nxt + p * pe + 3;
-        double *D2 = p != pout ? nullptr : m < K ? mid + (int64_t)(m - 1) * pe : remote + 3;
-        for (int c = tid; c < hw; c += nt) {  // (row, column) of the window, 32-bit index math
-          const int yy = DIM == 3 ? c / w : 0, xx = c - yy * w;
-          const int64_t x = xa + xx, y = ya + yy;
-          const int64_t e = (DIM == 3 ? y * pitch : 0) + x;
-          const bool in = x >= 1 && x <= nx - 2 && (DIM == 2 || (y >= 1 && y <= ny - 2));
-          const double *A = Sc + e;
-          double v;
-          if (!in) {
-            v = __ldcg(A);
-          } else if (DIM == 2) {  // oracle order: x+1, x-1, y+1, y-1 (then z+1, z-1), then the scale
-            v = 0.25 * (((__ldcg(A + 1) + __ldcg(A - 1)) + __ldcg(Sp + e)) + __ldcg(Sm + e));
-          } else {
-            v = kC6 * (((((__ldcg(A + 1) + __ldcg(A - 1)) + __ldcg(A + pitch)) + __ldcg(A - pitch)) + __ldcg(Sp + e)) +
-                       __ldcg(Sm + e));
-          }
-          D[e] = v;
-          if (D2) D2[e] = v;
-        }
-      }
-    }
+    // level m (compile-time per phase: the march and its loads are fully unrolled)
+    if (m == 1) tb_edge_phase<DIM, K, 1>(g, top, C, cur, E, nxt, mid, remote, ub, ue);
+    if constexpr (K >= 2) if (m == 2) tb_edge_phase<DIM, K, 2>(g, top, C, cur, E, nxt, mid, remote, ub, ue);
+    if constexpr (K >= 3) if (m == 3) tb_edge_phase<DIM, K, 3>(g, top, C, cur, E, nxt, mid, remote, ub, ue);
+    if constexpr (K >= 4) if (m == 4) tb_edge_phase<DIM, K, 4>(g, top, C, cur, E, nxt, mid, remote, ub, ue);
+    if constexpr (K >= 5) if (m == 5) tb_edge_phase<DIM, K, 5>(g, top, C, cur, E, nxt, mid, remote, ub, ue);
     __syncthreads();  // every thread's stores (local, neighbour's) precede the release below
     if (tid == 0 && !drop) st_release_sys(fout, (unsigned long long)(tg + m));
     if (mark) halo_mark(SL, P, side, tg + m - 1 - P.t0, 2);

@@ -196,13 +196,14 @@ def test_slab_bytes_matches_layout():
         kmax = 5
         scratch = (kmax - 1) + sum(2 * kmax - m for m in range(1, kmax))
         assert scratch == 34
-        assert b == (c + 2 + scratch) * g["plane_elems"] * 8
+        # + 8 doubles of read slack (JB_BUF_SLACK: vectorised edge-zone pair loads at the last column)
+        assert b == ((c + 2 + scratch) * g["plane_elems"] + 8) * 8
         total += c
     assert total == 62
     # 3D: K <= 3: 2 slots + 5 level-1 + 4 level-2 planes
     g3 = jb.jacobi_geometry(40, 30, 64, 7)
     s, c = jb.jacobi_decompose(64, 3, 1)
-    assert jb.jacobi_slab_bytes(40, 30, 64, 7, 3, 1) == (c + 2 + 11) * g3["plane_elems"] * 8
+    assert jb.jacobi_slab_bytes(40, 30, 64, 7, 3, 1) == ((c + 2 + 11) * g3["plane_elems"] + 8) * 8
 
 
 def test_set_allocator_rejects_half():
