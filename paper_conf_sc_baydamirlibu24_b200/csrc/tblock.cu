@@ -277,6 +277,27 @@ __device__ __forceinline__ void tbk_level1(const TbkLane &L, const double *sm, c
   }
 }
 
+// Level 1 from level-0 pairs already in registers (S, Cm, N rows; W / E: the centre row's cells
+// left of pair 0 and right of the last pair) — the software-pipelined steady state of tbk_march.
+template <int PPT, bool FAST>
+__device__ __forceinline__ void tbk_level1_regs(const TbkLane &L, const double2 *S0, const double2 *C0,
+                                                const double2 *N0, double Wl, double Er, double2 *V) {
+#pragma unroll
+  for (int i = 0; i < PPT; ++i) {
+    const double W = i == 0 ? Wl : C0[i - 1].y;
+    const double E = i == PPT - 1 ? Er : C0[i + 1].x;
+    // oracle order: ((x+1) + (x-1)) + (y+1) + (y-1), then * 0.25
+    const double l0 = 0.25 * (((C0[i].y + W) + N0[i].x) + S0[i].x);
+    const double l1 = 0.25 * (((E + C0[i].x) + N0[i].y) + S0[i].y);
+    if (FAST) {
+      V[i] = make_double2(l0, l1);
+    } else {
+      V[i].x = (L.ok >> i & 1u) ? l0 : C0[i].x;  // (steady rows are interior; columns may not be)
+      V[i].y = (L.full >> i & 1u) ? l1 : C0[i].y;
+    }
+  }
+}
+
 // A double from lane src (two 32-bit shuffles, halves kept in place).
 __device__ __forceinline__ double shfl_d(double v, int src) {
   double r;
@@ -345,6 +366,25 @@ __device__ __forceinline__ void tbk_march(const TbkLane &L, const Ring &R, RingP
   if (Rs <= r1) pn = ring_add(q, (uint32_t)(Rs - r0), R.S);
   R.wait_full(pm);
   R.wait_full(pc);
+  // Software pipelining of the steady state (LAG = 1): the level-0 pairs of the three rows a
+  // step reads live in registers Z[m % 3] (newest row of step m), and right after level 1 the
+  // step already waits for and loads the NEXT step's new row (one 16-byte LDS) and its centre
+  // row's two x neighbours, so their shared-memory latency overlaps levels 2 .. K instead of
+  // heading the next step's dependency chain (and 3 instead of 5 LDS per step).
+  constexpr bool PF = NS == 3;
+  double2 Z[3][PPT];
+  double zW = 0.0, zE = 0.0;
+  RingPos pnn = pn;  // steady steps: the next step's newest row
+  auto zload = [&](double2 *z, const RingPos &p) {
+    const double *st = R.stage(p) + L.j0;
+#pragma unroll
+    for (int i = 0; i < PPT; ++i) z[i] = lds2(st + 2 * i);
+  };
+  auto weload = [&](const RingPos &p) {
+    const double *st = R.stage(p) + L.j0;
+    zW = st[-1];
+    zE = st[2 * PPT];
+  };
   auto step = [&](auto u_ct, auto steady_ct, int Rr) {
     constexpr int U = decltype(u_ct)::value;
     constexpr bool ST = decltype(steady_ct)::value;
@@ -352,12 +392,26 @@ __device__ __forceinline__ void tbk_march(const TbkLane &L, const Ring &R, RingP
     constexpr int SN = (U + NS - (LAG - 1)) % NS, SC = (U + NS - LAG) % NS, SS = (U + 2 * NS - LAG - 1) % NS;
     // level k computes row Rr-1-LAG(k-1) if it lies in its range [a-(K-k), b+(K-k)] ∩ [0, C+1]
     auto need = [&](int k, int r) { return r >= max(a - (K - k), 0) && r <= min(b + (K - k), C + 1); };
-    if (ST || Rr <= r1) R.wait_full(pn);
-    // (y-1, centre, y+1) rows: the march's older / newer neighbours, swapped when it runs down
-    if (ST || need(1, Rr - 1))
-      tbk_level1<PPT, FAST, ST>(L, R.stage(REV ? pn : pm), R.stage(pc), R.stage(REV ? pm : pn), Rr - 1 >= 1 && Rr - 1 <= C,
-                                X[0][U]);
-    if (ST || (Rr - 2 >= r0 && Rr - 2 <= r1)) R.release(pm, lane);  // row Rr-2 is no longer needed
+    if (ST && PF) {
+      // level-0 rows Rr (newest, Z[U]), Rr-1 (centre, Z[U+2]), Rr-2 (Z[U+1]), preloaded
+      constexpr int ZN = U % 3, ZC = (U + 2) % 3, ZO = (U + 1) % 3;
+      tbk_level1_regs<PPT, FAST>(L, Z[REV ? ZN : ZO], Z[ZC], Z[REV ? ZO : ZN], zW, zE, X[0][U]);
+      R.release(pm, lane);  // row Rr-2: its last reads were the preloads
+      // next step (steady steps end before r1): its newest row into Z[U+1] (row Rr-2's, now
+      // dead), W / E of its centre row Rr
+      pnn = pn;
+      pnn.advance(R.S);
+      R.wait_full(pnn);
+      zload(Z[ZO], pnn);
+      weload(pn);
+    } else {
+      if (ST || Rr <= r1) R.wait_full(pn);
+      // (y-1, centre, y+1) rows: the march's older / newer neighbours, swapped when it runs down
+      if (ST || need(1, Rr - 1))
+        tbk_level1<PPT, FAST, ST>(L, R.stage(REV ? pn : pm), R.stage(pc), R.stage(REV ? pm : pn),
+                                  Rr - 1 >= 1 && Rr - 1 <= C, X[0][U]);
+      if (ST || (Rr - 2 >= r0 && Rr - 2 <= r1)) R.release(pm, lane);  // row Rr-2 is no longer needed
+    }
 #pragma unroll
     for (int k = 2; k < K; ++k) {
       const int r = Rr - 1 - LAG * (k - 1);
@@ -372,7 +426,9 @@ __device__ __forceinline__ void tbk_march(const TbkLane &L, const Ring &R, RingP
     o += ostep;
     pm = pc;
     pc = pn;
-    if (Rr + 1 <= r1) {  // branch-free ring advance
+    if (ST && PF) {
+      pn = pnn;
+    } else if (Rr + 1 <= r1) {  // branch-free ring advance
       const uint32_t sl = pn.slot + 1u;
       const bool wrap = sl == R.S;
       pn.slot = wrap ? 0u : sl;
@@ -394,8 +450,17 @@ __device__ __forceinline__ void tbk_march(const TbkLane &L, const Ring &R, RingP
   int Rr = Rs;
   if (nsteady > 0) {
     for (; Rr < Ws; Rr += NS) group(TF{}, Rr);  // the prefix keeps the group phase (set rotation)
-    if (Rr + NS - 1 <= We) {
-      const int Rend = Rr + ((We - Rr + 1) / NS) * NS;
+    // (with the preloads the steady steps end at We - 1: every one has a next row in the ring)
+    const int Wend = PF ? We - 1 : We;
+    if (Rr + NS - 1 <= Wend) {
+      const int Rend = Rr + ((Wend - Rr + 1) / NS) * NS;
+      if constexpr (PF) {  // preload the first steady step's rows (Rr, Rr-1, Rr-2 -> Z[0], Z[2], Z[1])
+        R.wait_full(pn);
+        zload(Z[0], pn);
+        zload(Z[2], pc);
+        zload(Z[1], pm);
+        weload(pc);
+      }
       for (; Rr < Rend; Rr += NS) group(TT{}, Rr);
     }
   }
@@ -905,7 +970,7 @@ __device__ __forceinline__ void tb_edge_phase(const JbGeom &g, bool top, int64_t
       const int x = xp0 + 2 * (c - ry * npx), y = ya + ry;
       const int64_t e = (DIM == 3 ? (int64_t)y * pitch : 0) + x;
       const bool yin = DIM == 2 || (y >= 1 && y <= ny - 2);
-      const bool in0 = yin && x >= 1 && x <= nx - 2, in1 = yin && x + 1 <= nx - 2;
+      const bool in0 = yin && x >= 1 && x <= nx - 2, in1 = yin && x + 1 >= 1 && x + 1 <= nx - 2;
       const bool st0 = x >= xa, st1 = x + 1 <= xb;
       // y neighbours of the Dirichlet rows are never used: keep their loads inside the plane
       const int64_t yn = (DIM == 3 && y < ny - 1) ? pitch : 0, ys = (DIM == 3 && y > 0) ? -pitch : 0;
