@@ -690,7 +690,7 @@ int run_cpufree_k1(jacobi_ctx *h, int64_t iters) {
 // over the interior planes the edge zones leave, and the ring shortened to the smem budget.
 // (K, pairs per lane, variant) of the time-blocked kernel for this handle; K = 0: none fits.
 // variant: 2D odd K = the wavefront lag (1, 2); 3D odd K = rows per warp of the tile.
-void tblock_choice(const jacobi_ctx *h, int *k_out, int *ppt_out, int *var_out) {
+void tblock_choice(const jacobi_ctx *h, int *k_out, int *ppt_out, int *var_out, int *ws_out) {
   const int kmax = h->dim == 2 ? JB_TB_KMAX2 : JB_TB_KMAX3;
   int k = h->tb_k >= 2 ? (int)std::min<int64_t>(h->tb_k, kmax) : (h->dim == 2 ? JB_TB_K2D : JB_TB_K3D);
   // every slab needs its edge zones (2K planes) when it has neighbours: shallower blocks otherwise
@@ -712,12 +712,13 @@ void tblock_choice(const jacobi_ctx *h, int *k_out, int *ppt_out, int *var_out) 
     var = dflt_var(k);
   }
   if (!fits(k)) k = 0;
+  *ws_out = (h->tb_ws != 0 && k > 0 && jbk::tblock_ncw(h->dim, k, ppt, var, 1, 1) > 0) ? 1 : 0;
   *k_out = k;
   *ppt_out = ppt;
   *var_out = var;
 }
 
-int run_tblock(jacobi_ctx *h, int64_t iters, int K, int ppt, int lag) {
+int run_tblock(jacobi_ctx *h, int64_t iters, int K, int ppt, int lag, int ws) {
   auto groups = launch_groups(h);
   std::vector<LaunchPlan> plans(groups.size());
   // roles must match across slabs; two CTAs per SM only for K = 2
@@ -750,7 +751,7 @@ int run_tblock(jacobi_ctx *h, int64_t iters, int K, int ppt, int lag) {
       g.units = g.units_x * g.units_y;
       g.stage_doubles = g.rh * g.ws;
     } else if (K > 2) {  // odd K: JB_NCW warps x (64 ppt - 2(K-1)) output columns per strip
-      g.tx = jbk::tblock_ncw(2, K, ppt, lag, 1) * (64 * ppt - 2 * (K - 1));
+      g.tx = jbk::tblock_ncw(2, K, ppt, lag, 1, ws) * (64 * ppt - 2 * (K - 1));
       g.ws = g.tx + 2 * K + 2;
       g.units_x = (int)((h->nx - 2 + g.tx - 1) / g.tx);
       g.units_y = 1;
@@ -802,7 +803,7 @@ int run_tblock(jacobi_ctx *h, int64_t iters, int K, int ppt, int lag) {
     if (jbk::tblock_smem(g) > (size_t)smem_optin) return JACOBI_EINVAL;
     L.smem = jbk::tblock_smem(g);
     int occ = 0;
-    CK(jbk::prepare_tblock(g, K, ppt, lag, per_sm, L.smem, &occ));
+    CK(jbk::prepare_tblock(g, K, ppt, lag, per_sm, ws, L.smem, &occ));
     if (occ < per_sm) {
       if (getenv("JACOBI_DEBUG")) fprintf(stderr, "[jacobi] tblock: occupancy %d < %d (smem %zu)\n", occ, per_sm, L.smem);
       return JACOBI_ENOCOOP;
@@ -829,7 +830,7 @@ int run_tblock(jacobi_ctx *h, int64_t iters, int K, int ppt, int lag) {
     CK(cudaSetDevice(L.device));
     Slab &s0 = h->slabs[L.slab_idx[0]];
     CK(cudaEventRecord(s0.ev0, L.stream));
-    CK(jbk::launch_tblock(L.P, K, ppt, lag, per_sm, L.grid, L.smem, L.stream));
+    CK(jbk::launch_tblock(L.P, K, ppt, lag, per_sm, ws, L.grid, L.smem, L.stream));
     ++h->last_launches;
     CK(cudaEventRecord(s0.ev1, L.stream));
   }
@@ -859,16 +860,27 @@ int run_cpufree(jacobi_ctx *h, int64_t iters) {
   h->last_launches = 0;
   h->last_tblock = 0;
   h->last_tb_k = 0;
+  h->last_tb_ws = 0;
   h->last_resident = 0;
   const bool nocomp = h->flags & JACOBI_FLAG_NO_COMPUTE;
   // P > 1: every slab needs the two edge zones (>= 2K planes); the NVSHMEM variant keeps jb_sweep
-  int K = 0, ppt = 0, lag = 1;
-  tblock_choice(h, &K, &ppt, &lag);
+  int K = 0, ppt = 0, lag = 1, ws = 0;
+  tblock_choice(h, &K, &ppt, &lag, &ws);
   const bool eligible = h->tblock != 0 && !nocomp && h->norm_every <= 0 && h->kind != KIND_SHMEM && K >= 2;
   if (h->tblock == 1 && !eligible) return JACOBI_EINVAL;
-  // auto picks it where it measured faster than the per-iteration kernel: 2D, and 3D slabs
-  // without neighbours (3D edge zones are whole planes: slower than per-iteration at P > 1)
-  const bool use = eligible && (h->tblock == 1 || h->dim == 2 || h->total == 1);
+  // auto picks it where it measured faster than the per-iteration kernel: 2D always; 3D when the
+  // slabs have no neighbours, or when every slab has >= 64 CTAs — the 3D edge zones are whole
+  // planes (K phases x 2K-m planes per side, computed by at most a quarter of the slab's CTAs),
+  // which pays with a GPU per slab (and with 2 virtual slabs: C3 397 -> 414 Gcell/s) but not when
+  // 4-8 virtual slabs share one GPU's CTAs
+  bool use3 = h->total == 1;
+  if (!use3 && h->dim == 3) {
+    int sms = 0;
+    CK(cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, h->slabs[0].device));
+    use3 = true;
+    for (int id = 0; id < h->total; ++id) use3 = use3 && slab_ctas(h, id, sms) >= 64;
+  }
+  const bool use = eligible && (h->tblock == 1 || h->dim == 2 || use3);
   int64_t tb_iters = 0;
   if (use) {
     // odd K: any block count; K = 2: an even one (the result stays in buf[t & 1], R10)
@@ -880,11 +892,12 @@ int run_cpufree(jacobi_ctx *h, int64_t iters) {
   }
   double ms = 0;
   if (tb_iters > 0) {
-    int rc = run_tblock(h, tb_iters, K, ppt, lag);
+    int rc = run_tblock(h, tb_iters, K, ppt, lag, ws);
     if (rc) return rc;
     ms = h->last_ms_max;
     h->last_tblock = tb_iters;
     h->last_tb_k = K;
+    h->last_tb_ws = ws;
   }
   if (iters - tb_iters > 0) {
     int rc = run_cpufree_k1(h, iters - tb_iters);
@@ -1019,6 +1032,8 @@ static int64_t *param_slot(jacobi_t h, const char *name) {
   if (!std::strcmp(name, "tb_ppt")) return &h->tb_ppt;
   if (!std::strcmp(name, "tb_lag")) return &h->tb_lag;
   if (!std::strcmp(name, "tb_rpw")) return &h->tb_rpw;
+  if (!std::strcmp(name, "tb_ws")) return &h->tb_ws;
+  if (!std::strcmp(name, "last_tb_ws")) return &h->last_tb_ws;
   if (!std::strcmp(name, "last_tb_k")) return &h->last_tb_k;
   if (!std::strcmp(name, "last_tblock")) return &h->last_tblock;
   if (!std::strcmp(name, "halo_trace")) return &h->halo_trace;
@@ -1029,7 +1044,7 @@ static int64_t *param_slot(jacobi_t h, const char *name) {
 int jacobi_set_param(jacobi_t h, const char *name, int64_t value) {
   if (!h || !name) return JACOBI_EINVAL;
   if (!std::strcmp(name, "last_resident") || !std::strcmp(name, "last_tblock") || !std::strcmp(name, "last_tb_k") ||
-      !std::strcmp(name, "last_launches"))
+      !std::strcmp(name, "last_launches") || !std::strcmp(name, "last_tb_ws"))
     return JACOBI_EINVAL;  // read-only
   int64_t *p = param_slot(h, name);
   if (!p) return JACOBI_EINVAL;

@@ -34,10 +34,10 @@ cudaError_t prepare_resident(int dim, int cpp, size_t smem, int *blocks_per_sm);
 cudaError_t launch_resident(const JbParams &p, int cpp, int grid, size_t smem, cudaStream_t st);
 cudaError_t launch_neighbour_wait(const JbParams &p, unsigned long long target, cudaStream_t st);
 int tblock_ty();
-int tblock_ncw(int dim, int k, int ppt, int lag, int per_sm);
+int tblock_ncw(int dim, int k, int ppt, int lag, int per_sm, int ws = 0);
 size_t tblock_smem(const JbGeom &g);
-cudaError_t prepare_tblock(const JbGeom &g, int k, int ppt, int lag, int per_sm, size_t smem, int *blocks_per_sm);
-cudaError_t launch_tblock(const JbParams &p, int k, int ppt, int lag, int per_sm, int grid, size_t smem,
+cudaError_t prepare_tblock(const JbGeom &g, int k, int ppt, int lag, int per_sm, int ws, size_t smem, int *blocks_per_sm);
+cudaError_t launch_tblock(const JbParams &p, int k, int ppt, int lag, int per_sm, int ws, int grid, size_t smem,
                           cudaStream_t st);
 }  // namespace jbk
 
@@ -185,6 +185,8 @@ struct jacobi_ctx {
   int64_t tb_ppt = -1;         // 2D cell pairs per thread and level: -1 auto (4 for K <= 3, 2 for K = 5)
   int64_t tb_lag = -1;         // 2D odd K: wavefront lag between levels (1 or 2; -1 auto)
   int64_t tb_rpw = -1;         // 3D odd K: rows per warp of the tile (-1 auto)
+  int64_t tb_ws = -1;          // warp-specialised register split (12 compute warps; -1 auto = where built, 0 off)
+  int64_t last_tb_ws = 0;      // read-only: whether the last time-blocked run used it
   int64_t last_tb_k = 0;       // read-only: K of the last time-blocked run
   int64_t last_tblock = 0;     // read-only: iterations of the last CPU-Free run done time-blocked
   int64_t last_launches = 0;   // read-only: kernels this process launched in the last jacobi_run
@@ -254,11 +256,11 @@ int setup_norm(jacobi_ctx *h, LaunchPlan &L);
 int setup_trace(jacobi_ctx *h, LaunchPlan &L);
 int run_cpufree(jacobi_ctx *h, int64_t iters);
 int run_cpufree_k1(jacobi_ctx *h, int64_t iters);
-int run_tblock(jacobi_ctx *h, int64_t iters, int k, int ppt, int lag);
+int run_tblock(jacobi_ctx *h, int64_t iters, int k, int ppt, int lag, int ws);
 // Tensor maps of a slab's two buffers for TMA box loads of `cols` x `rows` elements (one plane).
 int slab_tensor_maps(jacobi_ctx *h, Slab &s, int cols, int rows);
 // Time-block depth and pairs per thread the runtime would use for this handle (K = 0: none).
-void tblock_choice(const jacobi_ctx *h, int *k, int *ppt, int *lag);
+void tblock_choice(const jacobi_ctx *h, int *k, int *ppt, int *lag, int *ws);
 int ensure_nccl(jacobi_ctx *h);
 int time_begin(jacobi_ctx *h);
 int time_end(jacobi_ctx *h, int64_t iters);

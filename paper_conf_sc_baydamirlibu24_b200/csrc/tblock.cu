@@ -920,7 +920,7 @@ __device__ __forceinline__ double2 ldcg2(const double *p) { return __ldcg(reinte
 // neighbours are the march's registers) and 2.5 in 3D, and every store is a 16-byte store into
 // the local scratch / next buffer and, for the outermost plane, straight into the neighbour's
 // slot or halo.  Same oracle order; cells outside the interior keep level m-1.
-template <int DIM, int K, int M>
+template <int DIM, int K, int M, int NT>
 __device__ __forceinline__ void tb_edge_phase(const JbGeom &g, bool top, int64_t C, const double *cur, double *E,
                                               double *nxt, double *mid, double *remote, int ub, int ue) {
   constexpr int NP = M < K ? 2 * K - M : K;  // level-M planes of this side
@@ -965,7 +965,7 @@ __device__ __forceinline__ void tb_edge_phase(const JbGeom &g, bool top, int64_t
     const int xp0 = (xa & 1) ? xa : xa - 1;  // first pair (x odd: 16-byte aligned)
     const int npx = (xb - xp0) / 2 + 1;
     const int items = npx * (yb - ya + 1);
-    for (int c = threadIdx.x; c < items; c += blockDim.x) {
+    for (int c = threadIdx.x; c < items; c += NT) {
       const int ry = DIM == 3 ? c / npx : 0;
       const int x = xp0 + 2 * (c - ry * npx), y = ya + ry;
       const int64_t e = (DIM == 3 ? (int64_t)y * pitch : 0) + x;
@@ -1006,7 +1006,9 @@ __device__ __forceinline__ void tb_edge_phase(const JbGeom &g, bool top, int64_t
 
 // Not inlined: its fully unrolled phases would otherwise raise the register pressure of the
 // interior march they share the kernel with (measured: spills in the hot loop).
-template <int DIM, int K>
+// Run by the consumer warps (threads 0 .. NT-1) only, ordered among themselves by named barrier
+// 2; the producer warp meanwhile already streams the block's interior rows.
+template <int DIM, int K, int NT>
 __device__ __noinline__ bool tb_edge(const JbGeom &g, const JbSlab &SL, const JbParams &P, int role, int ridx, int rcount,
                         const double *cur, double *nxt, double *remote, int64_t tg, int *s_flag) {
   const bool top = role == ROLE_TOP;
@@ -1020,6 +1022,7 @@ __device__ __noinline__ bool tb_edge(const JbGeom &g, const JbSlab &SL, const Jb
   const int tid = threadIdx.x;
   const bool drop = (P.flags & JACOBI_FLAG_DROP_SIGNAL) && SL.slab_id == 0;
   const int side = top ? 0 : 1;
+  auto bar_edge = [] { asm volatile("bar.sync 2, %0;" ::"n"(NT) : "memory"); };
   const bool mark = ridx == 0 && tid == 0;
   auto wait = [&](unsigned long long target) {
     if (tid < 32) {
@@ -1028,27 +1031,33 @@ __device__ __noinline__ bool tb_edge(const JbGeom &g, const JbSlab &SL, const Jb
       if (tid == 0) *s_flag = ok ? 0 : 1;
       if (mark) halo_mark(SL, P, side, (int64_t)target - P.t0, 1);
     }
-    __syncthreads();
+    bar_edge();
     return *s_flag == 0;
   };
 #pragma unroll
   for (int m = 1; m <= K; ++m) {
     if (!wait((unsigned long long)(tg + m - 1))) return false;
     // level m (compile-time per phase: the march and its loads are fully unrolled)
-    if (m == 1) tb_edge_phase<DIM, K, 1>(g, top, C, cur, E, nxt, mid, remote, ub, ue);
-    if constexpr (K >= 2) if (m == 2) tb_edge_phase<DIM, K, 2>(g, top, C, cur, E, nxt, mid, remote, ub, ue);
-    if constexpr (K >= 3) if (m == 3) tb_edge_phase<DIM, K, 3>(g, top, C, cur, E, nxt, mid, remote, ub, ue);
-    if constexpr (K >= 4) if (m == 4) tb_edge_phase<DIM, K, 4>(g, top, C, cur, E, nxt, mid, remote, ub, ue);
-    if constexpr (K >= 5) if (m == 5) tb_edge_phase<DIM, K, 5>(g, top, C, cur, E, nxt, mid, remote, ub, ue);
-    __syncthreads();  // every thread's stores (local, neighbour's) precede the release below
+    if (m == 1) tb_edge_phase<DIM, K, 1, NT>(g, top, C, cur, E, nxt, mid, remote, ub, ue);
+    if constexpr (K >= 2) if (m == 2) tb_edge_phase<DIM, K, 2, NT>(g, top, C, cur, E, nxt, mid, remote, ub, ue);
+    if constexpr (K >= 3) if (m == 3) tb_edge_phase<DIM, K, 3, NT>(g, top, C, cur, E, nxt, mid, remote, ub, ue);
+    if constexpr (K >= 4) if (m == 4) tb_edge_phase<DIM, K, 4, NT>(g, top, C, cur, E, nxt, mid, remote, ub, ue);
+    if constexpr (K >= 5) if (m == 5) tb_edge_phase<DIM, K, 5, NT>(g, top, C, cur, E, nxt, mid, remote, ub, ue);
+    bar_edge();  // every thread's stores (local, neighbour's) precede the release below
     if (tid == 0 && !drop) st_release_sys(fout, (unsigned long long)(tg + m));
     if (mark) halo_mark(SL, P, side, tg + m - 1 - P.t0, 2);
   }
   return true;
 }
 
-template <int NCW, int DIM, int K, int TP, int LAG, int RPW>
+// WS = 1: warp-specialised register split — 4 + NCW warps, the last warpgroup (warp NCW = the
+// producer, three idle warps) gives registers back with setmaxnreg.dec and the NCW consumer
+// warps (whole warpgroups) take them with setmaxnreg.inc: 12 compute warps at 160 registers
+// where one producer warp per CTA would leave 11 at 168 (each SM sub-partition holds 16 K
+// registers: 32 + 3 x 160 = 512 per lane slot).
+template <int NCW, int DIM, int K, int TP, int LAG, int RPW, int WS = 0>
 __device__ __forceinline__ void tb_body(const JbParams &P) {
+  static_assert(!WS || NCW % 4 == 0, "warp specialisation needs whole consumer warpgroups");
   static_assert(K == 2 || (K & 1), "K = 2 or odd");
   extern __shared__ __align__(128) unsigned char smem[];
   __shared__ int s_abort;
@@ -1079,6 +1088,7 @@ __device__ __forceinline__ void tb_body(const JbParams &P) {
 
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const bool producer = warp == NCW;
+  const bool consumer = warp < NCW;  // (WS: warps NCW+1 .. NCW+3 are idle)
   if (threadIdx.x == 0) {
     for (uint32_t i = 0; i < R.S; ++i) {
       mbar_init(&R.full[i], 1);
@@ -1092,20 +1102,29 @@ __device__ __forceinline__ void tb_body(const JbParams &P) {
     s_abort = 0;
   }
   __syncthreads();
-
   const int64_t C = SL.chunk;
   const int64_t nblocks = P.iters / K;
   RingPos q = {0u, 0u}, rq = {0u, 0u};
-  for (int64_t j = 0; j < nblocks; ++j) {
-    const double *cur = SL.buf[(P.t0 + j) & 1];
-    double *nxt = SL.buf[(P.t0 + j + 1) & 1];
-    const int64_t tg = P.t0 + K * j;  // global iteration at the start of this time block
-    if (role != ROLE_INT) {  // edge zone with its per-iteration exchange, then help the interior
-      double *remote = role == ROLE_TOP ? SL.peer_top[(P.t0 + j + 1) & 1] : SL.peer_bot[(P.t0 + j + 1) & 1];
-      if (!tb_edge<DIM, K>(g, SL, P, role, ridx, rcount, cur, nxt, remote, tg, &s_edge)) return;
-      fence_proxy_async_global();  // our generic-proxy stores before later bulk reads
-    }
-    if (producer) {
+  // The time blocks.  RG = which warps run this copy of the loop: 0 every warp (WS = 0), 1 the
+  // producer warpgroup, 2 the consumer warps (WS = 1: two separate loops, so the register limits
+  // of setmaxnreg apply to whole code regions; both meet at the same grid-barrier bar.sync 0).
+  auto blocks = [&](auto rg_ct) {
+    constexpr int RG = decltype(rg_ct)::value;
+    for (int64_t j = 0; j < nblocks; ++j) {
+      const double *cur = SL.buf[(P.t0 + j) & 1];
+      double *nxt = SL.buf[(P.t0 + j + 1) & 1];
+      const int64_t tg = P.t0 + K * j;  // global iteration at the start of this time block
+      if constexpr (RG != 1) {
+        if (role != ROLE_INT && consumer) {  // edge zone with its per-iteration exchange, then help the interior
+          double *remote = role == ROLE_TOP ? SL.peer_top[(P.t0 + j + 1) & 1] : SL.peer_bot[(P.t0 + j + 1) & 1];
+          // (a watchdog timeout inside raises the abort flag: the consumers still drain this block's
+          // interior items, so the producer never blocks, and the grid barrier below ends the run)
+          tb_edge<DIM, K, NCW * 32>(g, SL, P, role, ridx, rcount, cur, nxt, remote, tg, &s_edge);
+          fence_proxy_async_global();  // our generic-proxy stores before later bulk reads
+        }
+      }
+      if constexpr (RG != 2) {
+        if (producer) {
       fence_proxy_async_global();
       if (lane == 0 && c == 0) SL.work_ctr[(j + 1) & 1] = 0u;  // idle since block j-1
       // Guided self-scheduling over (plane block, strip) items, as jb_sweep.
@@ -1193,7 +1212,10 @@ __device__ __forceinline__ void tb_body(const JbParams &P) {
         mbar_arrive(&qfull[rq.slot]);
       }
       rq.advance(JB_RQ);
-    } else {
+        }
+      }
+      if constexpr (RG != 1) {
+        if (consumer) {
       while (true) {
         mbar_wait(&qfull[rq.slot], rq.phase);
         const TbDesc d = desc[rq.slot];
@@ -1209,21 +1231,36 @@ __device__ __forceinline__ void tb_body(const JbParams &P) {
         else tbk_item<K, TP, LAG>(g, R, q, d.unit, d.a, d.b, C, nxt, warp, lane);
       }
       fence_proxy_async_global();  // generic-proxy stores before the next block's bulk reads
+        }
+      }
+      // Device-side grid barrier between time blocks.
+      __syncthreads();
+      if (threadIdx.x == 0) {
+        red_release_gpu_add(SL.barrier, 1ull);
+        const bool okb = wait_geq<false>(SL.barrier, (unsigned long long)SL.cta_count * (j + 1), P);
+        s_abort = (!okb || *(volatile int *)(P.status + 1)) ? 1 : 0;
+      }
+      __syncthreads();
+      if (s_abort) return;
     }
-    // Device-side grid barrier between time blocks.
-    __syncthreads();
-    if (threadIdx.x == 0) {
-      red_release_gpu_add(SL.barrier, 1ull);
-      const bool okb = wait_geq<false>(SL.barrier, (unsigned long long)SL.cta_count * (j + 1), P);
-      s_abort = (!okb || *(volatile int *)(P.status + 1)) ? 1 : 0;
+    // End of run: the neighbour's last halo has landed before the kernel completes (as jb_sweep).
+    if constexpr (RG != 1) {
+      if (role != ROLE_INT && warp == 0 && nblocks > 0) {
+        if (role == ROLE_TOP) wait_slots(SL.flag_in_top, SL.k_in_top, (unsigned long long)(P.t0 + P.iters), P, lane);
+        else wait_slots(SL.flag_in_bot, SL.k_in_bot, (unsigned long long)(P.t0 + P.iters), P, lane);
+      }
     }
-    __syncthreads();
-    if (s_abort) return;
-  }
-  // End of run: the neighbour's last halo has landed before the kernel completes (as jb_sweep).
-  if (role != ROLE_INT && warp == 0 && nblocks > 0) {
-    if (role == ROLE_TOP) wait_slots(SL.flag_in_top, SL.k_in_top, (unsigned long long)(P.t0 + P.iters), P, lane);
-    else wait_slots(SL.flag_in_bot, SL.k_in_bot, (unsigned long long)(P.t0 + P.iters), P, lane);
+  };
+  if constexpr (WS) {
+    if (consumer) {
+      asm volatile("setmaxnreg.inc.sync.aligned.u32 160;" ::: "memory");
+      blocks(std::integral_constant<int, 2>{});
+    } else {
+      asm volatile("setmaxnreg.dec.sync.aligned.u32 32;" ::: "memory");
+      blocks(std::integral_constant<int, 1>{});
+    }
+  } else {
+    blocks(std::integral_constant<int, 0>{});
   }
 }
 
@@ -1233,6 +1270,11 @@ __device__ __forceinline__ void tb_body(const JbParams &P) {
 template <int DIM, int K, int TP, int NCW = JB_NCW, int LAG = 1, int RPW = 1>
 __global__ void __launch_bounds__((NCW + 1) * 32, 1) jb_tblock(const __grid_constant__ JbParams P) {
   tb_body<NCW, DIM, K, TP, LAG, RPW>(P);
+}
+// warp-specialised register split (tb_body WS = 1): NCW consumer warps + one producer warpgroup
+template <int DIM, int K, int TP, int NCW, int LAG = 1, int RPW = 1>
+__global__ void __launch_bounds__(NCW * 32 + 128, 1) jb_tblock_ws(const __grid_constant__ JbParams P) {
+  tb_body<NCW, DIM, K, TP, LAG, RPW, 1>(P);
 }
 template <int TP>
 __global__ void __maxnreg__(96) jb_tblock2d_x2(const __grid_constant__ JbParams P) {
@@ -1244,9 +1286,14 @@ constexpr int TB_TY = 4;  // 3D tile rows (level-1 rows TY+2 carried per plane i
 // Kernel for (dim, K, pairs per thread, wavefront lag, CTAs per SM) and its consumer warp count;
 // nullptr if not instantiated.  Odd K holds (LAG+2)(K-1) level rows per lane: beyond ~168
 // registers, i.e. 7 consumer warps (256 threads: up to 255 registers).
-const void *tblock_fn(int dim, int k, int ppt, int lag, int per_sm, int *ncw) {
 #define JB_TB(...) reinterpret_cast<const void *>(&__VA_ARGS__)
+const void *tblock_fn_plain(int dim, int k, int ppt, int lag, int per_sm, int ws, int *ncw) {
   *ncw = JB_NCW;
+  if (ws) {  // warp-specialised register split: 2D K = 5, one pair per lane, 12 consumer warps
+    *ncw = 12;
+    if (dim == 2 && k == 5 && ppt == 1 && lag == 1 && per_sm == 1) return JB_TB(jb_tblock_ws<2, 5, 1, 12, 1>);
+    return nullptr;
+  }
   if (dim == 3) {
     if (k == 2) return JB_TB(jb_tblock<3, 2, TB_TY>);
     // odd K: (K, PPT, RPW = `lag`) -> NCW consumer warps x RPW rows per tile
@@ -1276,7 +1323,13 @@ const void *tblock_fn(int dim, int k, int ppt, int lag, int per_sm, int *ncw) {
   if (k == 3 && ppt == 4) return JB_TB(jb_tblock<2, 3, 4, 7>);
   if (k == 5 && ppt == 2) return JB_TB(jb_tblock<2, 5, 2, 7>);
   return nullptr;
+}
 #undef JB_TB
+// ... and its block size: the consumer warps + one producer warp (WS: + a producer warpgroup).
+const void *tblock_fn(int dim, int k, int ppt, int lag, int per_sm, int ws, int *ncw, int *threads) {
+  const void *fn = tblock_fn_plain(dim, k, ppt, lag, per_sm, ws, ncw);
+  *threads = (*ncw + (ws ? 4 : 1)) * 32;
+  return fn;
 }
 
 }  // namespace
@@ -1285,9 +1338,9 @@ namespace jbk {
 
 int tblock_ty() { return TB_TY; }
 // consumer warps of the kernel for (dim, k, ppt) with one CTA per SM; 0 if not instantiated
-int tblock_ncw(int dim, int k, int ppt, int lag, int per_sm) {
-  int ncw = 0;
-  return tblock_fn(dim, k, ppt, lag, per_sm, &ncw) ? ncw : 0;
+int tblock_ncw(int dim, int k, int ppt, int lag, int per_sm, int ws) {
+  int ncw = 0, threads = 0;
+  return tblock_fn(dim, k, ppt, lag, per_sm, ws, &ncw, &threads) ? ncw : 0;
 }
 
 // Dynamic shared memory of the temporally blocked kernel: header + ring stages (+ the 3D
@@ -1297,24 +1350,25 @@ size_t tblock_smem(const JbGeom &g) {
   return (hdr + 127) / 128 * 128 + (size_t)g.stages * g.stage_doubles * 8 + (size_t)g.xch_doubles * 8;
 }
 
-cudaError_t prepare_tblock(const JbGeom &g, int k, int ppt, int lag, int per_sm, size_t smem, int *blocks_per_sm) {
-  int ncw = 0;
-  const void *fn = tblock_fn(g.dim, k, ppt, lag, per_sm, &ncw);
+cudaError_t prepare_tblock(const JbGeom &g, int k, int ppt, int lag, int per_sm, int ws, size_t smem,
+                           int *blocks_per_sm) {
+  int ncw = 0, threads = 0;
+  const void *fn = tblock_fn(g.dim, k, ppt, lag, per_sm, ws, &ncw, &threads);
   if (!fn) return cudaErrorInvalidValue;
   cudaError_t e = cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
   if (e != cudaSuccess) return e;
   e = cudaFuncSetAttribute(fn, cudaFuncAttributePreferredSharedMemoryCarveout, (int)cudaSharedmemCarveoutMaxShared);
   if (e != cudaSuccess) return e;
-  return cudaOccupancyMaxActiveBlocksPerMultiprocessor(blocks_per_sm, fn, (ncw + 1) * 32, smem);
+  return cudaOccupancyMaxActiveBlocksPerMultiprocessor(blocks_per_sm, fn, threads, smem);
 }
 
-cudaError_t launch_tblock(const JbParams &p, int k, int ppt, int lag, int per_sm, int grid, size_t smem,
+cudaError_t launch_tblock(const JbParams &p, int k, int ppt, int lag, int per_sm, int ws, int grid, size_t smem,
                           cudaStream_t st) {
   void *args[] = {const_cast<JbParams *>(&p)};
-  int ncw = 0;
-  const void *fn = tblock_fn(p.g.dim, k, ppt, lag, per_sm, &ncw);
+  int ncw = 0, threads = 0;
+  const void *fn = tblock_fn(p.g.dim, k, ppt, lag, per_sm, ws, &ncw, &threads);
   if (!fn) return cudaErrorInvalidValue;
-  return cudaLaunchCooperativeKernel(fn, dim3(grid), dim3((ncw + 1) * 32), args, smem, st);
+  return cudaLaunchCooperativeKernel(fn, dim3(grid), dim3(threads), args, smem, st);
 }
 
 }  // namespace jbk

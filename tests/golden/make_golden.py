@@ -3,7 +3,11 @@
 PAPER.md prints no numeric results and no worked example (its figures are images), so
 these fixtures are oracle regression anchors: SHA-256 digests of the bit patterns of oracle runs on
 the BASELINE.json workloads' small configs, plus a few sampled cell values for readability.
-Run:  python tests/golden/make_golden.py
+Run:  python tests/golden/make_golden.py          (small cases, seconds; re-derived by the CPU suite)
+      python tests/golden/make_golden.py --full   (C2 16384^2 and C3 512^3 at 1000 iterations, the
+                                                   full BASELINE.json workloads: ~0.3-1 h of CPU;
+                                                   too slow for the CPU suite, which re-derives the
+                                                   small cases only)
 """
 import hashlib
 import json
@@ -26,6 +30,14 @@ CASES = {
 }
 
 
+# Full-size workloads (BASELINE.json configs[1], configs[2]) at their 1000 iterations: the GPU
+# suite compares the CUDA path's whole field against these digests (full-length parity).
+FULL = {
+    "c2_2d_16384x16384_u12_5c24_1000it": ((16384, 16384), 1000),
+    "c3_3d_512x512x512_u12_5c24_1000it": ((512, 512, 512), 1000),
+}
+
+
 def digest(a: np.ndarray) -> str:
     return hashlib.sha256(np.ascontiguousarray(a, dtype=np.float64).tobytes()).hexdigest()
 
@@ -35,14 +47,16 @@ def compute(shape, iters):
 
 
 def main():
+    full = "--full" in sys.argv
     out = {}
-    for name, (shape, iters) in CASES.items():
+    for name, (shape, iters) in (FULL if full else CASES).items():
         r = compute(shape, iters)
         mid = tuple(s // 2 for s in shape)
         out[name] = {"shape": list(shape), "iters": iters, "seed": SEED_BENCH, "sha256": digest(r),
                      "center_value": float(r[mid]), "mean": float(r.mean()),
                      "generator": "tests/golden/make_golden.py (oracle.jacobi, C oracle)"}
-    with open(os.path.join(HERE, "oracle_digests.json"), "w") as f:
+        print(name, out[name]["sha256"], flush=True)
+    with open(os.path.join(HERE, "oracle_digests_full.json" if full else "oracle_digests.json"), "w") as f:
         json.dump(out, f, indent=1)
     print(json.dumps(out, indent=1))
 

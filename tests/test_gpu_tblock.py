@@ -399,8 +399,9 @@ def test_tblock_3d_invariants_and_mixing():
 
 
 def test_tblock_3d_auto_selection():
-    """3D auto: time-blocked K = 3 for a slab without neighbours, per-iteration with neighbours
-    (whole-plane edge zones measured slower there)."""
+    """3D auto: time-blocked K = 3 for a slab without neighbours and for slabs with neighbours
+    that have >= 64 CTAs each (a GPU per slab, or 2 virtual slabs); per-iteration when 4+ virtual
+    slabs share one GPU (whole-plane edge zones on too few CTAs measured slower there)."""
     with jb.Jacobi((20, 30, 40)) as j:
         j.set_param("resident", 0)
         j.run(8)
@@ -408,7 +409,14 @@ def test_tblock_3d_auto_selection():
     with jb.Jacobi((20, 30, 40), virtual=2) as j:
         j.set_param("resident", 0)
         j.run(8)
+        assert j.get_param("last_tblock") == 6 and j.get_param("last_tb_k") == K3_AUTO
+    f = u12((50, 30, 40), 3)
+    with jb.Jacobi(f.shape, virtual=4) as j:
+        j.set_param("resident", 0)
+        j.scatter(f)
+        j.run(8)
         assert j.get_param("last_tblock") == 0
+        assert_bitwise(j.gather(), oracle.jacobi(f, 8), "3D auto, 4 virtual slabs")
 
 
 def test_c3_1000_iters_tblock_equals_per_iteration():
