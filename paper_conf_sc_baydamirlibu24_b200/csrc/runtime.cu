@@ -734,7 +734,7 @@ int run_tblock(jacobi_ctx *h, int64_t iters, int K, int ppt, int lag, int ws) {
     if (rc) return rc;
     JbGeom &g = L.P.g;
     if (h->dim == 3 && K > 2) {  // odd K: NCW warps x RPW rows x 64 ppt columns, outputs shrink by 2(K-1)
-      const int ncw = jbk::tblock_ncw(3, K, ppt, lag, 1), ty_all = ncw * lag;
+      const int ncw = jbk::tblock_ncw(3, K, ppt, lag, 1, ws), ty_all = ncw * lag;
       g.tx = 64 * ppt - 2 * (K - 1);
       g.ty = ty_all - 2 * (K - 1);
       g.rh = ty_all + 2;

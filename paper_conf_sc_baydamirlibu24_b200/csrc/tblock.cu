@@ -1289,9 +1289,12 @@ constexpr int TB_TY = 4;  // 3D tile rows (level-1 rows TY+2 carried per plane i
 #define JB_TB(...) reinterpret_cast<const void *>(&__VA_ARGS__)
 const void *tblock_fn_plain(int dim, int k, int ppt, int lag, int per_sm, int ws, int *ncw) {
   *ncw = JB_NCW;
-  if (ws) {  // warp-specialised register split: 2D K = 5, one pair per lane, 12 consumer warps
+  if (ws) {  // warp-specialised register split, 12 consumer warps: 2D K = 5, one pair per lane;
+             // 3D K = 3, one pair per lane, 2 rows per warp (tiles of 24 rows: 20 output rows)
     *ncw = 12;
-    if (dim == 2 && k == 5 && ppt == 1 && lag == 1 && per_sm == 1) return JB_TB(jb_tblock_ws<2, 5, 1, 12, 1>);
+    if (per_sm != 1) return nullptr;
+    if (dim == 2 && k == 5 && ppt == 1 && lag == 1) return JB_TB(jb_tblock_ws<2, 5, 1, 12, 1>);
+    if (dim == 3 && k == 3 && ppt == 1 && lag == 2) return JB_TB(jb_tblock_ws<3, 3, 1, 12, 1, 2>);
     return nullptr;
   }
   if (dim == 3) {

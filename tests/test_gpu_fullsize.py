@@ -6,7 +6,11 @@
   faces are > k cells away reproduces those cells bit for bit (light-cone sampling).
 * C3 (3D 512^3): 5 iterations cell-for-cell; 1000 iterations P = 8 virtual slabs bit-identical
   to P = 1 and to the CPU-controlled baseline (decomposition invariance).
-* C4 (weak scaling, P = 2 shape 1024x512x512): P = 2 slabs == P = 1.
+* C4 (weak scaling, P = 2 shape 1024x512x512): P = 2 slabs == P = 1; the P = 8 shape
+  (4096x512x512, 8 GiB per buffer): 8 virtual slabs == 1 slab.
+* Full length, whole field: C2 and C3 after 1000 iterations (the bench launch configuration,
+  1 slab and 8 virtual slabs) against the SHA-256 digests of the oracle's own 1000-iteration runs
+  (tests/golden/oracle_digests_full.json, written by make_golden.py --full from oracle/ only).
 """
 import os
 
@@ -99,3 +103,36 @@ def test_c4_weak_p2_shape():
     shape = (1024, 512, 512)
     ref = run(shape, 50)
     assert bits_equal(run(shape, 50, virtual=2), ref)
+
+
+def _digest(a):
+    import hashlib
+    return hashlib.sha256(np.ascontiguousarray(a).tobytes()).hexdigest()
+
+
+def _full_golden():
+    import json
+    with open(os.path.join(os.path.dirname(__file__), "golden", "oracle_digests_full.json")) as f:
+        return json.load(f)
+
+
+@pytest.mark.parametrize("name", ["c2_2d_16384x16384_u12_5c24_1000it", "c3_3d_512x512x512_u12_5c24_1000it"])
+@pytest.mark.parametrize("virtual", [0, 8])
+def test_full_length_whole_field_vs_oracle_digest(name, virtual):
+    """Every cell of C2 / C3 after 1000 iterations == the oracle, bit for bit (P:355 fixed count):
+    the device initialises the same U12 field (seed 0x5C24), runs the benchmark's kernel choice
+    (time-blocked K = 5 / K = 3; edge zones between 8 virtual slabs), and the digest of the gathered
+    field must equal the digest of the oracle's run."""
+    g = _full_golden()[name]
+    with jb.Jacobi(tuple(g["shape"]), virtual=virtual) as j:
+        j.run(g["iters"])
+        assert j.get_param("last_tblock") > 0  # the time-blocked kernel the benchmark runs
+        got = j.gather()
+    assert _digest(got) == g["sha256"], f"{name} virtual={virtual}"
+
+
+def test_c4_weak_p8_shape_virtual8_equals_one_slab():
+    """C4 at P = 8 (512x512x4096, 8 GiB per buffer): 8 virtual slabs == 1 slab after 30 iterations."""
+    shape = (4096, 512, 512)
+    ref = run(shape, 30)
+    assert bits_equal(run(shape, 30, virtual=8), ref)
