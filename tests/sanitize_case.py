@@ -28,7 +28,11 @@ for shape, P in [((20, 70), 2), ((8, 9, 33), 2), ((30, 40), 1)]:
 for shape, P, prm in [((24, 70), 2, {}), ((20, 70), 2, {"tb_k": 2}), ((12, 9, 33), 2, {}),
                       ((12, 9, 33), 1, {}), ((12, 9, 33), 1, {"tb_k": 2}), ((30, 40), 1, {}),
                       ((30, 40), 1, {"tb_k": 3}), ((30, 40), 1, {"tb_k": 5, "tb_ppt": 2}),
-                      ((30, 40), 1, {"stages": 4}), ((30, 40), 1, {"tb_k": 2, "stages": 4})]:
+                      ((30, 40), 1, {"stages": 4}), ((30, 40), 1, {"tb_k": 2, "stages": 4}),
+                      # without the warp-specialised register split (the default uses it for
+                      # 2D K = 5 and 3D K = 3), and 3D edge zones between virtual slabs
+                      ((30, 40), 1, {"tb_ws": 0}), ((24, 70), 2, {"tb_ws": 0}), ((12, 9, 33), 1, {"tb_ws": 0}),
+                      ((16, 9, 33), 2, {"tb_ws": 0})]:
     f = u12(shape, 4)
     with jb.Jacobi(shape, virtual=P) if P > 1 else jb.Jacobi(shape) as j:
         j.set_param("tblock", 1)
