@@ -4,11 +4,13 @@
 launch per iteration + cudaMemcpyPeerAsync halo copies + host synchronisation), with
 and without compute (the "no compute" runs of P:238-241), at P = 2/4/8 slabs.
 
-On a 1-GPU box the P slabs are VIRTUAL (jacobi_create_virtual: P slab groups of thread blocks
-on one device running the complete flag/halo protocol; the baseline launches P kernels and
-2(P-1) peer copies per iteration on the same device).  This measures the orchestration cost
-(launch + host sync vs device flags + grid barrier) that the paper's claim is about; it does
-not exercise NVLink.  Per-iteration time = (T(2N) - T(N)) / N, cancelling launch skew.
+With at least P visible GPUs the P slabs live on P PHYSICAL devices (jacobi_create(ngpus=P): UVA
+peer stores over NVLink, NCCL send/recv for the NCCL baseline).  On a box with fewer GPUs they are
+VIRTUAL (jacobi_create_virtual: P slab groups of thread blocks on one device running the complete
+flag/halo protocol; the baseline launches P kernels and 2(P-1) peer copies per iteration on the
+same device) — that measures the orchestration cost (launch + host sync vs device flags + grid
+barrier) the paper's claim is about, not NVLink.  Every row says which (`virtual`).  Per-iteration
+time = (T(2N) - T(N)) / N, cancelling launch skew; median of 5.
 
     python bench_latency.py [--iters N] [--out profiles/latency.json]
 """
@@ -44,6 +46,14 @@ def per_iter_us(j: jb.Jacobi, n: int, reps: int = 5) -> float:
     return vals[len(vals) // 2]
 
 
+def n_devices() -> int:
+    try:
+        import torch
+        return torch.cuda.device_count()
+    except Exception:
+        return 1
+
+
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--iters", type=int, default=500)
@@ -51,15 +61,18 @@ def main():
     ap.add_argument("--out", default="")
     args = ap.parse_args()
     rows = []
+    ndev = n_devices()
     for name, shape in SHAPES.items():
         for P in [int(p) for p in args.slabs.split(",")]:
-            with jb.Jacobi(shape, virtual=P) if P > 1 else jb.Jacobi(shape) as j:
-                for mname, mode in MODES.items():
+            real = P == 1 or ndev >= P
+            modes = dict(MODES, **({"baseline_nccl": jb.MODE_BASELINE_NCCL} if real else {}))
+            with jb.Jacobi(shape, ngpus=P) if real else jb.Jacobi(shape, virtual=P) as j:
+                for mname, mode in modes.items():
                     for nocomp in (False, True):
                         j.set_mode(mode, jb.FLAG_NO_COMPUTE if nocomp else 0)
                         j.run(50)  # warm-up
                         us = per_iter_us(j, args.iters)
-                        row = {"config": name, "slabs": P, "virtual": P > 1, "mode": mname,
+                        row = {"config": name, "slabs": P, "virtual": not real, "mode": mname,
                                "no_compute": nocomp, "us_per_iter": round(us, 3)}
                         if mname == "cpufree" and not nocomp:
                             row["kernel"] = ("resident" if j.get_param("last_resident") else
@@ -74,11 +87,13 @@ def main():
     for r in rows:
         if r["mode"] != "cpufree":
             continue
-        for bname in MODES:
+        for bname in list(MODES) + ["baseline_nccl"]:
             if bname == "cpufree":
                 continue
-            b = next(x for x in rows if x["mode"] == bname and x["config"] == r["config"]
-                     and x["slabs"] == r["slabs"] and x["no_compute"] == r["no_compute"])
+            b = next((x for x in rows if x["mode"] == bname and x["config"] == r["config"]
+                      and x["slabs"] == r["slabs"] and x["no_compute"] == r["no_compute"]), None)
+            if b is None:
+                continue
             summary.append({"config": r["config"], "slabs": r["slabs"], "no_compute": r["no_compute"],
                             "baseline": bname, "cpufree_us": r["us_per_iter"], "baseline_us": b["us_per_iter"],
                             "reduction_pct": (round(100 * (b["us_per_iter"] - r["us_per_iter"]) / b["us_per_iter"], 1)
@@ -89,7 +104,8 @@ def main():
     if args.out:
         with open(args.out, "w") as f:
             json.dump({"rows": rows, "summary": summary,
-                       "note": "virtual slabs on one B200 (see module docstring); paper's 58.8% (8xA100) is context only"},
+                       "gpus_visible": ndev,
+                       "note": "rows with virtual=true: P slabs on one B200 (module docstring); paper's 58.8% (8xA100) is context only"},
                       f, indent=1)
 
 

@@ -117,18 +117,22 @@ def _full_golden():
 
 
 @pytest.mark.parametrize("name", ["c2_2d_16384x16384_u12_5c24_1000it", "c3_3d_512x512x512_u12_5c24_1000it"])
-@pytest.mark.parametrize("virtual", [0, 8])
-def test_full_length_whole_field_vs_oracle_digest(name, virtual):
+@pytest.mark.parametrize("virtual,params", [(0, {}), (8, {}), (8, {"tblock": 1}), (2, {"tb_ws": 0})])
+def test_full_length_whole_field_vs_oracle_digest(name, virtual, params):
     """Every cell of C2 / C3 after 1000 iterations == the oracle, bit for bit (P:355 fixed count):
     the device initialises the same U12 field (seed 0x5C24), runs the benchmark's kernel choice
-    (time-blocked K = 5 / K = 3; edge zones between 8 virtual slabs), and the digest of the gathered
-    field must equal the digest of the oracle's run."""
+    (1 slab: time-blocked K = 5 / K = 3, warp-specialised), 8 virtual slabs (auto: 2D time-blocked
+    with edge zones, 3D per-iteration; forced: 3D time-blocked with edge zones), 2 virtual slabs
+    without the register split; the digest of the gathered field must equal the oracle's."""
     g = _full_golden()[name]
     with jb.Jacobi(tuple(g["shape"]), virtual=virtual) as j:
+        for k, v in params.items():
+            j.set_param(k, v)
         j.run(g["iters"])
-        assert j.get_param("last_tblock") > 0  # the time-blocked kernel the benchmark runs
+        if virtual == 0 or params.get("tblock") == 1 or name.startswith("c2"):
+            assert j.get_param("last_tblock") > 0  # the time-blocked kernel the benchmark runs
         got = j.gather()
-    assert _digest(got) == g["sha256"], f"{name} virtual={virtual}"
+    assert _digest(got) == g["sha256"], f"{name} virtual={virtual} {params}"
 
 
 def test_c4_weak_p8_shape_virtual8_equals_one_slab():
