@@ -886,9 +886,14 @@ int run_cpufree(jacobi_ctx *h, int64_t iters) {
     // odd K: any block count; K = 2: an even one (the result stays in buf[t & 1], R10)
     const int64_t step = (K & 1) ? K : 2 * K;
     tb_iters = iters / step * step;
-    // auto: slabs that fit on chip run the resident kernel (faster for those small grids);
-    // decided over every slab of the run so that all ranks take the same kernel
-    if (h->tblock < 0 && h->resident != 0 && resident_fits_all(h)) tb_iters = 0;
+    // auto: slabs that fit on chip run the resident kernel (faster for those small grids:
+    // C1 2D 256^2 2.2 vs 3.1 us/iteration) — except a single slab of >= 2^18 interior cells,
+    // where the time-blocked kernel's K iterations per barrier win (C5b 2D 1024^2: 3.3 vs 4.6
+    // us/iteration); decided over every slab of the run so that all ranks take
+    // the same kernel
+    const int64_t cells = (h->nx - 2) * (h->dim == 3 ? (h->ny - 2) * (h->nz - 2) : (h->ny - 2));
+    const bool big_single = h->total == 1 && cells >= ((int64_t)1 << 18);
+    if (h->tblock < 0 && h->resident != 0 && !big_single && resident_fits_all(h)) tb_iters = 0;
   }
   double ms = 0;
   if (tb_iters > 0) {

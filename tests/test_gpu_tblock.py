@@ -175,6 +175,12 @@ def test_tblock_auto_selection_and_errors():
         j.set_mode(jb.MODE_CPUFREE, jb.FLAG_NO_COMPUTE)  # no-compute runs keep jb_sweep
         with pytest.raises(jb.JacobiError):
             j.run(4)
+    with jb.Jacobi((1024, 1024)) as j:  # C5b: one slab of >= 2^18 cells prefers time blocking
+        j.run(10)
+        assert j.get_param("last_tblock") == 10 and j.get_param("last_resident") == 0
+    with jb.Jacobi((1024, 1024), virtual=2) as j:  # ... but with neighbours it stays on chip
+        j.run(10)
+        assert j.get_param("last_tblock") == 0 and j.get_param("last_resident") == 1
     with jb.Jacobi((6, 8, 10)) as j:  # 3D with the norm: per-iteration kernels only
         j.set_param("tblock", 1)
         j.set_tolerance(0.0, 2)
