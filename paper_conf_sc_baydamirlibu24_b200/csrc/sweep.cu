@@ -167,7 +167,8 @@ __device__ __forceinline__ void produce_planes(const JbGeom &g, const double *cu
 // plane costs one 16-byte LDS + two 8-byte LDS (x-1, x+2) per pair.
 template <int PPT, bool NOCOMP, bool NORM>
 __device__ __forceinline__ void consume_run_2d(const JbGeom &g, const Ring &R, RingPos &q, const Run &run,
-                                               double *nxt, double *remote, int ctid, int lane, double &acc) {
+                                               const double *cur, double *nxt, double *remote, int ctid, int lane,
+                                               double &acc) {
   const int64_t x0 = 1 + (int64_t)run.unit * g.tx;
   const int vx = (int)min((int64_t)g.tx, g.nx - 1 - x0);
   const int txp = g.tx >> 1;
@@ -183,18 +184,16 @@ __device__ __forceinline__ void consume_run_2d(const JbGeom &g, const Ring &R, R
   }
   const int64_t col = 3 + x0 + 2 * ctid;
   const int64_t L = run.p1 - run.p0 + 1;
-  if (NOCOMP) {
+  if (NOCOMP) {  // no-compute: the owned edge plane goes to the neighbour as-is,
+                 // 16-byte loads straight from the current buffer (L2), no ring stages
     for (int64_t p = 0; p < L; ++p) {
-      R.wait_full(q);
-      const double *sc = R.stage(q) + j0;
+      const double *src = cur + (run.p0 + p) * g.plane_elems + col;
 #pragma unroll
       for (int i = 0; i < PPT; ++i)
         if ((ok >> i & 1u) && remote) {
-          const double2 v = lds2(sc + 2 * i * JB_NC);
+          const double2 v = __ldcg(reinterpret_cast<const double2 *>(src + 2 * i * JB_NC));
           store_pair(remote + col + 2 * i * JB_NC, v.x, v.y, full >> i & 1u);
         }
-      R.release(q, lane);
-      q.advance(R.S);
     }
     return;
   }
@@ -257,7 +256,8 @@ __device__ __forceinline__ void consume_run_2d(const JbGeom &g, const Ring &R, R
 // 16 B (z-1) per pair.
 template <bool NOCOMP, bool NORM>
 __device__ __forceinline__ void consume_run_3d(const JbGeom &g, const Ring &R, RingPos &q, const Run &run,
-                                               double *nxt, double *remote, int ctid, int lane, double &acc) {
+                                               const double *cur, double *nxt, double *remote, int ctid, int lane,
+                                               double &acc) {
   const int ux = run.unit % g.units_x, uy = run.unit / g.units_x;
   const int64_t x0 = 1 + (int64_t)ux * g.tx;
   const int vx = (int)min((int64_t)g.tx, g.nx - 1 - x0);
@@ -274,19 +274,16 @@ __device__ __forceinline__ void consume_run_3d(const JbGeom &g, const Ring &R, R
   const int64_t col = (y0 + rb) * g.pitch + 3 + x0 + 2 * kk;
   const int64_t L = run.p1 - run.p0 + 1;
   const int srow = (rb + 1) * ws + j;  // stage offset of (row rb, pair kk) center
-  if (NOCOMP) {
+  if (NOCOMP) {  // no-compute: the owned edge plane to the neighbour as-is, straight from L2
     for (int64_t p = 0; p < L; ++p) {
-      R.wait_full(q);
       if (remote && ok) {
-        const double *c = R.stage(q) + srow;
+        const double *c = cur + (run.p0 + p) * g.plane_elems + col;
         double *o = remote + col;
-        for (int r = rb; r < re; ++r, c += ws, o += g.pitch) {
-          const double2 v = lds2(c);
+        for (int r = rb; r < re; ++r, c += g.pitch, o += g.pitch) {
+          const double2 v = __ldcg(reinterpret_cast<const double2 *>(c));
           store_pair(o, v.x, v.y, full);
         }
       }
-      R.release(q, lane);
-      q.advance(R.S);
     }
     return;
   }
@@ -348,15 +345,16 @@ __device__ __forceinline__ void consume_run_3d(const JbGeom &g, const Ring &R, R
 
 template <int DIM, bool NOCOMP, bool NORM>
 __device__ __forceinline__ void consume_run(const JbGeom &g, const Ring &R, RingPos &q, const Run &run,
-                                            double *nxt, double *remote, int ctid, int lane, double &acc) {
+                                            const double *cur, double *nxt, double *remote, int ctid, int lane,
+                                            double &acc) {
   if (DIM == 3) {
-    consume_run_3d<NOCOMP, NORM>(g, R, q, run, nxt, remote, ctid, lane, acc);
+    consume_run_3d<NOCOMP, NORM>(g, R, q, run, cur, nxt, remote, ctid, lane, acc);
     return;
   }
   const int ppt = g.tx / (2 * JB_NC);
-  if (ppt >= 4) consume_run_2d<4, NOCOMP, NORM>(g, R, q, run, nxt, remote, ctid, lane, acc);
-  else if (ppt == 2) consume_run_2d<2, NOCOMP, NORM>(g, R, q, run, nxt, remote, ctid, lane, acc);
-  else consume_run_2d<1, NOCOMP, NORM>(g, R, q, run, nxt, remote, ctid, lane, acc);
+  if (ppt >= 4) consume_run_2d<4, NOCOMP, NORM>(g, R, q, run, cur, nxt, remote, ctid, lane, acc);
+  else if (ppt == 2) consume_run_2d<2, NOCOMP, NORM>(g, R, q, run, cur, nxt, remote, ctid, lane, acc);
+  else consume_run_2d<1, NOCOMP, NORM>(g, R, q, run, cur, nxt, remote, ctid, lane, acc);
 }
 
 // ---------------------------------------------------------------- run-descriptor queue
@@ -548,8 +546,7 @@ __global__ void __launch_bounds__(JB_THREADS, 1) jb_sweep(const __grid_constant_
         while (sched.next(run)) {
           if (NOCOMP) {
             wait_flag();  // remote stores of this run must follow the neighbour's signal
-            publish(Q, rq, RUN_WORK, run, lane);
-            produce_planes(g, cur, run.unit, run.p0, run.p1, q, R, lane);
+            publish(Q, rq, RUN_WORK, run, lane);  // (the consumers copy from L2: no stages)
           } else if (role != ROLE_INT) {
             // boundary tile (one plane): halo is p-1 (top) or p+1 (bottom)
             publish(Q, rq, RUN_WORK, run, lane,
@@ -640,7 +637,7 @@ __global__ void __launch_bounds__(JB_THREADS, 1) jb_sweep(const __grid_constant_
         run.p1 = d.p1;
         double acc = 0.0;
         if (NORM && check) {
-          consume_run<DIM, NOCOMP, NORM>(g, R, q, run, nxt, remote, ctid, lane, acc);
+          consume_run<DIM, NOCOMP, NORM>(g, R, q, run, cur, nxt, remote, ctid, lane, acc);
           // deterministic per-run sum: xor tree in each warp, then warps in order
           for (int o = 16; o > 0; o >>= 1) acc = acc + __shfl_xor_sync(0xffffffffu, acc, o);
           if (lane == 0) s_red[warp] = acc;
@@ -652,7 +649,7 @@ __global__ void __launch_bounds__(JB_THREADS, 1) jb_sweep(const __grid_constant_
           }
           named_bar_consumers();
         } else {
-          consume_run<DIM, NOCOMP, false>(g, R, q, run, nxt, remote, ctid, lane, acc);
+          consume_run<DIM, NOCOMP, false>(g, R, q, run, cur, nxt, remote, ctid, lane, acc);
         }
       }
       // Our generic-proxy stores must be ordered before later bulk (async-proxy) reads.

@@ -1233,14 +1233,20 @@ __device__ __forceinline__ void tb_body(const JbParams &P) {
       fence_proxy_async_global();  // generic-proxy stores before the next block's bulk reads
         }
       }
-      // Device-side grid barrier between time blocks.
-      __syncthreads();
+      // Device-side grid barrier between time blocks.  WS: the two warp-role loops reach
+      // it at different instructions, so it is a named barrier over all 16 warps (bar.sync is
+      // aligned per warp only; CUDA's __syncthreads would have to be one instruction).
+      auto cta_sync = [] {
+        if constexpr (WS) asm volatile("bar.sync 3, %0;" ::"n"((NCW + 4) * 32) : "memory");
+        else __syncthreads();
+      };
+      cta_sync();
       if (threadIdx.x == 0) {
         red_release_gpu_add(SL.barrier, 1ull);
         const bool okb = wait_geq<false>(SL.barrier, (unsigned long long)SL.cta_count * (j + 1), P);
         s_abort = (!okb || *(volatile int *)(P.status + 1)) ? 1 : 0;
       }
-      __syncthreads();
+      cta_sync();
       if (s_abort) return;
     }
     // End of run: the neighbour's last halo has landed before the kernel completes (as jb_sweep).
