@@ -183,6 +183,8 @@ int jacobi_set_mode(jacobi_t h, int mode, int flags);
  * kernel), "last_tblock" (iterations of the last CPU-Free run done time-blocked), "last_tb_k"
  * (its K, 0 if none), "last_launches" (kernels this process launched in the last jacobi_run, all
  * GPUs).  Measurement: "halo_trace" (see jacobi_halo_trace; 0 = off, <= 2^20).
+ * "barrier" (the CPU-Free kernels' device-side grid barrier: 0 = one counter per slab with
+ * red.release + acquire spin (default), 1 = per-CTA arrival flags polled in parallel by every CTA).
  * Unknown names return JACOBI_EINVAL. */
 int jacobi_set_param(jacobi_t h, const char *name, int64_t value);
 int jacobi_get_param(jacobi_t h, const char *name, int64_t *value);

@@ -97,10 +97,27 @@ class JacobiError(RuntimeError):
         super().__init__(f"{what}: {strerror(code)} ({code})" if what else f"{strerror(code)} ({code})")
 
 
+def _torch_nccl() -> str | None:
+    """Path of the libnccl.so.2 PyTorch ships (nvidia-nccl wheel), if any — without importing torch."""
+    import importlib.util
+    try:
+        spec = importlib.util.find_spec("nvidia.nccl")
+    except (ImportError, ValueError):
+        return None
+    for base in (spec.submodule_search_locations or []) if spec else []:
+        p = os.path.join(base, "lib", "libnccl.so.2")
+        if os.path.exists(p):
+            return p
+    return None
+
+
 def lib() -> ctypes.CDLL:
     """Load the CUDA extension.  Fails loudly if it has not been built (no fallback)."""
     global _lib
     if _lib is None:
+        nccl = _torch_nccl()  # the NCCL baseline uses the same libnccl as PyTorch (one per process)
+        if nccl and "JACOBI_NCCL_LIB" not in os.environ:
+            os.environ["JACOBI_NCCL_LIB"] = nccl
         if not os.path.exists(LIB_PATH):
             raise RuntimeError(f"CUDA extension missing: {LIB_PATH} (run __graft_entry__.build())")
         L = ctypes.CDLL(LIB_PATH)

@@ -193,6 +193,61 @@ __device__ __forceinline__ void halo_mark(const JbSlab &SL, const JbParams &P, i
     SL.halo_trace[((int64_t)side * P.halo_trace_n + e) * 3 + which] = globaltimer();
 }
 
+__device__ __forceinline__ unsigned long long ld_relaxed_gpu(const unsigned long long *p) {
+  unsigned long long v;
+  asm volatile("ld.relaxed.gpu.global.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
+  return v;
+}
+__device__ __forceinline__ void fence_acq_rel_gpu() { asm volatile("fence.acq_rel.gpu;" ::: "memory"); }
+
+// Device-side grid barrier of a slab's CTAs (P:372 grid.sync()), called by warp 0 of every CTA
+// after a CTA barrier (whose cumulativity puts the whole CTA's writes before the arrival), followed
+// by a CTA barrier.  epoch = the global iteration count after this barrier (unique and increasing
+// across runs); k = the barrier's 1-based index in this launch (counter form).  Two forms:
+//  * counter (default): lane 0 red.release.gpu.add 1 on the slab counter, spins until it reaches
+//    cta_count * k (acquire);
+//  * flags (SL.bar_flags): lane 0 st.release.gpu of the epoch into this CTA's own slot; the warp
+//    polls all cta_count slots with relaxed loads issued in parallel (lane i: slots i, i+32, ..),
+//    then one fence.acq_rel.gpu (the acquire pattern) — no atomic serialised on one L2 address.
+// Returns false on abort / watchdog timeout (as wait_slots).
+__device__ bool slab_barrier(const JbSlab &SL, const JbParams &P, int c, unsigned long long k,
+                             unsigned long long epoch, int lane) {
+  if (!SL.bar_flags) {
+    bool ok = true;
+    if (lane == 0) {
+      red_release_gpu_add(SL.barrier, 1ull);
+      ok = wait_geq<false>(SL.barrier, (unsigned long long)SL.cta_count * k, P);
+    }
+    return __shfl_sync(0xffffffffu, ok ? 1 : 0, 0) != 0;
+  }
+  if (lane == 0) st_release_gpu(SL.bar_flags + c, epoch);
+  const int n = SL.cta_count;
+  const unsigned long long t_start = globaltimer();
+  uint32_t cnt = 0;
+  volatile int *abort_flag = P.status + 1;
+  while (true) {
+    bool mine = true;
+#pragma unroll 4
+    for (int s = lane; s < n; s += 32) mine &= ld_relaxed_gpu(SL.bar_flags + s) >= epoch;
+    if (__all_sync(0xffffffffu, mine)) break;
+    if ((++cnt & 127u) == 0) {
+      int stop = 0;
+      if (lane == 0) {
+        if (*abort_flag) {
+          stop = 1;
+        } else if (globaltimer() - t_start > P.timeout_ns) {
+          atomicCAS(P.status, 0, JACOBI_ETIMEOUT);
+          atomicExch(P.status + 1, 1);
+          stop = 1;
+        }
+      }
+      if (__shfl_sync(0xffffffffu, stop, 0)) return false;
+    }
+  }
+  fence_acq_rel_gpu();
+  return true;
+}
+
 // Position in the shared-memory ring: slot and the parity of the current use of that slot.
 struct RingPos {
   uint32_t slot, phase;

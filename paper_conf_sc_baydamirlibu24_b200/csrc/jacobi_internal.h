@@ -124,6 +124,10 @@ struct JbSlab {
   // the first boundary CTA of each side records %globaltimer at wait begin / flag acquired /
   // signal released: halo_trace[(side * n + e) * 3 + {0, 1, 2}], side 0 = top, 1 = bottom.
   unsigned long long *halo_trace;
+  // Grid barrier with per-CTA arrival flags (knob "barrier" = 1; null: the counter barrier): CTA c
+  // stores the barrier's epoch (the global iteration count after it) into bar_flags[c] and warp 0
+  // of every CTA polls all cta_count flags — no atomic serialised on one address.
+  unsigned long long *bar_flags;
 };
 
 struct JbParams {

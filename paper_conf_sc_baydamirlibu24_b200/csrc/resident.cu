@@ -207,10 +207,9 @@ __global__ void __launch_bounds__(JB_RNT, 1) jb_resident(const __grid_constant__
       if (tid == 0) st_release_gpu(SL.blk_flags + c, (unsigned long long)(tg + 1));
       continue;
     }
-    if (tid == 0) {
-      red_release_gpu_add(SL.barrier, 1ull);
-      const bool ok = wait_geq<false>(SL.barrier, (unsigned long long)SL.cta_count * (t + 1), P);
-      s_abort = (!ok || *(volatile int *)(P.status + 1)) ? 1 : 0;
+    if (tid < 32) {
+      const bool ok = slab_barrier(SL, P, c, (unsigned long long)(t + 1), (unsigned long long)(tg + 1), tid);
+      if (tid == 0) s_abort = (!ok || *(volatile int *)(P.status + 1)) ? 1 : 0;
     }
     __syncthreads();
     if (s_abort) return;

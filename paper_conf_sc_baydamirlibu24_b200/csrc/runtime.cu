@@ -82,6 +82,7 @@ void free_slab(Slab &s, const Allocator &a) {
   if (s.norm_peers) cudaFree(s.norm_peers);
   if (s.tmap) cudaFree(s.tmap);
   if (s.trace) cudaFree(s.trace);
+  if (s.bar_flags) cudaFree(s.bar_flags);
   if (s.ev0) cudaEventDestroy(s.ev0);
   if (s.ev1) cudaEventDestroy(s.ev1);
   if (s.ev_sync) cudaEventDestroy(s.ev_sync);
@@ -558,6 +559,20 @@ int setup_trace(jacobi_ctx *h, LaunchPlan &L) {
     CK(cudaMemsetAsync(s.trace, 0, (size_t)n * 6 * sizeof(unsigned long long), L.stream));
     s.trace_n = n;
     L.P.s[k].halo_trace = s.trace;
+  }
+  // grid-barrier form (knob "barrier"): per-CTA arrival flags, allocated once and zeroed; their
+  // epochs (global iteration counts) only grow, so stale slots never satisfy a later barrier
+  for (size_t k = 0; k < L.slab_idx.size(); ++k) {
+    Slab &s = h->slabs[L.slab_idx[k]];
+    L.P.s[k].bar_flags = nullptr;
+    if (h->barrier != 1) continue;
+    if (L.P.s[k].cta_count > JB_MAX_BLOCKS) return JACOBI_EINVAL;
+    CK(cudaSetDevice(s.device));
+    if (!s.bar_flags) {
+      CK(cudaMalloc(&s.bar_flags, JB_MAX_BLOCKS * sizeof(unsigned long long)));
+      CK(cudaMemset(s.bar_flags, 0, JB_MAX_BLOCKS * sizeof(unsigned long long)));
+    }
+    L.P.s[k].bar_flags = s.bar_flags;
   }
   return JACOBI_OK;
 }
@@ -1042,6 +1057,7 @@ static int64_t *param_slot(jacobi_t h, const char *name) {
   if (!std::strcmp(name, "last_tb_k")) return &h->last_tb_k;
   if (!std::strcmp(name, "last_tblock")) return &h->last_tblock;
   if (!std::strcmp(name, "halo_trace")) return &h->halo_trace;
+  if (!std::strcmp(name, "barrier")) return &h->barrier;
   if (!std::strcmp(name, "last_launches")) return &h->last_launches;
   return nullptr;
 }

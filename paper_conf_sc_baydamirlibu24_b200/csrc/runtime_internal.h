@@ -72,9 +72,14 @@ struct NcclApi {
   ncclResult_t (*GroupEnd)() = nullptr;
   bool load() {
     if (lib) return true;
-    const char *names[] = {"libnccl.so.2", "libnccl.so"};
+    // JACOBI_NCCL_LIB (set by the Python binding to the NCCL that PyTorch ships) first: the
+    // process must not end up with two different libnccl.so.2 — a system NCCL loaded here
+    // first would be reused by a later `import torch` (same soname) and lack its symbols.
+    // Loaded RTLD_LOCAL: the library's symbols are only reached through the pointers below.
+    const char *env = getenv("JACOBI_NCCL_LIB");
+    const char *names[] = {env ? env : "libnccl.so.2", "libnccl.so.2", "libnccl.so"};
     for (const char *n : names) {
-      lib = dlopen(n, RTLD_NOW | RTLD_GLOBAL);
+      lib = dlopen(n, RTLD_NOW | RTLD_LOCAL);
       if (lib) break;
     }
     if (!lib) return false;
@@ -153,6 +158,7 @@ struct Slab {
   double *partials = nullptr;               // N4: per-run partial sums (device)
   int64_t partials_cap = 0;
   JbCtrl **norm_peers = nullptr;            // N4: device array of every slab's control block
+  unsigned long long *bar_flags = nullptr;  // flag-array grid barrier: one slot per CTA (device)
   unsigned long long *trace = nullptr;  // halo-exchange trace of the last CPU-Free run (device)
   int64_t trace_cap = 0;                // its capacity (exchanges per side)
   int64_t trace_n = 0;                  // exchanges per side recorded by the last run (its stride)
@@ -190,6 +196,7 @@ struct jacobi_ctx {
   int64_t last_tb_k = 0;       // read-only: K of the last time-blocked run
   int64_t last_tblock = 0;     // read-only: iterations of the last CPU-Free run done time-blocked
   int64_t last_launches = 0;   // read-only: kernels this process launched in the last jacobi_run
+  int64_t barrier = 0;         // grid barrier of the CPU-Free kernels: 0 counter, 1 per-CTA flags
   int64_t halo_trace = 0;      // measurement: record the first n halo exchanges of each CPU-Free run
                                // (%globaltimer wait begin / flag acquired / signal; jacobi_halo_trace)
   int64_t norm_every = 0;      // N4: check the update norm every k iterations (0 = off)

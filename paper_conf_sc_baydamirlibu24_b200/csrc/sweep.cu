@@ -660,10 +660,9 @@ __global__ void __launch_bounds__(JB_THREADS, 1) jb_sweep(const __grid_constant_
 
     // Device-side grid barrier of this slab's CTAs (P:372 grid.sync()).
     __syncthreads();
-    if (threadIdx.x == 0) {
-      red_release_gpu_add(SL.barrier, 1ull);
-      const bool ok = wait_geq<false>(SL.barrier, (unsigned long long)SL.cta_count * (t + 1), P);
-      s_abort = (!ok || *(volatile int *)(P.status + 1)) ? 1 : 0;
+    if (warp == 0) {
+      const bool ok = slab_barrier(SL, P, c, (unsigned long long)(t + 1), (unsigned long long)(tg + 1), lane);
+      if (lane == 0) s_abort = (!ok || *(volatile int *)(P.status + 1)) ? 1 : 0;
     }
     __syncthreads();
     if (s_abort) return;

@@ -1022,7 +1022,7 @@ __device__ __noinline__ bool tb_edge(const JbGeom &g, const JbSlab &SL, const Jb
   const int tid = threadIdx.x;
   const bool drop = (P.flags & JACOBI_FLAG_DROP_SIGNAL) && SL.slab_id == 0;
   const int side = top ? 0 : 1;
-  auto bar_edge = [] { asm volatile("bar.sync 2, %0;" ::"n"(NT) : "memory"); };
+  auto bar_edge = [] { asm volatile("barrier.sync 2, %0;" ::"n"(NT) : "memory"); };  // non-.aligned
   const bool mark = ridx == 0 && tid == 0;
   auto wait = [&](unsigned long long target) {
     if (tid < 32) {
@@ -1237,14 +1237,14 @@ __device__ __forceinline__ void tb_body(const JbParams &P) {
       // it at different instructions, so it is a named barrier over all 16 warps (bar.sync is
       // aligned per warp only; CUDA's __syncthreads would have to be one instruction).
       auto cta_sync = [] {
-        if constexpr (WS) asm volatile("bar.sync 3, %0;" ::"n"((NCW + 4) * 32) : "memory");
+        // non-.aligned form: lanes of a warp may arrive unconverged after the march's branches
+        if constexpr (WS) asm volatile("barrier.sync 3, %0;" ::"n"((NCW + 4) * 32) : "memory");
         else __syncthreads();
       };
       cta_sync();
-      if (threadIdx.x == 0) {
-        red_release_gpu_add(SL.barrier, 1ull);
-        const bool okb = wait_geq<false>(SL.barrier, (unsigned long long)SL.cta_count * (j + 1), P);
-        s_abort = (!okb || *(volatile int *)(P.status + 1)) ? 1 : 0;
+      if (warp == 0) {
+        const bool okb = slab_barrier(SL, P, c, (unsigned long long)(j + 1), (unsigned long long)(tg + K), lane);
+        if (lane == 0) s_abort = (!okb || *(volatile int *)(P.status + 1)) ? 1 : 0;
       }
       cta_sync();
       if (s_abort) return;

@@ -14,6 +14,7 @@ import paper_conf_sc_baydamirlibu24_b200 as jb
 from jacobi_inputs import SEED_BENCH, integer_field, nv_field, u12
 
 pytestmark = pytest.mark.gpu
+ROOT_DIR = __import__("os").path.dirname(__import__("os").path.dirname(__import__("os").path.abspath(__file__)))
 
 
 def bits_equal(a, b):
@@ -402,3 +403,19 @@ def test_gpu_matches_golden_digests():
                 j.run(g["iters"])
                 r = j.gather()
             assert hashlib.sha256(np.ascontiguousarray(r).tobytes()).hexdigest() == g["sha256"], (name, virtual)
+
+
+def test_nccl_baseline_then_import_torch():
+    """The NCCL baseline loads the same libnccl.so.2 PyTorch ships (JACOBI_NCCL_LIB, set by the
+    binding): running it BEFORE `import torch` must not leave a different NCCL in the process
+    (a system NCCL of the same soname would be reused by torch and miss its symbols)."""
+    import subprocess
+    import sys
+    code = ("import sys; sys.path.insert(0, %r)\n"
+            "import numpy as np, paper_conf_sc_baydamirlibu24_b200 as jb\n"
+            "with jb.Jacobi((40, 64)) as j:\n"
+            "    j.set_mode(jb.MODE_BASELINE_NCCL); j.run(3)\n"
+            "import torch\n"
+            "print('TORCH_OK', torch.cuda.is_available())\n") % ROOT_DIR
+    r = subprocess.run([sys.executable, "-c", code], capture_output=True, text=True, timeout=300)
+    assert "TORCH_OK True" in r.stdout, (r.stdout + r.stderr)[-3000:]
