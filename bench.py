@@ -516,7 +516,8 @@ def main():
         # ---- CPU-controlled baselines (per-iteration launch + copy/NCCL + host sync), short run
         base = {}
         b_iters = min(iters, 200)
-        bmodes = [("memcpy", jb.MODE_BASELINE_MEMCPY), ("nccl", jb.MODE_BASELINE_NCCL)]
+        # (NCCL needs one GPU per rank: not with virtual slabs sharing one GPU)
+        bmodes = [("memcpy", jb.MODE_BASELINE_MEMCPY)] + ([] if args.virtual > 1 else [("nccl", jb.MODE_BASELINE_NCCL)])
         if single_multi:
             bmodes += [("overlap", jb.MODE_BASELINE_OVERLAP), ("p2p", jb.MODE_BASELINE_P2P),
                        ("graph", jb.MODE_BASELINE_GRAPH)]
@@ -537,7 +538,7 @@ def main():
 
         # ---- per-iteration halo latency (no-compute runs) and NVLink evidence at N > 1
         if n_gpus > 1 or args.virtual > 1:
-            hmodes = [("cpufree", jb.MODE_CPUFREE), ("baseline_nccl", jb.MODE_BASELINE_NCCL)]
+            hmodes = [("cpufree", jb.MODE_CPUFREE)] + ([] if args.virtual > 1 else [("baseline_nccl", jb.MODE_BASELINE_NCCL)])
             if world == 1:
                 hmodes += [("baseline_memcpy", jb.MODE_BASELINE_MEMCPY), ("baseline_graph", jb.MODE_BASELINE_GRAPH)]
             halo = halo_latency(j, jb, hmodes, max_over_ranks)

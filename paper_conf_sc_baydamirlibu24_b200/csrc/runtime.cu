@@ -884,16 +884,23 @@ int run_cpufree(jacobi_ctx *h, int64_t iters) {
   const bool eligible = h->tblock != 0 && !nocomp && h->norm_every <= 0 && h->kind != KIND_SHMEM && K >= 2;
   if (h->tblock == 1 && !eligible) return JACOBI_EINVAL;
   // auto picks it where it measured faster than the per-iteration kernel: 2D always; 3D when the
-  // slabs have no neighbours, or when every slab has >= 64 CTAs — the 3D edge zones are whole
-  // planes (K phases x 2K-m planes per side, computed by at most a quarter of the slab's CTAs),
-  // which pays with a GPU per slab (and with 2 virtual slabs: C3 397 -> 414 Gcell/s) but not when
-  // 4-8 virtual slabs share one GPU's CTAs
+  // slabs have no neighbours, or when every slab has a GPU of its own (>= 100 CTAs), or >= 64
+  // CTAs and >= 2^22 interior cells — the 3D edge zones are whole planes (K phases x 2K-m planes
+  // per side, computed by at most a quarter of the slab's CTAs, one neighbour flag round trip per
+  // phase): with 2 virtual slabs that pays for C3 (467 vs 384 Gcell/s) but not for the 128^3
+  // latency grid (22.7 vs 18.5 us/iteration), and it does not with 4-8 virtual slabs
   bool use3 = h->total == 1;
   if (!use3 && h->dim == 3) {
     int sms = 0;
     CK(cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, h->slabs[0].device));
     use3 = true;
-    for (int id = 0; id < h->total; ++id) use3 = use3 && slab_ctas(h, id, sms) >= 64;
+    for (int id = 0; id < h->total; ++id) {
+      int64_t st, ch;
+      jbplan::decompose(h->n_out, h->total, id, &st, &ch);
+      const int n = slab_ctas(h, id, sms);
+      const int64_t cells = ch * (h->nx - 2) * (h->ny - 2);
+      use3 = use3 && (n >= 100 || (n >= 64 && cells >= ((int64_t)1 << 22)));
+    }
   }
   const bool use = eligible && (h->tblock == 1 || h->dim == 2 || use3);
   int64_t tb_iters = 0;

@@ -406,8 +406,9 @@ def test_tblock_3d_invariants_and_mixing():
 
 def test_tblock_3d_auto_selection():
     """3D auto: time-blocked K = 3 for a slab without neighbours and for slabs with neighbours
-    that have >= 64 CTAs each (a GPU per slab, or 2 virtual slabs); per-iteration when 4+ virtual
-    slabs share one GPU (whole-plane edge zones on too few CTAs measured slower there)."""
+    that have a GPU each (>= 100 CTAs) or >= 64 CTAs and >= 2^22 cells (2 virtual slabs of a
+    large grid); per-iteration for small slabs with few CTAs and when 4+ virtual slabs share one
+    GPU (whole-plane edge zones on too few CTAs measured slower there)."""
     with jb.Jacobi((20, 30, 40)) as j:
         j.set_param("resident", 0)
         j.run(8)
@@ -415,7 +416,14 @@ def test_tblock_3d_auto_selection():
     with jb.Jacobi((20, 30, 40), virtual=2) as j:
         j.set_param("resident", 0)
         j.run(8)
+        assert j.get_param("last_tblock") == 0
+    f = u12((36, 512, 512), 4)  # 17 planes x 510^2 cells per slab >= 2^22
+    with jb.Jacobi(f.shape, virtual=2) as j:
+        j.set_param("resident", 0)
+        j.scatter(f)
+        j.run(8)
         assert j.get_param("last_tblock") == 6 and j.get_param("last_tb_k") == K3_AUTO
+        assert_bitwise(j.gather(), oracle.jacobi(f, 8, 8), "3D auto, 2 large virtual slabs")
     f = u12((50, 30, 40), 3)
     with jb.Jacobi(f.shape, virtual=4) as j:
         j.set_param("resident", 0)
