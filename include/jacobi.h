@@ -170,18 +170,21 @@ int jacobi_set_mode(jacobi_t h, int mode, int flags);
  * compute advance K iterations per pass over HBM — temporal blocking; slabs
  * with neighbours keep the per-iteration halo exchange through edge zones, which need 2K planes
  * per slab — for every whole multiple of K iterations (2K for K = 2), the rest per iteration:
- * -1 auto (default: 2D runs, not when the slab fits on chip, where the resident kernel is used),
- * 0 never, 1 always incl. 3D (EINVAL when a slab has < 4 planes with P > 1, with the norm, in
- * no-compute mode or in the NVSHMEM variant)), "tb_k" (iterations per time block: -1 auto = 5 in
+ * -1 auto (default: 2D runs — except slabs that fit on chip, which use the resident kernel, unless a
+ * single slab of >= 2^18 interior cells; 3D runs of one slab, or of slabs with a GPU each / >= 64
+ * CTAs and >= 2^22 cells each), 0 never, 1 always (EINVAL when a slab has < 2K planes with P > 1,
+ * with the norm, in no-compute mode or in the NVSHMEM variant)), "tb_k" (iterations per time block: -1 auto = 5 in
  * 2D, 3 in 3D; 2D accepts 2, 3, 5, 3D 2, 3 — a deeper K than the slabs fit falls back to 3, then 2),
  * "tb_ppt" (2D cell pairs per lane and level: K = 2: from tile_x; K = 3: 2 or 4; K = 5: 1 (default,
  * 11 consumer warps) or 2 (7 warps); 3D K = 3: 1 (default) or 2), "tb_rpw" (3D K = 3: rows per
  * warp, 2 (default, 11 warps) or 3 (7 warps)),
- * "tb_lag" (odd K: wavefront skew between levels, 1 default or 2), "tb_min_block" (smallest
+ * "tb_ws" (warp-specialised register split of the time-blocked kernel — 12 compute warps at 160
+ * registers via setmaxnreg, built for 2D K = 5 / 1 pair per lane and 3D K = 3 / 2 rows per warp:
+ * -1 auto (default: where built), 0 off), "tb_lag" (odd K: wavefront skew between levels, 1 default or 2), "tb_min_block" (smallest
  * dynamic plane block of that kernel, default 16), "tb_ctas" (its CTAs per SM, 1 or 2; 2 only
  * for K = 2 and P = 1).  Read-only: "last_resident" (1 if the last CPU-Free run used the resident
  * kernel), "last_tblock" (iterations of the last CPU-Free run done time-blocked), "last_tb_k"
- * (its K, 0 if none), "last_launches" (kernels this process launched in the last jacobi_run, all
+ * (its K, 0 if none), "last_tb_ws" (1 if it used the register split), "last_launches" (kernels this process launched in the last jacobi_run, all
  * GPUs).  Measurement: "halo_trace" (see jacobi_halo_trace; 0 = off, <= 2^20).
  * "barrier" (the CPU-Free kernels' device-side grid barrier: 0 = one counter per slab with
  * red.release + acquire spin (default), 1 = per-CTA arrival flags polled in parallel by every CTA).

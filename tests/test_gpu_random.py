@@ -30,6 +30,7 @@ def cases(draw):
         "min_block": draw(st.sampled_from([1, 3, 8])),
         "dyn_help": draw(st.sampled_from([0, 1])),
         "block_sync": draw(st.sampled_from([0, 1])),
+        "barrier": draw(st.sampled_from([0, 0, 1])),
     }
     mode = draw(st.sampled_from(["MODE_CPUFREE", "MODE_CPUFREE", "MODE_BASELINE_MEMCPY",
                                  "MODE_BASELINE_P2P", "MODE_BASELINE_OVERLAP"]))
@@ -81,7 +82,9 @@ def tblock_cases(draw):
         var = {"tb_lag": draw(st.sampled_from([1, 2]))}
     params = {"resident": 0, "tblock": 1, "tb_k": k, "tb_ppt": ppt, **var,
               "tb_min_block": draw(st.sampled_from([1, 2, 5, 16, 40])),
-              "stages": draw(st.sampled_from([-1, 4, 6]))}
+              "stages": draw(st.sampled_from([-1, 4, 6])),
+              "tb_ws": draw(st.sampled_from([-1, 0])),       # warp-specialised register split on / off
+              "barrier": draw(st.sampled_from([0, 0, 1]))}   # grid barrier: counter / per-CTA flags
     iters = draw(st.integers(1, 26))
     seed = draw(st.integers(0, 2 ** 31))
     return shape, P, params, iters, seed
