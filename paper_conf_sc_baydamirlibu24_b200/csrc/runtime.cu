@@ -790,6 +790,25 @@ int run_tblock(jacobi_ctx *h, int64_t iters, int K, int ppt, int lag, int ws) {
         if (rc) return rc;
         d.tmap = s.tmap;
       }
+      if (per_sm == 1 && (s.has_top || s.has_bot)) {
+        // Boundary roles of the time-blocked plan: plan_launch split the CTAs by the per-iteration
+        // tiles (C2: 8 strips of 2048), but the edge zones are distributed over THIS geometry's
+        // units (C2: 25 strips of 672 with the register split) — one CTA per unit, up to a quarter
+        // of the slab per side.  Every slab computes its own and its neighbours' counts with the
+        // same deterministic function (neighbour_roles), so the flag slots agree.
+        const int64_t sch = h->schedule;
+        h->schedule = 2;
+        int nt = 0, nb = 0, kt = 0, kb = 0;
+        neighbour_roles(h, s.id, sms, g.units, &nt, &nb);
+        if (s.has_top) neighbour_roles(h, s.id - 1, sms, g.units, nullptr, &kt);
+        if (s.has_bot) neighbour_roles(h, s.id + 1, sms, g.units, &kb, nullptr);
+        h->schedule = sch;
+        d.n_top = s.has_top ? nt : 0;
+        d.n_bot = s.has_bot ? nb : 0;
+        d.k_in_top = kt;
+        d.k_in_bot = kb;
+        if (d.n_top + d.n_bot >= d.cta_count) return JACOBI_ENOCOOP;
+      }
       const int64_t npl = d.tb_hi - d.tb_lo + 1;
       const int ni = d.cta_count - d.n_top - d.n_bot;
       d.dyn_items = 0;
