@@ -278,6 +278,17 @@ struct Ring {
 
 // ---------------------------------------------------------------- small load/store helpers
 __device__ __forceinline__ double2 lds2(const double *p) { return *reinterpret_cast<const double2 *>(p); }
+// 32-bit shared-window addresses (sptr): one register per address, no generic-to-shared conversion
+__device__ __forceinline__ double2 lds2_s(uint32_t a) {
+  double2 v;
+  asm volatile("ld.shared.v2.f64 {%0, %1}, [%2];" : "=d"(v.x), "=d"(v.y) : "r"(a) : "memory");
+  return v;
+}
+__device__ __forceinline__ double lds_s(uint32_t a) {
+  double v;
+  asm volatile("ld.shared.f64 %0, [%1];" : "=d"(v) : "r"(a) : "memory");
+  return v;
+}
 
 __device__ __forceinline__ void store_pair(double *p, double o0, double o1, bool pair) {
   if (pair) *reinterpret_cast<double2 *>(p) = make_double2(o0, o1);

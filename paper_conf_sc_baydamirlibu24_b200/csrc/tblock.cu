@@ -348,7 +348,10 @@ __device__ __forceinline__ void tbk_levelk(const TbkLane &L, const double2 *S, c
 // (three dependent fp64 operations after it: + y+1, + y-1, * 1/4), marching down it is y-1
 // (two: + y-1, * 1/4), so the dependency chain through the K levels of a step is ~25 % shorter
 // — same operations, same order, bit-identical results.
-template <int K, int PPT, int LAG, bool FAST, bool REV>
+// SD: the stage stride in doubles when it is a compile-time constant of the kernel variant (0:
+// runtime R.stage_doubles) — the steady-state preloads then address shared memory with one 32-bit
+// register and a constant stride.
+template <int K, int PPT, int LAG, bool FAST, bool REV, int SD = 0>
 __device__ __forceinline__ void tbk_march(const TbkLane &L, const Ring &R, RingPos q, int a, int b, int C, int r0,
                                           int r1, double *dst, int64_t pe, int lane) {
   constexpr int NS = LAG + 2;
@@ -375,15 +378,17 @@ __device__ __forceinline__ void tbk_march(const TbkLane &L, const Ring &R, RingP
   double2 Z[3][PPT];
   double zW = 0.0, zE = 0.0;
   RingPos pnn = pn;  // steady steps: the next step's newest row
+  const uint32_t sbase = sptr(R.stages) + 8u * (uint32_t)L.j0;
+  const uint32_t sstride = 8u * (uint32_t)(SD > 0 ? SD : R.stage_doubles);
   auto zload = [&](double2 *z, const RingPos &p) {
-    const double *st = R.stage(p) + L.j0;
+    const uint32_t st = sbase + p.slot * sstride;
 #pragma unroll
-    for (int i = 0; i < PPT; ++i) z[i] = lds2(st + 2 * i);
+    for (int i = 0; i < PPT; ++i) z[i] = lds2_s(st + 16u * i);
   };
   auto weload = [&](const RingPos &p) {
-    const double *st = R.stage(p) + L.j0;
-    zW = st[-1];
-    zE = st[2 * PPT];
+    const uint32_t st = sbase + p.slot * sstride;
+    zW = lds_s(st - 8u);
+    zE = lds_s(st + 16u * PPT);
   };
   auto step = [&](auto u_ct, auto steady_ct, int Rr) {
     constexpr int U = decltype(u_ct)::value;
@@ -470,7 +475,7 @@ __device__ __forceinline__ void tbk_march(const TbkLane &L, const Ring &R, RingP
   if (Re <= r1) R.release(pc, lane);
 }
 
-template <int K, int PPT, int LAG>
+template <int K, int PPT, int LAG, int SD = 0>
 __device__ __forceinline__ void tbk_item(const JbGeom &g, const Ring &R, RingPos &q, int unit, int64_t a, int64_t b,
                                          int64_t C, double *out, int warp, int lane) {
   constexpr int WO = 64 * PPT - 2 * (K - 1);
@@ -505,8 +510,8 @@ __device__ __forceinline__ void tbk_item(const JbGeom &g, const Ring &R, RingPos
   // march downwards (TB_REV): rows in mirrored coordinates r' = C+1-r
   const int ma = TB_REV ? (int)(C + 1 - b) : (int)a, mb = TB_REV ? (int)(C + 1 - a) : (int)b;
   const int m0 = TB_REV ? (int)(C + 1 - r1) : (int)r0, m1 = TB_REV ? (int)(C + 1 - r0) : (int)r1;
-  if (fast) tbk_march<K, PPT, LAG, true, TB_REV>(L, R, q0, ma, mb, (int)C, m0, m1, dst, g.plane_elems, lane);
-  else tbk_march<K, PPT, LAG, false, TB_REV>(L, R, q0, ma, mb, (int)C, m0, m1, dst, g.plane_elems, lane);
+  if (fast) tbk_march<K, PPT, LAG, true, TB_REV, SD>(L, R, q0, ma, mb, (int)C, m0, m1, dst, g.plane_elems, lane);
+  else tbk_march<K, PPT, LAG, false, TB_REV, SD>(L, R, q0, ma, mb, (int)C, m0, m1, dst, g.plane_elems, lane);
 }
 
 // ---------------------------------------------------------------- 3D (7-point)
@@ -1228,7 +1233,9 @@ __device__ __forceinline__ void tb_body(const JbParams &P) {
                                      lane);
         else if constexpr (DIM == 3) tb3_item<TP>(g, R, q, d.unit, d.a, d.b, C, nxt, warp, lane);
         else if constexpr (K == 2) tb2_item<TP>(g, R, q, d.unit, d.a, d.b, C, nxt, warp, lane);
-        else tbk_item<K, TP, LAG>(g, R, q, d.unit, d.a, d.b, C, nxt, warp, lane);
+        // (stage stride of the 2D odd-K strips: run_tblock sets ws = NCW (64 TP - 2(K-1)) + 2K + 2)
+        else tbk_item<K, TP, LAG, NCW * (64 * TP - 2 * (K - 1)) + 2 * K + 2>(g, R, q, d.unit, d.a, d.b, C, nxt, warp,
+                                                                              lane);
       }
       fence_proxy_async_global();  // generic-proxy stores before the next block's bulk reads
         }
