@@ -23,7 +23,9 @@ buffers: scatter + run + gather per step), ``cpu_controlled`` (the per-iteration
 baselines), ``clocks``; at N > 1 ``halo_us`` (per-iteration time of
 no-compute runs, CPU-Free vs the CPU-controlled baselines), ``halo_traffic`` (halo
 bytes per iteration and GB/s vs NVLink's 900 GB/s) and ``halo_spans_*`` (in-kernel %globaltimer
-wait -> flag -> signal spans of the boundary blocks, jacobi_halo_trace).
+wait -> flag -> signal spans of the boundary blocks, jacobi_halo_trace).  ``parity``: where
+tests/golden holds the oracle's digest of the workload (C1, C2, C3 at their lengths), the SHA-256
+of the whole field the e2e step produced on the N GPUs, compared with it.
 
 ``--impl reference``: there is no reference implementation to install (PAPER.md only), so
 the reference arm is the CPU oracle timed on this host.
@@ -220,6 +222,51 @@ def emit(line: dict) -> None:
     os.write(_JSON_FD if _JSON_FD is not None else 1, (json.dumps(line) + "\n").encode())
 
 
+def golden_digest(shape, iters):
+    """The oracle digest of this workload (U12 seed 0x5C24, `iters` iterations), if committed."""
+    want = list(shape if shape[0] > 1 else shape[1:])
+    for fn in ("oracle_digests_full.json", "oracle_digests.json"):
+        try:
+            with open(os.path.join(ROOT, "tests", "golden", fn)) as f:
+                d = json.load(f)
+        except OSError:
+            continue
+        for name, g in d.items():
+            if g["shape"] == want and g["iters"] == iters and g.get("seed") == 0x5C24:
+                return dict(g, name=name)
+    return None
+
+
+def assemble_field(h_out, shape, lo, hi, desc, world, rank, dist, torch):
+    """The whole gathered field on rank 0: one process holds it in h_out already; with one rank
+    per GPU every rank sends its owned outer planes (+ the global boundary plane it holds) to rank
+    0 over torch.distributed (gloo, CPU tensors)."""
+    import numpy as np
+    nz, ny, nx = shape
+    plane = nx * (ny if nz > 1 else 1)
+    n_out = nz if nz > 1 else ny
+    flat = h_out.numpy()
+    if world == 1:
+        return flat[: n_out * plane]
+    start, chunk = desc["start"], desc["chunk"]
+    a = start - 1 if start == 1 else start                     # first plane this rank owns / holds
+    b = start + chunk + 1 if start + chunk == n_out - 1 else start + chunk
+    mine = torch.from_numpy(np.ascontiguousarray(flat[(a - lo) * plane:(b - lo) * plane]))
+    rng = torch.tensor([a, b], dtype=torch.int64)
+    if rank != 0:
+        dist.send(rng, 0)
+        dist.send(mine, 0)
+        return None
+    full = np.empty(n_out * plane, dtype=np.float64)
+    full[a * plane:b * plane] = mine.numpy()
+    for r in range(1, world):
+        dist.recv(rng, r)
+        buf = torch.empty(int(rng[1] - rng[0]) * plane, dtype=torch.float64)
+        dist.recv(buf, r)
+        full[int(rng[0]) * plane:int(rng[1]) * plane] = buf.numpy()
+    return full
+
+
 def halo_latency(j, jb, modes, max_over_ranks, n=200):
     """Per-iteration time of no-compute runs (halo copies, flags and barriers only),
     (T(2n) - T(n)) / n to cancel the launch cost; µs.  Modes a handle does not support are
@@ -310,7 +357,7 @@ def main():
         return 2
     local = local % max(ndev, 1)  # (more ranks than GPUs only in functional tests: time-sliced)
 
-    import numpy as np  # noqa: F401
+    import numpy as np
     import torch
     import paper_conf_sc_baydamirlibu24_b200 as jb
 
@@ -611,6 +658,21 @@ def main():
                        "h2d_bytes_per_step": int(h2d_total), "d2h_bytes_per_step": int(d2h_total),
                        "ms_per_step": 1e3 * e2e_s / args.steps,
                        "path": "jacobi_scatter (pinned H2D) + jacobi_run + jacobi_gather (pinned D2H)"}
+
+        # ---- parity of the measured configuration: the e2e step above scattered the U12 field and
+        #      ran exactly `iters` iterations through the C ABI on these N GPUs, so the gathered
+        #      field is compared (SHA-256 of the whole field) with the digest of the CPU oracle's
+        #      own run of that workload, where tests/golden holds one (C1, C2, C3 at their
+        #      lengths; written by tests/golden/make_golden.py from oracle/ only)
+        gold = golden_digest(shape, iters)
+        if gold is not None:
+            full = assemble_field(h_out, shape, lo, hi, desc, world, rank, dist, torch)
+            if rank == 0:
+                import hashlib
+                got = hashlib.sha256(np.ascontiguousarray(full).tobytes()).hexdigest()
+                line["parity"] = {"match": got == gold["sha256"], "sha256": got, "oracle_sha256": gold["sha256"],
+                                  "what": f"whole {shape} field after {iters} iterations on {n_gpus} GPU(s) "
+                                          f"(e2e step) vs the oracle digest {gold['name']}"}
 
         # ---- CPU oracle on this host's cores (rank 0, N = 1 only), bounded sample
         if rank == 0 and n_gpus == 1:
