@@ -108,7 +108,10 @@ int jacobi_open_peers(jacobi_t h, const void *top_blob, const void *bottom_blob)
  * order): also opens every rank's control block, which the residual-norm all-reduce needs. */
 int jacobi_open_ranks(jacobi_t h, const void *blobs, int world);
 /* NCCL baseline in dist mode: rank 0 creates a 128-byte ncclUniqueId, every rank passes it to
- * jacobi_nccl_init (collective).  libnccl.so.2 is loaded with dlopen on first use. */
+ * jacobi_nccl_init (collective).  libnccl.so.2 is loaded with dlopen (RTLD_LOCAL) on first use —
+ * the file named by the environment variable JACOBI_NCCL_LIB if set (the Python binding sets it
+ * to the NCCL PyTorch ships, so the process never holds two different libnccl.so.2), else the
+ * default search path. */
 int jacobi_nccl_unique_id(void *out128);
 int jacobi_nccl_init(jacobi_t h, const void *id128);
 
