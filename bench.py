@@ -599,10 +599,12 @@ def main():
                 gbs = sides * plane_bytes / (halo["cpufree"] * 1e-6) / 1e9
                 msg["achieved_gbs_per_direction_nocompute"] = gbs
                 msg["frac_of_nvlink"] = gbs / 900.0
-            if tb_iters == 0 and not resident:
-                # compute runs of the per-iteration kernel deliver one plane per side per iteration
-                gbs = sides * plane_bytes / (1e-3 * launch_ms / iters) / 1e9
-                msg["halo_gbs_during_compute_run"] = gbs
+            # every CPU-Free kernel delivers one outer plane per side and iteration (the
+            # time-blocked one as its K edge-zone phases: level-m planes into the neighbour's
+            # slots, the last into its halo), so the halo rate of the timed compute run is:
+            gbs = sides * plane_bytes / (1e-3 * launch_ms / iters) / 1e9
+            msg["halo_gbs_during_compute_run"] = gbs
+            msg["halo_frac_of_nvlink_during_compute_run"] = gbs / 900.0
             line["halo_us"] = halo
             line["halo_traffic"] = msg
             if args.virtual > 1:
