@@ -45,6 +45,9 @@ __device__ __forceinline__ void tma_box3(void *dst, const void *tmap, int c0, in
 
 // The odd-K marches run towards row / plane 0 (shorter fp64 dependency chain, see tbk_march).
 constexpr bool TB_REV = true;
+#ifndef TB3_PF
+#define TB3_PF 1  // 3D odd-K march: level-0 planes of the steady state kept in registers (tb3k_march)
+#endif
 
 // Position `off` stages after p in the ring.
 __device__ __forceinline__ RingPos ring_add(RingPos p, uint32_t off, uint32_t S) {
@@ -728,6 +731,44 @@ __device__ __forceinline__ void tb3k_level1(const Tb3kLane &L, int sr0, int ws, 
   }
 }
 
+// Level 1 as tb3k_level1 (steady state: every row and plane interior), with the warp's own
+// level-0 rows of the three planes already in registers (Dn: z-1, Cc: z, Up: z+1); only the
+// centre plane's rows just above / below the warp and the x neighbours at the lane pair's ends
+// come from the centre plane's stage zc.
+template <int PPT, int RPW, bool FAST>
+__device__ __forceinline__ void tb3k_level1_regs(const Tb3kLane &L, int sr0, int ws, const double *zc,
+                                                 const double2 (*Dn)[PPT], const double2 (*Cc)[PPT],
+                                                 const double2 (*Up)[PPT], double2 (*V)[PPT]) {
+  double2 T[PPT], B[PPT];  // centre-plane rows sr0-1 and sr0+RPW
+#pragma unroll
+  for (int i = 0; i < PPT; ++i) {
+    T[i] = lds2(zc + (sr0 - 1) * ws + L.j0 + 2 * i);
+    B[i] = lds2(zc + (sr0 + RPW) * ws + L.j0 + 2 * i);
+  }
+#pragma unroll
+  for (int j = 0; j < RPW; ++j) {
+    const int o = (sr0 + j) * ws + L.j0;
+    const double Wl = zc[o - 1], Er = zc[o + 2 * PPT];
+#pragma unroll
+    for (int i = 0; i < PPT; ++i) {
+      const double2 C = Cc[j][i];
+      const double2 N = j + 1 < RPW ? Cc[j + 1 < RPW ? j + 1 : j][i] : B[i];
+      const double2 S = j > 0 ? Cc[j > 0 ? j - 1 : j][i] : T[i];
+      const double W = i == 0 ? Wl : Cc[j][i > 0 ? i - 1 : 0].y;
+      const double E = i == PPT - 1 ? Er : Cc[j][i + 1 < PPT ? i + 1 : i].x;
+      // oracle order: x+1, x-1, y+1, y-1, z+1, z-1, then * fl(1/6)
+      const double l0 = kC6 * (((((C.y + W) + N.x) + S.x) + Up[j][i].x) + Dn[j][i].x);
+      const double l1 = kC6 * (((((E + C.x) + N.y) + S.y) + Up[j][i].y) + Dn[j][i].y);
+      if (FAST) {
+        V[j][i] = make_double2(l0, l1);
+      } else {
+        V[j][i].x = (L.rok >> j & 1u) && (L.ok >> i & 1u) ? l0 : C.x;
+        V[j][i].y = (L.rok >> j & 1u) && (L.full >> i & 1u) ? l1 : C.y;
+      }
+    }
+  }
+}
+
 // Level k >= 2 of the warp's rows of the centre plane Zc (level k-1 planes Zm, Zc, Zp); yT / yB:
 // the level-(k-1) rows just above / below the warp (other warps' boundary rows).  STORE: level
 // K, pair i of row j stored at o + j·pitch + 2i.
@@ -797,12 +838,37 @@ __device__ __forceinline__ void tb3k_march(const Tb3kLane &L, const JbGeom &g, c
       *reinterpret_cast<double2 *>(xrow(k1, par, warp, 1) + 2 * (lane * PPT + i)) = V[RPW - 1][i];
     }
   };
+  // Steady state (TB3_PF): the warp's own level-0 rows of the three planes a step reads stay in
+  // registers Z[m % 3] (newest plane of step m), so each step loads only its new plane's own rows
+  // and the centre plane's two rows just outside the warp: RPW + 2 instead of 3 RPW + 2 row
+  // loads (LDS.128) per step — the 3D march is bound by its shared-memory pipe.
+  // (Loading the next step's plane right after level 1, as the 2D march does, needs more live
+  // registers here and spills: measured slower.)
+  constexpr bool PF = TB3_PF;
+  double2 Z[PF ? 3 : 1][RPW][PPT];
+  auto zload = [&](double2 (*z)[PPT], const RingPos &p) {
+    const double *st = R.stage(p) + sr0 * ws + L.j0;
+#pragma unroll
+    for (int j = 0; j < RPW; ++j)
+#pragma unroll
+      for (int i = 0; i < PPT; ++i) z[j][i] = lds2(st + j * ws + 2 * i);
+  };
   auto step = [&](auto u_ct, auto steady_ct, int Rr) {
     constexpr int U = decltype(u_ct)::value;
     constexpr bool ST = decltype(steady_ct)::value;
     constexpr int SN = U, SC = (U + NS - 1) % NS, SS = (U + NS - 2) % NS;
     const int par = Rr & 1, prv = par ^ 1;
     auto need = [&](int k, int r) { return r >= max(a - (K - k), 0) && r <= min(b + (K - k), C + 1); };
+    if (ST && PF) {
+      // level-0 planes Rr (newest, Z[U]), Rr-1 (centre, Z[U+2]), Rr-2 (Z[U+1])
+      constexpr int ZN = PF ? U % 3 : 0, ZC = PF ? (U + 2) % 3 : 0, ZO = PF ? (U + 1) % 3 : 0;
+      R.wait_full(pn);
+      zload(Z[ZN], pn);
+      bar_consumers<NCW>();  // the previous step's exchange rows are visible; its reads are done
+      tb3k_level1_regs<PPT, RPW, FAST>(L, sr0, ws, R.stage(pc), Z[REV ? ZN : ZO], Z[ZC], Z[REV ? ZO : ZN], X[0][U]);
+      publish(0, par, X[0][U]);
+      R.release(pm, lane);  // plane Rr-2: its last reads were the register loads
+    } else {
     if (ST || Rr <= r1) R.wait_full(pn);
     bar_consumers<NCW>();  // the previous step's exchange rows are visible; its reads are done
     if (ST || need(1, Rr - 1)) {
@@ -812,6 +878,7 @@ __device__ __forceinline__ void tb3k_march(const Tb3kLane &L, const JbGeom &g, c
       publish(0, par, X[0][U]);
     }
     if (ST || (Rr - 2 >= r0 && Rr - 2 <= r1)) R.release(pm, lane);
+    }
 #pragma unroll
     for (int k = 2; k <= K; ++k) {
       const int r = Rr - k;
@@ -835,7 +902,7 @@ __device__ __forceinline__ void tb3k_march(const Tb3kLane &L, const JbGeom &g, c
     o += ostep;
     pm = pc;
     pc = pn;
-    if (Rr + 1 <= r1) {
+    if ((ST && PF) || Rr + 1 <= r1) {  // (steady steps always have a next plane)
       const uint32_t sl = pn.slot + 1u;
       const bool wrap = sl == R.S;
       pn.slot = wrap ? 0u : sl;
@@ -853,8 +920,15 @@ __device__ __forceinline__ void tb3k_march(const Tb3kLane &L, const JbGeom &g, c
   int Rr = Rs;
   if (Ws <= We) {
     for (; Rr < Ws; Rr += NS) group(TF{}, Rr);
-    if (Rr + NS - 1 <= We) {
-      const int Rend = Rr + ((We - Rr + 1) / NS) * NS;
+    // (the steady steps end at We - 1: every one has a next plane in the ring)
+    const int Wend = PF ? We - 1 : We;
+    if (Rr + NS - 1 <= Wend) {
+      const int Rend = Rr + ((Wend - Rr + 1) / NS) * NS;
+      if constexpr (PF) {  // the first steady step's older planes (Rr-1, Rr-2 -> Z[2], Z[1])
+        R.wait_full(pn);
+        zload(Z[PF ? 2 : 0], pc);
+        zload(Z[PF ? 1 : 0], pm);
+      }
       for (; Rr < Rend; Rr += NS) group(TT{}, Rr);
     }
   }
@@ -1060,6 +1134,9 @@ __device__ __noinline__ bool tb_edge(const JbGeom &g, const JbSlab &SL, const Jb
 // warps (whole warpgroups) take them with setmaxnreg.inc: 12 compute warps at 160 registers
 // where one producer warp per CTA would leave 11 at 168 (each SM sub-partition holds 16 K
 // registers: 32 + 3 x 160 = 512 per lane slot).
+#ifndef JB_WS_REGS
+#define JB_WS_REGS 160  // consumer registers of the warp-specialised split
+#endif
 template <int NCW, int DIM, int K, int TP, int LAG, int RPW, int WS = 0>
 __device__ __forceinline__ void tb_body(const JbParams &P) {
   static_assert(!WS || NCW % 4 == 0, "warp specialisation needs whole consumer warpgroups");
@@ -1266,7 +1343,7 @@ __device__ __forceinline__ void tb_body(const JbParams &P) {
   };
   if constexpr (WS) {
     if (consumer) {
-      asm volatile("setmaxnreg.inc.sync.aligned.u32 160;" ::: "memory");
+      asm volatile("setmaxnreg.inc.sync.aligned.u32 %0;" ::"n"(JB_WS_REGS) : "memory");
       blocks(std::integral_constant<int, 2>{});
     } else {
       asm volatile("setmaxnreg.dec.sync.aligned.u32 32;" ::: "memory");
@@ -1310,6 +1387,7 @@ const void *tblock_fn_plain(int dim, int k, int ppt, int lag, int per_sm, int ws
     if (dim == 3 && k == 3 && ppt == 1 && lag == 2) return JB_TB(jb_tblock_ws<3, 3, 1, 12, 1, 2>);
     return nullptr;
   }
+#ifndef JB_TB_ONLY_WS  // (development builds: only the warp-specialised kernels)
   if (dim == 3) {
     if (k == 2) return JB_TB(jb_tblock<3, 2, TB_TY>);
     // odd K: (K, PPT, RPW = `lag`) -> NCW consumer warps x RPW rows per tile
@@ -1338,6 +1416,7 @@ const void *tblock_fn_plain(int dim, int k, int ppt, int lag, int per_sm, int ws
   if (k == 3 && ppt == 2) return JB_TB(jb_tblock<2, 3, 2, 7>);
   if (k == 3 && ppt == 4) return JB_TB(jb_tblock<2, 3, 4, 7>);
   if (k == 5 && ppt == 2) return JB_TB(jb_tblock<2, 5, 2, 7>);
+#endif
   return nullptr;
 }
 #undef JB_TB
