@@ -1134,9 +1134,6 @@ __device__ __noinline__ bool tb_edge(const JbGeom &g, const JbSlab &SL, const Jb
 // warps (whole warpgroups) take them with setmaxnreg.inc: 12 compute warps at 160 registers
 // where one producer warp per CTA would leave 11 at 168 (each SM sub-partition holds 16 K
 // registers: 32 + 3 x 160 = 512 per lane slot).
-#ifndef JB_WS_REGS
-#define JB_WS_REGS 160  // consumer registers of the warp-specialised split
-#endif
 template <int NCW, int DIM, int K, int TP, int LAG, int RPW, int WS = 0>
 __device__ __forceinline__ void tb_body(const JbParams &P) {
   static_assert(!WS || NCW % 4 == 0, "warp specialisation needs whole consumer warpgroups");
@@ -1343,7 +1340,10 @@ __device__ __forceinline__ void tb_body(const JbParams &P) {
   };
   if constexpr (WS) {
     if (consumer) {
-      asm volatile("setmaxnreg.inc.sync.aligned.u32 %0;" ::"n"(JB_WS_REGS) : "memory");
+      // 32 (producer warpgroup) + NCW/4 consumer warpgroups x WSR <= 512 registers per lane slot
+      // (8 consumer warps: 232, not 240 — measured: the .inc to 240 never completes)
+      constexpr int WSR = NCW == 12 ? 160 : NCW == 8 ? 232 : 120;
+      asm volatile("setmaxnreg.inc.sync.aligned.u32 %0;" ::"n"(WSR) : "memory");
       blocks(std::integral_constant<int, 2>{});
     } else {
       asm volatile("setmaxnreg.dec.sync.aligned.u32 32;" ::: "memory");
