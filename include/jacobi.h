@@ -191,6 +191,13 @@ int jacobi_set_mode(jacobi_t h, int mode, int flags);
  * GPUs).  Measurement: "halo_trace" (see jacobi_halo_trace; 0 = off, <= 2^20).
  * "barrier" (the CPU-Free kernels' device-side grid barrier: 0 = one counter per slab with
  * red.release + acquire spin (default), 1 = per-CTA arrival flags polled in parallel by every CTA).
+ * "halo_ll" (streaming CPU-Free kernel, not with the norm: halo cells travel as tagged 16-byte LL
+ * cells {tag:lo32, tag:hi32} that the receiving boundary CTAs poll and unpack into their halo
+ * plane, instead of plain peer stores + one sys-scope release flag per boundary CTA and
+ * iteration (P:394's signal); the first / last halo of every run keep the flags, so runs of every
+ * kind mix.  -1 auto (default: off), 0 off, 1 on.  DESIGN.md §5.11: removes the 1.5-3.9 us
+ * MEMBAR.SYS of each release but doubles the halo bytes — measured equal or slower except 2D
+ * no-compute / latency runs at 4-8 slabs).
  * Unknown names return JACOBI_EINVAL. */
 int jacobi_set_param(jacobi_t h, const char *name, int64_t value);
 int jacobi_get_param(jacobi_t h, const char *name, int64_t *value);

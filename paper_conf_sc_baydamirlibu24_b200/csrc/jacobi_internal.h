@@ -21,6 +21,7 @@
 #define JB_TB_LAG 1             // default wavefront lag of the odd-K march
 #define JB_TB_KMAX3 3           // deepest time block of the 3D time-blocked kernel
 #define JB_TB_K3D 3             // its default depth (auto; slabs without neighbours only)
+#define JB_LL_AUTO 0             // halo_ll = -1 (auto): LL halo protocol of the streaming kernel on/off
 #define JB_TB_RPW3 2            // 3D odd K: default rows per warp (x 11 warps)
 
 // Scratch planes after each slab buffer for the time-blocked kernel's edge zones of depth K
@@ -35,6 +36,13 @@ static inline int64_t jb_edge_planes(int dim) { return jb_edge_planes_k(dim == 2
 // Doubles of ONE field buffer of a slab with `chunk` owned planes.
 static inline int64_t jb_buf_doubles(int64_t chunk, int dim, int64_t plane_elems) {
   return (chunk + 2 + jb_edge_planes(dim)) * plane_elems + JB_BUF_SLACK;
+}
+
+// LL receive area of a slab buffer (JbSlab::ll_in_*): 2 planes of doubles (one 16-byte LL cell per
+// cell of the halo plane) per side — side 0 from the top neighbour, 1 from the bottom one — in the
+// last 4 edge-scratch planes (the streaming kernel never uses that scratch otherwise).
+static inline unsigned long long *jb_ll_area(double *buf, int64_t chunk, int dim, int64_t plane_elems, int side) {
+  return reinterpret_cast<unsigned long long *>(buf + (chunk + 2 + jb_edge_planes(dim) - 4 + 2 * side) * plane_elems);
 }
 
 // Grid geometry in HBM and the tile shape of the march.
@@ -128,6 +136,16 @@ struct JbSlab {
   // stores the barrier's epoch (the global iteration count after it) into bar_flags[c] and warp 0
   // of every CTA polls all cta_count flags — no atomic serialised on one address.
   unsigned long long *bar_flags;
+  // LL halo protocol (knob "halo_ll", streaming CPU-Free kernel): every halo cell
+  // travels as a 16-byte LL cell {tag:lo32, tag:hi32} (two single-copy-atomic 8-byte words), so
+  // the receiver polls the data itself and neither side issues a sys-scope fence per iteration.
+  // ll_out_*[p]: the neighbour's receive area for iteration parity p; ll_in_*[p]: this slab's own
+  // (from the top / bottom neighbour).  Null: the flag protocol above.  Areas live in the last 4
+  // edge-scratch planes of buf[p] (jb_ll_area).
+  unsigned long long *ll_out_top[2];
+  unsigned long long *ll_out_bot[2];
+  const unsigned long long *ll_in_top[2];
+  const unsigned long long *ll_in_bot[2];
 };
 
 struct JbParams {

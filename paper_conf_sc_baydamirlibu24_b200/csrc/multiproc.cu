@@ -123,6 +123,7 @@ int jacobi_open_peers(jacobi_t h, const void *top_blob, const void *bottom_blob)
     int rc = open(top_blob, h->rank - 1, bufs, &ctrl, &chunk);
     if (rc) return rc;
     for (int p = 0; p < 2; ++p) s.peer_top[p] = bufs[p] + (chunk + 1) * pe;
+    for (int p = 0; p < 2; ++p) s.ll_out_top[p] = jb_ll_area(bufs[p], chunk, h->dim, pe, 1);
     s.mid_top_out = bufs[1] + (chunk + 2) * pe;
     s.flag_out_top = &ctrl->flag_in[1][0];
   }
@@ -133,6 +134,7 @@ int jacobi_open_peers(jacobi_t h, const void *top_blob, const void *bottom_blob)
     int rc = open(bottom_blob, h->rank + 1, bufs, &ctrl, &chunk);
     if (rc) return rc;
     for (int p = 0; p < 2; ++p) s.peer_bot[p] = bufs[p];
+    for (int p = 0; p < 2; ++p) s.ll_out_bot[p] = jb_ll_area(bufs[p], chunk, h->dim, pe, 0);
     s.mid_bot_out = bufs[0] + (chunk + 2) * pe;
     s.flag_out_bot = &ctrl->flag_in[0][0];
   }

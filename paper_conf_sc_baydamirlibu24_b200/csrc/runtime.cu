@@ -103,6 +103,7 @@ void link_local(jacobi_ctx *h) {
     if (s.has_top) {
       Slab &o = h->slabs[i - 1];
       for (int p = 0; p < 2; ++p) s.peer_top[p] = o.buf[p] + (o.chunk + 1) * pe;
+      for (int p = 0; p < 2; ++p) s.ll_out_top[p] = jb_ll_area(o.buf[p], o.chunk, h->dim, pe, 1);
       s.mid_top_out = o.buf[1] + (o.chunk + 2) * pe;  // its E_bot (slot 0)
       s.flag_out_top = &o.ctrl->flag_in[1][0];
       s.peer_top_dev = o.device;
@@ -110,6 +111,7 @@ void link_local(jacobi_ctx *h) {
     if (s.has_bot) {
       Slab &o = h->slabs[i + 1];
       for (int p = 0; p < 2; ++p) s.peer_bot[p] = o.buf[p];
+      for (int p = 0; p < 2; ++p) s.ll_out_bot[p] = jb_ll_area(o.buf[p], o.chunk, h->dim, pe, 0);
       s.mid_bot_out = o.buf[0] + (o.chunk + 2) * pe;  // its E_top (slot 0)
       s.flag_out_bot = &o.ctrl->flag_in[0][0];
       s.peer_bot_dev = o.device;
@@ -577,6 +579,29 @@ int setup_trace(jacobi_ctx *h, LaunchPlan &L) {
   return JACOBI_OK;
 }
 
+// LL halo protocol (knob "halo_ll") for a streaming CPU-Free launch: the
+// receive areas of this launch's slabs and the neighbours' (set at link time); null = flags.
+bool ll_enabled(const jacobi_ctx *h) {
+  if (h->kind == KIND_SHMEM || h->halo_ll == 0) return false;
+  return h->halo_ll > 0 || JB_LL_AUTO;
+}
+void setup_ll(jacobi_ctx *h, LaunchPlan &L) {
+  const bool on = ll_enabled(h);
+  const int64_t pe = h->geom.plane_elems;
+  for (size_t k = 0; k < L.slab_idx.size(); ++k) {
+    Slab &s = h->slabs[L.slab_idx[k]];
+    JbSlab &d = L.P.s[k];
+    for (int p = 0; p < 2; ++p) {
+      d.ll_out_top[p] = on && s.has_top ? s.ll_out_top[p] : nullptr;
+      d.ll_out_bot[p] = on && s.has_bot ? s.ll_out_bot[p] : nullptr;
+      d.ll_in_top[p] = on && s.has_top ? jb_ll_area(s.buf[p], s.chunk, h->dim, pe, 0) : nullptr;
+      d.ll_in_bot[p] = on && s.has_bot ? jb_ll_area(s.buf[p], s.chunk, h->dim, pe, 1) : nullptr;
+    }
+    if (on && ((s.has_top && !s.ll_out_top[0]) || (s.has_bot && !s.ll_out_bot[0])))
+      for (int p = 0; p < 2; ++p) d.ll_out_top[p] = d.ll_out_bot[p] = nullptr, d.ll_in_top[p] = d.ll_in_bot[p] = nullptr;
+  }
+}
+
 int run_cpufree_k1(jacobi_ctx *h, int64_t iters) {
   const bool nocomp = h->flags & JACOBI_FLAG_NO_COMPUTE;
   const bool norm = !nocomp && h->norm_every > 0;
@@ -603,6 +628,7 @@ int run_cpufree_k1(jacobi_ctx *h, int64_t iters) {
       h->schedule = sched;
       if (rc) return rc;
       if (norm && (rc = setup_norm(h, plans[i]))) return rc;
+      if (!norm) setup_ll(h, plans[i]);
     }
     plans[i].P.t0 = h->t;
     plans[i].P.iters = iters;
@@ -1084,6 +1110,7 @@ static int64_t *param_slot(jacobi_t h, const char *name) {
   if (!std::strcmp(name, "last_tblock")) return &h->last_tblock;
   if (!std::strcmp(name, "halo_trace")) return &h->halo_trace;
   if (!std::strcmp(name, "barrier")) return &h->barrier;
+  if (!std::strcmp(name, "halo_ll")) return &h->halo_ll;
   if (!std::strcmp(name, "last_launches")) return &h->last_launches;
   return nullptr;
 }

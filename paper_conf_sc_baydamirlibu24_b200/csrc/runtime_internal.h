@@ -139,6 +139,8 @@ struct Slab {
   double *peer_top[2] = {nullptr, nullptr};
   double *peer_bot[2] = {nullptr, nullptr};
   double *mid_top_out = nullptr, *mid_bot_out = nullptr;  // neighbours' time-blocked edge slots
+  unsigned long long *ll_out_top[2] = {nullptr, nullptr};  // neighbours' LL receive areas (halo_ll)
+  unsigned long long *ll_out_bot[2] = {nullptr, nullptr};
   unsigned long long *flag_out_top = nullptr, *flag_out_bot = nullptr;
   int peer_top_dev = -1, peer_bot_dev = -1;
   int shm_pe_top = -1, shm_pe_bot = -1;  // NVSHMEM variant: neighbour PEs
@@ -198,6 +200,7 @@ struct jacobi_ctx {
   int64_t last_launches = 0;   // read-only: kernels this process launched in the last jacobi_run
   int64_t barrier = 0;         // grid barrier of the CPU-Free kernels: 0 counter, 1 per-CTA flags
   int64_t halo_trace = 0;      // measurement: record the first n halo exchanges of each CPU-Free run
+  int64_t halo_ll = -1;        // LL halo protocol of the streaming CPU-Free kernel (§5.11): -1 auto, 0 off, 1 on
                                // (%globaltimer wait begin / flag acquired / signal; jacobi_halo_trace)
   int64_t norm_every = 0;      // N4: check the update norm every k iterations (0 = off)
   double tol = 0.0;            // N4: stop once the norm <= tol

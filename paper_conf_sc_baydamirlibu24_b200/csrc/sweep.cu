@@ -104,6 +104,82 @@ __device__ Sched make_sched(const JbGeom &g, const JbSlab &S, int role, int ridx
   return s;
 }
 
+// ---------------------------------------------------------------- LL halo protocol
+// The flag protocol pays one sys-scope release (MEMBAR.SYS: 1.5 us alone, 3.9 us with every CTA
+// issuing one, profiles/r02_ubench_fence.txt) per boundary CTA and iteration.  LL cells carry
+// the iteration in each 8-byte word, so a cell is valid exactly when both of its words show the
+// tag of the awaited iteration — no fence, no flag.  Tags are a bijective mix of the global
+// iteration, odd (never 0, so untouched memory never matches; iterations only grow, so stale
+// cells of earlier runs never match either).
+__device__ __forceinline__ uint32_t ll_tag(int64_t tg) { return ((uint32_t)tg * 2654435761u ^ 0x6a09e667u) | 1u; }
+__device__ __forceinline__ void ll_store(unsigned long long *p, double v, uint32_t tag) {
+  const unsigned long long t = (unsigned long long)tag << 32;
+  const unsigned long long w0 = t | (uint32_t)__double2loint(v), w1 = t | (uint32_t)__double2hiint(v);
+  asm volatile("st.relaxed.sys.global.v2.u64 [%0], {%1, %2};" ::"l"(p), "l"(w0), "l"(w1) : "memory");
+}
+__device__ __forceinline__ void ll_store_pair(unsigned long long *p, double o0, double o1, bool pair, uint32_t tag) {
+  ll_store(p, o0, tag);
+  if (pair) ll_store(p + 2, o1, tag);
+}
+__device__ __forceinline__ ulonglong2 ll_load(const unsigned long long *p) {
+  ulonglong2 v;
+  asm volatile("ld.relaxed.sys.global.v2.u64 {%0, %1}, [%2];" : "=l"(v.x), "=l"(v.y) : "l"(p) : "memory");
+  return v;
+}
+
+// Receiver side: every thread of a boundary CTA polls the LL cells of the halo-plane cells its
+// units' edge tiles read (the cells straight above / below the tile: the edge plane's y-1 / y+1
+// (2D) or z-1 / z+1 (3D) neighbours) and writes them into the halo plane of the current buffer,
+// in batches of 4 independent cells per thread.  False: watchdog / abort.
+__device__ bool ll_unpack(const JbGeom &g, const Sched &sc, double *halo, const unsigned long long *ll, uint32_t tag,
+                          const JbParams &P) {
+  constexpr int B = 4;
+  const int nth = blockDim.x;
+  const unsigned long long t_start = globaltimer();
+  volatile int *abort_flag = P.status + 1;
+  for (int u = sc.ub; u < sc.ue; ++u) {
+    const int ux = u % g.units_x, uy = u / g.units_x;
+    const int64_t x0 = 1 + (int64_t)ux * g.tx;
+    const int vx = (int)min((int64_t)g.tx, g.nx - 1 - x0);
+    const int64_t y0 = g.dim == 3 ? 1 + (int64_t)uy * g.ty : 0;
+    const int vy = g.dim == 3 ? (int)min((int64_t)g.ty, g.ny - 1 - y0) : 1;
+    const int n = vx * vy;
+    for (int i0 = (int)threadIdx.x; i0 < n; i0 += B * nth) {
+      int64_t idx[B];
+#pragma unroll
+      for (int b = 0; b < B; ++b) {
+        const int i = i0 + b * nth;
+        const int r = i / vx;
+        idx[b] = i < n ? (y0 + r) * g.pitch + 3 + x0 + (i - r * vx) : -1;
+      }
+      ulonglong2 v[B];
+      uint32_t cnt = 0;
+      while (true) {
+        bool ok = true;
+#pragma unroll
+        for (int b = 0; b < B; ++b)
+          if (idx[b] >= 0) {
+            v[b] = ll_load(ll + 2 * idx[b]);
+            ok &= (uint32_t)(v[b].x >> 32) == tag && (uint32_t)(v[b].y >> 32) == tag;
+          }
+        if (ok) break;
+        if ((++cnt & 63u) == 0) {
+          if (*abort_flag) return false;
+          if (globaltimer() - t_start > P.timeout_ns) {
+            atomicCAS(P.status, 0, JACOBI_ETIMEOUT);
+            atomicExch(P.status + 1, 1);
+            return false;
+          }
+        }
+      }
+#pragma unroll
+      for (int b = 0; b < B; ++b)
+        if (idx[b] >= 0) halo[idx[b]] = __hiloint2double((int)(uint32_t)v[b].y, (int)(uint32_t)v[b].x);
+    }
+  }
+  return true;
+}
+
 // ---------------------------------------------------------------- producer
 // Where one tile's stage comes from: the rows of tile `unit` (1 in 2D; ty + 2 in 3D incl. the y
 // halo rows), each row the x window [x0-2, x0+tx+2) of 16-byte aligned doubles, one
@@ -167,7 +243,8 @@ __device__ __forceinline__ void produce_planes(const JbGeom &g, const double *cu
 // plane costs one 16-byte LDS + two 8-byte LDS (x-1, x+2) per pair.
 template <int PPT, bool NOCOMP, bool NORM>
 __device__ __forceinline__ void consume_run_2d(const JbGeom &g, const Ring &R, RingPos &q, const Run &run,
-                                               const double *cur, double *nxt, double *remote, int ctid, int lane,
+                                               const double *cur, double *nxt, double *remote,
+                                               unsigned long long *rll, uint32_t tag, int ctid, int lane,
                                                double &acc) {
   const int64_t x0 = 1 + (int64_t)run.unit * g.tx;
   const int vx = (int)min((int64_t)g.tx, g.nx - 1 - x0);
@@ -190,9 +267,10 @@ __device__ __forceinline__ void consume_run_2d(const JbGeom &g, const Ring &R, R
       const double *src = cur + (run.p0 + p) * g.plane_elems + col;
 #pragma unroll
       for (int i = 0; i < PPT; ++i)
-        if ((ok >> i & 1u) && remote) {
+        if ((ok >> i & 1u) && (remote || rll)) {
           const double2 v = __ldcg(reinterpret_cast<const double2 *>(src + 2 * i * JB_NC));
-          store_pair(remote + col + 2 * i * JB_NC, v.x, v.y, full >> i & 1u);
+          if (rll) ll_store_pair(rll + 2 * (col + 2 * i * JB_NC), v.x, v.y, full >> i & 1u, tag);
+          else store_pair(remote + col + 2 * i * JB_NC, v.x, v.y, full >> i & 1u);
         }
     }
     return;
@@ -212,6 +290,7 @@ __device__ __forceinline__ void consume_run_2d(const JbGeom &g, const Ring &R, R
     }
   double *dst = nxt + run.p0 * g.plane_elems + col;
   double *rem = remote ? remote + col : nullptr;
+  unsigned long long *rl = rll ? rll + 2 * col : nullptr;
   const int64_t pe = g.plane_elems;
   for (int64_t p = 0; p < L; ++p) {
     R.wait_full(pp);
@@ -226,7 +305,8 @@ __device__ __forceinline__ void consume_run_2d(const JbGeom &g, const Ring &R, R
         const double o1 = 0.25 * (((E + C[i].x) + N.y) + S[i].y);
         if (ok >> i & 1u) {
           store_pair(dst + 2 * i * JB_NC, o0, o1, full >> i & 1u);
-          if (rem) store_pair(rem + 2 * i * JB_NC, o0, o1, full >> i & 1u);
+          if (rl) ll_store_pair(rl + 4 * i * JB_NC, o0, o1, full >> i & 1u, tag);
+          else if (rem) store_pair(rem + 2 * i * JB_NC, o0, o1, full >> i & 1u);
           if (NORM) {  // update norm (N4): fixed per-thread order
             const double d0 = o0 - C[i].x;
             acc = acc + d0 * d0;
@@ -256,7 +336,8 @@ __device__ __forceinline__ void consume_run_2d(const JbGeom &g, const Ring &R, R
 // 16 B (z-1) per pair.
 template <bool NOCOMP, bool NORM>
 __device__ __forceinline__ void consume_run_3d(const JbGeom &g, const Ring &R, RingPos &q, const Run &run,
-                                               const double *cur, double *nxt, double *remote, int ctid, int lane,
+                                               const double *cur, double *nxt, double *remote,
+                                               unsigned long long *rll, uint32_t tag, int ctid, int lane,
                                                double &acc) {
   const int ux = run.unit % g.units_x, uy = run.unit / g.units_x;
   const int64_t x0 = 1 + (int64_t)ux * g.tx;
@@ -276,12 +357,20 @@ __device__ __forceinline__ void consume_run_3d(const JbGeom &g, const Ring &R, R
   const int srow = (rb + 1) * ws + j;  // stage offset of (row rb, pair kk) center
   if (NOCOMP) {  // no-compute: the owned edge plane to the neighbour as-is, straight from L2
     for (int64_t p = 0; p < L; ++p) {
-      if (remote && ok) {
+      if ((remote || rll) && ok) {
         const double *c = cur + (run.p0 + p) * g.plane_elems + col;
-        double *o = remote + col;
-        for (int r = rb; r < re; ++r, c += g.pitch, o += g.pitch) {
-          const double2 v = __ldcg(reinterpret_cast<const double2 *>(c));
-          store_pair(o, v.x, v.y, full);
+        if (rll) {
+          unsigned long long *o = rll + 2 * col;
+          for (int r = rb; r < re; ++r, c += g.pitch, o += 2 * g.pitch) {
+            const double2 v = __ldcg(reinterpret_cast<const double2 *>(c));
+            ll_store_pair(o, v.x, v.y, full, tag);
+          }
+        } else {
+          double *o = remote + col;
+          for (int r = rb; r < re; ++r, c += g.pitch, o += g.pitch) {
+            const double2 v = __ldcg(reinterpret_cast<const double2 *>(c));
+            store_pair(o, v.x, v.y, full);
+          }
         }
       }
     }
@@ -295,6 +384,7 @@ __device__ __forceinline__ void consume_run_3d(const JbGeom &g, const Ring &R, R
   R.wait_full(pc);
   double *dst = nxt + run.p0 * g.plane_elems + col;
   double *rem = remote ? remote + col : nullptr;
+  unsigned long long *rlb = rll ? rll + 2 * col : nullptr;
   for (int64_t p = 0; p < L; ++p) {
     R.wait_full(pp);
     if (rb < re) {
@@ -303,6 +393,7 @@ __device__ __forceinline__ void consume_run_3d(const JbGeom &g, const Ring &R, R
       const double *d = R.stage(pm) + srow;
       double2 S = lds2(c - ws), C = lds2(c);
       double *o = dst, *ro = rem;
+      unsigned long long *rl = rlb;
 #pragma unroll 2
       for (int r = rb; r < re; ++r) {
         const double2 N = lds2(c + ws);
@@ -313,7 +404,8 @@ __device__ __forceinline__ void consume_run_3d(const JbGeom &g, const Ring &R, R
         const double o1 = kC6 * (((((e + C.x) + N.y) + S.y) + U.y) + D.y);
         if (ok) {
           store_pair(o, o0, o1, full);
-          if (ro) store_pair(ro, o0, o1, full);
+          if (rl) ll_store_pair(rl, o0, o1, full, tag);
+          else if (ro) store_pair(ro, o0, o1, full);
           if (NORM) {  // update norm (N4): fixed per-thread order
             const double d0 = o0 - C.x;
             acc = acc + d0 * d0;
@@ -330,6 +422,7 @@ __device__ __forceinline__ void consume_run_3d(const JbGeom &g, const Ring &R, R
         d += ws;
         o += g.pitch;
         if (ro) ro += g.pitch;
+        if (rl) rl += 2 * g.pitch;
       }
     }
     R.release(pm, lane);
@@ -345,16 +438,17 @@ __device__ __forceinline__ void consume_run_3d(const JbGeom &g, const Ring &R, R
 
 template <int DIM, bool NOCOMP, bool NORM>
 __device__ __forceinline__ void consume_run(const JbGeom &g, const Ring &R, RingPos &q, const Run &run,
-                                            const double *cur, double *nxt, double *remote, int ctid, int lane,
+                                            const double *cur, double *nxt, double *remote,
+                                            unsigned long long *rll, uint32_t tag, int ctid, int lane,
                                             double &acc) {
   if (DIM == 3) {
-    consume_run_3d<NOCOMP, NORM>(g, R, q, run, cur, nxt, remote, ctid, lane, acc);
+    consume_run_3d<NOCOMP, NORM>(g, R, q, run, cur, nxt, remote, rll, tag, ctid, lane, acc);
     return;
   }
   const int ppt = g.tx / (2 * JB_NC);
-  if (ppt >= 4) consume_run_2d<4, NOCOMP, NORM>(g, R, q, run, cur, nxt, remote, ctid, lane, acc);
-  else if (ppt == 2) consume_run_2d<2, NOCOMP, NORM>(g, R, q, run, cur, nxt, remote, ctid, lane, acc);
-  else consume_run_2d<1, NOCOMP, NORM>(g, R, q, run, cur, nxt, remote, ctid, lane, acc);
+  if (ppt >= 4) consume_run_2d<4, NOCOMP, NORM>(g, R, q, run, cur, nxt, remote, rll, tag, ctid, lane, acc);
+  else if (ppt == 2) consume_run_2d<2, NOCOMP, NORM>(g, R, q, run, cur, nxt, remote, rll, tag, ctid, lane, acc);
+  else consume_run_2d<1, NOCOMP, NORM>(g, R, q, run, cur, nxt, remote, rll, tag, ctid, lane, acc);
 }
 
 // ---------------------------------------------------------------- run-descriptor queue
@@ -517,6 +611,31 @@ __global__ void __launch_bounds__(JB_THREADS, 1) jb_sweep(const __grid_constant_
     if (role == ROLE_TOP && !SL.use_shm) remote = SL.peer_top[(tg + 1) & 1];
     if (role == ROLE_BOT && !SL.use_shm) remote = SL.peer_bot[(tg + 1) & 1];
     const bool active = !(NOCOMP && role == ROLE_INT);
+    // LL halo protocol (§5.11): iterations after the run's first receive LL cells, iterations
+    // before its last send them; the first / last halo of a run keep the flag protocol, so flags
+    // and halo planes are valid between runs of any kind.
+    const unsigned long long *llin = nullptr;
+    unsigned long long *llout = nullptr, *rll = nullptr;
+    if (PERSIST && !NORM && role != ROLE_INT) {
+      if (t > 0) llin = role == ROLE_TOP ? SL.ll_in_top[tg & 1] : SL.ll_in_bot[tg & 1];
+      if (t + 1 < P.iters) llout = role == ROLE_TOP ? SL.ll_out_top[(tg + 1) & 1] : SL.ll_out_bot[(tg + 1) & 1];
+      if (llout && !drop_signal) {  // (a dropped signal: plain halo stores, no LL cells)
+        rll = llout;
+        remote = nullptr;
+      }
+    }
+    const uint32_t tag_out = ll_tag(tg + 1);
+    if (llin) {
+      // receive this iteration's halo: every thread of the boundary CTA unpacks LL cells into the
+      // halo plane of cur, then the producer's bulk copies read it (generic -> async proxy fence)
+      const bool mark = threadIdx.x == JB_NC && ridx == 0;
+      if (mark) halo_mark(SL, P, role == ROLE_BOT, t, 0);
+      double *halo = SL.buf[tg & 1] + (role == ROLE_TOP ? 0 : SL.chunk + 1) * g.plane_elems;
+      ll_unpack(g, sched0, halo, llin, ll_tag(tg), P);  // (false: abort flag up, the barrier ends the run)
+      fence_proxy_async_global();
+      __syncthreads();
+      if (mark) halo_mark(SL, P, role == ROLE_BOT, t, 1);
+    }
 
     if (producer) {
       // Every lane that issues bulk copies orders them after the grid barrier's acquire (and the
@@ -527,7 +646,7 @@ __global__ void __launch_bounds__(JB_THREADS, 1) jb_sweep(const __grid_constant_
       // boundary blocks wait until the neighbour committed the halo of the previous time
       // step.  With compute, the two owned planes of the first boundary tile are already in
       // flight while we wait; only the halo plane's load waits for the flag.
-      bool waited = !(PERSIST && role != ROLE_INT);
+      bool waited = !(PERSIST && role != ROLE_INT) || llin != nullptr;
       auto wait_flag = [&]() {
         if (!waited) {
           const bool mark = PERSIST && lane == 0 && ridx == 0;
@@ -624,11 +743,14 @@ __global__ void __launch_bounds__(JB_THREADS, 1) jb_sweep(const __grid_constant_
           }
 #endif
           if (PERSIST && ctid == 0 && !drop_signal) {
-            unsigned long long *fo = role == ROLE_TOP ? SL.flag_out_top : SL.flag_out_bot;
-            st_release_sys(fo + ridx, (unsigned long long)(tg + 1));
+            if (!llout) {
+              unsigned long long *fo = role == ROLE_TOP ? SL.flag_out_top : SL.flag_out_bot;
+              st_release_sys(fo + ridx, (unsigned long long)(tg + 1));
+            }  // (LL: the cells carry their iteration, nothing to signal)
             if (ridx == 0) halo_mark(SL, P, role == ROLE_BOT, t, 2);
           }
           remote = nullptr;  // later (interior) runs stay local
+          rll = nullptr;
           continue;
         }
         Run run;
@@ -637,7 +759,7 @@ __global__ void __launch_bounds__(JB_THREADS, 1) jb_sweep(const __grid_constant_
         run.p1 = d.p1;
         double acc = 0.0;
         if (NORM && check) {
-          consume_run<DIM, NOCOMP, NORM>(g, R, q, run, cur, nxt, remote, ctid, lane, acc);
+          consume_run<DIM, NOCOMP, NORM>(g, R, q, run, cur, nxt, remote, rll, tag_out, ctid, lane, acc);
           // deterministic per-run sum: xor tree in each warp, then warps in order
           for (int o = 16; o > 0; o >>= 1) acc = acc + __shfl_xor_sync(0xffffffffu, acc, o);
           if (lane == 0) s_red[warp] = acc;
@@ -649,7 +771,7 @@ __global__ void __launch_bounds__(JB_THREADS, 1) jb_sweep(const __grid_constant_
           }
           named_bar_consumers();
         } else {
-          consume_run<DIM, NOCOMP, false>(g, R, q, run, cur, nxt, remote, ctid, lane, acc);
+          consume_run<DIM, NOCOMP, false>(g, R, q, run, cur, nxt, remote, rll, tag_out, ctid, lane, acc);
         }
       }
       // Our generic-proxy stores must be ordered before later bulk (async-proxy) reads.

@@ -14,7 +14,8 @@ for shape, P in [((20, 70), 2), ((8, 9, 33), 2), ((30, 40), 1)]:
     f = u12(shape, 3)
     for params, mode in [({"resident": 0}, jb.MODE_CPUFREE), ({"resident": 1}, jb.MODE_CPUFREE),
                          ({}, jb.MODE_BASELINE_MEMCPY), ({}, jb.MODE_BASELINE_P2P),
-                         ({"resident": 0, "norm_every": 2}, jb.MODE_CPUFREE)]:
+                         ({"resident": 0, "norm_every": 2}, jb.MODE_CPUFREE),
+                         ({"resident": 0, "tblock": 0, "halo_ll": 1}, jb.MODE_CPUFREE)]:  # LL halos
         with jb.Jacobi(shape, virtual=P) if P > 1 else jb.Jacobi(shape) as j:
             for k, v in params.items():
                 j.set_param(k, v)
