@@ -326,6 +326,7 @@ def main():
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--ref-iters", type=int, default=2, help="oracle iterations per reference step")
     ap.add_argument("--no-extras", action="store_true", help="skip e2e / cpu_baseline / baselines")
+    ap.add_argument("--no-pipeline", action="store_true", help="skip the pipelined e2e (two fields)")
     ap.add_argument("--no-clocks", action="store_true", help="(diagnostic) no nvidia-smi sampling")
     ap.add_argument("--virtual", type=int, default=0, help="(measurement aid) P slabs on one GPU")
     ap.add_argument("--param", action="append", default=[], help="tuning knob name=value (jacobi_set_param)")
@@ -660,6 +661,52 @@ def main():
                        "h2d_bytes_per_step": int(h2d_total), "d2h_bytes_per_step": int(d2h_total),
                        "ms_per_step": 1e3 * e2e_s / args.steps,
                        "path": "jacobi_scatter (pinned H2D) + jacobi_run + jacobi_gather (pinned D2H)"}
+
+        # ---- e2e, pipelined (one process): two fields on the device; while one step runs, a second
+        #      host thread gathers the previous step's result and scatters the next step's input on
+        #      the other field, through the same public calls (H2D / D2H overlap the compute; every
+        #      step still copies its whole input in and its whole result out inside the timed region)
+        if world == 1 and args.steps >= 2 and not args.no_pipeline:
+            import threading
+            j2 = jb.Jacobi(shape, virtual=args.virtual) if args.virtual else jb.Jacobi(shape, ngpus=n_gpus)
+            for kv in args.param:
+                k, v = kv.split("=")
+                j2.set_param(k, int(v))
+            hs = [j, j2]
+            h_out2 = torch.empty_like(h_out, pin_memory=True)
+            outs = [h_out.data_ptr() - lo * plane * 8, h_out2.data_ptr() - lo * plane * 8]
+            j2.run(iters)  # warm the second handle's plan
+            err = []
+
+            def copies(i):
+                try:
+                    if i >= 1:
+                        jb.jacobi_gather_ptr(hs[(i - 1) % 2].h, outs[(i - 1) % 2])
+                    if i + 1 < args.steps:
+                        jb.jacobi_scatter_ptr(hs[(i + 1) % 2].h, base_in)
+                except Exception as e:  # noqa: BLE001
+                    err.append(e)
+
+            t0 = time.perf_counter()
+            jb.jacobi_scatter_ptr(hs[0].h, base_in)
+            for i in range(args.steps):
+                th = threading.Thread(target=copies, args=(i,))
+                th.start()
+                hs[i % 2].run(iters)
+                th.join()
+            jb.jacobi_gather_ptr(hs[(args.steps - 1) % 2].h, outs[(args.steps - 1) % 2])
+            e2p_s = time.perf_counter() - t0
+            if err:
+                raise err[0]
+            same = bool(np.array_equal(h_out.numpy().view(np.uint64), h_out2.numpy().view(np.uint64)))
+            line["e2e_pipelined"] = {"value": cells * iters * args.steps / e2p_s / 1e9, "unit": UNIT,
+                                     "h2d_bytes_per_step": int(nbytes), "d2h_bytes_per_step": int(d2h),
+                                     "ms_per_step": 1e3 * e2p_s / args.steps, "fields": 2,
+                                     "results_identical": same,
+                                     "path": "two handles: jacobi_run of step i || (jacobi_gather of step i-1 + "
+                                             "jacobi_scatter of step i+1) on a second host thread"}
+            j2.close()
+            del h_out2
 
         # ---- parity of the measured configuration: the e2e step above scattered the U12 field and
         #      ran exactly `iters` iterations through the C ABI on these N GPUs, so the gathered
