@@ -449,12 +449,16 @@ def main():
     tb_iters = jb.jacobi_get_param(j.h, "last_tblock")
     tb_k = max(jb.jacobi_get_param(j.h, "last_tb_k"), 1)
     resident = bool(jb.jacobi_get_param(j.h, "last_resident"))
+    cluster_nc = jb.jacobi_get_param(j.h, "last_cluster")
     alg_bytes = round(local_cells * (16 * (iters - tb_iters) + 16 / tb_k * tb_iters))
     achieved = alg_bytes / (launch_ms / 1e3) / 1e9
     dimk = 2 if shape[0] == 1 else 3
     if tb_iters:
         kname = f"jb_tblock<{dimk},{tb_k},*> (persistent CPU-Free kernel, {tb_k} iterations per HBM pass)"
         kkind = "tblock"
+    elif cluster_nc:
+        kname = f"jb_cluster2d (one {cluster_nc}-CTA thread-block cluster, grid on chip, DSMEM halos, cluster barrier)"
+        kkind = "cluster"
     elif resident:
         kname = f"jb_resident<{dimk},*> (persistent CPU-Free kernel, on-chip resident)"
         kkind = "resident"

@@ -75,7 +75,8 @@ def main():
                         row = {"config": name, "slabs": P, "virtual": not real, "mode": mname,
                                "no_compute": nocomp, "us_per_iter": round(us, 3)}
                         if mname == "cpufree" and not nocomp:
-                            row["kernel"] = ("resident" if j.get_param("last_resident") else
+                            row["kernel"] = ("cluster" if j.get_param("last_cluster") else
+                                             "resident" if j.get_param("last_resident") else
                                              "tblock" if j.get_param("last_tblock") else "streaming")
                         if not nocomp:
                             cells = (shape[2] - 2) * (shape[1] - 2) * (shape[0] - 2 if shape[0] > 1 else 1)

@@ -191,6 +191,12 @@ int jacobi_set_mode(jacobi_t h, int mode, int flags);
  * GPUs).  Measurement: "halo_trace" (see jacobi_halo_trace; 0 = off, <= 2^20).
  * "barrier" (the CPU-Free kernels' device-side grid barrier: 0 = one counter per slab with
  * red.release + acquire spin (default), 1 = per-CTA arrival flags polled in parallel by every CTA).
+ * "cluster" (CPU-Free runs of ONE 2D slab that fits in the shared memory of one thread-block
+ * cluster of <= 16 CTAs, both time levels: the whole grid stays on chip, halo rows between the
+ * cluster's CTAs are read through DSMEM and the iteration barrier of P:372 is the hardware cluster
+ * barrier; with compute, no norm: -1 auto (default: used while "resident" and "tblock" are auto
+ * too — C1 2D 256^2 1.29 vs 2.33 us/iteration), 0 never, 1 always (EINVAL where it does not
+ * apply)); read-only "last_cluster" (its cluster size in the last CPU-Free run, 0 if not used).
  * "halo_ll" (streaming CPU-Free kernel, not with the norm: halo cells travel as tagged 16-byte LL
  * cells {tag:lo32, tag:hi32} that the receiving boundary CTAs poll and unpack into their halo
  * plane, instead of plain peer stores + one sys-scope release flag per boundary CTA and

@@ -9,7 +9,7 @@ HERE = os.path.dirname(os.path.abspath(__file__))
 ROOT = os.path.dirname(HERE)
 CSRC = os.path.join(HERE, "csrc")
 LIB = os.path.join(HERE, "libjacobi_b200.so")
-SOURCES = ["sweep.cu", "resident.cu", "tblock.cu", "util.cu", "runtime.cu", "baselines.cu", "multiproc.cu", "plan.cpp"]
+SOURCES = ["sweep.cu", "resident.cu", "tblock.cu", "cluster.cu", "util.cu", "runtime.cu", "baselines.cu", "multiproc.cu", "plan.cpp"]
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
 
 ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]

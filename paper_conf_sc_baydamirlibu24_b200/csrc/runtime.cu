@@ -916,12 +916,71 @@ int run_tblock(jacobi_ctx *h, int64_t iters, int K, int ppt, int lag, int ws) {
 // CPU-Free run: the temporally blocked kernel for as many whole pairs of time blocks as fit when
 // the run is eligible (one slab without neighbours, 2D, compute, no norm, not on-chip resident),
 // the per-iteration kernels (streaming / resident) for the rest.  Device times add up.
+// One-cluster on-chip kernel (cluster.cu) for a single 2D slab that fits in the
+// shared memory of one thread-block cluster: cluster size (0: not eligible) and shared memory.
+int cluster_plan(jacobi_ctx *h, size_t *smem) {
+  if (h->total != 1 || h->slabs.size() != 1 || h->dim != 2 || h->kind == KIND_SHMEM) return 0;
+  if ((h->flags & JACOBI_FLAG_NO_COMPUTE) || h->norm_every > 0) return 0;
+  Slab &s = h->slabs[0];
+  CK(cudaSetDevice(s.device));
+  int optin = 0;
+  CK(cudaDeviceGetAttribute(&optin, cudaDevAttrMaxSharedMemoryPerBlockOptin, s.device));
+  return jbk::cluster_choice(h->geom, s.chunk, std::min(optin, JB_SMEM_DEFAULT) - 1024, smem);
+}
+
+int run_cluster(jacobi_ctx *h, int64_t iters, int nc, size_t smem) {
+  Slab &s = h->slabs[0];
+  CK(cudaSetDevice(s.device));
+  JbParams P;
+  std::memset(&P, 0, sizeof(P));
+  P.g = h->geom;
+  P.nslabs = 1;
+  P.flags = h->flags;
+  P.t0 = h->t;
+  P.iters = iters;
+  P.timeout_ns = (unsigned long long)h->timeout_ms * 1000000ull;
+  P.status = s.ctrl->status;
+  JbSlab &d = P.s[0];
+  d.buf[0] = s.buf[0];
+  d.buf[1] = s.buf[1];
+  d.chunk = s.chunk;
+  d.cta_count = nc;
+  CK(reset_run_counters(s, s.stream));
+  ++h->last_launches;
+  CK(cudaEventRecord(s.ev0, s.stream));
+  CK(jbk::launch_cluster(P, nc, smem, s.stream));
+  ++h->last_launches;
+  CK(cudaEventRecord(s.ev1, s.stream));
+  CK(cudaEventSynchronize(s.ev1));
+  float ms = 0;
+  CK(cudaEventElapsedTime(&ms, s.ev0, s.ev1));
+  s.last_ms = ms;
+  h->last_ms_max = ms;
+  int rc = read_status(s);
+  if (rc) return rc;
+  h->t += iters;
+  return JACOBI_OK;
+}
+
 int run_cpufree(jacobi_ctx *h, int64_t iters) {
   h->last_launches = 0;
   h->last_tblock = 0;
   h->last_tb_k = 0;
   h->last_tb_ws = 0;
   h->last_resident = 0;
+  h->last_cluster = 0;
+  if (h->cluster != 0) {  // auto (JB_CLUSTER_AUTO): only while the other kernel knobs are auto too
+    size_t smem = 0;
+    const int nc = cluster_plan(h, &smem);
+    if (h->cluster == 1 && nc == 0) return JACOBI_EINVAL;
+    const bool use = nc > 0 && (h->cluster == 1 || (JB_CLUSTER_AUTO && h->tblock < 0 && h->resident < 0));
+    if (use) {
+      int rc = run_cluster(h, iters, nc, smem);
+      if (rc) return rc;
+      h->last_cluster = nc;
+      return JACOBI_OK;
+    }
+  }
   const bool nocomp = h->flags & JACOBI_FLAG_NO_COMPUTE;
   // P > 1: every slab needs the two edge zones (>= 2K planes); the NVSHMEM variant keeps jb_sweep
   int K = 0, ppt = 0, lag = 1, ws = 0;
@@ -1111,6 +1170,8 @@ static int64_t *param_slot(jacobi_t h, const char *name) {
   if (!std::strcmp(name, "halo_trace")) return &h->halo_trace;
   if (!std::strcmp(name, "barrier")) return &h->barrier;
   if (!std::strcmp(name, "halo_ll")) return &h->halo_ll;
+  if (!std::strcmp(name, "cluster")) return &h->cluster;
+  if (!std::strcmp(name, "last_cluster")) return &h->last_cluster;
   if (!std::strcmp(name, "last_launches")) return &h->last_launches;
   return nullptr;
 }
@@ -1118,7 +1179,7 @@ static int64_t *param_slot(jacobi_t h, const char *name) {
 int jacobi_set_param(jacobi_t h, const char *name, int64_t value) {
   if (!h || !name) return JACOBI_EINVAL;
   if (!std::strcmp(name, "last_resident") || !std::strcmp(name, "last_tblock") || !std::strcmp(name, "last_tb_k") ||
-      !std::strcmp(name, "last_launches") || !std::strcmp(name, "last_tb_ws"))
+      !std::strcmp(name, "last_launches") || !std::strcmp(name, "last_tb_ws") || !std::strcmp(name, "last_cluster"))
     return JACOBI_EINVAL;  // read-only
   int64_t *p = param_slot(h, name);
   if (!p) return JACOBI_EINVAL;

@@ -33,6 +33,8 @@ cudaError_t launch_flag_max(unsigned long long *flags, int n, unsigned long long
 cudaError_t prepare_resident(int dim, int cpp, size_t smem, int *blocks_per_sm);
 cudaError_t launch_resident(const JbParams &p, int cpp, int grid, size_t smem, cudaStream_t st);
 cudaError_t launch_neighbour_wait(const JbParams &p, unsigned long long target, cudaStream_t st);
+int cluster_choice(const JbGeom &g, int64_t chunk, int smem_optin, size_t *smem_out);
+cudaError_t launch_cluster(const JbParams &p, int nc, size_t smem, cudaStream_t st);
 int tblock_ty();
 int tblock_ncw(int dim, int k, int ppt, int lag, int per_sm, int ws = 0);
 size_t tblock_smem(const JbGeom &g);
@@ -200,6 +202,8 @@ struct jacobi_ctx {
   int64_t last_launches = 0;   // read-only: kernels this process launched in the last jacobi_run
   int64_t barrier = 0;         // grid barrier of the CPU-Free kernels: 0 counter, 1 per-CTA flags
   int64_t halo_trace = 0;      // measurement: record the first n halo exchanges of each CPU-Free run
+  int64_t cluster = -1;        // one-cluster on-chip kernel for small 2D grids (§5.12): -1 auto, 0 off, 1 force
+  int64_t last_cluster = 0;    // read-only: cluster size of the last CPU-Free run (0: not used)
   int64_t halo_ll = -1;        // LL halo protocol of the streaming CPU-Free kernel (§5.11): -1 auto, 0 off, 1 on
                                // (%globaltimer wait begin / flag acquired / signal; jacobi_halo_trace)
   int64_t norm_every = 0;      // N4: check the update norm every k iterations (0 = off)

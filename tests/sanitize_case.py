@@ -43,4 +43,12 @@ for shape, P, prm in [((24, 70), 2, {}), ((20, 70), 2, {"tb_k": 2}), ((12, 9, 33
         j.scatter(f)
         j.run(8)
         ok &= bool(np.array_equal(j.gather(), oracle.jacobi(f, 8)))
+# one-cluster kernel (DSMEM halo rows, cluster barriers), 16- and small clusters
+for shape in [(30, 40), (5, 70), (40, 13)]:
+    f = u12(shape, 5)
+    with jb.Jacobi(shape) as j:
+        j.set_param("cluster", 1)
+        j.scatter(f)
+        j.run(6)
+        ok &= bool(np.array_equal(j.gather(), oracle.jacobi(f, 6)))
 print("SANITIZE_CASE_OK" if ok else "SANITIZE_CASE_MISMATCH")

@@ -147,8 +147,11 @@ def test_tblock_invariants_and_special_fields(kv):
 
 def test_tblock_auto_selection_and_errors():
     f = u12((64, 96), 1)
-    with jb.Jacobi(f.shape) as j:  # fits on chip: auto keeps the resident kernel
+    with jb.Jacobi(f.shape) as j:  # fits in one cluster: auto takes the cluster kernel (§5.12)
         j.scatter(f)
+        j.run(8)
+        assert j.get_param("last_tblock") == 0 and j.get_param("last_cluster") > 0
+        j.set_param("cluster", 0)  # ... else the on-chip resident kernel
         j.run(8)
         assert j.get_param("last_tblock") == 0 and j.get_param("last_resident") == 1
         j.set_param("resident", 0)
