@@ -204,6 +204,11 @@ int jacobi_set_mode(jacobi_t h, int mode, int flags);
  * kind mix.  -1 auto (default: off), 0 off, 1 on.  DESIGN.md §5.11: removes the 1.5-3.9 us
  * MEMBAR.SYS of each release but doubles the halo bytes — measured equal or slower except 2D
  * no-compute / latency runs at 4-8 slabs).
+ * "flag_scope" (memory scope of the halo flags' release store and acquire poll, P:364-365 /
+ * P:394's signal and wait: -1 auto (default: .gpu for virtual slabs — every neighbour is a thread
+ * block group of the same launch on the same GPU — and .sys otherwise, which a neighbour on another
+ * GPU or in another process needs), 0 .sys always, 1 .gpu (EINVAL unless the handle was made by
+ * jacobi_create_virtual).  DESIGN.md §5.13: a .sys release costs 1.5-3.9 us, a .gpu one 0.4 us.
  * Unknown names return JACOBI_EINVAL. */
 int jacobi_set_param(jacobi_t h, const char *name, int64_t value);
 int jacobi_get_param(jacobi_t h, const char *name, int64_t *value);

@@ -98,6 +98,17 @@ __device__ __forceinline__ void st_release_gpu(unsigned long long *p, unsigned l
 __device__ __forceinline__ void st_release_sys(unsigned long long *p, unsigned long long v) {
   asm volatile("st.release.sys.global.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
 }
+// Halo flags: .sys scope when a neighbour may sit on another GPU or in another
+// process; .gpu when the host marked the launch as one device (virtual slabs, JB_PFLAG_GPU_SCOPE):
+// the release then skips the system-wide MEMBAR (1.5-3.9 us measured, profiles/r02_ubench_fence.txt).
+__device__ __forceinline__ bool flag_gpu_scope(const JbParams &P) { return (P.flags & JB_PFLAG_GPU_SCOPE) != 0; }
+__device__ __forceinline__ void st_release_flag(const JbParams &P, unsigned long long *p, unsigned long long v) {
+  if (flag_gpu_scope(P)) st_release_gpu(p, v);
+  else st_release_sys(p, v);
+}
+__device__ __forceinline__ unsigned long long ld_acquire_flag(const JbParams &P, const unsigned long long *p) {
+  return flag_gpu_scope(P) ? ld_acquire_gpu(p) : ld_acquire_sys(p);
+}
 __device__ __forceinline__ void red_release_gpu_add(unsigned long long *p, unsigned long long v) {
   asm volatile("red.release.gpu.global.add.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
 }
@@ -139,7 +150,7 @@ __device__ bool wait_slots(const unsigned long long *slots, int k, unsigned long
   uint32_t n = 0;
   volatile int *abort_flag = P.status + 1;
   while (true) {
-    const bool ok = lane >= k || ld_acquire_sys(slots + lane) >= target;
+    const bool ok = lane >= k || ld_acquire_flag(P, slots + lane) >= target;
     if (__all_sync(0xffffffffu, ok)) return true;
     if ((++n & 127u) == 0) {
       int stop = 0;

@@ -22,6 +22,8 @@
 #define JB_TB_KMAX3 3           // deepest time block of the 3D time-blocked kernel
 #define JB_TB_K3D 3             // its default depth (auto; slabs without neighbours only)
 #define JB_CLUSTER_AUTO 1        // cluster = -1 (auto): one-cluster kernel for small single 2D slabs on/off
+#define JB_PFLAG_GPU_SCOPE (1 << 30)  // JbParams::flags (internal): every peer of the launch is on this GPU -> halo
+                                      // flags released / acquired at .gpu instead of .sys scope (knob flag_scope)
 #define JB_LL_AUTO 0             // halo_ll = -1 (auto): LL halo protocol of the streaming kernel on/off
 #define JB_TB_RPW3 2            // 3D odd K: default rows per warp (x 11 warps)
 

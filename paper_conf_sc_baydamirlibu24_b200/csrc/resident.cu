@@ -192,8 +192,8 @@ __global__ void __launch_bounds__(JB_RNT, 1) jb_resident(const __grid_constant__
     if (top_blk || bot_blk) {
       __syncthreads();  // every thread's peer stores precede thread 0's release (CTA scope)
       if (tid == 0 && !((P.flags & JACOBI_FLAG_DROP_SIGNAL) && SL.slab_id == 0)) {
-        if (top_blk) st_release_sys(SL.flag_out_top + by, (unsigned long long)(tg + 1));
-        if (bot_blk) st_release_sys(SL.flag_out_bot + by, (unsigned long long)(tg + 1));
+        if (top_blk) st_release_flag(P, SL.flag_out_top + by, (unsigned long long)(tg + 1));
+        if (bot_blk) st_release_flag(P, SL.flag_out_bot + by, (unsigned long long)(tg + 1));
         if (by == 0) {
           if (top_blk) halo_mark(SL, P, 0, t, 2);
           if (bot_blk) halo_mark(SL, P, 1, t, 2);

@@ -238,6 +238,13 @@ void neighbour_roles(const jacobi_ctx *h, int id, int sms, int units, int *nt_ou
 // virtual mode).  persist=false plans the discrete baseline kernel (no boundary roles).
 
 
+// JB_PFLAG_GPU_SCOPE when every slab of the launch lives on one GPU in this process (virtual
+// slabs): the halo flags then need only .gpu scope (knob flag_scope).
+static int flag_scope_bits(const jacobi_ctx *h) {
+  const bool gpu = h->kind == KIND_VIRTUAL && h->flag_scope != 0;
+  return gpu ? JB_PFLAG_GPU_SCOPE : 0;
+}
+
 int plan_launch(jacobi_ctx *h, const std::vector<int> &idx, LaunchKind lk, bool nocomp, LaunchPlan &L,
                 int grid_override) {
   const bool persist = lk == LK_PERSIST;
@@ -284,7 +291,7 @@ int plan_launch(jacobi_ctx *h, const std::vector<int> &idx, LaunchKind lk, bool 
   std::memset(&P, 0, sizeof(P));
   P.g = g;
   P.nslabs = nslab;
-  P.flags = h->flags;
+  P.flags = h->flags | flag_scope_bits(h);
   P.timeout_ns = (unsigned long long)h->timeout_ms * 1000000ull;
   P.status = s0.ctrl->status;
   int begin = 0;
@@ -412,7 +419,7 @@ int plan_resident(jacobi_ctx *h, const std::vector<int> &idx, LaunchPlan &L) {
   P.g.res_rs = (int)((h->nx + 2) / 2 * 2);  // round_up(nx + 1, 2)
   if ((h->slabs[idx[0]].chunk + 3) * P.g.plane_elems >= ((int64_t)1 << 31)) return JACOBI_EINVAL;
   P.nslabs = (int)idx.size();
-  P.flags = h->flags;
+  P.flags = h->flags | flag_scope_bits(h);
   P.timeout_ns = (unsigned long long)h->timeout_ms * 1000000ull;
   P.status = s0.ctrl->status;
   auto tiling = [&](int id, int *nbz, int *nby, int *cpp, size_t *sm) {
@@ -935,7 +942,7 @@ int run_cluster(jacobi_ctx *h, int64_t iters, int nc, size_t smem) {
   std::memset(&P, 0, sizeof(P));
   P.g = h->geom;
   P.nslabs = 1;
-  P.flags = h->flags;
+  P.flags = h->flags | flag_scope_bits(h);
   P.t0 = h->t;
   P.iters = iters;
   P.timeout_ns = (unsigned long long)h->timeout_ms * 1000000ull;
@@ -1170,6 +1177,7 @@ static int64_t *param_slot(jacobi_t h, const char *name) {
   if (!std::strcmp(name, "halo_trace")) return &h->halo_trace;
   if (!std::strcmp(name, "barrier")) return &h->barrier;
   if (!std::strcmp(name, "halo_ll")) return &h->halo_ll;
+  if (!std::strcmp(name, "flag_scope")) return &h->flag_scope;
   if (!std::strcmp(name, "cluster")) return &h->cluster;
   if (!std::strcmp(name, "last_cluster")) return &h->last_cluster;
   if (!std::strcmp(name, "last_launches")) return &h->last_launches;
@@ -1187,6 +1195,7 @@ int jacobi_set_param(jacobi_t h, const char *name, int64_t value) {
   if (!std::strcmp(name, "tile_x") && value > 4096) return JACOBI_EINVAL;
   if (!std::strcmp(name, "tile_y") && value > 30) return JACOBI_EINVAL;
   if (!std::strcmp(name, "halo_trace") && (value < 0 || value > (1 << 20))) return JACOBI_EINVAL;
+  if (!std::strcmp(name, "flag_scope") && value > 0 && h->kind != KIND_VIRTUAL) return JACOBI_EINVAL;  // .gpu needs one device
   *p = value;
   h->plan_gen++;
   return JACOBI_OK;

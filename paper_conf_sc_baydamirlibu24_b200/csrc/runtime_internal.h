@@ -192,7 +192,7 @@ struct jacobi_ctx {
   int64_t tb_min_block = 16;   // smallest dynamic plane block of the temporally blocked kernel
   int64_t tb_ctas = 1;         // CTAs per SM of the temporally blocked kernel (1 or 2; K = 2 only)
   int64_t tb_k = -1;           // iterations per time block: -1 auto (2D: JB_TB_K2D = 5, 3D: JB_TB_K3D = 3); 2, 3, 5
-  int64_t tb_ppt = -1;         // 2D cell pairs per thread and level: -1 auto (4 for K <= 3, 2 for K = 5)
+  int64_t tb_ppt = -1;         // 2D cell pairs per thread and level: -1 auto (K = 2, 3: 4; K = 5: JB_TB_PPT5 = 1; 3D: 1)
   int64_t tb_lag = -1;         // 2D odd K: wavefront lag between levels (1 or 2; -1 auto)
   int64_t tb_rpw = -1;         // 3D odd K: rows per warp of the tile (-1 auto)
   int64_t tb_ws = -1;          // warp-specialised register split (12 compute warps; -1 auto = where built, 0 off)
@@ -204,6 +204,7 @@ struct jacobi_ctx {
   int64_t halo_trace = 0;      // measurement: record the first n halo exchanges of each CPU-Free run
   int64_t cluster = -1;        // one-cluster on-chip kernel for small 2D grids (§5.12): -1 auto, 0 off, 1 force
   int64_t last_cluster = 0;    // read-only: cluster size of the last CPU-Free run (0: not used)
+  int64_t flag_scope = -1;     // halo flag scope: -1 auto (.gpu for virtual slabs, .sys otherwise), 0 sys, 1 gpu
   int64_t halo_ll = -1;        // LL halo protocol of the streaming CPU-Free kernel (§5.11): -1 auto, 0 off, 1 on
                                // (%globaltimer wait begin / flag acquired / signal; jacobi_halo_trace)
   int64_t norm_every = 0;      // N4: check the update norm every k iterations (0 = off)

@@ -745,7 +745,7 @@ __global__ void __launch_bounds__(JB_THREADS, 1) jb_sweep(const __grid_constant_
           if (PERSIST && ctid == 0 && !drop_signal) {
             if (!llout) {
               unsigned long long *fo = role == ROLE_TOP ? SL.flag_out_top : SL.flag_out_bot;
-              st_release_sys(fo + ridx, (unsigned long long)(tg + 1));
+              st_release_flag(P, fo + ridx, (unsigned long long)(tg + 1));
             }  // (LL: the cells carry their iteration, nothing to signal)
             if (ridx == 0) halo_mark(SL, P, role == ROLE_BOT, t, 2);
           }
@@ -801,7 +801,7 @@ __global__ void __launch_bounds__(JB_THREADS, 1) jb_sweep(const __grid_constant_
           if (lane < SL.norm_slabs) {  // lane g delivers this slab's sum to slab g
             JbCtrl *dst = SL.norm_peers[lane];
             dst->norm_val[k & 1][SL.slab_id] = v;
-            st_release_sys(&dst->norm_flag[SL.slab_id], (unsigned long long)(k + 1));
+            st_release_flag(P, &dst->norm_flag[SL.slab_id], (unsigned long long)(k + 1));
           }
         }
         const bool ok = wait_slots(mine->norm_flag, SL.norm_slabs, (unsigned long long)(k + 1), P, lane);

@@ -1123,7 +1123,7 @@ __device__ __noinline__ bool tb_edge(const JbGeom &g, const JbSlab &SL, const Jb
     if constexpr (K >= 4) if (m == 4) tb_edge_phase<DIM, K, 4, NT>(g, top, C, cur, E, nxt, mid, remote, ub, ue);
     if constexpr (K >= 5) if (m == 5) tb_edge_phase<DIM, K, 5, NT>(g, top, C, cur, E, nxt, mid, remote, ub, ue);
     bar_edge();  // every thread's stores (local, neighbour's) precede the release below
-    if (tid == 0 && !drop) st_release_sys(fout, (unsigned long long)(tg + m));
+    if (tid == 0 && !drop) st_release_flag(P, fout, (unsigned long long)(tg + m));
     if (mark) halo_mark(SL, P, side, tg + m - 1 - P.t0, 2);
   }
   return true;

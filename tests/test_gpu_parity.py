@@ -419,3 +419,27 @@ def test_nccl_baseline_then_import_torch():
             "print('TORCH_OK', torch.cuda.is_available())\n") % ROOT_DIR
     r = subprocess.run([sys.executable, "-c", code], capture_output=True, text=True, timeout=300)
     assert "TORCH_OK True" in r.stdout, (r.stdout + r.stderr)[-3000:]
+
+
+# ---------------------------------------------------------------- halo flag scope
+@pytest.mark.parametrize("shape,virtual", [((66, 300), 3), ((23, 20, 70), 2), ((130, 1030), 4)])
+@pytest.mark.parametrize("kernel", [{"resident": 0, "tblock": 0}, {"resident": 1}, {"resident": 0, "tblock": 1},
+                                    {"resident": 0, "tblock": 0, "halo_ll": 1}])
+@pytest.mark.parametrize("scope", [0, 1])
+def test_flag_scope_virtual_bitwise(shape, virtual, kernel, scope):
+    """Virtual slabs with halo flags at .sys (flag_scope 0) and .gpu scope (1; auto for virtual
+    slabs): the same bits as the oracle, for the streaming, resident, time-blocked and LL kernels."""
+    f = u12(shape, 11)
+    got = run_gpu(f, 23, virtual=virtual, params={**kernel, "flag_scope": scope})
+    assert_bitwise(got, oracle.jacobi(f, 23), f"{shape} P={virtual} {kernel} scope={scope}")
+
+
+def test_flag_scope_knob():
+    """.gpu scope is refused for a handle whose slabs may live on other GPUs / processes."""
+    with jb.Jacobi((40, 40)) as j:
+        assert j.get_param("flag_scope") == -1
+        with pytest.raises(jb.JacobiError):
+            j.set_param("flag_scope", 1)
+        j.set_param("flag_scope", 0)
+    with jb.Jacobi((40, 40), virtual=2) as j:
+        j.set_param("flag_scope", 1)
