@@ -221,17 +221,61 @@ __device__ __forceinline__ void fence_acq_rel_gpu() { asm volatile("fence.acq_re
 //    polls all cta_count slots with relaxed loads issued in parallel (lane i: slots i, i+32, ..),
 //    then one fence.acq_rel.gpu (the acquire pattern) — no atomic serialised on one L2 address.
 // Returns false on abort / watchdog timeout (as wait_slots).
+// sig (lane 0, optional): a halo flag (P:394's signal) to raise with value sigv as part of the
+// arrival — one release fence (at the flag's scope) then relaxed stores of the flag and the
+// arrival, instead of the flag's own release store followed by the arrival's release.
+__device__ __forceinline__ void fence_acq_rel_sys() { asm volatile("fence.acq_rel.sys;" ::: "memory"); }
+__device__ __forceinline__ void st_relaxed_sys(unsigned long long *p, unsigned long long v) {
+  asm volatile("st.relaxed.sys.global.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
+}
+__device__ __forceinline__ void red_relaxed_gpu_add(unsigned long long *p, unsigned long long v) {
+  asm volatile("red.relaxed.gpu.global.add.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
+}
+__device__ __forceinline__ void st_relaxed_gpu(unsigned long long *p, unsigned long long v) {
+  asm volatile("st.relaxed.gpu.global.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
+}
 __device__ bool slab_barrier(const JbSlab &SL, const JbParams &P, int c, unsigned long long k,
-                             unsigned long long epoch, int lane) {
+                             unsigned long long epoch, int lane, unsigned long long *sig = nullptr,
+                             unsigned long long sigv = 0) {
+  // release pattern: fence, then relaxed stores of the flag and the arrival
+  auto fence_and_signal = [&]() {
+    if (flag_gpu_scope(P)) {
+      fence_acq_rel_gpu();
+      st_relaxed_gpu(sig, sigv);
+    } else {
+      fence_acq_rel_sys();
+      st_relaxed_sys(sig, sigv);
+    }
+  };
+  // The abort flag (another CTA's watchdog / error) is read right AFTER the arrival (not before:
+  // the arrival's release fence would wait for the load), so its L2 round trip overlaps the spin
+  // instead of following the barrier on every iteration's critical path; an abort raised later
+  // is seen by the spins (every 128 polls) or at the next barrier.
+  int aborted = 0;
   if (!SL.bar_flags) {
     bool ok = true;
     if (lane == 0) {
-      red_release_gpu_add(SL.barrier, 1ull);
-      ok = wait_geq<false>(SL.barrier, (unsigned long long)SL.cta_count * k, P);
+      if (sig) {
+        fence_and_signal();
+        red_relaxed_gpu_add(SL.barrier, 1ull);
+      } else {
+        red_release_gpu_add(SL.barrier, 1ull);
+      }
+      aborted = *(volatile int *)(P.status + 1);
+      ok = wait_geq<false>(SL.barrier, (unsigned long long)SL.cta_count * k, P) && !aborted;
     }
     return __shfl_sync(0xffffffffu, ok ? 1 : 0, 0) != 0;
   }
-  if (lane == 0) st_release_gpu(SL.bar_flags + c, epoch);
+  if (lane == 0) {
+    if (sig) {
+      fence_and_signal();
+      st_relaxed_gpu(SL.bar_flags + c, epoch);
+    } else {
+      st_release_gpu(SL.bar_flags + c, epoch);
+    }
+    aborted = *(volatile int *)(P.status + 1);
+  }
+  aborted = __shfl_sync(0xffffffffu, aborted, 0);
   const int n = SL.cta_count;
   const unsigned long long t_start = globaltimer();
   uint32_t cnt = 0;
@@ -256,7 +300,7 @@ __device__ bool slab_barrier(const JbSlab &SL, const JbParams &P, int c, unsigne
     }
   }
   fence_acq_rel_gpu();
-  return true;
+  return !aborted;
 }
 
 // Position in the shared-memory ring: slot and the parity of the current use of that slot.

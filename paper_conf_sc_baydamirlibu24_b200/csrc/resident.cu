@@ -17,7 +17,7 @@ namespace {
 template <int DIM, int CPP>
 __global__ void __launch_bounds__(JB_RNT, 1) jb_resident(const __grid_constant__ JbParams P) {
   extern __shared__ __align__(16) double tile[];
-  __shared__ int s_abort;
+  __shared__ int s_abort, s_abort_pw;
   const JbGeom &g = P.g;
   int si = 0;
   while (si + 1 < P.nslabs && (int)blockIdx.x >= P.s[si + 1].cta_begin) ++si;
@@ -74,7 +74,7 @@ __global__ void __launch_bounds__(JB_RNT, 1) jb_resident(const __grid_constant__
       if (bot_blk && lz == zb - 1) bot_face |= 1u << i;
     }
   }
-  if (tid == 0) s_abort = 0;
+  if (tid == 0) s_abort = s_abort_pw = 0;
   // neighbour blocks (face-sharing) for the relaxed synchronisation
   const bool relaxed = SL.res_relaxed != 0;
   int nbr[4], n_nbr = 0;
@@ -124,7 +124,9 @@ __global__ void __launch_bounds__(JB_RNT, 1) jb_resident(const __grid_constant__
     double *nxt = SL.buf[(tg + 1) & 1];
     // (1) halo: wait for the neighbour GPU's edge plane (and, with relaxed sync, for the
     //     neighbour blocks' faces of the previous iteration), then refresh the ring from L2
-    if (t > 0 && (top_blk || bot_blk || relaxed)) {
+    // (with the grid barrier, boundary blocks acquired the neighbour's flag during the last
+    //  barrier: the pre-wait below)
+    if (t > 0 && relaxed) {
       if (tid == 0 && by == 0) {
         if (top_blk) halo_mark(SL, P, 0, t, 0);
         if (bot_blk) halo_mark(SL, P, 1, t, 0);
@@ -209,10 +211,27 @@ __global__ void __launch_bounds__(JB_RNT, 1) jb_resident(const __grid_constant__
     }
     if (tid < 32) {
       const bool ok = slab_barrier(SL, P, c, (unsigned long long)(t + 1), (unsigned long long)(tg + 1), tid);
-      if (tid == 0) s_abort = (!ok || *(volatile int *)(P.status + 1)) ? 1 : 0;
+      if (tid == 0) s_abort = ok ? 0 : 1;  // (slab_barrier also reports an abort flag)
+    } else if (tid < 64 && (top_blk || bot_blk) && t + 1 < P.iters) {
+      // Pre-wait (P:394's wait, off the critical path): the neighbour raises the next
+      // iteration's flag in its own iteration t, independent of this slab's barrier, so warp 1
+      // polls it while warp 0 spins on the barrier instead of paying an L2 round trip after it.
+      const int ln = tid - 32;
+      if (ln == 0 && by == 0) {
+        if (top_blk) halo_mark(SL, P, 0, t + 1, 0);
+        if (bot_blk) halo_mark(SL, P, 1, t + 1, 0);
+      }
+      bool ok = true;
+      if (top_blk) ok &= wait_slots(SL.flag_in_top, SL.k_in_top, (unsigned long long)(tg + 1), P, ln);
+      if (bot_blk) ok &= wait_slots(SL.flag_in_bot, SL.k_in_bot, (unsigned long long)(tg + 1), P, ln);
+      if (ln == 0 && !ok) s_abort_pw = 1;
+      if (ln == 0 && by == 0) {
+        if (top_blk) halo_mark(SL, P, 0, t + 1, 1);
+        if (bot_blk) halo_mark(SL, P, 1, t + 1, 1);
+      }
     }
     __syncthreads();
-    if (s_abort) return;
+    if (s_abort || s_abort_pw) return;
   }
   // End of run: the neighbours' last halo planes have landed before the kernel completes.
   if (tid < 32 && P.iters > 0) {

@@ -599,11 +599,15 @@ __global__ void __launch_bounds__(JB_THREADS, 1) jb_sweep(const __grid_constant_
   RingPos q = {0u, 0u};   // data ring: producer and consumers advance identical copies
   RingPos rq = {0u, 0u};  // run queue
 
-  __shared__ int s_stop;
-  if (threadIdx.x == 0) s_stop = 0;
+  __shared__ int s_stop, s_abort_pw;
+  if (threadIdx.x == 0) s_stop = s_abort_pw = 0;
   int64_t done = P.iters;
+  bool prewaited = false;  // producer of a boundary CTA: this iteration's halo flag was acquired during the last barrier
   for (int64_t t = 0; t < P.iters; ++t) {
     const int64_t tg = P.t0 + t;
+    const bool pw = prewaited;
+    prewaited = false;
+    unsigned long long *sig_pending = nullptr;  // thread 0 (NOCOMP): flag to raise at the barrier
     const bool check = NORM && P.norm_every > 0 && (t + 1) % P.norm_every == 0;
     const double *cur = SL.buf[tg & 1];
     double *nxt = SL.buf[(tg + 1) & 1];
@@ -642,11 +646,11 @@ __global__ void __launch_bounds__(JB_THREADS, 1) jb_sweep(const __grid_constant_
       // generic-proxy stores it covers) with its own proxy fence.
       fence_proxy_async_global();
       // The claim counter of the next iteration is idle now (last used in iteration t-1).
-      if (lane == 0 && c == 0 && SL.work_ctr) SL.work_ctr[(tg + 1) & 1] = 0u;
+      if (!NOCOMP && lane == 0 && c == 0 && SL.work_ctr) SL.work_ctr[(tg + 1) & 1] = 0u;
       // boundary blocks wait until the neighbour committed the halo of the previous time
       // step.  With compute, the two owned planes of the first boundary tile are already in
       // flight while we wait; only the halo plane's load waits for the flag.
-      bool waited = !(PERSIST && role != ROLE_INT) || llin != nullptr;
+      bool waited = !(PERSIST && role != ROLE_INT) || llin != nullptr || pw;
       auto wait_flag = [&]() {
         if (!waited) {
           const bool mark = PERSIST && lane == 0 && ridx == 0;
@@ -745,7 +749,10 @@ __global__ void __launch_bounds__(JB_THREADS, 1) jb_sweep(const __grid_constant_
           if (PERSIST && ctid == 0 && !drop_signal) {
             if (!llout) {
               unsigned long long *fo = role == ROLE_TOP ? SL.flag_out_top : SL.flag_out_bot;
-              st_release_flag(P, fo + ridx, (unsigned long long)(tg + 1));
+              // no-compute: the CTA's next action is the grid barrier, so the signal shares the
+              // arrival's release fence (slab_barrier): one fence instead of two serialised ones
+              if (NOCOMP) sig_pending = fo + ridx;
+              else st_release_flag(P, fo + ridx, (unsigned long long)(tg + 1));
             }  // (LL: the cells carry their iteration, nothing to signal)
             if (ridx == 0) halo_mark(SL, P, role == ROLE_BOT, t, 2);
           }
@@ -783,11 +790,27 @@ __global__ void __launch_bounds__(JB_THREADS, 1) jb_sweep(const __grid_constant_
     // Device-side grid barrier of this slab's CTAs (P:372 grid.sync()).
     __syncthreads();
     if (warp == 0) {
-      const bool ok = slab_barrier(SL, P, c, (unsigned long long)(t + 1), (unsigned long long)(tg + 1), lane);
-      if (lane == 0) s_abort = (!ok || *(volatile int *)(P.status + 1)) ? 1 : 0;
+      const bool ok = slab_barrier(SL, P, c, (unsigned long long)(t + 1), (unsigned long long)(tg + 1), lane,
+                                   sig_pending, (unsigned long long)(tg + 1));
+      if (lane == 0) s_abort = ok ? 0 : 1;  // (slab_barrier also reports an abort flag)
+    } else if (PERSIST && producer && role != ROLE_INT && t + 1 < P.iters &&
+               (NORM || (role == ROLE_TOP ? SL.ll_in_top[(tg + 1) & 1] : SL.ll_in_bot[(tg + 1) & 1]) == nullptr)) {
+      // Pre-wait (P:394's wait, moved off the critical path): the neighbour's flag for the next
+      // iteration does not depend on this slab's barrier (the neighbour raises it in its own
+      // iteration t), so the boundary CTA's producer polls it while warp 0 spins on the barrier,
+      // instead of paying another L2 round trip after it.
+      const bool mark = lane == 0 && ridx == 0;
+      if (mark) halo_mark(SL, P, role == ROLE_BOT, t + 1, 0);
+      const bool ok = role == ROLE_TOP ? wait_slots(SL.flag_in_top, SL.k_in_top, (unsigned long long)(tg + 1), P, lane)
+                                       : wait_slots(SL.flag_in_bot, SL.k_in_bot, (unsigned long long)(tg + 1), P, lane);
+      if (mark) halo_mark(SL, P, role == ROLE_BOT, t + 1, 1);
+      __syncwarp();
+      fence_proxy_async_global();  // every copying lane: halo rows written by the neighbour
+      prewaited = ok;
+      if (!ok && lane == 0) s_abort_pw = 1;
     }
     __syncthreads();
-    if (s_abort) return;
+    if (s_abort || s_abort_pw) return;
     if (NORM && check) {
       // N4: all-reduce of the update norm over every slab (device-side, through the JbCtrl
       // norm slots of each slab), identical on every CTA of every GPU, then the stop decision.

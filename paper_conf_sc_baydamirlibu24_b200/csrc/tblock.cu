@@ -1325,7 +1325,7 @@ __device__ __forceinline__ void tb_body(const JbParams &P) {
       cta_sync();
       if (warp == 0) {
         const bool okb = slab_barrier(SL, P, c, (unsigned long long)(j + 1), (unsigned long long)(tg + K), lane);
-        if (lane == 0) s_abort = (!okb || *(volatile int *)(P.status + 1)) ? 1 : 0;
+        if (lane == 0) s_abort = okb ? 0 : 1;  // (slab_barrier also reports an abort flag)
       }
       cta_sync();
       if (s_abort) return;
