@@ -161,8 +161,8 @@ int jacobi_run(jacobi_t h, int64_t iters);
 int jacobi_set_mode(jacobi_t h, int mode, int flags);
 /* Tuning knobs (none changes results): "tile_x", "tile_y", "stages", "boundary_ctas",
  * "ctas" (persistent grid size per slab group, 0 = all co-resident), "schedule" (interior
- * work distribution: -1 auto = 2, 0 static linear, 1 static lockstep, 2 dynamic guided
- * self-scheduling), "min_block" (smallest dynamic block, planes, default 8), "dyn_help"
+ * work distribution: -1 auto = 2 for grids of >= 2^17 interior cells per CTA of the job, else 0;
+ * 0 static linear, 1 static lockstep, 2 dynamic guided self-scheduling), "min_block" (smallest dynamic block, planes, default 8), "dyn_help"
  * (1: boundary blocks join the dynamic interior after signalling), "resident" (CPU-Free runs
  * with compute keep each slab on chip — PERKS-style, P:335-337, P:406-408 — when it fits in the
  * shared memory/registers of its CTAs: -1 auto (default), 0 never, 1 always (EINVAL if it does
@@ -173,9 +173,9 @@ int jacobi_set_mode(jacobi_t h, int mode, int flags);
  * compute advance K iterations per pass over HBM — temporal blocking; slabs
  * with neighbours keep the per-iteration halo exchange through edge zones, which need 2K planes
  * per slab — for every whole multiple of K iterations (2K for K = 2), the rest per iteration:
- * -1 auto (default: 2D runs — except slabs that fit on chip, which use the resident kernel, unless a
- * single slab of >= 2^18 interior cells; 3D runs of one slab, or of slabs with a GPU each / >= 64
- * CTAs and >= 2^22 cells each), 0 never, 1 always (EINVAL when a slab has < 2K planes with P > 1,
+ * -1 auto (default: a single slab — except 2D slabs that fit on chip, which use the resident
+ * kernel, unless of >= 2^18 interior cells; slabs with neighbours when the grid has >= 2^16 (2D) /
+ * 3 x 2^16 (3D, and >= 64 CTAs per slab) interior cells per CTA of the job), 0 never, 1 always (EINVAL when a slab has < 2K planes with P > 1,
  * with the norm, in no-compute mode or in the NVSHMEM variant)), "tb_k" (iterations per time block: -1 auto = 5 in
  * 2D, 3 in 3D; 2D accepts 2, 3, 5, 3D 2, 3 — a deeper K than the slabs fit falls back to 3, then 2),
  * "tb_ppt" (2D cell pairs per lane and level: K = 2: from tile_x; K = 3: 2 or 4; K = 5: 1 (default,

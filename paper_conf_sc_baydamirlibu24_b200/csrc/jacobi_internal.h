@@ -25,6 +25,9 @@
 #define JB_PFLAG_GPU_SCOPE (1 << 30)  // JbParams::flags (internal): every peer of the launch is on this GPU -> halo
                                       // flags released / acquired at .gpu instead of .sys scope (knob flag_scope)
 #define JB_LL_AUTO 0             // halo_ll = -1 (auto): LL halo protocol of the streaming kernel on/off
+#define JB_DYN_MIN_CELLS (1 << 17)          // auto schedule: dynamic from this many interior cells per CTA (else static)
+#define JB_TB2_NB_MIN_CELLS (1 << 16)       // auto: 2D time-blocked kernel for slabs with neighbours from this many cells per CTA
+#define JB_TB3_NB_MIN_CELLS (3 << 16)       // ... and 3D (plus >= 64 CTAs per slab)
 #define JB_TB_RPW3 2            // 3D odd K: default rows per warp (x 11 warps)
 
 // Scratch planes after each slab buffer for the time-blocked kernel's edge zones of depth K

@@ -196,6 +196,25 @@ int launch_ctas(const jacobi_ctx *h, int sms) {
   return total;
 }
 
+// Interior cells of the whole grid per CTA of the whole job (every slab's CTAs on every GPU):
+// the same number on every rank, so the policies below agree across processes.
+int64_t cells_per_cta(const jacobi_ctx *h, int sms) {
+  const int64_t cells = (h->nx - 2) * (h->dim == 3 ? (h->ny - 2) * (h->nz - 2) : (h->ny - 2));
+  const int64_t devices = h->kind == KIND_VIRTUAL ? 1 : h->total;
+  return cells / std::max<int64_t>(1, (int64_t)launch_ctas(h, sms) * devices);
+}
+
+// Interior schedule of the per-iteration kernel: knob "schedule" 0 / 1 static, 2 dynamic; auto
+// (-1): dynamic guided self-scheduling for large grids (it absorbs the B200's per-SM speed spread
+// on HBM-bound sweeps: C2 / C3 0.93-0.99 of copy), static linear for grids of < JB_DYN_MIN_CELLS
+// interior cells per CTA, whose L2-resident iterations are latency-bound and where every claim
+// (an atomic plus the block-table reads) sits on the critical path: 3D 128^3 18.0 -> 12.5 us,
+// 2D 2048^2 with 2-8 virtual slabs 15.7 -> 11.1-12.2 us per iteration.
+bool schedule_dynamic(const jacobi_ctx *h, int sms) {
+  if (h->schedule >= 0) return h->schedule == 2;
+  return cells_per_cta(h, sms) >= JB_DYN_MIN_CELLS;
+}
+
 // CTAs of slab `id` in its CPU-Free launch.
 int slab_ctas(const jacobi_ctx *h, int id, int sms) {
   const int total = launch_ctas(h, sms);
@@ -204,9 +223,9 @@ int slab_ctas(const jacobi_ctx *h, int id, int sms) {
 }
 
 // Boundary / interior split of a slab's CTAs (reconstructed P:398-404; R11).
-void split_roles(const jacobi_ctx *h, int count, int64_t inner, bool top, bool bot, int units, int *nt,
+void split_roles(const jacobi_ctx *h, int sms, int count, int64_t inner, bool top, bool bot, int units, int *nt,
                  int *nb, int *ni) {
-  const bool dynamic = h->schedule == 2 || h->schedule < 0;
+  const bool dynamic = schedule_dynamic(h, sms);
   int override_ps = (int)h->boundary_ctas;
   if (override_ps <= 0 && dynamic && h->dyn_help && inner > 0 && (top || bot)) {
     // Boundary CTAs join the dynamic interior after signalling, so give every boundary unit its
@@ -227,7 +246,7 @@ void neighbour_roles(const jacobi_ctx *h, int id, int sms, int units, int *nt_ou
   const bool top = id > 0, bot = id < h->total - 1;
   const int64_t inner = (bot ? chunk - 1 : chunk) - (top ? 2 : 1) + 1;
   int nt, nb, ni;
-  split_roles(h, slab_ctas(h, id, sms), inner, top, bot, units, &nt, &nb, &ni);
+  split_roles(h, sms, slab_ctas(h, id, sms), inner, top, bot, units, &nt, &nb, &ni);
   if (nt_out) *nt_out = nt;
   if (nb_out) *nb_out = nb;
 }
@@ -338,8 +357,8 @@ int plan_launch(jacobi_ctx *h, const std::vector<int> &idx, LaunchKind lk, bool 
     const int64_t inner = hi - lo + 1;
     int nt, nb, ni;
     if (count < (top ? 1 : 0) + (bot ? 1 : 0) + (inner > 0 ? 1 : 0)) return JACOBI_ENOCOOP;
-    const bool dynamic = h->schedule == 2 || h->schedule < 0;
-    split_roles(h, count, inner, top, bot, g.units, &nt, &nb, &ni);
+    const bool dynamic = schedule_dynamic(h, sms);
+    split_roles(h, sms, count, inner, top, bot, g.units, &nt, &nb, &ni);
     d.n_top = nt;
     d.n_bot = nb;
     if (persist || lk == LK_P2P) {
@@ -994,26 +1013,23 @@ int run_cpufree(jacobi_ctx *h, int64_t iters) {
   tblock_choice(h, &K, &ppt, &lag, &ws);
   const bool eligible = h->tblock != 0 && !nocomp && h->norm_every <= 0 && h->kind != KIND_SHMEM && K >= 2;
   if (h->tblock == 1 && !eligible) return JACOBI_EINVAL;
-  // auto picks it where it measured faster than the per-iteration kernel: 2D always; 3D when the
-  // slabs have no neighbours, or when every slab has a GPU of its own (>= 100 CTAs), or >= 64
-  // CTAs and >= 2^22 interior cells — the 3D edge zones are whole planes (K phases x 2K-m planes
-  // per side, computed by at most a quarter of the slab's CTAs, one neighbour flag round trip per
-  // phase): with 2 virtual slabs that pays for C3 (467 vs 384 Gcell/s) but not for the 128^3
-  // latency grid (22.7 vs 18.5 us/iteration), and it does not with 4-8 virtual slabs
-  bool use3 = h->total == 1;
-  if (!use3 && h->dim == 3) {
+  // auto picks it where it measured faster than the per-iteration kernel: always for a slab
+  // without neighbours; with neighbours the K phases of edge zones (each waiting for the
+  // neighbour's previous phase) must be amortised by enough interior work per CTA — 2D >= 2^16
+  // interior cells per CTA of the job (2048^2 with 2-8 virtual slabs, 28 K: 17.3 vs 11.0-12.2
+  // us/iteration per-iteration; 4096^2, 113 K: 22.6-28.0 vs 42-44), 3D >= 3 * 2^16 and >= 64
+  // CTAs per slab (256^3 with 2 virtual slabs, 111 K: 57.9 vs 49.8 us; 384^3, 380 K: 139 vs 191;
+  // C3 with 2 virtual slabs 467 vs 384 Gcell/s; with 8, 18 CTAs per slab: 251 vs 340 — DESIGN.md
+  // §5.9, §5.14).
+  bool use_tb = h->total == 1;
+  if (!use_tb) {
     int sms = 0;
     CK(cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, h->slabs[0].device));
-    use3 = true;
-    for (int id = 0; id < h->total; ++id) {
-      int64_t st, ch;
-      jbplan::decompose(h->n_out, h->total, id, &st, &ch);
-      const int n = slab_ctas(h, id, sms);
-      const int64_t cells = ch * (h->nx - 2) * (h->ny - 2);
-      use3 = use3 && (n >= 100 || (n >= 64 && cells >= ((int64_t)1 << 22)));
-    }
+    const int64_t cpc = cells_per_cta(h, sms);
+    use_tb = cpc >= (h->dim == 3 ? JB_TB3_NB_MIN_CELLS : JB_TB2_NB_MIN_CELLS);
+    for (int id = 0; id < h->total && use_tb && h->dim == 3; ++id) use_tb = slab_ctas(h, id, sms) >= 64;
   }
-  const bool use = eligible && (h->tblock == 1 || h->dim == 2 || use3);
+  const bool use = eligible && (h->tblock == 1 || use_tb);
   int64_t tb_iters = 0;
   if (use) {
     // odd K: any block count; K = 2: an even one (the result stays in buf[t & 1], R10)

@@ -274,12 +274,13 @@ def test_tblock_virtual_mixing_and_decomposition():
     exp = oracle.jacobi(f, 37)
     with jb.Jacobi(f.shape, virtual=4) as j:
         j.set_param("resident", 0)
+        j.set_param("tblock", 1)  # (auto keeps this small grid per-iteration: 2D auto selection test)
         j.scatter(f)
         j.run(8)
         assert j.get_param("last_tblock") == 5     # chunk 17: K = 5
         j.set_param("tblock", 0)
         j.run(3)
-        j.set_param("tblock", -1)
+        j.set_param("tblock", 1)
         j.set_mode(jb.MODE_BASELINE_MEMCPY)
         j.run(2)
         j.set_mode(jb.MODE_CPUFREE)
@@ -409,9 +410,9 @@ def test_tblock_3d_invariants_and_mixing():
 
 def test_tblock_3d_auto_selection():
     """3D auto: time-blocked K = 3 for a slab without neighbours and for slabs with neighbours
-    that have a GPU each (>= 100 CTAs) or >= 64 CTAs and >= 2^22 cells (2 virtual slabs of a
-    large grid); per-iteration for small slabs with few CTAs and when 4+ virtual slabs share one
-    GPU (whole-plane edge zones on too few CTAs measured slower there)."""
+    when the grid has >= 3 x 2^16 interior cells per CTA of the job and every slab >= 64 CTAs
+    (2 virtual slabs of a large grid); per-iteration for smaller grids and when 4+ virtual slabs
+    share one GPU (whole-plane edge zones on too few CTAs measured slower there)."""
     with jb.Jacobi((20, 30, 40)) as j:
         j.set_param("resident", 0)
         j.run(8)
@@ -420,7 +421,14 @@ def test_tblock_3d_auto_selection():
         j.set_param("resident", 0)
         j.run(8)
         assert j.get_param("last_tblock") == 0
-    f = u12((36, 512, 512), 4)  # 17 planes x 510^2 cells per slab >= 2^22
+    f = u12((36, 512, 512), 4)  # 34 x 510^2 cells: 60 K per CTA < 3 x 2^16
+    with jb.Jacobi(f.shape, virtual=2) as j:
+        j.set_param("resident", 0)
+        j.scatter(f)
+        j.run(8)
+        assert j.get_param("last_tblock") == 0
+        assert_bitwise(j.gather(), oracle.jacobi(f, 8, 8), "3D auto, 2 mid-size virtual slabs")
+    f = u12((130, 512, 512), 4)  # 128 x 510^2 cells: 225 K per CTA
     with jb.Jacobi(f.shape, virtual=2) as j:
         j.set_param("resident", 0)
         j.scatter(f)
@@ -452,3 +460,17 @@ def test_c3_1000_iters_tblock_equals_per_iteration():
             assert j.get_param("last_tb_k") == k
             assert j.get_param("last_tblock") == tb_iters(1000, k)
             assert_bitwise(j.gather(), ref, f"C3 tblock P={P or 1} K={k}")
+
+
+def test_tblock_2d_auto_selection():
+    """2D auto with neighbours: time-blocked K = 5 when the grid has >= 2^16 interior cells per
+    CTA of the job (3202^2 over 148 CTAs: 69 K), per-iteration below (1026^2: 7 K) — where the
+    per-iteration kernel's static schedule measured faster; bitwise either way."""
+    for n, tb in [(1026, 0), (3202, 10)]:
+        f = u12((n, n), 5)
+        with jb.Jacobi(f.shape, virtual=2) as j:
+            j.set_param("resident", 0)
+            j.scatter(f)
+            j.run(10)
+            assert j.get_param("last_tblock") == tb, n
+            assert_bitwise(j.gather(), oracle.jacobi(f, 10, 8), f"2D auto {n}^2, 2 virtual slabs")
