@@ -226,10 +226,12 @@ int slab_ctas(const jacobi_ctx *h, int id, int sms) {
 void split_roles(const jacobi_ctx *h, int sms, int count, int64_t inner, bool top, bool bot, int units, int *nt,
                  int *nb, int *ni) {
   const bool dynamic = schedule_dynamic(h, sms);
+  const bool nocomp = (h->flags & JACOBI_FLAG_NO_COMPUTE) != 0;
   int override_ps = (int)h->boundary_ctas;
-  if (override_ps <= 0 && dynamic && h->dyn_help && inner > 0 && (top || bot)) {
-    // Boundary CTAs join the dynamic interior after signalling, so give every boundary unit its
-    // own CTA (shortest halo critical path), up to a quarter of the grid per side.
+  if (override_ps <= 0 && ((dynamic && h->dyn_help) || nocomp) && inner > 0 && (top || bot)) {
+    // Boundary CTAs join the dynamic interior after signalling (or, without compute, the
+    // interior has nothing to do), so give every boundary unit its own CTA (shortest halo
+    // critical path), up to a quarter of the grid per side.
     override_ps = (int)std::max<int64_t>(1, std::min<int64_t>(units, count / 4));
   }
   override_ps = std::min(override_ps, JB_MAXK);

@@ -641,10 +641,13 @@ __global__ void __launch_bounds__(JB_THREADS, 1) jb_sweep(const __grid_constant_
       if (mark) halo_mark(SL, P, role == ROLE_BOT, t, 1);
     }
 
-    if (producer) {
+    // (no-compute: interior CTAs have no runs — they only join the barrier — and no CTA issues
+    //  bulk copies, so the queue hand-off and the generic -> async proxy fences are skipped)
+    if (NOCOMP && role == ROLE_INT) {
+    } else if (producer) {
       // Every lane that issues bulk copies orders them after the grid barrier's acquire (and the
       // generic-proxy stores it covers) with its own proxy fence.
-      fence_proxy_async_global();
+      if (!NOCOMP) fence_proxy_async_global();
       // The claim counter of the next iteration is idle now (last used in iteration t-1).
       if (!NOCOMP && lane == 0 && c == 0 && SL.work_ctr) SL.work_ctr[(tg + 1) & 1] = 0u;
       // boundary blocks wait until the neighbour committed the halo of the previous time
@@ -659,7 +662,7 @@ __global__ void __launch_bounds__(JB_THREADS, 1) jb_sweep(const __grid_constant_
           else wait_slots(SL.flag_in_bot, SL.k_in_bot, (unsigned long long)tg, P, lane);
           if (mark) halo_mark(SL, P, role == ROLE_BOT, t, 1);
           __syncwarp();
-          fence_proxy_async_global();  // every copying lane: halo rows written by the neighbour
+          if (!NOCOMP) fence_proxy_async_global();  // every copying lane: halo rows written by the neighbour
           waited = true;
         }
       };
@@ -782,7 +785,7 @@ __global__ void __launch_bounds__(JB_THREADS, 1) jb_sweep(const __grid_constant_
         }
       }
       // Our generic-proxy stores must be ordered before later bulk (async-proxy) reads.
-      fence_proxy_async_global();
+      if (!NOCOMP) fence_proxy_async_global();
     }
     if (!PERSIST) break;
     if (P.trace && t < 8 && threadIdx.x == 0) P.trace[t * gridDim.x + blockIdx.x] = globaltimer();
@@ -805,7 +808,7 @@ __global__ void __launch_bounds__(JB_THREADS, 1) jb_sweep(const __grid_constant_
                                        : wait_slots(SL.flag_in_bot, SL.k_in_bot, (unsigned long long)(tg + 1), P, lane);
       if (mark) halo_mark(SL, P, role == ROLE_BOT, t + 1, 1);
       __syncwarp();
-      fence_proxy_async_global();  // every copying lane: halo rows written by the neighbour
+      if (!NOCOMP) fence_proxy_async_global();  // every copying lane: halo rows written by the neighbour
       prewaited = ok;
       if (!ok && lane == 0) s_abort_pw = 1;
     }
