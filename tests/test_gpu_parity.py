@@ -443,3 +443,25 @@ def test_flag_scope_knob():
         j.set_param("flag_scope", 0)
     with jb.Jacobi((40, 40), virtual=2) as j:
         j.set_param("flag_scope", 1)
+
+
+@pytest.mark.parametrize("params,flags", [({"resident": 0, "tblock": 0}, 0),
+                                          ({"resident": 0, "tblock": 0}, jb.FLAG_NO_COMPUTE),
+                                          ({"resident": 1}, 0), ({"resident": 1, "block_sync": 1}, 0),
+                                          ({"resident": 0, "tblock": 1}, 0)])
+@pytest.mark.parametrize("scope", [0, 1])
+def test_watchdog_every_kernel(params, flags, scope):
+    """DROP_SIGNAL on slab 0 with every CPU-Free kernel and both flag scopes: the waits that moved
+    into the barrier (pre-wait) and the no-compute signal folded into the arrival still end in
+    JACOBI_ETIMEOUT, not a hang, and the next run on a new handle is bitwise."""
+    with jb.Jacobi((40, 200), virtual=2) as j:
+        j.set_param("timeout_ms", 300)
+        j.set_param("flag_scope", scope)
+        for k, v in params.items():
+            j.set_param(k, v)
+        j.set_mode(jb.MODE_CPUFREE, jb.FLAG_DROP_SIGNAL | flags)
+        with pytest.raises(jb.JacobiError) as e:
+            j.run(10)
+        assert e.value.code == jb.JACOBI_ETIMEOUT
+    f = u12((40, 200), 1)
+    assert_bitwise(run_gpu(f, 5, virtual=2, params=params), oracle.jacobi(f, 5), f"after timeout {params}")
