@@ -225,7 +225,7 @@ def emit(line: dict) -> None:
 def golden_digest(shape, iters):
     """The oracle digest of this workload (U12 seed 0x5C24, `iters` iterations), if committed."""
     want = list(shape if shape[0] > 1 else shape[1:])
-    for fn in ("oracle_digests_full.json", "oracle_digests.json"):
+    for fn in ("oracle_digests_full.json", "oracle_digests_latency.json", "oracle_digests.json"):
         try:
             with open(os.path.join(ROOT, "tests", "golden", fn)) as f:
                 d = json.load(f)

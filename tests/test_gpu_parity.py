@@ -405,6 +405,26 @@ def test_gpu_matches_golden_digests():
             assert hashlib.sha256(np.ascontiguousarray(r).tobytes()).hexdigest() == g["sha256"], (name, virtual)
 
 
+@pytest.mark.parametrize("virtual", [0, 2, 4, 8])
+@pytest.mark.parametrize("mode", ["auto", "graph"])
+def test_gpu_matches_latency_digests(virtual, mode):
+    """C5 latency workloads (3D 128^3, 2D 1024^2) at 1000 iterations with 1-8 slabs, the auto
+    kernel (time-blocked / static-schedule streaming / resident) and the CUDA-graph baseline: the
+    whole field equals the committed oracle digest (tests/golden/oracle_digests_latency.json)."""
+    import hashlib
+    import json
+    import os
+    with open(os.path.join(os.path.dirname(__file__), "golden", "oracle_digests_latency.json")) as f:
+        gold = json.load(f)
+    for name, g in gold.items():
+        with jb.Jacobi(tuple(g["shape"]), virtual=virtual) as j:  # created with U12 seed 0x5C24
+            if mode == "graph":
+                j.set_mode(jb.MODE_BASELINE_GRAPH)
+            j.run(g["iters"])
+            r = j.gather()
+        assert hashlib.sha256(np.ascontiguousarray(r).tobytes()).hexdigest() == g["sha256"], (name, virtual, mode)
+
+
 def test_nccl_baseline_then_import_torch():
     """The NCCL baseline loads the same libnccl.so.2 PyTorch ships (JACOBI_NCCL_LIB, set by the
     binding): running it BEFORE `import torch` must not leave a different NCCL in the process
