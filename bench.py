@@ -627,6 +627,18 @@ def main():
                 j.set_mode(jb.MODE_CPUFREE)
         else:
             line["halo_us"] = None  # one slab: no halo; see bench_latency.py (virtual slabs)
+            # Context at N = 1: the same grid split into 2 VIRTUAL slabs on this GPU (thread-block
+            # groups running the complete flag / halo protocol; no NVLink), no-compute per-iteration
+            # time of the CPU-Free kernel vs the CPU-controlled baselines.
+            try:
+                with jb.Jacobi(shape, virtual=2) as jv:
+                    line["halo_us_virtual2"] = dict(
+                        halo_latency(jv, jb, [("cpufree", jb.MODE_CPUFREE),
+                                              ("baseline_memcpy", jb.MODE_BASELINE_MEMCPY),
+                                              ("baseline_graph", jb.MODE_BASELINE_GRAPH)], lambda x: x),
+                        note="2 virtual slabs of this grid on one GPU (no NVLink); us per no-compute iteration")
+            except (jb.JacobiError, ValueError) as e:
+                line["halo_us_virtual2"] = {"error": str(e)}
 
         # ---- e2e through the C ABI with pinned host buffers (scatter + run + gather per step)
         from jacobi_inputs import u12_flat
