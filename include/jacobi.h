@@ -287,6 +287,15 @@ int jacobi_tb_split(int ctas, int64_t chunk, int has_top, int has_bottom, int64_
                     int override_per_side, int *out3);
 /* Geometry chosen for a grid: out[0..7] = pitch, plane_elems, tile_x, tile_y, units_x,
  * units_y, stage_rows, stage_row_doubles.  tile_x/tile_y <= 0 pick defaults. */
+/* Host-only (no GPU needed): the auto policies of DESIGN.md §5.14 for a grid split into `nslabs`
+ * slabs — one GPU each with `sms` SMs (virtual_slabs = 0), or all on one GPU (virtual_slabs = 1).
+ * out4[0] = interior cells per CTA of the whole job, out4[1] = 1 if the per-iteration kernel's
+ * interior schedule is dynamic (knob schedule = -1), out4[2] = 1 if CPU-Free runs with compute
+ * take the time-blocked kernel (knob tblock = -1; always 1 for one slab), out4[3] = CTAs of the
+ * smallest slab.  Functions of the global problem only, so every rank decides the same.
+ * Bad extents / stencil, nslabs < 1, sms < 1, out4 NULL: JACOBI_EINVAL. */
+int jacobi_auto_policy(int64_t nx, int64_t ny, int64_t nz, int stencil, int nslabs, int virtual_slabs, int sms,
+                       int64_t *out4);
 int jacobi_geometry(int64_t nx, int64_t ny, int64_t nz, int stencil, int tile_x, int tile_y,
                     int64_t *out8);
 int jacobi_version(void);

@@ -67,6 +67,7 @@ _SIGS = {
     "jacobi_decompose": ([_i64, _c.c_int, _c.c_int, _c.POINTER(_i64), _c.POINTER(_i64)], _c.c_int),
     "jacobi_tb_split": ([_c.c_int, _i64, _c.c_int, _c.c_int, _i64, _c.c_int, _c.POINTER(_c.c_int)], _c.c_int),
     "jacobi_geometry": ([_i64, _i64, _i64, _c.c_int, _c.c_int, _c.c_int, _c.POINTER(_i64)], _c.c_int),
+    "jacobi_auto_policy": ([_i64, _i64, _i64, _c.c_int, _c.c_int, _c.c_int, _c.c_int, _c.POINTER(_i64)], _c.c_int),
     "jacobi_version": ([], _c.c_int),
     "jacobi_set_allocator": ([_p, _p, _p], _c.c_int),
     "jacobi_open_ranks": ([_p, _p, _c.c_int], _c.c_int),
@@ -342,6 +343,14 @@ def jacobi_geometry(nx, ny, nz, stencil, tile_x=0, tile_y=0) -> dict:
     o = (_i64 * 8)()
     _check(lib().jacobi_geometry(nx, ny, nz, stencil, tile_x, tile_y, o), "jacobi_geometry")
     return dict(zip(GEOMETRY_KEYS, list(o)))
+
+
+def jacobi_auto_policy(nx, ny, nz, stencil, nslabs, virtual=False, sms=148) -> dict:
+    """Host-only auto policies of the C ABI: cells per CTA of the job, dynamic
+    interior schedule, time-blocked kernel, CTAs of the smallest slab."""
+    o = (_i64 * 4)()
+    _check(lib().jacobi_auto_policy(nx, ny, nz, stencil, nslabs, 1 if virtual else 0, sms, o), "jacobi_auto_policy")
+    return {"cells_per_cta": o[0], "dynamic_schedule": bool(o[1]), "tblock": bool(o[2]), "min_slab_ctas": o[3]}
 
 
 def jacobi_version() -> int:

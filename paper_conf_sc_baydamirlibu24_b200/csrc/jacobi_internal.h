@@ -197,6 +197,10 @@ void tb_split(int ctas, int64_t inner_planes, int has_top, int has_bot, int64_t 
 int choose_ty(int64_t ny, int units_x, int n_int, int smem_bytes, int ws);
 int tallest_ty(int64_t ny, int smem_bytes, int ws);
 int lockstep_k(int units, int n_int, int64_t inner_planes);
+// Auto policies of DESIGN.md §5.14 (global inputs only: identical on every rank).
+int64_t cells_per_cta(int64_t nx, int64_t ny, int64_t nz, int dim, int64_t job_ctas);
+bool schedule_dynamic_auto(int64_t cells_per_cta);
+bool tblock_neighbours_auto(int dim, int64_t cells_per_cta, int min_slab_ctas);
 // Number of plane blocks of the guided dynamic schedule (see JbSlab::dyn_min_blk).
 int64_t dyn_blocks(int64_t npl, int units, int n, int min_blk, int32_t *table = nullptr);
 // Resident (on-chip) tiling of a slab of `chunk` planes over at most `count` CTAs: nbz x nby

@@ -97,6 +97,18 @@ void tb_split(int ctas, int64_t inner, int has_top, int has_bot, int64_t units, 
   if (inner <= 0) *n_int = std::max(*n_int, 0);
 }
 
+// Auto policies, functions of the global problem only, so that every rank /
+// process takes the same decision: interior cells of the grid per CTA of the whole job.
+int64_t cells_per_cta(int64_t nx, int64_t ny, int64_t nz, int dim, int64_t job_ctas) {
+  const int64_t cells = (nx - 2) * (dim == 3 ? (ny - 2) * (nz - 2) : (ny - 2));
+  return cells / std::max<int64_t>(1, job_ctas);
+}
+bool schedule_dynamic_auto(int64_t cpc) { return cpc >= JB_DYN_MIN_CELLS; }
+bool tblock_neighbours_auto(int dim, int64_t cpc, int min_slab_ctas) {
+  if (dim == 3) return cpc >= JB_TB3_NB_MIN_CELLS && min_slab_ctas >= 64;
+  return cpc >= JB_TB2_NB_MIN_CELLS;
+}
+
 int lockstep_k(int units, int n_int, int64_t inner) {
   if (units <= 0 || n_int < units || inner <= 0) return 0;
   int64_t k = n_int / units;
@@ -224,6 +236,21 @@ int jacobi_geometry(int64_t nx, int64_t ny, int64_t nz, int stencil, int tile_x,
     return JACOBI_EINVAL;
   out8[0] = g.pitch; out8[1] = g.plane_elems; out8[2] = g.tx; out8[3] = g.ty;
   out8[4] = g.units_x; out8[5] = g.units_y; out8[6] = g.rh; out8[7] = g.ws;
+  return JACOBI_OK;
+}
+
+int jacobi_auto_policy(int64_t nx, int64_t ny, int64_t nz, int stencil, int nslabs, int virtual_slabs, int sms,
+                       int64_t *out4) {
+  if (!out4 || nx < 3 || ny < 3 || nslabs < 1 || sms < 1) return JACOBI_EINVAL;
+  if (!((stencil == 5 && nz == 1) || (stencil == 7 && nz >= 3))) return JACOBI_EINVAL;
+  const int dim = stencil == 5 ? 2 : 3;
+  const int64_t job_ctas = virtual_slabs ? sms : (int64_t)sms * nslabs;
+  const int min_slab_ctas = virtual_slabs ? sms / nslabs : sms;
+  const int64_t cpc = jbplan::cells_per_cta(nx, ny, nz, dim, job_ctas);
+  out4[0] = cpc;
+  out4[1] = jbplan::schedule_dynamic_auto(cpc) ? 1 : 0;
+  out4[2] = nslabs == 1 ? 1 : (jbplan::tblock_neighbours_auto(dim, cpc, min_slab_ctas) ? 1 : 0);
+  out4[3] = min_slab_ctas;
   return JACOBI_OK;
 }
 

@@ -199,9 +199,8 @@ int launch_ctas(const jacobi_ctx *h, int sms) {
 // Interior cells of the whole grid per CTA of the whole job (every slab's CTAs on every GPU):
 // the same number on every rank, so the policies below agree across processes.
 int64_t cells_per_cta(const jacobi_ctx *h, int sms) {
-  const int64_t cells = (h->nx - 2) * (h->dim == 3 ? (h->ny - 2) * (h->nz - 2) : (h->ny - 2));
   const int64_t devices = h->kind == KIND_VIRTUAL ? 1 : h->total;
-  return cells / std::max<int64_t>(1, (int64_t)launch_ctas(h, sms) * devices);
+  return jbplan::cells_per_cta(h->nx, h->ny, h->nz, h->dim, (int64_t)launch_ctas(h, sms) * devices);
 }
 
 // Interior schedule of the per-iteration kernel: knob "schedule" 0 / 1 static, 2 dynamic; auto
@@ -212,7 +211,7 @@ int64_t cells_per_cta(const jacobi_ctx *h, int sms) {
 // 2D 2048^2 with 2-8 virtual slabs 15.7 -> 11.1-12.2 us per iteration.
 bool schedule_dynamic(const jacobi_ctx *h, int sms) {
   if (h->schedule >= 0) return h->schedule == 2;
-  return cells_per_cta(h, sms) >= JB_DYN_MIN_CELLS;
+  return jbplan::schedule_dynamic_auto(cells_per_cta(h, sms));
 }
 
 // CTAs of slab `id` in its CPU-Free launch.
@@ -1027,9 +1026,9 @@ int run_cpufree(jacobi_ctx *h, int64_t iters) {
   if (!use_tb) {
     int sms = 0;
     CK(cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, h->slabs[0].device));
-    const int64_t cpc = cells_per_cta(h, sms);
-    use_tb = cpc >= (h->dim == 3 ? JB_TB3_NB_MIN_CELLS : JB_TB2_NB_MIN_CELLS);
-    for (int id = 0; id < h->total && use_tb && h->dim == 3; ++id) use_tb = slab_ctas(h, id, sms) >= 64;
+    int min_ctas = sms;
+    for (int id = 0; id < h->total; ++id) min_ctas = std::min(min_ctas, slab_ctas(h, id, sms));
+    use_tb = jbplan::tblock_neighbours_auto(h->dim, cells_per_cta(h, sms), min_ctas);
   }
   const bool use = eligible && (h->tblock == 1 || use_tb);
   int64_t tb_iters = 0;

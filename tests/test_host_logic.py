@@ -19,7 +19,7 @@ def built():
 
 def test_library_exports_every_header_symbol():
     names = jb.header_functions()
-    assert len(names) == len(jb._SIGS) == 31
+    assert len(names) == len(jb._SIGS) == 32
     L = ctypes.CDLL(jb.LIB_PATH)
     missing = [n for n in names if not hasattr(L, n)]
     assert not missing, missing
@@ -227,3 +227,36 @@ def test_halo_spans_summary():
     assert sp["wait_us"] == 1.0 and sp["put_us"] == 2.0 and sp["span_us"] == 3.0
     assert sp["period_us"] == 5.0 and sp["exchanges"] == n - 2
     assert jb.halo_spans(np.zeros((2, 4, 3), dtype=np.uint64))["span_us"] is None
+
+
+# ---------------------------------------------------------------- auto policies
+@pytest.mark.parametrize("shape,stencil,P,virtual,dyn,tb", [
+    # measured choices of profiles/r02_sched_sweep_*.jsonl
+    ((128, 128, 128), 7, 1, False, False, True),    # C5a: static schedule; one slab: time-blocked
+    ((128, 128, 128), 7, 2, True, False, False),    # 2 virtual slabs: per-iteration, static
+    ((256, 256, 256), 7, 2, True, False, False),    # 111 K cells per CTA: per-iteration
+    ((384, 384, 384), 7, 2, True, True, True),      # 380 K: time-blocked
+    ((384, 384, 384), 7, 4, True, True, False),     # 37 CTAs per slab < 64
+    ((512, 512, 512), 7, 2, True, True, True),      # C3 with 2 virtual slabs
+    ((512, 512, 512), 7, 8, True, True, False),     # 18 CTAs per slab
+    ((512, 512, 512), 7, 2, False, True, True),     # C3 on 2 GPUs: 227 K per CTA
+    ((512, 512, 512), 7, 8, False, False, False),   # C3 on 8 GPUs: 56 K per CTA
+    ((1, 2048, 2048), 5, 2, True, False, False),    # 28 K: per-iteration
+    ((1, 4096, 4096), 5, 2, True, False, True),     # 113 K: time-blocked, static interior (unused)
+    ((1, 16384, 16384), 5, 8, False, True, True),   # C2 on 8 GPUs: 227 K per CTA
+    ((1, 16384, 16384), 5, 8, True, True, True),    # C2 with 8 virtual slabs
+])
+def test_auto_policy_thresholds(shape, stencil, P, virtual, dyn, tb):
+    nz, ny, nx = shape
+    pol = jb.jacobi_auto_policy(nx, ny, nz, stencil, P, virtual)
+    cells = (nx - 2) * (ny - 2) * (nz - 2 if stencil == 7 else 1)
+    assert pol["cells_per_cta"] == cells // (148 if virtual else 148 * P)
+    assert pol["dynamic_schedule"] == dyn, pol
+    assert pol["tblock"] == tb, pol
+    assert pol["min_slab_ctas"] == (148 // P if virtual else 148)
+
+
+def test_auto_policy_rejects():
+    for args in [(2, 9, 1, 5, 1, 0, 148), (9, 9, 3, 5, 1, 0, 148), (9, 9, 1, 5, 0, 0, 148), (9, 9, 1, 5, 1, 0, 0)]:
+        with pytest.raises(jb.JacobiError):
+            jb.jacobi_auto_policy(*args)
