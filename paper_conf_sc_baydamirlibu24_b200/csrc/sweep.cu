@@ -643,7 +643,45 @@ __global__ void __launch_bounds__(JB_THREADS, 1) jb_sweep(const __grid_constant_
 
     // (no-compute: interior CTAs have no runs — they only join the barrier — and no CTA issues
     //  bulk copies, so the queue hand-off and the generic -> async proxy fences are skipped)
+    // No-compute boundary CTA with the flag protocol: the consumer warps copy their runs directly
+    // (the schedule is static), without the producer's run queue — three hand-offs fewer on the
+    // halo's critical path.  The neighbour's flag was acquired during the last barrier (pre-wait;
+    // t = 0: consumer warp 0 waits here first).
+    bool nc_direct = false;
+#ifdef JB_NVSHMEM
+    const bool shm_nc = SL.use_shm;
+#else
+    const bool shm_nc = false;
+#endif
+    if (NOCOMP && PERSIST && role != ROLE_INT && !llin && !llout && !shm_nc) nc_direct = true;
     if (NOCOMP && role == ROLE_INT) {
+    } else if (nc_direct) {
+      if (!producer) {
+        if (t == 0) {
+          if (warp == 0) {
+            const bool mark = lane == 0 && ridx == 0;
+            if (mark) halo_mark(SL, P, role == ROLE_BOT, t, 0);
+            const bool okw = role == ROLE_TOP ? wait_slots(SL.flag_in_top, SL.k_in_top, (unsigned long long)tg, P, lane)
+                                              : wait_slots(SL.flag_in_bot, SL.k_in_bot, (unsigned long long)tg, P, lane);
+            if (mark) halo_mark(SL, P, role == ROLE_BOT, t, 1);
+            if (lane == 0 && !okw) s_abort_pw = 1;
+          }
+          named_bar_consumers();
+        }
+        if (!s_abort_pw) {
+          Sched sched = sched0;
+          Run run;
+          double acc = 0.0;
+          while (sched.next(run))
+            consume_run<DIM, NOCOMP, false>(g, R, q, run, cur, nxt, remote, nullptr, tag_out, ctid, lane, acc);
+        }
+        // (the CTA barrier before the grid barrier orders every consumer's peer stores before
+        //  thread 0's release of the flag)
+        if (ctid == 0 && !drop_signal) {
+          sig_pending = (role == ROLE_TOP ? SL.flag_out_top : SL.flag_out_bot) + ridx;
+          if (ridx == 0) halo_mark(SL, P, role == ROLE_BOT, t, 2);
+        }
+      }
     } else if (producer) {
       // Every lane that issues bulk copies orders them after the grid barrier's acquire (and the
       // generic-proxy stores it covers) with its own proxy fence.
