@@ -40,11 +40,15 @@ __device__ __forceinline__ unsigned cl_n() { unsigned r; asm volatile("mov.u32 %
 // MODE 4: MODE 0 + fence.proxy.async by every thread (as the streaming kernel does)
 // MODE 5: cluster-hierarchical: cluster barrier, rank 0 counter (clusters arrive), cluster barrier
 // MODE 6: counter, volatile spin + fence after
+// MODE 7: production arrival, lane 0 of NPW warps polls (naturally staggered), the first to see
+//         the count raises a shared-memory flag the others also watch
 // bounded spin: a barrier that never completes (CTAs not co-resident) gives up after 0.5 s
 #define SPIN(cond) { const uint64_t ts_ = gt(); while (cond) { if (*(volatile unsigned long long *)(out + 148)) break; if (gt() - ts_ > 500000000ull) { out[148] = 1; break; } } }
 template <int MODE>
 __global__ void k(unsigned long long *ctr, unsigned long long *flag, int n, unsigned long long *out, int nunits) {
   const int tid = threadIdx.x;
+  __shared__ volatile int s_done[2];
+  if (tid == 0) s_done[0] = s_done[1] = 0;
   __syncthreads();
   uint64_t t0 = gt();
   for (int i = 0; i < n; ++i) {
@@ -57,6 +61,22 @@ __global__ void k(unsigned long long *ctr, unsigned long long *flag, int n, unsi
         SPIN(ld_acq(ctr) < target)
       }
       cl_arrive(); cl_wait();
+      continue;
+    }
+    if (MODE >= 7) {
+      const int NPW = MODE - 5;  // 7: 2 warps, 8: 3, 9: 4
+      __syncthreads();
+      const int par = i & 1;
+      if (tid == 0) { s_done[par ^ 1] = 0; red_rel(ctr, 1ull); }
+      if ((tid & 31) == 0 && (tid >> 5) < NPW) {
+        const uint64_t ts_ = gt();
+        while (!s_done[par]) {
+          if (ld_acq(ctr) >= target) { s_done[par] = 1; break; }
+          if (*(volatile unsigned long long *)(out + 148)) break;
+          if (gt() - ts_ > 500000000ull) { out[148] = 1; break; }
+        }
+      }
+      __syncthreads();
       continue;
     }
     __syncthreads();
@@ -108,10 +128,12 @@ int main() {
   cudaMalloc(&ctr, 256); cudaMalloc(&flag, 256); cudaMalloc(&out, 149 * 8); cudaMemset(out, 0, 149 * 8);
   const char *names[] = {"counter red.release + ld.acquire spin (production)", "counter, relaxed spin + fence",
                          "atom.acq_rel + last-arriver release flag", "counter without release (incorrect)",
-                         "production + fence.proxy.async", "cluster-hierarchical", "counter, volatile spin + fence"};
+                         "production + fence.proxy.async", "cluster-hierarchical", "counter, volatile spin + fence",
+                         "production arrival, 2 polling warps", "production arrival, 3 polling warps",
+                         "production arrival, 4 polling warps"};
   for (int grid : {1, 8, 32, 74, 148}) {
-    for (int m = 0; m < 7; ++m) {
-      if (m == 5) continue;
+    for (int m = 0; m < 10; ++m) {
+      if (m == 5 || m == 1 || m == 2 || m == 3 || m == 4 || m == 6) continue;
       float v = 0;
       for (int rep = 0; rep < 2; ++rep) {
         if (m == 0) v = run<0>(grid, 1, ctr, flag, out);
@@ -120,11 +142,15 @@ int main() {
         if (m == 3) v = run<3>(grid, 1, ctr, flag, out);
         if (m == 4) v = run<4>(grid, 1, ctr, flag, out);
         if (m == 6) v = run<6>(grid, 1, ctr, flag, out);
+        if (m == 7) v = run<7>(grid, 1, ctr, flag, out);
+        if (m == 8) v = run<8>(grid, 1, ctr, flag, out);
+        if (m == 9) v = run<9>(grid, 1, ctr, flag, out);
       }
       printf("ctas %3d  %-52s %8.1f ns/barrier\n", grid, names[m], v);
     }
   }
-  for (int cl : {2, 4, 8, 16}) {
+  for (int cl : {0}) {  // (cluster-hierarchical: profiles/r02_ubench_barrier.txt)
+    if (!cl) continue;
     for (int grid : {cl * 8, 144}) {
       if (cl == 16) {
         cudaFuncSetAttribute(k<5>, cudaFuncAttributeNonPortableClusterSizeAllowed, 1);
