@@ -236,15 +236,18 @@ __device__ __forceinline__ void st_relaxed_gpu(unsigned long long *p, unsigned l
 }
 __device__ bool slab_barrier(const JbSlab &SL, const JbParams &P, int c, unsigned long long k,
                              unsigned long long epoch, int lane, unsigned long long *sig = nullptr,
-                             unsigned long long sigv = 0) {
-  // release pattern: fence, then relaxed stores of the flag and the arrival
+                             unsigned long long sigv = 0, unsigned long long *sig2 = nullptr) {
+  // release pattern: fence, then relaxed stores of the flag(s) and the arrival (sig2: a second
+  // flag with the same value — a block that borders both neighbours)
   auto fence_and_signal = [&]() {
     if (flag_gpu_scope(P)) {
       fence_acq_rel_gpu();
       st_relaxed_gpu(sig, sigv);
+      if (sig2) st_relaxed_gpu(sig2, sigv);
     } else {
       fence_acq_rel_sys();
       st_relaxed_sys(sig, sigv);
+      if (sig2) st_relaxed_sys(sig2, sigv);
     }
   };
   // The abort flag (another CTA's watchdog / error) is read right AFTER the arrival (not before:

@@ -191,11 +191,20 @@ __global__ void __launch_bounds__(JB_RNT, 1) jb_resident(const __grid_constant__
         if (bot_face >> i & 1u) store_pair(rb + (gofs[i] - (pz0 + zb - 1) * pe), v[i].x, v[i].y, fl);
       }
     }
+    // Signal: with the grid barrier the block's next action is its arrival, so the
+    // flag(s) share the arrival's release fence (slab_barrier; one fence instead of two
+    // serialised ones); with relaxed sync a release store of its own.
+    unsigned long long *sig_top = nullptr, *sig_bot = nullptr;
     if (top_blk || bot_blk) {
-      __syncthreads();  // every thread's peer stores precede thread 0's release (CTA scope)
+      if (relaxed) __syncthreads();  // every thread's peer stores precede thread 0's release (CTA scope)
       if (tid == 0 && !((P.flags & JACOBI_FLAG_DROP_SIGNAL) && SL.slab_id == 0)) {
-        if (top_blk) st_release_flag(P, SL.flag_out_top + by, (unsigned long long)(tg + 1));
-        if (bot_blk) st_release_flag(P, SL.flag_out_bot + by, (unsigned long long)(tg + 1));
+        if (relaxed) {
+          if (top_blk) st_release_flag(P, SL.flag_out_top + by, (unsigned long long)(tg + 1));
+          if (bot_blk) st_release_flag(P, SL.flag_out_bot + by, (unsigned long long)(tg + 1));
+        } else {
+          if (top_blk) sig_top = SL.flag_out_top + by;
+          if (bot_blk) sig_bot = SL.flag_out_bot + by;
+        }
         if (by == 0) {
           if (top_blk) halo_mark(SL, P, 0, t, 2);
           if (bot_blk) halo_mark(SL, P, 1, t, 2);
@@ -210,7 +219,9 @@ __global__ void __launch_bounds__(JB_RNT, 1) jb_resident(const __grid_constant__
       continue;
     }
     if (tid < 32) {
-      const bool ok = slab_barrier(SL, P, c, (unsigned long long)(t + 1), (unsigned long long)(tg + 1), tid);
+      const bool ok = slab_barrier(SL, P, c, (unsigned long long)(t + 1), (unsigned long long)(tg + 1), tid,
+                                   sig_top ? sig_top : sig_bot, (unsigned long long)(tg + 1),
+                                   sig_top ? sig_bot : nullptr);
       if (tid == 0) s_abort = ok ? 0 : 1;  // (slab_barrier also reports an abort flag)
     } else if (tid < 64 && (top_blk || bot_blk) && t + 1 < P.iters) {
       // Pre-wait (P:394's wait, off the critical path): the neighbour raises the next

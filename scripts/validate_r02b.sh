@@ -1,7 +1,7 @@
 #!/bin/bash
 # Final round-2 validation on the GPU box (gpurun): GPU test suite, smoke, bench lines of every
 # config (+ virtual-slab lines, the reference arm), the C5 latency sweep, and the launch list of
-# the default bench command — all under gpurun_out/ (prefix f_).
+# the default bench command — all under gpurun_out/ (prefix f_; re-run as the last validation of the round).
 out=gpurun_out
 nvidia-smi --query-gpu=name,clocks.sm,clocks.max.sm,power.limit,temperature.gpu --format=csv > $out/f_smi.txt
 timeout 1200 python -m pytest tests -m gpu -q > $out/f_pytest_gpu.log 2>&1; echo "rc=$?" >> $out/f_pytest_gpu.log
