@@ -45,6 +45,9 @@ __device__ __forceinline__ void tma_box3(void *dst, const void *tmap, int c0, in
 
 // The odd-K marches run towards row / plane 0 (shorter fp64 dependency chain, see tbk_march).
 constexpr bool TB_REV = true;
+#ifndef TB2_HOIST
+#define TB2_HOIST 1  // 2D odd-K march: shuffle every level's centre-row x neighbours at the step start
+#endif
 #ifndef TB3_PF
 #define TB3_PF 1  // 3D odd-K march: level-0 planes of the steady state kept in registers (tb3k_march)
 #endif
@@ -316,9 +319,10 @@ __device__ __forceinline__ double shfl_d(double v, int src) {
 // STORE: level K, written to o (this lane's pair 0 in the output row) instead of V.
 template <int PPT, bool FAST, bool STEADY, bool STORE>
 __device__ __forceinline__ void tbk_levelk(const TbkLane &L, const double2 *S, const double2 *Cm, const double2 *N,
-                                           bool rowin, int lane, double2 *V, double *o) {
-  const double Wl = shfl_d(Cm[PPT - 1].y, (lane + 31) & 31);
-  const double Er = shfl_d(Cm[0].x, (lane + 1) & 31);
+                                           bool rowin, int lane, double2 *V, double *o, const double *WE = nullptr) {
+  // WE: this level's x neighbours of the centre row, already shuffled (TB2_HOIST)
+  const double Wl = WE ? WE[0] : shfl_d(Cm[PPT - 1].y, (lane + 31) & 31);
+  const double Er = WE ? WE[1] : shfl_d(Cm[0].x, (lane + 1) & 31);
 #pragma unroll
   for (int i = 0; i < PPT; ++i) {
     const double W = i == 0 ? Wl : Cm[i - 1].y;
@@ -400,6 +404,16 @@ __device__ __forceinline__ void tbk_march(const TbkLane &L, const Ring &R, RingP
     constexpr int SN = (U + NS - (LAG - 1)) % NS, SC = (U + NS - LAG) % NS, SS = (U + 2 * NS - LAG - 1) % NS;
     // level k computes row Rr-1-LAG(k-1) if it lies in its range [a-(K-k), b+(K-k)] ∩ [0, C+1]
     auto need = [&](int k, int r) { return r >= max(a - (K - k), 0) && r <= min(b + (K - k), C + 1); };
+    // TB2_HOIST: the x neighbours of every level's centre row (computed in the previous step) are
+    // shuffled at the start of the step, off the chain through this step's newest rows
+    double WE[K - 1][2];
+    if (TB2_HOIST && ST) {
+#pragma unroll
+      for (int k = 2; k <= K; ++k) {
+        WE[k - 2][0] = shfl_d(X[k - 2][SC][PPT - 1].y, (lane + 31) & 31);
+        WE[k - 2][1] = shfl_d(X[k - 2][SC][0].x, (lane + 1) & 31);
+      }
+    }
     if (ST && PF) {
       // level-0 rows Rr (newest, Z[U]), Rr-1 (centre, Z[U+2]), Rr-2 (Z[U+1]), preloaded
       constexpr int ZN = U % 3, ZC = (U + 2) % 3, ZO = (U + 1) % 3;
@@ -425,12 +439,13 @@ __device__ __forceinline__ void tbk_march(const TbkLane &L, const Ring &R, RingP
       const int r = Rr - 1 - LAG * (k - 1);
       if (ST || need(k, r))
         tbk_levelk<PPT, FAST, ST, false>(L, X[k - 2][REV ? SN : SS], X[k - 2][SC], X[k - 2][REV ? SS : SN],
-                                         r >= 1 && r <= C, lane, X[k - 1][U], nullptr);
+                                         r >= 1 && r <= C, lane, X[k - 1][U], nullptr,
+                                         (TB2_HOIST && ST) ? WE[k - 2] : nullptr);
     }
     const int ro = Rr - 1 - LAG * (K - 1);
     if (ST || (ro >= a && ro <= b))
       tbk_levelk<PPT, FAST, ST, true>(L, X[K - 2][REV ? SN : SS], X[K - 2][SC], X[K - 2][REV ? SS : SN], true, lane,
-                                      nullptr, o);
+                                      nullptr, o, (TB2_HOIST && ST) ? WE[K - 2] : nullptr);
     o += ostep;
     pm = pc;
     pc = pn;
