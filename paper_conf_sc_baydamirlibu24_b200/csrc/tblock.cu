@@ -305,6 +305,27 @@ __device__ __forceinline__ void tbk_level1_regs(const TbkLane &L, const double2 
 }
 
 // A double from lane src (two 32-bit shuffles, halves kept in place).
+// A double from lane l-1 (up) / l+1 (down): constant deltas, no lane index (whose S2R read the
+// compiler re-issues inside the 2D march and whose latency the shuffles then wait for: C2 +3-4 %;
+// the 3D march keeps the indexed form, measured equal-or-better there).  Lane 0 / 31
+// keep their own value — like the wrapped value before, it only reaches cells outside the valid
+// span (each level loses one column per segment end).
+__device__ __forceinline__ double shfl_up_d(double v) {
+  double r;
+  asm("{\n .reg .b32 lo, hi;\n mov.b64 {lo, hi}, %1;\n shfl.sync.up.b32 lo, lo, 1, 0x0, -1;\n"
+      " shfl.sync.up.b32 hi, hi, 1, 0x0, -1;\n mov.b64 %0, {lo, hi};\n}"
+      : "=d"(r)
+      : "d"(v));
+  return r;
+}
+__device__ __forceinline__ double shfl_down_d(double v) {
+  double r;
+  asm("{\n .reg .b32 lo, hi;\n mov.b64 {lo, hi}, %1;\n shfl.sync.down.b32 lo, lo, 1, 0x1f, -1;\n"
+      " shfl.sync.down.b32 hi, hi, 1, 0x1f, -1;\n mov.b64 %0, {lo, hi};\n}"
+      : "=d"(r)
+      : "d"(v));
+  return r;
+}
 __device__ __forceinline__ double shfl_d(double v, int src) {
   double r;
   asm("{\n .reg .b32 lo, hi;\n mov.b64 {lo, hi}, %1;\n shfl.sync.idx.b32 lo, lo, %2, 0x1f, -1;\n"
@@ -321,8 +342,8 @@ template <int PPT, bool FAST, bool STEADY, bool STORE>
 __device__ __forceinline__ void tbk_levelk(const TbkLane &L, const double2 *S, const double2 *Cm, const double2 *N,
                                            bool rowin, int lane, double2 *V, double *o, const double *WE = nullptr) {
   // WE: this level's x neighbours of the centre row, already shuffled (TB2_HOIST)
-  const double Wl = WE ? WE[0] : shfl_d(Cm[PPT - 1].y, (lane + 31) & 31);
-  const double Er = WE ? WE[1] : shfl_d(Cm[0].x, (lane + 1) & 31);
+  const double Wl = WE ? WE[0] : shfl_up_d(Cm[PPT - 1].y);
+  const double Er = WE ? WE[1] : shfl_down_d(Cm[0].x);
 #pragma unroll
   for (int i = 0; i < PPT; ++i) {
     const double W = i == 0 ? Wl : Cm[i - 1].y;
@@ -410,8 +431,8 @@ __device__ __forceinline__ void tbk_march(const TbkLane &L, const Ring &R, RingP
     if (TB2_HOIST && ST) {
 #pragma unroll
       for (int k = 2; k <= K; ++k) {
-        WE[k - 2][0] = shfl_d(X[k - 2][SC][PPT - 1].y, (lane + 31) & 31);
-        WE[k - 2][1] = shfl_d(X[k - 2][SC][0].x, (lane + 1) & 31);
+        WE[k - 2][0] = shfl_up_d(X[k - 2][SC][PPT - 1].y);
+        WE[k - 2][1] = shfl_down_d(X[k - 2][SC][0].x);
       }
     }
     if (ST && PF) {
