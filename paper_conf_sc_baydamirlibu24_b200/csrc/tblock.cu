@@ -406,7 +406,12 @@ __device__ __forceinline__ void tbk_march(const TbkLane &L, const Ring &R, RingP
   double2 Z[3][PPT];
   double zW = 0.0, zE = 0.0;
   RingPos pnn = pn;  // steady steps: the next step's newest row
-  const uint32_t sbase = sptr(R.stages) + 8u * (uint32_t)L.j0;
+  // shared-window addresses fixed for the march, kept in registers (not re-derived from S2R
+  // reads inside the loop, whose latency the dependent instructions would wait for)
+  const uint32_t sbase = opaque_u32(sptr(R.stages) + 8u * (uint32_t)L.j0);
+  const uint32_t fbase = opaque_u32(sptr(R.full)), ebase = opaque_u32(sptr(R.empty));
+  auto wait_full_s = [&](const RingPos &p) { mbar_wait_s(fbase + 8u * p.slot, p.phase); };
+  auto release_s = [&](const RingPos &p) { mbar_arrive_s(ebase + 8u * p.slot); };
   const uint32_t sstride = 8u * (uint32_t)(SD > 0 ? SD : R.stage_doubles);
   auto zload = [&](double2 *z, const RingPos &p) {
     const uint32_t st = sbase + p.slot * sstride;
@@ -439,12 +444,12 @@ __device__ __forceinline__ void tbk_march(const TbkLane &L, const Ring &R, RingP
       // level-0 rows Rr (newest, Z[U]), Rr-1 (centre, Z[U+2]), Rr-2 (Z[U+1]), preloaded
       constexpr int ZN = U % 3, ZC = (U + 2) % 3, ZO = (U + 1) % 3;
       tbk_level1_regs<PPT, FAST>(L, Z[REV ? ZN : ZO], Z[ZC], Z[REV ? ZO : ZN], zW, zE, X[0][U]);
-      R.release(pm, lane);  // row Rr-2: its last reads were the preloads
+      release_s(pm);  // row Rr-2: its last reads were the preloads
       // next step (steady steps end before r1): its newest row into Z[U+1] (row Rr-2's, now
       // dead), W / E of its centre row Rr
       pnn = pn;
       pnn.advance(R.S);
-      R.wait_full(pnn);
+      wait_full_s(pnn);
       zload(Z[ZO], pnn);
       weload(pn);
     } else {
