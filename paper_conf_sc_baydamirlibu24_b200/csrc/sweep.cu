@@ -265,12 +265,15 @@ __device__ __forceinline__ void consume_run_2d(const JbGeom &g, const Ring &R, R
                  // 16-byte loads straight from the current buffer (L2), no ring stages
     for (int64_t p = 0; p < L; ++p) {
       const double *src = cur + (run.p0 + p) * g.plane_elems + col;
+      double2 v[PPT];  // every pair's load issued before the stores (one L2 round trip)
+#pragma unroll
+      for (int i = 0; i < PPT; ++i)
+        if ((ok >> i & 1u) && (remote || rll)) v[i] = __ldcg(reinterpret_cast<const double2 *>(src + 2 * i * JB_NC));
 #pragma unroll
       for (int i = 0; i < PPT; ++i)
         if ((ok >> i & 1u) && (remote || rll)) {
-          const double2 v = __ldcg(reinterpret_cast<const double2 *>(src + 2 * i * JB_NC));
-          if (rll) ll_store_pair(rll + 2 * (col + 2 * i * JB_NC), v.x, v.y, full >> i & 1u, tag);
-          else store_pair(remote + col + 2 * i * JB_NC, v.x, v.y, full >> i & 1u);
+          if (rll) ll_store_pair(rll + 2 * (col + 2 * i * JB_NC), v[i].x, v[i].y, full >> i & 1u, tag);
+          else store_pair(remote + col + 2 * i * JB_NC, v[i].x, v[i].y, full >> i & 1u);
         }
     }
     return;
@@ -366,10 +369,17 @@ __device__ __forceinline__ void consume_run_3d(const JbGeom &g, const Ring &R, R
             ll_store_pair(o, v.x, v.y, full, tag);
           }
         } else {
+          // loads of up to 4 rows issued before their stores: one L2 round trip per 4 rows on the
+          // halo's critical path instead of one per row
           double *o = remote + col;
-          for (int r = rb; r < re; ++r, c += g.pitch, o += g.pitch) {
-            const double2 v = __ldcg(reinterpret_cast<const double2 *>(c));
-            store_pair(o, v.x, v.y, full);
+          for (int r = rb; r < re; r += 4, c += 4 * g.pitch, o += 4 * g.pitch) {
+            double2 v[4];
+#pragma unroll
+            for (int u = 0; u < 4; ++u)
+              if (r + u < re) v[u] = __ldcg(reinterpret_cast<const double2 *>(c + u * g.pitch));
+#pragma unroll
+            for (int u = 0; u < 4; ++u)
+              if (r + u < re) store_pair(o + u * g.pitch, v[u].x, v[u].y, full);
           }
         }
       }
